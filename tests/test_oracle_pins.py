@@ -1,0 +1,568 @@
+"""Pins for the CPU oracle (oracle/ll_oracle.py) against what the paper and the
+mathematics fix — NOT against the oracle itself.  Each test names its pin.
+All run on CPU (-m "not gpu")."""
+import itertools
+import json
+import os
+
+import numpy as np
+import pytest
+
+from oracle import ll_oracle as O
+from workloads import configs as W
+from workloads import gen
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def load(name):
+    with open(os.path.join(GOLD, name)) as f:
+        return json.load(f)
+
+
+def L_of(spec):
+    return O.Layout(*W.spec_to_bases(spec))
+
+
+# ----------------------------------------------------------------------------- GV1/GV2
+
+def fig1_A_from_matrix():
+    g = load("fig1_table1.json")
+    rows = g["matrix_A_rows"]
+    out_dims = [tuple(d) for d in g["out_dims"]]
+    names = ["reg", "reg", "lane", "lane", "lane", "lane", "lane", "warp"]
+    bases = {"reg": [], "lane": [], "warp": []}
+    for col in range(8):
+        i = sum(rows[f"i{k}"][col] << k for k in range(4))
+        j = sum(rows[f"j{k}"][col] << k for k in range(4))
+        bases[names[col]].append((i, j))
+    return O.Layout([tuple(d) for d in g["in_dims"]], out_dims, bases), g
+
+
+def test_table1_rows_reproduced_by_matrix_A():
+    """GV1: every printed row of Table 1 equals A·v with the P:140 matrix,
+    and the min-index preimage maps it back (A is bijective)."""
+    A, g = fig1_A_from_matrix()
+    first = O.preimage_min(A)
+    for i, j, r, t, w in g["table1_ij_reg_thread_warp"]:
+        h = O.hw_flat(A.in_dims, (r, t, w))
+        assert O.logical_coords(A.out_dims, O.apply(A, h)) == (i, j)
+        assert first[O.logical_flat(A.out_dims, (i, j))] == h
+    assert O.is_injective(A) and O.is_surjective(A)
+
+
+def test_worked_example_r1_t9_w0():
+    """GV2: loc_r1=(0,1), loc_t9=(2,2), loc_w0=(0,0), XOR=(2,3)."""
+    A, g = fig1_A_from_matrix()
+    ex = g["worked_example"]
+    loc = lambda r, t, w: O.logical_coords(A.out_dims, O.apply(A, O.hw_flat(A.in_dims, (r, t, w))))
+    assert loc(ex["reg"], 0, 0) == tuple(ex["loc_reg"])
+    assert loc(0, ex["thread"], 0) == tuple(ex["loc_thread"])
+    assert loc(0, 0, ex["warp"]) == tuple(ex["loc_warp"])
+    assert loc(ex["reg"], ex["thread"], ex["warp"]) == tuple(ex["ij"])
+
+
+def test_blocked_constructor_is_fig1_A():
+    """GV3 (P:128 vs P:140): blocked([2,2],[4,8],[2,1],[1,0]) on 16x16 == matrix A."""
+    A, g = fig1_A_from_matrix()
+    p = g["blocked_params_P128"]
+    Lb = O.blocked(p["shape"], p["size_per_thread"], p["threads_per_warp"], p["warps_per_cta"], p["order"])
+    assert Lb.cols == A.cols
+
+
+def test_fig1_literal_tables_match_matrix():
+    A, _ = fig1_A_from_matrix()
+    assert L_of(W.C1_A).cols == A.cols
+
+
+@pytest.mark.parametrize("which,ctor", [
+    ("c2B", lambda: O.blocked([128, 128], [8, 8], [2, 16], [4, 1], [1, 0])),
+    ("c3A", lambda: O.blocked([256, 128], [1, 8], [2, 16], [4, 1], [1, 0])),
+    ("c3B", lambda: O.blocked([256, 128], [8, 1], [32, 1], [1, 4], [0, 1])),
+    ("c3bA", lambda: O.blocked([256, 128], [8, 8], [2, 16], [4, 1], [1, 0])),
+    ("c3bB", lambda: O.blocked([256, 128], [8, 8], [32, 1], [1, 4], [0, 1])),
+    ("c2A", lambda: O.mma_acc([128, 128], 4)),
+])
+def test_constructors_match_appendix_tables(which, ctor):
+    tbl = {"c2B": W.c2(0)[1], "c3A": W.c3(0)[0], "c3B": W.c3(0)[1],
+           "c3bA": W.c3b(0)[0], "c3bB": W.c3b(0)[1], "c2A": W.c2(0)[0]}[which]
+    lit = L_of(tbl)
+    got = ctor()
+    # compare per hardware bit, on the tile dims (drop the empty batch dim)
+    assert [c for c in got.cols] == [c for c in lit.cols]
+
+
+def test_mma_acc_matches_ptx_fragment():
+    """Prop 9.2 vs the PTX m16n8 C/D fragment [HW]: element d[k] of lane l
+    sits at row = l/4 + 8*(k/2 % 2), col = 2*(l % 4) + k % 2, repeated over n in
+    8-column blocks then over m in 16-row blocks (wgmma: warps along M, 16 rows)."""
+    L = O.mma_acc([128, 128], 4)
+    ntile = 128 // 8
+    for h in range(1 << L.d_in):
+        r = h & 127
+        lane = (h >> 7) & 31
+        warp = h >> 12
+        q = r & 3                 # position in the m16n8 fragment
+        nrep = (r >> 2) & (ntile - 1)
+        mrep = r >> (2 + 4)
+        row = lane // 4 + 8 * (q // 2) + 16 * warp + 64 * mrep
+        col = 2 * (lane % 4) + q % 2 + 8 * nrep
+        # the register numbering of Prop 9.2 is reg0 -> j0, reg1 -> i3 (G17)
+        assert O.logical_coords(L.out_dims, O.apply(L, h)) == (row, col)
+
+
+# ----------------------------------------------------------------------------- GV4
+
+def test_mma_swizzle_linear_and_C_rows():
+    """GV4: the [[I_n, C],[0, I_m]] layout equals the Def 4.11 formula at all
+    4096 points, and its C rows equal the P:264 values."""
+    g = load("mma_swizzle_C.json")
+    m, n = g["m"], g["n"]
+    for case in g["cases"]:
+        vec, pp, mp = case["vec"], case["per_phase"], case["max_phase"]
+        assert O.mma_swizzle_C(m, n, vec, pp, mp) == case["C"]
+        L = O.mma_swizzle_layout(m, n, vec, pp, mp)
+        for i in range(1 << m):
+            for j in range(1 << n):
+                off = O.apply(L, j | (i << n))
+                assert off == (i << n) + O.mma_swizzle_offset(i, j, vec, pp, mp)
+        assert O.is_memory(L)
+
+
+# ----------------------------------------------------------------------------- predicates
+
+@pytest.mark.parametrize("ctor", [
+    lambda: O.blocked([16, 16], [2, 2], [4, 8], [2, 1], [1, 0]),
+    lambda: O.blocked([8, 8], [1, 1], [4, 8], [2, 1], [1, 0]),     # broadcast: 64 < 256 slots
+    lambda: O.mma_acc([64, 32], 4),
+    lambda: O.mma_acc([16, 8], 1),
+])
+def test_blocked_and_mma_are_distributed(ctor):
+    """P:206 (blocked), P:212 (mma) with Def 4.10."""
+    assert O.is_distributed(ctor())
+
+
+def test_sliced_is_surjective_maybe_not_injective():
+    """Remark P:224: a slice stays surjective, may lose injectivity."""
+    L = O.blocked([16, 16], [2, 2], [4, 8], [2, 1], [1, 0])
+    S = O.sliced(L, 1)
+    assert O.is_surjective(S) and not O.is_injective(S)
+    zero = [c for c in S.cols if c == 0]
+    assert len(zero) == 4          # the j bits became zero (broadcast) columns
+
+
+# ----------------------------------------------------------------------------- inverse
+
+def test_right_inverse_equals_min_index_preimage_random():
+    """Slack-zero Gaussian elimination == brute-force min-index
+    preimage, and A∘A^+ = I (Def 4.5)."""
+    rng = np.random.default_rng(7)
+    for trial in range(600):
+        d_out = int(rng.integers(1, 7))
+        d_in = int(rng.integers(d_out, 10))
+        cols = gen.random_surjective_cols(rng, d_out, d_in)
+        L = O.layout_from_cols([("h", d_in)], [("x", d_out)], cols)
+        first = O.preimage_min(L)
+        xs = np.arange(1 << d_out, dtype=np.uint64)
+        assert np.array_equal(O.apply_inverse_all(L, xs).astype(np.int64), first)
+        assert np.array_equal(O.apply_all(L, first.astype(np.uint64)), xs)
+
+
+def test_inverse_of_injective_is_two_sided():
+    rng = np.random.default_rng(11)
+    for _ in range(50):
+        d = int(rng.integers(1, 9))
+        cols = gen.random_memory_cols(rng, d)
+        L = O.layout_from_cols([("offset", d)], [("x", d)], cols)
+        Li = O.right_inverse(L)
+        hs = np.arange(1 << d, dtype=np.uint64)
+        assert np.array_equal(O.apply_all(Li, O.apply_all(L, hs)), hs)     # A^+∘A = I
+        assert O.is_memory(L)
+
+
+def test_left_inverse_fails_for_broadcast():
+    """A^+∘A = I iff A is injective (zero columns are lost)."""
+    L = O.blocked([8, 8], [1, 1], [4, 8], [2, 1], [1, 0])
+    Li = O.right_inverse(L)
+    hs = np.arange(1 << L.d_in, dtype=np.uint64)
+    assert not np.array_equal(O.apply_all(Li, O.apply_all(L, hs)), hs)
+
+
+def test_nonsurjective_has_no_right_inverse():
+    L = O.layout_from_cols([("h", 3)], [("x", 3)], [1, 2, 3])
+    with pytest.raises(ValueError):
+        O.right_inverse(L)
+    with pytest.raises(ValueError):
+        O.preimage_min(L)
+
+
+# ----------------------------------------------------------------------------- compose etc.
+
+def test_compose_is_function_composition_and_associative():
+    """Def 4.2: (L2∘L1)(u) = L2(L1(u)); associativity."""
+    rng = np.random.default_rng(3)
+    for _ in range(40):
+        a, b, c, d = (int(x) for x in rng.integers(1, 7, size=4))
+        L1 = O.layout_from_cols([("u", a)], [("v", b)], [int(x) for x in rng.integers(0, 1 << b, a)])
+        L2 = O.layout_from_cols([("v", b)], [("w", c)], [int(x) for x in rng.integers(0, 1 << c, b)])
+        L3 = O.layout_from_cols([("w", c)], [("z", d)], [int(x) for x in rng.integers(0, 1 << d, c)])
+        C = O.compose(L2, L1)
+        for u in range(1 << a):
+            assert O.apply(C, u) == O.apply(L2, O.apply(L1, u))
+        assert O.compose(L3, C).cols == O.compose(O.compose(L3, L2), L1).cols
+
+
+def test_product_then_left_division_roundtrip():
+    """(M1 × M2) /_l M1 = M2 (Defs 4.3, 4.4)."""
+    M1 = O.blocked([4, 4], [2, 2], [2, 2], [1, 1], [1, 0])
+    M2 = O.blocked([8, 4], [1, 2], [4, 2], [2, 1], [1, 0])
+    M1 = O.Layout(M1.in_dims, [("d0", 2), ("d1", 2)], M1.bases)
+    P = O.product(M1, M2)
+    Q = O.left_divide(P, M1)
+    assert Q.cols == M2.cols
+    # block-diagonal structure: M1 bits stay inside M1's range
+    with pytest.raises(ValueError):
+        O.left_divide(P, M2)
+
+
+def test_left_divide_ldst_tile():
+    """Thm 5.1 with the vectorised ld/st tile: a layout whose two lowest
+    register bits are the two lowest offset bits is divisible by id_2^{Reg,Off}."""
+    T = O.Layout([("reg", 2)], [("offset", 2)], {"reg": [(1,), (2,)]})
+    L = O.Layout([("reg", 3), ("lane", 1)], [("offset", 4)], {"reg": [(1,), (2,), (8,)], "lane": [(4,)]})
+    R = O.left_divide(L, T)
+    assert R.cols == [2, 1]
+    L_bad = O.Layout([("reg", 3), ("lane", 1)], [("offset", 4)], {"reg": [(2,), (1,), (8,)], "lane": [(4,)]})
+    with pytest.raises(ValueError):
+        O.left_divide(L_bad, T)
+
+
+# ----------------------------------------------------------------------------- convert
+
+def test_convert_closed_form_pack():
+    """O5: convert(pack_A(T)) == pack_B(T) for Fig. 1 A -> B and the batch variant."""
+    rng = np.random.default_rng(1001)
+    A, B = L_of(W.C1_A), L_of(W.C1_B)
+    T = gen.random_bits(rng, 256, 4)
+    assert np.array_equal(O.convert(A, B, O.pack(A, T)), O.pack(B, T))
+    A2, B2 = (L_of(s) for s in W.c1_batched(3))
+    T2 = gen.random_bits(rng, 256 * 8, 4)
+    assert np.array_equal(O.convert(A2, B2, O.pack(A2, T2)), O.pack(B2, T2))
+
+
+def test_convert_identity_and_transpose_library():
+    """A = B is the identity; row-major -> column-major memory layouts is
+    numpy.transpose (a library routine)."""
+    rng = np.random.default_rng(5)
+    out = [("i", 3), ("j", 4)]
+    row = O.identity_memory(out)
+    col = O.layout_from_cols([("offset", 7)], out, [1 << (4 + k) for k in range(3)] + [1 << k for k in range(4)])
+    T = gen.random_bits(rng, 128, 2)
+    assert np.array_equal(O.convert(row, row, T), T)
+    got = O.convert(row, col, T)
+    assert np.array_equal(got, T.reshape(8, 16).T.reshape(-1))
+
+
+def test_convert_random_exhaustive_small():
+    """Exhaustive 2^8 spaces (E1 subsample): random bijective B against Fig. 1 A;
+    closed form and A-consistency; broadcast variant with zero columns."""
+    rng = np.random.default_rng(2024)
+    A = L_of(W.C1_A)
+    hw = [("reg", 2), ("lane", 5), ("warp", 1)]
+    T = gen.random_bits(rng, 256, 4)
+    for _ in range(200):
+        B = L_of(gen.random_distributed(rng, W.C1_OUT, hw))
+        assert np.array_equal(O.convert(A, B, O.pack(A, T)), O.pack(B, T))
+    out7 = [("i", 3), ("j", 4)]
+    T7 = gen.random_bits(rng, 128, 4)
+    for _ in range(200):
+        A7 = L_of(gen.random_distributed(rng, out7, hw, zero_ok=["reg"]))
+        B7 = L_of(gen.random_distributed(rng, out7, hw, zero_ok=["lane"]))
+        src = O.pack(A7, T7)
+        assert O.is_consistent(A7, src)
+        assert np.array_equal(O.convert(A7, B7, src), O.pack(B7, T7))
+
+
+def test_convert_at_matches_full_convert():
+    rng = np.random.default_rng(9)
+    A, B = (L_of(s) for s in W.c1_batched(4))
+    T = gen.random_bits(rng, 256 * 16, 4)
+    src = O.pack(A, T)
+    full = O.convert(A, B, src)
+    hs = rng.integers(0, 1 << B.d_in, size=500).astype(np.uint64)
+    assert np.array_equal(O.convert_at(A, B, src, hs), full[hs.astype(np.int64)])
+
+
+# ----------------------------------------------------------------------------- class
+
+def test_class_special_cases():
+    """O7 on cases the paper fixes: A = B is NOOP; swapping A's register bits is a
+    register permutation; Fig.1 A->B^T needs smem (warp bit moves)."""
+    A = L_of(W.C1_A)
+    assert O.classify(A, A) == "NOOP"
+    swapped = {"out": W.C1_OUT, "in": [("reg", ["i0", "j0"]), ("lane", ["j1", "j2", "j3", "i1", "i2"]), ("warp", ["i3"])]}
+    assert O.classify(A, L_of(swapped)) == "REGPERM"
+    lane_perm = {"out": W.C1_OUT, "in": [("reg", ["j0", "i0"]), ("lane", ["j2", "j1", "j3", "i1", "i2"]), ("warp", ["i3"])]}
+    assert O.classify(A, L_of(lane_perm)) == "SHUFFLE"
+    assert O.classify(A, L_of(W.C1_B)) == "SMEM"
+    A2, B2 = (L_of(s) for s in W.c1_batched(2))
+    blk = {"out": A2.out_dims, "in": [("reg", ["j0", "i0"]), ("lane", ["j1", "j2", "j3", "i1", "i2"]),
+                                       ("warp", ["b0"]), ("block", ["i3", "b1"])]}
+    assert O.classify(A2, L_of(blk)) == "CTA"
+
+
+def test_class_configs_2_3():
+    A, B = (L_of(s) for s in W.c2(0))
+    assert O.classify(A, B) == "SHUFFLE"
+    A, B = (L_of(s) for s in W.c3(0))
+    assert O.classify(A, B) == "SMEM"
+
+
+def test_class_config5_device():
+    for p in (1, 2):
+        A, B = (L_of(s) for s in W.c5(p, n=4))
+        assert O.classify(A, B) == "DEVICE"
+
+
+def test_class_config5_p0_noop_and_transpose_cta():
+    A, B = (L_of(s) for s in W.c5(0, n=4))
+    assert O.classify(A, B) == "NOOP"
+    A, B = (L_of(s) for s in W.c5T(0, n=3))
+    assert O.classify(A, B) == "CTA"
+
+
+# ----------------------------------------------------------------------------- shuffle
+
+def test_shuffle_cosets_hold_one_vector_per_lane():
+    """for each i, R(i) ⊕ span(V∪I∪G) contains exactly one vectorised element
+    per thread of A and of B; the rounds cover every register once.  Checked
+    exhaustively (all 2^|R| cosets) on random SHUFFLE-class pairs."""
+    rng = np.random.default_rng(42)
+    out = [("i", 4), ("j", 4)]
+    hw = [("reg", 3), ("lane", 5)]
+    tested = 0
+    for _ in range(400):
+        A = L_of(gen.random_distributed(rng, out, hw))
+        B = L_of(gen.random_distributed(rng, out, hw))
+        if O.classify(A, B) != "SHUFFLE":
+            continue
+        for w in (1, 2, 4):
+            s = O.shuffle_sets(A, B, w)
+            assert s["rounds"] == 1 << ((3 + 5) - len(s["V"]) - len(s["I"]) - len(s["G"]))
+            base = O.span(s["V"] + s["I"] + s["G"])
+            vecspan = O.span(s["V"])
+            Ainv, Binv = O.preimage_min(A), O.preimage_min(B)
+            seen_a = set()
+            for ri in range(s["rounds"]):
+                r = 0
+                for t, c in enumerate(s["R"]):
+                    if (ri >> t) & 1:
+                        r ^= c
+                coset = {r ^ x for x in base}
+                for L, inv, seen in ((A, Ainv, seen_a), (B, Binv, None)):
+                    lanes = {}
+                    for x in coset:
+                        h = int(inv[x])
+                        lane = (h >> 3) & 31
+                        lanes.setdefault(lane, set()).add(x)
+                    assert sorted(lanes) == list(range(32))
+                    for lane, xs in lanes.items():
+                        x0 = min(xs)
+                        assert xs == {x0 ^ v for v in vecspan}   # one vector per lane
+                        if seen is not None:
+                            seen.add(x0)
+            assert len(seen_a) * len(vecspan) == 256
+        tested += 1
+    assert tested >= 20
+
+
+# ----------------------------------------------------------------------------- swizzle
+
+def _fig5():
+    g = load("fig5_swizzle.json")
+    out = [tuple(d) for d in g["out_dims"]]
+    A = L_of({"out": out, "in": [(k, v) for k, v in g["A"].items()]})
+    B = L_of({"out": out, "in": [(k, v) for k, v in g["B"].items()]})
+    return A, B, g
+
+
+def test_fig5_swizzle_reproduces_P426_schedule():
+    """GV5 (P:426 under the G3 reconstruction): Vec=[r0], Bank=[c0], Seg=[c0^c1, r1];
+    the read schedule printed in the paper; no conflicts in reads or writes."""
+    A, B, g = _fig5()
+    sw = O.optimal_swizzle(A, B, g["elem_bytes"], segment_bytes=g["segment_bytes"],
+                           bank_bytes=g["bank_bytes"])
+    flat = lambda name: O.logical_flat(A.out_dims, W.bit_coords(A.out_dims, name))
+    assert sw["Vec"] == [flat("r0")]
+    assert sw["Bank"] == [flat("c0")]
+    assert sw["Seg"] == [flat("c0") ^ flat("c1"), flat("r1")]
+    S = O.smem_layout_from_swizzle(sw, A.out_dims)
+    off = O.preimage_min(S)
+    nbank = g["segment_bytes"] // g["bank_bytes"]
+    for rd in g["reads_P426"]:
+        t = rd["thread"]
+        # element ids of the paper: id = 4r + c
+        elems = []
+        for r0 in (0, 1):
+            h = r0 | (t << 2)
+            x = O.apply(A, h)
+            r, c = O.logical_coords(A.out_dims, x)
+            elems.append(4 * r + c)
+            assert int(off[x]) % nbank == rd["banks"][r0]
+            assert int(off[x]) // nbank == rd["transaction"]  # segment index
+        assert elems == rd["elements"]
+    for L in (A, B):
+        wf, ideal = O.smem_wavefronts(S, L, g["elem_bytes"], sw["Vec"], bank_bytes=g["bank_bytes"],
+                                      n_banks=nbank)
+        assert wf == ideal == 4      # "four transactions without bank conflicts"
+
+
+@pytest.mark.parametrize("cfg", ["c1", "c3", "c3b"])
+def test_swizzle_conflict_free_on_configs(cfg):
+    """Lemma 9.4: the constructed S gives the ideal wavefront count for
+    both the store (A) and the load (B) of configs 1, 3 and 3b."""
+    A, B = {"c1": lambda: (L_of(W.C1_A), L_of(W.C1_B)),
+            "c3": lambda: tuple(L_of(s) for s in W.c3(0)),
+            "c3b": lambda: tuple(L_of(s) for s in W.c3b(0))}[cfg]()
+    w = {"c1": 4, "c3": 2, "c3b": 2}[cfg]
+    sw = O.optimal_swizzle(A, B, w)
+    S = O.smem_layout_from_swizzle(sw, A.out_dims)
+    assert O.is_memory(S) or all(bin(c).count("1") <= 2 for c in S.cols)
+    for L in (A, B):
+        wf, ideal = O.smem_wavefronts(S, L, w, sw["Vec"])
+        assert wf == ideal
+
+
+def test_unswizzled_config3_conflicts():
+    """Sanity of the bank model: a row-major (unswizzled) buffer for config 3 is
+    conflicted on the column-order side (4-way st / 32-way ld)."""
+    A, B = (L_of(s) for s in W.c3(0))
+    row = O.identity_memory(A.out_dims)
+    # 1-element (2-byte) accesses
+    wfA, idA = O.smem_wavefronts(row, A, 2, [])
+    wfB, idB = O.smem_wavefronts(row, B, 2, [])
+    assert wfA == 4 * idA      # 16 lanes at 16 B stride + the i0 lane: 4-way
+    assert wfB == 32 * idB     # lanes run along i (256 B apart): all in one bank
+
+
+def _all_subspaces(d, k):
+    """All k-dim subspaces of F2^d as sorted tuples of their reduced bases."""
+    seen = set()
+    for combo in itertools.combinations(range(1, 1 << d), k):
+        if O.rank(list(combo)) == k:
+            key = tuple(sorted(O.span(list(combo))))
+            if key not in seen:
+                seen.add(key)
+                yield list(combo)
+
+
+def test_lemma95_bruteforce():
+    """Lemma 9.5: largest subspace with trivial intersection with U ∪ V has dim
+    d - max(dim U, dim V); brute force over all subspaces of F2^4."""
+    rng = np.random.default_rng(0)
+    d = 4
+    for _ in range(25):
+        U = [int(x) for x in rng.integers(1, 1 << d, size=int(rng.integers(1, 3)))]
+        V = [int(x) for x in rng.integers(1, 1 << d, size=int(rng.integers(1, 3)))]
+        su, sv = O.span(U), O.span(V)
+        best = 0
+        for k in range(d, 0, -1):
+            if any(not ((O.span(b) - {0}) & (su | sv)) for b in _all_subspaces(d, k)):
+                best = k
+                break
+        assert best == O.lemma95_optimum(U, V, d)
+
+
+def test_swizzle_optimal_exhaustive_toy():
+    """E2 (Lemmas 9.4-9.6): with a toy bank geometry (4 banks of 4 B per segment) and
+    4 lanes, whenever some Seg subspace is conflict-free for both A and B, the
+    paper's construction is conflict-free too; and it is conflict-free exactly when
+    ℓ ≤ d - max(dim U, dim V) with U, V the Vec+Bank-lane spans (Lemma 9.5)."""
+    rng = np.random.default_rng(77)
+    out = [("r", 3), ("c", 2)]
+    hw = [("reg", 3), ("lane", 2)]
+    checked = 0
+    for _ in range(60):
+        A = L_of(gen.random_distributed(rng, out, hw))
+        B = L_of(gen.random_distributed(rng, out, hw))
+        w = 4
+        sw = O.optimal_swizzle(A, B, w, segment_bytes=16, bank_bytes=4)
+        if not sw["Vec"]:
+            continue
+        S = O.smem_layout_from_swizzle(sw, A.out_dims)
+        tot = sum(O.smem_wavefronts(S, L, w, sw["Vec"], n_banks=4)[0] for L in (A, B))
+        ideal = sum(O.smem_wavefronts(S, L, w, sw["Vec"], n_banks=4)[1] for L in (A, B))
+        # brute force over all Seg subspaces complementing Vec
+        d = 5
+        best = None
+        for seg in _all_subspaces(d, sw["ell"]) if sw["ell"] > 0 else [[]]:
+            if O.rank(sw["Vec"] + seg) != len(sw["Vec"]) + len(seg):
+                continue
+            bank = O.complete_basis(sw["Vec"] + seg, d)
+            S2 = O.smem_layout_from_swizzle({"Vec": sw["Vec"], "Bank": bank, "Seg": seg}, A.out_dims)
+            t2 = sum(O.smem_wavefronts(S2, L, w, sw["Vec"], n_banks=4)[0] for L in (A, B))
+            best = t2 if best is None else min(best, t2)
+        if best == ideal:
+            assert tot == ideal
+        checked += 1
+    assert checked >= 20
+
+
+# ----------------------------------------------------------------------------- gather / reduce
+
+@pytest.mark.parametrize("family", ["mma", "blocked"])
+def test_gather_is_take_along_axis(family):
+    """O10 vs numpy.take_along_axis on the tile-reshaped tensor."""
+    rng = np.random.default_rng(1004)
+    L = L_of(W.c4("gather", family, n_i=8, n_j=7))     # [256, 128] with [128, 32] tiles
+    n = 1 << L.d_in
+    T = gen.random_bits(rng, n, 4)
+    Ti = rng.integers(0, 32, size=n).astype(np.int32)
+    out = O.gather(L, 1, O.pack(L, T), O.pack(L, Ti))
+    ref = np.take_along_axis(T.reshape(256, 4, 32), Ti.reshape(256, 4, 32).astype(np.int64), axis=2)
+    assert np.array_equal(out, O.pack(L, ref.reshape(-1)))
+
+
+@pytest.mark.parametrize("family", ["mma", "blocked"])
+def test_reduce_fp64_and_fixed_order(family):
+    """O11: fp64 reference equals numpy's sum over [128,128] tiles; the fixed-order
+    fp32 replica is within 1e-6 relative (U[0,1) inputs, no cancellation)."""
+    rng = np.random.default_rng(1005)
+    L = L_of(W.c4("reduce", family, n_i=8, n_j=8))     # [256, 256] with [128,128] tiles
+    n = 1 << L.d_in
+    T = rng.random(n, dtype=np.float32)
+    src = O.pack(L, T)
+    ref = O.reduce_ref_fp64(L, 1, src)
+    lib = T.astype(np.float64).reshape(256, 2, 128).sum(axis=2).reshape(-1)
+    assert np.allclose(ref, lib, rtol=1e-12)
+    rep = O.reduce_fixed_order_fp32(L, 1, src)
+    assert np.all(np.abs(rep - ref) <= 1e-6 * np.abs(ref))
+
+
+def test_reduce_broadcast_dedup():
+    """duplicated (zero-column) data is reduced once, not twice."""
+    L = O.blocked([8, 16], [1, 2], [4, 8], [4, 1], [1, 0])      # 32 rows of slots for 8 rows: i-broadcast
+    L = O.Layout(L.in_dims, L.out_dims, L.bases)
+    assert any(c == 0 for c in L.cols)
+    rng = np.random.default_rng(3)
+    T = rng.random(128, dtype=np.float32)
+    src = O.pack(L, T)
+    rep = O.reduce_fixed_order_fp32(L, 1, src)
+    ref = T.astype(np.float64).reshape(8, 16).sum(axis=1)
+    assert np.allclose(rep, ref, rtol=1e-6)
+
+
+def test_distributed_rank_slices_concatenate():
+    """O12: the per-rank slices of B, for config-5 layouts at small size, are the
+    column shards of the logical tensor (an all_to_all of row shards)."""
+    rng = np.random.default_rng(1006)
+    n = 4
+    for p in (1, 2):
+        A, B = (L_of(s) for s in W.c5(p, n=n))
+        T = gen.random_bits(rng, 1 << (2 * n), 2)
+        P = 1 << p
+        M = T.reshape(1 << n, 1 << n)
+        for r in range(P):
+            got = O.convert_distributed_rank(A, B, T, r)
+            cols = M[:, r * (16 // P):(r + 1) * (16 // P)]
+            assert np.array_equal(got, cols.reshape(-1))
