@@ -1,0 +1,237 @@
+/*
+ * ll.h — C ABI of the B200-native linear-layout conversion library (libll.so).
+ *
+ * The method is "Linear Layouts: Robust Code Generation of Efficient Tensor
+ * Computation Using F2" (ASPLOS '26).  Citations "P:L" are line numbers of the
+ * paper text, with the section / definition given.
+ *
+ * CONVENTIONS
+ *  - A layout is a linear map over F2 from labelled input (hardware) bits to
+ *    labelled output (logical) bits (Def 4.1).  Input dims are named
+ *    "reg", "lane", "warp", "block", "dev" (distributed layouts, Def 4.10) or
+ *    "offset", "dev" (memory layouts, Def 4.14); output dims carry any names.
+ *  - Hardware flat index h: the input dims' bits concatenated in declaration
+ *    order, the FIRST declared dim least significant (P:138, P:148 footnote).
+ *  - Logical flat index: row-major over the output dims in declaration order,
+ *    the LAST dim fastest ("j is the fastest moving dimension").
+ *  - A buffer "packed in layout L" is a dense array of 2^{d_in} elements of
+ *    elem_bytes each; position h holds the logical element L(h).  A "dev" input
+ *    dim must be declared last; rank r holds the slice dev = r.
+ *  - Conversion is the pull form of B^{-1} ∘ A: for every dst index
+ *    h, dst[h] = src[h'] for a preimage h' with A(h') = B(h).  The planner picks
+ *    h' = Q(h), Q = A^+ ∘ B with the slack-zero right inverse and
+ *    the identity on dims where A and B agree.
+ *  - Precondition: src is A-consistent (A(h1) = A(h2) ⇒ equal elements); this
+ *    always holds for data written through a layout.
+ *
+ * OWNERSHIP AND ERRORS
+ *  - Handles (ll_layout, ll_plan, ll_comm) are created by the *_create / ll_plan_*
+ *    calls and freed by the matching *_destroy.  Layouts and plans are immutable;
+ *    a plan copies what it needs, so layouts may be destroyed after planning.
+ *  - Device pointers are caller-owned (e.g. torch tensors), must be 16-byte
+ *    aligned and stay alive until the stream work completes.
+ *  - Every call returns an ll_status; nothing throws across the ABI;
+ *    ll_last_error() returns a thread-local detail string.
+ *  - ll_convert / ll_gather / ll_reduce are asynchronous on `stream`, never
+ *    allocate device memory and never synchronise; asynchronous faults surface
+ *    at the caller's synchronisation as CUDA errors.  There is no CPU fallback:
+ *    the device entry points return LL_ERR_CUDA when no usable GPU is present.
+ */
+#ifndef LL_H_
+#define LL_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  LL_OK = 0,
+  LL_ERR_INVALID_ARG = 1,
+  LL_ERR_DIM_MISMATCH = 2,
+  LL_ERR_NOT_SURJECTIVE = 3,
+  LL_ERR_NOT_INVERTIBLE = 4,
+  LL_ERR_NOT_DIVISIBLE = 5,
+  LL_ERR_UNSUPPORTED = 6,
+  LL_ERR_ALIAS = 7,
+  LL_ERR_MISALIGNED = 8,
+  LL_ERR_CUDA = 9,
+  LL_ERR_NVRTC = 10,
+  LL_ERR_NCCL = 11,
+  LL_ERR_OOM = 12
+} ll_status;
+
+/* The paper's conversion classes (P:364-373 and the smem fallback P:391),
+ * extended with the cross-CTA and cross-GPU levels of the north star. */
+typedef enum {
+  LL_CLASS_NOOP = 0,    /* A(h) = B(h) for all h ("equivalent layouts")   */
+  LL_CLASS_REGPERM = 1, /* (B^{-1}∘A)_Reg is a register permutation  */
+  LL_CLASS_SHUFFLE = 2, /* warp part is the identity: warp shuffles  */
+  LL_CLASS_SMEM = 3,    /* shared-memory round trip with optimal swizzle */
+  LL_CLASS_CTA = 4,     /* mixes block (or memory-offset) bits                   */
+  LL_CLASS_DEVICE = 5   /* mixes device bits: pack -> all-to-all -> unpack       */
+} ll_class;
+
+typedef struct ll_layout ll_layout;
+typedef struct ll_plan ll_plan;
+typedef struct ll_comm ll_comm;
+
+/* A labelled dimension: name and log2 of its size. */
+typedef struct {
+  const char* name;
+  int log2_size;
+} ll_dim;
+
+typedef struct {
+  int force_class;      /* -1 = auto; else an ll_class to execute (SHUFFLE/SMEM) */
+  int max_vec_bytes;    /* global-memory vector bound, default 16    */
+  int sigma;            /* 0 = coalesced HBM access (default), 1 = faithful      */
+  int tile_bytes;       /* target CTA tile bytes when folding/choosing tiles (0 = default) */
+  int thread_bytes;     /* target bytes per thread (0 = default)                 */
+  int generic;          /* 1 = force the runtime-generic kernel                   */
+  ll_comm* comm;        /* required for DEVICE plans                              */
+} ll_plan_opts;
+
+/* Fill *opts with defaults (force_class = -1, max_vec_bytes = 16, ...). */
+void ll_plan_opts_default(ll_plan_opts* opts);
+
+/* ---------------------------------------------------------------- layouts --
+ * ll_layout_create (row a1; Def 4.1, matrix form P:140-148).
+ *   in[n_in], out[n_out]: dims (names, log2 sizes); in-dim names must be unique.
+ *   bases: Σ_i in[i].log2_size rows × n_out int64 coordinates; row k is the
+ *          output coordinate hit by input bit k (hardware flat order).  Each
+ *          coordinate must be < 2^{out log2_size}.  Copied; caller keeps ownership.
+ *   *L: new handle.  Errors: LL_ERR_INVALID_ARG (bad sizes/names, > 64 bits).   */
+ll_status ll_layout_create(const ll_dim* in, int n_in, const ll_dim* out, int n_out,
+                           const int64_t* bases, ll_layout** L);
+void ll_layout_destroy(ll_layout* L);
+
+/* Shape queries: numbers of dims / total bits, and a dim's name and log2 size. */
+ll_status ll_layout_info(const ll_layout* L, int* n_in, int* n_out, int* d_in, int* d_out);
+ll_status ll_layout_dim(const ll_layout* L, int is_out, int index, const char** name, int* log2_size);
+/* bases: d_in × n_out int64 (same format as ll_layout_create). */
+ll_status ll_layout_bases(const ll_layout* L, int64_t* bases);
+
+/* Evaluate L on one hardware coordinate tuple: XOR of the columns of the set bits
+ * (P:136-148).  in_coords[n_in] -> out_coords[n_out]. */
+ll_status ll_layout_apply(const ll_layout* L, const int64_t* in_coords, int64_t* out_coords);
+
+/* Predicates: surjective, injective (rank), distributed (Def 4.10),
+ * memory (Def 4.14).  Any output pointer may be NULL. */
+ll_status ll_layout_props(const ll_layout* L, int* surjective, int* injective,
+                          int* distributed, int* memory);
+
+/* Composition outer∘inner (Def 4.2): requires inner's output dims to
+ * equal outer's input dims (names and sizes, same order); else DIM_MISMATCH. */
+ll_status ll_compose(const ll_layout* outer, const ll_layout* inner, ll_layout** out);
+
+/* Right inverse (Def 4.5): Gaussian elimination over F2, free
+ * variables 0, pivots in ascending column order; equals the min-index
+ * preimage.  The result maps L's output dims to L's input dims.  Exact inverse
+ * when L is bijective.  Errors: LL_ERR_NOT_SURJECTIVE. */
+ll_status ll_invert(const ll_layout* L, ll_layout** out);
+
+/* Product L1 × L2 (Def 4.3), label-wise: same-named dims concatenate
+ * with L1's bits low; L2's images are shifted above L1's range. */
+ll_status ll_product(const ll_layout* L1, const ll_layout* L2, ll_layout** out);
+
+/* Left division M /_l M1 (Def 4.4): M2 such that M = M1 × M2
+ * label-wise, or LL_ERR_NOT_DIVISIBLE.  Used for SIMD tiles (Thm 5.1). */
+ll_status ll_left_divide(const ll_layout* M, const ll_layout* M1, ll_layout** M2);
+
+/* Basis of ker(L) as hardware flat indices (broadcast directions; zero columns of
+ * distributed layouts).  hw_vectors has room for d_in entries;
+ * *n receives the count. */
+ll_status ll_kernel_basis(const ll_layout* L, int64_t* hw_vectors, int* n);
+
+/* ---------------------------------------------------------------- conversion --
+ * ll_plan_convert (rows a2-a4, a6-a9).  Host only.
+ *   A, B: same output dims; A surjective.  elem_bytes in {1, 2, 4, 8}.
+ *   opts: NULL for defaults.  Computes Q = A^+ ∘ B, the paper's class (lowest
+ *   hardware level Q must cross), and an execution plan: NOOP (memcpy), a
+ *   specialised sm_100a tile kernel (register permutation / warp shuffles /
+ *   swizzled smem round trip / cross-CTA tiled exchange), the runtime-generic
+ *   kernel (broadcast and non-permutation maps), or DEVICE (pack, all-to-all over
+ *   NVLink, unpack; needs opts->comm).  The specialised kernel is compiled with
+ *   NVRTC for sm_100a on first use (cached on disk).
+ *   Errors: DIM_MISMATCH, NOT_SURJECTIVE, INVALID_ARG, UNSUPPORTED. */
+ll_status ll_plan_convert(const ll_layout* A, const ll_layout* B, int elem_bytes,
+                          const ll_plan_opts* opts, ll_plan** plan);
+ll_status ll_plan_class(const ll_plan* plan, ll_class* cls);
+/* Workspace needed by ll_convert (> 0 only for DEVICE plans). */
+ll_status ll_plan_workspace_bytes(const ll_plan* plan, size_t* bytes);
+/* JSON description: class, executed exchange, V/I/E/F/G/R, swizzle columns,
+ * rounds, predicted wavefronts, launch geometry.  Truncates to cap bytes. */
+ll_status ll_plan_describe(const ll_plan* plan, char* json, size_t cap);
+/* Specialised CUDA source of the plan's kernel (empty if none). */
+ll_status ll_plan_source(const ll_plan* plan, char* buf, size_t cap, size_t* needed);
+/* Compile/load the plan's kernel now (otherwise done by the first launch). */
+ll_status ll_plan_prepare(ll_plan* plan);
+void ll_plan_destroy(ll_plan* plan);
+
+/* ll_convert (rows a5-a10): dst[h] = src[Q(h)] on `stream` (a cudaStream_t).
+ *   src: device buffer packed in A (2^{A.d_in} elements, local slice for dev);
+ *   dst: device buffer packed in B; must not alias src unless the plan is NOOP
+ *   (LL_ERR_ALIAS); 16-byte aligned (LL_ERR_MISALIGNED).
+ *   workspace: NULL unless ll_plan_workspace_bytes > 0.
+ *   DEVICE plans are collective: every rank calls with the same plan. */
+ll_status ll_convert(const void* src, void* dst, void* workspace, const ll_plan* plan,
+                     void* stream);
+
+/* ---------------------------------------------------------------- gather --
+ * ll_plan_gather (row a11; §5.5).  src, idx and dst share layout L
+ * (P:430).  Along logical dim `axis`, K = 2^(non-block axis bits of L); these
+ * must be the low bits of the axis coordinate.  out[x] = src[x with the axis
+ * coordinate's low bits replaced by idx[x] & (K-1)] (take_along_axis inside each
+ * tile; out-of-range indices are masked).  Warp shuffles are used
+ * when L_Wrp^axis = 0. */
+ll_status ll_plan_gather(const ll_layout* L, int axis, int elem_bytes,
+                         const ll_plan_opts* opts, ll_plan** plan);
+/* src, dst: packed in L; idx: int32 packed in L. */
+ll_status ll_gather(const void* src, const int32_t* idx, void* dst, const ll_plan* plan,
+                    void* stream);
+
+/* ---------------------------------------------------------------- reduce --
+ * ll_plan_reduce (row a12; Table 4).  Sum (fp32) along
+ * logical dim `axis` over the non-block axis bits of L (within each CTA tile):
+ * an in-register tree over Reg axis bits, shfl.bfly over Lane axis bits and smem
+ * over Warp axis bits, in that fixed order (reg, lane, warp ascending);
+ * broadcast (zero-column) bits are skipped, each output is written once. */
+ll_status ll_plan_reduce(const ll_layout* L, int axis, const ll_plan_opts* opts, ll_plan** plan);
+/* Number of output elements. */
+ll_status ll_plan_reduce_out_elems(const ll_plan* plan, size_t* n);
+/* src: fp32 packed in L; dst: fp32 logical row-major with the axis replaced by
+ * its block part (one write per element). */
+ll_status ll_reduce(const float* src, float* dst, const ll_plan* plan, void* stream);
+
+/* ---------------------------------------------------------------- comm --
+ * NCCL communicator for DEVICE plans: nccl_unique_id is the 128-byte
+ * ncclUniqueId produced by rank 0 and broadcast by the caller (e.g. over a torch
+ * process group).  NCCL is loaded with dlopen on first use (LL_ERR_NCCL if
+ * absent). */
+ll_status ll_comm_create(const void* nccl_unique_id, int nranks, int rank, ll_comm** comm);
+ll_status ll_comm_get_unique_id(void* nccl_unique_id /* 128 bytes */);
+void ll_comm_destroy(ll_comm* comm);
+
+/* ---------------------------------------------------------------- test hooks --
+ * ll_plan_simulate: host emulation of a specialised tile plan's schedule (the
+ * same tables the kernel is specialised with: load addresses, pre/post register
+ * networks, shuffle rounds and source lanes, smem offsets).  For validating the
+ * planner on machines without a GPU; never used by ll_convert.  src/dst are HOST
+ * buffers.  LL_ERR_UNSUPPORTED for non-tile plans. */
+ll_status ll_plan_simulate(const ll_plan* plan, const void* src, void* dst);
+
+/* ll_jit_precompile: NVRTC-compile the plan's kernel into the on-disk cubin cache
+ * without loading it (works without a GPU; used by the build to pre-populate the
+ * cache for the benchmark configurations). */
+ll_status ll_jit_precompile(const ll_plan* plan);
+
+const char* ll_last_error(void);
+const char* ll_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* LL_H_ */

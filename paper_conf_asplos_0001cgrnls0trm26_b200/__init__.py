@@ -1,0 +1,366 @@
+"""Python binding of libll.so — the B200-native linear-layout conversion library.
+
+Argument marshalling only: every step of the hot path runs in libll.so (host
+planner in C++, sm_100a kernels specialised with NVRTC).  PyTorch is used for
+device memory and streams.  There is no CPU fallback: if libll.so is missing the
+import fails; on a machine without a GPU the device calls raise LLError(LL_ERR_CUDA).
+
+Names follow the C ABI of include/ll.h (ll_layout_create, ll_compose, ll_invert,
+ll_plan_convert, ll_convert, ll_plan_gather, ll_gather, ll_plan_reduce, ll_reduce).
+"""
+from __future__ import annotations
+
+import ctypes as C
+import json
+import os
+from typing import Dict, List, Optional, Sequence, Tuple
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_LIB_PATH = os.path.join(_HERE, "libll.so")
+
+if not os.path.exists(_LIB_PATH):
+    raise ImportError(f"{_LIB_PATH} is missing: build it with `python -c 'import __graft_entry__ as g; g.build()'`")
+_lib = C.CDLL(_LIB_PATH)
+
+STATUS = ["OK", "INVALID_ARG", "DIM_MISMATCH", "NOT_SURJECTIVE", "NOT_INVERTIBLE", "NOT_DIVISIBLE",
+          "UNSUPPORTED", "ALIAS", "MISALIGNED", "CUDA", "NVRTC", "NCCL", "OOM"]
+CLASSES = ["NOOP", "REGPERM", "SHUFFLE", "SMEM", "CTA", "DEVICE"]
+
+
+class LLError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"LL_ERR_{STATUS[status] if status < len(STATUS) else status}: {msg}")
+        self.status = status
+
+
+class _Dim(C.Structure):
+    _fields_ = [("name", C.c_char_p), ("log2_size", C.c_int)]
+
+
+class _Opts(C.Structure):
+    _fields_ = [("force_class", C.c_int), ("max_vec_bytes", C.c_int), ("sigma", C.c_int),
+                ("tile_bytes", C.c_int), ("thread_bytes", C.c_int), ("generic", C.c_int),
+                ("comm", C.c_void_p)]
+
+
+_P = C.c_void_p
+_PP = C.POINTER(C.c_void_p)
+_sig = {
+    "ll_layout_create": [C.POINTER(_Dim), C.c_int, C.POINTER(_Dim), C.c_int, C.POINTER(C.c_int64), _PP],
+    "ll_layout_info": [_P, C.POINTER(C.c_int)] * 1 + [C.POINTER(C.c_int)] * 3,
+    "ll_layout_dim": [_P, C.c_int, C.c_int, C.POINTER(C.c_char_p), C.POINTER(C.c_int)],
+    "ll_layout_bases": [_P, C.POINTER(C.c_int64)],
+    "ll_layout_apply": [_P, C.POINTER(C.c_int64), C.POINTER(C.c_int64)],
+    "ll_layout_props": [_P] + [C.POINTER(C.c_int)] * 4,
+    "ll_compose": [_P, _P, _PP],
+    "ll_invert": [_P, _PP],
+    "ll_product": [_P, _P, _PP],
+    "ll_left_divide": [_P, _P, _PP],
+    "ll_kernel_basis": [_P, C.POINTER(C.c_int64), C.POINTER(C.c_int)],
+    "ll_plan_convert": [_P, _P, C.c_int, C.POINTER(_Opts), _PP],
+    "ll_plan_class": [_P, C.POINTER(C.c_int)],
+    "ll_plan_workspace_bytes": [_P, C.POINTER(C.c_size_t)],
+    "ll_plan_describe": [_P, C.c_char_p, C.c_size_t],
+    "ll_plan_source": [_P, C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t)],
+    "ll_plan_prepare": [_P],
+    "ll_jit_precompile": [_P],
+    "ll_convert": [_P, _P, _P, _P, _P],
+    "ll_plan_gather": [_P, C.c_int, C.c_int, C.POINTER(_Opts), _PP],
+    "ll_gather": [_P, _P, _P, _P, _P],
+    "ll_plan_reduce": [_P, C.c_int, C.POINTER(_Opts), _PP],
+    "ll_plan_reduce_out_elems": [_P, C.POINTER(C.c_size_t)],
+    "ll_reduce": [_P, _P, _P, _P],
+    "ll_plan_simulate": [_P, _P, _P],
+    "ll_comm_create": [_P, C.c_int, C.c_int, _PP],
+    "ll_comm_get_unique_id": [_P],
+}
+for _name, _args in _sig.items():
+    _f = getattr(_lib, _name)
+    _f.argtypes = _args
+    _f.restype = C.c_int
+_lib.ll_layout_destroy.argtypes = [_P]
+_lib.ll_layout_destroy.restype = None
+_lib.ll_plan_destroy.argtypes = [_P]
+_lib.ll_plan_destroy.restype = None
+_lib.ll_comm_destroy.argtypes = [_P]
+_lib.ll_comm_destroy.restype = None
+_lib.ll_last_error.restype = C.c_char_p
+_lib.ll_version.restype = C.c_char_p
+_lib.ll_plan_opts_default.argtypes = [C.POINTER(_Opts)]
+_lib.ll_plan_opts_default.restype = None
+
+EXPORTED = sorted(list(_sig) + ["ll_layout_destroy", "ll_plan_destroy", "ll_comm_destroy", "ll_last_error",
+                                "ll_version", "ll_plan_opts_default"])
+
+
+def _check(st: int):
+    if st != 0:
+        raise LLError(st, _lib.ll_last_error().decode(errors="replace"))
+
+
+def library_path() -> str:
+    return _LIB_PATH
+
+
+def version() -> str:
+    return _lib.ll_version().decode()
+
+
+def _opts(force_class=None, max_vec_bytes=16, sigma=0, tile_bytes=0, thread_bytes=0, generic=False, comm=None):
+    o = _Opts()
+    _lib.ll_plan_opts_default(C.byref(o))
+    if force_class is not None:
+        o.force_class = CLASSES.index(force_class) if isinstance(force_class, str) else int(force_class)
+    o.max_vec_bytes = max_vec_bytes
+    o.sigma = {"coalesced": 0, "faithful": 1}.get(sigma, sigma) if isinstance(sigma, str) else int(sigma)
+    o.tile_bytes = tile_bytes
+    o.thread_bytes = thread_bytes
+    o.generic = int(bool(generic))
+    o.comm = comm.handle if comm is not None else None
+    return o
+
+
+class Layout:
+    """ll_layout: a linear layout between labelled F2 spaces (Def 4.1)."""
+
+    def __init__(self, in_dims: Sequence[Tuple[str, int]], out_dims: Sequence[Tuple[str, int]],
+                 bases: Dict[str, Sequence[Sequence[int]]] = None, _handle=None):
+        if _handle is not None:
+            self.handle = _handle
+            return
+        ins = (_Dim * max(1, len(in_dims)))(*[_Dim(n.encode(), b) for n, b in in_dims])
+        outs = (_Dim * max(1, len(out_dims)))(*[_Dim(n.encode(), b) for n, b in out_dims])
+        rows = []
+        for n, b in in_dims:
+            vecs = list((bases or {}).get(n, []))
+            if len(vecs) != b:
+                raise ValueError(f"dim {n}: {len(vecs)} basis vectors for {b} bits")
+            rows += [list(v) for v in vecs]
+        arr = (C.c_int64 * max(1, len(rows) * len(out_dims)))(*[c for r in rows for c in r])
+        h = C.c_void_p()
+        _check(_lib.ll_layout_create(ins, len(in_dims), outs, len(out_dims), arr, C.byref(h)))
+        self.handle = h
+
+    @classmethod
+    def from_spec(cls, spec) -> "Layout":
+        """From a literal spec {"out": [(name, bits)], "in": [(dim, [logical bit names])]}."""
+        from workloads.configs import spec_to_bases
+        in_dims, out_dims, bases = spec_to_bases(spec)
+        return cls(in_dims, out_dims, bases)
+
+    def __del__(self):
+        h = getattr(self, "handle", None)
+        if h:
+            _lib.ll_layout_destroy(h)
+            self.handle = None
+
+    def _info(self):
+        a, b, c, d = C.c_int(), C.c_int(), C.c_int(), C.c_int()
+        _check(_lib.ll_layout_info(self.handle, C.byref(a), C.byref(b), C.byref(c), C.byref(d)))
+        return a.value, b.value, c.value, d.value
+
+    def dims(self, out: bool):
+        n_in, n_out, _, _ = self._info()
+        res = []
+        for i in range(n_out if out else n_in):
+            nm, sz = C.c_char_p(), C.c_int()
+            _check(_lib.ll_layout_dim(self.handle, int(out), i, C.byref(nm), C.byref(sz)))
+            res.append((nm.value.decode(), sz.value))
+        return res
+
+    @property
+    def in_dims(self):
+        return self.dims(False)
+
+    @property
+    def out_dims(self):
+        return self.dims(True)
+
+    @property
+    def d_in(self):
+        return self._info()[2]
+
+    @property
+    def d_out(self):
+        return self._info()[3]
+
+    def bases(self) -> List[Tuple[int, ...]]:
+        _, n_out, d_in, _ = self._info()
+        arr = (C.c_int64 * max(1, d_in * n_out))()
+        _check(_lib.ll_layout_bases(self.handle, arr))
+        return [tuple(arr[k * n_out:(k + 1) * n_out]) for k in range(d_in)]
+
+    def cols(self) -> List[int]:
+        """Logical flat index (row-major, last dim fastest) per input bit."""
+        out = self.out_dims
+        res = []
+        for v in self.bases():
+            f = 0
+            for (n, b), c in zip(out, v):
+                f = (f << b) | c
+            res.append(f)
+        return res
+
+    def apply(self, in_coords: Sequence[int]) -> Tuple[int, ...]:
+        n_in, n_out, _, _ = self._info()
+        a = (C.c_int64 * max(1, n_in))(*in_coords)
+        b = (C.c_int64 * max(1, n_out))()
+        _check(_lib.ll_layout_apply(self.handle, a, b))
+        return tuple(b[:n_out])
+
+    def props(self) -> Dict[str, bool]:
+        v = [C.c_int() for _ in range(4)]
+        _check(_lib.ll_layout_props(self.handle, *[C.byref(x) for x in v]))
+        return dict(zip(["surjective", "injective", "distributed", "memory"], [bool(x.value) for x in v]))
+
+    def compose(self, inner: "Layout") -> "Layout":
+        """self ∘ inner (Def 4.2)."""
+        h = C.c_void_p()
+        _check(_lib.ll_compose(self.handle, inner.handle, C.byref(h)))
+        return Layout(None, None, _handle=h)
+
+    def invert(self) -> "Layout":
+        h = C.c_void_p()
+        _check(_lib.ll_invert(self.handle, C.byref(h)))
+        return Layout(None, None, _handle=h)
+
+    def product(self, other: "Layout") -> "Layout":
+        h = C.c_void_p()
+        _check(_lib.ll_product(self.handle, other.handle, C.byref(h)))
+        return Layout(None, None, _handle=h)
+
+    def left_divide(self, M1: "Layout") -> "Layout":
+        h = C.c_void_p()
+        _check(_lib.ll_left_divide(self.handle, M1.handle, C.byref(h)))
+        return Layout(None, None, _handle=h)
+
+    def kernel_basis(self) -> List[int]:
+        arr = (C.c_int64 * 64)()
+        n = C.c_int()
+        _check(_lib.ll_kernel_basis(self.handle, arr, C.byref(n)))
+        return list(arr[:n.value])
+
+
+# ---- ABI-named functions -------------------------------------------------------------
+def ll_layout_create(in_dims, out_dims, bases) -> Layout:
+    return Layout(in_dims, out_dims, bases)
+
+
+def ll_compose(outer: Layout, inner: Layout) -> Layout:
+    return outer.compose(inner)
+
+
+def ll_invert(L: Layout) -> Layout:
+    return L.invert()
+
+
+def _stream_ptr(stream):
+    if stream is None:
+        import torch
+        return C.c_void_p(torch.cuda.current_stream().cuda_stream)
+    if isinstance(stream, int):
+        return C.c_void_p(stream)
+    return C.c_void_p(stream.cuda_stream)
+
+
+def _ptr(t):
+    if t is None:
+        return None
+    if hasattr(t, "data_ptr"):
+        if not t.is_cuda:
+            raise LLError(1, "device entry points take CUDA tensors")
+        return C.c_void_p(t.data_ptr())
+    return C.c_void_p(int(t))
+
+
+class Plan:
+    """ll_plan: a conversion (ll_plan_convert), gather or reduce plan."""
+
+    def __init__(self, handle, kind: str):
+        self.handle = handle
+        self.kind = kind
+
+    def __del__(self):
+        h = getattr(self, "handle", None)
+        if h:
+            _lib.ll_plan_destroy(h)
+            self.handle = None
+
+    @property
+    def cls(self) -> str:
+        c = C.c_int()
+        _check(_lib.ll_plan_class(self.handle, C.byref(c)))
+        return CLASSES[c.value]
+
+    def describe(self) -> dict:
+        buf = C.create_string_buffer(1 << 20)
+        _check(_lib.ll_plan_describe(self.handle, buf, len(buf)))
+        return json.loads(buf.value.decode())
+
+    def source(self) -> str:
+        n = C.c_size_t()
+        _check(_lib.ll_plan_source(self.handle, None, 0, C.byref(n)))
+        buf = C.create_string_buffer(n.value + 1)
+        _check(_lib.ll_plan_source(self.handle, buf, len(buf), C.byref(n)))
+        return buf.value.decode()
+
+    def workspace_bytes(self) -> int:
+        n = C.c_size_t()
+        _check(_lib.ll_plan_workspace_bytes(self.handle, C.byref(n)))
+        return n.value
+
+    def prepare(self):
+        _check(_lib.ll_plan_prepare(self.handle))
+        return self
+
+    def precompile(self):
+        _check(_lib.ll_jit_precompile(self.handle))
+        return self
+
+    def out_elems(self) -> int:
+        n = C.c_size_t()
+        _check(_lib.ll_plan_reduce_out_elems(self.handle, C.byref(n)))
+        return n.value
+
+    def simulate(self, src: np.ndarray, dst_elems: int) -> np.ndarray:
+        """Host emulation of the plan's kernel schedule (test hook, no GPU)."""
+        src = np.ascontiguousarray(src)
+        dst = np.zeros(dst_elems, dtype=src.dtype)
+        _check(_lib.ll_plan_simulate(self.handle, src.ctypes.data_as(C.c_void_p), dst.ctypes.data_as(C.c_void_p)))
+        return dst
+
+
+def ll_plan_convert(A: Layout, B: Layout, elem_bytes: int, **opts) -> Plan:
+    h = C.c_void_p()
+    o = _opts(**opts)
+    _check(_lib.ll_plan_convert(A.handle, B.handle, int(elem_bytes), C.byref(o), C.byref(h)))
+    return Plan(h, "convert")
+
+
+def ll_convert(src, dst, plan: Plan, stream=None, workspace=None):
+    """dst <- convert(src) on `stream` (torch CUDA tensors or raw device pointers)."""
+    _check(_lib.ll_convert(_ptr(src), _ptr(dst), _ptr(workspace), plan.handle, _stream_ptr(stream)))
+
+
+def ll_plan_gather(L: Layout, axis: int, elem_bytes: int, **opts) -> Plan:
+    h = C.c_void_p()
+    o = _opts(**opts)
+    _check(_lib.ll_plan_gather(L.handle, int(axis), int(elem_bytes), C.byref(o), C.byref(h)))
+    return Plan(h, "gather")
+
+
+def ll_gather(src, idx, dst, plan: Plan, stream=None):
+    _check(_lib.ll_gather(_ptr(src), _ptr(idx), _ptr(dst), plan.handle, _stream_ptr(stream)))
+
+
+def ll_plan_reduce(L: Layout, axis: int, **opts) -> Plan:
+    h = C.c_void_p()
+    o = _opts(**opts)
+    _check(_lib.ll_plan_reduce(L.handle, int(axis), C.byref(o), C.byref(h)))
+    return Plan(h, "reduce")
+
+
+def ll_reduce(src, dst, plan: Plan, stream=None):
+    _check(_lib.ll_reduce(_ptr(src), _ptr(dst), plan.handle, _stream_ptr(stream)))

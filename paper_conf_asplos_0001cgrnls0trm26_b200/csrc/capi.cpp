@@ -1,0 +1,483 @@
+// The C ABI of include/ll.h.  Every entry point converts internal errors into an
+// ll_status and a thread-local message (nothing throws across the ABI).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstring>
+#include <sstream>
+
+#include "ll_internal.hpp"
+
+namespace ll {
+const std::string& last_error_ref();
+std::string jit_precompile(const std::string& plan_src, const char* name);
+int launch_generic(const void* src, void* dst, const unsigned long long* cols, int nbits, unsigned long long nelem,
+                   int w, cudaStream_t stream, int sms);
+ll_status device_convert(const ConvPlan& P, const void* src, void* dst, void* ws, cudaStream_t st);
+void plan_device(ConvPlan& P, const ll_plan_opts* opts);
+}  // namespace ll
+
+using namespace ll;
+
+#define LL_TRY try {
+#define LL_CATCH                                                  \
+  }                                                               \
+  catch (const ll::Error& e) {                                    \
+    set_last_error(e.what());                                     \
+    return e.st;                                                  \
+  }                                                               \
+  catch (const std::bad_alloc&) {                                 \
+    set_last_error("out of host memory");                         \
+    return LL_ERR_OOM;                                            \
+  }                                                               \
+  catch (const std::exception& e) {                               \
+    set_last_error(e.what());                                     \
+    return LL_ERR_INVALID_ARG;                                    \
+  }                                                               \
+  return LL_OK;
+
+namespace {
+
+int num_sms() {
+  static int sms = -1;
+  if (sms < 0) {
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess)
+      sms = 148;
+  }
+  return sms;
+}
+
+void check_cuda(cudaError_t e, const char* what) {
+  if (e != cudaSuccess) fail(LL_ERR_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
+}
+
+// 8-byte elements are converted as pairs of 4-byte atoms: a new lowest input bit
+// maps to a new lowest logical bit (the product of the layout with a 1-bit identity,
+// Def 4.3).  Packed buffers are unchanged byte-wise.
+Layout atomize(const Layout& L) {
+  Layout R;
+  bool done = false;
+  for (auto& d : L.in) {
+    if (!done && (d.name == "reg" || d.name == "offset")) {
+      R.in.push_back({d.name, d.bits + 1});
+      done = true;
+    } else {
+      R.in.push_back(d);
+    }
+  }
+  if (!done) R.in.insert(R.in.begin(), Dim{"reg", 1});
+  R.out = L.out;
+  R.out.push_back({"__atom", 1});
+  // the new bit sits at position 0 of the first reg/offset dim, which is the first
+  // dim in every supported layout; otherwise at the very front
+  int pos = 0;
+  {
+    int p = 0;
+    bool found = false;
+    for (auto& d : L.in) {
+      if (d.name == "reg" || d.name == "offset") { pos = p; found = true; break; }
+      p += d.bits;
+    }
+    if (!found) pos = 0;
+  }
+  for (int k = 0; k < int(L.cols.size()); ++k) {
+    if (k == pos) R.cols.push_back(1);
+    R.cols.push_back(L.cols[k] << 1);
+  }
+  if (pos == int(L.cols.size())) R.cols.push_back(1);
+  return R;
+}
+
+void ensure_tile_kernel(ConvPlan& P) {
+  std::lock_guard<std::mutex> g(P.mu);
+  if (P.kernel) return;
+  if (P.source.empty()) P.source = codegen_tile(P);
+  P.kernel = jit_kernel(P.source, "ll_tile_kernel");
+  if (P.smem_bytes > 48 * 1024)
+    check_cuda(cudaFuncSetAttribute(P.kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, P.smem_bytes),
+               "cudaFuncSetAttribute");
+}
+
+unsigned grid_for(u64 ntiles) {
+  const char* e = getenv("LL_GRID_PER_SM");
+  int per = e ? atoi(e) : 0;
+  u64 cap = per > 0 ? u64(num_sms()) * per : u64(0x7fffffff);
+  u64 g = std::min<u64>(ntiles, cap);
+  return unsigned(std::max<u64>(g, 1));
+}
+
+ll_status convert_impl(const void* src, void* dst, void* ws, ConvPlan& P, cudaStream_t st) {
+  const size_t sbytes = P.src_elems * P.w, dbytes = P.dst_elems * P.w;
+  if ((reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst)) & 15)
+    fail(LL_ERR_MISALIGNED, "src and dst must be 16-byte aligned");
+  if (P.exec == EXEC_NOOP) {
+    if (src != dst) check_cuda(cudaMemcpyAsync(dst, src, dbytes, cudaMemcpyDeviceToDevice, st), "cudaMemcpyAsync");
+    return LL_OK;
+  }
+  const char* s8 = static_cast<const char*>(src);
+  const char* d8 = static_cast<const char*>(dst);
+  if (s8 < d8 + dbytes && d8 < s8 + sbytes) fail(LL_ERR_ALIAS, "src and dst overlap (only NOOP plans may alias)");
+  if (P.exec == EXEC_TILE) {
+    ensure_tile_kernel(P);
+    u64 ntiles = u64(1) << P.tile.grid_dst_bit.size();
+    unsigned long long nt = ntiles;
+    void* args[] = {const_cast<void**>(&src), &dst, &nt};
+    check_cuda(cudaLaunchKernel(P.kernel, dim3(grid_for(ntiles)), dim3(P.tile.threads()), args, size_t(P.smem_bytes), st),
+               "cudaLaunchKernel(ll_tile_kernel)");
+    return LL_OK;
+  }
+  if (P.exec == EXEC_GENERIC) {
+    const int nb = P.B.d_in() - (P.B.in_bits("dev"));
+    std::vector<unsigned long long> cols(P.Q.begin(), P.Q.begin() + nb);
+    int e = launch_generic(src, dst, cols.data(), nb, P.dst_elems, P.w, st, num_sms());
+    check_cuda(cudaError_t(e), "ll_generic_convert_kernel");
+    return LL_OK;
+  }
+  return device_convert(P, src, dst, ws, st);
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* ll_last_error(void) { return ll::last_error_ref().c_str(); }
+const char* ll_version(void) { return "ll-b200 0.1 (sm_100a)"; }
+
+void ll_plan_opts_default(ll_plan_opts* o) {
+  if (!o) return;
+  std::memset(o, 0, sizeof *o);
+  o->force_class = -1;
+  o->max_vec_bytes = 16;
+}
+
+ll_status ll_layout_create(const ll_dim* in, int n_in, const ll_dim* out, int n_out, const int64_t* bases,
+                           ll_layout** Lout) {
+  LL_TRY
+  if (!Lout || (n_in && !in) || (n_out && !out) || n_in < 0 || n_out < 0) fail(LL_ERR_INVALID_ARG, "null argument");
+  auto* h = new ll_layout();
+  std::unique_ptr<ll_layout> guard(h);
+  Layout& L = h->L;
+  int dout = 0;
+  for (int i = 0; i < n_out; ++i) {
+    if (!out[i].name || out[i].log2_size < 0 || out[i].log2_size > 62) fail(LL_ERR_INVALID_ARG, "bad output dim");
+    L.out.push_back({out[i].name, out[i].log2_size});
+    dout += out[i].log2_size;
+  }
+  int din = 0;
+  for (int i = 0; i < n_in; ++i) {
+    if (!in[i].name || in[i].log2_size < 0 || in[i].log2_size > 62) fail(LL_ERR_INVALID_ARG, "bad input dim");
+    for (int j = 0; j < i; ++j)
+      if (!std::strcmp(in[i].name, in[j].name)) fail(LL_ERR_INVALID_ARG, "duplicate input dim name");
+    L.in.push_back({in[i].name, in[i].log2_size});
+    din += in[i].log2_size;
+  }
+  if (din > 62 || dout > 62) fail(LL_ERR_INVALID_ARG, "more than 62 bits");
+  if (din && !bases) fail(LL_ERR_INVALID_ARG, "null bases");
+  for (int k = 0; k < din; ++k) {
+    u64 f = 0;
+    for (int i = 0; i < n_out; ++i) {
+      int64_t c = bases[size_t(k) * n_out + i];
+      if (c < 0 || (u64(c) >> L.out[i].bits)) fail(LL_ERR_INVALID_ARG, "basis coordinate out of range");
+      f = (f << L.out[i].bits) | u64(c);
+    }
+    L.cols.push_back(f);
+  }
+  *Lout = guard.release();
+  LL_CATCH
+}
+
+void ll_layout_destroy(ll_layout* L) { delete L; }
+
+ll_status ll_layout_info(const ll_layout* L, int* n_in, int* n_out, int* d_in, int* d_out) {
+  LL_TRY
+  if (!L) fail(LL_ERR_INVALID_ARG, "null layout");
+  if (n_in) *n_in = int(L->L.in.size());
+  if (n_out) *n_out = int(L->L.out.size());
+  if (d_in) *d_in = L->L.d_in();
+  if (d_out) *d_out = L->L.d_out();
+  LL_CATCH
+}
+
+ll_status ll_layout_dim(const ll_layout* L, int is_out, int index, const char** name, int* log2_size) {
+  LL_TRY
+  if (!L) fail(LL_ERR_INVALID_ARG, "null layout");
+  auto& v = is_out ? L->L.out : L->L.in;
+  if (index < 0 || index >= int(v.size())) fail(LL_ERR_INVALID_ARG, "dim index out of range");
+  if (name) *name = v[index].name.c_str();
+  if (log2_size) *log2_size = v[index].bits;
+  LL_CATCH
+}
+
+ll_status ll_layout_bases(const ll_layout* L, int64_t* bases) {
+  LL_TRY
+  if (!L || !bases) fail(LL_ERR_INVALID_ARG, "null argument");
+  const Layout& l = L->L;
+  for (size_t k = 0; k < l.cols.size(); ++k)
+    for (size_t i = 0; i < l.out.size(); ++i) {
+      int sh = l.out_shift(int(i));
+      bases[k * l.out.size() + i] = int64_t((l.cols[k] >> sh) & ((u64(1) << l.out[i].bits) - 1));
+    }
+  LL_CATCH
+}
+
+ll_status ll_layout_apply(const ll_layout* L, const int64_t* in_coords, int64_t* out_coords) {
+  LL_TRY
+  if (!L || !in_coords || !out_coords) fail(LL_ERR_INVALID_ARG, "null argument");
+  const Layout& l = L->L;
+  u64 h = 0;
+  int s = 0;
+  for (size_t i = 0; i < l.in.size(); ++i) {
+    if (in_coords[i] < 0 || (u64(in_coords[i]) >> l.in[i].bits)) fail(LL_ERR_INVALID_ARG, "coordinate out of range");
+    h |= u64(in_coords[i]) << s;
+    s += l.in[i].bits;
+  }
+  u64 x = l.apply(h);
+  for (size_t i = 0; i < l.out.size(); ++i)
+    out_coords[i] = int64_t((x >> l.out_shift(int(i))) & ((u64(1) << l.out[i].bits) - 1));
+  LL_CATCH
+}
+
+ll_status ll_layout_props(const ll_layout* L, int* surj, int* inj, int* dist, int* mem) {
+  LL_TRY
+  if (!L) fail(LL_ERR_INVALID_ARG, "null layout");
+  if (surj) *surj = L->L.surjective();
+  if (inj) *inj = L->L.injective();
+  if (dist) *dist = L->L.distributed();
+  if (mem) *mem = L->L.memory();
+  LL_CATCH
+}
+
+ll_status ll_compose(const ll_layout* outer, const ll_layout* inner, ll_layout** out) {
+  LL_TRY
+  if (!outer || !inner || !out) fail(LL_ERR_INVALID_ARG, "null argument");
+  auto* h = new ll_layout{compose(outer->L, inner->L)};
+  *out = h;
+  LL_CATCH
+}
+
+ll_status ll_invert(const ll_layout* L, ll_layout** out) {
+  LL_TRY
+  if (!L || !out) fail(LL_ERR_INVALID_ARG, "null argument");
+  *out = new ll_layout{invert(L->L)};
+  LL_CATCH
+}
+
+ll_status ll_product(const ll_layout* L1, const ll_layout* L2, ll_layout** out) {
+  LL_TRY
+  if (!L1 || !L2 || !out) fail(LL_ERR_INVALID_ARG, "null argument");
+  *out = new ll_layout{product(L1->L, L2->L)};
+  LL_CATCH
+}
+
+ll_status ll_left_divide(const ll_layout* M, const ll_layout* M1, ll_layout** M2) {
+  LL_TRY
+  if (!M || !M1 || !M2) fail(LL_ERR_INVALID_ARG, "null argument");
+  *M2 = new ll_layout{left_divide(M->L, M1->L)};
+  LL_CATCH
+}
+
+ll_status ll_kernel_basis(const ll_layout* L, int64_t* v, int* n) {
+  LL_TRY
+  if (!L || !v || !n) fail(LL_ERR_INVALID_ARG, "null argument");
+  auto k = kernel_basis(L->L);
+  for (size_t i = 0; i < k.size(); ++i) v[i] = int64_t(k[i]);
+  *n = int(k.size());
+  LL_CATCH
+}
+
+ll_status ll_plan_convert(const ll_layout* A, const ll_layout* B, int w, const ll_plan_opts* opts, ll_plan** plan) {
+  LL_TRY
+  if (!A || !B || !plan) fail(LL_ERR_INVALID_ARG, "null argument");
+  auto h = std::make_unique<ll_plan>();
+  h->kind = 0;
+  if (w == 8) {
+    // class of the original pair; execution on 4-byte atoms
+    auto P0 = plan_convert(A->L, B->L, 8, opts);
+    ll_class cls = P0->cls;
+    if (P0->exec == EXEC_TILE || P0->exec == EXEC_GENERIC) {
+      auto P = plan_convert(atomize(A->L), atomize(B->L), 4, opts);
+      P->cls = cls;
+      h->conv = std::move(P);
+    } else {
+      h->conv = std::move(P0);
+    }
+  } else {
+    h->conv = plan_convert(A->L, B->L, w, opts);
+  }
+  if (h->conv->exec == EXEC_DEVICE) plan_device(*h->conv, opts);
+  if (h->conv->exec == EXEC_TILE) h->conv->source = codegen_tile(*h->conv);
+  *plan = h.release();
+  LL_CATCH
+}
+
+ll_status ll_plan_class(const ll_plan* p, ll_class* cls) {
+  LL_TRY
+  if (!p || !cls || p->kind != 0) fail(LL_ERR_INVALID_ARG, "not a conversion plan");
+  *cls = p->conv->cls;
+  LL_CATCH
+}
+
+ll_status ll_plan_workspace_bytes(const ll_plan* p, size_t* bytes) {
+  LL_TRY
+  if (!p || !bytes) fail(LL_ERR_INVALID_ARG, "null argument");
+  *bytes = p->kind == 0 ? p->conv->workspace_bytes : 0;
+  LL_CATCH
+}
+
+ll_status ll_plan_describe(const ll_plan* p, char* json, size_t cap) {
+  LL_TRY
+  if (!p || !json || !cap) fail(LL_ERR_INVALID_ARG, "null argument");
+  std::string s;
+  if (p->kind == 0) s = describe(*p->conv);
+  else if (p->kind == 1) {
+    const GatherPlan& G = *p->gather;
+    std::ostringstream o;
+    o << "{\"kind\":\"gather\",\"sigma\":\"" << (G.sigma ? "faithful" : "coalesced") << "\",\"R\":" << G.R
+      << ",\"warp_bits\":" << G.Wb << ",\"K_bits\":" << G.K_bits << ",\"shuffles_per_elem\":" << (1 << G.cand_bits)
+      << ",\"ctas\":" << (u64(1) << G.grid_bit.size()) << "}";
+    s = o.str();
+  } else {
+    const ReducePlan& Rp = *p->reduce;
+    std::ostringstream o;
+    o << "{\"kind\":\"reduce\",\"R\":" << Rp.R << ",\"warp_bits\":" << Rp.Wb << ",\"tree_levels\":" << Rp.red_reg.size()
+      << ",\"bfly_stages\":" << Rp.red_lane.size() << ",\"warp_stages\":" << Rp.red_warp.size()
+      << ",\"dup_bits\":" << Rp.dup_bits.size() << ",\"out_elems\":" << Rp.out_elems
+      << ",\"ctas\":" << (u64(1) << Rp.grid_bit.size()) << "}";
+    s = o.str();
+  }
+  std::strncpy(json, s.c_str(), cap - 1);
+  json[cap - 1] = 0;
+  if (s.size() >= cap) fail(LL_ERR_INVALID_ARG, "describe: buffer too small");
+  LL_CATCH
+}
+
+ll_status ll_plan_source(const ll_plan* p, char* buf, size_t cap, size_t* needed) {
+  LL_TRY
+  if (!p) fail(LL_ERR_INVALID_ARG, "null plan");
+  std::string s;
+  if (p->kind == 0 && p->conv->exec == EXEC_TILE) s = p->conv->source;
+  if (p->kind == 1) s = codegen_gather(*p->gather);
+  if (p->kind == 2) s = codegen_reduce(*p->reduce);
+  if (needed) *needed = s.size() + 1;
+  if (buf && cap) {
+    std::strncpy(buf, s.c_str(), cap - 1);
+    buf[cap - 1] = 0;
+  }
+  LL_CATCH
+}
+
+ll_status ll_plan_prepare(ll_plan* p) {
+  LL_TRY
+  if (!p) fail(LL_ERR_INVALID_ARG, "null plan");
+  if (p->kind == 0 && p->conv->exec == EXEC_TILE) ensure_tile_kernel(*p->conv);
+  if (p->kind == 0 && p->conv->exec == EXEC_DEVICE) {
+    if (p->conv->pack && p->conv->pack->exec == EXEC_TILE) ensure_tile_kernel(*p->conv->pack);
+    if (p->conv->unpack && p->conv->unpack->exec == EXEC_TILE) ensure_tile_kernel(*p->conv->unpack);
+  }
+  if (p->kind == 1) {
+    std::lock_guard<std::mutex> g(p->gather->mu);
+    if (!p->gather->kernel) p->gather->kernel = jit_kernel(codegen_gather(*p->gather), "ll_gather_kernel");
+  }
+  if (p->kind == 2) {
+    std::lock_guard<std::mutex> g(p->reduce->mu);
+    if (!p->reduce->kernel) {
+      p->reduce->kernel = jit_kernel(codegen_reduce(*p->reduce), "ll_reduce_kernel");
+      if (p->reduce->smem_bytes > 48 * 1024)
+        check_cuda(cudaFuncSetAttribute(p->reduce->kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                        p->reduce->smem_bytes), "cudaFuncSetAttribute");
+    }
+  }
+  LL_CATCH
+}
+
+ll_status ll_jit_precompile(const ll_plan* p) {
+  LL_TRY
+  if (!p) fail(LL_ERR_INVALID_ARG, "null plan");
+  if (p->kind == 0 && p->conv->exec == EXEC_TILE) jit_precompile(p->conv->source, "ll_tile_kernel");
+  if (p->kind == 1) jit_precompile(codegen_gather(*p->gather), "ll_gather_kernel");
+  if (p->kind == 2) jit_precompile(codegen_reduce(*p->reduce), "ll_reduce_kernel");
+  LL_CATCH
+}
+
+void ll_plan_destroy(ll_plan* p) { delete p; }
+
+ll_status ll_convert(const void* src, void* dst, void* ws, const ll_plan* p, void* stream) {
+  LL_TRY
+  if (!p || p->kind != 0) fail(LL_ERR_INVALID_ARG, "not a conversion plan");
+  if (!src || !dst) fail(LL_ERR_INVALID_ARG, "null buffer");
+  return convert_impl(src, dst, ws, *p->conv, static_cast<cudaStream_t>(stream));
+  LL_CATCH
+}
+
+ll_status ll_plan_gather(const ll_layout* L, int axis, int w, const ll_plan_opts* opts, ll_plan** plan) {
+  LL_TRY
+  if (!L || !plan) fail(LL_ERR_INVALID_ARG, "null argument");
+  if (w == 8) fail(LL_ERR_UNSUPPORTED, "gather: elem_bytes 8 not supported");
+  auto h = std::make_unique<ll_plan>();
+  h->kind = 1;
+  h->gather = plan_gather(L->L, axis, w, opts);
+  *plan = h.release();
+  LL_CATCH
+}
+
+ll_status ll_gather(const void* src, const int32_t* idx, void* dst, const ll_plan* p, void* stream) {
+  LL_TRY
+  if (!p || p->kind != 1) fail(LL_ERR_INVALID_ARG, "not a gather plan");
+  if (!src || !idx || !dst) fail(LL_ERR_INVALID_ARG, "null buffer");
+  if ((reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(idx) | reinterpret_cast<uintptr_t>(dst)) & 15)
+    fail(LL_ERR_MISALIGNED, "buffers must be 16-byte aligned");
+  GatherPlan& G = *p->gather;
+  {
+    std::lock_guard<std::mutex> g(G.mu);
+    if (!G.kernel) G.kernel = jit_kernel(codegen_gather(G), "ll_gather_kernel");
+  }
+  unsigned long long nt = u64(1) << G.grid_bit.size();
+  void* args[] = {const_cast<void**>(&src), const_cast<int32_t**>(&idx), &dst, &nt};
+  check_cuda(cudaLaunchKernel(G.kernel, dim3(grid_for(nt)), dim3(32u << G.Wb), args, 0, static_cast<cudaStream_t>(stream)),
+             "cudaLaunchKernel(ll_gather_kernel)");
+  LL_CATCH
+}
+
+ll_status ll_plan_reduce(const ll_layout* L, int axis, const ll_plan_opts* opts, ll_plan** plan) {
+  LL_TRY
+  if (!L || !plan) fail(LL_ERR_INVALID_ARG, "null argument");
+  auto h = std::make_unique<ll_plan>();
+  h->kind = 2;
+  h->reduce = plan_reduce(L->L, axis, opts);
+  *plan = h.release();
+  LL_CATCH
+}
+
+ll_status ll_plan_reduce_out_elems(const ll_plan* p, size_t* n) {
+  LL_TRY
+  if (!p || p->kind != 2 || !n) fail(LL_ERR_INVALID_ARG, "not a reduce plan");
+  *n = size_t(p->reduce->out_elems);
+  LL_CATCH
+}
+
+ll_status ll_reduce(const float* src, float* dst, const ll_plan* p, void* stream) {
+  LL_TRY
+  if (!p || p->kind != 2) fail(LL_ERR_INVALID_ARG, "not a reduce plan");
+  if (!src || !dst) fail(LL_ERR_INVALID_ARG, "null buffer");
+  if (reinterpret_cast<uintptr_t>(src) & 15) fail(LL_ERR_MISALIGNED, "src must be 16-byte aligned");
+  ll_status st = ll_plan_prepare(const_cast<ll_plan*>(p));
+  if (st != LL_OK) return st;
+  ReducePlan& Rp = *p->reduce;
+  unsigned long long nt = u64(1) << Rp.grid_bit.size();
+  void* args[] = {const_cast<float**>(&src), &dst, &nt};
+  check_cuda(cudaLaunchKernel(Rp.kernel, dim3(grid_for(nt)), dim3(32u << Rp.Wb), args, size_t(Rp.smem_bytes),
+                              static_cast<cudaStream_t>(stream)),
+             "cudaLaunchKernel(ll_reduce_kernel)");
+  LL_CATCH
+}
+
+ll_status ll_plan_simulate(const ll_plan* p, const void* src, void* dst) {
+  LL_TRY
+  if (!p || p->kind != 0 || !src || !dst) fail(LL_ERR_INVALID_ARG, "bad argument");
+  if (p->conv->exec != EXEC_TILE) fail(LL_ERR_UNSUPPORTED, "simulate: only tile plans");
+  simulate_tile(*p->conv, static_cast<const uint8_t*>(src), static_cast<uint8_t*>(dst));
+  LL_CATCH
+}
+
+}  // extern "C"

@@ -1,0 +1,168 @@
+// Specialisation of the sm_100a kernel templates (ll_kernels.cuh): emits the plan
+// constants as a `struct P` of compile-time tables and instantiates the entry point.
+#include <sstream>
+#include <type_traits>
+
+#include "ll_internal.hpp"
+
+namespace ll {
+
+namespace {
+
+template <class T>
+std::string arr(const char* type, const char* name, const std::vector<T>& v) {
+  std::ostringstream o;
+  o << "  static constexpr " << type << " " << name << "[" << (v.empty() ? 1 : v.size()) << "] = {";
+  if (v.empty()) o << "0";
+  for (size_t i = 0; i < v.size(); ++i) o << (i ? "," : "") << v[i] << (sizeof(T) == 8 ? "ull" : (std::is_unsigned<T>::value ? "u" : ""));
+  o << "};\n";
+  return o.str();
+}
+
+std::string icon(const char* name, long long v) {
+  std::ostringstream o;
+  o << "  static constexpr int " << name << " = " << v << ";\n";
+  return o.str();
+}
+
+int ilog2i(u64 v) { return v ? 63 - __builtin_clzll(v) : -1; }
+
+// grid map: CTA index bit g -> offsets; contiguous when both sides are a run of bits
+void emit_grid(std::ostringstream& o, const std::vector<int>& gs, const std::vector<int>& gd, int shift_scale) {
+  bool contig = !gs.empty();
+  for (size_t g = 0; g < gs.size(); ++g)
+    if (gs[g] != gs[0] + int(g) || gd[g] != gd[0] + int(g)) contig = false;
+  if (gs.empty()) contig = true;
+  o << icon("G", gs.size());
+  o << "  static constexpr bool GRID_CONTIG = " << (contig ? "true" : "false") << ";\n";
+  o << icon("GRID_LD_SHIFT", gs.empty() ? 0 : gs[0] + shift_scale);
+  o << icon("GRID_ST_SHIFT", gd.empty() ? 0 : gd[0] + shift_scale);
+  std::vector<u64> ld, st;
+  for (size_t g = 0; g < gs.size(); ++g) {
+    ld.push_back(u64(1) << (gs[g] + shift_scale));
+    st.push_back(u64(1) << (gd[g] + shift_scale));
+  }
+  o << arr("u64", "GRID_LD", ld) << arr("u64", "GRID_ST", st);
+}
+
+}  // namespace
+
+std::string codegen_tile(const ConvPlan& Pl) {
+  const TilePlan& T = Pl.tile;
+  const int lw = ilog2i(u64(T.w));
+  std::ostringstream o;
+  o << "// plan: " << describe(Pl).substr(0, 0) << "\nstruct P {\n";
+  o << icon("W", T.w) << icon("R", T.R) << icon("WB", T.Wb)
+    << icon("NW", std::max<long long>(1, ((1ll << T.R) * T.w) / 4))
+    << icon("VLD", T.vld) << icon("VST", T.vst) << icon("XCHG", T.xchg) << icon("THREADS", T.threads());
+  std::vector<u64> ldc, stc;
+  for (int b = 0; b < T.n; ++b) {
+    ldc.push_back(u64(1) << (T.ld_bit[b] + lw));
+    stc.push_back(u64(1) << (T.st_bit[b] + lw));
+  }
+  o << arr("u64", "LD_COL", ldc) << arr("u64", "ST_COL", stc);
+  emit_grid(o, T.grid_src_bit, T.grid_dst_bit, lw);
+  // REGPERM
+  o << arr("int", "PERM", T.perm);
+  // SHUFFLE
+  o << icon("NSLOT", T.nslot) << icon("UW", std::max(1, T.unit_elems * T.w / 4)) << icon("ROUNDS", T.rounds)
+    << icon("NPRE", T.pre_x.size()) << icon("NPOST", T.post_x.size());
+  o << arr("int", "SEND_SLOT", T.send_slot) << arr("int", "RECV_SLOT", T.recv_slot)
+    << arr("u32", "SRC_LANE0", T.src_lane0)
+    << arr("u32", "SRC_LANE_COL", std::vector<uint32_t>(T.src_lane_col, T.src_lane_col + 5))
+    << arr("u32", "PRE_LMASK", T.pre_lmask) << arr("int", "PRE_X", T.pre_x)
+    << arr("u32", "POST_LMASK", T.post_lmask) << arr("int", "POST_X", T.post_x);
+  // SMEM
+  o << icon("SV", T.sm_v) << arr("int", "VSLOT_LD", T.vec_slot_ld) << arr("int", "VSLOT_ST", T.vec_slot_st)
+    << arr("u64", "SMOFF_LD", T.smoff_ld) << arr("u64", "SMOFF_ST", T.smoff_st);
+  o << "};\n";
+  o << "extern \"C\" __global__ void __launch_bounds__(" << T.threads()
+    << ") ll_tile_kernel(const u8* __restrict__ src, u8* __restrict__ dst, u64 ntiles) {\n"
+    << "  ll_tile_body<P>(src, dst, ntiles);\n}\n";
+  return o.str();
+}
+
+std::string codegen_gather(const GatherPlan& G) {
+  std::ostringstream o;
+  const int n = int(G.hw_bit.size());
+  o << "struct P {\n";
+  o << icon("W", G.w) << icon("R", G.R) << icon("WB", G.Wb)
+    << icon("NW", std::max<long long>(1, ((1ll << G.R) * G.w) / 4)) << icon("VLD", G.v);
+  std::vector<u64> ldc;
+  for (int b = 0; b < n; ++b) ldc.push_back(u64(1) << G.hw_bit[b]);   // element offsets
+  o << arr("u64", "LD_COL", ldc);
+  std::vector<int> none;
+  emit_grid(o, G.grid_bit, G.grid_bit, 0);
+  o << icon("KBITS", G.K_bits) << icon("CBITS", G.cand_bits);
+  o << arr("int", "AXIS_OF_LANE", G.axis_of_lane) << arr("int", "AXIS_LANE_POS", G.axis_lane_pos);
+  // candidate bits: the register bits that carry axis bits, in ascending order
+  std::vector<int> cand_reg, axis_cand_pos(G.K_bits, -1), axis_of_reg = G.axis_of_reg;
+  for (int b = 0; b < G.R; ++b)
+    if (G.axis_of_reg[b] >= 0) { axis_cand_pos[G.axis_of_reg[b]] = int(cand_reg.size()); cand_reg.push_back(b); }
+  o << arr("int", "AXIS_CAND_POS", axis_cand_pos) << arr("int", "CAND_REG", cand_reg)
+    << arr("int", "AXIS_OF_REG", axis_of_reg);
+  o << "  template <int E> static constexpr u32 axis_of_slot() { u32 a = 0;"
+       " for (int b = 0; b < R; ++b) if (((E >> b) & 1) && AXIS_OF_REG[b] >= 0) a ^= 1u << AXIS_OF_REG[b]; return a; }\n";
+  o << "  template <int E> static constexpr u32 cand_of_slot() { u32 c = 0;"
+       " for (int i = 0; i < CBITS; ++i) if ((E >> CAND_REG[i]) & 1) c |= 1u << i; return c; }\n";
+  o << "  template <int E, int C> static constexpr int slot_of() { int s = E;"
+       " for (int i = 0; i < CBITS; ++i) { s &= ~(1 << CAND_REG[i]); if ((C >> i) & 1) s |= 1 << CAND_REG[i]; } return s; }\n";
+  o << "};\n";
+  o << "extern \"C\" __global__ void __launch_bounds__(" << (32 << G.Wb)
+    << ") ll_gather_kernel(const u8* __restrict__ src, const u8* __restrict__ idx, u8* __restrict__ dst, u64 ntiles) {\n"
+    << "  ll_gather_body<P>(src, idx, dst, ntiles);\n}\n";
+  return o.str();
+}
+
+std::string codegen_reduce(const ReducePlan& Rp) {
+  const Layout& L = Rp.L;
+  std::ostringstream o;
+  o << "struct P {\n";
+  const int R = Rp.R;
+  int v = std::min(2, R);
+  o << icon("W", 4) << icon("R", R) << icon("WB", Rp.Wb) << icon("VLD", v);
+  std::vector<u64> ldc;
+  for (int b = 0; b < R + 5 + Rp.Wb; ++b) ldc.push_back(u64(4) << b);
+  o << arr("u64", "LD_COL", ldc);
+  std::vector<int> gsh;
+  emit_grid(o, Rp.grid_bit, Rp.grid_bit, 2);
+  std::vector<u64> gout;
+  for (int k : Rp.grid_bit) gout.push_back(Rp.out_col[k]);
+  o << arr("u64", "GRID_OUT", gout);
+  std::vector<u64> oc(Rp.out_col.begin(), Rp.out_col.begin() + (R + 5 + Rp.Wb));
+  o << arr("u64", "OUT_COL", oc);
+  auto rel = [&](const std::vector<int>& bits, int base) {
+    std::vector<int> r;
+    for (int k : bits) r.push_back(k - base);
+    return r;
+  };
+  auto rr = rel(Rp.red_reg, 0), rl = rel(Rp.red_lane, R), rw = rel(Rp.red_warp, R + 5);
+  int regmask = 0, dupreg = 0;
+  uint32_t nolane = 0, nowarp = 0, rwmask = 0;
+  for (int b : rr) regmask |= 1 << b;
+  for (int b : rl) nolane |= 1u << b;
+  for (int b : rw) { nowarp |= 1u << b; rwmask |= 1u << b; }
+  for (int k : Rp.dup_bits) {
+    if (k < R) dupreg |= 1 << k;
+    else if (k < R + 5) nolane |= 1u << (k - R);
+    else if (k < R + 5 + Rp.Wb) nowarp |= 1u << (k - R - 5);
+  }
+  o << icon("NRED_REG", rr.size()) << arr("int", "RED_REG", rr) << icon("RED_REG_MASK", regmask)
+    << icon("DUP_REG_MASK", dupreg) << icon("NRED_LANE", rl.size()) << arr("int", "RED_LANE", rl)
+    << icon("NRED_WARP", rw.size()) << arr("int", "RED_WARP", rw);
+  o << "  static constexpr u32 NOSTORE_LANE_MASK = " << nolane << "u;\n"
+    << "  static constexpr u32 NOSTORE_WARP_MASK = " << nowarp << "u;\n"
+    << "  static constexpr u32 RED_WARP_MASK = " << rwmask << "u;\n";
+  o << "  template <int I> static constexpr int done_mask() { int m = 0; for (int j = 0; j < I; ++j) m |= 1 << RED_REG[j]; return m; }\n";
+  o << "  template <int E> static constexpr u64 out_of_slot() { u64 c = 0; for (int b = 0; b < R; ++b) if ((E >> b) & 1) c ^= OUT_COL[b]; return c; }\n";
+  o << "  template <int E> static constexpr int live_index() { int k = 0, t = 0;"
+       " for (int b = 0; b < R; ++b) { if ((RED_REG_MASK | DUP_REG_MASK) & (1 << b)) continue; if ((E >> b) & 1) k |= 1 << t; ++t; } return k; }\n";
+  o << "};\n";
+  o << "extern \"C\" __global__ void __launch_bounds__(" << (32 << Rp.Wb)
+    << ") ll_reduce_kernel(const float* __restrict__ src, float* __restrict__ dst, u64 ntiles) {\n"
+    << "  ll_reduce_body<P>(src, dst, ntiles);\n}\n";
+  (void)L;
+  return o.str();
+}
+
+}  // namespace ll

@@ -1,0 +1,249 @@
+// Linear layouts and their F2 algebra (row a2; Defs 4.1-4.5).
+#include <algorithm>
+#include <sstream>
+
+#include "ll_internal.hpp"
+
+namespace ll {
+
+static thread_local std::string g_last_error;
+void set_last_error(const std::string& m) { g_last_error = m; }
+const std::string& last_error_ref() { return g_last_error; }
+[[noreturn]] void fail(ll_status s, const std::string& msg) { throw Error(s, msg); }
+
+int dim_level(const std::string& n) {
+  if (n == "reg" || n == "register") return 0;
+  if (n == "lane" || n == "thr" || n == "thread") return 1;
+  if (n == "warp" || n == "wrp") return 2;
+  if (n == "block" || n == "cta" || n == "offset") return 3;
+  if (n == "dev" || n == "device") return 4;
+  return -1;
+}
+
+int Layout::d_in() const { int s = 0; for (auto& d : in) s += d.bits; return s; }
+int Layout::d_out() const { int s = 0; for (auto& d : out) s += d.bits; return s; }
+int Layout::in_pos(const std::string& name) const {
+  int p = 0;
+  for (auto& d : in) { if (d.name == name) return p; p += d.bits; }
+  return -1;
+}
+int Layout::in_bits(const std::string& name) const {
+  for (auto& d : in) if (d.name == name) return d.bits;
+  return 0;
+}
+int Layout::out_shift(int idx) const {
+  int s = 0;
+  for (size_t i = idx + 1; i < out.size(); ++i) s += out[i].bits;
+  return s;
+}
+int Layout::rank() const {
+  Echelon e;
+  for (u64 c : cols) e.insert(c);
+  return e.rank;
+}
+bool Layout::distributed() const {
+  // Def 4.10: surjective; every column has at most one set bit; no
+  // repeated non-zero columns.
+  if (!surjective()) return false;
+  std::vector<u64> nz;
+  for (u64 c : cols) {
+    if (popc(c) > 1) return false;
+    if (c) nz.push_back(c);
+  }
+  std::sort(nz.begin(), nz.end());
+  return std::adjacent_find(nz.begin(), nz.end()) == nz.end();
+}
+bool Layout::memory() const {
+  // Def 4.14: invertible, columns with 1 or 2 set bits.
+  if (d_in() != d_out() || !surjective()) return false;
+  for (u64 c : cols) if (popc(c) < 1 || popc(c) > 2) return false;
+  return true;
+}
+bool Layout::unit_columns() const {
+  if (d_in() != d_out()) return false;
+  u64 seen = 0;
+  for (u64 c : cols) {
+    if (popc(c) != 1 || (seen & c)) return false;
+    seen |= c;
+  }
+  return true;
+}
+
+u64 apply_cols(const std::vector<u64>& cols, u64 v) {
+  u64 x = 0;
+  for (size_t k = 0; k < cols.size(); ++k) if ((v >> k) & 1) x ^= cols[k];
+  return x;
+}
+
+std::vector<u64> right_inverse_cols(const Layout& L) {
+  // Gaussian elimination over F2: process the columns in ascending order;
+  // a column that reduces to zero is a free variable and stays 0 (slack = 0).
+  Echelon e;
+  for (size_t k = 0; k < L.cols.size(); ++k) e.insert(L.cols[k], u64(1) << k);
+  if (e.rank != L.d_out()) fail(LL_ERR_NOT_SURJECTIVE, "layout is not surjective (P:194)");
+  std::vector<u64> out(L.d_out());
+  for (int t = 0; t < L.d_out(); ++t) {
+    u64 c = 0;
+    u64 r = e.reduce(u64(1) << t, &c);
+    if (r) fail(LL_ERR_NOT_SURJECTIVE, "layout is not surjective (P:194)");
+    out[t] = c;
+  }
+  return out;
+}
+
+std::vector<u64> kernel_basis(const Layout& L) {
+  Echelon e;
+  std::vector<u64> ker;
+  for (size_t k = 0; k < L.cols.size(); ++k) {
+    u64 c = u64(1) << k;
+    u64 r = e.reduce(L.cols[k], &c);
+    if (r) e.insert(r, c);      // (reduce again inside insert is a no-op)
+    else ker.push_back(c);      // column k depends on earlier ones: kernel vector
+  }
+  return ker;
+}
+
+static u64 coords_to_flat(const std::vector<Dim>& dims, const std::vector<u64>& c) {
+  u64 f = 0;
+  for (size_t i = 0; i < dims.size(); ++i) f = (f << dims[i].bits) | c[i];
+  return f;
+}
+static std::vector<u64> flat_to_coords(const std::vector<Dim>& dims, u64 f) {
+  std::vector<u64> c(dims.size());
+  for (int i = int(dims.size()) - 1; i >= 0; --i) {
+    c[i] = dims[i].bits ? (f & ((u64(1) << dims[i].bits) - 1)) : 0;
+    f = dims[i].bits >= 64 ? 0 : (f >> dims[i].bits);
+  }
+  return c;
+}
+static u64 hw_to_flat_hw(const std::vector<Dim>& dims, const std::vector<u64>& c) {
+  // hardware flat: first dim least significant
+  u64 h = 0; int s = 0;
+  for (size_t i = 0; i < dims.size(); ++i) { h |= c[i] << s; s += dims[i].bits; }
+  return h;
+}
+static std::vector<u64> hw_coords(const std::vector<Dim>& dims, u64 h) {
+  std::vector<u64> c(dims.size());
+  for (size_t i = 0; i < dims.size(); ++i) {
+    c[i] = dims[i].bits ? (h & ((u64(1) << dims[i].bits) - 1)) : 0;
+    h >>= dims[i].bits;
+  }
+  return c;
+}
+
+// Re-express a layout whose *output* is a hardware space (e.g. an inverse) — its
+// output coordinates are the named dims, flattened row-major like any output.
+Layout compose(const Layout& outer, const Layout& inner) {
+  // Def 4.2: (outer ∘ inner)(u) = outer(inner(u)); label-wise matrix product.
+  if (inner.out != outer.in) fail(LL_ERR_DIM_MISMATCH, "compose: inner.out != outer.in");
+  Layout R;
+  R.in = inner.in;
+  R.out = outer.out;
+  for (u64 c : inner.cols) {
+    // c is a logical flat over inner.out (row-major); outer's input is hardware
+    // flat (first dim lowest): convert coordinates.
+    auto coords = flat_to_coords(inner.out, c);
+    u64 h = hw_to_flat_hw(outer.in, coords);
+    R.cols.push_back(outer.apply(h));
+  }
+  return R;
+}
+
+Layout invert(const Layout& L) {
+  // Def 4.5: right inverse as a layout from L's output dims to L's input dims.
+  auto hc = right_inverse_cols(L);   // per logical flat bit (lowest first)
+  Layout R;
+  R.in = L.out;
+  R.out = L.in;
+  // R's input bits in hardware-flat order: first dim of L.out lowest.  Logical
+  // flat bit of (dim i, bit b) = out_shift(i) + b.
+  for (size_t i = 0; i < L.out.size(); ++i) {
+    int sh = L.out_shift(int(i));
+    for (int b = 0; b < L.out[i].bits; ++b) {
+      u64 h = hc[sh + b];
+      R.cols.push_back(coords_to_flat(L.in, hw_coords(L.in, h)));
+    }
+  }
+  return R;
+}
+
+static std::vector<Dim> merge_dims(const std::vector<Dim>& a, const std::vector<Dim>& b) {
+  std::vector<Dim> r = a;
+  for (auto& d : b) {
+    bool found = false;
+    for (auto& x : r) if (x.name == d.name) { x.bits += d.bits; found = true; }
+    if (!found) r.push_back(d);
+  }
+  return r;
+}
+
+Layout product(const Layout& L1, const Layout& L2) {
+  // Def 4.3, label-wise: dims with the same name concatenate, L1's
+  // bits low; L2's images are shifted above L1's range in every output dim.
+  Layout R;
+  R.in = merge_dims(L1.in, L2.in);
+  R.out = merge_dims(L1.out, L2.out);
+  auto coord_in = [&](const Layout& S, u64 col, int shift_by_L1) {
+    auto c = flat_to_coords(S.out, col);
+    std::vector<u64> rc(R.out.size(), 0);
+    for (size_t i = 0; i < S.out.size(); ++i) {
+      size_t j = 0;
+      while (R.out[j].name != S.out[i].name) ++j;
+      int sh = 0;
+      if (shift_by_L1)
+        for (auto& d : L1.out) if (d.name == S.out[i].name) sh = d.bits;
+      rc[j] = c[i] << sh;
+    }
+    return coords_to_flat(R.out, rc);
+  };
+  for (auto& d : R.in) {
+    int p1 = L1.in_pos(d.name), b1 = L1.in_bits(d.name);
+    int p2 = L2.in_pos(d.name), b2 = L2.in_bits(d.name);
+    for (int k = 0; k < b1; ++k) R.cols.push_back(coord_in(L1, L1.cols[p1 + k], 0));
+    for (int k = 0; k < b2; ++k) R.cols.push_back(coord_in(L2, L2.cols[p2 + k], 1));
+  }
+  return R;
+}
+
+Layout left_divide(const Layout& M, const Layout& M1) {
+  // Def 4.4: M /_l M1 = M2 iff M = diag(M1, M2) label-wise.
+  Layout R;
+  for (auto& d : M.in) R.in.push_back({d.name, d.bits - M1.in_bits(d.name)});
+  for (size_t i = 0; i < M.out.size(); ++i) {
+    int b1 = 0;
+    for (auto& d : M1.out) if (d.name == M.out[i].name) b1 = d.bits;
+    R.out.push_back({M.out[i].name, M.out[i].bits - b1});
+  }
+  for (auto& d : R.in) if (d.bits < 0) fail(LL_ERR_NOT_DIVISIBLE, "M1 has more input bits than M");
+  for (auto& d : R.out) if (d.bits < 0) fail(LL_ERR_NOT_DIVISIBLE, "M1 has more output bits than M");
+  for (auto& d : M1.in) if (M.in_pos(d.name) < 0 && d.bits) fail(LL_ERR_NOT_DIVISIBLE, "M1 dim missing in M");
+  for (auto& d : M.in) {
+    int p = M.in_pos(d.name);
+    int k1 = M1.in_bits(d.name);
+    int p1 = M1.in_pos(d.name);
+    for (int k = 0; k < d.bits; ++k) {
+      auto c = flat_to_coords(M.out, M.cols[p + k]);
+      if (k < k1) {
+        auto c1 = flat_to_coords(M1.out, M1.cols[p1 + k]);
+        for (size_t i = 0; i < M.out.size(); ++i) {
+          u64 want = 0;
+          for (size_t j = 0; j < M1.out.size(); ++j)
+            if (M1.out[j].name == M.out[i].name) want = c1[j];
+          if (c[i] != want) fail(LL_ERR_NOT_DIVISIBLE, "left division: low bits differ from M1");
+        }
+      } else {
+        std::vector<u64> rc(M.out.size());
+        for (size_t i = 0; i < M.out.size(); ++i) {
+          int b1 = 0;
+          for (auto& x : M1.out) if (x.name == M.out[i].name) b1 = x.bits;
+          if (c[i] & ((u64(1) << b1) - 1)) fail(LL_ERR_NOT_DIVISIBLE, "left division: overlaps M1's range");
+          rc[i] = c[i] >> b1;
+        }
+        R.cols.push_back(coords_to_flat(R.out, rc));
+      }
+    }
+  }
+  return R;
+}
+
+}  // namespace ll

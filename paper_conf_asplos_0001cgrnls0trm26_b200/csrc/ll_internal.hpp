@@ -1,0 +1,248 @@
+// Internal declarations of the linear-layout library (host side).
+//
+// Layer map:
+//   f2      — F2 vector/matrix helpers over uint64 columns (§2.4)
+//   Layout  — labelled linear layouts (Def 4.1) and their algebra
+//             (Defs 4.2-4.5)
+//   plan    — conversion planner: pull map Q = A^+ ∘ B, class selection
+//             (P:350-373), kernel decomposition, shuffle plan and
+//             optimal swizzle; gather and
+//             reduce plans
+//   codegen — specialisation of the sm_100a kernel templates (ll_kernels.cuh)
+//   jit     — NVRTC compilation + cubin cache + cudaLibrary loading
+//   capi    — the C ABI of include/ll.h
+#pragma once
+#include <cstdint>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <stdexcept>
+#include <string>
+#include <vector>
+
+#include "../../include/ll.h"
+
+namespace ll {
+
+using u64 = uint64_t;
+
+// Error carrying an ll_status across internal layers; never crosses the ABI.
+struct Error : std::runtime_error {
+  ll_status st;
+  Error(ll_status s, const std::string& m) : std::runtime_error(m), st(s) {}
+};
+[[noreturn]] void fail(ll_status s, const std::string& msg);
+void set_last_error(const std::string& msg);
+
+inline int popc(u64 v) { return __builtin_popcountll(v); }
+inline int lead(u64 v) { return 63 - __builtin_clzll(v); }
+inline bool parity(u64 v) { return popc(v) & 1; }
+
+// ------------------------------------------------------------------ F2 helpers
+// Row-echelon basis keyed by leading bit, tracking for every stored vector the
+// combination (over some index space) that produced it.
+struct Echelon {
+  u64 vec[64] = {0};
+  u64 comb[64] = {0};
+  bool has[64] = {false};
+  int rank = 0;
+  // Reduce v (with running combination c); returns the residue.
+  u64 reduce(u64 v, u64* c = nullptr) const {
+    while (v) {
+      int l = lead(v);
+      if (!has[l]) return v;
+      v ^= vec[l];
+      if (c) *c ^= comb[l];
+    }
+    return 0;
+  }
+  // Insert v (with combination c); returns true if it was independent.
+  bool insert(u64 v, u64 c = 0) {
+    v = reduce(v, &c);
+    if (!v) return false;
+    int l = lead(v);
+    has[l] = true; vec[l] = v; comb[l] = c; ++rank;
+    return true;
+  }
+  bool contains(u64 v) const { return reduce(v) == 0; }
+};
+
+// ------------------------------------------------------------------ layouts
+struct Dim {
+  std::string name;
+  int bits;
+  bool operator==(const Dim& o) const { return name == o.name && bits == o.bits; }
+  bool operator!=(const Dim& o) const { return !(*this == o); }
+};
+
+// Hardware level of an input dim (reg < lane < warp < block < dev).  "offset"
+// (memory layouts, Def 4.14) lives at the block level.  Unknown names: -1.
+int dim_level(const std::string& name);
+
+struct Layout {
+  std::vector<Dim> in, out;
+  // cols[k]: logical flat index (row-major over `out`, last dim fastest)
+  // hit by hardware bit k (hardware flat order: first input dim lowest).
+  std::vector<u64> cols;
+
+  int d_in() const;
+  int d_out() const;
+  int in_pos(const std::string& name) const;   // first hardware bit of dim, -1
+  int in_bits(const std::string& name) const;  // 0 if absent
+  int out_shift(int out_index) const;          // flat shift of output dim
+  u64 apply(u64 h) const {
+    u64 x = 0;
+    for (size_t k = 0; k < cols.size(); ++k)
+      if ((h >> k) & 1) x ^= cols[k];
+    return x;
+  }
+  int rank() const;
+  bool surjective() const { return rank() == d_out(); }
+  bool injective() const { return rank() == d_in(); }
+  bool distributed() const;   // Def 4.10
+  bool memory() const;        // Def 4.14
+  bool unit_columns() const;  // every column a single bit (a bijective permutation)
+};
+
+// Slack-zero right inverse: per logical flat bit t, the hardware
+// index of the solution with free variables 0 and pivots in ascending column order.
+std::vector<u64> right_inverse_cols(const Layout& L);
+u64 apply_cols(const std::vector<u64>& cols, u64 v);
+// Basis of ker(L) (hardware vectors).
+std::vector<u64> kernel_basis(const Layout& L);
+
+Layout compose(const Layout& outer, const Layout& inner);     // Def 4.2
+Layout invert(const Layout& L);                                // Def 4.5
+Layout product(const Layout& L1, const Layout& L2);            // Def 4.3
+Layout left_divide(const Layout& M, const Layout& M1);         // Def 4.4
+
+// ------------------------------------------------------------------ plans
+enum ExecKind { EXEC_NOOP = 0, EXEC_TILE = 1, EXEC_GENERIC = 2, EXEC_DEVICE = 3 };
+enum TileXchg { X_COPY = 0, X_REGPERM = 1, X_SHUFFLE = 2, X_SMEM = 3 };
+enum SigmaMode { SIGMA_COALESCED = 0, SIGMA_FAITHFUL = 1 };
+
+// Kernel decomposition of a conversion whose pull map is a bit permutation:
+// a CTA owns `n` tile bits; kernel hardware inside the CTA is (R reg bits,
+// 5 lane bits, Wb warp bits).  For every kernel hardware bit b:
+//   ld_bit[b] = src packed bit it loads from (L_ld = A ∘ σ_ld), lcol_ld[b] = A.col
+//   st_bit[b] = dst packed bit it stores to  (L_st = B ∘ σ_st), lcol_st[b] = B.col
+// Kernel bit order: reg 0..R-1, lane 0..4, warp 0..Wb-1.
+struct TilePlan {
+  int w = 4;            // element bytes
+  int n = 0;            // tile bits
+  int R = 0, Wb = 0;    // kernel reg / warp bits (lanes = 5)
+  int vld = 0, vst = 0; // elements per global vector = 1 << v
+  std::vector<int> ld_bit, st_bit;
+  std::vector<u64> lcol_ld, lcol_st;
+  std::vector<int> grid_src_bit, grid_dst_bit;   // CTA index bit g -> packed bits
+  int sigma = SIGMA_COALESCED;
+  int xchg = X_COPY;
+
+  // --- REGPERM: out slot e <- in slot perm[e]
+  std::vector<int> perm;
+
+  // --- SHUFFLE; units of `unit_elems` elements (one 32-bit word for
+  // w<4, one element for w>=4); all unit indices are register-unit indices.
+  int unit_elems = 1, nslot = 0;
+  std::vector<u64> V, I, E, F, G, Rb;          // logical vectors (describe)
+  int rounds = 0;
+  std::vector<int> send_slot, recv_slot;       // per round (after pre-permutation)
+  std::vector<uint32_t> src_lane0;             // per round: source lane for lane 0
+  uint32_t src_lane_col[5] = {0, 0, 0, 0, 0};  // linear part: lane bit t -> XOR
+  std::vector<uint32_t> pre_lmask, post_lmask; // per stage: lane mask (parity predicate)
+  std::vector<int> pre_x, post_x;              // per stage: slot XOR constant
+
+  // --- SMEM: smem layout M: offset bits (Vec, Bank, Seg)
+  std::vector<u64> sw_vec, sw_bank, sw_seg, sw_H, sw_C;
+  int sm_v = 0;                               // |Vec|
+  std::vector<int> vec_slot_ld, vec_slot_st;  // reg bit positions of Vec in L_ld / L_st
+  // smem element offset contributed by each kernel hardware bit (M^{-1} ∘ L)
+  std::vector<u64> smoff_ld, smoff_st;
+  u64 smem_elems = 0;
+  long predicted_wavefronts_st = -1, predicted_wavefronts_ld = -1, ideal_wavefronts = -1;
+
+  int threads() const { return 32 << Wb; }
+  int elems_per_thread() const { return 1 << R; }
+};
+
+struct ConvPlan {
+  Layout A, B;          // original (local) layouts
+  int w = 4;
+  ll_class cls = LL_CLASS_NOOP;   // the paper's class of A -> B
+  int exec = EXEC_NOOP;
+  std::vector<u64> Q;   // pull map: dst bit k -> src packed index (A^+ ∘ B, adjusted)
+  u64 src_elems = 0, dst_elems = 0;
+  TilePlan tile;
+  // DEVICE plans
+  int dev_bits = 0;
+  size_t workspace_bytes = 0;
+  ll_comm* comm = nullptr;
+  std::unique_ptr<ConvPlan> pack, unpack;   // local stages of a DEVICE plan
+  std::string source;   // specialised kernel source (EXEC_TILE)
+  std::string kernel_key;
+  void* kernel = nullptr;   // cudaKernel_t once loaded
+  int smem_bytes = 0;
+  std::mutex mu;
+};
+
+std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, const ll_plan_opts* opts);
+std::string describe(const ConvPlan& P);
+
+struct GatherPlan {
+  Layout L;
+  int axis = 0, w = 4;
+  int exec = EXEC_TILE;
+  int sigma = SIGMA_COALESCED;
+  int R = 0, Wb = 0, v = 0;
+  int K_bits = 0;          // in-tile axis bits (K = 1 << K_bits)
+  std::vector<int> hw_bit; // kernel bit -> packed bit (same for src, idx, dst)
+  std::vector<u64> lcol;   // kernel bit -> logical column
+  std::vector<int> grid_bit;
+  // axis bit t (0..K_bits-1): position in the kernel: reg bit or lane bit (-1)
+  std::vector<int> axis_reg_pos, axis_lane_pos;
+  std::vector<int> axis_of_reg;  // kernel reg bit -> axis bit index or -1
+  std::vector<int> axis_of_lane;
+  int cand_bits = 0;       // |L_Reg^axis| in the kernel layout
+  std::string source;
+  void* kernel = nullptr;
+  std::mutex mu;
+};
+std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const ll_plan_opts* opts);
+
+struct ReducePlan {
+  Layout L;
+  int axis = 0;
+  int exec = EXEC_TILE;
+  int R = 0, Wb = 0;
+  std::vector<int> grid_bit;      // CTA index bit -> packed bit
+  std::vector<int> red_reg, red_lane, red_warp;   // reduced kernel bits (L order)
+  std::vector<int> dup_bits;      // zero-column kernel bits (de-dup)
+  std::vector<u64> out_col;       // per packed bit: output flat offset (0 for reduced/dup)
+  u64 out_elems = 0;
+  std::string source;
+  void* kernel = nullptr;
+  int smem_bytes = 0;
+  std::mutex mu;
+};
+std::unique_ptr<ReducePlan> plan_reduce(const Layout& L, int axis, const ll_plan_opts* opts);
+
+// ------------------------------------------------------------------ codegen / jit
+std::string codegen_tile(const ConvPlan& P);
+std::string codegen_gather(const GatherPlan& P);
+std::string codegen_reduce(const ReducePlan& P);
+// Compile (or fetch from cache) and return a cudaKernel_t for `source`.
+void* jit_kernel(const std::string& source, const char* name);
+const char* kernel_template();   // embedded ll_kernels.cuh
+
+// ------------------------------------------------------------------ host simulation (tests)
+void simulate_tile(const ConvPlan& P, const uint8_t* src, uint8_t* dst);
+
+}  // namespace ll
+
+struct ll_layout { ll::Layout L; };
+struct ll_plan {
+  int kind;   // 0 conv, 1 gather, 2 reduce
+  std::unique_ptr<ll::ConvPlan> conv;
+  std::unique_ptr<ll::GatherPlan> gather;
+  std::unique_ptr<ll::ReducePlan> reduce;
+};

@@ -1,0 +1,536 @@
+// ll_kernels.cuh — sm_100a kernel templates for the linear-layout conversion hot path.
+//
+// Hand-written CUDA; specialised per plan by codegen.cpp, which emits a `struct P`
+// of compile-time tables (plan constants) and instantiates the entry points at the
+// end of this file.  Compiled with NVRTC for sm_100a (jit.cpp) and cached.
+//
+// Every register index below is a compile-time constant (static_for), so the
+// per-thread register file is addressed statically: register permutations are
+// free renamings, lane-dependent choices are selp networks (P:371-389 via the
+// affine decomposition of DESIGN.md §5.2).
+//
+// Rows of SURVEY §8(a): a5 HBM load (ld_tile), a6 REGPERM, a7 SHUFFLE, a8 SMEM,
+// a9 CTA (grid map), a10 HBM store (st_tile), a11 gather, a12 reduce.
+
+typedef unsigned int u32;
+typedef unsigned long long u64;
+typedef unsigned short u16;
+typedef unsigned char u8;
+
+// ------------------------------------------------------------------ compile-time loops
+template <int V> struct IC { static constexpr int value = V; };
+template <int I, int N, bool Small = (N - I <= 1)> struct SFor;
+template <int I, int N> struct SFor<I, N, true> {
+  template <class F> __device__ __forceinline__ static void run(F& f) {
+    if constexpr (N - I == 1) f(IC<I>{});
+  }
+};
+template <int I, int N> struct SFor<I, N, false> {
+  template <class F> __device__ __forceinline__ static void run(F& f) {
+    SFor<I, (I + N) / 2>::run(f);
+    SFor<(I + N) / 2, N>::run(f);
+  }
+};
+template <int N, class F> __device__ __forceinline__ void static_for(F&& f) { SFor<0, N>::run(f); }
+
+// ------------------------------------------------------------------ element access
+// Registers are 32-bit words; an element of W bytes (W in 1, 2, 4) at slot e lives
+// in word e*W/4 at byte (e*W) % 4.
+template <int W, int E> __device__ __forceinline__ u32 get_e(const u32* r) {
+  if constexpr (W == 4) return r[E];
+  else if constexpr (W == 2) return (r[E >> 1] >> (16 * (E & 1))) & 0xffffu;
+  else return (r[E >> 2] >> (8 * (E & 3))) & 0xffu;
+}
+template <int W, int E> __device__ __forceinline__ void set_e(u32* r, u32 v) {
+  if constexpr (W == 4) r[E] = v;
+  else if constexpr (W == 2) {
+    constexpr int s = 16 * (E & 1);
+    r[E >> 1] = (r[E >> 1] & ~(0xffffu << s)) | (v << s);
+  } else {
+    constexpr int s = 8 * (E & 3);
+    r[E >> 2] = (r[E >> 2] & ~(0xffu << s)) | (v << s);
+  }
+}
+
+// ------------------------------------------------------------------ global memory
+__device__ __forceinline__ void ldg_v4(const u8* p, u32& a, u32& b, u32& c, u32& d) {
+  asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(a), "=r"(b), "=r"(c), "=r"(d) : "l"(p));
+}
+__device__ __forceinline__ void ldg_v2(const u8* p, u32& a, u32& b) {
+  asm volatile("ld.global.nc.L1::no_allocate.v2.u32 {%0,%1}, [%2];" : "=r"(a), "=r"(b) : "l"(p));
+}
+__device__ __forceinline__ u32 ldg_b32(const u8* p) {
+  u32 a;
+  asm volatile("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(a) : "l"(p));
+  return a;
+}
+__device__ __forceinline__ void stg_v4(u8* p, u32 a, u32 b, u32 c, u32 d) {
+  asm volatile("st.global.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(a), "r"(b), "r"(c), "r"(d) : "memory");
+}
+__device__ __forceinline__ void stg_v2(u8* p, u32 a, u32 b) {
+  asm volatile("st.global.v2.u32 [%0], {%1,%2};" ::"l"(p), "r"(a), "r"(b) : "memory");
+}
+__device__ __forceinline__ void stg_b32(u8* p, u32 a) {
+  asm volatile("st.global.u32 [%0], %1;" ::"l"(p), "r"(a) : "memory");
+}
+
+// Load vector K of the thread (2^VL elements of W bytes starting at slot K<<VL).
+template <int W, int VL, int K, int NW>
+__device__ __forceinline__ void load_vec(u32 (&r)[NW], const u8* p) {
+  constexpr int VB = W << VL;                 // vector bytes
+  constexpr int E0 = K << VL;
+  if constexpr (VB == 16) {
+    ldg_v4(p, r[E0 * W / 4 + 0], r[E0 * W / 4 + 1], r[E0 * W / 4 + 2], r[E0 * W / 4 + 3]);
+  } else if constexpr (VB == 8) {
+    ldg_v2(p, r[E0 * W / 4 + 0], r[E0 * W / 4 + 1]);
+  } else if constexpr (VB == 4) {
+    r[E0 * W / 4] = ldg_b32(p);
+  } else if constexpr (VB == 2) {
+    set_e<2, E0 * W / 2>(r, u32(*reinterpret_cast<const u16*>(p)));
+  } else {
+    set_e<1, E0>(r, u32(*p));
+  }
+}
+template <int W, int VL, int K, int NW>
+__device__ __forceinline__ void store_vec(const u32 (&r)[NW], u8* p) {
+  constexpr int VB = W << VL;
+  constexpr int E0 = K << VL;
+  if constexpr (VB == 16) {
+    stg_v4(p, r[E0 * W / 4 + 0], r[E0 * W / 4 + 1], r[E0 * W / 4 + 2], r[E0 * W / 4 + 3]);
+  } else if constexpr (VB == 8) {
+    stg_v2(p, r[E0 * W / 4 + 0], r[E0 * W / 4 + 1]);
+  } else if constexpr (VB == 4) {
+    stg_b32(p, r[E0 * W / 4]);
+  } else if constexpr (VB == 2) {
+    *reinterpret_cast<u16*>(p) = u16(get_e<2, E0 * W / 2>(r));
+  } else {
+    *p = u8(get_e<1, E0>(r));
+  }
+}
+
+// Byte offset (within the tile) of thread-local vector K: XOR of the per-register-bit
+// columns (compile time).
+template <class P, int K> struct LdOff {
+  static constexpr u64 value() {
+    u64 o = 0;
+    for (int b = P::VLD; b < P::R; ++b) if (((K << P::VLD) >> b) & 1) o ^= P::LD_COL[b];
+    return o;
+  }
+};
+template <class P, int K> struct StOff {
+  static constexpr u64 value() {
+    u64 o = 0;
+    for (int b = P::VST; b < P::R; ++b) if (((K << P::VST) >> b) & 1) o ^= P::ST_COL[b];
+    return o;
+  }
+};
+
+// Per-thread base from the lane / warp columns (runtime lane, warp).
+template <class P, bool LD>
+__device__ __forceinline__ u64 thread_base(u32 lane, u32 warp) {
+  u64 o = 0;
+  static_for<5>([&](auto t) {
+    constexpr int T = decltype(t)::value;
+    u64 c;
+    if constexpr (LD) c = P::LD_COL[P::R + T]; else c = P::ST_COL[P::R + T];
+    if ((lane >> T) & 1) o ^= c;
+  });
+  static_for<P::WB>([&](auto t) {
+    constexpr int T = decltype(t)::value;
+    u64 c;
+    if constexpr (LD) c = P::LD_COL[P::R + 5 + T]; else c = P::ST_COL[P::R + 5 + T];
+    if ((warp >> T) & 1) o ^= c;
+  });
+  return o;
+}
+
+template <class P, bool LD>
+__device__ __forceinline__ u64 tile_base(u64 t) {
+  if constexpr (P::GRID_CONTIG) {
+    if constexpr (LD) return t << P::GRID_LD_SHIFT; else return t << P::GRID_ST_SHIFT;
+  } else {
+    u64 o = 0;
+    static_for<P::G>([&](auto g) {
+      constexpr int Gi = decltype(g)::value;
+      u64 c;
+      if constexpr (LD) c = P::GRID_LD[Gi]; else c = P::GRID_ST[Gi];
+      if ((t >> Gi) & 1) o ^= c;
+    });
+    return o;
+  }
+}
+
+// ------------------------------------------------------------------ exchanges
+// a6 REGPERM: out slot e <- in slot PERM[e]; free renaming for W = 4.
+template <class P>
+__device__ __forceinline__ void xchg_regperm(const u32 (&r)[P::NW], u32 (&o)[P::NW]) {
+  static_for<(1 << P::R)>([&](auto e) {
+    constexpr int E = decltype(e)::value;
+    set_e<P::W, E>(o, get_e<P::W, P::PERM[E]>(r));
+  });
+}
+
+// Conditional-swap network: slot j <-> slot j^X[s] when parity(lane & MASK[s]).
+template <class P, bool PRE>
+__device__ __forceinline__ void xor_net(u32 (&r)[P::NW], u32 lane) {
+  constexpr int NST = PRE ? P::NPRE : P::NPOST;
+  static_for<NST>([&](auto s) {
+    constexpr int S = decltype(s)::value;
+    constexpr u32 MASK = PRE ? P::PRE_LMASK[S] : P::POST_LMASK[S];
+    constexpr int X = PRE ? P::PRE_X[S] : P::POST_X[S];
+    const bool p = __popc(lane & MASK) & 1;
+    static_for<P::NSLOT>([&](auto j) {
+      constexpr int J = decltype(j)::value;
+      constexpr int K = J ^ X;
+      if constexpr (K > J) {
+        static_for<P::UW>([&](auto q) {
+          constexpr int Q = decltype(q)::value;
+          const u32 a = r[J * P::UW + Q], b = r[K * P::UW + Q];
+          r[J * P::UW + Q] = p ? b : a;
+          r[K * P::UW + Q] = p ? a : b;
+        });
+      }
+    });
+  });
+}
+
+// a7 SHUFFLE: pre-permutation (slot ^= M·lane), 2^|R| rounds of
+// shfl.sync.idx moving one 32-bit unit each, static renaming, post-permutation.
+template <class P>
+__device__ __forceinline__ void xchg_shuffle(u32 (&r)[P::NW], u32 (&o)[P::NW], u32 lane) {
+  xor_net<P, true>(r, lane);
+  u32 lx = 0;
+  static_for<5>([&](auto t) {
+    constexpr int T = decltype(t)::value;
+    if ((lane >> T) & 1) lx ^= P::SRC_LANE_COL[T];
+  });
+  static_for<P::ROUNDS>([&](auto rr) {
+    constexpr int RR = decltype(rr)::value;
+    constexpr int S = P::SEND_SLOT[RR];
+    const int sl = int(P::SRC_LANE0[RR] ^ lx);
+    static_for<P::UW>([&](auto q) {
+      constexpr int Q = decltype(q)::value;
+      r[S * P::UW + Q] = __shfl_sync(0xffffffffu, r[S * P::UW + Q], sl);
+    });
+  });
+  static_for<P::ROUNDS>([&](auto rr) {
+    constexpr int RR = decltype(rr)::value;
+    static_for<P::UW>([&](auto q) {
+      constexpr int Q = decltype(q)::value;
+      o[P::RECV_SLOT[RR] * P::UW + Q] = r[P::SEND_SLOT[RR] * P::UW + Q];
+    });
+  });
+  xor_net<P, false>(o, lane);
+}
+
+// Shared-memory vector access of 2^SV elements (SV = |Vec|) at element offset off.
+template <int W, int SV>
+__device__ __forceinline__ void sts_vec(u32 addr, const u32* v) {
+  constexpr int VB = W << SV;
+  if constexpr (VB == 16)
+    asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(addr), "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]) : "memory");
+  else if constexpr (VB == 8)
+    asm volatile("st.shared.v2.u32 [%0], {%1,%2};" ::"r"(addr), "r"(v[0]), "r"(v[1]) : "memory");
+  else if constexpr (VB == 4)
+    asm volatile("st.shared.u32 [%0], %1;" ::"r"(addr), "r"(v[0]) : "memory");
+  else if constexpr (VB == 2)
+    asm volatile("st.shared.u16 [%0], %1;" ::"r"(addr), "h"(u16(v[0])) : "memory");
+  else
+    asm volatile("st.shared.u8 [%0], %1;" ::"r"(addr), "r"(v[0]) : "memory");
+}
+template <int W, int SV>
+__device__ __forceinline__ void lds_vec(u32 addr, u32* v) {
+  constexpr int VB = W << SV;
+  if constexpr (VB == 16)
+    asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]) : "r"(addr) : "memory");
+  else if constexpr (VB == 8)
+    asm volatile("ld.shared.v2.u32 {%0,%1}, [%2];" : "=r"(v[0]), "=r"(v[1]) : "r"(addr) : "memory");
+  else if constexpr (VB == 4)
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v[0]) : "r"(addr) : "memory");
+  else if constexpr (VB == 2) {
+    u16 h;
+    asm volatile("ld.shared.u16 %0, [%1];" : "=h"(h) : "r"(addr) : "memory");
+    v[0] = h;
+  } else {
+    u32 b;
+    asm volatile("ld.shared.u8 %0, [%1];" : "=r"(b) : "r"(addr) : "memory");
+    v[0] = b & 0xffu;
+  }
+}
+
+template <class P, int K, bool ST> struct SmVec {
+  // register slot of vector K's element 0 (non-Vec register bits enumerate K) and
+  // its smem element offset (M^{-1} ∘ L of those bits)
+  static constexpr int base_slot() {
+    int s = 0, k = K, t = 0;
+    for (int b = 0; b < P::R; ++b) {
+      bool isvec = false;
+      for (int i = 0; i < P::SV; ++i) if ((ST ? P::VSLOT_LD[i] : P::VSLOT_ST[i]) == b) isvec = true;
+      if (isvec) continue;
+      if ((k >> t) & 1) s |= 1 << b;
+      ++t;
+    }
+    return s;
+  }
+  static constexpr u64 off() {
+    u64 o = 0;
+    int s = base_slot();
+    for (int b = 0; b < P::R; ++b) if ((s >> b) & 1) o ^= (ST ? P::SMOFF_LD[b] : P::SMOFF_ST[b]);
+    return o;
+  }
+  template <int I> static constexpr int slot() {
+    int s = base_slot();
+    for (int i = 0; i < P::SV; ++i) if ((I >> i) & 1) s ^= 1 << (ST ? P::VSLOT_LD[i] : P::VSLOT_ST[i]);
+    return s;
+  }
+};
+
+template <class P, bool ST>
+__device__ __forceinline__ u32 smem_thread_base(u32 lane, u32 warp) {
+  u32 o = 0;
+  static_for<5>([&](auto t) {
+    constexpr int T = decltype(t)::value;
+    constexpr u32 c = u32(ST ? P::SMOFF_LD[P::R + T] : P::SMOFF_ST[P::R + T]);
+    if ((lane >> T) & 1) o ^= c;
+  });
+  static_for<P::WB>([&](auto t) {
+    constexpr int T = decltype(t)::value;
+    constexpr u32 c = u32(ST ? P::SMOFF_LD[P::R + 5 + T] : P::SMOFF_ST[P::R + 5 + T]);
+    if ((warp >> T) & 1) o ^= c;
+  });
+  return o;
+}
+
+// a8 SMEM: st.shared through M^{-1}∘L_ld, barrier,
+// ld.shared through M^{-1}∘L_st; M is the optimal swizzle (conflict-free).
+template <class P>
+__device__ __forceinline__ void xchg_smem(const u32 (&r)[P::NW], u32 (&o)[P::NW], u32 lane, u32 warp, u32 sbase) {
+  constexpr int VE = 1 << P::SV;
+  constexpr int VW = (P::W * VE + 3) / 4;
+  const u32 tst = smem_thread_base<P, true>(lane, warp);
+  static_for<(1 << (P::R - P::SV))>([&](auto k) {
+    constexpr int K = decltype(k)::value;
+    u32 v[VW > 0 ? VW : 1];
+    static_for<VW>([&](auto q) { v[decltype(q)::value] = 0; });
+    static_for<VE>([&](auto i) {
+      constexpr int I = decltype(i)::value;
+      constexpr int S = SmVec<P, K, true>::template slot<I>();
+      set_e<P::W, I>(v, get_e<P::W, S>(r));
+    });
+    constexpr u32 off = u32(SmVec<P, K, true>::off());
+    sts_vec<P::W, P::SV>(sbase + (tst ^ off) * P::W, v);
+  });
+  __syncthreads();
+  const u32 tld = smem_thread_base<P, false>(lane, warp);
+  static_for<(1 << (P::R - P::SV))>([&](auto k) {
+    constexpr int K = decltype(k)::value;
+    u32 v[VW > 0 ? VW : 1];
+    constexpr u32 off = u32(SmVec<P, K, false>::off());
+    lds_vec<P::W, P::SV>(sbase + (tld ^ off) * P::W, v);
+    static_for<VE>([&](auto i) {
+      constexpr int I = decltype(i)::value;
+      constexpr int S = SmVec<P, K, false>::template slot<I>();
+      set_e<P::W, S>(o, get_e<P::W, I>(v));
+    });
+  });
+}
+
+// ------------------------------------------------------------------ tile kernel
+template <class P>
+__device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, u8* __restrict__ dst, u64 ntiles) {
+  extern __shared__ __align__(16) u8 ll_smem[];
+  const u32 lane = threadIdx.x & 31u;
+  const u32 warp = threadIdx.x >> 5;
+  const u64 ld_thr = thread_base<P, true>(lane, warp);
+  const u64 st_thr = thread_base<P, false>(lane, warp);
+  const u32 sbase = u32(__cvta_generic_to_shared(ll_smem));
+  for (u64 t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    const u8* s = src + (tile_base<P, true>(t) ^ ld_thr);
+    u8* d = dst + (tile_base<P, false>(t) ^ st_thr);
+    u32 r[P::NW];
+    // a5: HBM load of the src tile (16-byte vectors; coalesced under σ_ld)
+    static_for<(1 << (P::R - P::VLD))>([&](auto k) {
+      constexpr int K = decltype(k)::value;
+      load_vec<P::W, P::VLD, K>(r, s + LdOff<P, K>::value());
+    });
+    u32 o[P::NW];
+    if constexpr (P::XCHG == 0) {
+      static_for<P::NW>([&](auto q) { o[decltype(q)::value] = r[decltype(q)::value]; });
+    } else if constexpr (P::XCHG == 1) {
+      static_for<P::NW>([&](auto q) { o[decltype(q)::value] = 0; });
+      xchg_regperm<P>(r, o);
+    } else if constexpr (P::XCHG == 2) {
+      xchg_shuffle<P>(r, o, lane);
+    } else {
+      static_for<P::NW>([&](auto q) { o[decltype(q)::value] = 0; });
+      xchg_smem<P>(r, o, lane, warp, sbase);
+    }
+    // a10: HBM store of the dst tile
+    static_for<(1 << (P::R - P::VST))>([&](auto k) {
+      constexpr int K = decltype(k)::value;
+      store_vec<P::W, P::VST, K>(o, d + StOff<P, K>::value());
+    });
+    if constexpr (P::XCHG == 3) __syncthreads();   // smem reuse by the next tile
+  }
+}
+
+// ------------------------------------------------------------------ gather (a11)
+// P:428-432 (G15 reading): per output slot, read idx, locate the source
+// (register candidates, lane) and run 2^{|L_Reg^axis|} shuffle rounds, keeping the
+// value whose candidate equals the source register.
+template <class P>
+__device__ __forceinline__ void ll_gather_body(const u8* __restrict__ src, const u8* __restrict__ idx,
+                                               u8* __restrict__ dst, u64 ntiles) {
+  const u32 lane = threadIdx.x & 31u;
+  const u32 warp = threadIdx.x >> 5;
+  const u64 thr = thread_base<P, true>(lane, warp);           // element offsets (x W below)
+  // axis coordinate contributed by this lane
+  u32 a_lane = 0;
+  static_for<5>([&](auto t) {
+    constexpr int T = decltype(t)::value;
+    if constexpr (P::AXIS_OF_LANE[T] >= 0) if ((lane >> T) & 1) a_lane ^= 1u << P::AXIS_OF_LANE[T];
+  });
+  for (u64 t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    const u64 eoff = tile_base<P, true>(t) ^ thr;
+    u32 r[P::NW];
+    u32 ix[1 << P::R];
+    static_for<(1 << (P::R - P::VLD))>([&](auto k) {
+      constexpr int K = decltype(k)::value;
+      load_vec<P::W, P::VLD, K>(r, src + (eoff ^ LdOff<P, K>::value()) * P::W);
+      load_vec<4, P::VLD, K>(ix, idx + (eoff ^ LdOff<P, K>::value()) * 4);
+    });
+    u32 o[P::NW];
+    static_for<P::NW>([&](auto q) { o[decltype(q)::value] = 0; });
+    static_for<(1 << P::R)>([&](auto e) {
+      constexpr int E = decltype(e)::value;
+      // axis coordinate of slot E's element and its candidate part
+      constexpr u32 a_reg = P::template axis_of_slot<E>();
+      const u32 kidx = ix[E] & ((1u << P::KBITS) - 1u);
+      const u32 dlt = kidx ^ (a_reg ^ a_lane);
+      u32 sl = lane, ct = 0;
+      static_for<P::KBITS>([&](auto tt) {
+        constexpr int T = decltype(tt)::value;
+        const u32 bit = (dlt >> T) & 1u;
+        if constexpr (P::AXIS_LANE_POS[T] >= 0) sl ^= bit << P::AXIS_LANE_POS[T];
+        if constexpr (P::AXIS_CAND_POS[T] >= 0) ct ^= bit << P::AXIS_CAND_POS[T];
+      });
+      ct ^= P::template cand_of_slot<E>();
+      u32 res = 0;
+      static_for<(1 << P::CBITS)>([&](auto c) {
+        constexpr int C = decltype(c)::value;
+        constexpr int S = P::template slot_of<E, C>();
+        const u32 v = __shfl_sync(0xffffffffu, get_e<P::W, S>(r), int(sl));
+        res = (u32(C) == ct) ? v : res;
+      });
+      set_e<P::W, E>(o, res);
+    });
+    static_for<(1 << (P::R - P::VLD))>([&](auto k) {
+      constexpr int K = decltype(k)::value;
+      store_vec<P::W, P::VLD, K>(o, dst + (eoff ^ LdOff<P, K>::value()) * P::W);
+    });
+  }
+}
+
+// ------------------------------------------------------------------ reduce (a12)
+// in-register tree over the Reg axis bits, shfl.bfly over the Lane axis
+// bits, smem over the Warp axis bits — in the layout's bit order (reg, lane, warp
+// ascending); zero-column (broadcast) bits are skipped and de-duplicated at store.
+template <class P>
+__device__ __forceinline__ void ll_reduce_body(const float* __restrict__ src, float* __restrict__ dst, u64 ntiles) {
+  extern __shared__ __align__(16) u8 ll_smem[];
+  float* sm = reinterpret_cast<float*>(ll_smem);
+  const u32 lane = threadIdx.x & 31u;
+  const u32 warp = threadIdx.x >> 5;
+  u64 othr = 0;
+  static_for<5>([&](auto t) {
+    constexpr int T = decltype(t)::value;
+    if ((lane >> T) & 1) othr ^= P::OUT_COL[P::R + T];
+  });
+  static_for<P::WB>([&](auto t) {
+    constexpr int T = decltype(t)::value;
+    if ((warp >> T) & 1) othr ^= P::OUT_COL[P::R + 5 + T];
+  });
+  const bool lane_store = (lane & P::NOSTORE_LANE_MASK) == 0;
+  const bool warp_store = (warp & P::NOSTORE_WARP_MASK) == 0;
+  for (u64 t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    u64 oblk = 0;
+    static_for<P::G>([&](auto g) {
+      constexpr int Gi = decltype(g)::value;
+      if ((t >> Gi) & 1) oblk ^= P::GRID_OUT[Gi];
+    });
+    const u8* s = reinterpret_cast<const u8*>(src) + (tile_base<P, true>(t) ^ thread_base<P, true>(lane, warp));
+    u32 r[1 << P::R];
+    static_for<(1 << (P::R - P::VLD))>([&](auto k) {
+      constexpr int K = decltype(k)::value;
+      load_vec<4, P::VLD, K>(r, s + LdOff<P, K>::value());
+    });
+    // register tree, in the layout's register-bit order
+    static_for<P::NRED_REG>([&](auto i) {
+      constexpr int B = P::RED_REG[decltype(i)::value];
+      static_for<(1 << P::R)>([&](auto e) {
+        constexpr int E = decltype(e)::value;
+        if constexpr (((E >> B) & 1) == 0 && (E & P::template done_mask<decltype(i)::value>()) == 0 &&
+                      (E & P::DUP_REG_MASK) == 0) {
+          r[E] = __float_as_uint(__fadd_rn(__uint_as_float(r[E]), __uint_as_float(r[E | (1 << B)])));
+        }
+      });
+    });
+    // butterfly over the lane axis bits
+    static_for<P::NRED_LANE>([&](auto i) {
+      constexpr int L = P::RED_LANE[decltype(i)::value];
+      static_for<(1 << P::R)>([&](auto e) {
+        constexpr int E = decltype(e)::value;
+        if constexpr ((E & (P::RED_REG_MASK | P::DUP_REG_MASK)) == 0) {
+          const float x = __uint_as_float(r[E]);
+          r[E] = __float_as_uint(__fadd_rn(x, __shfl_xor_sync(0xffffffffu, x, 1 << L)));
+        }
+      });
+    });
+    // warps through smem
+    if constexpr (P::NRED_WARP > 0) {
+      static_for<(1 << P::R)>([&](auto e) {
+        constexpr int E = decltype(e)::value;
+        if constexpr ((E & (P::RED_REG_MASK | P::DUP_REG_MASK)) == 0)
+          sm[(P::template live_index<E>() * (32 << P::WB)) + threadIdx.x] = __uint_as_float(r[E]);
+      });
+      __syncthreads();
+      if ((warp & P::RED_WARP_MASK) == 0) {
+        static_for<(1 << P::R)>([&](auto e) {
+          constexpr int E = decltype(e)::value;
+          if constexpr ((E & (P::RED_REG_MASK | P::DUP_REG_MASK)) == 0) {
+            float v[1 << P::NRED_WARP];
+            static_for<(1 << P::NRED_WARP)>([&](auto m) {
+              constexpr int M = decltype(m)::value;
+              u32 wsel = warp;
+              static_for<P::NRED_WARP>([&](auto q) {
+                constexpr int Q = decltype(q)::value;
+                if ((M >> Q) & 1) wsel |= 1u << P::RED_WARP[Q];
+              });
+              v[M] = sm[(P::template live_index<E>() * (32 << P::WB)) + wsel * 32 + lane];
+            });
+            static_for<P::NRED_WARP>([&](auto q) {
+              constexpr int Q = decltype(q)::value;
+              static_for<(1 << P::NRED_WARP)>([&](auto m) {
+                constexpr int M = decltype(m)::value;
+                if constexpr (((M >> Q) & 1) == 0 && (M & ((1 << Q) - 1)) == 0)
+                  v[M] = __fadd_rn(v[M], v[M | (1 << Q)]);
+              });
+            });
+            r[E] = __float_as_uint(v[0]);
+          }
+        });
+      }
+      __syncthreads();
+    }
+    if (lane_store && warp_store) {
+      static_for<(1 << P::R)>([&](auto e) {
+        constexpr int E = decltype(e)::value;
+        if constexpr ((E & (P::RED_REG_MASK | P::DUP_REG_MASK)) == 0) {
+          constexpr u64 oc = P::template out_of_slot<E>();
+          dst[oblk ^ othr ^ oc] = __uint_as_float(r[E]);
+        }
+      });
+    }
+  }
+}

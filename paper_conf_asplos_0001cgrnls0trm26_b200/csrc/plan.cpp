@@ -1,0 +1,828 @@
+// Conversion planner (rows a3, a4, a6-a9) plus gather (a11) and
+// reduce (a12) plans.
+#include <algorithm>
+#include <cstring>
+#include <sstream>
+
+#include "ll_internal.hpp"
+
+namespace ll {
+
+namespace {
+
+int ilog2(u64 v) { return v ? lead(v) : -1; }
+
+int default_int(const ll_plan_opts* o, int ll_plan_opts::*f, int dflt) {
+  if (!o) return dflt;
+  int v = o->*f;
+  return v > 0 ? v : dflt;
+}
+
+// Bits of the layout belonging to dims of level <= maxlev / == lev.
+std::vector<int> bits_at_level(const Layout& L, int lev_lo, int lev_hi) {
+  std::vector<int> r;
+  int p = 0;
+  for (auto& d : L.in) {
+    int lv = dim_level(d.name);
+    if (lv >= lev_lo && lv <= lev_hi)
+      for (int k = 0; k < d.bits; ++k) r.push_back(p + k);
+    p += d.bits;
+  }
+  return r;
+}
+
+int dev_bits(const Layout& L) { return L.in_bits("dev") + L.in_bits("device"); }
+
+}  // namespace
+
+// ---------------------------------------------------------------------------
+// Pull map and class.  Q[k] = A^+(B.col[k]) with the slack-zero right
+// inverse (rule (2)).  The class is the lowest level λ such that Q can be
+// adjusted by ker(A) (a choice of preimage) to be the identity on every input dim
+// above λ (rule (1)) — equal to the existential class of SURVEY O7.
+// ---------------------------------------------------------------------------
+static int classify_and_adjust(const Layout& A, const Layout& B, std::vector<u64>& Q) {
+  auto Ainv = right_inverse_cols(A);
+  Q.assign(B.cols.size(), 0);
+  for (size_t k = 0; k < B.cols.size(); ++k) Q[k] = apply_cols(Ainv, B.cols[k]);
+  auto ker = kernel_basis(A);
+  for (int lev = 0; lev <= 4; ++lev) {
+    // high-dim mask of A and, for each B bit in a high dim, its A counterpart
+    u64 hiA = 0;
+    int p = 0;
+    for (auto& d : A.in) {
+      if (dim_level(d.name) > lev) for (int t = 0; t < d.bits; ++t) hiA |= u64(1) << (p + t);
+      p += d.bits;
+    }
+    bool ok = true;
+    std::vector<u64> target(B.cols.size(), 0);
+    p = 0;
+    for (auto& d : B.in) {
+      if (dim_level(d.name) > lev) {
+        int pa = A.in_pos(d.name), ba = A.in_bits(d.name);
+        for (int t = 0; t < d.bits; ++t) {
+          if (pa < 0 || t >= ba) { ok = false; break; }
+          target[p + t] = u64(1) << (pa + t);
+        }
+      }
+      if (!ok) break;
+      p += d.bits;
+    }
+    if (!ok) continue;
+    Echelon ek;
+    for (size_t i = 0; i < ker.size(); ++i) ek.insert(ker[i] & hiA, u64(1) << i);
+    std::vector<u64> adj(Q.size());
+    for (size_t k = 0; k < Q.size() && ok; ++k) {
+      u64 delta = (Q[k] & hiA) ^ target[k];
+      u64 c = 0;
+      if (ek.reduce(delta, &c)) { ok = false; break; }
+      u64 fix = 0;
+      for (size_t i = 0; i < ker.size(); ++i) if ((c >> i) & 1) fix ^= ker[i];
+      adj[k] = Q[k] ^ fix;
+    }
+    if (!ok) continue;
+    Q = adj;
+    return lev;
+  }
+  fail(LL_ERR_UNSUPPORTED, "no class found (internal)");
+}
+
+// ---------------------------------------------------------------------------
+// Kernel decomposition (σ_ld, σ_st) of a permutation Q over one CTA tile.
+//   S: src packed bits of the tile (ascending), D: dst packed bits (ascending);
+//   colA(s) = A.cols[s], colB(d) = B.cols[d]; the two sets of logical vectors are
+//   equal.  prefer_warp: logical vectors preferred as kernel warps (in order).
+// Coalesced σ: kreg[0, v) = lowest v tile bits (one 16-byte
+// vector), klane = the next 5 bits (a warp instruction covers 512 contiguous
+// bytes), kernel warps = common vectors where possible, remaining bits -> regs.
+// ---------------------------------------------------------------------------
+static void assign_sigma_coalesced(TilePlan& T, const Layout& A, const Layout& B,
+                                   const std::vector<int>& S, const std::vector<int>& D,
+                                   const std::vector<u64>& prefer_warp, int maxvec, int thread_bytes) {
+  const int n = int(S.size());
+  const int w = T.w;
+  T.n = n;
+  int R = std::max(0, ilog2(std::max(1, thread_bytes / w)));
+  int Wb = n - 5 - R;
+  if (Wb < 0) Wb = 0;
+  if (Wb > 5) Wb = 5;
+  R = n - 5 - Wb;
+  if (R < 0) fail(LL_ERR_UNSUPPORTED, "tile smaller than one warp");
+  T.R = R;
+  T.Wb = Wb;
+  int v = std::min(std::max(0, ilog2(std::max(1, maxvec / w))), R);
+  T.vld = T.vst = v;
+  T.ld_bit.assign(n, -1);
+  T.st_bit.assign(n, -1);
+  for (int b = 0; b < v; ++b) { T.ld_bit[b] = S[b]; T.st_bit[b] = D[b]; }
+  for (int t = 0; t < 5; ++t) { T.ld_bit[R + t] = S[v + t]; T.st_bit[R + t] = D[v + t]; }
+  std::vector<int> restS(S.begin() + v + 5, S.end()), restD(D.begin() + v + 5, D.end());
+  auto findS = [&](u64 c) { for (size_t i = 0; i < restS.size(); ++i) if (A.cols[restS[i]] == c) return int(i); return -1; };
+  auto findD = [&](u64 c) { for (size_t i = 0; i < restD.size(); ++i) if (B.cols[restD[i]] == c) return int(i); return -1; };
+  // 1. vectorisation set: logical vectors that can be register bits on
+  //    both sides — the forced low registers of one side placed among the free
+  //    registers of the other — in A's register order, within max_vec_bytes (G9).
+  std::vector<int> regS, regD;   // free register bits reserved for Vec (packed bits)
+  {
+    std::vector<u64> order;
+    for (int b = 0; b < v; ++b) order.push_back(A.cols[S[b]]);
+    for (int b = 0; b < v; ++b) order.push_back(B.cols[D[b]]);
+    auto forcedA = [&](u64 c) { for (int b = 0; b < v; ++b) if (A.cols[S[b]] == c) return true; return false; };
+    auto forcedB = [&](u64 c) { for (int b = 0; b < v; ++b) if (B.cols[D[b]] == c) return true; return false; };
+    int nv = 0;
+    const int free_regs = R - v;
+    std::vector<u64> chosen;
+    for (u64 c : order) {
+      if ((2 << nv) * w > maxvec) break;
+      if (std::find(chosen.begin(), chosen.end(), c) != chosen.end()) continue;
+      bool inA = forcedA(c), inB = forcedB(c);
+      if (inA && inB) { ++nv; chosen.push_back(c); continue; }
+      int is = inA ? -1 : findS(c), id = inB ? -1 : findD(c);
+      if ((!inA && (is < 0 || int(regS.size()) >= free_regs)) || (!inB && (id < 0 || int(regD.size()) >= free_regs)))
+        continue;
+      if (!inA) { regS.push_back(restS[is]); restS.erase(restS.begin() + is); }
+      if (!inB) { regD.push_back(restD[id]); restD.erase(restD.begin() + id); }
+      ++nv;
+      chosen.push_back(c);
+    }
+  }
+  // 2. kernel warps: common logical vectors first (preferred ones, then ascending src
+  //    position), so that warp-level classes (SHUFFLE/REGPERM) stay available
+  std::vector<u64> cand = prefer_warp;
+  for (int s : restS) cand.push_back(A.cols[s]);
+  int wi = 0;
+  for (u64 c : cand) {
+    if (wi == Wb) break;
+    int is = findS(c), id = findD(c);
+    if (is < 0 || id < 0) continue;
+    T.ld_bit[R + 5 + wi] = restS[is];
+    T.st_bit[R + 5 + wi] = restD[id];
+    restS.erase(restS.begin() + is);
+    restD.erase(restD.begin() + id);
+    ++wi;
+  }
+  // not enough common vectors: take the highest remaining bits on each side
+  while (wi < Wb) {
+    T.ld_bit[R + 5 + wi] = restS.back(); restS.pop_back();
+    T.st_bit[R + 5 + wi] = restD.back(); restD.pop_back();
+    ++wi;
+  }
+  // 3. remaining register bits: reserved Vec bits first, then ascending
+  std::sort(restS.begin(), restS.end());
+  std::sort(restD.begin(), restD.end());
+  regS.insert(regS.end(), restS.begin(), restS.end());
+  regD.insert(regD.end(), restD.begin(), restD.end());
+  for (int b = v; b < R; ++b) { T.ld_bit[b] = regS[b - v]; T.st_bit[b] = regD[b - v]; }
+  T.sigma = SIGMA_COALESCED;
+}
+
+static void assign_sigma_faithful(TilePlan& T, const Layout& A, const Layout& B,
+                                  const std::vector<int>& foldS, const std::vector<int>& foldD, int maxvec) {
+  // kernel hardware = A's (reg, lane, warp) for loads and B's for stores, plus
+  // folded block bits as extra warps.
+  auto reg = [](const Layout& L, const char* nm) {
+    std::vector<int> r; int p = L.in_pos(nm);
+    for (int k = 0; k < L.in_bits(nm); ++k) r.push_back(p + k);
+    return r;
+  };
+  auto rA = reg(A, "reg"), lA = reg(A, "lane"), wA = reg(A, "warp");
+  auto rB = reg(B, "reg"), lB = reg(B, "lane"), wB = reg(B, "warp");
+  if (lA.size() != 5 || lB.size() != 5 || rA.size() != rB.size() || wA.size() != wB.size())
+    fail(LL_ERR_UNSUPPORTED, "faithful σ needs 5 lane bits and equal reg/warp sizes");
+  T.R = int(rA.size());
+  T.Wb = int(wA.size() + foldS.size());
+  T.n = T.R + 5 + T.Wb;
+  if (T.Wb > 5) fail(LL_ERR_UNSUPPORTED, "too many warps");
+  T.ld_bit.clear(); T.st_bit.clear();
+  for (int b : rA) T.ld_bit.push_back(b);
+  for (int b : lA) T.ld_bit.push_back(b);
+  for (int b : wA) T.ld_bit.push_back(b);
+  for (int b : foldS) T.ld_bit.push_back(b);
+  for (int b : rB) T.st_bit.push_back(b);
+  for (int b : lB) T.st_bit.push_back(b);
+  for (int b : wB) T.st_bit.push_back(b);
+  for (int b : foldD) T.st_bit.push_back(b);
+  int v = std::min(std::max(0, ilog2(std::max(1, maxvec / T.w))), T.R);
+  T.vld = T.vst = v;
+  T.sigma = SIGMA_FAITHFUL;
+}
+
+// ---------------------------------------------------------------- exchange plans
+static void plan_regperm(TilePlan& T) {
+  // (B^{-1}∘A)_Reg is a register permutation: out slot e holds the
+  // logical element of L_st slot e, found in the L_ld slot with the same register
+  // logical vectors (lanes and warps agree).
+  std::vector<int> map(T.R, -1);
+  for (int b = 0; b < T.R; ++b)
+    for (int a = 0; a < T.R; ++a)
+      if (T.lcol_ld[a] == T.lcol_st[b]) map[b] = a;
+  for (int b = 0; b < T.R; ++b)
+    if (map[b] < 0) fail(LL_ERR_UNSUPPORTED, "regperm: register sets differ (internal)");
+  T.perm.assign(size_t(1) << T.R, 0);
+  for (u64 e = 0; e < (u64(1) << T.R); ++e) {
+    u64 s = 0;
+    for (int b = 0; b < T.R; ++b) if ((e >> b) & 1) s |= u64(1) << map[b];
+    T.perm[e] = int(s);
+  }
+}
+
+// Fit f(l) = c ⊕ Σ_t l_t·col_t over lane bits; returns false if f is not affine.
+static bool fit_affine(const std::vector<int>& f, int& c, int col[5]) {
+  c = f[0];
+  for (int t = 0; t < 5; ++t) col[t] = f[1 << t] ^ c;
+  for (int l = 0; l < 32; ++l) {
+    int g = c;
+    for (int t = 0; t < 5; ++t) if ((l >> t) & 1) g ^= col[t];
+    if (g != f[l]) return false;
+  }
+  return true;
+}
+
+// Conditional-swap stages realising "slot j <- slot j ⊕ (Σ_t l_t col_t)".
+static void xor_network(const int col[5], std::vector<uint32_t>& lmask, std::vector<int>& xs) {
+  Echelon e;
+  std::vector<u64> basis;
+  for (int t = 0; t < 5; ++t)
+    if (col[t] && e.insert(u64(col[t]), u64(1) << basis.size())) basis.push_back(0);
+  // recompute basis vectors from the echelon combos: store original vectors
+  basis.clear();
+  Echelon e2;
+  std::vector<u64> orig;
+  for (int t = 0; t < 5; ++t)
+    if (col[t] && e2.insert(u64(col[t]), u64(1) << orig.size())) orig.push_back(u64(col[t]));
+  lmask.assign(orig.size(), 0);
+  xs.assign(orig.size(), 0);
+  for (size_t i = 0; i < orig.size(); ++i) xs[i] = int(orig[i]);
+  for (int t = 0; t < 5; ++t) {
+    if (!col[t]) continue;
+    u64 c = 0;
+    e2.reduce(u64(col[t]), &c);   // col[t] = Σ_i c_i orig[i]
+    for (size_t i = 0; i < orig.size(); ++i) if ((c >> i) & 1) lmask[i] |= 1u << t;
+  }
+}
+
+static bool plan_shuffle(TilePlan& T) {
+  // P:371-389 on the kernel layouts L_ld -> L_st within one warp.
+  const int R = T.R, w = T.w;
+  const int u = w < 4 ? ilog2(4 / w) : 0;        // reg bits inside one 32-bit unit
+  if (u > R) return false;
+  for (int b = 0; b < u; ++b) if (T.lcol_ld[b] != T.lcol_st[b]) return false;   // word units
+  T.unit_elems = 1 << u;
+  T.nslot = 1 << (R - u);
+  // V: the common register vectors forming one 32-bit unit.
+  T.V.assign(T.lcol_ld.begin(), T.lcol_ld.begin() + u);
+  std::vector<u64> aThr(T.lcol_ld.begin() + R, T.lcol_ld.begin() + R + 5);
+  std::vector<u64> bThr(T.lcol_st.begin() + R, T.lcol_st.begin() + R + 5);
+  T.I.clear(); T.E.clear(); T.F.clear(); T.G.clear(); T.Rb.clear();
+  for (u64 c : aThr) if (std::find(bThr.begin(), bThr.end(), c) != bThr.end()) T.I.push_back(c);
+  for (u64 c : aThr) if (std::find(T.I.begin(), T.I.end(), c) == T.I.end()) T.E.push_back(c);
+  for (u64 c : bThr) if (std::find(T.I.begin(), T.I.end(), c) == T.I.end()) T.F.push_back(c);
+  std::sort(T.E.begin(), T.E.end());     // "ascending order" (G8)
+  std::sort(T.F.begin(), T.F.end());
+  if (T.E.size() != T.F.size()) return false;
+  for (size_t i = 0; i < T.E.size(); ++i) T.G.push_back(T.E[i] ^ T.F[i]);
+  // R completes V ∪ I ∪ G to the warp space
+  Echelon ech;
+  for (u64 c : T.V) ech.insert(c);
+  for (u64 c : T.I) ech.insert(c);
+  for (u64 c : T.G) ech.insert(c);
+  std::vector<u64> wsp(T.lcol_ld.begin(), T.lcol_ld.begin() + R + 5);
+  std::sort(wsp.begin(), wsp.end());
+  for (u64 c : wsp) if (ech.insert(c)) T.Rb.push_back(c);
+  T.rounds = 1 << T.Rb.size();
+  if (T.rounds != T.nslot) return false;
+  // inverse maps logical -> (reg, lane) for L_ld and L_st (within the warp)
+  auto inv_of = [&](const std::vector<u64>& lc) {
+    Echelon e;
+    for (int b = 0; b < R + 5; ++b) e.insert(lc[b], u64(1) << b);
+    return e;
+  };
+  Echelon invLd = inv_of(T.lcol_ld), invSt = inv_of(T.lcol_st);
+  auto hw_of = [&](const Echelon& e, u64 x) {
+    u64 c = 0;
+    if (e.reduce(x, &c)) fail(LL_ERR_UNSUPPORTED, "shuffle: element outside warp space");
+    return c;
+  };
+  // span(V ∪ I ∪ G) enumerated once
+  std::vector<u64> gens = T.V;
+  gens.insert(gens.end(), T.I.begin(), T.I.end());
+  gens.insert(gens.end(), T.G.begin(), T.G.end());
+  std::vector<u64> spanv(size_t(1) << gens.size(), 0);
+  for (size_t m = 1; m < spanv.size(); ++m) {
+    int t = __builtin_ctzll(m);
+    spanv[m] = spanv[m & (m - 1)] ^ gens[t];
+  }
+  const u64 umask = (u64(1) << u) - 1;
+  std::vector<int> send(32), srcl(32), recv(32);
+  T.send_slot.assign(T.rounds, 0);
+  T.recv_slot.assign(T.rounds, 0);
+  T.src_lane0.assign(T.rounds, 0);
+  int Mcol[5] = {0}, Kcol[5] = {0}, Ncol[5] = {0};
+  for (int r = 0; r < T.rounds; ++r) {
+    u64 base = 0;
+    for (size_t t = 0; t < T.Rb.size(); ++t) if ((r >> t) & 1) base ^= T.Rb[t];
+    std::fill(send.begin(), send.end(), -1);
+    std::fill(srcl.begin(), srcl.end(), -1);
+    for (u64 s : spanv) {
+      u64 x = base ^ s;
+      u64 hl = hw_of(invLd, x), hs = hw_of(invSt, x);
+      int lane_ld = int((hl >> R) & 31), lane_st = int((hs >> R) & 31);
+      int unit_ld = int((hl & ((u64(1) << R) - 1)) >> u);
+      int unit_st = int((hs & ((u64(1) << R) - 1)) >> u);
+      if ((hl & umask) != (hs & umask)) return false;
+      if (send[lane_ld] >= 0 && send[lane_ld] != unit_ld) return false;
+      send[lane_ld] = unit_ld;
+      if (srcl[lane_st] >= 0 && srcl[lane_st] != lane_ld) return false;
+      srcl[lane_st] = lane_ld;
+      recv[lane_st] = unit_st;
+    }
+    for (int l = 0; l < 32; ++l) if (send[l] < 0 || srcl[l] < 0) return false;
+    int c, col[5];
+    if (!fit_affine(send, c, col)) return false;
+    if (r == 0) std::copy(col, col + 5, Mcol);
+    else if (!std::equal(col, col + 5, Mcol)) return false;
+    T.send_slot[r] = c;
+    if (!fit_affine(srcl, c, col)) return false;
+    if (r == 0) std::copy(col, col + 5, Kcol);
+    else if (!std::equal(col, col + 5, Kcol)) return false;
+    T.src_lane0[r] = uint32_t(c);
+    if (!fit_affine(recv, c, col)) return false;
+    if (r == 0) std::copy(col, col + 5, Ncol);
+    else if (!std::equal(col, col + 5, Ncol)) return false;
+    T.recv_slot[r] = c;
+  }
+  for (int t = 0; t < 5; ++t) T.src_lane_col[t] = uint32_t(Kcol[t]);
+  xor_network(Mcol, T.pre_lmask, T.pre_x);
+  xor_network(Ncol, T.post_lmask, T.post_x);
+  // send slots must be a bijection over the rounds (in-place exchange)
+  std::vector<int> seen(T.nslot, 0);
+  for (int r = 0; r < T.rounds; ++r) if (seen[T.send_slot[r]]++) return false;
+  return true;
+}
+
+// Simulated wavefront count (Lemma 9.4 model) of a kernel layout
+// accessing smem through offsets `smoff` (per kernel bit) with `v` vector bits.
+static long sim_wavefronts(const TilePlan& T, const std::vector<u64>& smoff,
+                           const std::vector<int>& vec_slots, long* ideal) {
+  const int R = T.R, w = T.w, v = int(vec_slots.size());
+  const int a = (1 << v) * w;
+  const int lanes_per_phase = a > 4 ? std::max(1, 128 / a) : 32;
+  std::vector<int> other;
+  for (int b = 0; b < R; ++b)
+    if (std::find(vec_slots.begin(), vec_slots.end(), b) == vec_slots.end()) other.push_back(b);
+  long total = 0, id = 0;
+  for (int wi = 0; wi < (1 << T.Wb); ++wi) {
+    u64 wbase = 0;
+    for (int t = 0; t < T.Wb; ++t) if ((wi >> t) & 1) wbase ^= smoff[R + 5 + t];
+    for (u64 ri = 0; ri < (u64(1) << other.size()); ++ri) {
+      u64 rbase = wbase;
+      for (size_t t = 0; t < other.size(); ++t) if ((ri >> t) & 1) rbase ^= smoff[other[t]];
+      u64 addr[32];
+      for (int l = 0; l < 32; ++l) {
+        u64 o = rbase;
+        for (int t = 0; t < 5; ++t) if ((l >> t) & 1) o ^= smoff[R + t];
+        addr[l] = o * w;
+      }
+      for (int p0 = 0; p0 < 32; p0 += lanes_per_phase) {
+        std::map<int, std::vector<u64>> bank;
+        for (int l = p0; l < p0 + lanes_per_phase; ++l)
+          for (int b = 0; b < a; b += std::min(a, 4)) {
+            u64 word = (addr[l] + b) / 4;
+            auto& vv = bank[int(word % 32)];
+            if (std::find(vv.begin(), vv.end(), word) == vv.end()) vv.push_back(word);
+          }
+        size_t mx = 0;
+        for (auto& kv : bank) mx = std::max(mx, kv.second.size());
+        total += long(mx);
+        id += (lanes_per_phase * a + 127) / 128;
+      }
+    }
+  }
+  if (ideal) *ideal = id;
+  return total;
+}
+
+static void plan_smem(TilePlan& T, int maxvec) {
+  // Optimal swizzling (appendix) on the kernel layouts.
+  const int R = T.R, w = T.w, n = T.n;
+  // 1. Vec: common register vectors, in L_ld register order, within max_vec_bytes.
+  T.sw_vec.clear(); T.vec_slot_ld.clear(); T.vec_slot_st.clear();
+  for (int b = 0; b < R; ++b) {
+    u64 c = T.lcol_ld[b];
+    int bs = -1;
+    for (int q = 0; q < R; ++q) if (T.lcol_st[q] == c) bs = q;
+    if (bs < 0) continue;
+    if ((int(1) << (T.sw_vec.size() + 1)) * w > maxvec) break;
+    T.sw_vec.push_back(c);
+    T.vec_slot_ld.push_back(b);
+    T.vec_slot_st.push_back(bs);
+  }
+  const int v = int(T.sw_vec.size());
+  T.sm_v = v;
+  const int vec_bytes = (1 << v) * w;
+  // 2. b = log2(128 / (2^v w))
+  int b = std::max(0, ilog2(u64(std::max(1, 128 / vec_bytes))));
+  if (b > n - v) b = n - v;
+  // 3. A_Bank, B_Bank: drop the last log2 max(1, 2^v w / 4) thread vectors
+  int drop = ilog2(u64(std::max(1, vec_bytes / 4)));
+  std::vector<u64> aThr(T.lcol_ld.begin() + R, T.lcol_ld.begin() + R + 5);
+  std::vector<u64> bThr(T.lcol_st.begin() + R, T.lcol_st.begin() + R + 5);
+  std::vector<u64> aBank(aThr.begin(), aThr.end() - drop), bBank(bThr.begin(), bThr.end() - drop);
+  // 4. E, F, H
+  std::vector<u64> E, F;
+  for (u64 c : aBank) if (std::find(bBank.begin(), bBank.end(), c) == bBank.end()) E.push_back(c);
+  for (u64 c : bBank) if (std::find(aBank.begin(), aBank.end(), c) == aBank.end()) F.push_back(c);
+  if (E.size() > F.size()) std::swap(E, F);
+  std::sort(E.begin(), E.end());
+  std::sort(F.begin(), F.end());
+  T.sw_H.clear();
+  for (size_t i = 0; i < E.size(); ++i) T.sw_H.push_back(E[i] ^ F[i]);
+  // 5. C completes span(Vec ∪ A_Bank ∪ B_Bank) inside the tile space
+  std::vector<u64> space(T.lcol_ld.begin(), T.lcol_ld.end());
+  std::sort(space.begin(), space.end());
+  Echelon ep;
+  for (u64 c : T.sw_vec) ep.insert(c);
+  for (u64 c : aBank) ep.insert(c);
+  for (u64 c : bBank) ep.insert(c);
+  T.sw_C.clear();
+  for (u64 c : space) if (ep.insert(c)) T.sw_C.push_back(c);
+  // 6. Seg: ℓ vectors from H then C; else unused A_Bank, then A_Thr (G14)
+  const int ell = n - v - b;
+  Echelon es;
+  for (u64 c : T.sw_vec) es.insert(c);
+  T.sw_seg.clear();
+  auto try_add = [&](u64 c) {
+    if (int(T.sw_seg.size()) < ell && es.insert(c)) T.sw_seg.push_back(c);
+  };
+  for (u64 c : T.sw_H) try_add(c);
+  for (u64 c : T.sw_C) try_add(c);
+  for (u64 c : aBank) try_add(c);
+  for (u64 c : aThr) try_add(c);
+  for (u64 c : space) try_add(c);
+  // 7. Bank completes span(Vec ∪ Seg)
+  T.sw_bank.clear();
+  for (u64 c : space) if (es.insert(c)) T.sw_bank.push_back(c);
+  if (int(T.sw_vec.size() + T.sw_bank.size() + T.sw_seg.size()) != n)
+    fail(LL_ERR_UNSUPPORTED, "swizzle: basis incomplete (internal)");
+  // M: offset bit -> logical (Vec, Bank, Seg); invert to get smem offsets.
+  std::vector<u64> M = T.sw_vec;
+  M.insert(M.end(), T.sw_bank.begin(), T.sw_bank.end());
+  M.insert(M.end(), T.sw_seg.begin(), T.sw_seg.end());
+  Echelon em;
+  for (size_t o = 0; o < M.size(); ++o) em.insert(M[o], u64(1) << o);
+  auto minv = [&](u64 x) { u64 c = 0; if (em.reduce(x, &c)) fail(LL_ERR_UNSUPPORTED, "swizzle: not invertible"); return c; };
+  T.smoff_ld.resize(n);
+  T.smoff_st.resize(n);
+  for (int k = 0; k < n; ++k) { T.smoff_ld[k] = minv(T.lcol_ld[k]); T.smoff_st[k] = minv(T.lcol_st[k]); }
+  for (int i = 0; i < v; ++i)
+    if (T.smoff_ld[T.vec_slot_ld[i]] != (u64(1) << i) || T.smoff_st[T.vec_slot_st[i]] != (u64(1) << i))
+      fail(LL_ERR_UNSUPPORTED, "swizzle: vector bits not lowest (internal)");
+  T.smem_elems = u64(1) << n;
+  long id1 = 0, id2 = 0;
+  T.predicted_wavefronts_st = sim_wavefronts(T, T.smoff_ld, T.vec_slot_ld, &id1);
+  T.predicted_wavefronts_ld = sim_wavefronts(T, T.smoff_st, T.vec_slot_st, &id2);
+  T.ideal_wavefronts = id1 + id2;
+}
+
+// ---------------------------------------------------------------------------
+static void build_tile(ConvPlan& P, const std::vector<int>& S0, const std::vector<int>& D0,
+                       std::vector<int> gridS, std::vector<int> gridD, const ll_plan_opts* opts,
+                       bool in_cta) {
+  const Layout &A = P.A, &B = P.B;
+  TilePlan& T = P.tile;
+  T = TilePlan();
+  T.w = P.w;
+  int maxvec = default_int(opts, &ll_plan_opts::max_vec_bytes, 16);
+  int sigma = opts ? opts->sigma : 0;
+  int tile_bytes = default_int(opts, &ll_plan_opts::tile_bytes, 16384);
+  std::vector<int> S = S0, D = D0;
+  // fold low grid bits into the tile while it is small (common vectors)
+  std::vector<int> foldS, foldD;
+  while (!gridD.empty() && (u64(1) << S.size()) * u64(P.w) < u64(tile_bytes) && S.size() < 20) {
+    foldS.push_back(gridS.front()); foldD.push_back(gridD.front());
+    S.push_back(gridS.front()); D.push_back(gridD.front());
+    gridS.erase(gridS.begin()); gridD.erase(gridD.begin());
+  }
+  std::vector<int> Ss = S, Ds = D;
+  std::sort(Ss.begin(), Ss.end());
+  std::sort(Ds.begin(), Ds.end());
+  if (S.size() < 5) fail(LL_ERR_UNSUPPORTED, "tile smaller than a warp");
+  if (sigma == SIGMA_FAITHFUL && in_cta) {
+    assign_sigma_faithful(T, A, B, foldS, foldD, maxvec);
+  } else {
+    std::vector<u64> prefer;
+    int pw = A.in_pos("warp");
+    for (int k = 0; k < A.in_bits("warp"); ++k) prefer.push_back(A.cols[pw + k]);
+    for (int s : foldS) prefer.push_back(A.cols[s]);
+    int thread_bytes = default_int(opts, &ll_plan_opts::thread_bytes, 256);
+    assign_sigma_coalesced(T, A, B, Ss, Ds, prefer, maxvec, thread_bytes);
+  }
+  T.grid_src_bit = gridS;
+  T.grid_dst_bit = gridD;
+  T.lcol_ld.resize(T.n);
+  T.lcol_st.resize(T.n);
+  for (int b = 0; b < T.n; ++b) { T.lcol_ld[b] = A.cols[T.ld_bit[b]]; T.lcol_st[b] = B.cols[T.st_bit[b]]; }
+  // exchange class of L_ld -> L_st
+  bool same_lane = true, same_warp = true, same_reg = true;
+  for (int t = 0; t < 5; ++t) same_lane &= T.lcol_ld[T.R + t] == T.lcol_st[T.R + t];
+  for (int t = 0; t < T.Wb; ++t) same_warp &= T.lcol_ld[T.R + 5 + t] == T.lcol_st[T.R + 5 + t];
+  for (int t = 0; t < T.R; ++t) same_reg &= T.lcol_ld[t] == T.lcol_st[t];
+  int force = opts ? opts->force_class : -1;
+  if (force == LL_CLASS_SMEM) {
+    T.xchg = X_SMEM;
+  } else if (same_lane && same_warp) {
+    T.xchg = same_reg ? X_COPY : X_REGPERM;
+  } else if (same_warp && plan_shuffle(T)) {
+    T.xchg = X_SHUFFLE;
+  } else {
+    if (force == LL_CLASS_SHUFFLE) fail(LL_ERR_UNSUPPORTED, "SHUFFLE forced but the kernel layouts need smem");
+    T.xchg = X_SMEM;
+  }
+  if (T.xchg == X_REGPERM) plan_regperm(T);
+  if (T.xchg == X_SMEM) plan_smem(T, maxvec);
+  if (T.xchg == X_SMEM && (T.smem_elems * u64(T.w)) > 200 * 1024)
+    fail(LL_ERR_UNSUPPORTED, "smem tile too large");
+  P.smem_bytes = T.xchg == X_SMEM ? int(T.smem_elems * T.w) : 0;
+}
+
+// CTA class (Q mixes block/offset bits): choose the dst bits a CTA owns so that both
+// the loads and the stores are coalesced.
+static void choose_cta_tile(const ConvPlan& P, const std::vector<int>& pi, int nloc, int c_bits,
+                            int target_bits, std::vector<int>& S, std::vector<int>& D,
+                            std::vector<int>& gS, std::vector<int>& gD) {
+  std::vector<int> inv(nloc, -1);
+  for (int k = 0; k < nloc; ++k) inv[pi[k]] = k;
+  std::vector<char> inT(nloc, 0);
+  for (int k = 0; k < std::min(c_bits, nloc); ++k) { inT[k] = 1; inT[inv[k]] = 1; }
+  int cnt = 0;
+  for (int k = 0; k < nloc; ++k) cnt += inT[k];
+  for (int k = 0; k < nloc && cnt < target_bits; ++k) if (!inT[k]) { inT[k] = 1; ++cnt; }
+  S.clear(); D.clear(); gS.clear(); gD.clear();
+  for (int k = 0; k < nloc; ++k) {
+    if (inT[k]) { D.push_back(k); S.push_back(pi[k]); }
+    else { gD.push_back(k); gS.push_back(pi[k]); }
+  }
+}
+
+std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, const ll_plan_opts* opts) {
+  if (w != 1 && w != 2 && w != 4 && w != 8) fail(LL_ERR_INVALID_ARG, "elem_bytes must be 1, 2, 4 or 8");
+  if (A.out != B.out) fail(LL_ERR_DIM_MISMATCH, "A and B must have the same output dims");
+  for (auto* L : {&A, &B}) {
+    for (auto& d : L->in)
+      if (dim_level(d.name) < 0) fail(LL_ERR_INVALID_ARG, "unknown input dim name '" + d.name + "'");
+    if (L->d_in() > 62) fail(LL_ERR_INVALID_ARG, "more than 62 input bits");
+    int pd = L->in_pos("dev");
+    if (pd >= 0 && pd + L->in_bits("dev") != L->d_in()) fail(LL_ERR_INVALID_ARG, "dev must be the last input dim");
+  }
+  if (!A.surjective()) fail(LL_ERR_NOT_SURJECTIVE, "A is not surjective (Def 4.5, P:194)");
+  auto P = std::make_unique<ConvPlan>();
+  P->A = A; P->B = B; P->w = w;
+  int lev = classify_and_adjust(A, B, P->Q);
+  bool noop = A.in == B.in && A.cols == B.cols;
+  P->cls = noop ? LL_CLASS_NOOP : ll_class(LL_CLASS_REGPERM + lev);
+  const int dA = dev_bits(A), dB = dev_bits(B);
+  const int nA = A.d_in() - dA, nB = B.d_in() - dB;
+  P->src_elems = u64(1) << nA;
+  P->dst_elems = u64(1) << nB;
+  P->dev_bits = std::max(dA, dB);
+  if (noop) { P->exec = EXEC_NOOP; return P; }
+  if (P->cls == LL_CLASS_DEVICE) {
+    P->exec = EXEC_DEVICE;
+    return P;   // completed by plan_device (dist.cpp)
+  }
+  // local pull map: dst local bit -> src local index (no dev components by class)
+  bool generic = opts && opts->generic;
+  bool perm = A.unit_columns() && B.unit_columns() && nA == nB;
+  if (!generic && perm) {
+    std::vector<int> pi(nB);
+    for (int k = 0; k < nB; ++k) {
+      u64 q = P->Q[k];
+      if (popc(q) != 1 || lead(q) >= nA) { perm = false; break; }
+      pi[k] = lead(q);
+    }
+    if (perm) {
+      try {
+        std::vector<int> S, D, gS, gD;
+        if (lev <= 2) {
+          D = bits_at_level(B, 0, 2);
+          for (int k : D) S.push_back(pi[k]);
+          for (int k : bits_at_level(B, 3, 3)) { gD.push_back(k); gS.push_back(pi[k]); }
+          build_tile(*P, S, D, gS, gD, opts, true);
+        } else {
+          int maxvec = default_int(opts, &ll_plan_opts::max_vec_bytes, 16);
+          int v = std::max(0, ilog2(u64(std::max(1, maxvec / w))));
+          int tb = default_int(opts, &ll_plan_opts::tile_bytes, 16384);
+          int target = std::max(v + 5, ilog2(u64(std::max(1, tb / w))));
+          int c_bits = v + 5;
+          choose_cta_tile(*P, pi, nB, c_bits, target, S, D, gS, gD);
+          if (int(S.size()) > 15) {   // too large for smem: coalesce to 128-byte lines only
+            choose_cta_tile(*P, pi, nB, v + 3, target, S, D, gS, gD);
+          }
+          build_tile(*P, S, D, gS, gD, opts, false);
+        }
+        P->exec = EXEC_TILE;
+        return P;
+      } catch (const Error& e) {
+        if (opts && opts->force_class >= 0) throw;
+        // fall through to the generic kernel
+      }
+    }
+  }
+  P->exec = EXEC_GENERIC;
+  return P;
+}
+
+// ---------------------------------------------------------------- describe
+static std::string vec_json(const std::vector<u64>& v) {
+  std::ostringstream o;
+  o << "[";
+  for (size_t i = 0; i < v.size(); ++i) o << (i ? "," : "") << v[i];
+  o << "]";
+  return o.str();
+}
+template <class T>
+static std::string ivec_json(const std::vector<T>& v) {
+  std::ostringstream o;
+  o << "[";
+  for (size_t i = 0; i < v.size(); ++i) o << (i ? "," : "") << v[i];
+  o << "]";
+  return o.str();
+}
+
+std::string describe(const ConvPlan& P) {
+  static const char* cls[] = {"NOOP", "REGPERM", "SHUFFLE", "SMEM", "CTA", "DEVICE"};
+  static const char* ex[] = {"noop", "tile", "generic", "device"};
+  static const char* xc[] = {"copy", "regperm", "shuffle", "smem"};
+  std::ostringstream o;
+  o << "{\"class\":\"" << cls[P.cls] << "\",\"exec\":\"" << ex[P.exec] << "\",\"elem_bytes\":" << P.w
+    << ",\"src_elems\":" << P.src_elems << ",\"dst_elems\":" << P.dst_elems
+    << ",\"Q\":" << vec_json(P.Q);
+  if (P.exec == EXEC_TILE) {
+    const TilePlan& T = P.tile;
+    o << ",\"tile\":{\"xchg\":\"" << xc[T.xchg] << "\",\"sigma\":\"" << (T.sigma ? "faithful" : "coalesced")
+      << "\",\"n\":" << T.n << ",\"R\":" << T.R << ",\"warp_bits\":" << T.Wb << ",\"threads\":" << T.threads()
+      << ",\"vld\":" << T.vld << ",\"vst\":" << T.vst << ",\"ctas\":" << (u64(1) << T.grid_dst_bit.size())
+      << ",\"ld_bit\":" << ivec_json(T.ld_bit) << ",\"st_bit\":" << ivec_json(T.st_bit)
+      << ",\"L_ld\":" << vec_json(T.lcol_ld) << ",\"L_st\":" << vec_json(T.lcol_st)
+      << ",\"grid_src_bit\":" << ivec_json(T.grid_src_bit) << ",\"grid_dst_bit\":" << ivec_json(T.grid_dst_bit);
+    if (T.xchg == X_SHUFFLE)
+      o << ",\"V\":" << vec_json(T.V) << ",\"I\":" << vec_json(T.I) << ",\"E\":" << vec_json(T.E)
+        << ",\"F\":" << vec_json(T.F) << ",\"G\":" << vec_json(T.G) << ",\"R_basis\":" << vec_json(T.Rb)
+        << ",\"rounds\":" << T.rounds << ",\"pre_stages\":" << T.pre_x.size()
+        << ",\"post_stages\":" << T.post_x.size() << ",\"unit_elems\":" << T.unit_elems;
+    if (T.xchg == X_SMEM)
+      o << ",\"Vec\":" << vec_json(T.sw_vec) << ",\"Bank\":" << vec_json(T.sw_bank) << ",\"Seg\":" << vec_json(T.sw_seg)
+        << ",\"H\":" << vec_json(T.sw_H) << ",\"C\":" << vec_json(T.sw_C)
+        << ",\"smem_bytes\":" << T.smem_elems * T.w
+        << ",\"wavefronts_st\":" << T.predicted_wavefronts_st << ",\"wavefronts_ld\":" << T.predicted_wavefronts_ld
+        << ",\"ideal_wavefronts\":" << T.ideal_wavefronts;
+    o << "}";
+  }
+  if (P.exec == EXEC_DEVICE) {
+    o << ",\"dev_bits\":" << P.dev_bits << ",\"workspace_bytes\":" << P.workspace_bytes;
+    if (P.pack) o << ",\"pack\":" << describe(*P.pack);
+    if (P.unpack) o << ",\"unpack\":" << describe(*P.unpack);
+  }
+  o << "}";
+  return o.str();
+}
+
+// ---------------------------------------------------------------------------
+// Gather (§5.5)
+// ---------------------------------------------------------------------------
+std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const ll_plan_opts* opts) {
+  if (w != 1 && w != 2 && w != 4 && w != 8) fail(LL_ERR_INVALID_ARG, "elem_bytes must be 1, 2, 4 or 8");
+  if (axis < 0 || axis >= int(L.out.size())) fail(LL_ERR_INVALID_ARG, "axis out of range");
+  if (!L.unit_columns()) fail(LL_ERR_UNSUPPORTED, "gather: L must be a bijective distributed layout");
+  if (L.in_bits("lane") != 5) fail(LL_ERR_UNSUPPORTED, "gather: 5 lane bits required");
+  auto G = std::make_unique<GatherPlan>();
+  G->L = L; G->axis = axis; G->w = w;
+  const int sh = L.out_shift(axis), ab = L.out[axis].bits;
+  const u64 amask = ((ab >= 64) ? ~u64(0) : ((u64(1) << ab) - 1)) << sh;
+  auto tileb = bits_at_level(L, 0, 2);
+  auto blk = bits_at_level(L, 3, 3);
+  // in-tile axis bits must be the low K bits of the axis coordinate (O10)
+  std::vector<int> axis_bits;
+  for (int k : tileb) if (L.cols[k] & amask) axis_bits.push_back(k);
+  G->K_bits = int(axis_bits.size());
+  for (int t = 0; t < G->K_bits; ++t) {
+    bool found = false;
+    for (int k : axis_bits) if (L.cols[k] == (u64(1) << (sh + t))) found = true;
+    if (!found) fail(LL_ERR_UNSUPPORTED, "gather: in-tile axis bits must be the low axis bits");
+  }
+  for (int k : bits_at_level(L, 2, 2))
+    if (L.cols[k] & amask) fail(LL_ERR_UNSUPPORTED, "gather: L_Wrp^axis != 0 (P:430)");
+  // kernel decomposition: faithful (L itself) or coalesced σ; pick the one with
+  // fewer shuffle candidates 2^{|L_Reg^axis|}, coalesced on ties.
+  const int ev = std::max(w, 4);   // idx is int32: one σ for both
+  int maxvec = default_int(opts, &ll_plan_opts::max_vec_bytes, 16);
+  int v = std::min(ilog2(u64(std::max(1, maxvec / ev))), L.in_bits("reg"));
+  auto regb = bits_at_level(L, 0, 0), laneb = bits_at_level(L, 1, 1), warpb = bits_at_level(L, 2, 2);
+  const int R = int(regb.size());
+  auto cand_of = [&](const std::vector<int>& hw) {
+    int c = 0;
+    for (int b = 0; b < R; ++b) if (L.cols[hw[b]] & amask) ++c;
+    return c;
+  };
+  std::vector<int> faith;
+  for (int k : regb) faith.push_back(k);
+  for (int k : laneb) faith.push_back(k);
+  for (int k : warpb) faith.push_back(k);
+  std::vector<int> coal(faith.size());
+  // tile bits in packed order: reg (0..R-1), lane (R..R+4), warp
+  std::vector<int> Ts = tileb;
+  std::sort(Ts.begin(), Ts.end());
+  for (int b = 0; b < v; ++b) coal[b] = Ts[b];
+  for (int t = 0; t < 5; ++t) coal[R + t] = Ts[v + t];
+  {
+    std::vector<int> rest(Ts.begin() + v + 5, Ts.end());
+    // warps keep L's warp bits (axis-free) so L_Wrp^axis stays 0
+    std::vector<int> wr;
+    for (int k : warpb) { wr.push_back(k); rest.erase(std::find(rest.begin(), rest.end(), k)); }
+    for (int b = v; b < R; ++b) coal[b] = rest[b - v];
+    for (size_t t = 0; t < wr.size(); ++t) coal[R + 5 + t] = wr[t];
+    // coalesced σ only valid if the warp bits were not consumed by reg/lane positions
+    for (int b = 0; b < R + 5; ++b)
+      if (std::find(warpb.begin(), warpb.end(), coal[b]) != warpb.end()) { coal.clear(); break; }
+  }
+  int sigma = opts ? opts->sigma : 0;
+  bool use_coal = !coal.empty() && sigma != SIGMA_FAITHFUL && cand_of(coal) <= cand_of(faith);
+  G->hw_bit = use_coal ? coal : faith;
+  G->sigma = use_coal ? SIGMA_COALESCED : SIGMA_FAITHFUL;
+  G->R = R;
+  G->Wb = int(warpb.size());
+  G->v = use_coal ? v : std::min(ilog2(u64(std::max(1, maxvec / ev))), R);
+  G->grid_bit = blk;
+  G->lcol.resize(G->hw_bit.size());
+  for (size_t b = 0; b < G->hw_bit.size(); ++b) G->lcol[b] = L.cols[G->hw_bit[b]];
+  G->axis_reg_pos.assign(G->K_bits, -1);
+  G->axis_lane_pos.assign(G->K_bits, -1);
+  G->axis_of_reg.assign(R, -1);
+  G->axis_of_lane.assign(5, -1);
+  G->cand_bits = 0;
+  for (int t = 0; t < G->K_bits; ++t) {
+    u64 c = u64(1) << (sh + t);
+    for (int b = 0; b < R; ++b) if (G->lcol[b] == c) { G->axis_reg_pos[t] = b; G->axis_of_reg[b] = t; ++G->cand_bits; }
+    for (int l = 0; l < 5; ++l) if (G->lcol[R + l] == c) { G->axis_lane_pos[t] = l; G->axis_of_lane[l] = t; }
+  }
+  return G;
+}
+
+// ---------------------------------------------------------------------------
+// Reduce: faithful kernel layout so the fixed order (reg, lane, warp
+// ascending) is exactly the layout's.
+// ---------------------------------------------------------------------------
+std::unique_ptr<ReducePlan> plan_reduce(const Layout& L, int axis, const ll_plan_opts* opts) {
+  (void)opts;
+  if (axis < 0 || axis >= int(L.out.size())) fail(LL_ERR_INVALID_ARG, "axis out of range");
+  if (!L.distributed()) fail(LL_ERR_UNSUPPORTED, "reduce: L must be a distributed layout (Def 4.10)");
+  if (L.in_bits("lane") != 5) fail(LL_ERR_UNSUPPORTED, "reduce: 5 lane bits required");
+  if (L.in.size() < 1 || L.in[0].name != "reg") fail(LL_ERR_UNSUPPORTED, "reduce: dims must be reg, lane, warp[, block]");
+  auto Rp = std::make_unique<ReducePlan>();
+  Rp->L = L; Rp->axis = axis;
+  const int sh = L.out_shift(axis), ab = L.out[axis].bits;
+  const u64 amask = ((u64(1) << ab) - 1) << sh;
+  Rp->R = L.in_bits("reg");
+  Rp->Wb = L.in_bits("warp");
+  // K: number of in-tile (non-block) axis bits; they must be the low axis bits
+  int K = 0;
+  for (int k : bits_at_level(L, 0, 2)) if (L.cols[k] & amask) ++K;
+  for (int t = 0; t < K; ++t) {
+    bool f = false;
+    for (int k : bits_at_level(L, 0, 2)) if (L.cols[k] == (u64(1) << (sh + t))) f = true;
+    if (!f) fail(LL_ERR_UNSUPPORTED, "reduce: in-tile axis bits must be the low axis bits");
+  }
+  auto classify_bits = [&](int lev, std::vector<int>& red) {
+    for (int k : bits_at_level(L, lev, lev)) {
+      if (L.cols[k] == 0) Rp->dup_bits.push_back(k);
+      else if (L.cols[k] & amask) red.push_back(k);
+    }
+  };
+  classify_bits(0, Rp->red_reg);
+  classify_bits(1, Rp->red_lane);
+  classify_bits(2, Rp->red_warp);
+  for (int k : bits_at_level(L, 3, 3)) {
+    if (L.cols[k] == 0) Rp->dup_bits.push_back(k);
+    else Rp->grid_bit.push_back(k);
+  }
+  // output flat offset per hardware bit: logical x -> row-major output with the axis
+  // replaced by its block part (axis / K)
+  Rp->out_col.assign(L.d_in(), 0);
+  for (int k = 0; k < L.d_in(); ++k) {
+    u64 c = L.cols[k];
+    if (!c || (std::find(Rp->red_reg.begin(), Rp->red_reg.end(), k) != Rp->red_reg.end()) ||
+        (std::find(Rp->red_lane.begin(), Rp->red_lane.end(), k) != Rp->red_lane.end()) ||
+        (std::find(Rp->red_warp.begin(), Rp->red_warp.end(), k) != Rp->red_warp.end()))
+      continue;
+    u64 lower = c & ((u64(1) << sh) - 1);
+    u64 a = (c & amask) >> sh;
+    u64 upper = c >> (sh + ab);
+    int na_bits = ab - K;
+    Rp->out_col[k] = (((upper << na_bits) | (a >> K)) << sh) | lower;
+  }
+  Rp->out_elems = u64(1) << (L.d_out() - K);
+  Rp->smem_bytes = Rp->red_warp.empty() ? 0 : int((u64(4) << (L.in_bits("reg") + 5 + Rp->Wb)));
+  return Rp;
+}
+
+}  // namespace ll

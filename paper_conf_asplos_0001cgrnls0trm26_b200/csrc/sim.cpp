@@ -1,0 +1,100 @@
+// Host emulation of a specialised tile plan's schedule (test hook ll_plan_simulate).
+// It executes exactly the tables the kernel is specialised with — σ_ld / σ_st
+// addresses, the pre / post conditional-swap networks, the shuffle rounds with their
+// source lanes and slots, the swizzled smem offsets — one warp at a time, so the
+// planner can be validated without a GPU.  It is never used by ll_convert.
+#include <cstring>
+
+#include "ll_internal.hpp"
+
+namespace ll {
+
+void simulate_tile(const ConvPlan& P, const uint8_t* src, uint8_t* dst) {
+  if (P.exec != EXEC_TILE) fail(LL_ERR_UNSUPPORTED, "simulate: not a tile plan");
+  const TilePlan& T = P.tile;
+  const int w = T.w, R = T.R, n = T.n;
+  const int E = 1 << R, NT = T.threads();
+  const u64 ntiles = u64(1) << T.grid_dst_bit.size();
+  auto off = [&](const std::vector<int>& bits, u64 hw) {
+    u64 o = 0;
+    for (int b = 0; b < n; ++b) if ((hw >> b) & 1) o |= u64(1) << bits[b];
+    return o;
+  };
+  std::vector<uint64_t> in(size_t(NT) * E), out(size_t(NT) * E);
+  std::vector<uint8_t> smem(T.xchg == X_SMEM ? T.smem_elems * w : 0);
+  auto getv = [&](const uint8_t* p) { uint64_t v = 0; std::memcpy(&v, p, w); return v; };
+  for (u64 t = 0; t < ntiles; ++t) {
+    u64 sb = 0, db = 0;
+    for (size_t g = 0; g < T.grid_dst_bit.size(); ++g)
+      if ((t >> g) & 1) { sb |= u64(1) << T.grid_src_bit[g]; db |= u64(1) << T.grid_dst_bit[g]; }
+    for (int th = 0; th < NT; ++th)
+      for (int e = 0; e < E; ++e) {
+        u64 hw = u64(e) | (u64(th) << R);
+        in[size_t(th) * E + e] = getv(src + (sb | off(T.ld_bit, hw)) * w);
+      }
+    if (T.xchg == X_COPY) {
+      out = in;
+    } else if (T.xchg == X_REGPERM) {
+      for (int th = 0; th < NT; ++th)
+        for (int e = 0; e < E; ++e) out[size_t(th) * E + e] = in[size_t(th) * E + T.perm[e]];
+    } else if (T.xchg == X_SHUFFLE) {
+      const int U = T.unit_elems;
+      for (int wp = 0; wp < (1 << T.Wb); ++wp) {
+        // pre network: slot j <-> j ^ X when parity(lane & mask)
+        auto net = [&](std::vector<uint64_t>& buf, const std::vector<uint32_t>& mk, const std::vector<int>& xs) {
+          for (size_t s = 0; s < xs.size(); ++s)
+            for (int l = 0; l < 32; ++l) {
+              if (!parity(u64(l) & mk[s])) continue;
+              uint64_t* r = &buf[size_t(wp * 32 + l) * E];
+              for (int j = 0; j < T.nslot; ++j) {
+                int k = j ^ xs[s];
+                if (k > j) for (int q = 0; q < U; ++q) std::swap(r[j * U + q], r[k * U + q]);
+              }
+            }
+        };
+        net(in, T.pre_lmask, T.pre_x);
+        for (int rr = 0; rr < T.rounds; ++rr) {
+          int S = T.send_slot[rr];
+          uint64_t sent[32][8];
+          for (int l = 0; l < 32; ++l)
+            for (int q = 0; q < U; ++q) sent[l][q] = in[size_t(wp * 32 + l) * E + S * U + q];
+          for (int l = 0; l < 32; ++l) {
+            uint32_t lx = 0;
+            for (int b = 0; b < 5; ++b) if ((l >> b) & 1) lx ^= T.src_lane_col[b];
+            int sl = int((T.src_lane0[rr] ^ lx) & 31);
+            for (int q = 0; q < U; ++q) in[size_t(wp * 32 + l) * E + S * U + q] = sent[sl][q];
+          }
+        }
+        for (int l = 0; l < 32; ++l)
+          for (int rr = 0; rr < T.rounds; ++rr)
+            for (int q = 0; q < U; ++q)
+              out[size_t(wp * 32 + l) * E + T.recv_slot[rr] * U + q] = in[size_t(wp * 32 + l) * E + T.send_slot[rr] * U + q];
+        net(out, T.post_lmask, T.post_x);
+      }
+    } else {
+      for (int th = 0; th < NT; ++th)
+        for (int e = 0; e < E; ++e) {
+          u64 hw = u64(e) | (u64(th) << R);
+          u64 so = 0;
+          for (int b = 0; b < n; ++b) if ((hw >> b) & 1) so ^= T.smoff_ld[b];
+          std::memcpy(&smem[so * w], &in[size_t(th) * E + e], w);
+        }
+      for (int th = 0; th < NT; ++th)
+        for (int e = 0; e < E; ++e) {
+          u64 hw = u64(e) | (u64(th) << R);
+          u64 so = 0;
+          for (int b = 0; b < n; ++b) if ((hw >> b) & 1) so ^= T.smoff_st[b];
+          uint64_t v = 0;
+          std::memcpy(&v, &smem[so * w], w);
+          out[size_t(th) * E + e] = v;
+        }
+    }
+    for (int th = 0; th < NT; ++th)
+      for (int e = 0; e < E; ++e) {
+        u64 hw = u64(e) | (u64(th) << R);
+        std::memcpy(dst + (db | off(T.st_bit, hw)) * w, &out[size_t(th) * E + e], w);
+      }
+  }
+}
+
+}  // namespace ll

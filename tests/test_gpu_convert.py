@@ -1,0 +1,208 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle, element by
+element, bit-exact (movement is integer work).  Needs a B200 (-m gpu)."""
+import numpy as np
+import pytest
+
+from oracle import ll_oracle as O
+from workloads import configs as W
+from workloads import gen
+from tests._util import empty_device, from_device, to_device
+
+pytestmark = pytest.mark.gpu
+
+ll = pytest.importorskip("paper_conf_asplos_0001cgrnls0trm26_b200")
+
+
+def both(spec):
+    return ll.Layout.from_spec(spec), O.Layout(*W.spec_to_bases(spec))
+
+
+def run_convert(sa, sb, w, seed, **opts):
+    A, OA = both(sa)
+    B, OB = both(sb)
+    rng = np.random.default_rng(seed)
+    T = gen.random_bits(rng, 1 << OA.d_out, w)
+    src = O.pack(OA, T)
+    plan = ll.ll_plan_convert(A, B, w, **opts)
+    d_src = to_device(src)
+    d_dst = empty_device(1 << OB.d_in, w)
+    ll.ll_convert(d_src, d_dst, plan)
+    import torch
+    torch.cuda.synchronize()
+    got = from_device(d_dst, w)
+    ref = O.convert(OA, OB, src)
+    return got, ref, plan
+
+
+CASES = [
+    ("c1", (W.C1_A, W.C1_B), 4),
+    ("c1_batch", W.c1_batched(6), 4),
+    ("c2", W.c2(3), 2),
+    ("c3", W.c3(2), 2),
+    ("c3b", W.c3b(2), 2),
+]
+
+
+@pytest.mark.parametrize("name,specs,w", CASES, ids=[c[0] for c in CASES])
+@pytest.mark.parametrize("force", [None, "SMEM"])
+def test_configs_small_bitexact(name, specs, w, force):
+    got, ref, plan = run_convert(specs[0], specs[1], w, 1001, force_class=force)
+    assert plan.describe()["exec"] == "tile"
+    assert np.array_equal(got, ref)
+
+
+@pytest.mark.parametrize("name,specs,w", CASES[:4], ids=[c[0] for c in CASES[:4]])
+def test_configs_faithful_sigma(name, specs, w):
+    got, ref, plan = run_convert(specs[0], specs[1], w, 7, sigma="faithful")
+    assert np.array_equal(got, ref)
+
+
+@pytest.mark.parametrize("w", [1, 2, 4, 8])
+def test_random_distributed_bijective(w):
+    rng = np.random.default_rng(100 + w)
+    out = [("b", 3), ("i", 5), ("j", 5)]
+    hw = [("reg", 2), ("lane", 5), ("warp", 3)]
+    for case in range(6):
+        sa = gen.random_distributed(rng, out[1:], hw)
+        sb = gen.random_distributed(rng, out[1:], hw)
+        # batch bits as block dims, identical in A and B
+        sa = {"out": out, "in": sa["in"] + [("block", ["b0", "b1", "b2"])]}
+        sb = {"out": out, "in": sb["in"] + [("block", ["b0", "b1", "b2"])]}
+        got, ref, plan = run_convert(sa, sb, w, case)
+        assert np.array_equal(got, ref), (case, plan.describe()["class"])
+
+
+def test_random_cta_class():
+    rng = np.random.default_rng(5)
+    out = [("i", 6), ("j", 6)]
+    for case in range(6):
+        cols_a = rng.permutation(12)
+        cols_b = rng.permutation(12)
+        name = lambda k: f"j{k}" if k < 6 else f"i{k - 6}"
+        sa = {"out": out, "in": [("offset", [name(k) for k in cols_a])]}
+        sb = {"out": out, "in": [("offset", [name(k) for k in cols_b])]}
+        got, ref, plan = run_convert(sa, sb, 2, case)
+        assert np.array_equal(got, ref), plan.describe()["class"]
+
+
+def test_broadcast_generic():
+    rng = np.random.default_rng(9)
+    out = [("i", 3), ("j", 4)]
+    hw = [("reg", 2), ("lane", 5), ("warp", 1)]
+    for case in range(5):
+        sa = gen.random_distributed(rng, out, hw, zero_ok=["reg"])
+        sb = gen.random_distributed(rng, out, hw, zero_ok=["lane"])
+        got, ref, plan = run_convert(sa, sb, 4, case)
+        assert np.array_equal(got, ref)
+
+
+def test_memory_swizzle_generic():
+    """Def 4.14 memory layouts with 2-bit columns (R2): non-permutation pull map."""
+    rng = np.random.default_rng(21)
+    for case in range(5):
+        d = 10
+        ca = gen.random_memory_cols(rng, d)
+        cb = gen.random_memory_cols(rng, d)
+        out = [("x", d)]
+        OA = O.layout_from_cols([("offset", d)], out, ca)
+        OB = O.layout_from_cols([("offset", d)], out, cb)
+        A = ll.Layout([("offset", d)], out, {"offset": [(c,) for c in ca]})
+        B = ll.Layout([("offset", d)], out, {"offset": [(c,) for c in cb]})
+        src = gen.random_bits(rng, 1 << d, 4)
+        plan = ll.ll_plan_convert(A, B, 4)
+        d_src, d_dst = to_device(src), empty_device(1 << d, 4)
+        ll.ll_convert(d_src, d_dst, plan)
+        assert np.array_equal(from_device(d_dst, 4), O.convert(OA, OB, src))
+
+
+def test_noop_memcpy():
+    A, OA = both(W.C1_A)
+    plan = ll.ll_plan_convert(A, A, 4)
+    assert plan.cls == "NOOP"
+    src = gen.random_bits(np.random.default_rng(0), 256, 4)
+    d_src, d_dst = to_device(src), empty_device(256, 4)
+    ll.ll_convert(d_src, d_dst, plan)
+    assert np.array_equal(from_device(d_dst, 4), src)
+
+
+def test_config2_full_size_sampled():
+    """BASELINE config 2 at full size (65536 tiles, 2 GiB in) in the launch
+    configuration bench.py times; 2^20 sampled outputs checked against the oracle's
+    pull map one by one."""
+    import torch
+    sa, sb = W.c2(16)
+    A, OA = both(sa)
+    B, OB = both(sb)
+    plan = ll.ll_plan_convert(A, B, 2)
+    n = 1 << 30
+    g = torch.Generator(device="cuda").manual_seed(1002)
+    src = torch.randint(-2 ** 15, 2 ** 15, (n,), dtype=torch.int16, device="cuda", generator=g)
+    dst = torch.empty_like(src)
+    ll.ll_convert(src, dst, plan)
+    torch.cuda.synchronize()
+    rng = np.random.default_rng(3)
+    hs = np.concatenate([rng.integers(0, n, size=1 << 20), np.arange(4096), n - 1 - np.arange(4096)]).astype(np.uint64)
+    hsrc = O.apply_inverse_all(OA, O.apply_all(OB, hs)).astype(np.int64)
+    got = dst[torch.from_numpy(hs.astype(np.int64)).cuda()].cpu().numpy()
+    want = src[torch.from_numpy(hsrc).cuda()].cpu().numpy()
+    assert np.array_equal(got, want)
+    del src, dst
+    torch.cuda.empty_cache()
+
+
+def test_config3_full_size_sampled():
+    import torch
+    sa, sb = W.c3(14)
+    A, OA = both(sa)
+    B, OB = both(sb)
+    plan = ll.ll_plan_convert(A, B, 2)
+    n = 1 << 29
+    g = torch.Generator(device="cuda").manual_seed(1003)
+    src = torch.randint(-2 ** 15, 2 ** 15, (n,), dtype=torch.int16, device="cuda", generator=g)
+    dst = torch.empty_like(src)
+    ll.ll_convert(src, dst, plan)
+    torch.cuda.synchronize()
+    rng = np.random.default_rng(4)
+    hs = np.concatenate([rng.integers(0, n, size=1 << 20), np.arange(4096)]).astype(np.uint64)
+    hsrc = O.apply_inverse_all(OA, O.apply_all(OB, hs)).astype(np.int64)
+    got = dst[torch.from_numpy(hs.astype(np.int64)).cuda()].cpu().numpy()
+    want = src[torch.from_numpy(hsrc).cuda()].cpu().numpy()
+    assert np.array_equal(got, want)
+
+
+@pytest.mark.parametrize("family", ["mma", "blocked"])
+@pytest.mark.parametrize("sigma", ["coalesced", "faithful"])
+def test_gather_bitexact(family, sigma):
+    """O10: gather via shuffles vs the oracle (take_along_axis)."""
+    rng = np.random.default_rng(1004)
+    spec = W.c4("gather", family, n_i=9, n_j=7)
+    L, OL = both(spec)
+    n = 1 << OL.d_in
+    T = gen.random_bits(rng, n, 4)
+    Ti = rng.integers(-1000, 1000, size=n).astype(np.int32)   # masked to [0, K) (G16)
+    src, idx = O.pack(OL, T), O.pack(OL, Ti)
+    ref = O.gather(OL, 1, src, idx)
+    plan = ll.ll_plan_gather(L, 1, 4, sigma=sigma)
+    d_dst = empty_device(n, 4)
+    ll.ll_gather(to_device(src), to_device(idx.view(np.uint32)), d_dst, plan)
+    assert np.array_equal(from_device(d_dst, 4), ref)
+
+
+@pytest.mark.parametrize("family", ["mma", "blocked"])
+def test_reduce_tolerance_and_fixed_order(family):
+    """O11: ≤ 1e-6 relative vs fp64 and bit-exact vs the fixed-order fp32 replica."""
+    import torch
+    rng = np.random.default_rng(1005)
+    spec = W.c4("reduce", family, n_i=9, n_j=9)
+    L, OL = both(spec)
+    n = 1 << OL.d_in
+    T = rng.random(n, dtype=np.float32)
+    src = O.pack(OL, T)
+    plan = ll.ll_plan_reduce(L, 1)
+    out = torch.empty(plan.out_elems(), dtype=torch.float32, device="cuda")
+    ll.ll_reduce(torch.from_numpy(src).cuda(), out, plan)
+    got = out.cpu().numpy()
+    ref = O.reduce_ref_fp64(OL, 1, src)
+    assert np.all(np.abs(got - ref) <= 1e-6 * np.abs(ref))
+    rep = O.reduce_fixed_order_fp32(OL, 1, src)
+    assert np.array_equal(got.view(np.uint32), rep.view(np.uint32))

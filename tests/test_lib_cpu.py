@@ -1,0 +1,257 @@
+"""CPU tests of libll.so: the C ABI loads and exports every declared symbol; the
+host F2 algebra and the planner agree with the oracle; the specialised plans'
+schedules (emulated on the host with the same tables the kernels are compiled
+from) reproduce the oracle's conversion; swizzles are bank-conflict free under the
+oracle's Lemma 9.4 model; the kernel templates compile for sm_100a (NVRTC)."""
+import ctypes
+import os
+import re
+
+import numpy as np
+import pytest
+
+from oracle import ll_oracle as O
+from workloads import configs as W
+from workloads import gen
+
+ll = pytest.importorskip("paper_conf_asplos_0001cgrnls0trm26_b200")
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def both(spec):
+    return ll.Layout.from_spec(spec), O.Layout(*W.spec_to_bases(spec))
+
+
+def test_exports_every_declared_symbol():
+    hdr = open(os.path.join(ROOT, "include", "ll.h")).read()
+    names = set(re.findall(r"^\s*(?:ll_status|void|const char\*)\s+(ll_\w+)\s*\(", hdr, re.M))
+    assert len(names) >= 30
+    lib = ctypes.CDLL(ll.library_path())
+    missing = [n for n in sorted(names) if not hasattr(lib, n)]
+    assert not missing, missing
+
+
+def test_layout_roundtrip_and_apply():
+    L, OL = both(W.C1_A)
+    assert L.cols() == OL.cols
+    for h in range(256):
+        coords = O.hw_coords(OL.in_dims, h)
+        assert L.apply(coords) == O.logical_coords(OL.out_dims, O.apply(OL, h))
+    # predicates are properties of the matrix: a permutation matrix satisfies both
+    # Def 4.10 and Def 4.14
+    assert L.props() == dict(surjective=O.is_surjective(OL), injective=O.is_injective(OL),
+                             distributed=O.is_distributed(OL), memory=O.is_memory(OL))
+
+
+def test_algebra_vs_oracle_random():
+    rng = np.random.default_rng(12)
+    for _ in range(60):
+        d_out = int(rng.integers(1, 6))
+        d_in = int(rng.integers(d_out, 9))
+        cols = gen.random_surjective_cols(rng, d_out, d_in)
+        OL = O.layout_from_cols([("h", d_in)], [("x", d_out)], cols)
+        L = ll.Layout([("h", d_in)], [("x", d_out)], {"h": [(c,) for c in cols]})
+        # right inverse (Def 4.5): equals the oracle's brute-force min-index preimage
+        Li = L.invert()
+        first = O.preimage_min(OL)
+        assert [b[0] for b in Li.bases()] == [int(first[1 << t]) for t in range(d_out)]
+        # kernel dimension
+        assert len(L.kernel_basis()) == d_in - d_out
+        # compose with a random map (Def 4.2)
+        d2 = int(rng.integers(1, 6))
+        c2 = [int(x) for x in rng.integers(0, 1 << d2, size=d_out)]
+        OM = O.layout_from_cols([("x", d_out)], [("y", d2)], c2)
+        M = ll.Layout([("x", d_out)], [("y", d2)], {"x": [(c,) for c in c2]})
+        assert M.compose(L).cols() == O.compose(OM, OL).cols
+        p = L.props()
+        assert p["surjective"] and p["injective"] == (d_in == d_out)
+
+
+def test_product_and_left_division_vs_oracle():
+    OA = O.blocked([4, 4], [2, 2], [2, 2], [1, 1], [1, 0])
+    OB = O.blocked([8, 4], [1, 2], [4, 2], [2, 1], [1, 0])
+    OA = O.Layout(OA.in_dims, [("d0", 2), ("d1", 2)], OA.bases)
+    A = ll.Layout(OA.in_dims, OA.out_dims, OA.bases)
+    B = ll.Layout(OB.in_dims, OB.out_dims, OB.bases)
+    P = A.product(B)
+    OP = O.product(OA, OB)
+    assert P.cols() == OP.cols
+    assert P.left_divide(A).cols() == OB.cols
+    with pytest.raises(ll.LLError):
+        P.left_divide(B)
+
+
+def test_errors():
+    A, _ = both(W.C1_A)
+    B2, _ = both(W.c2(0)[0])
+    with pytest.raises(ll.LLError, match="DIM_MISMATCH"):
+        ll.ll_plan_convert(A, B2, 4)
+    N = ll.Layout([("offset", 3)], [("x", 3)], {"offset": [(1,), (2,), (3,)]})
+    with pytest.raises(ll.LLError, match="NOT_SURJECTIVE"):
+        ll.ll_plan_convert(N, N, 4)
+    with pytest.raises(ll.LLError, match="INVALID_ARG"):
+        ll.ll_plan_convert(A, A, 3)
+    with pytest.raises(ll.LLError):
+        ll.Layout([("reg", 1)], [("x", 1)], {"reg": [(2,)]})
+
+
+@pytest.mark.parametrize("cfg", ["c1", "c2", "c3"])
+def test_planner_class_matches_oracle_configs(cfg):
+    sa, sb = {"c1": (W.C1_A, W.C1_B), "c2": W.c2(0), "c3": W.c3(0)}[cfg]
+    A, OA = both(sa)
+    B, OB = both(sb)
+    assert ll.ll_plan_convert(A, B, 4).cls == O.classify(OA, OB)
+
+
+def test_planner_class_matches_oracle_exhaustive_sample():
+    """E1 (sampled): random relabelings B of Fig. 1's space, with and without
+    broadcast columns; the planner's class equals the existential class O7."""
+    rng = np.random.default_rng(31)
+    A, OA = both(W.C1_A)
+    hw = [("reg", 2), ("lane", 5), ("warp", 1)]
+    for _ in range(300):
+        sb = gen.random_distributed(rng, W.C1_OUT, hw)
+        B, OB = both(sb)
+        assert ll.ll_plan_convert(A, B, 4).cls == O.classify(OA, OB)
+    out7 = [("i", 3), ("j", 4)]
+    for _ in range(300):
+        sa = gen.random_distributed(rng, out7, hw, zero_ok=["reg", "warp"])
+        sb = gen.random_distributed(rng, out7, hw, zero_ok=["lane", "reg"])
+        A7, OA7 = both(sa)
+        B7, OB7 = both(sb)
+        assert ll.ll_plan_convert(A7, B7, 4).cls == O.classify(OA7, OB7)
+
+
+def _sim_check(sa, sb, w, seed, **opts):
+    A, OA = both(sa)
+    B, OB = both(sb)
+    plan = ll.ll_plan_convert(A, B, w, **opts)
+    rng = np.random.default_rng(seed)
+    T = gen.random_bits(rng, 1 << OA.d_out, w)
+    src = O.pack(OA, T)
+    d = plan.describe()
+    if d["exec"] != "tile":
+        return d
+    got = plan.simulate(src, 1 << OB.d_in)
+    assert np.array_equal(got, O.convert(OA, OB, src)), d
+    return d
+
+
+@pytest.mark.parametrize("force", [None, "SMEM"])
+@pytest.mark.parametrize("sigma", ["coalesced", "faithful"])
+def test_simulated_schedule_configs(force, sigma):
+    for sa, sb, w in [(W.C1_A, W.C1_B, 4), (*W.c1_batched(5), 4), (*W.c2(1), 2), (*W.c3(1), 2), (*W.c3b(1), 2)]:
+        d = _sim_check(sa, sb, w, 1, force_class=force, sigma=sigma)
+        assert d["exec"] == "tile"
+        if force == "SMEM":
+            assert d["tile"]["xchg"] == "smem"
+
+
+def test_simulated_schedule_random_distributed():
+    rng = np.random.default_rng(77)
+    out = [("i", 5), ("j", 5)]
+    hw = [("reg", 2), ("lane", 5), ("warp", 3)]
+    seen = set()
+    for case in range(80):
+        sa = gen.random_distributed(rng, out, hw)
+        sb = gen.random_distributed(rng, out, hw)
+        w = [1, 2, 4, 8][case % 4]
+        d = _sim_check(sa, sb, w, case)
+        seen.add((d["class"], d.get("tile", {}).get("xchg")))
+    assert ("SMEM", "smem") in seen
+
+
+def test_simulated_schedule_regperm_shuffle_classes():
+    """REGPERM and SHUFFLE class pairs built by permuting only
+    register bits / register+lane bits of a random layout."""
+    rng = np.random.default_rng(8)
+    out = [("i", 5), ("j", 5)]
+    hw = [("reg", 3), ("lane", 5), ("warp", 2)]
+    for case in range(40):
+        sa = gen.random_distributed(rng, out, hw)
+        ins = dict(sa["in"])
+        if case % 2 == 0:
+            regs = list(ins["reg"])
+            rng.shuffle(regs)
+            sb = {"out": out, "in": [("reg", regs), ("lane", ins["lane"]), ("warp", ins["warp"])]}
+            want = "REGPERM"
+        else:
+            pool = list(ins["reg"]) + list(ins["lane"])
+            rng.shuffle(pool)
+            sb = {"out": out, "in": [("reg", pool[:3]), ("lane", pool[3:]), ("warp", ins["warp"])]}
+            want = "SHUFFLE"
+        A, OA = both(sa)
+        B, OB = both(sb)
+        if O.classify(OA, OB) != want:
+            continue
+        for w in (2, 4):
+            d = _sim_check(sa, sb, w, case, sigma="faithful")
+            assert d["class"] == want
+
+
+def test_simulated_schedule_cta_class():
+    rng = np.random.default_rng(5)
+    out = [("i", 6), ("j", 6)]
+    name = lambda k: f"j{k}" if k < 6 else f"i{k - 6}"
+    for case in range(20):
+        sa = {"out": out, "in": [("offset", [name(k) for k in rng.permutation(12)])]}
+        sb = {"out": out, "in": [("offset", [name(k) for k in rng.permutation(12)])]}
+        d = _sim_check(sa, sb, [1, 2, 4][case % 3], case)
+        assert d["class"] in ("CTA", "NOOP")
+
+
+def test_swizzle_plans_conflict_free_under_oracle_model():
+    """The planner's smem layout (Vec, Bank, Seg) gives the ideal number of wavefronts
+    for the store (L_ld) and load (L_st) sides under the oracle's simulator."""
+    for sa, sb, w in [(W.C1_A, W.C1_B, 4), (*W.c2(0), 2), (*W.c3(0), 2), (*W.c3b(0), 2)]:
+        A, OA = both(sa)
+        B, OB = both(sb)
+        t = ll.ll_plan_convert(A, B, w, force_class="SMEM").describe()["tile"]
+        out = OA.out_dims
+        mk = lambda cols: O.layout_from_cols([("reg", t["R"]), ("lane", 5), ("warp", t["warp_bits"])], out, cols)
+        Lld, Lst = mk(t["L_ld"]), mk(t["L_st"])
+        S = O.layout_from_cols([("offset", t["n"])], out, t["Vec"] + t["Bank"] + t["Seg"])
+        assert O.is_memory(S) or O.is_surjective(S)
+        for L in (Lld, Lst):
+            wf, ideal = O.smem_wavefronts(S, L, w, t["Vec"])
+            assert wf == ideal
+        assert t["wavefronts_st"] + t["wavefronts_ld"] == t["ideal_wavefronts"]
+
+
+def test_shuffle_plan_invariants_config2():
+    """O9: rounds = 2^{(n_reg+5) - |V| - |I| - |G|}; G = {e_i ^ f_i} with E, F
+    ascending; one 32-bit unit per lane per round."""
+    A, _ = both(W.c2(0)[0])
+    B, _ = both(W.c2(0)[1])
+    t = ll.ll_plan_convert(A, B, 2).describe()["tile"]
+    assert t["xchg"] == "shuffle"
+    assert t["rounds"] == 1 << ((t["R"] + 5) - len(t["V"]) - len(t["I"]) - len(t["G"]))
+    assert t["E"] == sorted(t["E"]) and t["F"] == sorted(t["F"])
+    assert t["G"] == [e ^ f for e, f in zip(t["E"], t["F"])]
+    assert t["unit_elems"] * 2 == 4
+
+
+def test_kernels_compile_for_sm100a():
+    """NVRTC specialisation of each kernel family for sm_100a (no GPU needed)."""
+    for sa, sb, w, fc in [(*W.c2(16), 2, None), (*W.c3(14), 2, None), (W.C1_A, W.C1_B, 4, "SMEM")]:
+        A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
+        p = ll.ll_plan_convert(A, B, w, force_class=fc)
+        p.precompile()
+        assert "ll_tile_kernel" in p.source()
+    L = ll.Layout.from_spec(W.c4("gather", "mma"))
+    ll.ll_plan_gather(L, 1, 4).precompile()
+    L = ll.Layout.from_spec(W.c4("reduce", "blocked"))
+    ll.ll_plan_reduce(L, 1).precompile()
+
+
+def test_device_entry_fails_loudly_without_gpu():
+    try:
+        import torch
+        if torch.cuda.is_available():
+            pytest.skip("GPU present")
+    except ImportError:
+        pass
+    A, B = ll.Layout.from_spec(W.C1_A), ll.Layout.from_spec(W.C1_B)
+    p = ll.ll_plan_convert(A, B, 4)
+    with pytest.raises(ll.LLError, match="CUDA"):
+        ll.ll_convert(1 << 20, 2 << 20, p, stream=0)

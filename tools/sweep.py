@@ -1,0 +1,113 @@
+"""Developer sweep: time ll_convert / ll_gather / ll_reduce on the BASELINE configs
+under several plan options (CUDA events, inputs > L2).  Not the bench contract."""
+import argparse
+import json
+import os
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import torch  # noqa: E402
+
+import paper_conf_asplos_0001cgrnls0trm26_b200 as ll  # noqa: E402
+from workloads import configs as W  # noqa: E402
+
+
+def time_fn(fn, iters=20, warmup=5):
+    for _ in range(warmup):
+        fn()
+    torch.cuda.synchronize()
+    ts = []
+    for _ in range(iters):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        fn()
+        b.record()
+        b.synchronize()
+        ts.append(a.elapsed_time(b))
+    ts.sort()
+    return ts[len(ts) // 2]
+
+
+def conv_case(name, sa, sb, w, **opts):
+    A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
+    p = ll.ll_plan_convert(A, B, w, **opts)
+    n = 1 << A.d_in
+    src = torch.randint(-2 ** 15, 2 ** 15, (n * w // 2,), dtype=torch.int16, device="cuda")
+    dst = torch.empty_like(src)
+    p.prepare()
+    ms = time_fn(lambda: ll.ll_convert(src, dst, p))
+    gbs = 2 * n * w / ms / 1e6
+    d = p.describe()
+    t = d.get("tile", {})
+    print(json.dumps({"case": name, "opts": opts, "class": d["class"], "xchg": t.get("xchg"), "ms": round(ms, 4),
+                      "GBps": round(gbs, 1), "frac_6539": round(gbs / 6539.5, 3)}), flush=True)
+    del src, dst
+    torch.cuda.empty_cache()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--quick", action="store_true")
+    args = ap.parse_args()
+    # raw copy roofline reference
+    n = 1 << 30
+    a = torch.empty(n, dtype=torch.int16, device="cuda")
+    b = torch.empty_like(a)
+    ms = time_fn(lambda: b.copy_(a))
+    print(json.dumps({"case": "torch_copy_2GiB", "ms": round(ms, 4), "GBps": round(4 * n / ms / 1e6, 1)}), flush=True)
+    del a, b
+    for grid in ["0", "4", "8", "16"]:
+        os.environ["LL_GRID_PER_SM"] = grid
+        sa, sb = W.c2(16)
+        conv_case(f"c2 grid{grid}", sa, sb, 2)
+    os.environ["LL_GRID_PER_SM"] = "0"
+    sa, sb = W.c2(16)
+    for opts in [dict(force_class="SMEM"), dict(sigma="faithful"), dict(thread_bytes=128), dict(thread_bytes=64)]:
+        conv_case("c2", sa, sb, 2, **opts)
+    sa, sb = W.c3(14)
+    for opts in [dict(), dict(thread_bytes=128), dict(thread_bytes=64), dict(sigma="faithful")]:
+        conv_case("c3", sa, sb, 2, **opts)
+    sa, sb = W.c3b(14)
+    conv_case("c3b", sa, sb, 2)
+    sa, sb = W.c1_batched(20)
+    for opts in [dict(), dict(force_class="SMEM"), dict(tile_bytes=65536), dict(thread_bytes=16)]:
+        conv_case("c1batch", sa, sb, 4, **opts)
+    # gather / reduce (4096 x 4096 fp32)
+    for fam in ["mma", "blocked"]:
+        for sig in ["coalesced", "faithful"]:
+            L = ll.Layout.from_spec(W.c4("gather", fam))
+            p = ll.ll_plan_gather(L, 1, 4, sigma=sig)
+            p.prepare()
+            n = 1 << 24
+            sets = [(torch.randint(-2 ** 31, 2 ** 31 - 1, (n,), dtype=torch.int32, device="cuda"),
+                     torch.randint(0, 32, (n,), dtype=torch.int32, device="cuda"),
+                     torch.empty(n, dtype=torch.int32, device="cuda")) for _ in range(4)]
+            it = [0]
+
+            def g():
+                s = sets[it[0] % 4]
+                it[0] += 1
+                ll.ll_gather(s[0], s[1], s[2], p)
+            ms = time_fn(g)
+            print(json.dumps({"case": f"gather {fam} {sig}", "desc": p.describe(), "ms": round(ms, 4),
+                              "GBps": round(12 * n / ms / 1e6, 1)}), flush=True)
+        L = ll.Layout.from_spec(W.c4("reduce", fam))
+        p = ll.ll_plan_reduce(L, 1)
+        p.prepare()
+        n = 1 << 24
+        sets = [(torch.rand(n, device="cuda"), torch.empty(p.out_elems(), device="cuda")) for _ in range(4)]
+        it = [0]
+
+        def r():
+            s = sets[it[0] % 4]
+            it[0] += 1
+            ll.ll_reduce(s[0], s[1], p)
+        ms = time_fn(r)
+        print(json.dumps({"case": f"reduce {fam}", "ms": round(ms, 4), "GBps": round((4 * n + 4 * p.out_elems()) / ms / 1e6, 1)}), flush=True)
+
+
+if __name__ == "__main__":
+    main()
