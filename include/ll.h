@@ -213,7 +213,19 @@ ll_status ll_reduce(const float* src, float* dst, const ll_plan* plan, void* str
  * absent). */
 ll_status ll_comm_create(const void* nccl_unique_id, int nranks, int rank, ll_comm** comm);
 ll_status ll_comm_get_unique_id(void* nccl_unique_id /* 128 bytes */);
+/* Single-process loopback communicator of nranks (power of two) virtual ranks: the
+ * src / dst / workspace buffers passed to ll_convert hold all ranks' slices back to
+ * back, and the exchange is a set of device memcpys.  For tests of the DEVICE
+ * decomposition on one GPU. */
+ll_status ll_comm_create_loopback(int nranks, ll_comm** comm);
 void ll_comm_destroy(ll_comm* comm);
+
+/* The stages of a DEVICE plan: pack (src -> send layout, receiver
+ * rank bits on top) and unpack (recv layout, source rank bits on top -> dst); NULL
+ * when a stage is the identity.  Every rank exchanges chunk_elems elements with
+ * every peer.  The stage handles are owned by `plan` (do not destroy them). */
+ll_status ll_plan_device_stages(const ll_plan* plan, ll_plan** pack, ll_plan** unpack,
+                                size_t* chunk_elems, int* nranks);
 
 /* ---------------------------------------------------------------- test hooks --
  * ll_plan_simulate: host emulation of a specialised tile plan's schedule (the

@@ -75,6 +75,8 @@ _sig = {
     "ll_plan_simulate": [_P, _P, _P],
     "ll_comm_create": [_P, C.c_int, C.c_int, _PP],
     "ll_comm_get_unique_id": [_P],
+    "ll_comm_create_loopback": [C.c_int, _PP],
+    "ll_plan_device_stages": [_P, _PP, _PP, C.POINTER(C.c_size_t), C.POINTER(C.c_int)],
 }
 for _name, _args in _sig.items():
     _f = getattr(_lib, _name)
@@ -91,6 +93,7 @@ _lib.ll_version.restype = C.c_char_p
 _lib.ll_plan_opts_default.argtypes = [C.POINTER(_Opts)]
 _lib.ll_plan_opts_default.restype = None
 
+_lib.ll_comm_create_loopback.restype = C.c_int
 EXPORTED = sorted(list(_sig) + ["ll_layout_destroy", "ll_plan_destroy", "ll_comm_destroy", "ll_last_error",
                                 "ll_version", "ll_plan_opts_default"])
 
@@ -324,6 +327,15 @@ class Plan:
         _check(_lib.ll_plan_reduce_out_elems(self.handle, C.byref(n)))
         return n.value
 
+    def device_stages(self):
+        """(pack, unpack, chunk_elems, nranks) of a DEVICE plan; stages are None when
+        they are the identity.  Stage plans are views owned by this plan."""
+        pk, up = C.c_void_p(), C.c_void_p()
+        ch, nr = C.c_size_t(), C.c_int()
+        _check(_lib.ll_plan_device_stages(self.handle, C.byref(pk), C.byref(up), C.byref(ch), C.byref(nr)))
+        wrap = lambda h: _Stage(h, self) if h.value else None
+        return wrap(pk), wrap(up), ch.value, nr.value
+
     def simulate(self, src: np.ndarray, dst_elems: int) -> np.ndarray:
         """Host emulation of the plan's kernel schedule (test hook, no GPU)."""
         src = np.ascontiguousarray(src)
@@ -332,11 +344,58 @@ class Plan:
         return dst
 
 
+class _Stage(Plan):
+    """A borrowed stage view of a DEVICE plan (kept alive by its parent)."""
+
+    def __init__(self, handle, parent):
+        super().__init__(handle, "convert")
+        self.parent = parent
+
+    def __del__(self):
+        self.handle = None
+
+
+class Comm:
+    """ll_comm: NCCL communicator (one per rank) or a single-process loopback."""
+
+    def __init__(self, handle, nranks):
+        self.handle, self.nranks = handle, nranks
+
+    @classmethod
+    def loopback(cls, nranks: int) -> "Comm":
+        h = C.c_void_p()
+        _check(_lib.ll_comm_create_loopback(int(nranks), C.byref(h)))
+        return cls(h, nranks)
+
+    @classmethod
+    def from_process_group(cls, group=None) -> "Comm":
+        """Bootstrap NCCL: rank 0's ncclUniqueId is broadcast over the torch group."""
+        import torch.distributed as dist
+        rank, world = dist.get_rank(group), dist.get_world_size(group)
+        uid = (C.c_char * 128)()
+        if rank == 0:
+            _check(_lib.ll_comm_get_unique_id(uid))
+        obj = [bytes(uid)]
+        dist.broadcast_object_list(obj, src=0, group=group)
+        uid = (C.c_char * 128).from_buffer_copy(obj[0])
+        h = C.c_void_p()
+        _check(_lib.ll_comm_create(uid, world, rank, C.byref(h)))
+        return cls(h, world)
+
+    def __del__(self):
+        h = getattr(self, "handle", None)
+        if h:
+            _lib.ll_comm_destroy(h)
+            self.handle = None
+
+
 def ll_plan_convert(A: Layout, B: Layout, elem_bytes: int, **opts) -> Plan:
     h = C.c_void_p()
     o = _opts(**opts)
     _check(_lib.ll_plan_convert(A.handle, B.handle, int(elem_bytes), C.byref(o), C.byref(h)))
-    return Plan(h, "convert")
+    p = Plan(h, "convert")
+    p.comm = opts.get("comm")   # keep the communicator alive as long as the plan
+    return p
 
 
 def ll_convert(src, dst, plan: Plan, stream=None, workspace=None):

@@ -89,6 +89,9 @@ Layout atomize(const Layout& L) {
   return R;
 }
 
+}  // namespace
+
+namespace ll {
 void ensure_tile_kernel(ConvPlan& P) {
   std::lock_guard<std::mutex> g(P.mu);
   if (P.kernel) return;
@@ -99,6 +102,9 @@ void ensure_tile_kernel(ConvPlan& P) {
                "cudaFuncSetAttribute");
 }
 
+}  // namespace ll
+
+namespace {
 unsigned grid_for(u64 ntiles) {
   const char* e = getenv("LL_GRID_PER_SM");
   int per = e ? atoi(e) : 0;
@@ -107,6 +113,9 @@ unsigned grid_for(u64 ntiles) {
   return unsigned(std::max<u64>(g, 1));
 }
 
+}  // namespace
+
+namespace ll {
 ll_status convert_impl(const void* src, void* dst, void* ws, ConvPlan& P, cudaStream_t st) {
   const size_t sbytes = P.src_elems * P.w, dbytes = P.dst_elems * P.w;
   if ((reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst)) & 15)
@@ -137,7 +146,7 @@ ll_status convert_impl(const void* src, void* dst, void* ws, ConvPlan& P, cudaSt
   return device_convert(P, src, dst, ws, st);
 }
 
-}  // namespace
+}  // namespace ll
 
 extern "C" {
 
@@ -305,7 +314,17 @@ ll_status ll_plan_convert(const ll_layout* A, const ll_layout* B, int w, const l
   } else {
     h->conv = plan_convert(A->L, B->L, w, opts);
   }
-  if (h->conv->exec == EXEC_DEVICE) plan_device(*h->conv, opts);
+  if (h->conv->exec == EXEC_DEVICE) {
+    plan_device(*h->conv, opts);
+    ConvPlan* st[2] = {h->conv->pack.get(), h->conv->unpack.get()};
+    for (int i = 0; i < 2; ++i)
+      if (st[i]) {
+        h->stage[i] = std::make_unique<ll_plan>();
+        h->stage[i]->kind = 0;
+        h->stage[i]->borrowed = st[i];
+        if (st[i]->exec == EXEC_TILE) st[i]->source = codegen_tile(*st[i]);
+      }
+  }
   if (h->conv->exec == EXEC_TILE) h->conv->source = codegen_tile(*h->conv);
   *plan = h.release();
   LL_CATCH
@@ -314,14 +333,14 @@ ll_status ll_plan_convert(const ll_layout* A, const ll_layout* B, int w, const l
 ll_status ll_plan_class(const ll_plan* p, ll_class* cls) {
   LL_TRY
   if (!p || !cls || p->kind != 0) fail(LL_ERR_INVALID_ARG, "not a conversion plan");
-  *cls = p->conv->cls;
+  *cls = p->cp().cls;
   LL_CATCH
 }
 
 ll_status ll_plan_workspace_bytes(const ll_plan* p, size_t* bytes) {
   LL_TRY
   if (!p || !bytes) fail(LL_ERR_INVALID_ARG, "null argument");
-  *bytes = p->kind == 0 ? p->conv->workspace_bytes : 0;
+  *bytes = p->kind == 0 ? p->cp().workspace_bytes : 0;
   LL_CATCH
 }
 
@@ -329,7 +348,7 @@ ll_status ll_plan_describe(const ll_plan* p, char* json, size_t cap) {
   LL_TRY
   if (!p || !json || !cap) fail(LL_ERR_INVALID_ARG, "null argument");
   std::string s;
-  if (p->kind == 0) s = describe(*p->conv);
+  if (p->kind == 0) s = describe(p->cp());
   else if (p->kind == 1) {
     const GatherPlan& G = *p->gather;
     std::ostringstream o;
@@ -356,7 +375,7 @@ ll_status ll_plan_source(const ll_plan* p, char* buf, size_t cap, size_t* needed
   LL_TRY
   if (!p) fail(LL_ERR_INVALID_ARG, "null plan");
   std::string s;
-  if (p->kind == 0 && p->conv->exec == EXEC_TILE) s = p->conv->source;
+  if (p->kind == 0 && p->cp().exec == EXEC_TILE) s = p->cp().source;
   if (p->kind == 1) s = codegen_gather(*p->gather);
   if (p->kind == 2) s = codegen_reduce(*p->reduce);
   if (needed) *needed = s.size() + 1;
@@ -370,10 +389,10 @@ ll_status ll_plan_source(const ll_plan* p, char* buf, size_t cap, size_t* needed
 ll_status ll_plan_prepare(ll_plan* p) {
   LL_TRY
   if (!p) fail(LL_ERR_INVALID_ARG, "null plan");
-  if (p->kind == 0 && p->conv->exec == EXEC_TILE) ensure_tile_kernel(*p->conv);
-  if (p->kind == 0 && p->conv->exec == EXEC_DEVICE) {
-    if (p->conv->pack && p->conv->pack->exec == EXEC_TILE) ensure_tile_kernel(*p->conv->pack);
-    if (p->conv->unpack && p->conv->unpack->exec == EXEC_TILE) ensure_tile_kernel(*p->conv->unpack);
+  if (p->kind == 0 && p->cp().exec == EXEC_TILE) ensure_tile_kernel(p->cp());
+  if (p->kind == 0 && p->cp().exec == EXEC_DEVICE) {
+    if (p->cp().pack && p->cp().pack->exec == EXEC_TILE) ensure_tile_kernel(*p->cp().pack);
+    if (p->cp().unpack && p->cp().unpack->exec == EXEC_TILE) ensure_tile_kernel(*p->cp().unpack);
   }
   if (p->kind == 1) {
     std::lock_guard<std::mutex> g(p->gather->mu);
@@ -394,19 +413,21 @@ ll_status ll_plan_prepare(ll_plan* p) {
 ll_status ll_jit_precompile(const ll_plan* p) {
   LL_TRY
   if (!p) fail(LL_ERR_INVALID_ARG, "null plan");
-  if (p->kind == 0 && p->conv->exec == EXEC_TILE) jit_precompile(p->conv->source, "ll_tile_kernel");
+  if (p->kind == 0 && p->cp().exec == EXEC_TILE) jit_precompile(p->cp().source, "ll_tile_kernel");
   if (p->kind == 1) jit_precompile(codegen_gather(*p->gather), "ll_gather_kernel");
   if (p->kind == 2) jit_precompile(codegen_reduce(*p->reduce), "ll_reduce_kernel");
   LL_CATCH
 }
 
-void ll_plan_destroy(ll_plan* p) { delete p; }
+void ll_plan_destroy(ll_plan* p) {
+  if (p && !p->borrowed) delete p;   // stage views are owned by their DEVICE plan
+}
 
 ll_status ll_convert(const void* src, void* dst, void* ws, const ll_plan* p, void* stream) {
   LL_TRY
   if (!p || p->kind != 0) fail(LL_ERR_INVALID_ARG, "not a conversion plan");
   if (!src || !dst) fail(LL_ERR_INVALID_ARG, "null buffer");
-  return convert_impl(src, dst, ws, *p->conv, static_cast<cudaStream_t>(stream));
+  return convert_impl(src, dst, ws, p->cp(), static_cast<cudaStream_t>(stream));
   LL_CATCH
 }
 
@@ -472,11 +493,24 @@ ll_status ll_reduce(const float* src, float* dst, const ll_plan* p, void* stream
   LL_CATCH
 }
 
+ll_status ll_plan_device_stages(const ll_plan* p, ll_plan** pack, ll_plan** unpack, size_t* chunk_elems,
+                                int* nranks) {
+  LL_TRY
+  if (!p || p->kind != 0) fail(LL_ERR_INVALID_ARG, "not a conversion plan");
+  const ConvPlan& P = p->cp();
+  if (P.exec != EXEC_DEVICE) fail(LL_ERR_INVALID_ARG, "not a DEVICE plan");
+  if (pack) *pack = p->stage[0].get();
+  if (unpack) *unpack = p->stage[1].get();
+  if (chunk_elems) *chunk_elems = size_t(P.chunk_elems);
+  if (nranks) *nranks = P.nranks;
+  LL_CATCH
+}
+
 ll_status ll_plan_simulate(const ll_plan* p, const void* src, void* dst) {
   LL_TRY
   if (!p || p->kind != 0 || !src || !dst) fail(LL_ERR_INVALID_ARG, "bad argument");
-  if (p->conv->exec != EXEC_TILE) fail(LL_ERR_UNSUPPORTED, "simulate: only tile plans");
-  simulate_tile(*p->conv, static_cast<const uint8_t*>(src), static_cast<uint8_t*>(dst));
+  if (p->cp().exec != EXEC_TILE) fail(LL_ERR_UNSUPPORTED, "simulate: only tile plans");
+  simulate_tile(p->cp(), static_cast<const uint8_t*>(src), static_cast<uint8_t*>(dst));
   LL_CATCH
 }
 

@@ -173,11 +173,14 @@ struct ConvPlan {
   std::vector<u64> Q;   // pull map: dst bit k -> src packed index (A^+ ∘ B, adjusted)
   u64 src_elems = 0, dst_elems = 0;
   TilePlan tile;
-  // DEVICE plans
+  // DEVICE plans (pack -> all-to-all -> unpack)
   int dev_bits = 0;
   size_t workspace_bytes = 0;
   ll_comm* comm = nullptr;
-  std::unique_ptr<ConvPlan> pack, unpack;   // local stages of a DEVICE plan
+  std::unique_ptr<ConvPlan> pack, unpack;   // local stages of a DEVICE plan (null = identity)
+  u64 chunk_elems = 0;                      // elements exchanged with every peer
+  int nranks = 1;
+  u64 local_elems = 0;
   std::string source;   // specialised kernel source (EXEC_TILE)
   std::string kernel_key;
   void* kernel = nullptr;   // cudaKernel_t once loaded
@@ -243,6 +246,14 @@ struct ll_layout { ll::Layout L; };
 struct ll_plan {
   int kind;   // 0 conv, 1 gather, 2 reduce
   std::unique_ptr<ll::ConvPlan> conv;
+  ll::ConvPlan* borrowed = nullptr;          // sub-plan handles (DEVICE stages)
+  std::unique_ptr<ll_plan> stage[2];         // pack / unpack views of a DEVICE plan
   std::unique_ptr<ll::GatherPlan> gather;
   std::unique_ptr<ll::ReducePlan> reduce;
+  ll::ConvPlan& cp() const { return borrowed ? *borrowed : *conv; }
+};
+struct ll_comm {
+  int nranks = 1, rank = 0;
+  bool loopback = false;   // all ranks' slices in one process (tests); memcpy exchange
+  void* nccl = nullptr;    // ncclComm_t
 };

@@ -1,0 +1,155 @@
+"""DEVICE class (row a9): pack -> all-to-all -> unpack.
+
+CPU (gloo, world_size 2 and 4): each rank builds the real plan, runs its pack /
+unpack stages with the host schedule emulation (ll_plan_simulate) and exchanges the
+chunks with torch.distributed.all_to_all_single over gloo; every rank's slice must
+equal the oracle's closed form (O12).  GPU (1 B200): the loopback communicator runs
+the same decomposition with the CUDA kernels and device memcpys for P = 2, 4, 8."""
+import os
+import socket
+
+import numpy as np
+import pytest
+
+from oracle import ll_oracle as O
+from workloads import configs as W
+from workloads import gen
+
+ll = pytest.importorskip("paper_conf_asplos_0001cgrnls0trm26_b200")
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _rank_src(OA, T, r):
+    la, off = O.rank_slice(OA, r)
+    xs = O.apply_all(la, np.arange(1 << la.d_in, dtype=np.uint64)) ^ np.uint64(off)
+    return T[xs.astype(np.int64)]
+
+
+def _worker(rank, world, port, n, q):
+    import torch
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        p = world.bit_length() - 1
+        for make in (W.c5, W.c5T):
+            sa, sb = make(p, n=n)
+            OA, OB = O.Layout(*W.spec_to_bases(sa)), O.Layout(*W.spec_to_bases(sb))
+            A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
+            # the communicator handle is only consulted for its size at plan time
+            plan = ll.ll_plan_convert(A, B, 2, comm=ll.Comm.loopback(world))
+            assert plan.cls == "DEVICE"
+            pack, unpack, chunk, nr = plan.device_stages()
+            assert nr == world
+            T = gen.random_bits(np.random.default_rng(1006), 1 << (2 * n), 2)
+            src = _rank_src(OA, T, rank)
+            send = pack.simulate(src, src.size) if pack else src
+            # gloo has no 16-bit all_to_all: move the bf16 bits as int32 pairs
+            recv = torch.empty(src.size // 2, dtype=torch.int32)
+            dist.all_to_all_single(recv, torch.from_numpy(send.view(np.int32).copy()),
+                                   [chunk // 2] * world, [chunk // 2] * world)
+            recv = recv.numpy().view(np.uint16)
+            got = unpack.simulate(recv, recv.size) if unpack else recv
+            want = O.convert_distributed_rank(OA, OB, T, rank)
+            assert np.array_equal(got, want), (make.__name__, rank)
+        q.put((rank, "ok"))
+    except Exception as e:  # pragma: no cover - reported to the parent
+        q.put((rank, repr(e)))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 4])
+def test_device_decomposition_gloo(world):
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, 5, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = dict(q.get(timeout=300) for _ in procs)
+    for p in procs:
+        p.join(timeout=60)
+    assert all(v == "ok" for v in res.values()), res
+
+
+def test_device_plan_errors():
+    sa, sb = W.c5(1, n=4)
+    A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
+    with pytest.raises(ll.LLError, match="comm"):
+        ll.ll_plan_convert(A, B, 2)
+    with pytest.raises(ll.LLError):
+        ll.ll_plan_convert(A, B, 2, comm=ll.Comm.loopback(4))   # 2 ranks' worth of dev bits
+
+
+def test_device_p1_is_noop_and_5T_is_cta():
+    sa, sb = W.c5(0, n=5)
+    assert ll.ll_plan_convert(ll.Layout.from_spec(sa), ll.Layout.from_spec(sb), 2).cls == "NOOP"
+    sa, sb = W.c5T(0, n=5)
+    p = ll.ll_plan_convert(ll.Layout.from_spec(sa), ll.Layout.from_spec(sb), 2)
+    assert p.cls == "CTA" and p.describe()["exec"] == "tile"
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("p", [1, 2, 3])
+@pytest.mark.parametrize("make", ["c5", "c5T"])
+def test_device_loopback_gpu(p, make):
+    import torch
+    from tests._util import empty_device, from_device, to_device
+    n = 9
+    sa, sb = getattr(W, make)(p, n=n)
+    OA, OB = O.Layout(*W.spec_to_bases(sa)), O.Layout(*W.spec_to_bases(sb))
+    A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
+    P = 1 << p
+    plan = ll.ll_plan_convert(A, B, 2, comm=ll.Comm.loopback(P))
+    T = gen.random_bits(np.random.default_rng(1006), 1 << (2 * n), 2)
+    src = np.concatenate([_rank_src(OA, T, r) for r in range(P)])
+    d_src, d_dst = to_device(src), empty_device(src.size, 2)
+    ws = torch.empty(max(1, plan.workspace_bytes()), dtype=torch.uint8, device="cuda")
+    ll.ll_convert(d_src, d_dst, plan, workspace=ws)
+    got = from_device(d_dst, 2).reshape(P, -1)
+    for r in range(P):
+        assert np.array_equal(got[r], O.convert_distributed_rank(OA, OB, T, r)), r
+
+
+@pytest.mark.gpu
+def test_device_loopback_config5_large():
+    """Config 5 shape at P = 8 with a 2^13 x 2^13 bf16 tensor (128 MiB): every rank's
+    slice checked on sampled outputs against the oracle's closed form."""
+    import torch
+    n, p = 13, 3
+    sa, sb = W.c5(p, n=n)
+    OA, OB = O.Layout(*W.spec_to_bases(sa)), O.Layout(*W.spec_to_bases(sb))
+    A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
+    P = 1 << p
+    plan = ll.ll_plan_convert(A, B, 2, comm=ll.Comm.loopback(P))
+    total = 1 << (2 * n)
+    g = torch.Generator(device="cuda").manual_seed(1006)
+    T = torch.randint(-2 ** 15, 2 ** 15, (total,), dtype=torch.int16, device="cuda", generator=g)
+    # rank slices of A: src_r[h] = T[A(h, dev=r)], built from the oracle's index map
+    nloc = total // P
+    rng = np.random.default_rng(0)
+    src = torch.empty(total, dtype=torch.int16, device="cuda")
+    for r in range(P):
+        la, off = O.rank_slice(OA, r)
+        xs = O.apply_all(la, np.arange(nloc, dtype=np.uint64)) ^ np.uint64(off)
+        src[r * nloc:(r + 1) * nloc] = T[torch.from_numpy(xs.astype(np.int64)).cuda()]
+    dst = torch.empty_like(src)
+    ws = torch.empty(max(1, plan.workspace_bytes()), dtype=torch.uint8, device="cuda")
+    ll.ll_convert(src, dst, plan, workspace=ws)
+    torch.cuda.synchronize()
+    for r in range(P):
+        hs = rng.integers(0, nloc, size=1 << 16).astype(np.uint64)
+        lb, offb = O.rank_slice(OB, r)
+        xs = (O.apply_all(lb, hs) ^ np.uint64(offb)).astype(np.int64)
+        got = dst[r * nloc + torch.from_numpy(hs.astype(np.int64)).cuda()]
+        assert torch.equal(got, T[torch.from_numpy(xs).cuda()]), r

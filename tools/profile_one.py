@@ -1,0 +1,49 @@
+"""Run one hot-path kernel a few times (for ncu captures): --case c2 | c2smem | c3 |
+c3b | c1b | c1bsmem | gather_mma | gather_blocked | reduce_mma | reduce_blocked."""
+import argparse
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import torch  # noqa: E402
+
+import paper_conf_asplos_0001cgrnls0trm26_b200 as ll  # noqa: E402
+from workloads import configs as W  # noqa: E402
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--case", default="c2")
+ap.add_argument("--iters", type=int, default=3)
+a = ap.parse_args()
+
+conv = {"c2": (W.c2(16), 2, {}), "c2smem": (W.c2(16), 2, {"force_class": "SMEM"}),
+        "c3": (W.c3(14), 2, {}), "c3b": (W.c3b(14), 2, {}), "c1b": (W.c1_batched(20), 4, {}),
+        "c1bsmem": (W.c1_batched(20), 4, {"force_class": "SMEM"})}
+if a.case in conv:
+    (sa, sb), w, opts = conv[a.case]
+    A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
+    p = ll.ll_plan_convert(A, B, w, **opts)
+    n = (1 << A.d_in) * w // 2
+    src = torch.randint(-2 ** 15, 2 ** 15, (n,), dtype=torch.int16, device="cuda")
+    dst = torch.empty_like(src)
+    for _ in range(a.iters):
+        ll.ll_convert(src, dst, p)
+elif a.case.startswith("gather"):
+    fam = a.case.split("_")[1]
+    p = ll.ll_plan_gather(ll.Layout.from_spec(W.c4("gather", fam)), 1, 4)
+    n = 1 << 24
+    s = torch.randint(0, 1 << 30, (n,), dtype=torch.int32, device="cuda")
+    i = torch.randint(0, 32, (n,), dtype=torch.int32, device="cuda")
+    d = torch.empty_like(s)
+    for _ in range(a.iters):
+        ll.ll_gather(s, i, d, p)
+else:
+    fam = a.case.split("_")[1]
+    p = ll.ll_plan_reduce(ll.Layout.from_spec(W.c4("reduce", fam)), 1)
+    s = torch.rand(1 << 24, device="cuda")
+    d = torch.empty(p.out_elems(), device="cuda")
+    for _ in range(a.iters):
+        ll.ll_reduce(s, d, p)
+torch.cuda.synchronize()
+print("done", a.case)
