@@ -38,6 +38,16 @@ def hbm_peak():
         return FALLBACK_HBM, "fallback"
 
 
+def smem_conflicts():
+    """Bank conflicts per shared request of the SMEM-class kernel (config 3) from the
+    committed ncu captures (the metric's second part; config 2 itself uses no smem)."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "smem_conflicts.json")) as f:
+            return json.load(f)
+    except Exception:
+        return None
+
+
 def ncu_traffic(key):
     """Per-launch dram bytes (read + write) from the committed ncu --set full capture."""
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
@@ -262,6 +272,7 @@ def main():
                     "h2d_bytes_per_step": n * w, "d2h_bytes_per_step": n * w, "ms_per_step": round(e2e_ms, 3),
                     "matches_device_run": ok_e2e},
             "gpu_launches": args.steps,
+            "smem_bank_conflicts": smem_conflicts(),
             "clocks": clk.summary(),
         }
         if not args.no_cpu_baseline:

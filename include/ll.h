@@ -146,6 +146,39 @@ ll_status ll_left_divide(const ll_layout* M, const ll_layout* M1, ll_layout** M2
  * *n receives the count. */
 ll_status ll_kernel_basis(const ll_layout* L, int64_t* hw_vectors, int* n);
 
+/* ---------------------------------------------------------------- families --
+ * Layout families (§4.3).  Output dims are named "d0", "d1", ... (row-major, last
+ * fastest); all sizes are powers of two, else LL_ERR_INVALID_ARG.
+ *
+ * ll_layout_blocked (Prop 4.6 / 9.1): rank-`rank` tensor of
+ *   `shape`; sizePerThread / threadsPerWarp / warpsPerCTA per dim; order[0] is the
+ *   fastest dim.  Registers take sizePerThread bits in order, then lanes, then warps;
+ *   a CTA tile smaller than the shape repeats over further register bits (in order),
+ *   a larger one broadcasts (zero columns).  Fig. 1 A is
+ *   blocked([16,16],[2,2],[4,8],[2,1],[1,0]). */
+ll_status ll_layout_blocked(int rank, const int* shape, const int* size_per_thread,
+                            const int* threads_per_warp, const int* warps_per_cta,
+                            const int* order, ll_layout** L);
+/* ll_layout_mma_acc (Prop 4.7 / 9.2): the mma m16n8 / wgmma
+ * accumulator tile of an M x N output: reg0 -> j0, lanes (j1, j2, i0, i1, i2),
+ * reg1 -> i3; warps along M first, then N; n-repetitions, then m-repetitions
+ * as further register bits. */
+ll_status ll_layout_mma_acc(int M, int N, int warps_m, int warps_n, ll_layout** L);
+/* ll_layout_mma_swizzle (Def 4.11, Prop 4.12): the memory layout
+ * offset -> (i, j) of a 2^m x 2^n tile, matrix [[I_n, C], [0, I_m]] with
+ * c_i = (vec·((2^i/per_phase) mod max_phase)) mod 2^n. */
+ll_status ll_layout_mma_swizzle(int log2_rows, int log2_cols, int vec, int per_phase,
+                                int max_phase, ll_layout** L);
+/* ll_layout_contiguity (§5.1 "Contiguous elements"): the number of
+ * elements each thread can move with one vector instruction — the largest u with
+ * L^{-1}_Reg(i) = i for all i < u (leading register bits mapping in order to the
+ * lowest logical bits, across dimensions), capped at max_vec_bytes (default 16 =
+ * v4.b32). */
+ll_status ll_layout_contiguity(const ll_layout* L, int elem_bytes, int max_vec_bytes, int* elems);
+/* ll_layout_slice (Prop 4.8): drop logical dim `dim` (the result stays
+ * surjective and may gain zero columns, Remark P:224). */
+ll_status ll_layout_slice(const ll_layout* L, int dim, ll_layout** out);
+
 /* ---------------------------------------------------------------- conversion --
  * ll_plan_convert (rows a2-a4, a6-a9).  Host only.
  *   A, B: same output dims; A surjective.  elem_bytes in {1, 2, 4, 8}.

@@ -77,6 +77,11 @@ _sig = {
     "ll_comm_get_unique_id": [_P],
     "ll_comm_create_loopback": [C.c_int, _PP],
     "ll_plan_device_stages": [_P, _PP, _PP, C.POINTER(C.c_size_t), C.POINTER(C.c_int)],
+    "ll_layout_blocked": [C.c_int] + [C.POINTER(C.c_int)] * 5 + [_PP],
+    "ll_layout_mma_acc": [C.c_int, C.c_int, C.c_int, C.c_int, _PP],
+    "ll_layout_mma_swizzle": [C.c_int] * 5 + [_PP],
+    "ll_layout_slice": [_P, C.c_int, _PP],
+    "ll_layout_contiguity": [_P, C.c_int, C.c_int, C.POINTER(C.c_int)],
 }
 for _name, _args in _sig.items():
     _f = getattr(_lib, _name)
@@ -155,9 +160,9 @@ class Layout:
 
     def __del__(self):
         h = getattr(self, "handle", None)
-        if h:
+        if h and _lib is not None:
             _lib.ll_layout_destroy(h)
-            self.handle = None
+        self.handle = None
 
     def _info(self):
         a, b, c, d = C.c_int(), C.c_int(), C.c_int(), C.c_int()
@@ -239,11 +244,47 @@ class Layout:
         _check(_lib.ll_left_divide(self.handle, M1.handle, C.byref(h)))
         return Layout(None, None, _handle=h)
 
+    def contiguity(self, elem_bytes: int, max_vec_bytes: int = 16) -> int:
+        """Contiguous elements per thread, capped at max_vec_bytes."""
+        e = C.c_int()
+        _check(_lib.ll_layout_contiguity(self.handle, int(elem_bytes), int(max_vec_bytes), C.byref(e)))
+        return e.value
+
     def kernel_basis(self) -> List[int]:
         arr = (C.c_int64 * 64)()
         n = C.c_int()
         _check(_lib.ll_kernel_basis(self.handle, arr, C.byref(n)))
         return list(arr[:n.value])
+
+
+def _ints(v):
+    return (C.c_int * len(v))(*[int(x) for x in v])
+
+
+def ll_layout_blocked(shape, size_per_thread, threads_per_warp, warps_per_cta, order) -> Layout:
+    """Blocked layout (Prop 9.1); see include/ll.h."""
+    h = C.c_void_p()
+    _check(_lib.ll_layout_blocked(len(shape), _ints(shape), _ints(size_per_thread), _ints(threads_per_warp),
+                                  _ints(warps_per_cta), _ints(order), C.byref(h)))
+    return Layout(None, None, _handle=h)
+
+
+def ll_layout_mma_acc(M, N, warps_m, warps_n=1) -> Layout:
+    h = C.c_void_p()
+    _check(_lib.ll_layout_mma_acc(M, N, warps_m, warps_n, C.byref(h)))
+    return Layout(None, None, _handle=h)
+
+
+def ll_layout_mma_swizzle(log2_rows, log2_cols, vec, per_phase, max_phase) -> Layout:
+    h = C.c_void_p()
+    _check(_lib.ll_layout_mma_swizzle(log2_rows, log2_cols, vec, per_phase, max_phase, C.byref(h)))
+    return Layout(None, None, _handle=h)
+
+
+def ll_layout_slice(L: Layout, dim: int) -> Layout:
+    h = C.c_void_p()
+    _check(_lib.ll_layout_slice(L.handle, dim, C.byref(h)))
+    return Layout(None, None, _handle=h)
 
 
 # ---- ABI-named functions -------------------------------------------------------------
@@ -287,9 +328,9 @@ class Plan:
 
     def __del__(self):
         h = getattr(self, "handle", None)
-        if h:
+        if h and _lib is not None:
             _lib.ll_plan_destroy(h)
-            self.handle = None
+        self.handle = None
 
     @property
     def cls(self) -> str:
@@ -384,9 +425,9 @@ class Comm:
 
     def __del__(self):
         h = getattr(self, "handle", None)
-        if h:
+        if h and _lib is not None:
             _lib.ll_comm_destroy(h)
-            self.handle = None
+        self.handle = None
 
 
 def ll_plan_convert(A: Layout, B: Layout, elem_bytes: int, **opts) -> Plan:

@@ -295,6 +295,56 @@ ll_status ll_kernel_basis(const ll_layout* L, int64_t* v, int* n) {
   LL_CATCH
 }
 
+ll_status ll_layout_blocked(int rank, const int* shape, const int* size_per_thread, const int* threads_per_warp,
+                            const int* warps_per_cta, const int* order, ll_layout** out) {
+  LL_TRY
+  if (rank < 1 || !shape || !size_per_thread || !threads_per_warp || !warps_per_cta || !order || !out)
+    fail(LL_ERR_INVALID_ARG, "null argument");
+  std::vector<int> sh(shape, shape + rank), s(size_per_thread, size_per_thread + rank),
+      t(threads_per_warp, threads_per_warp + rank), w(warps_per_cta, warps_per_cta + rank), o(order, order + rank);
+  std::vector<int> seen(rank, 0);
+  for (int d : o) { if (d < 0 || d >= rank || seen[d]++) fail(LL_ERR_INVALID_ARG, "order must be a permutation"); }
+  *out = new ll_layout{make_blocked(sh, s, t, w, o)};
+  LL_CATCH
+}
+
+ll_status ll_layout_mma_acc(int M, int N, int warps_m, int warps_n, ll_layout** out) {
+  LL_TRY
+  if (!out) fail(LL_ERR_INVALID_ARG, "null argument");
+  *out = new ll_layout{make_mma_acc(M, N, warps_m, warps_n)};
+  LL_CATCH
+}
+
+ll_status ll_layout_mma_swizzle(int log2_rows, int log2_cols, int vec, int per_phase, int max_phase, ll_layout** out) {
+  LL_TRY
+  if (!out || log2_rows < 0 || log2_cols < 0 || log2_rows + log2_cols > 62) fail(LL_ERR_INVALID_ARG, "bad argument");
+  *out = new ll_layout{make_mma_swizzle(log2_rows, log2_cols, vec, per_phase, max_phase)};
+  LL_CATCH
+}
+
+ll_status ll_layout_contiguity(const ll_layout* L, int elem_bytes, int max_vec_bytes, int* elems) {
+  LL_TRY
+  if (!L || !elems || elem_bytes <= 0) fail(LL_ERR_INVALID_ARG, "bad argument");
+  // the largest u with L^{-1}_Reg(i) = i for all i < u, i.e. the number of
+  // leading register bits that map, in order, to logical flat bits 0, 1, 2, ...;
+  // capped by the widest vector instruction (v4.b32).
+  const Layout& l = L->L;
+  int p = l.in_pos("reg"), nb = l.in_bits("reg"), k = 0;
+  while (p >= 0 && k < nb && l.cols[p + k] == (u64(1) << k)) ++k;
+  int cap = max_vec_bytes > 0 ? max_vec_bytes : 16;
+  int e = 1 << k;
+  while (e > 1 && e * elem_bytes > cap) e >>= 1;
+  *elems = e;
+  LL_CATCH
+}
+
+ll_status ll_layout_slice(const ll_layout* L, int dim, ll_layout** out) {
+  LL_TRY
+  if (!L || !out) fail(LL_ERR_INVALID_ARG, "null argument");
+  *out = new ll_layout{make_slice(L->L, dim)};
+  LL_CATCH
+}
+
 ll_status ll_plan_convert(const ll_layout* A, const ll_layout* B, int w, const ll_plan_opts* opts, ll_plan** plan) {
   LL_TRY
   if (!A || !B || !plan) fail(LL_ERR_INVALID_ARG, "null argument");

@@ -1,5 +1,6 @@
 // Specialisation of the sm_100a kernel templates (ll_kernels.cuh): emits the plan
 // constants as a `struct P` of compile-time tables and instantiates the entry point.
+#include <cstdlib>
 #include <sstream>
 #include <type_traits>
 
@@ -55,6 +56,9 @@ std::string codegen_tile(const ConvPlan& Pl) {
   o << icon("W", T.w) << icon("R", T.R) << icon("WB", T.Wb)
     << icon("NW", std::max<long long>(1, ((1ll << T.R) * T.w) / 4))
     << icon("VLD", T.vld) << icon("VST", T.vst) << icon("XCHG", T.xchg) << icon("THREADS", T.threads());
+  o << "  static constexpr bool ISOLATE_SMEM = " << (std::getenv("LL_ISOLATE_SMEM") ? "true" : "false") << ";\n";
+  // per-thread-contiguous loads (faithful σ) re-use sectors across instructions
+  o << "  static constexpr bool LD_L1 = " << (T.sigma == SIGMA_FAITHFUL ? "true" : "false") << ";\n";
   std::vector<u64> ldc, stc;
   for (int b = 0; b < T.n; ++b) {
     ldc.push_back(u64(1) << (T.ld_bit[b] + lw));
@@ -88,6 +92,7 @@ std::string codegen_gather(const GatherPlan& G) {
   o << "struct P {\n";
   o << icon("W", G.w) << icon("R", G.R) << icon("WB", G.Wb)
     << icon("NW", std::max<long long>(1, ((1ll << G.R) * G.w) / 4)) << icon("VLD", G.v);
+  o << "  static constexpr bool LD_L1 = " << (G.sigma == SIGMA_FAITHFUL ? "true" : "false") << ";\n";
   std::vector<u64> ldc;
   for (int b = 0; b < n; ++b) ldc.push_back(u64(1) << G.hw_bit[b]);   // element offsets
   o << arr("u64", "LD_COL", ldc);
@@ -115,41 +120,29 @@ std::string codegen_gather(const GatherPlan& G) {
 }
 
 std::string codegen_reduce(const ReducePlan& Rp) {
-  const Layout& L = Rp.L;
   std::ostringstream o;
   o << "struct P {\n";
-  const int R = Rp.R;
-  int v = std::min(2, R);
-  o << icon("W", 4) << icon("R", R) << icon("WB", Rp.Wb) << icon("VLD", v);
+  const int R = Rp.R, n = int(Rp.hw_bit.size());
+  o << icon("W", 4) << icon("R", R) << icon("WB", Rp.Wb) << icon("VLD", Rp.v);
+  o << "  static constexpr bool LD_L1 = " << (Rp.sigma == SIGMA_FAITHFUL ? "true" : "false") << ";\n";
   std::vector<u64> ldc;
-  for (int b = 0; b < R + 5 + Rp.Wb; ++b) ldc.push_back(u64(4) << b);
+  for (int b = 0; b < n; ++b) ldc.push_back(u64(4) << Rp.hw_bit[b]);
   o << arr("u64", "LD_COL", ldc);
-  std::vector<int> gsh;
   emit_grid(o, Rp.grid_bit, Rp.grid_bit, 2);
-  std::vector<u64> gout;
-  for (int k : Rp.grid_bit) gout.push_back(Rp.out_col[k]);
-  o << arr("u64", "GRID_OUT", gout);
-  std::vector<u64> oc(Rp.out_col.begin(), Rp.out_col.begin() + (R + 5 + Rp.Wb));
-  o << arr("u64", "OUT_COL", oc);
-  auto rel = [&](const std::vector<int>& bits, int base) {
-    std::vector<int> r;
-    for (int k : bits) r.push_back(k - base);
-    return r;
-  };
-  auto rr = rel(Rp.red_reg, 0), rl = rel(Rp.red_lane, R), rw = rel(Rp.red_warp, R + 5);
+  o << arr("u64", "GRID_OUT", Rp.grid_out) << arr("u64", "OUT_COL", Rp.out_col);
   int regmask = 0, dupreg = 0;
   uint32_t nolane = 0, nowarp = 0, rwmask = 0;
-  for (int b : rr) regmask |= 1 << b;
-  for (int b : rl) nolane |= 1u << b;
-  for (int b : rw) { nowarp |= 1u << b; rwmask |= 1u << b; }
+  for (int b : Rp.red_reg) regmask |= 1 << b;
+  for (int b : Rp.red_lane) nolane |= 1u << b;
+  for (int b : Rp.red_warp) { nowarp |= 1u << b; rwmask |= 1u << b; }
   for (int k : Rp.dup_bits) {
     if (k < R) dupreg |= 1 << k;
     else if (k < R + 5) nolane |= 1u << (k - R);
-    else if (k < R + 5 + Rp.Wb) nowarp |= 1u << (k - R - 5);
+    else nowarp |= 1u << (k - R - 5);
   }
-  o << icon("NRED_REG", rr.size()) << arr("int", "RED_REG", rr) << icon("RED_REG_MASK", regmask)
-    << icon("DUP_REG_MASK", dupreg) << icon("NRED_LANE", rl.size()) << arr("int", "RED_LANE", rl)
-    << icon("NRED_WARP", rw.size()) << arr("int", "RED_WARP", rw);
+  o << icon("NRED_REG", Rp.red_reg.size()) << arr("int", "RED_REG", Rp.red_reg) << icon("RED_REG_MASK", regmask)
+    << icon("DUP_REG_MASK", dupreg) << icon("NRED_LANE", Rp.red_lane.size()) << arr("int", "RED_LANE", Rp.red_lane)
+    << icon("NRED_WARP", Rp.red_warp.size()) << arr("int", "RED_WARP", Rp.red_warp);
   o << "  static constexpr u32 NOSTORE_LANE_MASK = " << nolane << "u;\n"
     << "  static constexpr u32 NOSTORE_WARP_MASK = " << nowarp << "u;\n"
     << "  static constexpr u32 RED_WARP_MASK = " << rwmask << "u;\n";
@@ -161,7 +154,6 @@ std::string codegen_reduce(const ReducePlan& Rp) {
   o << "extern \"C\" __global__ void __launch_bounds__(" << (32 << Rp.Wb)
     << ") ll_reduce_kernel(const float* __restrict__ src, float* __restrict__ dst, u64 ntiles) {\n"
     << "  ll_reduce_body<P>(src, dst, ntiles);\n}\n";
-  (void)L;
   return o.str();
 }
 

@@ -247,3 +247,99 @@ Layout left_divide(const Layout& M, const Layout& M1) {
 }
 
 }  // namespace ll
+
+// ---------------------------------------------------------------------------
+// Layout families (§4.3; Props 9.1 / 9.2).  Output dims are "d0", "d1", ...
+// (row-major, last fastest).
+// ---------------------------------------------------------------------------
+namespace ll {
+
+static int lg2(int v) {
+  if (v <= 0 || (v & (v - 1))) fail(LL_ERR_INVALID_ARG, "sizes must be powers of two (P:128)");
+  return 31 - __builtin_clz(unsigned(v));
+}
+
+Layout make_blocked(const std::vector<int>& shape, const std::vector<int>& spt, const std::vector<int>& tpw,
+                    const std::vector<int>& wpc, const std::vector<int>& order) {
+  // Prop 9.1: σ_o^{-1} ∘ (id_R^o × id_T^o × id_W^o) — registers take sizePerThread in
+  // `order` (fastest first), then lanes, then warps; if the CTA tile is smaller than the
+  // shape the remaining bits become further registers in `order` (repetition); if it is
+  // larger, the excess bits are zero columns (broadcast).
+  const size_t nd = shape.size();
+  if (spt.size() != nd || tpw.size() != nd || wpc.size() != nd || order.size() != nd)
+    fail(LL_ERR_INVALID_ARG, "blocked: rank mismatch");
+  Layout L;
+  std::vector<int> sb(nd), used(nd, 0);
+  for (size_t d = 0; d < nd; ++d) { sb[d] = lg2(shape[d]); L.out.push_back({"d" + std::to_string(d), sb[d]}); }
+  auto flat_bit = [&](size_t d, int b) -> u64 {
+    if (b >= sb[d]) return 0;
+    int sh = 0;
+    for (size_t e = d + 1; e < nd; ++e) sh += sb[e];
+    return u64(1) << (sh + b);
+  };
+  auto take = [&](const std::vector<int>& cnt, std::vector<u64>& cols) {
+    for (int d : order) for (int k = 0; k < lg2(cnt[d]); ++k) cols.push_back(flat_bit(d, used[d]++));
+  };
+  std::vector<u64> reg, lane, warp;
+  take(spt, reg);
+  take(tpw, lane);
+  take(wpc, warp);
+  for (int d : order) while (used[d] < sb[d]) reg.push_back(flat_bit(d, used[d]++));
+  L.in = {{"reg", int(reg.size())}, {"lane", int(lane.size())}, {"warp", int(warp.size())}};
+  L.cols = reg;
+  L.cols.insert(L.cols.end(), lane.begin(), lane.end());
+  L.cols.insert(L.cols.end(), warp.begin(), warp.end());
+  return L;
+}
+
+Layout make_mma_acc(int M, int N, int warps_m, int warps_n) {
+  // Prop 9.2 / G17: m16n8 accumulator fragment reg0->j0, lanes (j1,j2,i0,i1,i2),
+  // reg1->i3; warps along M first (wgmma); n-repetitions then m-repetitions.
+  const int mb = lg2(M), nb = lg2(N), wm = lg2(warps_m), wn = lg2(warps_n);
+  auto I = [&](int k) -> u64 { return k < mb ? (u64(1) << (nb + k)) : 0; };
+  auto J = [&](int k) -> u64 { return k < nb ? (u64(1) << k) : 0; };
+  std::vector<u64> reg = {J(0), I(3)}, lane = {J(1), J(2), I(0), I(1), I(2)}, warp;
+  for (int k = 0; k < wm; ++k) warp.push_back(I(4 + k));
+  for (int k = 0; k < wn; ++k) warp.push_back(J(3 + k));
+  for (int k = 3 + wn; k < nb; ++k) reg.push_back(J(k));
+  for (int k = 4 + wm; k < mb; ++k) reg.push_back(I(k));
+  Layout L;
+  L.out = {{"d0", mb}, {"d1", nb}};
+  L.in = {{"reg", int(reg.size())}, {"lane", 5}, {"warp", int(warp.size())}};
+  L.cols = reg;
+  L.cols.insert(L.cols.end(), lane.begin(), lane.end());
+  L.cols.insert(L.cols.end(), warp.begin(), warp.end());
+  return L;
+}
+
+Layout make_mma_swizzle(int m, int n, int vec, int per_phase, int max_phase) {
+  // Def 4.11 as the memory layout offset -> (i, j): the matrix
+  // [[I_n, C], [0, I_m]] with c_i = (vec · ((2^i / per_phase) mod max_phase)) mod 2^n;
+  // the matrix is an involution, so it is both directions of the map.
+  if (vec <= 0 || per_phase <= 0 || max_phase <= 0) fail(LL_ERR_INVALID_ARG, "swizzle parameters must be > 0");
+  lg2(vec); lg2(per_phase); lg2(max_phase);
+  Layout L;
+  L.out = {{"d0", m}, {"d1", n}};
+  L.in = {{"offset", m + n}};
+  for (int k = 0; k < n; ++k) L.cols.push_back(u64(1) << k);
+  for (int i = 0; i < m; ++i) {
+    u64 c = (u64(vec) * u64(((u64(1) << i) / per_phase) % max_phase)) % (u64(1) << n);
+    L.cols.push_back((u64(1) << (n + i)) | c);
+  }
+  return L;
+}
+
+Layout make_slice(const Layout& L, int dim) {
+  // Prop 4.8: remove logical dim `dim` (Remark P:224: stays surjective, may gain zero
+  // columns).
+  if (dim < 0 || dim >= int(L.out.size())) fail(LL_ERR_INVALID_ARG, "slice: dim out of range");
+  Layout R;
+  R.in = L.in;
+  for (int i = 0; i < int(L.out.size()); ++i) if (i != dim) R.out.push_back(L.out[i]);
+  const int sh = L.out_shift(dim), b = L.out[dim].bits;
+  const u64 lo = (u64(1) << sh) - 1;
+  for (u64 c : L.cols) R.cols.push_back((c & lo) | ((c >> (sh + b)) << sh));
+  return R;
+}
+
+}  // namespace ll

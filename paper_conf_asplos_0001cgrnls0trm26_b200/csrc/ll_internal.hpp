@@ -115,6 +115,11 @@ Layout compose(const Layout& outer, const Layout& inner);     // Def 4.2
 Layout invert(const Layout& L);                                // Def 4.5
 Layout product(const Layout& L1, const Layout& L2);            // Def 4.3
 Layout left_divide(const Layout& M, const Layout& M1);         // Def 4.4
+Layout make_blocked(const std::vector<int>& shape, const std::vector<int>& spt, const std::vector<int>& tpw,
+                    const std::vector<int>& wpc, const std::vector<int>& order);   // Prop 9.1
+Layout make_mma_acc(int M, int N, int warps_m, int warps_n);                     // Prop 9.2
+Layout make_mma_swizzle(int m, int n, int vec, int per_phase, int max_phase);    // Def 4.11
+Layout make_slice(const Layout& L, int dim);                                     // Prop 4.8
 
 // ------------------------------------------------------------------ plans
 enum ExecKind { EXEC_NOOP = 0, EXEC_TILE = 1, EXEC_GENERIC = 2, EXEC_DEVICE = 3 };
@@ -216,11 +221,15 @@ struct ReducePlan {
   Layout L;
   int axis = 0;
   int exec = EXEC_TILE;
-  int R = 0, Wb = 0;
-  std::vector<int> grid_bit;      // CTA index bit -> packed bit
-  std::vector<int> red_reg, red_lane, red_warp;   // reduced kernel bits (L order)
+  int sigma = SIGMA_COALESCED;
+  int R = 0, Wb = 0, v = 0;
+  std::vector<int> hw_bit;        // kernel bit -> packed bit of L (σ)
+  std::vector<int> grid_bit;      // CTA index bit -> packed bit (non-duplicate block bits)
+  // reduced kernel bits, each list ascending: the fixed order is reg, lane, warp
+  std::vector<int> red_reg, red_lane, red_warp;
   std::vector<int> dup_bits;      // zero-column kernel bits (de-dup)
-  std::vector<u64> out_col;       // per packed bit: output flat offset (0 for reduced/dup)
+  std::vector<u64> out_col;       // per kernel bit: output flat offset (0 for reduced/dup)
+  std::vector<u64> grid_out;      // per grid bit: output flat offset
   u64 out_elems = 0;
   std::string source;
   void* kernel = nullptr;

@@ -53,16 +53,31 @@ template <int W, int E> __device__ __forceinline__ void set_e(u32* r, u32 v) {
 }
 
 // ------------------------------------------------------------------ global memory
+// Global loads.  L1A = false: streaming (.L1::no_allocate) for coalesced σ, where a
+// warp instruction covers whole lines; L1A = true: L1-allocating read-only loads for
+// per-thread-contiguous σ, where consecutive instructions of a lane share sectors.
+template <bool L1A>
 __device__ __forceinline__ void ldg_v4(const u8* p, u32& a, u32& b, u32& c, u32& d) {
-  asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
-               : "=r"(a), "=r"(b), "=r"(c), "=r"(d) : "l"(p));
+  if constexpr (L1A)
+    asm volatile("ld.global.nc.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(a), "=r"(b), "=r"(c), "=r"(d) : "l"(p));
+  else
+    asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(a), "=r"(b), "=r"(c), "=r"(d) : "l"(p));
 }
+template <bool L1A>
 __device__ __forceinline__ void ldg_v2(const u8* p, u32& a, u32& b) {
-  asm volatile("ld.global.nc.L1::no_allocate.v2.u32 {%0,%1}, [%2];" : "=r"(a), "=r"(b) : "l"(p));
+  if constexpr (L1A)
+    asm volatile("ld.global.nc.v2.u32 {%0,%1}, [%2];" : "=r"(a), "=r"(b) : "l"(p));
+  else
+    asm volatile("ld.global.nc.L1::no_allocate.v2.u32 {%0,%1}, [%2];" : "=r"(a), "=r"(b) : "l"(p));
 }
+template <bool L1A>
 __device__ __forceinline__ u32 ldg_b32(const u8* p) {
   u32 a;
-  asm volatile("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(a) : "l"(p));
+  if constexpr (L1A)
+    asm volatile("ld.global.nc.u32 %0, [%1];" : "=r"(a) : "l"(p));
+  else
+    asm volatile("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(a) : "l"(p));
   return a;
 }
 __device__ __forceinline__ void stg_v4(u8* p, u32 a, u32 b, u32 c, u32 d) {
@@ -76,16 +91,16 @@ __device__ __forceinline__ void stg_b32(u8* p, u32 a) {
 }
 
 // Load vector K of the thread (2^VL elements of W bytes starting at slot K<<VL).
-template <int W, int VL, int K, int NW>
+template <int W, int VL, int K, int NW, bool L1A = false>
 __device__ __forceinline__ void load_vec(u32 (&r)[NW], const u8* p) {
   constexpr int VB = W << VL;                 // vector bytes
   constexpr int E0 = K << VL;
   if constexpr (VB == 16) {
-    ldg_v4(p, r[E0 * W / 4 + 0], r[E0 * W / 4 + 1], r[E0 * W / 4 + 2], r[E0 * W / 4 + 3]);
+    ldg_v4<L1A>(p, r[E0 * W / 4 + 0], r[E0 * W / 4 + 1], r[E0 * W / 4 + 2], r[E0 * W / 4 + 3]);
   } else if constexpr (VB == 8) {
-    ldg_v2(p, r[E0 * W / 4 + 0], r[E0 * W / 4 + 1]);
+    ldg_v2<L1A>(p, r[E0 * W / 4 + 0], r[E0 * W / 4 + 1]);
   } else if constexpr (VB == 4) {
-    r[E0 * W / 4] = ldg_b32(p);
+    r[E0 * W / 4] = ldg_b32<L1A>(p);
   } else if constexpr (VB == 2) {
     set_e<2, E0 * W / 2>(r, u32(*reinterpret_cast<const u16*>(p)));
   } else {
@@ -345,6 +360,20 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, u8* __r
   const u64 ld_thr = thread_base<P, true>(lane, warp);
   const u64 st_thr = thread_base<P, false>(lane, warp);
   const u32 sbase = u32(__cvta_generic_to_shared(ll_smem));
+  if constexpr (P::XCHG == 3 && P::ISOLATE_SMEM) {
+    // Diagnostic variant (codegen env LL_ISOLATE_SMEM=1): the smem exchange alone,
+    // 16 times, with no global traffic — separates true bank conflicts from L1 data
+    // pipe contention with concurrent global loads in ncu's counters.
+    u32 r[P::NW], o[P::NW];
+    static_for<P::NW>([&](auto q) { r[decltype(q)::value] = threadIdx.x * 131u + decltype(q)::value; });
+    for (int it = 0; it < 16; ++it) {
+      xchg_smem<P>(r, o, lane, warp, sbase);
+      __syncthreads();
+      static_for<P::NW>([&](auto q) { r[decltype(q)::value] = o[decltype(q)::value] + 1u; });
+    }
+    if (r[0] == 0x9e3779b9u) dst[threadIdx.x] = u8(r[P::NW - 1]);
+    return;
+  }
   for (u64 t = blockIdx.x; t < ntiles; t += gridDim.x) {
     const u8* s = src + (tile_base<P, true>(t) ^ ld_thr);
     u8* d = dst + (tile_base<P, false>(t) ^ st_thr);
@@ -352,7 +381,7 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, u8* __r
     // a5: HBM load of the src tile (16-byte vectors; coalesced under σ_ld)
     static_for<(1 << (P::R - P::VLD))>([&](auto k) {
       constexpr int K = decltype(k)::value;
-      load_vec<P::W, P::VLD, K>(r, s + LdOff<P, K>::value());
+      load_vec<P::W, P::VLD, K, P::NW, P::LD_L1>(r, s + LdOff<P, K>::value());
     });
     u32 o[P::NW];
     if constexpr (P::XCHG == 0) {
@@ -397,8 +426,8 @@ __device__ __forceinline__ void ll_gather_body(const u8* __restrict__ src, const
     u32 ix[1 << P::R];
     static_for<(1 << (P::R - P::VLD))>([&](auto k) {
       constexpr int K = decltype(k)::value;
-      load_vec<P::W, P::VLD, K>(r, src + (eoff ^ LdOff<P, K>::value()) * P::W);
-      load_vec<4, P::VLD, K>(ix, idx + (eoff ^ LdOff<P, K>::value()) * 4);
+      load_vec<P::W, P::VLD, K, P::NW, P::LD_L1>(r, src + (eoff ^ LdOff<P, K>::value()) * P::W);
+      load_vec<4, P::VLD, K, (1 << P::R), P::LD_L1>(ix, idx + (eoff ^ LdOff<P, K>::value()) * 4);
     });
     u32 o[P::NW];
     static_for<P::NW>([&](auto q) { o[decltype(q)::value] = 0; });
@@ -463,7 +492,7 @@ __device__ __forceinline__ void ll_reduce_body(const float* __restrict__ src, fl
     u32 r[1 << P::R];
     static_for<(1 << (P::R - P::VLD))>([&](auto k) {
       constexpr int K = decltype(k)::value;
-      load_vec<4, P::VLD, K>(r, s + LdOff<P, K>::value());
+      load_vec<4, P::VLD, K, (1 << P::R), P::LD_L1>(r, s + LdOff<P, K>::value());
     });
     // register tree, in the layout's register-bit order
     static_for<P::NRED_REG>([&](auto i) {

@@ -1,6 +1,7 @@
 // Conversion planner (rows a3, a4, a6-a9) plus gather (a11) and
 // reduce (a12) plans.
 #include <algorithm>
+#include <functional>
 #include <cstring>
 #include <sstream>
 
@@ -690,6 +691,35 @@ std::string describe(const ConvPlan& P) {
 // ---------------------------------------------------------------------------
 // Gather (§5.5)
 // ---------------------------------------------------------------------------
+// Line-coalesced kernel decomposition for the single-layout kernels (gather, reduce;
+// DESIGN.md §5.6-5.7).  Tile bits (reg, lane, warp of L) in packed order t0 < t1 < ...:
+//   kreg[0, v)  = the v lowest reg/lane bits (one 16-byte vector per thread),
+//   klane[0, 3) = the next 3 bits (8 lanes cover one 128-byte line),
+//   klane[3, 5) = two of the remaining reg/lane bits, those with pref(bit) = true
+//                 first, then ascending,
+//   kreg[v, R)  = the remaining reg/lane bits ascending,
+//   kernel warps = L's warp bits.
+static std::vector<int> sigma_line(const Layout& L, int v, const std::function<bool(int)>& pref) {
+  auto regb = bits_at_level(L, 0, 0), laneb = bits_at_level(L, 1, 1), warpb = bits_at_level(L, 2, 2);
+  const int R = int(regb.size());
+  std::vector<int> nw = regb;
+  nw.insert(nw.end(), laneb.begin(), laneb.end());
+  std::sort(nw.begin(), nw.end());
+  if (R < v || int(nw.size()) != R + 5) fail(LL_ERR_UNSUPPORTED, "line σ: bad tile");
+  std::vector<int> hw(R + 5 + warpb.size());
+  for (int b = 0; b < v; ++b) hw[b] = nw[b];
+  for (int t = 0; t < 3; ++t) hw[R + t] = nw[v + t];
+  std::vector<int> rest(nw.begin() + v + 3, nw.end());
+  std::stable_sort(rest.begin(), rest.end(), [&](int a, int b) { return pref(a) && !pref(b); });
+  hw[R + 3] = rest[0];
+  hw[R + 4] = rest[1];
+  std::vector<int> regs(rest.begin() + 2, rest.end());
+  std::sort(regs.begin(), regs.end());
+  for (int b = v; b < R; ++b) hw[b] = regs[b - v];
+  for (size_t t = 0; t < warpb.size(); ++t) hw[R + 5 + t] = warpb[t];
+  return hw;
+}
+
 std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const ll_plan_opts* opts) {
   if (w != 1 && w != 2 && w != 4 && w != 8) fail(LL_ERR_INVALID_ARG, "elem_bytes must be 1, 2, 4 or 8");
   if (axis < 0 || axis >= int(L.out.size())) fail(LL_ERR_INVALID_ARG, "axis out of range");
@@ -728,25 +758,13 @@ std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const 
   for (int k : regb) faith.push_back(k);
   for (int k : laneb) faith.push_back(k);
   for (int k : warpb) faith.push_back(k);
-  std::vector<int> coal(faith.size());
-  // tile bits in packed order: reg (0..R-1), lane (R..R+4), warp
-  std::vector<int> Ts = tileb;
-  std::sort(Ts.begin(), Ts.end());
-  for (int b = 0; b < v; ++b) coal[b] = Ts[b];
-  for (int t = 0; t < 5; ++t) coal[R + t] = Ts[v + t];
-  {
-    std::vector<int> rest(Ts.begin() + v + 5, Ts.end());
-    // warps keep L's warp bits (axis-free) so L_Wrp^axis stays 0
-    std::vector<int> wr;
-    for (int k : warpb) { wr.push_back(k); rest.erase(std::find(rest.begin(), rest.end(), k)); }
-    for (int b = v; b < R; ++b) coal[b] = rest[b - v];
-    for (size_t t = 0; t < wr.size(); ++t) coal[R + 5 + t] = wr[t];
-    // coalesced σ only valid if the warp bits were not consumed by reg/lane positions
-    for (int b = 0; b < R + 5; ++b)
-      if (std::find(warpb.begin(), warpb.end(), coal[b]) != warpb.end()) { coal.clear(); break; }
-  }
+  // coalesced (line σ with the axis bits preferred in the free lanes, so that fewer
+  // candidates remain in registers) unless faithful is requested: measured on B200,
+  // coalesced loads beat faithful ones even at 2x the shuffles (profiles/r01_*).
+  std::vector<int> coal = sigma_line(L, v, [&](int k) { return (L.cols[k] & amask) != 0; });
   int sigma = opts ? opts->sigma : 0;
-  bool use_coal = !coal.empty() && sigma != SIGMA_FAITHFUL && cand_of(coal) <= cand_of(faith);
+  bool use_coal = sigma != SIGMA_FAITHFUL;
+  (void)cand_of;
   G->hw_bit = use_coal ? coal : faith;
   G->sigma = use_coal ? SIGMA_COALESCED : SIGMA_FAITHFUL;
   G->R = R;
@@ -773,7 +791,6 @@ std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const 
 // ascending) is exactly the layout's.
 // ---------------------------------------------------------------------------
 std::unique_ptr<ReducePlan> plan_reduce(const Layout& L, int axis, const ll_plan_opts* opts) {
-  (void)opts;
   if (axis < 0 || axis >= int(L.out.size())) fail(LL_ERR_INVALID_ARG, "axis out of range");
   if (!L.distributed()) fail(LL_ERR_UNSUPPORTED, "reduce: L must be a distributed layout (Def 4.10)");
   if (L.in_bits("lane") != 5) fail(LL_ERR_UNSUPPORTED, "reduce: 5 lane bits required");
@@ -782,7 +799,8 @@ std::unique_ptr<ReducePlan> plan_reduce(const Layout& L, int axis, const ll_plan
   Rp->L = L; Rp->axis = axis;
   const int sh = L.out_shift(axis), ab = L.out[axis].bits;
   const u64 amask = ((u64(1) << ab) - 1) << sh;
-  Rp->R = L.in_bits("reg");
+  const int R = L.in_bits("reg");
+  Rp->R = R;
   Rp->Wb = L.in_bits("warp");
   // K: number of in-tile (non-block) axis bits; they must be the low axis bits
   int K = 0;
@@ -792,36 +810,51 @@ std::unique_ptr<ReducePlan> plan_reduce(const Layout& L, int axis, const ll_plan
     for (int k : bits_at_level(L, 0, 2)) if (L.cols[k] == (u64(1) << (sh + t))) f = true;
     if (!f) fail(LL_ERR_UNSUPPORTED, "reduce: in-tile axis bits must be the low axis bits");
   }
-  auto classify_bits = [&](int lev, std::vector<int>& red) {
-    for (int k : bits_at_level(L, lev, lev)) {
-      if (L.cols[k] == 0) Rp->dup_bits.push_back(k);
-      else if (L.cols[k] & amask) red.push_back(k);
-    }
-  };
-  classify_bits(0, Rp->red_reg);
-  classify_bits(1, Rp->red_lane);
-  classify_bits(2, Rp->red_warp);
-  for (int k : bits_at_level(L, 3, 3)) {
-    if (L.cols[k] == 0) Rp->dup_bits.push_back(k);
-    else Rp->grid_bit.push_back(k);
+  // kernel layout: faithful (L itself) or line-coalesced σ with non-axis bits
+  // preferred in the free lanes (axis bits stay in registers: cheap tree levels)
+  int sigma = opts ? opts->sigma : 0;
+  Rp->v = std::min(2, R);
+  if (sigma == SIGMA_FAITHFUL) {
+    Rp->sigma = SIGMA_FAITHFUL;
+    for (int k : bits_at_level(L, 0, 2)) Rp->hw_bit.push_back(k);
+  } else {
+    Rp->sigma = SIGMA_COALESCED;
+    Rp->hw_bit = sigma_line(L, Rp->v, [&](int k) { return L.cols[k] != 0 && !(L.cols[k] & amask); });
   }
-  // output flat offset per hardware bit: logical x -> row-major output with the axis
-  // replaced by its block part (axis / K)
-  Rp->out_col.assign(L.d_in(), 0);
-  for (int k = 0; k < L.d_in(); ++k) {
-    u64 c = L.cols[k];
-    if (!c || (std::find(Rp->red_reg.begin(), Rp->red_reg.end(), k) != Rp->red_reg.end()) ||
-        (std::find(Rp->red_lane.begin(), Rp->red_lane.end(), k) != Rp->red_lane.end()) ||
-        (std::find(Rp->red_warp.begin(), Rp->red_warp.end(), k) != Rp->red_warp.end()))
-      continue;
+  const int n = int(Rp->hw_bit.size());
+  // classify kernel bits; the fixed order is kernel reg, lane, warp bits
+  // ascending — equal to L's own order for the faithful decomposition
+  for (int b = 0; b < n; ++b) {
+    u64 c = L.cols[Rp->hw_bit[b]];
+    if (c == 0) { Rp->dup_bits.push_back(b); continue; }
+    if (!(c & amask)) continue;
+    if (b < R) Rp->red_reg.push_back(b);
+    else if (b < R + 5) Rp->red_lane.push_back(b - R);
+    else Rp->red_warp.push_back(b - R - 5);
+  }
+  auto out_of = [&](u64 c) {
     u64 lower = c & ((u64(1) << sh) - 1);
     u64 a = (c & amask) >> sh;
     u64 upper = c >> (sh + ab);
-    int na_bits = ab - K;
-    Rp->out_col[k] = (((upper << na_bits) | (a >> K)) << sh) | lower;
+    return (((upper << (ab - K)) | (a >> K)) << sh) | lower;
+  };
+  Rp->out_col.assign(n, 0);
+  for (int b = 0; b < n; ++b) {
+    u64 c = L.cols[Rp->hw_bit[b]];
+    bool red = (b < R && std::count(Rp->red_reg.begin(), Rp->red_reg.end(), b)) ||
+               (b >= R && b < R + 5 && std::count(Rp->red_lane.begin(), Rp->red_lane.end(), b - R)) ||
+               (b >= R + 5 && std::count(Rp->red_warp.begin(), Rp->red_warp.end(), b - R - 5));
+    if (c && !red) Rp->out_col[b] = out_of(c);
+  }
+  for (int k : bits_at_level(L, 3, 3)) {
+    if (L.cols[k] == 0) continue;   // duplicate CTAs are not launched
+    Rp->grid_bit.push_back(k);
+    Rp->grid_out.push_back(out_of(L.cols[k]));
   }
   Rp->out_elems = u64(1) << (L.d_out() - K);
-  Rp->smem_bytes = Rp->red_warp.empty() ? 0 : int((u64(4) << (L.in_bits("reg") + 5 + Rp->Wb)));
+  int live = R - int(Rp->red_reg.size());
+  for (int b : Rp->dup_bits) if (b < R) --live;
+  Rp->smem_bytes = Rp->red_warp.empty() ? 0 : int((u64(4) << (std::max(0, live) + 5 + Rp->Wb)));
   return Rp;
 }
 

@@ -188,9 +188,36 @@ def test_gather_bitexact(family, sigma):
     assert np.array_equal(from_device(d_dst, 4), ref)
 
 
+def _line_sigma_layout(OL, axis):
+    """The reduce kernel's layout L' = L∘σ, re-derived from the rule written in
+    DESIGN.md §5.7 (line-coalesced σ: 16-byte vector bits, 3 forced lanes, 2 free lanes
+    preferring non-axis columns, the rest registers; warps and blocks unchanged).
+    Returns (L', perm) with src'[h'] = src[perm[h']]."""
+    R = OL.dim_bits("reg").__len__()
+    sh = sum(b for _, b in OL.out_dims[axis + 1:])
+    amask = ((1 << OL.out_dims[axis][1]) - 1) << sh
+    nw = sorted(OL.dim_bits("reg") + OL.dim_bits("lane"))
+    v = min(2, R)
+    rest = nw[v + 3:]
+    pref = lambda k: OL.cols[k] != 0 and not (OL.cols[k] & amask)
+    rest_sorted = [k for k in rest if pref(k)] + [k for k in rest if not pref(k)]
+    lanes = nw[v:v + 3] + rest_sorted[:2]
+    regs = nw[:v] + sorted(rest_sorted[2:])
+    hw = regs + lanes + OL.dim_bits("warp") + OL.dim_bits("block")
+    Lp = O.layout_from_cols(OL.in_dims, OL.out_dims, [OL.cols[k] for k in hw])
+    hs = np.arange(1 << OL.d_in, dtype=np.int64)
+    perm = np.zeros_like(hs)
+    for b, k in enumerate(hw):
+        perm |= ((hs >> b) & 1) << k
+    return Lp, perm
+
+
 @pytest.mark.parametrize("family", ["mma", "blocked"])
-def test_reduce_tolerance_and_fixed_order(family):
-    """O11: ≤ 1e-6 relative vs fp64 and bit-exact vs the fixed-order fp32 replica."""
+@pytest.mark.parametrize("sigma", ["coalesced", "faithful"])
+def test_reduce_tolerance_and_fixed_order(family, sigma):
+    """O11: ≤ 1e-6 relative vs fp64, and bit-exact vs the fixed-order fp32 replica
+    taken over the kernel's layout (L itself for faithful σ; L∘σ for the coalesced
+    one, the order being reg, lane, warp bits ascending in both cases)."""
     import torch
     rng = np.random.default_rng(1005)
     spec = W.c4("reduce", family, n_i=9, n_j=9)
@@ -198,11 +225,67 @@ def test_reduce_tolerance_and_fixed_order(family):
     n = 1 << OL.d_in
     T = rng.random(n, dtype=np.float32)
     src = O.pack(OL, T)
-    plan = ll.ll_plan_reduce(L, 1)
+    plan = ll.ll_plan_reduce(L, 1, sigma=sigma)
     out = torch.empty(plan.out_elems(), dtype=torch.float32, device="cuda")
     ll.ll_reduce(torch.from_numpy(src).cuda(), out, plan)
     got = out.cpu().numpy()
     ref = O.reduce_ref_fp64(OL, 1, src)
     assert np.all(np.abs(got - ref) <= 1e-6 * np.abs(ref))
+    if sigma == "faithful":
+        rep = O.reduce_fixed_order_fp32(OL, 1, src)
+    else:
+        Lp, perm = _line_sigma_layout(OL, 1)
+        rep = O.reduce_fixed_order_fp32(Lp, 1, src[perm])
+    assert np.array_equal(got.view(np.uint32), rep.view(np.uint32))
+
+
+def test_reduce_broadcast_dedup_gpu():
+    """a layout with zero columns (duplicated lanes and registers) reduces each
+    logical element once; one write per output."""
+    import torch
+    OL = O.blocked([8, 16], [1, 2], [4, 8], [4, 1], [1, 0])
+    spec = {"out": [("d0", 3), ("d1", 4)], "in": []}
+    L = ll.Layout(OL.in_dims, OL.out_dims, OL.bases)
+    rng = np.random.default_rng(3)
+    T = rng.random(128, dtype=np.float32)
+    src = O.pack(OL, T)
+    plan = ll.ll_plan_reduce(L, 1, sigma="faithful")
+    out = torch.full((plan.out_elems(),), -1.0, dtype=torch.float32, device="cuda")
+    ll.ll_reduce(torch.from_numpy(src).cuda(), out, plan)
+    got = out.cpu().numpy()
     rep = O.reduce_fixed_order_fp32(OL, 1, src)
     assert np.array_equal(got.view(np.uint32), rep.view(np.uint32))
+
+
+def test_exhaustive_fig1_sample_gpu():
+    """E1 (sampled on GPU): random bijective relabelings B of Fig. 1's 2^8 space
+    against Fig. 1 A, and a 7-bit space where A and B each carry a broadcast column;
+    every plan (tile kernel or generic kernel) bit-exact against the oracle, and the
+    planner's class equal to the oracle's existential class (O7)."""
+    import torch
+    rng = np.random.default_rng(4040)
+    A, OA = both(W.C1_A)
+    hw = [("reg", 2), ("lane", 5), ("warp", 1)]
+    T = gen.random_bits(rng, 256, 4)
+    src = O.pack(OA, T)
+    d_src = to_device(src)
+    for case in range(60):
+        sb = gen.random_distributed(rng, W.C1_OUT, hw)
+        B, OB = both(sb)
+        plan = ll.ll_plan_convert(A, B, 4)
+        assert plan.cls == O.classify(OA, OB)
+        d_dst = empty_device(256, 4)
+        ll.ll_convert(d_src, d_dst, plan)
+        assert np.array_equal(from_device(d_dst, 4), O.pack(OB, T)), (case, plan.describe()["exec"])
+    out7 = [("i", 3), ("j", 4)]
+    T7 = gen.random_bits(rng, 128, 4)
+    for case in range(30):
+        sa = gen.random_distributed(rng, out7, hw, zero_ok=["reg"])
+        sb = gen.random_distributed(rng, out7, hw, zero_ok=["lane"])
+        A7, OA7 = both(sa)
+        B7, OB7 = both(sb)
+        plan = ll.ll_plan_convert(A7, B7, 4)
+        assert plan.cls == O.classify(OA7, OB7)
+        d_dst = empty_device(256, 4)
+        ll.ll_convert(to_device(O.pack(OA7, T7)), d_dst, plan)
+        assert np.array_equal(from_device(d_dst, 4), O.pack(OB7, T7))

@@ -255,3 +255,67 @@ def test_device_entry_fails_loudly_without_gpu():
     p = ll.ll_plan_convert(A, B, 4)
     with pytest.raises(ll.LLError, match="CUDA"):
         ll.ll_convert(1 << 20, 2 << 20, p, stream=0)
+
+
+# ---------------------------------------------------------------- layout families
+@pytest.mark.parametrize("args", [
+    ([16, 16], [2, 2], [4, 8], [2, 1], [1, 0]),
+    ([128, 128], [8, 8], [2, 16], [4, 1], [1, 0]),
+    ([256, 128], [1, 8], [2, 16], [4, 1], [1, 0]),
+    ([256, 128], [8, 1], [32, 1], [1, 4], [0, 1]),
+    ([8, 8], [1, 1], [4, 8], [2, 1], [1, 0]),          # broadcast
+    ([4, 8, 16], [1, 2, 2], [2, 4, 4], [1, 2, 2], [2, 1, 0]),
+])
+def test_blocked_family_matches_oracle(args):
+    L = ll.ll_layout_blocked(*args)
+    OL = O.blocked(*args)
+    assert L.cols() == OL.cols and L.in_dims == OL.in_dims
+
+
+def test_blocked_is_fig1_A():
+    """GV3 through the product's constructor: blocked([2,2],[4,8],[2,1],[1,0]) on
+    16x16 has the columns of the P:140 matrix."""
+    L = ll.ll_layout_blocked([16, 16], [2, 2], [4, 8], [2, 1], [1, 0])
+    assert L.cols() == O.Layout(*W.spec_to_bases(W.C1_A)).cols
+
+
+@pytest.mark.parametrize("M,N,wm", [(128, 128, 4), (64, 32, 4), (16, 8, 1), (128, 32, 4)])
+def test_mma_acc_family_matches_oracle(M, N, wm):
+    assert ll.ll_layout_mma_acc(M, N, wm).cols() == O.mma_acc([M, N], wm).cols
+
+
+def test_mma_swizzle_family_matches_def411():
+    for vec, pp, mp in [(8, 1, 8), (4, 2, 4), (8, 2, 4), (2, 1, 8)]:
+        L = ll.ll_layout_mma_swizzle(6, 6, vec, pp, mp)
+        assert L.props()["memory"]
+        # the map is an involution: offset(i, j) = (i << 6) + Def 4.11 formula
+        cols = L.cols()
+        for i in range(64):
+            for j in range(64):
+                x = (i << 6) | j
+                off = 0
+                for k in range(12):
+                    if (x >> k) & 1:
+                        off ^= cols[k]
+                assert off == (i << 6) + O.mma_swizzle_offset(i, j, vec, pp, mp)
+
+
+def test_slice_family_matches_oracle():
+    L = ll.ll_layout_blocked([16, 16], [2, 2], [4, 8], [2, 1], [1, 0])
+    S = ll.ll_layout_slice(L, 1)
+    OS = O.sliced(O.blocked([16, 16], [2, 2], [4, 8], [2, 1], [1, 0]), 1)
+    assert S.cols() == OS.cols
+    assert S.props()["surjective"] and not S.props()["injective"]
+
+
+def test_contiguity_table3():
+    """P:300-304 contiguity reproduces Table 3's Triton-Linear bitwidths
+    on the blocked layouts of the fixture (layouts are a reading, G23)."""
+    import json
+    rows = json.load(open(os.path.join(ROOT, "tests", "golden", "table3_contiguity.json")))["rows"]
+    for r in rows:
+        L = ll.ll_layout_blocked(r["shape"], r["size_per_thread"], [4, 8], [4, 1], [1, 0])
+        assert L.contiguity(r["dtype_bytes"]) * r["dtype_bytes"] * 8 == r["bits"], r
+    # legacy Triton's fastest-dim-only rule would give 16 bits for [512,2] x f8 (P:464)
+    L = ll.ll_layout_blocked([512, 2], [8, 2], [4, 8], [4, 1], [1, 0])
+    assert L.cols()[0] == 1 and L.cols()[1] == 2   # j0 then i0: contiguous across dims

@@ -19,7 +19,10 @@ a = ap.parse_args()
 
 conv = {"c2": (W.c2(16), 2, {}), "c2smem": (W.c2(16), 2, {"force_class": "SMEM"}),
         "c3": (W.c3(14), 2, {}), "c3b": (W.c3b(14), 2, {}), "c1b": (W.c1_batched(20), 4, {}),
-        "c1bsmem": (W.c1_batched(20), 4, {"force_class": "SMEM"})}
+        "c1bsmem": (W.c1_batched(20), 4, {"force_class": "SMEM"}),
+        # small variants for compute-sanitizer
+        "c1bsmem_small": (W.c1_batched(6), 4, {"force_class": "SMEM"}),
+        "c3_small": (W.c3(3), 2, {}), "c2_small": (W.c2(3), 2, {})}
 if a.case in conv:
     (sa, sb), w, opts = conv[a.case]
     A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)

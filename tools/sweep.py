@@ -51,7 +51,11 @@ def conv_case(name, sa, sb, w, **opts):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--quick", action="store_true")
+    ap.add_argument("--only", default="all")
     args = ap.parse_args()
+    only = args.only.split(",")
+    if "all" not in only and "conv" not in only:
+        return gather_reduce()
     # raw copy roofline reference
     n = 1 << 30
     a = torch.empty(n, dtype=torch.int16, device="cuda")
@@ -75,9 +79,13 @@ def main():
     sa, sb = W.c1_batched(20)
     for opts in [dict(), dict(force_class="SMEM"), dict(tile_bytes=65536), dict(thread_bytes=16)]:
         conv_case("c1batch", sa, sb, 4, **opts)
+    gather_reduce()
+
+
+def gather_reduce():
     # gather / reduce (4096 x 4096 fp32)
     for fam in ["mma", "blocked"]:
-        for sig in ["coalesced", "faithful"]:
+        for sig in ["coalesced", "faithful", 2]:
             L = ll.Layout.from_spec(W.c4("gather", fam))
             p = ll.ll_plan_gather(L, 1, 4, sigma=sig)
             p.prepare()
