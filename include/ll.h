@@ -169,6 +169,21 @@ ll_status ll_layout_mma_acc(int M, int N, int warps_m, int warps_n, ll_layout** 
  * c_i = (vec·((2^i/per_phase) mod max_phase)) mod 2^n. */
 ll_status ll_layout_mma_swizzle(int log2_rows, int log2_cols, int vec, int per_phase,
                                 int max_phase, ll_layout** L);
+/* ll_layout_mma_operand (Prop 4.7 / 9.2): input
+ * operand of mma (m16n8kK) / wgmma for `bitwidth`-bit elements (8, 16, 32).
+ *   is_rhs = 0: lhs, rows x cols = M x K:
+ *     id^{Reg,1}_{log2(32/b)} x id^{Thr,1}_2 x id^{Thr,0}_3 x id^{Reg,0}_1 x id^{Reg,1}_1
+ *   is_rhs = 1: rhs, rows x cols = K x N:
+ *     id^{Reg,0}_{log2(32/b)} x id^{Thr,0}_2 x id^{Thr,1}_3 x id^{Reg,1}_1
+ *   Repetitions over K, then over the other dim, become register bits.  warps_m /
+ *   warps_n split M / N; the operand's copies over the other dim's warps broadcast
+ *   (zero columns).  wgmma's lhs is warps_m = 4 (id^{Wrp,0}_2). */
+ll_status ll_layout_mma_operand(int is_rhs, int rows, int cols, int bitwidth, int warps_m,
+                                int warps_n, ll_layout** L);
+/* ll_layout_tmem_32x32b: the registers of a warpgroup after tcgen05.ld.32x32b from a
+ * 128 x N fp32 TMEM accumulator (Blackwell tensor memory): thread t of warp w
+ * holds row 32w + t, register r holds column r. */
+ll_status ll_layout_tmem_32x32b(int M, int N, ll_layout** L);
 /* ll_layout_contiguity (§5.1 "Contiguous elements"): the number of
  * elements each thread can move with one vector instruction — the largest u with
  * L^{-1}_Reg(i) = i for all i < u (leading register bits mapping in order to the

@@ -82,6 +82,8 @@ _sig = {
     "ll_layout_mma_swizzle": [C.c_int] * 5 + [_PP],
     "ll_layout_slice": [_P, C.c_int, _PP],
     "ll_layout_contiguity": [_P, C.c_int, C.c_int, C.POINTER(C.c_int)],
+    "ll_layout_mma_operand": [C.c_int] * 6 + [_PP],
+    "ll_layout_tmem_32x32b": [C.c_int, C.c_int, _PP],
 }
 for _name, _args in _sig.items():
     _f = getattr(_lib, _name)
@@ -278,6 +280,18 @@ def ll_layout_mma_acc(M, N, warps_m, warps_n=1) -> Layout:
 def ll_layout_mma_swizzle(log2_rows, log2_cols, vec, per_phase, max_phase) -> Layout:
     h = C.c_void_p()
     _check(_lib.ll_layout_mma_swizzle(log2_rows, log2_cols, vec, per_phase, max_phase, C.byref(h)))
+    return Layout(None, None, _handle=h)
+
+
+def ll_layout_mma_operand(is_rhs, rows, cols, bitwidth, warps_m=1, warps_n=1) -> Layout:
+    h = C.c_void_p()
+    _check(_lib.ll_layout_mma_operand(int(is_rhs), rows, cols, bitwidth, warps_m, warps_n, C.byref(h)))
+    return Layout(None, None, _handle=h)
+
+
+def ll_layout_tmem_32x32b(M, N) -> Layout:
+    h = C.c_void_p()
+    _check(_lib.ll_layout_tmem_32x32b(M, N, C.byref(h)))
     return Layout(None, None, _handle=h)
 
 

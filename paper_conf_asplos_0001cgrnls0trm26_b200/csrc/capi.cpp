@@ -338,6 +338,21 @@ ll_status ll_layout_contiguity(const ll_layout* L, int elem_bytes, int max_vec_b
   LL_CATCH
 }
 
+ll_status ll_layout_mma_operand(int is_rhs, int rows, int cols, int bitwidth, int warps_m, int warps_n,
+                                ll_layout** out) {
+  LL_TRY
+  if (!out) fail(LL_ERR_INVALID_ARG, "null argument");
+  *out = new ll_layout{make_mma_operand(is_rhs, rows, cols, bitwidth, warps_m, warps_n)};
+  LL_CATCH
+}
+
+ll_status ll_layout_tmem_32x32b(int M, int N, ll_layout** out) {
+  LL_TRY
+  if (!out) fail(LL_ERR_INVALID_ARG, "null argument");
+  *out = new ll_layout{make_tmem_32x32b(M, N)};
+  LL_CATCH
+}
+
 ll_status ll_layout_slice(const ll_layout* L, int dim, ll_layout** out) {
   LL_TRY
   if (!L || !out) fail(LL_ERR_INVALID_ARG, "null argument");

@@ -28,6 +28,14 @@ std::string icon(const char* name, long long v) {
 
 int ilog2i(u64 v) { return v ? 63 - __builtin_clzll(v) : -1; }
 
+// Store cache hint for the streaming outputs: 1 = .cs (evict-first; measured +0.5%
+// on config 2 and +3% on config 3, profiles/r01_sweep_hints.jsonl), 0 = default
+// write-back (env LL_ST_HINT=wb).
+int st_hint() {
+  const char* e = std::getenv("LL_ST_HINT");
+  return (e && std::string(e) == "wb") ? 0 : 1;
+}
+
 // grid map: CTA index bit g -> offsets; contiguous when both sides are a run of bits
 void emit_grid(std::ostringstream& o, const std::vector<int>& gs, const std::vector<int>& gd, int shift_scale) {
   bool contig = !gs.empty();
@@ -57,6 +65,7 @@ std::string codegen_tile(const ConvPlan& Pl) {
     << icon("NW", std::max<long long>(1, ((1ll << T.R) * T.w) / 4))
     << icon("VLD", T.vld) << icon("VST", T.vst) << icon("XCHG", T.xchg) << icon("THREADS", T.threads());
   o << "  static constexpr bool ISOLATE_SMEM = " << (std::getenv("LL_ISOLATE_SMEM") ? "true" : "false") << ";\n";
+  o << icon("ST_HINT", st_hint());
   // per-thread-contiguous loads (faithful σ) re-use sectors across instructions
   o << "  static constexpr bool LD_L1 = " << (T.sigma == SIGMA_FAITHFUL ? "true" : "false") << ";\n";
   std::vector<u64> ldc, stc;
@@ -93,6 +102,7 @@ std::string codegen_gather(const GatherPlan& G) {
   o << icon("W", G.w) << icon("R", G.R) << icon("WB", G.Wb)
     << icon("NW", std::max<long long>(1, ((1ll << G.R) * G.w) / 4)) << icon("VLD", G.v);
   o << "  static constexpr bool LD_L1 = " << (G.sigma == SIGMA_FAITHFUL ? "true" : "false") << ";\n";
+  o << icon("ST_HINT", st_hint());
   std::vector<u64> ldc;
   for (int b = 0; b < n; ++b) ldc.push_back(u64(1) << G.hw_bit[b]);   // element offsets
   o << arr("u64", "LD_COL", ldc);

@@ -343,3 +343,62 @@ Layout make_slice(const Layout& L, int dim) {
 }
 
 }  // namespace ll
+
+// ---------------------------------------------------------------------------
+// MMA input operands (Prop 9.2) and the tcgen05 TMEM
+// 32x32b load fragment (Blackwell tensor memory) as distributed layouts.
+// ---------------------------------------------------------------------------
+namespace ll {
+
+Layout make_mma_operand(int is_rhs, int rows, int cols, int bitwidth, int warps_m, int warps_n) {
+  // lhs (M x K, d0 = m, d1 = k):
+  //   id^{Reg,1}_{log2(32/b)} x id^{Thr,1}_2 x id^{Thr,0}_3 x id^{Reg,0}_1 x id^{Reg,1}_1
+  // rhs (K x N, d0 = k, d1 = n):
+  //   id^{Reg,0}_{log2(32/b)} x id^{Thr,0}_2 x id^{Thr,1}_3 x id^{Reg,1}_1
+  // then repetitions over the k dim, then the other dim, as register bits; warps along
+  // M then N: the operand's own dim is split, warps on the other dim broadcast (zero
+  // columns).
+  if (bitwidth != 8 && bitwidth != 16 && bitwidth != 32) fail(LL_ERR_INVALID_ARG, "operand bitwidth must be 8, 16 or 32");
+  const int rb = lg2(rows), cb = lg2(cols), kb = lg2(32 / bitwidth);
+  const int wm = lg2(warps_m), wn = lg2(warps_n);
+  // dims: lhs (d0 = m, d1 = k); rhs (d0 = k, d1 = n)
+  auto D0 = [&](int k) -> u64 { return k < rb ? (u64(1) << (cb + k)) : 0; };
+  auto D1 = [&](int k) -> u64 { return k < cb ? (u64(1) << k) : 0; };
+  std::vector<u64> reg, lane, warp;
+  int k_used = 0, o_used = 0;   // bits used on the k dim / the other dim
+  auto K = [&](int k) { return is_rhs ? D0(k) : D1(k); };
+  auto Oth = [&](int k) { return is_rhs ? D1(k) : D0(k); };
+  for (int t = 0; t < kb; ++t) reg.push_back(K(k_used++));
+  for (int t = 0; t < 2; ++t) lane.push_back(K(k_used++));
+  for (int t = 0; t < 3; ++t) lane.push_back(Oth(o_used++));
+  if (!is_rhs) { reg.push_back(Oth(o_used++)); }   // rows +8 (lhs only: 16-row tile)
+  reg.push_back(K(k_used++));                      // k + 8·(32/b)/... second k half
+  // warps: lhs splits M (i) over warps_m, broadcasts over warps_n; rhs the converse
+  for (int t = 0; t < wm; ++t) warp.push_back(is_rhs ? 0 : Oth(o_used++));
+  for (int t = 0; t < wn; ++t) warp.push_back(is_rhs ? Oth(o_used++) : 0);
+  const int kdim_bits = is_rhs ? rb : cb, odim_bits = is_rhs ? cb : rb;
+  while (k_used < kdim_bits) reg.push_back(K(k_used++));
+  while (o_used < odim_bits) reg.push_back(Oth(o_used++));
+  Layout L;
+  L.out = {{"d0", rb}, {"d1", cb}};
+  L.in = {{"reg", int(reg.size())}, {"lane", 5}, {"warp", int(warp.size())}};
+  L.cols = reg;
+  L.cols.insert(L.cols.end(), lane.begin(), lane.end());
+  L.cols.insert(L.cols.end(), warp.begin(), warp.end());
+  return L;
+}
+
+Layout make_tmem_32x32b(int M, int N) {
+  // tcgen05.ld.32x32b: warp w of a warpgroup reads TMEM lanes [32w, 32w + 32); thread
+  // t gets lane (row) 32w + t; consecutive registers are consecutive columns.
+  const int mb = lg2(M), nb = lg2(N);
+  if (mb != 7) fail(LL_ERR_INVALID_ARG, "tmem 32x32b fragment: M must be 128 (4 warps x 32 lanes)");
+  Layout L;
+  L.out = {{"d0", mb}, {"d1", nb}};
+  L.in = {{"reg", nb}, {"lane", 5}, {"warp", 2}};
+  for (int k = 0; k < nb; ++k) L.cols.push_back(u64(1) << k);
+  for (int k = 0; k < 7; ++k) L.cols.push_back(u64(1) << (nb + k));
+  return L;
+}
+
+}  // namespace ll

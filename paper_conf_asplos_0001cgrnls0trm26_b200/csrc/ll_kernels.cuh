@@ -80,14 +80,27 @@ __device__ __forceinline__ u32 ldg_b32(const u8* p) {
     asm volatile("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(a) : "l"(p));
   return a;
 }
+// Global stores.  HINT 0: default (write-back); 1: .cs (streaming, evict-first).
+template <int HINT>
 __device__ __forceinline__ void stg_v4(u8* p, u32 a, u32 b, u32 c, u32 d) {
-  asm volatile("st.global.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(a), "r"(b), "r"(c), "r"(d) : "memory");
+  if constexpr (HINT == 1)
+    asm volatile("st.global.cs.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(a), "r"(b), "r"(c), "r"(d) : "memory");
+  else
+    asm volatile("st.global.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(a), "r"(b), "r"(c), "r"(d) : "memory");
 }
+template <int HINT>
 __device__ __forceinline__ void stg_v2(u8* p, u32 a, u32 b) {
-  asm volatile("st.global.v2.u32 [%0], {%1,%2};" ::"l"(p), "r"(a), "r"(b) : "memory");
+  if constexpr (HINT == 1)
+    asm volatile("st.global.cs.v2.u32 [%0], {%1,%2};" ::"l"(p), "r"(a), "r"(b) : "memory");
+  else
+    asm volatile("st.global.v2.u32 [%0], {%1,%2};" ::"l"(p), "r"(a), "r"(b) : "memory");
 }
+template <int HINT>
 __device__ __forceinline__ void stg_b32(u8* p, u32 a) {
-  asm volatile("st.global.u32 [%0], %1;" ::"l"(p), "r"(a) : "memory");
+  if constexpr (HINT == 1)
+    asm volatile("st.global.cs.u32 [%0], %1;" ::"l"(p), "r"(a) : "memory");
+  else
+    asm volatile("st.global.u32 [%0], %1;" ::"l"(p), "r"(a) : "memory");
 }
 
 // Load vector K of the thread (2^VL elements of W bytes starting at slot K<<VL).
@@ -107,16 +120,16 @@ __device__ __forceinline__ void load_vec(u32 (&r)[NW], const u8* p) {
     set_e<1, E0>(r, u32(*p));
   }
 }
-template <int W, int VL, int K, int NW>
+template <int W, int VL, int K, int NW, int HINT = 0>
 __device__ __forceinline__ void store_vec(const u32 (&r)[NW], u8* p) {
   constexpr int VB = W << VL;
   constexpr int E0 = K << VL;
   if constexpr (VB == 16) {
-    stg_v4(p, r[E0 * W / 4 + 0], r[E0 * W / 4 + 1], r[E0 * W / 4 + 2], r[E0 * W / 4 + 3]);
+    stg_v4<HINT>(p, r[E0 * W / 4 + 0], r[E0 * W / 4 + 1], r[E0 * W / 4 + 2], r[E0 * W / 4 + 3]);
   } else if constexpr (VB == 8) {
-    stg_v2(p, r[E0 * W / 4 + 0], r[E0 * W / 4 + 1]);
+    stg_v2<HINT>(p, r[E0 * W / 4 + 0], r[E0 * W / 4 + 1]);
   } else if constexpr (VB == 4) {
-    stg_b32(p, r[E0 * W / 4]);
+    stg_b32<HINT>(p, r[E0 * W / 4]);
   } else if constexpr (VB == 2) {
     *reinterpret_cast<u16*>(p) = u16(get_e<2, E0 * W / 2>(r));
   } else {
@@ -398,7 +411,7 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, u8* __r
     // a10: HBM store of the dst tile
     static_for<(1 << (P::R - P::VST))>([&](auto k) {
       constexpr int K = decltype(k)::value;
-      store_vec<P::W, P::VST, K>(o, d + StOff<P, K>::value());
+      store_vec<P::W, P::VST, K, P::NW, P::ST_HINT>(o, d + StOff<P, K>::value());
     });
     if constexpr (P::XCHG == 3) __syncthreads();   // smem reuse by the next tile
   }
@@ -456,7 +469,7 @@ __device__ __forceinline__ void ll_gather_body(const u8* __restrict__ src, const
     });
     static_for<(1 << (P::R - P::VLD))>([&](auto k) {
       constexpr int K = decltype(k)::value;
-      store_vec<P::W, P::VLD, K>(o, dst + (eoff ^ LdOff<P, K>::value()) * P::W);
+      store_vec<P::W, P::VLD, K, P::NW, P::ST_HINT>(o, dst + (eoff ^ LdOff<P, K>::value()) * P::W);
     });
   }
 }

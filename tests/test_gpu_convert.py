@@ -289,3 +289,56 @@ def test_exhaustive_fig1_sample_gpu():
         d_dst = empty_device(256, 4)
         ll.ll_convert(to_device(O.pack(OA7, T7)), d_dst, plan)
         assert np.array_equal(from_device(d_dst, 4), O.pack(OB7, T7))
+
+
+@pytest.mark.parametrize("want", ["REGPERM", "SHUFFLE"])
+def test_class_kernels_faithful_gpu(want):
+    """Register permutation and warp shuffles executed on the
+    layouts' own hardware (faithful σ), so the executed exchange is the paper's class;
+    random pairs built by permuting register bits (REGPERM) or register+lane bits
+    (SHUFFLE) of a random distributed layout; 4-byte and 2-byte elements."""
+    rng = np.random.default_rng(606 if want == "REGPERM" else 607)
+    out = [("b", 4), ("i", 5), ("j", 5)]
+    hw = [("reg", 3), ("lane", 5), ("warp", 2)]
+    done = 0
+    for case in range(60):
+        sa = gen.random_distributed(rng, out[1:], hw)
+        ins = dict(sa["in"])
+        if want == "REGPERM":
+            regs = list(ins["reg"])
+            rng.shuffle(regs)
+            sb_in = [("reg", regs), ("lane", ins["lane"]), ("warp", ins["warp"])]
+        else:
+            pool = list(ins["reg"]) + list(ins["lane"])
+            rng.shuffle(pool)
+            sb_in = [("reg", pool[:3]), ("lane", pool[3:]), ("warp", ins["warp"])]
+        blk = [("block", ["b0", "b1", "b2", "b3"])]
+        sa = {"out": out, "in": sa["in"] + blk}
+        sb = {"out": out, "in": sb_in + blk}
+        OA, OB = O.Layout(*W.spec_to_bases(sa)), O.Layout(*W.spec_to_bases(sb))
+        if O.classify(OA, OB) != want:
+            continue
+        for w in (4, 2):
+            got, ref, plan = run_convert(sa, sb, w, case, sigma="faithful")
+            d = plan.describe()
+            assert d["class"] == want
+            if w == 4:
+                assert d["tile"]["xchg"] == {"REGPERM": "regperm", "SHUFFLE": "shuffle"}[want]
+            assert np.array_equal(got, ref), (case, w)
+        done += 1
+        if done == 8:
+            break
+    assert done >= 5
+
+
+@pytest.mark.parametrize("which", ["n1", "n2"])
+def test_next_rows_n1_n2_bitexact(which):
+    """§8(f) N1 (HBM pre-shuffle of a bf16 weight into mma rhs fragment order)
+    and N2 (tcgen05 TMEM 32x32b fragment -> coalesced blocked epilogue layout)."""
+    if which == "n1":
+        (sa, sb), w = W.n1_preshuffle(9, 8), 2
+    else:
+        (sa, sb), w = W.n2_tmem_epilogue(3), 4
+    got, ref, plan = run_convert(sa, sb, w, 77)
+    assert plan.describe()["exec"] == "tile"
+    assert np.array_equal(got, ref)

@@ -319,3 +319,72 @@ def test_contiguity_table3():
     # legacy Triton's fastest-dim-only rule would give 16 bits for [512,2] x f8
     L = ll.ll_layout_blocked([512, 2], [8, 2], [4, 8], [4, 1], [1, 0])
     assert L.cols()[0] == 1 and L.cols()[1] == 2   # j0 then i0: contiguous across dims
+
+
+# ---------------------------------------------------------------- N2: operand / TMEM families
+def _enum(L):
+    """(reg, lane, warp) -> logical coords for every hardware index of L."""
+    d = {}
+    ins = L.in_dims
+    nr, nl, nw = [dict(ins).get(k, 0) for k in ("reg", "lane", "warp")]
+    for w in range(1 << nw):
+        for l in range(1 << nl):
+            for r in range(1 << nr):
+                d[(r, l, w)] = L.apply([r, l, w][:len(ins)])
+    return d
+
+
+@pytest.mark.parametrize("bits", [16, 8, 32])
+def test_mma_lhs_matches_ptx_fragment(bits):
+    """Prop 9.2 lhs tile vs the PTX m16n8k{8,16,32} A fragment [HW]: element i of
+    lane (g = lane/4, t = lane%4) at row g + 8·((i/e)%2), col e·t + i%e + 4e·(i/(2e)),
+    e = 32/bits elements per 32-bit register."""
+    e = 32 // bits
+    K = 8 * e
+    L = ll.ll_layout_mma_operand(0, 16, K, bits)
+    for (r, lane, w), (row, col) in _enum(L).items():
+        g, t = lane // 4, lane % 4
+        assert row == g + 8 * ((r // e) % 2), (r, lane)
+        assert col == e * t + r % e + 4 * e * (r // (2 * e)), (r, lane)
+
+
+@pytest.mark.parametrize("bits", [16, 8, 32])
+def test_mma_rhs_matches_ptx_fragment(bits):
+    """Prop 9.2 rhs tile vs the PTX B fragment [HW]: element i at
+    k = e·t + i%e + 4e·(i/e), n = g."""
+    e = 32 // bits
+    K = 8 * e
+    L = ll.ll_layout_mma_operand(1, K, 8, bits)
+    for (r, lane, w), (k, n) in _enum(L).items():
+        g, t = lane // 4, lane % 4
+        assert k == e * t + r % e + 4 * e * (r // e) and n == g, (r, lane)
+
+
+def test_mma_acc_to_lhs_is_free():
+    """The m16n8 fp32 accumulator of a 16x16 tile has the columns of the m16n8k16 bf16
+    lhs operand (reg j0, i3, j3; lanes j1 j2 i0 i1 i2), so converting the accumulator
+    (after a per-element downcast) into the next mma's A operand is NOOP — the register
+    reuse FlashAttention exploits."""
+    acc = ll.ll_layout_mma_acc(16, 16, 1)
+    lhs = ll.ll_layout_mma_operand(0, 16, 16, 16)
+    assert acc.cols() == lhs.cols()
+    assert ll.ll_plan_convert(acc, lhs, 2).cls == "NOOP"
+
+
+def test_wgmma_lhs_and_broadcast_warps():
+    """wgmma lhs = mma lhs x id^{Wrp,0}_2; with warps along N the lhs is
+    broadcast over those warps (zero columns)."""
+    L = ll.ll_layout_mma_operand(0, 64, 16, 16, warps_m=4)
+    c = L.cols()
+    assert c[-2:] == [16 << 4, 16 << 5]          # warps -> i4, i5
+    L2 = ll.ll_layout_mma_operand(0, 16, 16, 16, warps_m=1, warps_n=2)
+    assert L2.cols()[-1] == 0 and L2.props()["surjective"] and not L2.props()["injective"]
+
+
+def test_tmem_fragment_family():
+    L = ll.ll_layout_tmem_32x32b(128, 64)
+    for (r, lane, w), (row, col) in _enum(L).items():
+        assert row == 32 * w + lane and col == r
+    B = ll.ll_layout_blocked([128, 64], [1, 4], [2, 16], [4, 1], [1, 0])
+    p = ll.ll_plan_convert(L, B, 4)
+    assert p.cls == "SMEM"

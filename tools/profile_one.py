@@ -22,7 +22,9 @@ conv = {"c2": (W.c2(16), 2, {}), "c2smem": (W.c2(16), 2, {"force_class": "SMEM"}
         "c1bsmem": (W.c1_batched(20), 4, {"force_class": "SMEM"}),
         # small variants for compute-sanitizer
         "c1bsmem_small": (W.c1_batched(6), 4, {"force_class": "SMEM"}),
-        "c3_small": (W.c3(3), 2, {}), "c2_small": (W.c2(3), 2, {})}
+        "c3_small": (W.c3(3), 2, {}), "c2_small": (W.c2(3), 2, {}),
+        "c5T": (W.c5T(0, n=15), 2, {}), "n1": (W.n1_preshuffle(14, 14), 2, {}),
+        "n2": (W.n2_tmem_epilogue(13), 4, {})}
 if a.case in conv:
     (sa, sb), w, opts = conv[a.case]
     A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)

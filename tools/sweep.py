@@ -54,6 +54,10 @@ def main():
     ap.add_argument("--only", default="all")
     args = ap.parse_args()
     only = args.only.split(",")
+    if "hints" in only:
+        return hints()
+    if "next" in only:
+        return next_rows()
     if "all" not in only and "conv" not in only:
         return gather_reduce()
     # raw copy roofline reference
@@ -82,10 +86,51 @@ def main():
     gather_reduce()
 
 
-def gather_reduce():
+def next_rows():
+    """§8(f) N1 pre-shuffle and N2 TMEM-fragment epilogue at scale; CTA-class transpose."""
+    conv_case("N1 preshuffle W[16384,16384] bf16 -> mma rhs fragments", *W.n1_preshuffle(14, 14), 2)
+    conv_case("N2 tmem 32x32b -> blocked, 8192 tiles 128x128 fp32", *W.n2_tmem_epilogue(13), 4)
+    sa, sb = W.c5T(0, n=15)
+    for opts in [dict(), dict(force_class="SMEM")]:
+        conv_case("c5T P=1 transpose", sa, sb, 2, **opts)
+
+
+def hints():
+    """Store hint, grid persistence, CTA-class transpose and DEVICE loopback."""
+    for hint in ["", "cs"]:
+        os.environ["LL_ST_HINT"] = hint
+        sa, sb = W.c2(16)
+        conv_case(f"c2 st_hint={hint or 'default'}", sa, sb, 2)
+        sa, sb = W.c3(14)
+        conv_case(f"c3 st_hint={hint or 'default'}", sa, sb, 2)
+    os.environ["LL_ST_HINT"] = ""
+    sa, sb = W.c5T(0, n=15)          # 2 GiB bf16 transpose (CTA class)
+    for opts in [dict(), dict(tile_bytes=32768), dict(tile_bytes=8192)]:
+        conv_case("c5T P=1 transpose", sa, sb, 2, **opts)
+    # config 5 DEVICE decomposition on one GPU (loopback: memcpy exchange), P = 8
+    sa, sb = W.c5(3, n=15)
+    A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
+    p = ll.ll_plan_convert(A, B, 2, comm=ll.Comm.loopback(8))
+    p.prepare()
+    n = 1 << 30
+    src = torch.randint(-2 ** 15, 2 ** 15, (n,), dtype=torch.int16, device="cuda")
+    dst = torch.empty_like(src)
+    ws = torch.empty(p.workspace_bytes(), dtype=torch.uint8, device="cuda")
+    ms = time_fn(lambda: ll.ll_convert(src, dst, p, workspace=ws), iters=10, warmup=3)
+    print(json.dumps({"case": "c5 P=8 loopback (pack + memcpy all-to-all)", "ms": round(ms, 4),
+                      "GBps_algorithmic": round(4 * n / ms / 1e6, 1)}), flush=True)
+    del src, dst, ws
+    torch.cuda.empty_cache()
+    for per in ["0", "4", "8", "16"]:
+        os.environ["LL_GRID_PER_SM"] = per
+        gather_reduce(tag=f" grid{per}", sigmas=["coalesced"])
+    os.environ["LL_GRID_PER_SM"] = "0"
+
+
+def gather_reduce(tag="", sigmas=("coalesced", "faithful")):
     # gather / reduce (4096 x 4096 fp32)
     for fam in ["mma", "blocked"]:
-        for sig in ["coalesced", "faithful", 2]:
+        for sig in sigmas:
             L = ll.Layout.from_spec(W.c4("gather", fam))
             p = ll.ll_plan_gather(L, 1, 4, sigma=sig)
             p.prepare()
@@ -100,7 +145,7 @@ def gather_reduce():
                 it[0] += 1
                 ll.ll_gather(s[0], s[1], s[2], p)
             ms = time_fn(g)
-            print(json.dumps({"case": f"gather {fam} {sig}", "desc": p.describe(), "ms": round(ms, 4),
+            print(json.dumps({"case": f"gather {fam} {sig}{tag}", "desc": p.describe(), "ms": round(ms, 4),
                               "GBps": round(12 * n / ms / 1e6, 1)}), flush=True)
         L = ll.Layout.from_spec(W.c4("reduce", fam))
         p = ll.ll_plan_reduce(L, 1)
@@ -114,7 +159,7 @@ def gather_reduce():
             it[0] += 1
             ll.ll_reduce(s[0], s[1], p)
         ms = time_fn(r)
-        print(json.dumps({"case": f"reduce {fam}", "ms": round(ms, 4), "GBps": round((4 * n + 4 * p.out_elems()) / ms / 1e6, 1)}), flush=True)
+        print(json.dumps({"case": f"reduce {fam}{tag}", "ms": round(ms, 4), "GBps": round((4 * n + 4 * p.out_elems()) / ms / 1e6, 1)}), flush=True)
 
 
 if __name__ == "__main__":

@@ -149,3 +149,29 @@ CONFIGS = {
     "c3": {"A": c3()[0], "B": c3()[1], "elem_bytes": 2, "dtype": "f16"},
     "c3b": {"A": c3b()[0], "B": c3b()[1], "elem_bytes": 2, "dtype": "f16"},
 }
+
+
+# ---- §8(f) N1: HBM operand pre-shuffle ----
+def n1_preshuffle(kb: int = 12, nb: int = 12):
+    """A bf16 weight W[K, N] (K = 2^kb, N = 2^nb) stored row-major (A), rewritten in
+    HBM into the packed fragment order of the mma m16n8k16 rhs operand (B; Prop 9.2,
+    P:676) for 64 x 32 tiles (4 k-steps, 4 warps along N): every thread's 8 bf16 of
+    a tile become one contiguous 16-byte vector."""
+    out = [("k", kb), ("n", nb)]
+    A = {"out": out, "in": [("offset", _b("n", 0, nb) + _b("k", 0, kb))]}
+    B = _spec(out, ["k0", "k3", "k4", "k5"], ["k1", "k2", "n0", "n1", "n2"], ["n3", "n4"],
+              _b("k", 6, kb) + _b("n", 5, nb))
+    return A, B
+
+
+# ---- §8(f) N2: tcgen05 TMEM 32x32b accumulator fragment -> coalesced blocked ----
+def n2_tmem_epilogue(nb: int = 13):
+    """A batch of 2^nb 128 x 128 fp32 accumulator tiles as loaded from TMEM by
+    tcgen05.ld.32x32b (thread t of warp w holds row 32w + t; register r column r)
+    converted to the blocked [1,4]/[2,16]/[4,1] row-major layout a coalesced epilogue
+    store wants."""
+    out = [("b", nb), ("i", 7), ("j", 7)]
+    A = _spec(out, _b("j", 0, 7), _b("i", 0, 5), ["i5", "i6"], _b("b", 0, nb))
+    B = _spec(out, ["j0", "j1", "j6", "i3", "i4", "i5", "i6"], ["j2", "j3", "j4", "j5", "i0"], ["i1", "i2"],
+              _b("b", 0, nb))
+    return A, B
