@@ -614,10 +614,12 @@ std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, 
           int v = std::max(0, ilog2(u64(std::max(1, maxvec / w))));
           int tb = default_int(opts, &ll_plan_opts::tile_bytes, 16384);
           int target = std::max(v + 5, ilog2(u64(std::max(1, tb / w))));
-          int c_bits = v + 5;
-          choose_cta_tile(*P, pi, nB, c_bits, target, S, D, gS, gD);
-          if (int(S.size()) > 15) {   // too large for smem: coalesce to 128-byte lines only
-            choose_cta_tile(*P, pi, nB, v + 3, target, S, D, gS, gD);
+          // the longest contiguous runs (2^c elements on both sides) whose tile fits in
+          // 64 KiB of smem: 512-byte runs, else 256, else 128 (one line)
+          const int max_bits = ilog2(u64(65536 / w));
+          for (int c_bits = v + 5; c_bits >= v + 3; --c_bits) {
+            choose_cta_tile(*P, pi, nB, c_bits, target, S, D, gS, gD);
+            if (int(S.size()) <= max_bits) break;
           }
           build_tile(*P, S, D, gS, gD, opts, false);
         }

@@ -91,8 +91,11 @@ def next_rows():
     conv_case("N1 preshuffle W[16384,16384] bf16 -> mma rhs fragments", *W.n1_preshuffle(14, 14), 2)
     conv_case("N2 tmem 32x32b -> blocked, 8192 tiles 128x128 fp32", *W.n2_tmem_epilogue(13), 4)
     sa, sb = W.c5T(0, n=15)
-    for opts in [dict(), dict(force_class="SMEM")]:
+    for opts in [dict(), dict(tile_bytes=65536), dict(thread_bytes=128), dict(thread_bytes=64),
+                 dict(tile_bytes=65536, thread_bytes=128)]:
         conv_case("c5T P=1 transpose", sa, sb, 2, **opts)
+    for opts in [dict(), dict(tile_bytes=65536), dict(thread_bytes=128)]:
+        conv_case("N1 preshuffle", *W.n1_preshuffle(14, 14), 2, **opts)
 
 
 def hints():
