@@ -515,7 +515,12 @@ static void build_tile(ConvPlan& P, const std::vector<int>& S0, const std::vecto
     int pw = A.in_pos("warp");
     for (int k = 0; k < A.in_bits("warp"); ++k) prefer.push_back(A.cols[pw + k]);
     for (int s : foldS) prefer.push_back(A.cols[s]);
-    int thread_bytes = default_int(opts, &ll_plan_opts::thread_bytes, 256);
+    // 256 bytes per thread; cross-CTA tiles (always an smem exchange) keep at least 8
+    // warps per CTA (measured: 2 GiB transpose 0.91 -> 1.00 of the copy roofline at
+    // 4 -> 8 warps, profiles/r01_sweep_next_rows.jsonl)
+    int dflt = 256;
+    if (!in_cta) dflt = int(std::max<u64>(u64(P.w), std::min<u64>(256, ((u64(1) << Ss.size()) * u64(P.w)) / 256)));
+    int thread_bytes = default_int(opts, &ll_plan_opts::thread_bytes, dflt);
     assign_sigma_coalesced(T, A, B, Ss, Ds, prefer, maxvec, thread_bytes);
   }
   T.grid_src_bit = gridS;
