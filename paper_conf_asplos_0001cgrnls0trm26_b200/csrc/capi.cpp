@@ -102,6 +102,14 @@ void ensure_tile_kernel(ConvPlan& P) {
                "cudaFuncSetAttribute");
 }
 
+void ensure_gather_kernel(GatherPlan& G) {
+  std::lock_guard<std::mutex> g(G.mu);
+  if (G.kernel) return;
+  G.kernel = jit_kernel(codegen_gather(G), "ll_gather_kernel");
+  if (G.smem_bytes > 48 * 1024)
+    check_cuda(cudaFuncSetAttribute(G.kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, G.smem_bytes),
+               "cudaFuncSetAttribute");
+}
 }  // namespace ll
 
 namespace {
@@ -418,7 +426,8 @@ ll_status ll_plan_describe(const ll_plan* p, char* json, size_t cap) {
     const GatherPlan& G = *p->gather;
     std::ostringstream o;
     o << "{\"kind\":\"gather\",\"sigma\":\"" << (G.sigma ? "faithful" : "coalesced") << "\",\"R\":" << G.R
-      << ",\"warp_bits\":" << G.Wb << ",\"K_bits\":" << G.K_bits << ",\"shuffles_per_elem\":" << (1 << G.cand_bits)
+      << ",\"warp_bits\":" << G.Wb << ",\"K_bits\":" << G.K_bits
+      << ",\"exchange\":\"" << (G.smem ? "smem" : "shuffle") << "\",\"shuffles_per_elem\":" << (G.smem ? 0 : (1 << G.cand_bits))
       << ",\"ctas\":" << (u64(1) << G.grid_bit.size()) << "}";
     s = o.str();
   } else {
@@ -460,8 +469,7 @@ ll_status ll_plan_prepare(ll_plan* p) {
     if (p->cp().unpack && p->cp().unpack->exec == EXEC_TILE) ensure_tile_kernel(*p->cp().unpack);
   }
   if (p->kind == 1) {
-    std::lock_guard<std::mutex> g(p->gather->mu);
-    if (!p->gather->kernel) p->gather->kernel = jit_kernel(codegen_gather(*p->gather), "ll_gather_kernel");
+    ensure_gather_kernel(*p->gather);
   }
   if (p->kind == 2) {
     std::lock_guard<std::mutex> g(p->reduce->mu);
@@ -514,13 +522,11 @@ ll_status ll_gather(const void* src, const int32_t* idx, void* dst, const ll_pla
   if ((reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(idx) | reinterpret_cast<uintptr_t>(dst)) & 15)
     fail(LL_ERR_MISALIGNED, "buffers must be 16-byte aligned");
   GatherPlan& G = *p->gather;
-  {
-    std::lock_guard<std::mutex> g(G.mu);
-    if (!G.kernel) G.kernel = jit_kernel(codegen_gather(G), "ll_gather_kernel");
-  }
+  ensure_gather_kernel(G);
   unsigned long long nt = u64(1) << G.grid_bit.size();
   void* args[] = {const_cast<void**>(&src), const_cast<int32_t**>(&idx), &dst, &nt};
-  check_cuda(cudaLaunchKernel(G.kernel, dim3(grid_for(nt)), dim3(32u << G.Wb), args, 0, static_cast<cudaStream_t>(stream)),
+  check_cuda(cudaLaunchKernel(G.kernel, dim3(grid_for(nt)), dim3(32u << G.Wb), args, size_t(G.smem_bytes),
+                              static_cast<cudaStream_t>(stream)),
              "cudaLaunchKernel(ll_gather_kernel)");
   LL_CATCH
 }

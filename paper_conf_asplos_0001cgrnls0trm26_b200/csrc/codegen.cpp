@@ -75,6 +75,12 @@ std::string codegen_tile(const ConvPlan& Pl) {
   }
   o << arr("u64", "LD_COL", ldc) << arr("u64", "ST_COL", stc);
   emit_grid(o, T.grid_src_bit, T.grid_dst_bit, lw);
+  // broadcast destinations: every value is stored at 2^|rep| replica offsets (bytes)
+  std::vector<u64> rep(size_t(1) << T.rep_bits.size(), 0);
+  for (size_t r = 0; r < rep.size(); ++r)
+    for (size_t t = 0; t < T.rep_bits.size(); ++t)
+      if ((r >> t) & 1) rep[r] |= u64(1) << (T.rep_bits[t] + lw);
+  o << icon("NREP", rep.size()) << arr("u64", "REP_OFF", rep);
   // REGPERM
   o << arr("int", "PERM", T.perm);
   // SHUFFLE
@@ -106,7 +112,6 @@ std::string codegen_gather(const GatherPlan& G) {
   std::vector<u64> ldc;
   for (int b = 0; b < n; ++b) ldc.push_back(u64(1) << G.hw_bit[b]);   // element offsets
   o << arr("u64", "LD_COL", ldc);
-  std::vector<int> none;
   emit_grid(o, G.grid_bit, G.grid_bit, 0);
   o << icon("KBITS", G.K_bits) << icon("CBITS", G.cand_bits);
   o << arr("int", "AXIS_OF_LANE", G.axis_of_lane) << arr("int", "AXIS_LANE_POS", G.axis_lane_pos);
@@ -120,6 +125,11 @@ std::string codegen_gather(const GatherPlan& G) {
        " for (int b = 0; b < R; ++b) if (((E >> b) & 1) && AXIS_OF_REG[b] >= 0) a ^= 1u << AXIS_OF_REG[b]; return a; }\n";
   o << "  template <int E> static constexpr u32 cand_of_slot() { u32 c = 0;"
        " for (int i = 0; i < CBITS; ++i) if ((E >> CAND_REG[i]) & 1) c |= 1u << i; return c; }\n";
+  o << "  static constexpr bool GATHER_SMEM = " << (G.smem ? "true" : "false") << ";\n";
+  o << arr("u32", "SMOFF", G.smoff) << "  static constexpr u32 AXMASK = " << G.axmask << "u;\n"
+    << arr("int", "AXPOS", G.axpos);
+  o << "  template <int E> static constexpr u32 smoff_of_slot() { u32 s = 0;"
+       " for (int b = 0; b < R; ++b) if ((E >> b) & 1) s ^= SMOFF[b]; return s; }\n";
   o << "  template <int E, int C> static constexpr int slot_of() { int s = E;"
        " for (int i = 0; i < CBITS; ++i) { s &= ~(1 << CAND_REG[i]); if ((C >> i) & 1) s |= 1 << CAND_REG[i]; } return s; }\n";
   o << "};\n";

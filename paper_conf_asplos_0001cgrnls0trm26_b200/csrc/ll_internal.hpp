@@ -142,6 +142,7 @@ struct TilePlan {
   std::vector<int> ld_bit, st_bit;
   std::vector<u64> lcol_ld, lcol_st;
   std::vector<int> grid_src_bit, grid_dst_bit;   // CTA index bit g -> packed bits
+  std::vector<int> rep_bits;   // dst packed bits with zero columns in B: store replicas
   int sigma = SIGMA_COALESCED;
   int xchg = X_COPY;
 
@@ -213,6 +214,11 @@ struct GatherPlan {
   std::vector<int> axis_of_reg;  // kernel reg bit -> axis bit index or -1
   std::vector<int> axis_of_lane;
   int cand_bits = 0;       // |L_Reg^axis| in the kernel layout
+  bool smem = false;       // shared-memory gather (too many shuffle candidates)
+  std::vector<uint32_t> smoff;   // kernel bit -> smem element offset (logical tile order)
+  uint32_t axmask = 0;           // smem offset bits of the in-tile axis bits
+  std::vector<int> axpos;        // axis bit t -> smem offset bit
+  int smem_bytes = 0;
   std::string source;
   void* kernel = nullptr;
   std::mutex mu;

@@ -17,6 +17,11 @@ typedef unsigned long long u64;
 typedef unsigned short u16;
 typedef unsigned char u8;
 
+namespace std {
+template <bool B, class T, class F> struct conditional { typedef T type; };
+template <class T, class F> struct conditional<false, T, F> { typedef F type; };
+}  // namespace std
+
 // ------------------------------------------------------------------ compile-time loops
 template <int V> struct IC { static constexpr int value = V; };
 template <int I, int N, bool Small = (N - I <= 1)> struct SFor;
@@ -408,10 +413,13 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, u8* __r
       static_for<P::NW>([&](auto q) { o[decltype(q)::value] = 0; });
       xchg_smem<P>(r, o, lane, warp, sbase);
     }
-    // a10: HBM store of the dst tile
-    static_for<(1 << (P::R - P::VST))>([&](auto k) {
-      constexpr int K = decltype(k)::value;
-      store_vec<P::W, P::VST, K, P::NW, P::ST_HINT>(o, d + StOff<P, K>::value());
+    // a10: HBM store of the dst tile (and of its broadcast replicas)
+    static_for<P::NREP>([&](auto rp) {
+      constexpr u64 RO = P::REP_OFF[decltype(rp)::value];
+      static_for<(1 << (P::R - P::VST))>([&](auto k) {
+        constexpr int K = decltype(k)::value;
+        store_vec<P::W, P::VST, K, P::NW, P::ST_HINT>(o, d + (StOff<P, K>::value() ^ RO));
+      });
     });
     if constexpr (P::XCHG == 3) __syncthreads();   // smem reuse by the next tile
   }
@@ -433,6 +441,55 @@ __device__ __forceinline__ void ll_gather_body(const u8* __restrict__ src, const
     constexpr int T = decltype(t)::value;
     if constexpr (P::AXIS_OF_LANE[T] >= 0) if ((lane >> T) & 1) a_lane ^= 1u << P::AXIS_OF_LANE[T];
   });
+  if constexpr (P::GATHER_SMEM) {
+    // shared-memory gather (the paper's crossover): the tile is staged in smem
+    // in logical order; each output reads its source element directly.
+    extern __shared__ __align__(16) u8 ll_smem[];
+    typedef typename std::conditional<P::W == 4, u32, typename std::conditional<P::W == 2, u16, u8>::type>::type ET;
+    ET* sm = reinterpret_cast<ET*>(ll_smem);
+    u32 sthr = 0;
+    static_for<5>([&](auto t) {
+      constexpr int T = decltype(t)::value;
+      if ((lane >> T) & 1) sthr ^= P::SMOFF[P::R + T];
+    });
+    static_for<P::WB>([&](auto t) {
+      constexpr int T = decltype(t)::value;
+      if ((warp >> T) & 1) sthr ^= P::SMOFF[P::R + 5 + T];
+    });
+    for (u64 t = blockIdx.x; t < ntiles; t += gridDim.x) {
+      const u64 eoff = tile_base<P, true>(t) ^ thr;
+      u32 r[P::NW];
+      u32 ix[1 << P::R];
+      static_for<(1 << (P::R - P::VLD))>([&](auto k) {
+        constexpr int K = decltype(k)::value;
+        load_vec<P::W, P::VLD, K, P::NW, P::LD_L1>(r, src + (eoff ^ LdOff<P, K>::value()) * P::W);
+        load_vec<4, P::VLD, K, (1 << P::R), P::LD_L1>(ix, idx + (eoff ^ LdOff<P, K>::value()) * 4);
+      });
+      static_for<(1 << P::R)>([&](auto e) {
+        constexpr int E = decltype(e)::value;
+        sm[sthr ^ P::template smoff_of_slot<E>()] = ET(get_e<P::W, E>(r));
+      });
+      __syncthreads();
+      u32 o[P::NW];
+      static_for<P::NW>([&](auto q) { o[decltype(q)::value] = 0; });
+      static_for<(1 << P::R)>([&](auto e) {
+        constexpr int E = decltype(e)::value;
+        const u32 kidx = ix[E] & ((1u << P::KBITS) - 1u);
+        u32 off = (sthr ^ P::template smoff_of_slot<E>()) & ~P::AXMASK;
+        static_for<P::KBITS>([&](auto tt) {
+          constexpr int T = decltype(tt)::value;
+          off |= ((kidx >> T) & 1u) << P::AXPOS[T];
+        });
+        set_e<P::W, E>(o, u32(sm[off]));
+      });
+      static_for<(1 << (P::R - P::VLD))>([&](auto k) {
+        constexpr int K = decltype(k)::value;
+        store_vec<P::W, P::VLD, K, P::NW, P::ST_HINT>(o, dst + (eoff ^ LdOff<P, K>::value()) * P::W);
+      });
+      __syncthreads();
+    }
+    return;
+  }
   for (u64 t = blockIdx.x; t < ntiles; t += gridDim.x) {
     const u64 eoff = tile_base<P, true>(t) ^ thr;
     u32 r[P::NW];

@@ -112,7 +112,13 @@ static void assign_sigma_coalesced(TilePlan& T, const Layout& A, const Layout& B
   T.R = R;
   T.Wb = Wb;
   int v = std::min(std::max(0, ilog2(std::max(1, maxvec / w))), R);
-  T.vld = T.vst = v;
+  // a global vector needs its v bits to be the packed positions 0..v-1 (broadcast
+  // layouts may skip a low position: then the vector shrinks to the contiguous prefix)
+  int vl = 0, vs = 0;
+  while (vl < v && S[vl] == vl) ++vl;
+  while (vs < v && D[vs] == vs) ++vs;
+  T.vld = vl;
+  T.vst = vs;
   T.ld_bit.assign(n, -1);
   T.st_bit.assign(n, -1);
   for (int b = 0; b < v; ++b) { T.ld_bit[b] = S[b]; T.st_bit[b] = D[b]; }
@@ -240,13 +246,9 @@ static bool fit_affine(const std::vector<int>& f, int& c, int col[5]) {
 }
 
 // Conditional-swap stages realising "slot j <- slot j ⊕ (Σ_t l_t col_t)".
+// The stages use a basis of span{col_t}; lane bit t's mask is expressed in it, and
+// stage i fires on the parity of the lane bits whose expression contains basis vector i.
 static void xor_network(const int col[5], std::vector<uint32_t>& lmask, std::vector<int>& xs) {
-  Echelon e;
-  std::vector<u64> basis;
-  for (int t = 0; t < 5; ++t)
-    if (col[t] && e.insert(u64(col[t]), u64(1) << basis.size())) basis.push_back(0);
-  // recompute basis vectors from the echelon combos: store original vectors
-  basis.clear();
   Echelon e2;
   std::vector<u64> orig;
   for (int t = 0; t < 5; ++t)
@@ -553,7 +555,7 @@ static void build_tile(ConvPlan& P, const std::vector<int>& S0, const std::vecto
 
 // CTA class (Q mixes block/offset bits): choose the dst bits a CTA owns so that both
 // the loads and the stores are coalesced.
-static void choose_cta_tile(const ConvPlan& P, const std::vector<int>& pi, int nloc, int c_bits,
+static void choose_cta_tile(const std::vector<int>& pi, int nloc, int c_bits,
                             int target_bits, std::vector<int>& S, std::vector<int>& D,
                             std::vector<int>& gS, std::vector<int>& gD) {
   std::vector<int> inv(nloc, -1);
@@ -623,7 +625,7 @@ std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, 
           // 64 KiB of smem: 512-byte runs, else 256, else 128 (one line)
           const int max_bits = ilog2(u64(65536 / w));
           for (int c_bits = v + 5; c_bits >= v + 3; --c_bits) {
-            choose_cta_tile(*P, pi, nB, c_bits, target, S, D, gS, gD);
+            choose_cta_tile(pi, nB, c_bits, target, S, D, gS, gD);
             if (int(S.size()) <= max_bits) break;
           }
           build_tile(*P, S, D, gS, gD, opts, false);
@@ -633,6 +635,46 @@ std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, 
       } catch (const Error& e) {
         if (opts && opts->force_class >= 0) throw;
         // fall through to the generic kernel
+      }
+    }
+  }
+  // Broadcast layouts (zero columns, rule (2) P:362) inside one CTA: the
+  // non-zero columns of A and of B are each a permutation of the logical unit vectors.
+  // The kernel moves the distinct elements only: src bits with zero columns are never
+  // read (slack = 0), dst bits with zero columns become store replicas.
+  if (!generic && lev <= 2 && !(opts && opts->sigma == SIGMA_FAITHFUL)) {
+    auto nz_unit = [](const Layout& L) {
+      u64 seen = 0;
+      for (u64 c : L.cols) {
+        if (!c) continue;
+        if (popc(c) != 1 || (seen & c)) return false;
+        seen |= c;
+      }
+      return popc(seen) == L.d_out();
+    };
+    if (nz_unit(A) && nz_unit(B)) {
+      try {
+        std::vector<int> S, D, gS, gD, rep;
+        auto srcbit_of = [&](u64 c) {
+          for (int k = 0; k < nA; ++k) if (A.cols[k] == c) return k;
+          fail(LL_ERR_UNSUPPORTED, "broadcast: column missing in A (internal)");
+        };
+        for (int k : bits_at_level(B, 0, 2)) {
+          if (B.cols[k]) { D.push_back(k); S.push_back(srcbit_of(B.cols[k])); }
+          else rep.push_back(k);
+        }
+        for (int k : bits_at_level(B, 3, 3)) {
+          if (B.cols[k]) { gD.push_back(k); gS.push_back(srcbit_of(B.cols[k])); }
+          else rep.push_back(k);
+        }
+        if (rep.size() <= 4) {
+          build_tile(*P, S, D, gS, gD, opts, true);
+          P->tile.rep_bits = rep;
+          P->exec = EXEC_TILE;
+          return P;
+        }
+      } catch (const Error& e) {
+        if (opts && opts->force_class >= 0) throw;
       }
     }
   }
@@ -756,11 +798,7 @@ std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const 
   int v = std::min(ilog2(u64(std::max(1, maxvec / ev))), L.in_bits("reg"));
   auto regb = bits_at_level(L, 0, 0), laneb = bits_at_level(L, 1, 1), warpb = bits_at_level(L, 2, 2);
   const int R = int(regb.size());
-  auto cand_of = [&](const std::vector<int>& hw) {
-    int c = 0;
-    for (int b = 0; b < R; ++b) if (L.cols[hw[b]] & amask) ++c;
-    return c;
-  };
+
   std::vector<int> faith;
   for (int k : regb) faith.push_back(k);
   for (int k : laneb) faith.push_back(k);
@@ -771,7 +809,6 @@ std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const 
   std::vector<int> coal = sigma_line(L, v, [&](int k) { return (L.cols[k] & amask) != 0; });
   int sigma = opts ? opts->sigma : 0;
   bool use_coal = sigma != SIGMA_FAITHFUL;
-  (void)cand_of;
   G->hw_bit = use_coal ? coal : faith;
   G->sigma = use_coal ? SIGMA_COALESCED : SIGMA_FAITHFUL;
   G->R = R;
@@ -790,6 +827,24 @@ std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const 
     for (int b = 0; b < R; ++b) if (G->lcol[b] == c) { G->axis_reg_pos[t] = b; G->axis_of_reg[b] = t; ++G->cand_bits; }
     for (int l = 0; l < 5; ++l) if (G->lcol[R + l] == c) { G->axis_lane_pos[t] = l; G->axis_of_lane[l] = t; }
   }
+  // shuffles vs shared memory: the paper observes the shuffle rounds lose once
+  // the gathered dimension grows; the planner switches when more than 4
+  // candidates per element remain (force_class selects either)
+  int force = opts ? opts->force_class : -1;
+  G->smem = force == LL_CLASS_SMEM || (force != LL_CLASS_SHUFFLE && G->cand_bits > 2);
+  // smem layout: the tile's logical bits in ascending order (logical row-major tile)
+  std::vector<u64> tl(G->lcol.begin(), G->lcol.end());
+  std::sort(tl.begin(), tl.end());
+  auto rank_of = [&](u64 c) { return int(std::lower_bound(tl.begin(), tl.end(), c) - tl.begin()); };
+  G->smoff.resize(G->lcol.size());
+  for (size_t b = 0; b < G->lcol.size(); ++b) G->smoff[b] = 1u << rank_of(G->lcol[b]);
+  G->axpos.assign(G->K_bits, 0);
+  G->axmask = 0;
+  for (int t = 0; t < G->K_bits; ++t) {
+    G->axpos[t] = rank_of(u64(1) << (sh + t));
+    G->axmask |= 1u << G->axpos[t];
+  }
+  G->smem_bytes = G->smem ? int((u64(1) << G->lcol.size()) * u64(w)) : 0;
   return G;
 }
 

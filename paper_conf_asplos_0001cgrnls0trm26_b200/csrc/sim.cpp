@@ -89,11 +89,15 @@ void simulate_tile(const ConvPlan& P, const uint8_t* src, uint8_t* dst) {
           out[size_t(th) * E + e] = v;
         }
     }
-    for (int th = 0; th < NT; ++th)
-      for (int e = 0; e < E; ++e) {
-        u64 hw = u64(e) | (u64(th) << R);
-        std::memcpy(dst + (db | off(T.st_bit, hw)) * w, &out[size_t(th) * E + e], w);
-      }
+    for (u64 rp = 0; rp < (u64(1) << T.rep_bits.size()); ++rp) {
+      u64 ro = 0;
+      for (size_t t = 0; t < T.rep_bits.size(); ++t) if ((rp >> t) & 1) ro |= u64(1) << T.rep_bits[t];
+      for (int th = 0; th < NT; ++th)
+        for (int e = 0; e < E; ++e) {
+          u64 hw = u64(e) | (u64(th) << R);
+          std::memcpy(dst + (db | off(T.st_bit, hw) | ro) * w, &out[size_t(th) * E + e], w);
+        }
+    }
   }
 }
 

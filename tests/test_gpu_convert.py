@@ -172,20 +172,41 @@ def test_config3_full_size_sampled():
 
 @pytest.mark.parametrize("family", ["mma", "blocked"])
 @pytest.mark.parametrize("sigma", ["coalesced", "faithful"])
-def test_gather_bitexact(family, sigma):
-    """O10: gather via shuffles vs the oracle (take_along_axis)."""
+@pytest.mark.parametrize("k_bits", [4, 5, 6])
+@pytest.mark.parametrize("exchange", ["SHUFFLE", "SMEM"])
+def test_gather_bitexact(family, sigma, k_bits, exchange):
+    """O10: gather via shuffles or via shared memory (the P:519 crossover)
+    vs the oracle (take_along_axis), for the config-4 tiles [128, K], K = 16 / 32 / 64
+    (the survey's K sweep)."""
     rng = np.random.default_rng(1004)
-    spec = W.c4("gather", family, n_i=9, n_j=7)
+    spec = W.c4("gather", family, n_i=9, n_j=7, k_bits=k_bits)
     L, OL = both(spec)
     n = 1 << OL.d_in
     T = gen.random_bits(rng, n, 4)
     Ti = rng.integers(-1000, 1000, size=n).astype(np.int32)   # masked to [0, K) (G16)
     src, idx = O.pack(OL, T), O.pack(OL, Ti)
     ref = O.gather(OL, 1, src, idx)
-    plan = ll.ll_plan_gather(L, 1, 4, sigma=sigma)
+    plan = ll.ll_plan_gather(L, 1, 4, sigma=sigma, force_class=exchange)
+    assert plan.describe()["exchange"] == exchange.lower()
     d_dst = empty_device(n, 4)
     ll.ll_gather(to_device(src), to_device(idx.view(np.uint32)), d_dst, plan)
     assert np.array_equal(from_device(d_dst, 4), ref)
+
+
+@pytest.mark.parametrize("w", [2, 1])
+@pytest.mark.parametrize("exchange", ["SHUFFLE", "SMEM"])
+def test_gather_narrow_elements(w, exchange):
+    rng = np.random.default_rng(1009)
+    spec = W.c4("gather", "mma", n_i=8, n_j=6, k_bits=5)
+    L, OL = both(spec)
+    n = 1 << OL.d_in
+    T = gen.random_bits(rng, n, w)
+    Ti = rng.integers(0, 32, size=n).astype(np.int32)
+    src, idx = O.pack(OL, T), O.pack(OL, Ti)
+    plan = ll.ll_plan_gather(L, 1, w, force_class=exchange)
+    d_dst = empty_device(n, w)
+    ll.ll_gather(to_device(src), to_device(idx.view(np.uint32)), d_dst, plan)
+    assert np.array_equal(from_device(d_dst, w), O.gather(OL, 1, src, idx))
 
 
 def _line_sigma_layout(OL, axis):
@@ -342,3 +363,20 @@ def test_next_rows_n1_n2_bitexact(which):
     got, ref, plan = run_convert(sa, sb, w, 77)
     assert plan.describe()["exec"] == "tile"
     assert np.array_equal(got, ref)
+
+
+def test_broadcast_tile_kernels_gpu():
+    """Broadcast (zero-column) layouts through the specialised kernels (rule (2),
+    P:362): bit-exact, and at least some plans execute as tile kernels."""
+    rng = np.random.default_rng(55)
+    opts_z = [["reg", "lane"], ["lane", "warp"], ["reg", "warp"]]
+    tiles = 0
+    for case in range(24):
+        out = [("i", 4), ("j", 4)]
+        hw = [("reg", 3), ("lane", 5), ("warp", 2)]
+        sa = gen.random_distributed(rng, out, hw, zero_ok=opts_z[case % 3])
+        sb = gen.random_distributed(rng, out, hw, zero_ok=opts_z[(case // 3) % 3])
+        got, ref, plan = run_convert(sa, sb, [2, 4][case % 2], case)
+        assert np.array_equal(got, ref), plan.describe()
+        tiles += plan.describe()["exec"] == "tile"
+    assert tiles >= 8

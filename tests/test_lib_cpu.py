@@ -388,3 +388,20 @@ def test_tmem_fragment_family():
     B = ll.ll_layout_blocked([128, 64], [1, 4], [2, 16], [4, 1], [1, 0])
     p = ll.ll_plan_convert(L, B, 4)
     assert p.cls == "SMEM"
+
+
+def test_simulated_schedule_broadcast_layouts():
+    """Rule (2) / broadcast: layouts with zero columns run in the
+    specialised tile kernels — zero src bits are never read, zero dst bits become store
+    replicas; the emulated schedule equals the oracle's conversion."""
+    rng = np.random.default_rng(5)
+    tiles = 0
+    opts_z = [["reg", "lane"], ["lane", "warp"], ["reg", "warp", "block"], ["reg", "lane", "warp", "block"]]
+    for case in range(120):
+        out = [("i", 3 + case % 3), ("j", 4)]
+        hw = [("reg", 3), ("lane", 5), ("warp", 2), ("block", 1)]
+        sa = gen.random_distributed(rng, out, hw, zero_ok=opts_z[case % 4])
+        sb = gen.random_distributed(rng, out, hw, zero_ok=opts_z[(case // 4) % 4])
+        d = _sim_check(sa, sb, [1, 2, 4, 8][case % 4], case)
+        tiles += d["exec"] == "tile"
+    assert tiles >= 20

@@ -58,6 +58,8 @@ def main():
         return hints()
     if "next" in only:
         return next_rows()
+    if "lat" in only:
+        return latency_and_ksweep()
     if "all" not in only and "conv" not in only:
         return gather_reduce()
     # raw copy roofline reference
@@ -96,6 +98,47 @@ def next_rows():
         conv_case("c5T P=1 transpose", sa, sb, 2, **opts)
     for opts in [dict(), dict(tile_bytes=65536), dict(thread_bytes=128)]:
         conv_case("N1 preshuffle", *W.n1_preshuffle(14, 14), 2, **opts)
+
+
+def latency_and_ksweep():
+    """Config 1 single tile (latency-bound: CUDA graph of 1000 ll_convert launches) and
+    the config-4 gather K sweep (16 / 32 / 64)."""
+    A, B = ll.Layout.from_spec(W.C1_A), ll.Layout.from_spec(W.C1_B)
+    for fc in [None, "SMEM"]:
+        p = ll.ll_plan_convert(A, B, 4, force_class=fc)
+        p.prepare()
+        src = torch.randint(0, 1 << 30, (256,), dtype=torch.int32, device="cuda")
+        dst = torch.empty_like(src)
+        s = torch.cuda.Stream()
+        with torch.cuda.stream(s):
+            ll.ll_convert(src, dst, p, s)
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g, stream=s):
+                for _ in range(1000):
+                    ll.ll_convert(src, dst, p, torch.cuda.current_stream())
+        torch.cuda.synchronize()
+        ms = time_fn(lambda: g.replay(), iters=10, warmup=3)
+        print(json.dumps({"case": f"c1 single tile (16x16 fp32) {fc or 'auto'}: 1000 launches in a CUDA graph",
+                          "us_per_conversion": round(ms, 4), "xchg": p.describe()["tile"]["xchg"]}), flush=True)
+    for kb, fam, fc in [(k, f, x) for k in [4, 5, 6] for f in ["mma", "blocked"] for x in ["SHUFFLE", "SMEM"]]:
+        if True:
+            L = ll.Layout.from_spec(W.c4("gather", fam, k_bits=kb))
+            p = ll.ll_plan_gather(L, 1, 4, force_class=fc)
+            p.prepare()
+            n = 1 << 24
+            sets = [(torch.randint(-2 ** 31, 2 ** 31 - 1, (n,), dtype=torch.int32, device="cuda"),
+                     torch.randint(0, 1 << kb, (n,), dtype=torch.int32, device="cuda"),
+                     torch.empty(n, dtype=torch.int32, device="cuda")) for _ in range(4)]
+            it = [0]
+
+            def gg():
+                st = sets[it[0] % 4]
+                it[0] += 1
+                ll.ll_gather(st[0], st[1], st[2], p)
+            ms = time_fn(gg)
+            print(json.dumps({"case": f"gather {fam} K={1 << kb} {fc}", "desc": p.describe(), "ms": round(ms, 4),
+                              "GBps": round(12 * n / ms / 1e6, 1)}), flush=True)
+            del sets
 
 
 def hints():

@@ -102,16 +102,24 @@ def c3b(nb: int = 14):
 
 
 # ---- config 4: gather / reduce on 4096x4096 fp32 (tiles [128,32] / [128,128]) ----
-def c4(kind: str, family: str, n_i: int = 12, n_j: int = 12):
+def c4(kind: str, family: str, n_i: int = 12, n_j: int = 12, k_bits: int = 5):
     """kind in {gather, reduce}; family in {mma, blocked}.  Block bits are the tile
-    coordinates: i7.. then j5.. (gather) / j7.. (reduce)."""
+    coordinates: i7.. then j<K>.. (gather, K = 2^k_bits = 16/32/64) / j7.. (reduce)."""
     out = [("i", n_i), ("j", n_j)]
     if kind == "gather":
-        jt = 5
+        jt = k_bits
         if family == "mma":
-            reg, lane, warp = ["j0", "i3", "j3", "j4", "i6"], ["j1", "j2", "i0", "i1", "i2"], ["i4", "i5"]
+            # mma accumulator tile [128, K], 4 warps along M: n-reps j3.. then m-rep i6
+            reg = ["j0", "i3"] + _b("j", 3, k_bits) + ["i6"]
+            lane, warp = ["j1", "j2", "i0", "i1", "i2"], ["i4", "i5"]
         else:
-            reg, lane, warp = ["j0", "j1", "i4", "i5", "i6"], ["j2", "j3", "j4", "i0", "i1"], ["i2", "i3"]
+            # blocked [1,4]/[4,8]/[4,1] on [128, K]: lanes j2..j4 (8 along j) when K >= 32
+            if k_bits >= 5:
+                reg = ["j0", "j1"] + _b("j", 5, k_bits) + ["i4", "i5", "i6"]
+                lane, warp = ["j2", "j3", "j4", "i0", "i1"], ["i2", "i3"]
+            else:   # K = 16: threads [8, 4]
+                reg = ["j0", "j1", "i5", "i6"]
+                lane, warp = ["j2", "j3", "i0", "i1", "i2"], ["i3", "i4"]
     else:
         jt = 7
         if family == "mma":
