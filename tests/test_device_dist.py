@@ -153,3 +153,18 @@ def test_device_loopback_config5_large():
         xs = (O.apply_all(lb, hs) ^ np.uint64(offb)).astype(np.int64)
         got = dst[r * nloc + torch.from_numpy(hs.astype(np.int64)).cuda()]
         assert torch.equal(got, T[torch.from_numpy(xs).cuda()]), r
+
+
+@pytest.mark.gpu
+def test_nccl_comm_bootstrap_single_rank():
+    """NCCL through dlopen: ncclGetUniqueId + ncclCommInitRank (one rank on this GPU)
+    and destroy — the bootstrap every DEVICE plan uses (the multi-GPU exchange itself
+    needs >1 GPU, unavailable in this run)."""
+    import ctypes
+    uid = (ctypes.c_char * 128)()
+    ll._check(ll._lib.ll_comm_get_unique_id(uid))
+    assert any(b != 0 for b in bytes(uid))
+    h = ctypes.c_void_p()
+    ll._check(ll._lib.ll_comm_create(uid, 1, 0, ctypes.byref(h)))
+    assert h.value
+    ll._lib.ll_comm_destroy(h)
