@@ -228,6 +228,17 @@ void ll_plan_destroy(ll_plan* plan);
 ll_status ll_convert(const void* src, void* dst, void* workspace, const ll_plan* plan,
                      void* stream);
 
+/* ll_convert_host: the same conversion end to end from HOST buffers (pinned for
+ * overlap): the batch is split into chunks of whole CTA tiles, and each chunk runs
+ * H2D copy -> ll_tile_kernel -> D2H copy on streams[c % n_streams], so that copies in
+ * both directions and the kernels of different chunks overlap.
+ *   dev_buf: caller-owned device scratch of dev_buf_bytes (split into n_streams slots;
+ *   each slot must hold at least one tile of src and dst).  Asynchronous: the caller
+ *   synchronises the streams.  Tile plans whose CTA grid is the top bits of both
+ *   buffers, and NOOP plans; else LL_ERR_UNSUPPORTED. */
+ll_status ll_convert_host(const void* src_host, void* dst_host, void* dev_buf, size_t dev_buf_bytes,
+                          const ll_plan* plan, int n_streams, void* const* streams);
+
 /* ---------------------------------------------------------------- gather --
  * ll_plan_gather (row a11; §5.5).  src, idx and dst share layout L
  * (P:430).  Along logical dim `axis`, K = 2^(non-block axis bits of L); these

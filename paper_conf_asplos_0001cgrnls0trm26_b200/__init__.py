@@ -20,6 +20,21 @@ import numpy as np
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _LIB_PATH = os.path.join(_HERE, "libll.so")
 
+# NCCL for DEVICE plans is dlopen'ed by libll.so on first use.  Point it at the same
+# libnccl.so.2 torch links (the venv's nvidia-nccl wheel), so that a later `import
+# torch` does not meet an older system libnccl.so.2 already loaded under that soname.
+if not os.environ.get("LL_NCCL_LIB"):
+    try:
+        import importlib.util as _ilu
+        _spec = _ilu.find_spec("nvidia.nccl")
+        for _d in (list(_spec.submodule_search_locations) if _spec and _spec.submodule_search_locations else []):
+            _cand = os.path.join(_d, "lib", "libnccl.so.2")
+            if os.path.exists(_cand):
+                os.environ["LL_NCCL_LIB"] = _cand
+                break
+    except Exception:
+        pass
+
 if not os.path.exists(_LIB_PATH):
     raise ImportError(f"{_LIB_PATH} is missing: build it with `python -c 'import __graft_entry__ as g; g.build()'`")
 _lib = C.CDLL(_LIB_PATH)
@@ -84,6 +99,7 @@ _sig = {
     "ll_layout_contiguity": [_P, C.c_int, C.c_int, C.POINTER(C.c_int)],
     "ll_layout_mma_operand": [C.c_int] * 6 + [_PP],
     "ll_layout_tmem_32x32b": [C.c_int, C.c_int, _PP],
+    "ll_convert_host": [_P, _P, _P, C.c_size_t, _P, C.c_int, C.POINTER(C.c_void_p)],
 }
 for _name, _args in _sig.items():
     _f = getattr(_lib, _name)
@@ -456,6 +472,15 @@ def ll_plan_convert(A: Layout, B: Layout, elem_bytes: int, **opts) -> Plan:
 def ll_convert(src, dst, plan: Plan, stream=None, workspace=None):
     """dst <- convert(src) on `stream` (torch CUDA tensors or raw device pointers)."""
     _check(_lib.ll_convert(_ptr(src), _ptr(dst), _ptr(workspace), plan.handle, _stream_ptr(stream)))
+
+
+def ll_convert_host(src_host, dst_host, dev_buf, plan: Plan, streams):
+    """End-to-end conversion from pinned HOST tensors through the device (chunked H2D ->
+    kernel -> D2H pipeline over `streams`); dev_buf is a CUDA tensor used as scratch."""
+    arr = (C.c_void_p * len(streams))(*[s.cuda_stream for s in streams])
+    _check(_lib.ll_convert_host(C.c_void_p(src_host.data_ptr()), C.c_void_p(dst_host.data_ptr()),
+                                C.c_void_p(dev_buf.data_ptr()), dev_buf.numel() * dev_buf.element_size(),
+                                plan.handle, len(streams), arr))
 
 
 def ll_plan_gather(L: Layout, axis: int, elem_bytes: int, **opts) -> Plan:

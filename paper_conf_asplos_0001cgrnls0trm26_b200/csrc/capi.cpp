@@ -113,6 +113,8 @@ void ensure_gather_kernel(GatherPlan& G) {
 }  // namespace ll
 
 namespace {
+int ilog2_u64(u64 v) { return v ? 63 - __builtin_clzll(v) : -1; }
+
 unsigned grid_for(u64 ntiles) {
   const char* e = getenv("LL_GRID_PER_SM");
   int per = e ? atoi(e) : 0;
@@ -427,7 +429,7 @@ ll_status ll_plan_describe(const ll_plan* p, char* json, size_t cap) {
     std::ostringstream o;
     o << "{\"kind\":\"gather\",\"sigma\":\"" << (G.sigma ? "faithful" : "coalesced") << "\",\"R\":" << G.R
       << ",\"warp_bits\":" << G.Wb << ",\"K_bits\":" << G.K_bits
-      << ",\"exchange\":\"" << (G.smem ? "smem" : "shuffle") << "\",\"shuffles_per_elem\":" << (G.smem ? 0 : (1 << G.cand_bits))
+      << ",\"exchange\":\"" << (G.smem ? "smem" : "shuffle") << "\",\"tma\":" << (G.tma ? "true" : "false") << ",\"shuffles_per_elem\":" << (G.smem ? 0 : (1 << G.cand_bits))
       << ",\"ctas\":" << (u64(1) << G.grid_bit.size()) << "}";
     s = o.str();
   } else {
@@ -436,6 +438,7 @@ ll_status ll_plan_describe(const ll_plan* p, char* json, size_t cap) {
     o << "{\"kind\":\"reduce\",\"R\":" << Rp.R << ",\"warp_bits\":" << Rp.Wb << ",\"tree_levels\":" << Rp.red_reg.size()
       << ",\"bfly_stages\":" << Rp.red_lane.size() << ",\"warp_stages\":" << Rp.red_warp.size()
       << ",\"dup_bits\":" << Rp.dup_bits.size() << ",\"out_elems\":" << Rp.out_elems
+      << ",\"tma\":" << (Rp.tma ? "true" : "false") << ",\"stages\":" << Rp.stages << ",\"sigma\":\"" << (Rp.sigma ? "faithful" : "coalesced") << "\""
       << ",\"ctas\":" << (u64(1) << Rp.grid_bit.size()) << "}";
     s = o.str();
   }
@@ -504,6 +507,56 @@ ll_status ll_convert(const void* src, void* dst, void* ws, const ll_plan* p, voi
   LL_CATCH
 }
 
+ll_status ll_convert_host(const void* src_host, void* dst_host, void* dev_buf, size_t dev_buf_bytes,
+                          const ll_plan* p, int n_streams, void* const* streams) {
+  LL_TRY
+  if (!p || p->kind != 0 || !src_host || !dst_host || !dev_buf || n_streams < 1 || !streams)
+    fail(LL_ERR_INVALID_ARG, "bad argument");
+  ConvPlan& P = p->cp();
+  if (P.exec != EXEC_TILE && P.exec != EXEC_NOOP)
+    fail(LL_ERR_UNSUPPORTED, "ll_convert_host: tile or NOOP plans only (device / generic plans: use ll_convert)");
+  const TilePlan& T = P.tile;
+  // chunks are runs of whole CTA tiles, contiguous in both buffers: the grid bits must be
+  // the top bits of src and dst, in the same order
+  const int lw = P.w == 1 ? 0 : P.w == 2 ? 1 : P.w == 4 ? 2 : 3;
+  u64 ntiles = 1, tile_src = P.src_elems * P.w, tile_dst = P.dst_elems * P.w;
+  if (P.exec == EXEC_TILE) {
+    const size_t g = T.grid_dst_bit.size();
+    int ns = int(ilog2_u64(P.src_elems)), nd = int(ilog2_u64(P.dst_elems));
+    for (size_t k = 0; k < g; ++k)
+      if (T.grid_src_bit[k] != ns - int(g) + int(k) || T.grid_dst_bit[k] != nd - int(g) + int(k))
+        fail(LL_ERR_UNSUPPORTED, "ll_convert_host: the CTA grid is not the top bits of both buffers");
+    ntiles = u64(1) << g;
+    tile_src >>= g;
+    tile_dst >>= g;
+    (void)lw;
+  }
+  const u64 slot_bytes = dev_buf_bytes / u64(n_streams);
+  u64 chunk = slot_bytes / (tile_src + tile_dst);
+  if (chunk == 0) fail(LL_ERR_INVALID_ARG, "ll_convert_host: dev_buf too small for one tile per stream");
+  chunk = std::min<u64>(chunk, std::max<u64>(1, ntiles / (2 * u64(n_streams))));   // >= 2 chunks per stream
+  u64 c = 0;
+  for (u64 t0 = 0; t0 < ntiles; t0 += chunk, ++c) {
+    const u64 nt = std::min<u64>(chunk, ntiles - t0);
+    cudaStream_t st = static_cast<cudaStream_t>(streams[c % u64(n_streams)]);
+    char* slot = static_cast<char*>(dev_buf) + (c % u64(n_streams)) * slot_bytes;
+    char* dsrc = slot;
+    char* ddst = (P.exec == EXEC_NOOP) ? slot : slot + ((nt * tile_src + 15) & ~u64(15));
+    check_cuda(cudaMemcpyAsync(dsrc, static_cast<const char*>(src_host) + t0 * tile_src, nt * tile_src,
+                               cudaMemcpyHostToDevice, st), "cudaMemcpyAsync(H2D)");
+    if (P.exec == EXEC_TILE) {
+      ensure_tile_kernel(P);
+      unsigned long long n = nt;
+      void* args[] = {&dsrc, &ddst, &n};
+      check_cuda(cudaLaunchKernel(P.kernel, dim3(grid_for(nt)), dim3(T.threads()), args, size_t(P.smem_bytes), st),
+                 "cudaLaunchKernel(ll_tile_kernel)");
+    }
+    check_cuda(cudaMemcpyAsync(static_cast<char*>(dst_host) + t0 * tile_dst, ddst, nt * tile_dst,
+                               cudaMemcpyDeviceToHost, st), "cudaMemcpyAsync(D2H)");
+  }
+  LL_CATCH
+}
+
 ll_status ll_plan_gather(const ll_layout* L, int axis, int w, const ll_plan_opts* opts, ll_plan** plan) {
   LL_TRY
   if (!L || !plan) fail(LL_ERR_INVALID_ARG, "null argument");
@@ -525,7 +578,13 @@ ll_status ll_gather(const void* src, const int32_t* idx, void* dst, const ll_pla
   ensure_gather_kernel(G);
   unsigned long long nt = u64(1) << G.grid_bit.size();
   void* args[] = {const_cast<void**>(&src), const_cast<int32_t**>(&idx), &dst, &nt};
-  check_cuda(cudaLaunchKernel(G.kernel, dim3(grid_for(nt)), dim3(32u << G.Wb), args, size_t(G.smem_bytes),
+  // the TMA pipeline is persistent: as many CTAs as fit in shared memory per SM
+  unsigned grid = grid_for(nt);
+  if (G.tma) {
+    u64 per_sm = std::max<u64>(1, std::min<u64>(8, (228u * 1024u) / u64(G.smem_bytes + 1024)));
+    grid = unsigned(std::min<u64>(nt, per_sm * u64(num_sms())));
+  }
+  check_cuda(cudaLaunchKernel(G.kernel, dim3(grid), dim3(32u << G.Wb), args, size_t(G.smem_bytes),
                               static_cast<cudaStream_t>(stream)),
              "cudaLaunchKernel(ll_gather_kernel)");
   LL_CATCH
@@ -558,7 +617,9 @@ ll_status ll_reduce(const float* src, float* dst, const ll_plan* p, void* stream
   ReducePlan& Rp = *p->reduce;
   unsigned long long nt = u64(1) << Rp.grid_bit.size();
   void* args[] = {const_cast<float**>(&src), &dst, &nt};
-  check_cuda(cudaLaunchKernel(Rp.kernel, dim3(grid_for(nt)), dim3(32u << Rp.Wb), args, size_t(Rp.smem_bytes),
+  // the TMA pipeline is persistent: one CTA per SM streams its tiles through the stages
+  unsigned grid = Rp.tma ? unsigned(std::min<u64>(nt, u64(num_sms()))) : grid_for(nt);
+  check_cuda(cudaLaunchKernel(Rp.kernel, dim3(grid), dim3(32u << Rp.Wb), args, size_t(Rp.smem_bytes),
                               static_cast<cudaStream_t>(stream)),
              "cudaLaunchKernel(ll_reduce_kernel)");
   LL_CATCH

@@ -126,6 +126,8 @@ std::string codegen_gather(const GatherPlan& G) {
   o << "  template <int E> static constexpr u32 cand_of_slot() { u32 c = 0;"
        " for (int i = 0; i < CBITS; ++i) if ((E >> CAND_REG[i]) & 1) c |= 1u << i; return c; }\n";
   o << "  static constexpr bool GATHER_SMEM = " << (G.smem ? "true" : "false") << ";\n";
+  o << "  static constexpr bool TMA = " << (G.tma ? "true" : "false") << ";\n";
+  o << "  static constexpr unsigned STAGES = " << std::max(1, G.stages) << "u;\n";
   o << arr("u32", "SMOFF", G.smoff) << "  static constexpr u32 AXMASK = " << G.axmask << "u;\n"
     << arr("int", "AXPOS", G.axpos);
   o << "  template <int E> static constexpr u32 smoff_of_slot() { u32 s = 0;"
@@ -145,6 +147,9 @@ std::string codegen_reduce(const ReducePlan& Rp) {
   const int R = Rp.R, n = int(Rp.hw_bit.size());
   o << icon("W", 4) << icon("R", R) << icon("WB", Rp.Wb) << icon("VLD", Rp.v);
   o << "  static constexpr bool LD_L1 = " << (Rp.sigma == SIGMA_FAITHFUL ? "true" : "false") << ";\n";
+  o << "  static constexpr bool TMA = " << (Rp.tma ? "true" : "false") << ";\n";
+  o << "  static constexpr unsigned WRED_BYTES = " << Rp.wred_bytes << "u;\n";
+  o << "  static constexpr unsigned STAGES = " << std::max(1, Rp.stages) << "u;\n";
   std::vector<u64> ldc;
   for (int b = 0; b < n; ++b) ldc.push_back(u64(4) << Rp.hw_bit[b]);
   o << arr("u64", "LD_COL", ldc);

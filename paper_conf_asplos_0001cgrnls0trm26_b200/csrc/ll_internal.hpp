@@ -219,6 +219,8 @@ struct GatherPlan {
   uint32_t axmask = 0;           // smem offset bits of the in-tile axis bits
   std::vector<int> axpos;        // axis bit t -> smem offset bit
   int smem_bytes = 0;
+  bool tma = false;        // stream the contiguous src / idx tiles with cp.async.bulk
+  int stages = 0;
   std::string source;
   void* kernel = nullptr;
   std::mutex mu;
@@ -239,6 +241,9 @@ struct ReducePlan {
   std::vector<u64> out_col;       // per kernel bit: output flat offset (0 for reduced/dup)
   std::vector<u64> grid_out;      // per grid bit: output flat offset
   u64 out_elems = 0;
+  bool tma = false;        // stage each contiguous CTA tile with cp.async.bulk (UBLKCP)
+  int wred_bytes = 0;      // smem for the warp-level stage
+  int stages = 0;          // TMA pipeline depth
   std::string source;
   void* kernel = nullptr;
   int smem_bytes = 0;

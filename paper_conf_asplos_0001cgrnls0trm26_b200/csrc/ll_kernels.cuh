@@ -429,9 +429,69 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, u8* __r
 // P:428-432 (G15 reading): per output slot, read idx, locate the source
 // (register candidates, lane) and run 2^{|L_Reg^axis|} shuffle rounds, keeping the
 // value whose candidate equals the source register.
+// ------------------------------------------------------------------ TMA bulk copies
+// cp.async.bulk (SASS UBLKCP) global -> shared, completion tracked by an mbarrier
+// (expect_tx / complete_tx), the Blackwell async-copy pipeline.
+__device__ __forceinline__ void mbar_init(u32 bar, u32 count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_fence_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void fence_proxy_async() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(u32 bar, u32 bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(u32 dst, const void* src, u32 bytes, u32 bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+               ::"r"(dst), "l"(src), "r"(bytes), "r"(bar) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(u32 bar, u32 parity) {
+  u32 ok = 0;
+  do {
+    asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+                 "selp.u32 %0, 1, 0, p;\n\t}" : "=r"(ok) : "r"(bar), "r"(parity) : "memory");
+  } while (!ok);
+}
+__device__ __forceinline__ void lds_v4(u32 addr, u32& a, u32& b, u32& c, u32& d) {
+  asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(a), "=r"(b), "=r"(c), "=r"(d) : "r"(addr) : "memory");
+}
+
+// Shared-memory vector load of thread-local vector K (2^VL elements of W bytes).
+template <int W, int VL, int K, int NW>
+__device__ __forceinline__ void load_vec_s(u32 (&r)[NW], u32 addr) {
+  constexpr int VB = W << VL;
+  constexpr int E0 = K << VL;
+  if constexpr (VB == 16) {
+    lds_v4(addr, r[E0 * W / 4 + 0], r[E0 * W / 4 + 1], r[E0 * W / 4 + 2], r[E0 * W / 4 + 3]);
+  } else if constexpr (VB == 8) {
+    asm volatile("ld.shared.v2.u32 {%0,%1}, [%2];" : "=r"(r[E0 * W / 4]), "=r"(r[E0 * W / 4 + 1]) : "r"(addr) : "memory");
+  } else if constexpr (VB == 4) {
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(r[E0 * W / 4]) : "r"(addr) : "memory");
+  } else if constexpr (VB == 2) {
+    u16 h;
+    asm volatile("ld.shared.u16 %0, [%1];" : "=h"(h) : "r"(addr) : "memory");
+    set_e<2, E0 * W / 2>(r, u32(h));
+  } else {
+    u32 b;
+    asm volatile("ld.shared.u8 %0, [%1];" : "=r"(b) : "r"(addr) : "memory");
+    set_e<1, E0>(r, b & 0xffu);
+  }
+}
+
+// ------------------------------------------------------------------ gather (a11)
+// P:428-432 (G15 reading): per output slot, read idx, locate the source
+// (register candidates, lane) and run 2^{|L_Reg^axis|} shuffle rounds, keeping the
+// value whose candidate equals the source register; or, past the P:519 crossover,
+// gather from the tile staged in shared memory.  With P::TMA the contiguous src and
+// idx tiles are streamed through an mbarrier pipeline of cp.async.bulk copies.
 template <class P>
 __device__ __forceinline__ void ll_gather_body(const u8* __restrict__ src, const u8* __restrict__ idx,
                                                u8* __restrict__ dst, u64 ntiles) {
+  extern __shared__ __align__(16) u8 ll_smem[];
+  typedef typename std::conditional<P::W == 4, u32, typename std::conditional<P::W == 2, u16, u8>::type>::type ET;
   const u32 lane = threadIdx.x & 31u;
   const u32 warp = threadIdx.x >> 5;
   const u64 thr = thread_base<P, true>(lane, warp);           // element offsets (x W below)
@@ -441,13 +501,15 @@ __device__ __forceinline__ void ll_gather_body(const u8* __restrict__ src, const
     constexpr int T = decltype(t)::value;
     if constexpr (P::AXIS_OF_LANE[T] >= 0) if ((lane >> T) & 1) a_lane ^= 1u << P::AXIS_OF_LANE[T];
   });
+  // smem: [stages][src tile | idx tile] (TMA) | gather area (GATHER_SMEM) | mbarriers
+  constexpr u32 NE = u32(1) << (P::R + 5 + P::WB);          // tile elements
+  constexpr u32 TBS = NE * P::W, TBI = NE * 4, TBST = TBS + TBI;
+  constexpr u32 NS = P::TMA ? P::STAGES : 0;
+  const u32 sbase = u32(__cvta_generic_to_shared(ll_smem));
+  const u32 bar0 = sbase + NS * TBST + (P::GATHER_SMEM ? TBS : 0);
+  ET* sm = reinterpret_cast<ET*>(ll_smem + NS * TBST);
+  u32 sthr = 0;
   if constexpr (P::GATHER_SMEM) {
-    // shared-memory gather (the paper's crossover): the tile is staged in smem
-    // in logical order; each output reads its source element directly.
-    extern __shared__ __align__(16) u8 ll_smem[];
-    typedef typename std::conditional<P::W == 4, u32, typename std::conditional<P::W == 2, u16, u8>::type>::type ET;
-    ET* sm = reinterpret_cast<ET*>(ll_smem);
-    u32 sthr = 0;
     static_for<5>([&](auto t) {
       constexpr int T = decltype(t)::value;
       if ((lane >> T) & 1) sthr ^= P::SMOFF[P::R + T];
@@ -456,22 +518,58 @@ __device__ __forceinline__ void ll_gather_body(const u8* __restrict__ src, const
       constexpr int T = decltype(t)::value;
       if ((warp >> T) & 1) sthr ^= P::SMOFF[P::R + 5 + T];
     });
-    for (u64 t = blockIdx.x; t < ntiles; t += gridDim.x) {
-      const u64 eoff = tile_base<P, true>(t) ^ thr;
-      u32 r[P::NW];
-      u32 ix[1 << P::R];
+  }
+  auto issue = [&](u64 tq, u32 q) {
+    mbar_expect_tx(bar0 + 8 * q, TBST);
+    const u64 eb = tile_base<P, true>(tq);
+    bulk_g2s(sbase + q * TBST, src + eb * P::W, TBS, bar0 + 8 * q);
+    bulk_g2s(sbase + q * TBST + TBS, idx + eb * 4, TBI, bar0 + 8 * q);
+  };
+  if constexpr (P::TMA) {
+    if (threadIdx.x == 0) {
+      for (u32 q = 0; q < NS; ++q) mbar_init(bar0 + 8 * q, 1);
+      mbar_fence_init();
+    }
+    __syncthreads();
+    if (threadIdx.x == 0)
+      for (u32 q = 0; q + 1 < NS; ++q)
+        if (blockIdx.x + u64(q) * gridDim.x < ntiles) issue(blockIdx.x + u64(q) * gridDim.x, q);
+  }
+  u32 i = 0;
+  for (u64 t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
+    const u64 eoff = tile_base<P, true>(t) ^ thr;
+    u32 r[P::NW];
+    u32 ix[1 << P::R];
+    if constexpr (P::TMA) {
+      const u32 st = i % NS;
+      const u64 tn = t + u64(NS - 1) * gridDim.x;
+      if (threadIdx.x == 0 && tn < ntiles) {
+        fence_proxy_async();
+        issue(tn, (i + NS - 1) % NS);
+      }
+      mbar_wait(bar0 + 8 * st, (i / NS) & 1u);
+      const u32 ts = sbase + st * TBST;
+      static_for<(1 << (P::R - P::VLD))>([&](auto k) {
+        constexpr int K = decltype(k)::value;
+        load_vec_s<P::W, P::VLD, K>(r, ts + u32((thr ^ LdOff<P, K>::value()) * P::W));
+        load_vec_s<4, P::VLD, K>(ix, ts + TBS + u32((thr ^ LdOff<P, K>::value()) * 4));
+      });
+    } else {
       static_for<(1 << (P::R - P::VLD))>([&](auto k) {
         constexpr int K = decltype(k)::value;
         load_vec<P::W, P::VLD, K, P::NW, P::LD_L1>(r, src + (eoff ^ LdOff<P, K>::value()) * P::W);
         load_vec<4, P::VLD, K, (1 << P::R), P::LD_L1>(ix, idx + (eoff ^ LdOff<P, K>::value()) * 4);
       });
+    }
+    u32 o[P::NW];
+    static_for<P::NW>([&](auto q) { o[decltype(q)::value] = 0; });
+    if constexpr (P::GATHER_SMEM) {
+      // stage the tile in logical order, then every output reads its source element
       static_for<(1 << P::R)>([&](auto e) {
         constexpr int E = decltype(e)::value;
         sm[sthr ^ P::template smoff_of_slot<E>()] = ET(get_e<P::W, E>(r));
       });
       __syncthreads();
-      u32 o[P::NW];
-      static_for<P::NW>([&](auto q) { o[decltype(q)::value] = 0; });
       static_for<(1 << P::R)>([&](auto e) {
         constexpr int E = decltype(e)::value;
         const u32 kidx = ix[E] & ((1u << P::KBITS) - 1u);
@@ -482,52 +580,36 @@ __device__ __forceinline__ void ll_gather_body(const u8* __restrict__ src, const
         });
         set_e<P::W, E>(o, u32(sm[off]));
       });
-      static_for<(1 << (P::R - P::VLD))>([&](auto k) {
-        constexpr int K = decltype(k)::value;
-        store_vec<P::W, P::VLD, K, P::NW, P::ST_HINT>(o, dst + (eoff ^ LdOff<P, K>::value()) * P::W);
+    } else {
+      static_for<(1 << P::R)>([&](auto e) {
+        constexpr int E = decltype(e)::value;
+        // axis coordinate of slot E's element and its candidate part
+        constexpr u32 a_reg = P::template axis_of_slot<E>();
+        const u32 kidx = ix[E] & ((1u << P::KBITS) - 1u);
+        const u32 dlt = kidx ^ (a_reg ^ a_lane);
+        u32 sl = lane, ct = 0;
+        static_for<P::KBITS>([&](auto tt) {
+          constexpr int T = decltype(tt)::value;
+          const u32 bit = (dlt >> T) & 1u;
+          if constexpr (P::AXIS_LANE_POS[T] >= 0) sl ^= bit << P::AXIS_LANE_POS[T];
+          if constexpr (P::AXIS_CAND_POS[T] >= 0) ct ^= bit << P::AXIS_CAND_POS[T];
+        });
+        ct ^= P::template cand_of_slot<E>();
+        u32 res = 0;
+        static_for<(1 << P::CBITS)>([&](auto c) {
+          constexpr int C = decltype(c)::value;
+          constexpr int S = P::template slot_of<E, C>();
+          const u32 v = __shfl_sync(0xffffffffu, get_e<P::W, S>(r), int(sl));
+          res = (u32(C) == ct) ? v : res;
+        });
+        set_e<P::W, E>(o, res);
       });
-      __syncthreads();
     }
-    return;
-  }
-  for (u64 t = blockIdx.x; t < ntiles; t += gridDim.x) {
-    const u64 eoff = tile_base<P, true>(t) ^ thr;
-    u32 r[P::NW];
-    u32 ix[1 << P::R];
-    static_for<(1 << (P::R - P::VLD))>([&](auto k) {
-      constexpr int K = decltype(k)::value;
-      load_vec<P::W, P::VLD, K, P::NW, P::LD_L1>(r, src + (eoff ^ LdOff<P, K>::value()) * P::W);
-      load_vec<4, P::VLD, K, (1 << P::R), P::LD_L1>(ix, idx + (eoff ^ LdOff<P, K>::value()) * 4);
-    });
-    u32 o[P::NW];
-    static_for<P::NW>([&](auto q) { o[decltype(q)::value] = 0; });
-    static_for<(1 << P::R)>([&](auto e) {
-      constexpr int E = decltype(e)::value;
-      // axis coordinate of slot E's element and its candidate part
-      constexpr u32 a_reg = P::template axis_of_slot<E>();
-      const u32 kidx = ix[E] & ((1u << P::KBITS) - 1u);
-      const u32 dlt = kidx ^ (a_reg ^ a_lane);
-      u32 sl = lane, ct = 0;
-      static_for<P::KBITS>([&](auto tt) {
-        constexpr int T = decltype(tt)::value;
-        const u32 bit = (dlt >> T) & 1u;
-        if constexpr (P::AXIS_LANE_POS[T] >= 0) sl ^= bit << P::AXIS_LANE_POS[T];
-        if constexpr (P::AXIS_CAND_POS[T] >= 0) ct ^= bit << P::AXIS_CAND_POS[T];
-      });
-      ct ^= P::template cand_of_slot<E>();
-      u32 res = 0;
-      static_for<(1 << P::CBITS)>([&](auto c) {
-        constexpr int C = decltype(c)::value;
-        constexpr int S = P::template slot_of<E, C>();
-        const u32 v = __shfl_sync(0xffffffffu, get_e<P::W, S>(r), int(sl));
-        res = (u32(C) == ct) ? v : res;
-      });
-      set_e<P::W, E>(o, res);
-    });
     static_for<(1 << (P::R - P::VLD))>([&](auto k) {
       constexpr int K = decltype(k)::value;
       store_vec<P::W, P::VLD, K, P::NW, P::ST_HINT>(o, dst + (eoff ^ LdOff<P, K>::value()) * P::W);
     });
+    if constexpr (P::TMA || P::GATHER_SMEM) __syncthreads();
   }
 }
 
@@ -536,9 +618,80 @@ __device__ __forceinline__ void ll_gather_body(const u8* __restrict__ src, const
 // bits, smem over the Warp axis bits — in the layout's bit order (reg, lane, warp
 // ascending); zero-column (broadcast) bits are skipped and de-duplicated at store.
 template <class P>
+__device__ __forceinline__ void ll_reduce_tile(u32 (&r)[1 << P::R], float* sm, u32 lane, u32 warp, u64 oblk,
+                                               u64 othr, bool do_store, float* __restrict__ dst) {
+  // register tree, in the kernel layout's register-bit order
+  static_for<P::NRED_REG>([&](auto i) {
+    constexpr int B = P::RED_REG[decltype(i)::value];
+    static_for<(1 << P::R)>([&](auto e) {
+      constexpr int E = decltype(e)::value;
+      if constexpr (((E >> B) & 1) == 0 && (E & P::template done_mask<decltype(i)::value>()) == 0 &&
+                    (E & P::DUP_REG_MASK) == 0) {
+        r[E] = __float_as_uint(__fadd_rn(__uint_as_float(r[E]), __uint_as_float(r[E | (1 << B)])));
+      }
+    });
+  });
+  // butterfly over the lane axis bits
+  static_for<P::NRED_LANE>([&](auto i) {
+    constexpr int L = P::RED_LANE[decltype(i)::value];
+    static_for<(1 << P::R)>([&](auto e) {
+      constexpr int E = decltype(e)::value;
+      if constexpr ((E & (P::RED_REG_MASK | P::DUP_REG_MASK)) == 0) {
+        const float x = __uint_as_float(r[E]);
+        r[E] = __float_as_uint(__fadd_rn(x, __shfl_xor_sync(0xffffffffu, x, 1 << L)));
+      }
+    });
+  });
+  // warps through smem
+  if constexpr (P::NRED_WARP > 0) {
+    static_for<(1 << P::R)>([&](auto e) {
+      constexpr int E = decltype(e)::value;
+      if constexpr ((E & (P::RED_REG_MASK | P::DUP_REG_MASK)) == 0)
+        sm[(P::template live_index<E>() * (32 << P::WB)) + threadIdx.x] = __uint_as_float(r[E]);
+    });
+    __syncthreads();
+    if ((warp & P::RED_WARP_MASK) == 0) {
+      static_for<(1 << P::R)>([&](auto e) {
+        constexpr int E = decltype(e)::value;
+        if constexpr ((E & (P::RED_REG_MASK | P::DUP_REG_MASK)) == 0) {
+          float v[1 << P::NRED_WARP];
+          static_for<(1 << P::NRED_WARP)>([&](auto m) {
+            constexpr int M = decltype(m)::value;
+            u32 wsel = warp;
+            static_for<P::NRED_WARP>([&](auto q) {
+              constexpr int Q = decltype(q)::value;
+              if ((M >> Q) & 1) wsel |= 1u << P::RED_WARP[Q];
+            });
+            v[M] = sm[(P::template live_index<E>() * (32 << P::WB)) + wsel * 32 + lane];
+          });
+          static_for<P::NRED_WARP>([&](auto q) {
+            constexpr int Q = decltype(q)::value;
+            static_for<(1 << P::NRED_WARP)>([&](auto m) {
+              constexpr int M = decltype(m)::value;
+              if constexpr (((M >> Q) & 1) == 0 && (M & ((1 << Q) - 1)) == 0)
+                v[M] = __fadd_rn(v[M], v[M | (1 << Q)]);
+            });
+          });
+          r[E] = __float_as_uint(v[0]);
+        }
+      });
+    }
+    __syncthreads();
+  }
+  if (do_store) {
+    static_for<(1 << P::R)>([&](auto e) {
+      constexpr int E = decltype(e)::value;
+      if constexpr ((E & (P::RED_REG_MASK | P::DUP_REG_MASK)) == 0) {
+        constexpr u64 oc = P::template out_of_slot<E>();
+        dst[oblk ^ othr ^ oc] = __uint_as_float(r[E]);
+      }
+    });
+  }
+}
+
+template <class P>
 __device__ __forceinline__ void ll_reduce_body(const float* __restrict__ src, float* __restrict__ dst, u64 ntiles) {
   extern __shared__ __align__(16) u8 ll_smem[];
-  float* sm = reinterpret_cast<float*>(ll_smem);
   const u32 lane = threadIdx.x & 31u;
   const u32 warp = threadIdx.x >> 5;
   u64 othr = 0;
@@ -550,86 +703,73 @@ __device__ __forceinline__ void ll_reduce_body(const float* __restrict__ src, fl
     constexpr int T = decltype(t)::value;
     if ((warp >> T) & 1) othr ^= P::OUT_COL[P::R + 5 + T];
   });
-  const bool lane_store = (lane & P::NOSTORE_LANE_MASK) == 0;
-  const bool warp_store = (warp & P::NOSTORE_WARP_MASK) == 0;
-  for (u64 t = blockIdx.x; t < ntiles; t += gridDim.x) {
+  const bool do_store = ((lane & P::NOSTORE_LANE_MASK) == 0) && ((warp & P::NOSTORE_WARP_MASK) == 0);
+  auto out_blk = [&](u64 t) {
     u64 oblk = 0;
     static_for<P::G>([&](auto g) {
       constexpr int Gi = decltype(g)::value;
       if ((t >> Gi) & 1) oblk ^= P::GRID_OUT[Gi];
     });
-    const u8* s = reinterpret_cast<const u8*>(src) + (tile_base<P, true>(t) ^ thread_base<P, true>(lane, warp));
-    u32 r[1 << P::R];
-    static_for<(1 << (P::R - P::VLD))>([&](auto k) {
-      constexpr int K = decltype(k)::value;
-      load_vec<4, P::VLD, K, (1 << P::R), P::LD_L1>(r, s + LdOff<P, K>::value());
-    });
-    // register tree, in the layout's register-bit order
-    static_for<P::NRED_REG>([&](auto i) {
-      constexpr int B = P::RED_REG[decltype(i)::value];
-      static_for<(1 << P::R)>([&](auto e) {
-        constexpr int E = decltype(e)::value;
-        if constexpr (((E >> B) & 1) == 0 && (E & P::template done_mask<decltype(i)::value>()) == 0 &&
-                      (E & P::DUP_REG_MASK) == 0) {
-          r[E] = __float_as_uint(__fadd_rn(__uint_as_float(r[E]), __uint_as_float(r[E | (1 << B)])));
-        }
-      });
-    });
-    // butterfly over the lane axis bits
-    static_for<P::NRED_LANE>([&](auto i) {
-      constexpr int L = P::RED_LANE[decltype(i)::value];
-      static_for<(1 << P::R)>([&](auto e) {
-        constexpr int E = decltype(e)::value;
-        if constexpr ((E & (P::RED_REG_MASK | P::DUP_REG_MASK)) == 0) {
-          const float x = __uint_as_float(r[E]);
-          r[E] = __float_as_uint(__fadd_rn(x, __shfl_xor_sync(0xffffffffu, x, 1 << L)));
-        }
-      });
-    });
-    // warps through smem
-    if constexpr (P::NRED_WARP > 0) {
-      static_for<(1 << P::R)>([&](auto e) {
-        constexpr int E = decltype(e)::value;
-        if constexpr ((E & (P::RED_REG_MASK | P::DUP_REG_MASK)) == 0)
-          sm[(P::template live_index<E>() * (32 << P::WB)) + threadIdx.x] = __uint_as_float(r[E]);
-      });
-      __syncthreads();
-      if ((warp & P::RED_WARP_MASK) == 0) {
-        static_for<(1 << P::R)>([&](auto e) {
-          constexpr int E = decltype(e)::value;
-          if constexpr ((E & (P::RED_REG_MASK | P::DUP_REG_MASK)) == 0) {
-            float v[1 << P::NRED_WARP];
-            static_for<(1 << P::NRED_WARP)>([&](auto m) {
-              constexpr int M = decltype(m)::value;
-              u32 wsel = warp;
-              static_for<P::NRED_WARP>([&](auto q) {
-                constexpr int Q = decltype(q)::value;
-                if ((M >> Q) & 1) wsel |= 1u << P::RED_WARP[Q];
-              });
-              v[M] = sm[(P::template live_index<E>() * (32 << P::WB)) + wsel * 32 + lane];
-            });
-            static_for<P::NRED_WARP>([&](auto q) {
-              constexpr int Q = decltype(q)::value;
-              static_for<(1 << P::NRED_WARP)>([&](auto m) {
-                constexpr int M = decltype(m)::value;
-                if constexpr (((M >> Q) & 1) == 0 && (M & ((1 << Q) - 1)) == 0)
-                  v[M] = __fadd_rn(v[M], v[M | (1 << Q)]);
-              });
-            });
-            r[E] = __float_as_uint(v[0]);
-          }
-        });
-      }
-      __syncthreads();
+    return oblk;
+  };
+  const u64 thr = thread_base<P, true>(lane, warp);
+  if constexpr (P::TMA) {
+    // The CTA tile of L is contiguous in HBM: one cp.async.bulk per tile into a
+    // double-buffered stage, completion on an mbarrier; the next tile's copy is in
+    // flight while this one is reduced.  Stage reads use the line-coalesced σ offsets
+    // (16-byte vectors, 8 lanes per 128-byte row: conflict-free).
+    constexpr u32 TB = u32(4) << (P::R + 5 + P::WB);
+    constexpr u32 NS = P::STAGES;
+    const u32 sbase = u32(__cvta_generic_to_shared(ll_smem));
+    const u32 bar0 = sbase + NS * TB + P::WRED_BYTES;
+    float* sm = reinterpret_cast<float*>(ll_smem + NS * TB);
+    if (threadIdx.x == 0) {
+      for (u32 q = 0; q < NS; ++q) mbar_init(bar0 + 8 * q, 1);
+      mbar_fence_init();
     }
-    if (lane_store && warp_store) {
-      static_for<(1 << P::R)>([&](auto e) {
-        constexpr int E = decltype(e)::value;
-        if constexpr ((E & (P::RED_REG_MASK | P::DUP_REG_MASK)) == 0) {
-          constexpr u64 oc = P::template out_of_slot<E>();
-          dst[oblk ^ othr ^ oc] = __uint_as_float(r[E]);
+    __syncthreads();
+    // prologue: the first NS - 1 tiles of this CTA are in flight before any compute
+    if (threadIdx.x == 0) {
+      for (u32 q = 0; q + 1 < NS; ++q) {
+        const u64 tq = blockIdx.x + u64(q) * gridDim.x;
+        if (tq < ntiles) {
+          mbar_expect_tx(bar0 + 8 * q, TB);
+          bulk_g2s(sbase + q * TB, reinterpret_cast<const u8*>(src) + tile_base<P, true>(tq), TB, bar0 + 8 * q);
         }
+      }
+    }
+    u32 i = 0;
+    for (u64 t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
+      const u32 st = i % NS;
+      // refill the stage consumed in the previous iteration with tile i + NS - 1
+      const u64 tn = t + u64(NS - 1) * gridDim.x;
+      if (threadIdx.x == 0 && tn < ntiles) {
+        const u32 sn = (i + NS - 1) % NS;
+        fence_proxy_async();
+        mbar_expect_tx(bar0 + 8 * sn, TB);
+        bulk_g2s(sbase + sn * TB, reinterpret_cast<const u8*>(src) + tile_base<P, true>(tn), TB, bar0 + 8 * sn);
+      }
+      mbar_wait(bar0 + 8 * st, (i / NS) & 1u);
+      u32 r[1 << P::R];
+      const u32 tb = sbase + st * TB + u32(thr);
+      static_for<(1 << (P::R - P::VLD))>([&](auto k) {
+        constexpr int K = decltype(k)::value;
+        constexpr int E0 = K << P::VLD;
+        lds_v4(tb + u32(LdOff<P, K>::value()), r[E0], r[E0 + 1], r[E0 + 2], r[E0 + 3]);
       });
+      ll_reduce_tile<P>(r, sm, lane, warp, out_blk(t), othr, do_store, dst);
+      __syncthreads();   // stage st is free before it is refilled next iteration
+    }
+  } else {
+    float* sm = reinterpret_cast<float*>(ll_smem);
+    for (u64 t = blockIdx.x; t < ntiles; t += gridDim.x) {
+      const u8* s = reinterpret_cast<const u8*>(src) + (tile_base<P, true>(t) ^ thr);
+      u32 r[1 << P::R];
+      static_for<(1 << (P::R - P::VLD))>([&](auto k) {
+        constexpr int K = decltype(k)::value;
+        load_vec<4, P::VLD, K, (1 << P::R), P::LD_L1>(r, s + LdOff<P, K>::value());
+      });
+      ll_reduce_tile<P>(r, sm, lane, warp, out_blk(t), othr, do_store, dst);
     }
   }
 }

@@ -844,7 +844,26 @@ std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const 
     G->axpos[t] = rank_of(u64(1) << (sh + t));
     G->axmask |= 1u << G->axpos[t];
   }
-  G->smem_bytes = G->smem ? int((u64(1) << G->lcol.size()) * u64(w)) : 0;
+  const u64 ne = u64(1) << G->lcol.size();
+  const u64 gbytes = G->smem ? ne * u64(w) : 0;
+  // TMA staging (cp.async.bulk of the contiguous src and idx tiles, 2 stages) with the
+  // line-coalesced σ; force_class = CTA keeps direct LDG loads (a diagnostic knob)
+  bool contiguous = true;
+  {
+    int p = 0;
+    for (auto& d : L.in) {
+      if (dim_level(d.name) <= 2 && p + d.bits > int(G->lcol.size())) contiguous = false;
+      p += d.bits;
+    }
+  }
+  G->stages = 2;
+  const u64 stage_bytes = ne * u64(w + 4);
+  // measured (profiles/r01_sweep_gather_tma.jsonl): the bulk-copy pipeline wins from
+  // 64 KiB stages (K = 64: +10-15%), direct LDG wins below (K = 16: +5-8%)
+  G->tma = G->sigma == SIGMA_COALESCED && contiguous && force != LL_CLASS_CTA &&
+           (stage_bytes >= 65536 || force == LL_CLASS_SHUFFLE || force == LL_CLASS_SMEM) &&
+           u64(G->stages) * stage_bytes + gbytes + 16 <= 200 * 1024 && (G->v + ilog2(u64(w))) >= 2;
+  G->smem_bytes = int(gbytes + (G->tma ? u64(G->stages) * stage_bytes + 8 * G->stages : 0));
   return G;
 }
 
@@ -916,7 +935,25 @@ std::unique_ptr<ReducePlan> plan_reduce(const Layout& L, int axis, const ll_plan
   Rp->out_elems = u64(1) << (L.d_out() - K);
   int live = R - int(Rp->red_reg.size());
   for (int b : Rp->dup_bits) if (b < R) --live;
-  Rp->smem_bytes = Rp->red_warp.empty() ? 0 : int((u64(4) << (std::max(0, live) + 5 + Rp->Wb)));
+  Rp->wred_bytes = Rp->red_warp.empty() ? 0 : int((u64(4) << (std::max(0, live) + 5 + Rp->Wb)));
+  // TMA staging (cp.async.bulk) when the CTA tile is contiguous in HBM (reg, lane, warp
+  // are L's lowest packed bits), the stage reads are 16-byte line-coalesced (σ), and two
+  // stages fit in smem; force_class = SHUFFLE keeps direct LDG loads
+  const u64 tile_bytes = u64(4) << (R + 5 + Rp->Wb);
+  bool contiguous = true;
+  {
+    int p = 0;
+    for (auto& d : L.in) {
+      if (dim_level(d.name) <= 2 && p + d.bits > R + 5 + Rp->Wb) contiguous = false;
+      p += d.bits;
+    }
+  }
+  int force = opts ? opts->force_class : -1;
+  Rp->stages = 0;
+  for (int ns = 4; ns >= 2; --ns)
+    if (u64(ns) * tile_bytes + u64(Rp->wred_bytes) + 8 * ns <= 200 * 1024) { Rp->stages = ns; break; }
+  Rp->tma = Rp->sigma == SIGMA_COALESCED && Rp->v == 2 && contiguous && force != LL_CLASS_SHUFFLE && Rp->stages;
+  Rp->smem_bytes = Rp->tma ? int(Rp->stages * tile_bytes + Rp->wred_bytes + 8 * Rp->stages) : Rp->wred_bytes;
   return Rp;
 }
 

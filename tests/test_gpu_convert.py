@@ -173,7 +173,7 @@ def test_config3_full_size_sampled():
 @pytest.mark.parametrize("family", ["mma", "blocked"])
 @pytest.mark.parametrize("sigma", ["coalesced", "faithful"])
 @pytest.mark.parametrize("k_bits", [4, 5, 6])
-@pytest.mark.parametrize("exchange", ["SHUFFLE", "SMEM"])
+@pytest.mark.parametrize("exchange", ["SHUFFLE", "SMEM", "LDG"])
 def test_gather_bitexact(family, sigma, k_bits, exchange):
     """O10: gather via shuffles or via shared memory (the P:519 crossover)
     vs the oracle (take_along_axis), for the config-4 tiles [128, K], K = 16 / 32 / 64
@@ -186,8 +186,15 @@ def test_gather_bitexact(family, sigma, k_bits, exchange):
     Ti = rng.integers(-1000, 1000, size=n).astype(np.int32)   # masked to [0, K) (G16)
     src, idx = O.pack(OL, T), O.pack(OL, Ti)
     ref = O.gather(OL, 1, src, idx)
-    plan = ll.ll_plan_gather(L, 1, 4, sigma=sigma, force_class=exchange)
-    assert plan.describe()["exchange"] == exchange.lower()
+    # SHUFFLE / SMEM: forced exchange (TMA-staged when coalesced); LDG: automatic
+    # exchange with direct global loads (force_class = CTA)
+    plan = ll.ll_plan_gather(L, 1, 4, sigma=sigma, force_class="CTA" if exchange == "LDG" else exchange)
+    d = plan.describe()
+    if exchange != "LDG":
+        assert d["exchange"] == exchange.lower()
+        assert d["tma"] == (sigma == "coalesced")
+    else:
+        assert not d["tma"]
     d_dst = empty_device(n, 4)
     ll.ll_gather(to_device(src), to_device(idx.view(np.uint32)), d_dst, plan)
     assert np.array_equal(from_device(d_dst, 4), ref)
@@ -234,7 +241,7 @@ def _line_sigma_layout(OL, axis):
 
 
 @pytest.mark.parametrize("family", ["mma", "blocked"])
-@pytest.mark.parametrize("sigma", ["coalesced", "faithful"])
+@pytest.mark.parametrize("sigma", ["coalesced", "coalesced-ldg", "faithful"])
 def test_reduce_tolerance_and_fixed_order(family, sigma):
     """O11: ≤ 1e-6 relative vs fp64, and bit-exact vs the fixed-order fp32 replica
     taken over the kernel's layout (L itself for faithful σ; L∘σ for the coalesced
@@ -246,7 +253,10 @@ def test_reduce_tolerance_and_fixed_order(family, sigma):
     n = 1 << OL.d_in
     T = rng.random(n, dtype=np.float32)
     src = O.pack(OL, T)
-    plan = ll.ll_plan_reduce(L, 1, sigma=sigma)
+    # "coalesced" stages tiles with cp.async.bulk (TMA), "coalesced-ldg" loads directly
+    plan = ll.ll_plan_reduce(L, 1, sigma=sigma.split("-")[0],
+                             force_class="SHUFFLE" if sigma == "coalesced-ldg" else None)
+    assert plan.describe()["tma"] == (sigma == "coalesced")
     out = torch.empty(plan.out_elems(), dtype=torch.float32, device="cuda")
     ll.ll_reduce(torch.from_numpy(src).cuda(), out, plan)
     got = out.cpu().numpy()
@@ -380,3 +390,22 @@ def test_broadcast_tile_kernels_gpu():
         assert np.array_equal(got, ref), plan.describe()
         tiles += plan.describe()["exec"] == "tile"
     assert tiles >= 8
+
+
+def test_convert_host_pipeline():
+    """ll_convert_host: pinned host src -> chunked H2D / kernel / D2H over two streams
+    -> pinned host dst, equal to the oracle."""
+    import torch
+    sa, sb = W.c2(6)
+    A, OA = both(sa)
+    B, OB = both(sb)
+    plan = ll.ll_plan_convert(A, B, 2)
+    rng = np.random.default_rng(8)
+    src = O.pack(OA, gen.random_bits(rng, 1 << OA.d_out, 2))
+    h_src = torch.from_numpy(src.view(np.int16).copy()).pin_memory()
+    h_dst = torch.zeros_like(h_src).pin_memory()
+    dev = torch.empty(1 << 20, dtype=torch.uint8, device="cuda")    # forces several chunks
+    streams = [torch.cuda.Stream(), torch.cuda.Stream()]
+    ll.ll_convert_host(h_src, h_dst, dev, plan, streams)
+    torch.cuda.synchronize()
+    assert np.array_equal(h_dst.numpy().view(np.uint16), O.convert(OA, OB, src))

@@ -15,18 +15,29 @@ import paper_conf_asplos_0001cgrnls0trm26_b200 as ll  # noqa: E402
 from workloads import configs as W  # noqa: E402
 
 
-def time_fn(fn, iters=20, warmup=5):
+def time_fn(fn, iters=20, warmup=5, batch=None):
+    """Median over `iters` samples of the time per call; each sample times `batch`
+    back-to-back calls between two events (default: 1, or 20 for calls < 100 us so that
+    small kernels are measured as a stream, not one launch latency each)."""
     for _ in range(warmup):
         fn()
     torch.cuda.synchronize()
-    ts = []
-    for _ in range(iters):
+    if batch is None:
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record()
         fn()
         b.record()
         b.synchronize()
-        ts.append(a.elapsed_time(b))
+        batch = 20 if a.elapsed_time(b) < 0.1 else 1
+    ts = []
+    for _ in range(iters):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        for _ in range(batch):
+            fn()
+        b.record()
+        b.synchronize()
+        ts.append(a.elapsed_time(b) / batch)
     ts.sort()
     return ts[len(ts) // 2]
 
@@ -120,7 +131,7 @@ def latency_and_ksweep():
         ms = time_fn(lambda: g.replay(), iters=10, warmup=3)
         print(json.dumps({"case": f"c1 single tile (16x16 fp32) {fc or 'auto'}: 1000 launches in a CUDA graph",
                           "us_per_conversion": round(ms, 4), "xchg": p.describe()["tile"]["xchg"]}), flush=True)
-    for kb, fam, fc in [(k, f, x) for k in [4, 5, 6] for f in ["mma", "blocked"] for x in ["SHUFFLE", "SMEM"]]:
+    for kb, fam, fc in [(k, f, x) for k in [4, 5, 6] for f in ["mma", "blocked"] for x in ["SHUFFLE", "SMEM", "CTA"]]:
         if True:
             L = ll.Layout.from_spec(W.c4("gather", fam, k_bits=kb))
             p = ll.ll_plan_gather(L, 1, 4, force_class=fc)
@@ -136,7 +147,7 @@ def latency_and_ksweep():
                 it[0] += 1
                 ll.ll_gather(st[0], st[1], st[2], p)
             ms = time_fn(gg)
-            print(json.dumps({"case": f"gather {fam} K={1 << kb} {fc}", "desc": p.describe(), "ms": round(ms, 4),
+            print(json.dumps({"case": f"gather {fam} K={1 << kb} {fc if fc != 'CTA' else 'auto-exchange, LDG (no TMA)'}", "desc": p.describe(), "ms": round(ms, 4),
                               "GBps": round(12 * n / ms / 1e6, 1)}), flush=True)
             del sets
 
@@ -193,19 +204,21 @@ def gather_reduce(tag="", sigmas=("coalesced", "faithful")):
             ms = time_fn(g)
             print(json.dumps({"case": f"gather {fam} {sig}{tag}", "desc": p.describe(), "ms": round(ms, 4),
                               "GBps": round(12 * n / ms / 1e6, 1)}), flush=True)
-        L = ll.Layout.from_spec(W.c4("reduce", fam))
-        p = ll.ll_plan_reduce(L, 1)
-        p.prepare()
-        n = 1 << 24
-        sets = [(torch.rand(n, device="cuda"), torch.empty(p.out_elems(), device="cuda")) for _ in range(4)]
-        it = [0]
+        for fc in [None, "SHUFFLE"]:
+            L = ll.Layout.from_spec(W.c4("reduce", fam))
+            p = ll.ll_plan_reduce(L, 1, force_class=fc)
+            p.prepare()
+            n = 1 << 24
+            sets = [(torch.rand(n, device="cuda"), torch.empty(p.out_elems(), device="cuda")) for _ in range(4)]
+            it = [0]
 
-        def r():
-            s = sets[it[0] % 4]
-            it[0] += 1
-            ll.ll_reduce(s[0], s[1], p)
-        ms = time_fn(r)
-        print(json.dumps({"case": f"reduce {fam}{tag}", "ms": round(ms, 4), "GBps": round((4 * n + 4 * p.out_elems()) / ms / 1e6, 1)}), flush=True)
+            def r():
+                s = sets[it[0] % 4]
+                it[0] += 1
+                ll.ll_reduce(s[0], s[1], p)
+            ms = time_fn(r)
+            print(json.dumps({"case": f"reduce {fam}{tag} {'tma' if p.describe()['tma'] else 'ldg'}", "ms": round(ms, 4),
+                              "GBps": round((4 * n + 4 * p.out_elems()) / ms / 1e6, 1)}), flush=True)
 
 
 if __name__ == "__main__":
