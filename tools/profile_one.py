@@ -35,18 +35,25 @@ if a.case in conv:
     for _ in range(a.iters):
         ll.ll_convert(src, dst, p)
 elif a.case.startswith("gather"):
-    fam = a.case.split("_")[1]
-    p = ll.ll_plan_gather(ll.Layout.from_spec(W.c4("gather", fam)), 1, 4)
-    n = 1 << 24
+    parts = a.case.split("_")
+    fam = parts[1]
+    kb = int(parts[2]) if len(parts) > 2 else 5
+    small = len(parts) > 3
+    spec = W.c4("gather", fam, k_bits=kb) if not small else W.c4("gather", fam, n_i=9, n_j=8, k_bits=kb)
+    p = ll.ll_plan_gather(ll.Layout.from_spec(spec), 1, 4)
+    n = 1 << (24 if not small else 17)
     s = torch.randint(0, 1 << 30, (n,), dtype=torch.int32, device="cuda")
     i = torch.randint(0, 32, (n,), dtype=torch.int32, device="cuda")
     d = torch.empty_like(s)
     for _ in range(a.iters):
         ll.ll_gather(s, i, d, p)
 else:
-    fam = a.case.split("_")[1]
-    p = ll.ll_plan_reduce(ll.Layout.from_spec(W.c4("reduce", fam)), 1)
-    s = torch.rand(1 << 24, device="cuda")
+    parts = a.case.split("_")
+    fam = parts[1]
+    small = len(parts) > 2
+    spec = W.c4("reduce", fam) if not small else W.c4("reduce", fam, n_i=9, n_j=9)
+    p = ll.ll_plan_reduce(ll.Layout.from_spec(spec), 1)
+    s = torch.rand(1 << (24 if not small else 18), device="cuda")
     d = torch.empty(p.out_elems(), device="cuda")
     for _ in range(a.iters):
         ll.ll_reduce(s, d, p)
