@@ -477,6 +477,49 @@ def mma_acc(shape, warps_m, warps_n=1) -> Layout:
     return Layout(in_dims, [("d0", mb), ("d1", nb)], {"reg": reg, "lane": lane, "warp": warp})
 
 
+def mma_operand(is_rhs: bool, shape, bitwidth: int, warps_m: int = 1, warps_n: int = 1) -> Layout:
+    """mma / wgmma input operand tiles (Prop 9.2), written from the paper:
+        lhs:  id^{Reg,1}_{log2(32/b)} x id^{Thr,1}_2 x id^{Thr,0}_3 x id^{Reg,0}_1 x id^{Reg,1}_1
+        rhs:  id^{Reg,0}_{log2(32/b)} x id^{Thr,0}_2 x id^{Thr,1}_3 x id^{Reg,1}_1
+    (the product is taken left to right, each factor's bits above the previous ones in
+    its dims).  Dims: lhs (d0 = M, d1 = K), rhs (d0 = K, d1 = N).  Repetitions: over the
+    K dim first, then the other dim, as register bits.  Warps: warps_m split M and
+    warps_n split N; the operand is broadcast over the other dim's warps
+    (zero columns)."""
+    rows, cols = shape
+    rb, cb = int(rows).bit_length() - 1, int(cols).bit_length() - 1
+    kb = (32 // bitwidth).bit_length() - 1
+    used = {0: 0, 1: 0}
+    def take(dim):
+        c = [0, 0]
+        nb = rb if dim == 0 else cb
+        if used[dim] < nb:
+            c[dim] = 1 << used[dim]
+        used[dim] += 1
+        return tuple(c)
+    kdim, odim = (0, 1) if is_rhs else (1, 0)
+    reg, lane, warp = [], [], []
+    reg += [take(kdim) for _ in range(kb)]
+    lane += [take(kdim) for _ in range(2)]
+    lane += [take(odim) for _ in range(3)]
+    if not is_rhs:
+        reg.append(take(odim))
+    reg.append(take(kdim))
+    wm, wn = int(warps_m).bit_length() - 1, int(warps_n).bit_length() - 1
+    for _ in range(wm):
+        warp.append((0, 0) if is_rhs else take(odim))
+    for _ in range(wn):
+        warp.append(take(odim) if is_rhs else (0, 0))
+    nbk = rb if is_rhs else cb
+    nbo = cb if is_rhs else rb
+    while used[kdim] < nbk:
+        reg.append(take(kdim))
+    while used[odim] < nbo:
+        reg.append(take(odim))
+    in_dims = [("reg", len(reg)), ("lane", 5), ("warp", len(warp))]
+    return Layout(in_dims, [("d0", rb), ("d1", cb)], {"reg": reg, "lane": lane, "warp": warp})
+
+
 def sliced(L: Layout, dim: int) -> Layout:
     """Slice: remove logical dim ``dim`` (Prop 4.8).  The result may be
     non-injective (zero columns) but stays surjective (Remark P:224)."""

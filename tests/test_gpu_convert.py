@@ -409,3 +409,63 @@ def test_convert_host_pipeline():
     ll.ll_convert_host(h_src, h_dst, dev, plan, streams)
     torch.cuda.synchronize()
     assert np.array_equal(h_dst.numpy().view(np.uint16), O.convert(OA, OB, src))
+
+
+# ---------------------------------------------------------------- N3: Table 4 families
+TABLE4_SHAPES = [(128, 16), (128, 128), (32, 128), (32, 32), (16, 16)]
+
+
+def _table4_layout(family, shape, rng):
+    """(oracle layout, product layout) of one Table 4 family on `shape`,
+    4 warps.  Sliced<F> is F on [a, b] times one extra register bit on a third
+    dim, sliced away (Prop 4.8): a broadcast register (zero column)."""
+    a, b = shape
+    if family == "blocked":
+        args = ([a, b], [1, 4], [8, 4], [4, 1], [1, 0])
+        return O.blocked(*args), ll.ll_layout_blocked(*args)
+    if family == "mma":
+        return O.mma_acc([a, b], 4), ll.ll_layout_mma_acc(a, b, 4)
+    if family == "mma_input":
+        return O.mma_operand(False, (a, b), 16, 4, 1), ll.ll_layout_mma_operand(0, a, b, 16, 4, 1)
+    if family.startswith("sliced_"):
+        OP, _ = _table4_layout(family[len("sliced_"):], shape, rng)
+        # parent over [a, b, 2]: the extra register bit hits the new dim, then slice it
+        out3 = list(OP.out_dims) + [("d2", 1)]
+        bases = {n: [tuple(v) + (0,) for v in OP.bases[n]] for n, _ in OP.in_dims}
+        bases["reg"] = bases["reg"] + [(0, 0, 1)]
+        in3 = [(n, nb + (1 if n == "reg" else 0)) for n, nb in OP.in_dims]
+        parent = O.Layout(in3, out3, bases)
+        OS = O.sliced(parent, 2)
+        return OS, ll.Layout(OS.in_dims, OS.out_dims, OS.bases)
+    # custom: a random distributed layout with broadcast lanes / registers
+    out = [("r", a.bit_length() - 1), ("c", b.bit_length() - 1)]
+    d = sum(x for _, x in out)
+    nreg = max(1, d - 7 + 2)
+    spec = gen.random_distributed(rng, out, [("reg", nreg), ("lane", 5), ("warp", 2)], zero_ok=["reg", "lane", "warp"])
+    OL = O.Layout(*W.spec_to_bases(spec))
+    return OL, ll.Layout(OL.in_dims, OL.out_dims, OL.bases)
+
+
+@pytest.mark.parametrize("family", ["blocked", "mma", "mma_input", "sliced_blocked", "sliced_mma",
+                                    "sliced_mma_input", "custom"])
+def test_table4_reduce_families(family):
+    """§8(f) N3: reductions (tl.sum along the last dim) over every Table 4 layout family
+    on the Table 4 shapes: ≤ 1e-6 relative vs fp64 and bit-exact vs the
+    fixed-order replica on the kernel layout; broadcast copies counted once."""
+    import torch
+    rng = np.random.default_rng(4747)
+    for shape in TABLE4_SHAPES:
+        OL, L = _table4_layout(family, shape, rng)
+        assert L.cols() == OL.cols
+        n = 1 << OL.d_in
+        T = rng.random(1 << OL.d_out, dtype=np.float32)
+        src = O.pack(OL, T)
+        plan = ll.ll_plan_reduce(L, 1)
+        out = torch.full((plan.out_elems(),), -1.0, dtype=torch.float32, device="cuda")
+        ll.ll_reduce(torch.from_numpy(src).cuda(), out, plan)
+        got = out.cpu().numpy()
+        ref = T.astype(np.float64).reshape(shape).sum(axis=1)
+        assert np.all(np.abs(got - ref) <= 1e-6 * np.abs(ref)), (family, shape)
+        Lp, perm = _line_sigma_layout(OL, 1)
+        rep = O.reduce_fixed_order_fp32(Lp, 1, src[perm])
+        assert np.array_equal(got.view(np.uint32), rep.view(np.uint32)), (family, shape)

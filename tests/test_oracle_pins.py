@@ -566,3 +566,22 @@ def test_distributed_rank_slices_concatenate():
             got = O.convert_distributed_rank(A, B, T, r)
             cols = M[:, r * (16 // P):(r + 1) * (16 // P)]
             assert np.array_equal(got, cols.reshape(-1))
+
+
+@pytest.mark.parametrize("bits", [16, 8, 32])
+def test_oracle_mma_operand_matches_ptx(bits):
+    """Prop 9.2 operand tiles in the oracle vs the PTX m16n8kK A / B
+    fragment formulas [HW] (g = lane/4, t = lane%4, e = 32/bits elements per register):
+    A: row = g + 8((i/e)%2), col = e·t + i%e + 4e·(i/(2e)); B: k = e·t + i%e + 4e·(i/e), n = g."""
+    e = 32 // bits
+    K = 8 * e
+    A = O.mma_operand(False, (16, K), bits)
+    B = O.mma_operand(True, (K, 8), bits)
+    for h in range(1 << A.d_in):
+        i, lane = h & ((1 << A.dim_bits("reg").__len__()) - 1), h >> len(A.dim_bits("reg"))
+        g, t = lane // 4, lane % 4
+        assert O.logical_coords(A.out_dims, O.apply(A, h)) == (g + 8 * ((i // e) % 2), e * t + i % e + 4 * e * (i // (2 * e)))
+    for h in range(1 << B.d_in):
+        i, lane = h & ((1 << len(B.dim_bits("reg"))) - 1), h >> len(B.dim_bits("reg"))
+        g, t = lane // 4, lane % 4
+        assert O.logical_coords(B.out_dims, O.apply(B, h)) == (e * t + i % e + 4 * e * (i // e), g)
