@@ -70,11 +70,22 @@ std::string codegen_tile(const ConvPlan& Pl) {
   o << "  static constexpr bool LD_L1 = " << (T.sigma == SIGMA_FAITHFUL ? "true" : "false") << ";\n";
   std::vector<u64> ldc, stc;
   for (int b = 0; b < T.n; ++b) {
-    ldc.push_back(u64(1) << (T.ld_bit[b] + lw));
+    ldc.push_back(T.ld_xcol.empty() ? (u64(1) << (T.ld_bit[b] + lw)) : (T.ld_xcol[b] << lw));
     stc.push_back(u64(1) << (T.st_bit[b] + lw));
   }
   o << arr("u64", "LD_COL", ldc) << arr("u64", "ST_COL", stc);
-  emit_grid(o, T.grid_src_bit, T.grid_dst_bit, lw);
+  if (T.grid_src_xcol.empty()) {
+    emit_grid(o, T.grid_src_bit, T.grid_dst_bit, lw);
+  } else {
+    // XOR grid: per-bit src / dst offsets (never contiguous shifts)
+    std::vector<u64> ld, st;
+    for (size_t g = 0; g < T.grid_dst_bit.size(); ++g) {
+      ld.push_back(T.grid_src_xcol[g] << lw);
+      st.push_back(u64(1) << (T.grid_dst_bit[g] + lw));
+    }
+    o << icon("G", T.grid_dst_bit.size()) << "  static constexpr bool GRID_CONTIG = false;\n"
+      << icon("GRID_LD_SHIFT", 0) << icon("GRID_ST_SHIFT", 0) << arr("u64", "GRID_LD", ld) << arr("u64", "GRID_ST", st);
+  }
   // broadcast destinations: every value is stored at 2^|rep| replica offsets (bytes)
   std::vector<u64> rep(size_t(1) << T.rep_bits.size(), 0);
   for (size_t r = 0; r < rep.size(); ++r)

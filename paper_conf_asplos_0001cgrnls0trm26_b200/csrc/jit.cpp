@@ -85,18 +85,25 @@ std::string compile(const std::string& full, const char* name) {
   return cubin;
 }
 
+// Read-only cache of the cubins build() pre-compiles for the benchmark / smoke plans
+// (travels with the tree); the writable cache (LL_JIT_CACHE) holds everything else.
+std::string prebuilt_dir() { return self_dir() + "/.ll_jit_prebuilt"; }
+
+std::string read_file(const std::string& path) {
+  std::ifstream f(path, std::ios::binary);
+  if (!f) return std::string();
+  std::stringstream ss;
+  ss << f.rdbuf();
+  return ss.str();
+}
+
 std::string cubin_for(const std::string& full, const char* name, std::string* key_out) {
   std::string key = key_of(full);
   if (key_out) *key_out = key;
   std::string path = cache_dir() + "/" + key + ".cubin";
-  {
-    std::ifstream f(path, std::ios::binary);
-    if (f) {
-      std::stringstream ss;
-      ss << f.rdbuf();
-      std::string s = ss.str();
-      if (!s.empty()) return s;
-    }
+  for (const std::string& p : {path, prebuilt_dir() + "/" + key + ".cubin"}) {
+    std::string s = read_file(p);
+    if (!s.empty()) return s;
   }
   std::string cubin = compile(full, name);
   std::string tmp = path + ".tmp" + std::to_string(getpid());

@@ -143,6 +143,10 @@ struct TilePlan {
   std::vector<u64> lcol_ld, lcol_st;
   std::vector<int> grid_src_bit, grid_dst_bit;   // CTA index bit g -> packed bits
   std::vector<int> rep_bits;   // dst packed bits with zero columns in B: store replicas
+  // Linear (XOR) copy plans: the src index of kernel bit b / grid bit g is an arbitrary
+  // F2 combination Q(dst bit) (swizzled memory layouts, Def 4.14; broadcast).  When
+  // non-empty these replace 1 << ld_bit / 1 << grid_src_bit.
+  std::vector<u64> ld_xcol, grid_src_xcol;
   int sigma = SIGMA_COALESCED;
   int xchg = X_COPY;
 

@@ -678,6 +678,62 @@ std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, 
       }
     }
   }
+  // Any other linear pull map (2-bit columns of swizzled memory layouts, Def 4.14 /
+  // P:240-276; broadcast across CTAs): a copy kernel in dst order — coalesced 16-byte
+  // stores, loads at src = Q(dst) (XOR of columns), vectorised over the low dst bits Q
+  // keeps in place.  Efficient when Q is row-local (swizzles); the generic kernel is
+  // kept for maps that scatter the low bits.
+  if (!generic && lev <= 3 && nB >= 5) {
+    int vmax = std::max(0, ilog2(u64(std::max(1, default_int(opts, &ll_plan_opts::max_vec_bytes, 16) / w))));
+    int v = 0;
+    while (v < vmax && v < nB && P->Q[v] == (u64(1) << v)) ++v;
+    // the low lane bits must keep whole 32-byte sectors together: Q maps dst bits [v, v+2)
+    // to src bits of single weight
+    bool rowlocal = true;
+    for (int k = v; k < std::min(nB, v + 2); ++k) if (popc(P->Q[k]) != 1) rowlocal = false;
+    if (rowlocal) {
+      TilePlan& T = P->tile;
+      T = TilePlan();
+      T.w = w;
+      const int tb = default_int(opts, &ll_plan_opts::tile_bytes, 16384);
+      int n = std::min(nB, std::max(v + 5, ilog2(u64(std::max(1, tb / w)))));
+      int thread_bytes = default_int(opts, &ll_plan_opts::thread_bytes, 64);
+      int R = std::max(v, ilog2(u64(std::max(1, thread_bytes / w))));
+      int Wb = std::min(5, std::max(0, n - 5 - R));
+      R = n - 5 - Wb;
+      if (R >= v) {
+        T.n = n; T.R = R; T.Wb = Wb;
+        T.vld = T.vst = v;
+        // dst bits in order: kreg[0,v), klane, kreg[v,R), kwarp; grid = the top bits
+        std::vector<int> order;
+        for (int k = 0; k < v; ++k) order.push_back(k);
+        std::vector<int> lane_bits, reg_bits, warp_bits;
+        int k = v;
+        for (int t = 0; t < 5; ++t) lane_bits.push_back(k++);
+        for (int t = v; t < R; ++t) reg_bits.push_back(k++);
+        for (int t = 0; t < Wb; ++t) warp_bits.push_back(k++);
+        T.st_bit = order;
+        T.st_bit.insert(T.st_bit.end(), reg_bits.begin(), reg_bits.end());
+        T.st_bit.insert(T.st_bit.end(), lane_bits.begin(), lane_bits.end());
+        T.st_bit.insert(T.st_bit.end(), warp_bits.begin(), warp_bits.end());
+        T.ld_bit = T.st_bit;   // (unused for the load side: ld_xcol)
+        for (int b : T.st_bit) T.ld_xcol.push_back(P->Q[b]);
+        for (int g = n; g < nB; ++g) {
+          T.grid_dst_bit.push_back(g);
+          T.grid_src_bit.push_back(g);
+          T.grid_src_xcol.push_back(P->Q[g]);
+        }
+        T.lcol_ld.assign(n, 0);
+        T.lcol_st.assign(n, 0);
+        for (int b = 0; b < n; ++b) T.lcol_st[b] = T.lcol_ld[b] = B.cols[T.st_bit[b]];
+        T.xchg = X_COPY;
+        T.sigma = SIGMA_COALESCED;
+        P->smem_bytes = 0;
+        P->exec = EXEC_TILE;
+        return P;
+      }
+    }
+  }
   P->exec = EXEC_GENERIC;
   return P;
 }

@@ -20,17 +20,26 @@ void simulate_tile(const ConvPlan& P, const uint8_t* src, uint8_t* dst) {
     for (int b = 0; b < n; ++b) if ((hw >> b) & 1) o |= u64(1) << bits[b];
     return o;
   };
+  auto ld_off = [&](u64 hw) {
+    if (T.ld_xcol.empty()) return off(T.ld_bit, hw);
+    u64 o = 0;
+    for (int b = 0; b < n; ++b) if ((hw >> b) & 1) o ^= T.ld_xcol[b];
+    return o;
+  };
   std::vector<uint64_t> in(size_t(NT) * E), out(size_t(NT) * E);
   std::vector<uint8_t> smem(T.xchg == X_SMEM ? T.smem_elems * w : 0);
   auto getv = [&](const uint8_t* p) { uint64_t v = 0; std::memcpy(&v, p, w); return v; };
   for (u64 t = 0; t < ntiles; ++t) {
     u64 sb = 0, db = 0;
     for (size_t g = 0; g < T.grid_dst_bit.size(); ++g)
-      if ((t >> g) & 1) { sb |= u64(1) << T.grid_src_bit[g]; db |= u64(1) << T.grid_dst_bit[g]; }
+      if ((t >> g) & 1) {
+        sb ^= T.grid_src_xcol.empty() ? (u64(1) << T.grid_src_bit[g]) : T.grid_src_xcol[g];
+        db |= u64(1) << T.grid_dst_bit[g];
+      }
     for (int th = 0; th < NT; ++th)
       for (int e = 0; e < E; ++e) {
         u64 hw = u64(e) | (u64(th) << R);
-        in[size_t(th) * E + e] = getv(src + (sb | off(T.ld_bit, hw)) * w);
+        in[size_t(th) * E + e] = getv(src + (sb ^ ld_off(hw)) * w);
       }
     if (T.xchg == X_COPY) {
       out = in;

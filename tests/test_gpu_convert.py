@@ -469,3 +469,24 @@ def test_table4_reduce_families(family):
         Lp, perm = _line_sigma_layout(OL, 1)
         rep = O.reduce_fixed_order_fp32(Lp, 1, src[perm])
         assert np.array_equal(got.view(np.uint32), rep.view(np.uint32)), (family, shape)
+
+
+def test_swizzled_memory_layout_gpu():
+    """Row-major -> Def 4.11 mma-swizzled memory layout of a 1024 x 1024 bf16 matrix
+    (vec 8, per_phase 1, max_phase 8 — the 128-byte swizzle pattern) on the XOR-column
+    copy kernel: element (i, j) lands at i*2^10 + Def 4.11 offset."""
+    import torch
+    m = n = 10
+    S = ll.ll_layout_mma_swizzle(m, n, 8, 1, 8)
+    R = ll.Layout([("offset", m + n)], [("d0", m), ("d1", n)],
+                  {"offset": [((1 << (k - n)) if k >= n else 0, (1 << k) if k < n else 0) for k in range(m + n)]})
+    plan = ll.ll_plan_convert(R, S, 2)
+    assert plan.describe()["exec"] == "tile"
+    T = gen.random_bits(np.random.default_rng(12), 1 << (m + n), 2)
+    d_dst = empty_device(1 << (m + n), 2)
+    ll.ll_convert(to_device(T), d_dst, plan)
+    got = from_device(d_dst, 2)
+    i = np.arange(1 << m)[:, None]
+    j = np.arange(1 << n)[None, :]
+    off = (i << n) + ((((i // 1) % 8) ^ (j // 8)) * 8 ^ (j % 8))
+    assert np.array_equal(got[off.reshape(-1)], T)

@@ -437,3 +437,29 @@ def test_exhaustive_fig1_all_40320():
     assert sum(counts.values()) == 40320
     # bijective relabelings never broadcast: NOOP exactly once (B = A)
     assert counts.get("NOOP") == 1
+
+
+@pytest.mark.parametrize("vec,pp,mp", [(8, 1, 8), (4, 2, 4), (8, 2, 4), (2, 1, 8)])
+def test_swizzled_memory_layout_xor_copy(vec, pp, mp):
+    """Row-major -> Def 4.11 mma-swizzled memory layout and back: the pull
+    map has 2-bit columns; the planner runs it as a vectorised XOR-column copy kernel
+    whose emulated schedule equals the oracle (and the Def 4.11 formula)."""
+    m = n = 6
+    rng = np.random.default_rng(vec * 100 + pp * 10 + mp)
+    row = O.identity_memory([("i", m), ("j", n)])
+    S = ll.ll_layout_mma_swizzle(m, n, vec, pp, mp)
+    R = ll.Layout(row.in_dims, [("d0", m), ("d1", n)], {"offset": [((c >> n), c & ((1 << n) - 1)) for c in row.cols]})
+    T = gen.random_bits(rng, 1 << (m + n), 2)
+    for A, B in ((R, S), (S, R)):
+        p = ll.ll_plan_convert(A, B, 2)
+        assert p.describe()["exec"] == "tile"
+        OA = O.layout_from_cols([("offset", m + n)], [("d0", m), ("d1", n)], A.cols())
+        OB = O.layout_from_cols([("offset", m + n)], [("d0", m), ("d1", n)], B.cols())
+        src = O.pack(OA, T)
+        assert np.array_equal(p.simulate(src, 1 << (m + n)), O.convert(OA, OB, src))
+    # the swizzled buffer holds element (i, j) at offset i*2^n + Def 4.11 offset
+    p = ll.ll_plan_convert(R, S, 2)
+    got = p.simulate(T, 1 << (m + n))
+    for i in range(0, 64, 5):
+        for j in range(0, 64, 3):
+            assert got[(i << n) + O.mma_swizzle_offset(i, j, vec, pp, mp)] == T[(i << n) + j]

@@ -99,8 +99,25 @@ def main():
     gather_reduce()
 
 
+def swizzle_case():
+    """Row-major -> Def 4.11 mma-swizzled memory layout, 16384 x 16384 bf16 (XOR copy)."""
+    m = n = 14
+    S = ll.ll_layout_mma_swizzle(m, n, 8, 1, 8)
+    R = ll.Layout([("offset", m + n)], [("d0", m), ("d1", n)],
+                  {"offset": [((1 << (k - n)) if k >= n else 0, (1 << k) if k < n else 0) for k in range(m + n)]})
+    p = ll.ll_plan_convert(R, S, 2)
+    p.prepare()
+    src = torch.randint(-2 ** 15, 2 ** 15, (1 << (m + n),), dtype=torch.int16, device="cuda")
+    dst = torch.empty_like(src)
+    ms = time_fn(lambda: ll.ll_convert(src, dst, p))
+    gbs = 4 * (1 << (m + n)) / ms / 1e6
+    print(json.dumps({"case": "row-major -> mma swizzle (Def 4.11) 16384^2 bf16", "exec": p.describe()["exec"],
+                      "ms": round(ms, 4), "GBps": round(gbs, 1), "frac_6539": round(gbs / 6539.5, 3)}), flush=True)
+
+
 def next_rows():
     """§8(f) N1 pre-shuffle and N2 TMEM-fragment epilogue at scale; CTA-class transpose."""
+    swizzle_case()
     conv_case("N1 preshuffle W[16384,16384] bf16 -> mma rhs fragments", *W.n1_preshuffle(14, 14), 2)
     conv_case("N2 tmem 32x32b -> blocked, 8192 tiles 128x128 fp32", *W.n2_tmem_epilogue(13), 4)
     sa, sb = W.c5T(0, n=15)
