@@ -74,6 +74,14 @@ typedef enum {
   LL_CLASS_DEVICE = 5   /* mixes device bits: pack -> all-to-all -> unpack       */
 } ll_class;
 
+/* How a DEVICE plan moves data between GPUs.
+ *   COLLECTIVE: pack -> all-to-all (grouped ncclSend/ncclRecv) -> unpack.
+ *   PEER: one tile kernel per rank loads its src tiles and stores 16-byte vectors
+ *         straight into the receivers' dst windows (NVLink peer memory, CUDA IPC),
+ *         between two flag barriers; needs ll_comm_create_peers (or a loopback comm).
+ *   AUTO: PEER when the communicator has peer windows, else COLLECTIVE. */
+typedef enum { LL_EXCHANGE_AUTO = 0, LL_EXCHANGE_COLLECTIVE = 1, LL_EXCHANGE_PEER = 2 } ll_exchange;
+
 typedef struct ll_layout ll_layout;
 typedef struct ll_plan ll_plan;
 typedef struct ll_comm ll_comm;
@@ -92,6 +100,7 @@ typedef struct {
   int thread_bytes;     /* target bytes per thread (0 = default)                 */
   int generic;          /* 1 = force the runtime-generic kernel                   */
   ll_comm* comm;        /* required for DEVICE plans                              */
+  int exchange;         /* DEVICE plans: an ll_exchange (default AUTO)            */
 } ll_plan_opts;
 
 /* Fill *opts with defaults (force_class = -1, max_vec_bytes = 16, ...). */
@@ -279,6 +288,32 @@ ll_status ll_comm_get_unique_id(void* nccl_unique_id /* 128 bytes */);
 ll_status ll_comm_create_loopback(int nranks, ll_comm** comm);
 void ll_comm_destroy(ll_comm* comm);
 
+/* Peer-window communicator (§8(f) N4, LL_EXCHANGE_PEER).  Every rank owns a dst
+ * window (>= the local dst size; ll_convert's dst must be exactly this rank's
+ * window) and a zero-initialised flag buffer of LL_PEER_FLAG_BYTES; both are
+ * caller-owned device memory, shared with the other ranks through CUDA IPC
+ * (ll_ipc_export / ll_ipc_import) and mapped into this process.
+ *   dst_windows[q], flag_bufs[q]: rank q's buffers as addressed from this process
+ *   (this rank's own: its local pointers).  nranks <= LL_MAX_PEERS, power of two.
+ * Copied; the caller keeps the mappings alive until ll_comm_destroy.  ll_convert
+ * on such a plan is collective and stream-ordered: entry barrier, one tile kernel,
+ * exit barrier (flag barriers spin on the GPU; a peer that never arrives traps the
+ * kernel after 30 s instead of hanging). */
+#define LL_PEER_FLAG_BYTES 512
+#define LL_MAX_PEERS 64
+ll_status ll_comm_create_peers(int nranks, int rank, void* const* dst_windows, void* const* flag_bufs,
+                               size_t window_bytes, ll_comm** comm);
+
+/* CUDA IPC of caller-owned device allocations (any pointer inside a cudaMalloc'd
+ * block, e.g. a torch tensor): export writes LL_IPC_HANDLE_BYTES (the block's
+ * cudaIpcMemHandle_t plus the pointer's offset in it); import maps it in another
+ * process (one mapping per block, reference counted) and returns the pointer;
+ * close drops the reference. */
+#define LL_IPC_HANDLE_BYTES 72
+ll_status ll_ipc_export(const void* dev_ptr, void* handle);
+ll_status ll_ipc_import(const void* handle, void** dev_ptr);
+ll_status ll_ipc_close(void* dev_ptr);
+
 /* The stages of a DEVICE plan: pack (src -> send layout, receiver
  * rank bits on top) and unpack (recv layout, source rank bits on top -> dst); NULL
  * when a stage is the identity.  Every rank exchanges chunk_elems elements with
@@ -291,7 +326,9 @@ ll_status ll_plan_device_stages(const ll_plan* plan, ll_plan** pack, ll_plan** u
  * same tables the kernel is specialised with: load addresses, pre/post register
  * networks, shuffle rounds and source lanes, smem offsets).  For validating the
  * planner on machines without a GPU; never used by ll_convert.  src/dst are HOST
- * buffers.  LL_ERR_UNSUPPORTED for non-tile plans. */
+ * buffers.  DEVICE plans with the peer exchange simulate their fused tile plan on
+ * all ranks' slices back to back (the loopback buffer convention).
+ * LL_ERR_UNSUPPORTED for other non-tile plans. */
 ll_status ll_plan_simulate(const ll_plan* plan, const void* src, void* dst);
 
 /* ll_jit_precompile: NVRTC-compile the plan's kernel into the on-disk cubin cache

@@ -57,7 +57,7 @@ class _Dim(C.Structure):
 class _Opts(C.Structure):
     _fields_ = [("force_class", C.c_int), ("max_vec_bytes", C.c_int), ("sigma", C.c_int),
                 ("tile_bytes", C.c_int), ("thread_bytes", C.c_int), ("generic", C.c_int),
-                ("comm", C.c_void_p)]
+                ("comm", C.c_void_p), ("exchange", C.c_int)]
 
 
 _P = C.c_void_p
@@ -92,6 +92,10 @@ _sig = {
     "ll_comm_get_unique_id": [_P],
     "ll_comm_create_loopback": [C.c_int, _PP],
     "ll_plan_device_stages": [_P, _PP, _PP, C.POINTER(C.c_size_t), C.POINTER(C.c_int)],
+    "ll_comm_create_peers": [C.c_int, C.c_int, _PP, _PP, C.c_size_t, _PP],
+    "ll_ipc_export": [_P, _P],
+    "ll_ipc_import": [_P, _PP],
+    "ll_ipc_close": [_P],
     "ll_layout_blocked": [C.c_int] + [C.POINTER(C.c_int)] * 5 + [_PP],
     "ll_layout_mma_acc": [C.c_int, C.c_int, C.c_int, C.c_int, _PP],
     "ll_layout_mma_swizzle": [C.c_int] * 5 + [_PP],
@@ -134,7 +138,13 @@ def version() -> str:
     return _lib.ll_version().decode()
 
 
-def _opts(force_class=None, max_vec_bytes=16, sigma=0, tile_bytes=0, thread_bytes=0, generic=False, comm=None):
+EXCHANGES = ("auto", "collective", "peer")
+PEER_FLAG_BYTES = 512
+IPC_HANDLE_BYTES = 72
+
+
+def _opts(force_class=None, max_vec_bytes=16, sigma=0, tile_bytes=0, thread_bytes=0, generic=False, comm=None,
+          exchange="auto"):
     o = _Opts()
     _lib.ll_plan_opts_default(C.byref(o))
     if force_class is not None:
@@ -145,6 +155,7 @@ def _opts(force_class=None, max_vec_bytes=16, sigma=0, tile_bytes=0, thread_byte
     o.thread_bytes = thread_bytes
     o.generic = int(bool(generic))
     o.comm = comm.handle if comm is not None else None
+    o.exchange = EXCHANGES.index(exchange) if isinstance(exchange, str) else int(exchange)
     return o
 
 
@@ -453,11 +464,62 @@ class Comm:
         _check(_lib.ll_comm_create(uid, world, rank, C.byref(h)))
         return cls(h, world)
 
+    @classmethod
+    def peers(cls, dst_window, flags, group=None) -> "Comm":
+        """Peer-window communicator (LL_EXCHANGE_PEER, §8(f) N4).  dst_window: this
+        rank's dst buffer (CUDA tensor, the `dst` of every ll_convert on it); flags:
+        a zeroed CUDA tensor of >= PEER_FLAG_BYTES.  The other ranks' buffers are
+        mapped with CUDA IPC; the handles travel over the torch process group."""
+        import torch.distributed as dist
+        rank, world = dist.get_rank(group), dist.get_world_size(group)
+        if flags.numel() * flags.element_size() < PEER_FLAG_BYTES:
+            raise ValueError("flags must hold at least PEER_FLAG_BYTES")
+        hd, hf = ipc_export(dst_window), ipc_export(flags)
+        allh = [None] * world
+        dist.all_gather_object(allh, (hd, hf), group=group)
+        opened, dptr, fptr = [], [], []
+        for q in range(world):
+            if q == rank:
+                dptr.append(dst_window.data_ptr())
+                fptr.append(flags.data_ptr())
+            else:
+                d, f = ipc_import(allh[q][0]), ipc_import(allh[q][1])
+                opened += [d, f]
+                dptr.append(d)
+                fptr.append(f)
+        da = (C.c_void_p * world)(*dptr)
+        fa = (C.c_void_p * world)(*fptr)
+        h = C.c_void_p()
+        _check(_lib.ll_comm_create_peers(world, rank, da, fa, dst_window.numel() * dst_window.element_size(),
+                                         C.byref(h)))
+        c = cls(h, world)
+        c._opened, c._keep = opened, (dst_window, flags)
+        return c
+
     def __del__(self):
         h = getattr(self, "handle", None)
         if h and _lib is not None:
             _lib.ll_comm_destroy(h)
         self.handle = None
+        for ptr in getattr(self, "_opened", []):
+            if _lib is not None:
+                _lib.ll_ipc_close(C.c_void_p(ptr))
+        self._opened = []
+
+
+def ipc_export(t) -> bytes:
+    """CUDA IPC handle (IPC_HANDLE_BYTES) of a CUDA tensor's memory."""
+    buf = (C.c_char * IPC_HANDLE_BYTES)()
+    _check(_lib.ll_ipc_export(C.c_void_p(t.data_ptr()), buf))
+    return bytes(buf)
+
+
+def ipc_import(handle: bytes) -> int:
+    """Map another process's exported buffer; returns its device address here."""
+    buf = (C.c_char * IPC_HANDLE_BYTES).from_buffer_copy(handle)
+    p = C.c_void_p()
+    _check(_lib.ll_ipc_import(buf, C.byref(p)))
+    return p.value
 
 
 def ll_plan_convert(A: Layout, B: Layout, elem_bytes: int, **opts) -> Plan:

@@ -36,7 +36,7 @@ using namespace ll;
   }                                                               \
   return LL_OK;
 
-namespace {
+namespace ll {
 
 int num_sms() {
   static int sms = -1;
@@ -52,6 +52,9 @@ void check_cuda(cudaError_t e, const char* what) {
   if (e != cudaSuccess) fail(LL_ERR_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
 }
 
+}  // namespace ll
+
+namespace ll {
 // 8-byte elements are converted as pairs of 4-byte atoms: a new lowest input bit
 // maps to a new lowest logical bit (the product of the layout with a 1-bit identity,
 // Def 4.3).  Packed buffers are unchanged byte-wise.
@@ -89,14 +92,14 @@ Layout atomize(const Layout& L) {
   return R;
 }
 
-}  // namespace
+}  // namespace ll
 
 namespace ll {
 void ensure_tile_kernel(ConvPlan& P) {
   std::lock_guard<std::mutex> g(P.mu);
   if (P.kernel) return;
   if (P.source.empty()) P.source = codegen_tile(P);
-  P.kernel = jit_kernel(P.source, "ll_tile_kernel");
+  P.kernel = jit_kernel(P.source, P.peer_shift >= 0 ? "ll_tile_peer_kernel" : "ll_tile_kernel");
   if (P.smem_bytes > 48 * 1024)
     check_cuda(cudaFuncSetAttribute(P.kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, P.smem_bytes),
                "cudaFuncSetAttribute");
@@ -124,6 +127,10 @@ unsigned grid_for(u64 ntiles) {
 }
 
 }  // namespace
+
+namespace ll {
+unsigned grid_for_tiles(u64 ntiles) { return grid_for(ntiles); }
+}  // namespace ll
 
 namespace ll {
 ll_status convert_impl(const void* src, void* dst, void* ws, ConvPlan& P, cudaStream_t st) {
@@ -453,6 +460,7 @@ ll_status ll_plan_source(const ll_plan* p, char* buf, size_t cap, size_t* needed
   if (!p) fail(LL_ERR_INVALID_ARG, "null plan");
   std::string s;
   if (p->kind == 0 && p->cp().exec == EXEC_TILE) s = p->cp().source;
+  if (p->kind == 0 && p->cp().fused) s = p->cp().fused->source;
   if (p->kind == 1) s = codegen_gather(*p->gather);
   if (p->kind == 2) s = codegen_reduce(*p->reduce);
   if (needed) *needed = s.size() + 1;
@@ -470,6 +478,7 @@ ll_status ll_plan_prepare(ll_plan* p) {
   if (p->kind == 0 && p->cp().exec == EXEC_DEVICE) {
     if (p->cp().pack && p->cp().pack->exec == EXEC_TILE) ensure_tile_kernel(*p->cp().pack);
     if (p->cp().unpack && p->cp().unpack->exec == EXEC_TILE) ensure_tile_kernel(*p->cp().unpack);
+    if (p->cp().fused) ensure_tile_kernel(*p->cp().fused);
   }
   if (p->kind == 1) {
     ensure_gather_kernel(*p->gather);
@@ -490,6 +499,12 @@ ll_status ll_jit_precompile(const ll_plan* p) {
   LL_TRY
   if (!p) fail(LL_ERR_INVALID_ARG, "null plan");
   if (p->kind == 0 && p->cp().exec == EXEC_TILE) jit_precompile(p->cp().source, "ll_tile_kernel");
+  if (p->kind == 0 && p->cp().exec == EXEC_DEVICE) {
+    const ConvPlan& P = p->cp();
+    for (const ConvPlan* q : {P.pack.get(), P.unpack.get()})
+      if (q && q->exec == EXEC_TILE) jit_precompile(q->source, "ll_tile_kernel");
+    if (P.fused) jit_precompile(P.fused->source, "ll_tile_peer_kernel");
+  }
   if (p->kind == 1) jit_precompile(codegen_gather(*p->gather), "ll_gather_kernel");
   if (p->kind == 2) jit_precompile(codegen_reduce(*p->reduce), "ll_reduce_kernel");
   LL_CATCH
@@ -641,8 +656,10 @@ ll_status ll_plan_device_stages(const ll_plan* p, ll_plan** pack, ll_plan** unpa
 ll_status ll_plan_simulate(const ll_plan* p, const void* src, void* dst) {
   LL_TRY
   if (!p || p->kind != 0 || !src || !dst) fail(LL_ERR_INVALID_ARG, "bad argument");
-  if (p->cp().exec != EXEC_TILE) fail(LL_ERR_UNSUPPORTED, "simulate: only tile plans");
-  simulate_tile(p->cp(), static_cast<const uint8_t*>(src), static_cast<uint8_t*>(dst));
+  // peer-exchange DEVICE plans: the fused tile plan over all ranks' slices back to back
+  const ConvPlan& P = p->cp().fused ? *p->cp().fused : p->cp();
+  if (P.exec != EXEC_TILE) fail(LL_ERR_UNSUPPORTED, "simulate: only tile plans");
+  simulate_tile(P, static_cast<const uint8_t*>(src), static_cast<uint8_t*>(dst));
   LL_CATCH
 }
 

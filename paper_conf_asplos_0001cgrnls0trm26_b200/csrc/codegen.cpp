@@ -106,9 +106,19 @@ std::string codegen_tile(const ConvPlan& Pl) {
   o << icon("SV", T.sm_v) << arr("int", "VSLOT_LD", T.vec_slot_ld) << arr("int", "VSLOT_ST", T.vec_slot_st)
     << arr("u64", "SMOFF_LD", T.smoff_ld) << arr("u64", "SMOFF_ST", T.smoff_st);
   o << "};\n";
-  o << "extern \"C\" __global__ void __launch_bounds__(" << T.threads()
-    << ") ll_tile_kernel(const u8* __restrict__ src, u8* __restrict__ dst, u64 ntiles) {\n"
-    << "  ll_tile_body<P>(src, dst, ntiles);\n}\n";
+  if (Pl.peer_shift >= 0) {
+    // DEVICE plan executed as peer stores (N4): global dst offsets, window per rank
+    const int sh = Pl.peer_shift + lw;
+    o << "extern \"C\" __global__ void __launch_bounds__(" << T.threads()
+      << ") ll_tile_peer_kernel(const u8* __restrict__ src, const __grid_constant__ LLPeers peers, u64 ntiles,"
+         " u64 tile0) {\n"
+      << "  ll_tile_body<P, DstPeers<" << sh << ">, " << (Pl.peer_reg ? "true" : "false") << ">(src, DstPeers<" << sh
+      << ">(&peers), ntiles, tile0);\n}\n";
+  } else {
+    o << "extern \"C\" __global__ void __launch_bounds__(" << T.threads()
+      << ") ll_tile_kernel(const u8* __restrict__ src, u8* __restrict__ dst, u64 ntiles) {\n"
+      << "  ll_tile_body<P>(src, DstLocal(dst), ntiles);\n}\n";
+  }
   return o.str();
 }
 

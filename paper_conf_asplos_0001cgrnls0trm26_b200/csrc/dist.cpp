@@ -13,6 +13,8 @@
 
 #include <algorithm>
 #include <cstring>
+#include <map>
+#include <mutex>
 
 #include "ll_internal.hpp"
 
@@ -58,6 +60,38 @@ Nccl& nccl() {
   return n;
 }
 
+// CUDA IPC mappings opened in this process (one per exported block).
+struct IpcMap { void* base; int refs; };
+struct IpcRegistry {
+  std::mutex mu;
+  std::map<std::string, IpcMap> by_handle;
+  std::vector<std::pair<void*, std::string>> mapped;
+};
+IpcRegistry& ipc_registry() {
+  static IpcRegistry r;
+  return r;
+}
+
+// Base and size of the allocation containing p (driver cuMemGetAddressRange through
+// the runtime's entry-point table; the library links only cudart).
+cudaError_t mem_range(const void* p, void** base, size_t* size) {
+  typedef int (*Fn)(unsigned long long*, size_t*, unsigned long long);
+  static Fn fn = nullptr;
+  if (!fn) {
+    void* f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    cudaError_t e = cudaGetDriverEntryPoint("cuMemGetAddressRange", &f, cudaEnableDefault, &q);
+    if (e != cudaSuccess) return e;
+    if (!f || q != cudaDriverEntryPointSuccess) return cudaErrorNotSupported;
+    fn = reinterpret_cast<Fn>(f);
+  }
+  unsigned long long b = 0;
+  int r = fn(&b, size, reinterpret_cast<unsigned long long>(p));
+  if (r != 0) return cudaErrorInvalidValue;
+  *base = reinterpret_cast<void*>(b);
+  return cudaSuccess;
+}
+
 void check_nccl(int r, const char* what) {
   if (r != 0) fail(LL_ERR_NCCL, std::string(what) + ": " + (nccl().errstr ? nccl().errstr(r) : "error"));
 }
@@ -98,8 +132,85 @@ Layout memory_layout(const std::vector<u64>& cols, const std::vector<Dim>& out) 
 
 }  // namespace
 
+// §8(f) N4: the DEVICE map as ONE tile kernel per rank.  The pair (A, B) is planned
+// over the GLOBAL packed index space (local bits, then the dev bits on top: the
+// layouts read as memory layouts of 2^{d_in} elements), which gives an ordinary CTA
+// tile plan.  Push form: every tile's loads must be rank-local, so the src dev bits
+// are grid bits; they are moved to the top of the CTA index, and rank r runs the
+// 2^{G-p} tiles above r * 2^{G-p}.  Its stores land in the receivers' windows through
+// the global dst offset's top bits (DstPeers in ll_kernels.cuh): no pack, exchange
+// buffer or unpack pass, and the NVLink transfer overlaps the loads tile by tile.
+void plan_peer(ConvPlan& P, const ll_plan_opts* opts) {
+  const Layout &A = P.A, &B = P.B;
+  const int p = A.in_bits("dev");
+  const int nloc = A.d_in() - p;
+  if (A.in_pos("dev") != nloc || B.in_pos("dev") != B.d_in() - p)
+    fail(LL_ERR_UNSUPPORTED, "peer exchange: the dev dimension must be declared last");
+  ll_plan_opts lo;
+  std::memset(&lo, 0, sizeof lo);
+  lo.force_class = -1;
+  lo.max_vec_bytes = opts->max_vec_bytes ? opts->max_vec_bytes : 16;
+  lo.tile_bytes = opts->tile_bytes;
+  lo.thread_bytes = opts->thread_bytes;
+  // 8-byte elements move as pairs of 4-byte atoms (one more, lowest, local bit)
+  Layout Ag = memory_layout(A.cols, A.out), Bg = memory_layout(B.cols, B.out);
+  int wk = P.w, nl = nloc;
+  if (P.w == 8) { Ag = atomize(Ag); Bg = atomize(Bg); wk = 4; nl = nloc + 1; }
+  u64 devmask = 0;
+  for (int t = 0; t < p; ++t) devmask |= u64(1) << (nl + t);
+  auto F = plan_convert(Ag, Bg, wk, &lo, devmask);
+  if (F->exec != EXEC_TILE || !F->tile.ld_xcol.empty() || !F->tile.rep_bits.empty())
+    fail(LL_ERR_UNSUPPORTED, "peer exchange: the global map has no permutation tile plan");
+  TilePlan& T = F->tile;
+  for (int b : T.ld_bit)
+    if (b >= nl) fail(LL_ERR_UNSUPPORTED, "peer exchange: a src tile spans ranks (use the collective exchange)");
+  std::vector<int> gs, gd;
+  std::vector<std::pair<int, int>> hi;
+  for (size_t g = 0; g < T.grid_src_bit.size(); ++g) {
+    if (T.grid_src_bit[g] >= nl) hi.push_back({T.grid_src_bit[g], T.grid_dst_bit[g]});
+    else { gs.push_back(T.grid_src_bit[g]); gd.push_back(T.grid_dst_bit[g]); }
+  }
+  if (int(hi.size()) != p) fail(LL_ERR_UNSUPPORTED, "peer exchange: src dev bits are not grid bits (internal)");
+  std::sort(hi.begin(), hi.end());
+  for (auto& h : hi) { gs.push_back(h.first); gd.push_back(h.second); }
+  T.grid_src_bit = gs;
+  T.grid_dst_bit = gd;
+  F->peer_shift = nl;
+  F->peer_reg = false;
+  for (int b = 0; b < T.R; ++b)
+    if (T.st_bit[b] >= nl) F->peer_reg = true;
+  F->source = codegen_tile(*F);
+  P.rank_tiles = u64(1) << (gs.size() - p);
+  P.fused = std::move(F);
+  P.exchange = LL_EXCHANGE_PEER;
+  P.nranks = opts->comm->nranks;
+  P.comm = opts->comm;
+  P.local_elems = u64(1) << nloc;
+  P.chunk_elems = u64(1) << (nloc - p);
+  P.workspace_bytes = 0;
+  P.src_elems = P.dst_elems = P.local_elems;
+}
+
 void plan_device(ConvPlan& P, const ll_plan_opts* opts) {
   if (!opts || !opts->comm) fail(LL_ERR_INVALID_ARG, "DEVICE plans require opts->comm (the map mixes device bits)");
+  {
+    const int p = P.A.in_bits("dev");
+    if (P.B.in_bits("dev") != p || p == 0) fail(LL_ERR_UNSUPPORTED, "DEVICE: A and B need the same number of dev bits");
+    if (!P.A.unit_columns() || !P.B.unit_columns())
+      fail(LL_ERR_UNSUPPORTED, "DEVICE: only bijective permutation layouts are supported");
+    if (opts->comm->nranks != (1 << p)) fail(LL_ERR_INVALID_ARG, "DEVICE: communicator size != 2^(dev bits)");
+    const bool windows = !opts->comm->peer_dst.empty();
+    int ex = opts->exchange;
+    if (ex == LL_EXCHANGE_AUTO) ex = windows ? LL_EXCHANGE_PEER : LL_EXCHANGE_COLLECTIVE;
+    if (ex == LL_EXCHANGE_PEER) {
+      if (!windows && !opts->comm->loopback)
+        fail(LL_ERR_INVALID_ARG, "peer exchange needs a communicator with peer windows (ll_comm_create_peers)");
+      plan_peer(P, opts);
+      return;
+    }
+    if (!opts->comm->nccl && !opts->comm->loopback)
+      fail(LL_ERR_INVALID_ARG, "collective exchange needs an NCCL (or loopback) communicator");
+  }
   const Layout &A = P.A, &B = P.B;
   const int p = A.in_bits("dev");
   if (B.in_bits("dev") != p || p == 0) fail(LL_ERR_UNSUPPORTED, "DEVICE: A and B need the same number of dev bits");
@@ -133,8 +244,10 @@ void plan_device(ConvPlan& P, const ll_plan_opts* opts) {
   Layout A1, S1, R1, B1;
   relabel(Al, S, A1, S1);
   relabel(R, Bl, R1, B1);
-  auto pack = plan_convert(A1, S1, P.w, &lo);
-  auto unpack = plan_convert(R1, B1, P.w, &lo);
+  int wk = P.w;
+  if (P.w == 8) { A1 = atomize(A1); S1 = atomize(S1); R1 = atomize(R1); B1 = atomize(B1); wk = 4; }
+  auto pack = plan_convert(A1, S1, wk, &lo);
+  auto unpack = plan_convert(R1, B1, wk, &lo);
   P.pack = pack->exec == EXEC_NOOP ? nullptr : std::move(pack);
   P.unpack = unpack->exec == EXEC_NOOP ? nullptr : std::move(unpack);
   P.nranks = comm->nranks;
@@ -147,8 +260,51 @@ void plan_device(ConvPlan& P, const ll_plan_opts* opts) {
   P.src_elems = P.dst_elems = P.local_elems;
 }
 
+void ensure_tile_kernel(ConvPlan& P);
+unsigned grid_for_tiles(u64 ntiles);
+int launch_peer_barrier(void* const* flags, int nranks, int rank, unsigned epoch, cudaStream_t st);
+
+namespace {
+void launch_peer_tiles(ConvPlan& F, const void* src, const LLPeersHost& tab, u64 ntiles, u64 tile0, cudaStream_t st) {
+  unsigned long long nt = ntiles, t0 = tile0;
+  void* args[] = {const_cast<void**>(&src), const_cast<LLPeersHost*>(&tab), &nt, &t0};
+  check_cuda(cudaLaunchKernel(F.kernel, dim3(grid_for_tiles(ntiles)), dim3(F.tile.threads()), args,
+                              size_t(F.smem_bytes), st),
+             "cudaLaunchKernel(ll_tile_peer_kernel)");
+}
+}  // namespace
+
+ll_status peer_convert(ConvPlan& P, const void* src, void* dst, cudaStream_t st) {
+  ll_comm* comm = P.comm;
+  ConvPlan& F = *P.fused;
+  ensure_tile_kernel(F);
+  const size_t lb = size_t(P.local_elems) * P.w;
+  LLPeersHost tab;
+  std::memset(&tab, 0, sizeof tab);
+  if (comm->loopback) {
+    // virtual ranks in one buffer: the windows are the slices; one launch per rank
+    for (int q = 0; q < P.nranks; ++q) tab.dst[q] = static_cast<char*>(dst) + q * lb;
+    for (int r = 0; r < P.nranks; ++r)
+      launch_peer_tiles(F, static_cast<const char*>(src) + r * lb, tab, P.rank_tiles, u64(r) * P.rank_tiles, st);
+    return LL_OK;
+  }
+  if (dst != comm->peer_dst[comm->rank])
+    fail(LL_ERR_INVALID_ARG, "peer exchange: dst must be this rank's registered window");
+  if (comm->window_bytes < lb) fail(LL_ERR_INVALID_ARG, "peer exchange: window smaller than the local dst");
+  for (int q = 0; q < P.nranks; ++q) tab.dst[q] = static_cast<char*>(comm->peer_dst[q]);
+  // entry barrier: every receiver is done with its window's previous contents
+  int e = launch_peer_barrier(comm->peer_flags.data(), P.nranks, comm->rank, ++comm->epoch, st);
+  check_cuda(cudaError_t(e), "ll_peer_barrier_kernel");
+  launch_peer_tiles(F, src, tab, P.rank_tiles, u64(comm->rank) * P.rank_tiles, st);
+  // exit barrier: every sender's stores into this window have landed
+  e = launch_peer_barrier(comm->peer_flags.data(), P.nranks, comm->rank, ++comm->epoch, st);
+  check_cuda(cudaError_t(e), "ll_peer_barrier_kernel");
+  return LL_OK;
+}
+
 ll_status device_convert(const ConvPlan& Pc, const void* src, void* dst, void* ws, cudaStream_t st) {
   ConvPlan& P = const_cast<ConvPlan&>(Pc);
+  if (P.exchange == LL_EXCHANGE_PEER) return peer_convert(P, src, dst, st);
   ll_comm* comm = P.comm;
   const size_t lb = size_t(P.local_elems) * P.w, cb = size_t(P.chunk_elems) * P.w;
   if (P.workspace_bytes && !ws) fail(LL_ERR_INVALID_ARG, "DEVICE plan needs a workspace (ll_plan_workspace_bytes)");
@@ -220,6 +376,98 @@ ll_status ll_comm_create(const void* id, int nranks, int rank, ll_comm** out) {
     ll::set_last_error(e.what());
     return e.st;
   }
+}
+
+ll_status ll_comm_create_peers(int nranks, int rank, void* const* dst_windows, void* const* flag_bufs,
+                               size_t window_bytes, ll_comm** out) {
+  try {
+    if (!out || !dst_windows || !flag_bufs || nranks < 1 || nranks > LL_MAX_PEERS || (nranks & (nranks - 1)) ||
+        rank < 0 || rank >= nranks)
+      ll::fail(LL_ERR_INVALID_ARG, "peer communicator: bad nranks / rank / buffers");
+    auto c = std::make_unique<ll_comm>();
+    c->nranks = nranks;
+    c->rank = rank;
+    c->window_bytes = window_bytes;
+    for (int q = 0; q < nranks; ++q) {
+      if (!dst_windows[q] || !flag_bufs[q]) ll::fail(LL_ERR_INVALID_ARG, "peer communicator: null window");
+      if ((reinterpret_cast<uintptr_t>(dst_windows[q]) & 15) || (reinterpret_cast<uintptr_t>(flag_bufs[q]) & 15))
+        ll::fail(LL_ERR_MISALIGNED, "peer communicator: windows must be 16-byte aligned");
+      c->peer_dst.push_back(dst_windows[q]);
+      c->peer_flags.push_back(flag_bufs[q]);
+    }
+    *out = c.release();
+    return LL_OK;
+  } catch (const ll::Error& e) {
+    ll::set_last_error(e.what());
+    return e.st;
+  }
+}
+
+ll_status ll_ipc_export(const void* ptr, void* handle) {
+  try {
+    if (!ptr || !handle) ll::fail(LL_ERR_INVALID_ARG, "null argument");
+    void* base = nullptr;
+    size_t size = 0;
+    ll::check_cuda(ll::mem_range(ptr, &base, &size), "cuMemGetAddressRange");
+    cudaIpcMemHandle_t h;
+    ll::check_cuda(cudaIpcGetMemHandle(&h, base), "cudaIpcGetMemHandle");
+    uint64_t off = static_cast<const char*>(ptr) - static_cast<char*>(base);
+    std::memcpy(handle, &h, sizeof h);
+    std::memcpy(static_cast<char*>(handle) + 64, &off, 8);
+    return LL_OK;
+  } catch (const ll::Error& e) {
+    ll::set_last_error(e.what());
+    return e.st;
+  }
+}
+
+ll_status ll_ipc_import(const void* handle, void** ptr) {
+  try {
+    if (!handle || !ptr) ll::fail(LL_ERR_INVALID_ARG, "null argument");
+    std::string key(static_cast<const char*>(handle), 64);
+    uint64_t off;
+    std::memcpy(&off, static_cast<const char*>(handle) + 64, 8);
+    auto& reg = ll::ipc_registry();
+    std::lock_guard<std::mutex> g(reg.mu);
+    auto it = reg.by_handle.find(key);
+    if (it == reg.by_handle.end()) {
+      cudaIpcMemHandle_t h;
+      std::memcpy(&h, handle, sizeof h);
+      void* base = nullptr;
+      ll::check_cuda(cudaIpcOpenMemHandle(&base, h, cudaIpcMemLazyEnablePeerAccess), "cudaIpcOpenMemHandle");
+      it = reg.by_handle.emplace(key, ll::IpcMap{base, 0}).first;
+    }
+    it->second.refs += 1;
+    *ptr = static_cast<char*>(it->second.base) + off;
+    reg.mapped.push_back({*ptr, key});
+    return LL_OK;
+  } catch (const ll::Error& e) {
+    ll::set_last_error(e.what());
+    return e.st;
+  }
+}
+
+ll_status ll_ipc_close(void* ptr) {
+  try {
+    auto& reg = ll::ipc_registry();
+    std::lock_guard<std::mutex> g(reg.mu);
+    for (size_t i = 0; i < reg.mapped.size(); ++i) {
+      if (reg.mapped[i].first != ptr) continue;
+      auto it = reg.by_handle.find(reg.mapped[i].second);
+      reg.mapped.erase(reg.mapped.begin() + i);
+      if (it != reg.by_handle.end() && --it->second.refs == 0) {
+        cudaError_t e = cudaIpcCloseMemHandle(it->second.base);
+        reg.by_handle.erase(it);
+        ll::check_cuda(e, "cudaIpcCloseMemHandle");
+      }
+      return LL_OK;
+    }
+    ll::fail(LL_ERR_INVALID_ARG, "ll_ipc_close: pointer was not imported");
+  } catch (const ll::Error& e) {
+    ll::set_last_error(e.what());
+    return e.st;
+  }
+  return LL_OK;
 }
 
 ll_status ll_comm_create_loopback(int nranks, ll_comm** out) {

@@ -50,4 +50,39 @@ int launch_generic(const void* src, void* dst, const unsigned long long* cols, i
   return int(cudaGetLastError());
 }
 
+// Flag barrier of the peer exchange (§8(f) N4).  flags[q] is rank q's flag buffer as
+// mapped here; slot s of it holds the last epoch rank s announced to q.  Thread q
+// announces `epoch` to rank q (release, system scope: the preceding kernel's peer
+// stores are ordered before it) and waits until rank q announced it here (acquire).
+// Epochs grow by one per barrier on every rank, so a peer can be at most one epoch
+// ahead.  A rank that never arrives traps the kernel after 30 s (no GPU hang).
+struct PeerFlags { unsigned* f[64]; };
+
+__global__ void ll_peer_barrier_kernel(PeerFlags flags, int nranks, int rank, unsigned epoch) {
+  const int q = threadIdx.x;
+  if (q < nranks) {
+    asm volatile("fence.acq_rel.sys;" ::: "memory");
+    asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(flags.f[q] + rank), "r"(epoch) : "memory");
+    const unsigned* mine = flags.f[rank] + q;
+    unsigned long long t0, t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+    while (true) {
+      unsigned v;
+      asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(mine) : "memory");
+      if (int(v - epoch) >= 0) break;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+      if (t - t0 > 30000000000ull) __trap();
+      __nanosleep(256);
+    }
+  }
+  __syncthreads();
+}
+
+int launch_peer_barrier(void* const* flags, int nranks, int rank, unsigned epoch, cudaStream_t st) {
+  PeerFlags f;
+  for (int i = 0; i < 64; ++i) f.f[i] = i < nranks ? static_cast<unsigned*>(flags[i]) : nullptr;
+  ll_peer_barrier_kernel<<<1, 64, 0, st>>>(f, nranks, rank, epoch);
+  return int(cudaGetLastError());
+}
+
 }  // namespace ll

@@ -12,6 +12,9 @@
 //   jit     — NVRTC compilation + cubin cache + cudaLibrary loading
 //   capi    — the C ABI of include/ll.h
 #pragma once
+#include <cuda_runtime.h>
+
+#include <atomic>
 #include <cstdint>
 #include <map>
 #include <memory>
@@ -193,6 +196,14 @@ struct ConvPlan {
   u64 chunk_elems = 0;                      // elements exchanged with every peer
   int nranks = 1;
   u64 local_elems = 0;
+  // DEVICE plans executed as peer stores (§8(f) N4): `fused` is one tile plan over the
+  // global packed index space whose grid bits carrying the src dev bits come last;
+  // rank r runs tiles [0, rank_tiles) with tile0 = r * rank_tiles.
+  int exchange = 0;                         // LL_EXCHANGE_COLLECTIVE / LL_EXCHANGE_PEER
+  std::unique_ptr<ConvPlan> fused;
+  u64 rank_tiles = 0;
+  int peer_shift = -1;    // >= 0: this tile plan is a peer kernel; log2 local elements
+  bool peer_reg = false;  // a dst register / replica bit crosses ranks
   std::string source;   // specialised kernel source (EXEC_TILE)
   std::string kernel_key;
   void* kernel = nullptr;   // cudaKernel_t once loaded
@@ -200,7 +211,13 @@ struct ConvPlan {
   std::mutex mu;
 };
 
-std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, const ll_plan_opts* opts);
+std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, const ll_plan_opts* opts,
+                                       u64 grid_only_src = 0);
+Layout atomize(const Layout& L);   // 8-byte elements as pairs of 4-byte atoms (capi.cpp)
+int num_sms();
+void check_cuda(cudaError_t e, const char* what);
+// host mirror of LLPeers (ll_kernels.cuh): kernel parameter of the peer tile kernel
+struct LLPeersHost { void* dst[64]; };
 std::string describe(const ConvPlan& P);
 
 struct GatherPlan {
@@ -282,4 +299,9 @@ struct ll_comm {
   int nranks = 1, rank = 0;
   bool loopback = false;   // all ranks' slices in one process (tests); memcpy exchange
   void* nccl = nullptr;    // ncclComm_t
+  // peer windows (N4): every rank's dst window and barrier-flag buffer, mapped into
+  // this process (CUDA IPC over NVLink); empty unless created by ll_comm_create_peers
+  std::vector<void*> peer_dst, peer_flags;
+  size_t window_bytes = 0;
+  std::atomic<unsigned> epoch{0};
 };

@@ -370,8 +370,34 @@ __device__ __forceinline__ void xchg_smem(const u32 (&r)[P::NW], u32 (&o)[P::NW]
 }
 
 // ------------------------------------------------------------------ tile kernel
-template <class P>
-__device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, u8* __restrict__ dst, u64 ntiles) {
+// Destination addressing of the tile kernel.  DstLocal: one buffer.  DstPeers (row
+// a9 DEVICE plans executed as peer stores, §8(f) N4): the dst offset is an offset in
+// the GLOBAL packed index space (local bits, then the dev bits on top); its top bits
+// select the receiving rank's window (NVLink peer memory mapped into this process).
+struct DstLocal {
+  u8* base;
+  __device__ __forceinline__ explicit DstLocal(u8* b) : base(b) {}
+  __device__ __forceinline__ u8* at(u64 off) const { return base + off; }
+};
+#ifndef LL_MAX_PEERS
+#define LL_MAX_PEERS 64
+#endif
+struct LLPeers {
+  u8* dst[LL_MAX_PEERS];
+};
+template <int SHIFT>
+struct DstPeers {
+  const LLPeers* p;
+  __device__ __forceinline__ explicit DstPeers(const LLPeers* q) : p(q) {}
+  __device__ __forceinline__ u8* at(u64 off) const {
+    return p->dst[off >> SHIFT] + (off & ((u64(1) << SHIFT) - 1));
+  }
+};
+
+// PEER_REG: some register / replica bit of the dst tile crosses ranks, so every
+// store picks its window; otherwise one window per thread and tile.
+template <class P, class Dst, bool PEER_REG = false>
+__device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, Dst D, u64 ntiles, u64 tile0 = 0) {
   extern __shared__ __align__(16) u8 ll_smem[];
   const u32 lane = threadIdx.x & 31u;
   const u32 warp = threadIdx.x >> 5;
@@ -389,12 +415,13 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, u8* __r
       __syncthreads();
       static_for<P::NW>([&](auto q) { r[decltype(q)::value] = o[decltype(q)::value] + 1u; });
     }
-    if (r[0] == 0x9e3779b9u) dst[threadIdx.x] = u8(r[P::NW - 1]);
+    if (r[0] == 0x9e3779b9u) *D.at(threadIdx.x) = u8(r[P::NW - 1]);
     return;
   }
   for (u64 t = blockIdx.x; t < ntiles; t += gridDim.x) {
     const u8* s = src + (tile_base<P, true>(t) ^ ld_thr);
-    u8* d = dst + (tile_base<P, false>(t) ^ st_thr);
+    const u64 doff = tile_base<P, false>(t | tile0) ^ st_thr;
+    u8* d = D.at(doff);
     u32 r[P::NW];
     // a5: HBM load of the src tile (16-byte vectors; coalesced under σ_ld)
     static_for<(1 << (P::R - P::VLD))>([&](auto k) {
@@ -418,7 +445,10 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, u8* __r
       constexpr u64 RO = P::REP_OFF[decltype(rp)::value];
       static_for<(1 << (P::R - P::VST))>([&](auto k) {
         constexpr int K = decltype(k)::value;
-        store_vec<P::W, P::VST, K, P::NW, P::ST_HINT>(o, d + (StOff<P, K>::value() ^ RO));
+        if constexpr (PEER_REG)
+          store_vec<P::W, P::VST, K, P::NW, P::ST_HINT>(o, D.at(doff + (StOff<P, K>::value() ^ RO)));
+        else
+          store_vec<P::W, P::VST, K, P::NW, P::ST_HINT>(o, d + (StOff<P, K>::value() ^ RO));
       });
     });
     if constexpr (P::XCHG == 3) __syncthreads();   // smem reuse by the next tile

@@ -490,7 +490,7 @@ static void plan_smem(TilePlan& T, int maxvec) {
 // ---------------------------------------------------------------------------
 static void build_tile(ConvPlan& P, const std::vector<int>& S0, const std::vector<int>& D0,
                        std::vector<int> gridS, std::vector<int> gridD, const ll_plan_opts* opts,
-                       bool in_cta) {
+                       bool in_cta, u64 grid_only_src = 0) {
   const Layout &A = P.A, &B = P.B;
   TilePlan& T = P.tile;
   T = TilePlan();
@@ -501,10 +501,13 @@ static void build_tile(ConvPlan& P, const std::vector<int>& S0, const std::vecto
   std::vector<int> S = S0, D = D0;
   // fold low grid bits into the tile while it is small (common vectors)
   std::vector<int> foldS, foldD;
-  while (!gridD.empty() && (u64(1) << S.size()) * u64(P.w) < u64(tile_bytes) && S.size() < 20) {
-    foldS.push_back(gridS.front()); foldD.push_back(gridD.front());
-    S.push_back(gridS.front()); D.push_back(gridD.front());
-    gridS.erase(gridS.begin()); gridD.erase(gridD.begin());
+  while ((u64(1) << S.size()) * u64(P.w) < u64(tile_bytes) && S.size() < 20) {
+    size_t g = 0;
+    while (g < gridS.size() && ((grid_only_src >> gridS[g]) & 1)) ++g;
+    if (g == gridS.size()) break;
+    foldS.push_back(gridS[g]); foldD.push_back(gridD[g]);
+    S.push_back(gridS[g]); D.push_back(gridD[g]);
+    gridS.erase(gridS.begin() + g); gridD.erase(gridD.begin() + g);
   }
   std::vector<int> Ss = S, Ds = D;
   std::sort(Ss.begin(), Ss.end());
@@ -555,16 +558,22 @@ static void build_tile(ConvPlan& P, const std::vector<int>& S0, const std::vecto
 
 // CTA class (Q mixes block/offset bits): choose the dst bits a CTA owns so that both
 // the loads and the stores are coalesced.
+// grid_only_src: src bits that must stay CTA-index bits (the src dev bits of a peer
+// exchange, whose tiles must load from one rank).
 static void choose_cta_tile(const std::vector<int>& pi, int nloc, int c_bits,
                             int target_bits, std::vector<int>& S, std::vector<int>& D,
-                            std::vector<int>& gS, std::vector<int>& gD) {
+                            std::vector<int>& gS, std::vector<int>& gD, u64 grid_only_src = 0) {
   std::vector<int> inv(nloc, -1);
   for (int k = 0; k < nloc; ++k) inv[pi[k]] = k;
   std::vector<char> inT(nloc, 0);
-  for (int k = 0; k < std::min(c_bits, nloc); ++k) { inT[k] = 1; inT[inv[k]] = 1; }
+  auto ok = [&](int d) { return !((grid_only_src >> pi[d]) & 1); };
+  for (int k = 0; k < std::min(c_bits, nloc); ++k) {
+    if (ok(k)) inT[k] = 1;
+    if (ok(inv[k])) inT[inv[k]] = 1;
+  }
   int cnt = 0;
   for (int k = 0; k < nloc; ++k) cnt += inT[k];
-  for (int k = 0; k < nloc && cnt < target_bits; ++k) if (!inT[k]) { inT[k] = 1; ++cnt; }
+  for (int k = 0; k < nloc && cnt < target_bits; ++k) if (!inT[k] && ok(k)) { inT[k] = 1; ++cnt; }
   S.clear(); D.clear(); gS.clear(); gD.clear();
   for (int k = 0; k < nloc; ++k) {
     if (inT[k]) { D.push_back(k); S.push_back(pi[k]); }
@@ -572,7 +581,8 @@ static void choose_cta_tile(const std::vector<int>& pi, int nloc, int c_bits,
   }
 }
 
-std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, const ll_plan_opts* opts) {
+std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, const ll_plan_opts* opts,
+                                       u64 grid_only_src) {
   if (w != 1 && w != 2 && w != 4 && w != 8) fail(LL_ERR_INVALID_ARG, "elem_bytes must be 1, 2, 4 or 8");
   if (A.out != B.out) fail(LL_ERR_DIM_MISMATCH, "A and B must have the same output dims");
   for (auto* L : {&A, &B}) {
@@ -611,7 +621,7 @@ std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, 
     if (perm) {
       try {
         std::vector<int> S, D, gS, gD;
-        if (lev <= 2) {
+        if (lev <= 2 && !grid_only_src) {
           D = bits_at_level(B, 0, 2);
           for (int k : D) S.push_back(pi[k]);
           for (int k : bits_at_level(B, 3, 3)) { gD.push_back(k); gS.push_back(pi[k]); }
@@ -625,10 +635,10 @@ std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, 
           // 64 KiB of smem: 512-byte runs, else 256, else 128 (one line)
           const int max_bits = ilog2(u64(65536 / w));
           for (int c_bits = v + 5; c_bits >= v + 3; --c_bits) {
-            choose_cta_tile(pi, nB, c_bits, target, S, D, gS, gD);
+            choose_cta_tile(pi, nB, c_bits, target, S, D, gS, gD, grid_only_src);
             if (int(S.size()) <= max_bits) break;
           }
-          build_tile(*P, S, D, gS, gD, opts, false);
+          build_tile(*P, S, D, gS, gD, opts, false, grid_only_src);
         }
         P->exec = EXEC_TILE;
         return P;
@@ -785,7 +795,11 @@ std::string describe(const ConvPlan& P) {
     o << "}";
   }
   if (P.exec == EXEC_DEVICE) {
-    o << ",\"dev_bits\":" << P.dev_bits << ",\"workspace_bytes\":" << P.workspace_bytes;
+    o << ",\"dev_bits\":" << P.dev_bits << ",\"workspace_bytes\":" << P.workspace_bytes
+      << ",\"exchange\":\"" << (P.exchange == LL_EXCHANGE_PEER ? "peer" : "collective") << "\"";
+    if (P.fused)
+      o << ",\"rank_tiles\":" << P.rank_tiles << ",\"peer_reg\":" << (P.fused->peer_reg ? "true" : "false")
+        << ",\"fused\":" << describe(*P.fused);
     if (P.pack) o << ",\"pack\":" << describe(*P.pack);
     if (P.unpack) o << ",\"unpack\":" << describe(*P.unpack);
   }

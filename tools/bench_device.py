@@ -4,6 +4,7 @@ grouped ncclSend/ncclRecv all-to-all over NVLink -> unpack (identity here).
 
     torchrun --nproc-per-node P --master-addr 127.0.0.1 tools/bench_device.py [--n 15]
     python tools/bench_device.py --loopback 8      # one GPU, P virtual ranks (memcpy exchange)
+    python tools/bench_device.py --loopback 8 --exchange peer   # one GPU, fused peer-store kernel
 
 Prints one JSON line: aggregate GB/s (2 x tensor bytes / time, max over ranks), the
 per-GPU NVLink bytes and their fraction of 900 GB/s per direction (nominal) and of the
@@ -28,6 +29,9 @@ def main():
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--loopback", type=int, default=0)
+    ap.add_argument("--exchange", default="collective", choices=["collective", "peer"],
+                    help="collective: pack -> all-to-all -> unpack; peer: one tile kernel storing into "
+                         "the receivers' windows (CUDA IPC over NVLink), §8(f) N4")
     args = ap.parse_args()
     rank, world = int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1))
     local = int(os.environ.get("LOCAL_RANK", 0))
@@ -40,19 +44,22 @@ def main():
         if world > 1:
             import torch.distributed as dist
             dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-            comm = ll.Comm.from_process_group()
+            comm = None if args.exchange == "peer" else ll.Comm.from_process_group()
         else:
             comm = None
     p = P.bit_length() - 1
-    sa, sb = W.c5(p, n=args.n)
-    A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
-    plan = ll.ll_plan_convert(A, B, 2, comm=comm) if p else ll.ll_plan_convert(A, B, 2)
-    plan.prepare()
     total = 1 << (2 * args.n)
     local_elems = total // P
     slices = P if args.loopback else 1
     src = torch.randint(-2 ** 15, 2 ** 15, (local_elems * slices,), dtype=torch.int16, device="cuda")
     dst = torch.empty_like(src)
+    if args.exchange == "peer" and not args.loopback and world > 1:
+        flags = torch.zeros(ll.PEER_FLAG_BYTES // 4, dtype=torch.int32, device="cuda")
+        comm = ll.Comm.peers(dst, flags)
+    sa, sb = W.c5(p, n=args.n)
+    A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
+    plan = ll.ll_plan_convert(A, B, 2, comm=comm, exchange=args.exchange) if p else ll.ll_plan_convert(A, B, 2)
+    plan.prepare()
     ws = torch.empty(max(16, plan.workspace_bytes()), dtype=torch.uint8, device="cuda")
     for _ in range(args.warmup):
         ll.ll_convert(src, dst, plan, workspace=ws)
@@ -76,7 +83,7 @@ def main():
         print(json.dumps({
             "workload": f"config 5: [{1 << args.n},{1 << args.n}] bf16 row-sharded -> column-sharded, P={P}"
                         + (" (loopback)" if args.loopback else ""),
-            "class": d["class"], "exec": d["exec"], "ms_per_step": round(ms, 4),
+            "class": d["class"], "exec": d["exec"], "exchange": d.get("exchange"), "ms_per_step": round(ms, 4),
             "value_GBps": round(2 * total * 2 / (ms / 1e3) / 1e9, 1),
             "nvlink_bytes_per_gpu_each_way": int(nvl),
             "nvlink_GBps_per_gpu": round(nvl / (ms / 1e3) / 1e9, 1) if P > 1 else None,
