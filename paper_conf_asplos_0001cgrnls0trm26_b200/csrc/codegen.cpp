@@ -74,6 +74,7 @@ std::string codegen_tile(const ConvPlan& Pl) {
     stc.push_back(u64(1) << (T.st_bit[b] + lw));
   }
   o << arr("u64", "LD_COL", ldc) << arr("u64", "ST_COL", stc);
+  o << "  static constexpr bool LD_XOR = " << (T.ld_xcol.empty() ? "false" : "true") << ";\n";
   if (T.grid_src_xcol.empty()) {
     emit_grid(o, T.grid_src_bit, T.grid_dst_bit, lw);
   } else {

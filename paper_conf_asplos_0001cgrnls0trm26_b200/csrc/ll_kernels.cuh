@@ -419,14 +419,20 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, Dst D, 
     return;
   }
   for (u64 t = blockIdx.x; t < ntiles; t += gridDim.x) {
-    const u8* s = src + (tile_base<P, true>(t) ^ ld_thr);
+    const u64 sofs = tile_base<P, true>(t) ^ ld_thr;
+    const u8* s = src + sofs;
     const u64 doff = tile_base<P, false>(t | tile0) ^ st_thr;
     u8* d = D.at(doff);
     u32 r[P::NW];
     // a5: HBM load of the src tile (16-byte vectors; coalesced under σ_ld)
     static_for<(1 << (P::R - P::VLD))>([&](auto k) {
       constexpr int K = decltype(k)::value;
-      load_vec<P::W, P::VLD, K, P::NW, P::LD_L1>(r, s + LdOff<P, K>::value());
+      // XOR-copy plans (non-permutation Q): register and thread offsets share bits,
+      // so they combine by XOR; permutation plans' bits are disjoint (immediate add)
+      if constexpr (P::LD_XOR)
+        load_vec<P::W, P::VLD, K, P::NW, P::LD_L1>(r, src + (sofs ^ LdOff<P, K>::value()));
+      else
+        load_vec<P::W, P::VLD, K, P::NW, P::LD_L1>(r, s + LdOff<P, K>::value());
     });
     u32 o[P::NW];
     if constexpr (P::XCHG == 0) {

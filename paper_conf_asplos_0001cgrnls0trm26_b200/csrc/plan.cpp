@@ -695,8 +695,16 @@ std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, 
   // kept for maps that scatter the low bits.
   if (!generic && lev <= 3 && nB >= 5) {
     int vmax = std::max(0, ilog2(u64(std::max(1, default_int(opts, &ll_plan_opts::max_vec_bytes, 16) / w))));
+    // vector bits: dst bits [0, v) map to src bits [0, v), and no other column reaches
+    // below bit v, so each vector's 2^v elements are contiguous and aligned in src
     int v = 0;
     while (v < vmax && v < nB && P->Q[v] == (u64(1) << v)) ++v;
+    for (;;) {
+      bool clean = true;
+      for (int k = v; k < nB; ++k) if (P->Q[k] & ((u64(1) << v) - 1)) clean = false;
+      if (clean || v == 0) break;
+      --v;
+    }
     // the low lane bits must keep whole 32-byte sectors together: Q maps dst bits [v, v+2)
     // to src bits of single weight
     bool rowlocal = true;

@@ -9,22 +9,27 @@
 
 namespace ll {
 
+namespace {
+struct struct_off { u64 thr, reg, elem; };
+}  // namespace
+
 void simulate_tile(const ConvPlan& P, const uint8_t* src, uint8_t* dst) {
   if (P.exec != EXEC_TILE) fail(LL_ERR_UNSUPPORTED, "simulate: not a tile plan");
   const TilePlan& T = P.tile;
   const int w = T.w, R = T.R, n = T.n;
   const int E = 1 << R, NT = T.threads();
   const u64 ntiles = u64(1) << T.grid_dst_bit.size();
-  auto off = [&](const std::vector<int>& bits, u64 hw) {
-    u64 o = 0;
-    for (int b = 0; b < n; ++b) if ((hw >> b) & 1) o |= u64(1) << bits[b];
-    return o;
-  };
+  // Address arithmetic exactly as ll_tile_body forms it: thread part (lane / warp
+  // columns) XOR the tile base; the register part of vector K (bits >= vld) added —
+  // or XORed for XOR-copy plans (LD_XOR) — and element i of the vector at +i.
+  const bool ld_xor = !T.ld_xcol.empty();
+  auto ld_col = [&](int b) { return ld_xor ? T.ld_xcol[b] : (u64(1) << T.ld_bit[b]); };
   auto ld_off = [&](u64 hw) {
-    if (T.ld_xcol.empty()) return off(T.ld_bit, hw);
-    u64 o = 0;
-    for (int b = 0; b < n; ++b) if ((hw >> b) & 1) o ^= T.ld_xcol[b];
-    return o;
+    const u64 vmask = (u64(1) << T.vld) - 1;
+    u64 thr = 0, reg = 0;
+    for (int b = R; b < n; ++b) if ((hw >> b) & 1) thr ^= ld_col(b);
+    for (int b = T.vld; b < R; ++b) if ((hw >> b) & 1) reg ^= ld_col(b);
+    return struct_off{thr, reg, hw & vmask};
   };
   std::vector<uint64_t> in(size_t(NT) * E), out(size_t(NT) * E);
   std::vector<uint8_t> smem(T.xchg == X_SMEM ? T.smem_elems * w : 0);
@@ -39,7 +44,10 @@ void simulate_tile(const ConvPlan& P, const uint8_t* src, uint8_t* dst) {
     for (int th = 0; th < NT; ++th)
       for (int e = 0; e < E; ++e) {
         u64 hw = u64(e) | (u64(th) << R);
-        in[size_t(th) * E + e] = getv(src + (sb ^ ld_off(hw)) * w);
+        struct_off a = ld_off(hw);
+        u64 base = sb ^ a.thr;
+        u64 idx = (ld_xor ? (base ^ a.reg) : (base + a.reg)) + a.elem;
+        in[size_t(th) * E + e] = getv(src + idx * w);
       }
     if (T.xchg == X_COPY) {
       out = in;
@@ -104,7 +112,12 @@ void simulate_tile(const ConvPlan& P, const uint8_t* src, uint8_t* dst) {
       for (int th = 0; th < NT; ++th)
         for (int e = 0; e < E; ++e) {
           u64 hw = u64(e) | (u64(th) << R);
-          std::memcpy(dst + (db | off(T.st_bit, hw) | ro) * w, &out[size_t(th) * E + e], w);
+          const u64 vmask = (u64(1) << T.vst) - 1;
+          u64 thr = 0, reg = 0;
+          for (int b = R; b < n; ++b) if ((hw >> b) & 1) thr ^= u64(1) << T.st_bit[b];
+          for (int b = T.vst; b < R; ++b) if ((hw >> b) & 1) reg ^= u64(1) << T.st_bit[b];
+          u64 idx = (db ^ thr) + (reg ^ ro) + (hw & vmask);
+          std::memcpy(dst + idx * w, &out[size_t(th) * E + e], w);
         }
     }
   }

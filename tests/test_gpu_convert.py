@@ -490,3 +490,30 @@ def test_swizzled_memory_layout_gpu():
     j = np.arange(1 << n)[None, :]
     off = (i << n) + ((((i // 1) % 8) ^ (j // 8)) * 8 ^ (j % 8))
     assert np.array_equal(got[off.reshape(-1)], T)
+
+
+@pytest.mark.gpu
+def test_e1_exhaustive_generic_gpu():
+    """E1 on the GPU, exhaustive: all 8! = 40320 bijective relabelings B
+    of Fig. 1's 2^8 space against Fig. 1 A, each executed by the runtime-generic
+    kernel (XOR-of-columns pull map) into its own slice of one device buffer, then
+    compared in one go with the oracle's pack_B(T)."""
+    import itertools
+    import torch
+    A, OA = both(W.C1_A)
+    T = gen.random_bits(np.random.default_rng(1001), 256, 4)
+    d_src = to_device(O.pack(OA, T))
+    unit = [1 << t for t in range(8)]
+    perms = list(itertools.permutations(range(8)))
+    d_dst = torch.empty((len(perms), 256), dtype=torch.int32, device="cuda")
+    want = np.empty((len(perms), 256), dtype=np.uint32)
+    for case, perm in enumerate(perms):
+        OB = O.layout_from_cols(OA.in_dims, OA.out_dims, [unit[p] for p in perm])
+        B = ll.Layout(OB.in_dims, OB.out_dims, OB.bases)
+        plan = ll.ll_plan_convert(A, B, 4, generic=True)
+        ll.ll_convert(d_src, d_dst[case], plan)
+        want[case] = O.pack(OB, T)
+    torch.cuda.synchronize()
+    got = d_dst.cpu().numpy().view(np.uint32)
+    bad = np.nonzero(~np.all(got == want, axis=1))[0]
+    assert bad.size == 0, [perms[i] for i in bad[:5]]

@@ -463,3 +463,30 @@ def test_swizzled_memory_layout_xor_copy(vec, pp, mp):
     for i in range(0, 64, 5):
         for j in range(0, 64, 3):
             assert got[(i << n) + O.mma_swizzle_offset(i, j, vec, pp, mp)] == T[(i << n) + j]
+
+
+@pytest.mark.parametrize("w", [1, 2, 4, 8])
+def test_random_memory_layouts_xor_copy_simulated(w):
+    """R2 random memory layouts (Def 4.14: 1- or 2-bit columns) <-> row-major, d = 5..10:
+    every XOR-copy tile plan's emulated schedule — with the kernel's own address
+    arithmetic (thread part XOR tile base, register part XOR, vector element +i) —
+    equals the oracle.  (A vector whose start another column reaches below bit v would
+    be misaligned: the planner narrows v.)"""
+    tiles = 0
+    for d in range(5, 11):
+        for seed in range(12):
+            rng = np.random.default_rng(seed * 7 + d + 1000 * w)
+            out = [("x", d)]
+            OA = O.Layout([("offset", d)], out, {"offset": [[1 << k] for k in range(d)]})
+            OB = O.layout_from_cols([("offset", d)], out, gen.random_memory_cols(rng, d))
+            A = ll.Layout(OA.in_dims, OA.out_dims, OA.bases)
+            B = ll.Layout(OB.in_dims, OB.out_dims, OB.bases)
+            T = gen.random_bits(rng, 1 << d, w)
+            for A_, B_, OA_, OB_ in ((A, B, OA, OB), (B, A, OB, OA)):
+                p = ll.ll_plan_convert(A_, B_, w)
+                if p.describe()["exec"] != "tile":
+                    continue
+                tiles += 1
+                s = O.pack(OA_, T)
+                assert np.array_equal(p.simulate(s, 1 << d), O.convert(OA_, OB_, s)), (d, seed)
+    assert tiles >= 40
