@@ -159,6 +159,111 @@ def run_reference(args):
     print(json.dumps(line), flush=True)
 
 
+def _time_stream(fn, torch, samples=10, batch=20, warmup=3):
+    """Median over `samples` of the time per call of `batch` back-to-back calls (CUDA
+    events on the current stream); small kernels are measured as a stream."""
+    for _ in range(warmup):
+        fn()
+    torch.cuda.synchronize()
+    ts = []
+    for _ in range(samples):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        for _ in range(batch):
+            fn()
+        b.record()
+        b.synchronize()
+        ts.append(a.elapsed_time(b) / batch)
+    ts.sort()
+    return ts[len(ts) // 2]
+
+
+def other_configs(ll, W, torch, peak):
+    """The other BASELINE configs (1, 3, 4, 5) measured live on this GPU, each against
+    the same copy roofline: GB/s = algorithmic bytes / median time per call.  Inputs
+    larger than L2, or 4 rotated buffer sets for config 4 (192 / 64.5 MiB per set)."""
+    out = []
+
+    def conv(name, sa, sb, w, comm=None, batch=5, **opts):
+        A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
+        p = ll.ll_plan_convert(A, B, w, comm=comm, **opts) if comm else ll.ll_plan_convert(A, B, w, **opts)
+        p.prepare()
+        n = 1 << A.d_in        # all ranks' slices for the loopback communicator (dev bits included)
+        src = torch.randint(-2 ** 15, 2 ** 15, (n * w // 2,), dtype=torch.int16, device="cuda")
+        dst = torch.empty_like(src)
+        ms = _time_stream(lambda: ll.ll_convert(src, dst, p), torch, batch=batch)
+        d = p.describe()
+        gbs = 2 * n * w / ms / 1e6
+        if "tile" in d:
+            ex = d["tile"]["xchg"]
+        elif d.get("exchange") == "peer":
+            ex = "peer stores: one %s tile kernel per rank" % d["fused"]["tile"]["xchg"]
+        else:
+            ex = d["exec"]
+        out.append({"workload": name, "class": d["class"], "executed": ex, "ms": round(ms, 4),
+                    "GBps": round(gbs, 1), "frac": round(gbs / peak, 3)})
+        del src, dst
+
+    # config 1 single tile: latency of one conversion in a CUDA graph of 1000
+    A, B = ll.Layout.from_spec(W.C1_A), ll.Layout.from_spec(W.C1_B)
+    p1 = ll.ll_plan_convert(A, B, 4)
+    p1.prepare()
+    s1 = torch.zeros(256, dtype=torch.int32, device="cuda")
+    d1 = torch.empty_like(s1)
+    st = torch.cuda.Stream()
+    with torch.cuda.stream(st):
+        ll.ll_convert(s1, d1, p1, st)
+        torch.cuda.synchronize()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=st):
+            for _ in range(1000):
+                ll.ll_convert(s1, d1, p1, st)
+    ms = _time_stream(g.replay, torch, batch=1)
+    out.append({"workload": "config 1: one 16x16 fp32 tile (2 warps), 1000 conversions in a CUDA graph",
+                "class": p1.cls, "us_per_conversion": round(ms, 4)})
+    conv("config 1 batch: 2^20 Fig.-1 tiles (16x16 fp32, A -> B = A^T), 1+1 GiB", *W.c1_batched(20), 4)
+    conv("config 3: 16384 tiles 256x128 fp16 blocked -> transposed blocked (optimal swizzle), 1+1 GiB", *W.c3(14), 2)
+    conv("config 5-T, P=1: 32768^2 bf16 row-major -> column-major, 2+2 GiB", *W.c5T(0), 2)
+    conv("config 5, P=8 loopback on one GPU: row- -> column-sharded, peer-store kernels, 2+2 GiB",
+         *W.c5(3), 2, comm=ll.Comm.loopback(8), exchange="peer")
+    # config 4: gather and reduce, [4096, 4096] fp32 in [128, K=32] / [128, 128] tiles
+    for fam in ("mma", "blocked"):
+        L = ll.Layout.from_spec(W.c4("gather", fam))
+        p = ll.ll_plan_gather(L, 1, 4)
+        n = 1 << L.d_in
+        sets = [(torch.randint(-2 ** 31, 2 ** 31 - 1, (n,), dtype=torch.int32, device="cuda"),
+                 torch.randint(0, 32, (n,), dtype=torch.int32, device="cuda"),
+                 torch.empty(n, dtype=torch.int32, device="cuda")) for _ in range(4)]
+        it = [0]
+
+        def g1():
+            s = sets[it[0] % 4]
+            it[0] += 1
+            ll.ll_gather(s[0], s[1], s[2], p)
+        ms = _time_stream(g1, torch)
+        d = p.describe()
+        gbs = 12 * n / ms / 1e6
+        out.append({"workload": f"config 4 gather: [4096,4096] fp32, {fam} [128,32] tiles", "class": "gather",
+                    "executed": d["exchange"] + (" (TMA stages)" if d.get("tma") else ""), "ms": round(ms, 4),
+                    "GBps": round(gbs, 1), "frac": round(gbs / peak, 3)})
+        L = ll.Layout.from_spec(W.c4("reduce", fam))
+        p = ll.ll_plan_reduce(L, 1)
+        rsets = [(torch.rand(n, device="cuda"), torch.empty(p.out_elems(), device="cuda")) for _ in range(4)]
+
+        def r1():
+            s = rsets[it[0] % 4]
+            it[0] += 1
+            ll.ll_reduce(s[0], s[1], p)
+        ms = _time_stream(r1, torch)
+        gbs = (4 * n + 4 * p.out_elems()) / ms / 1e6
+        out.append({"workload": f"config 4 reduce: [4096,4096] fp32 -> [4096,32], {fam} [128,128] tiles",
+                    "class": "reduce", "executed": "tree + shfl.bfly" + (" (TMA stages)" if p.describe().get("tma") else ""),
+                    "ms": round(ms, 4), "GBps": round(gbs, 1), "frac": round(gbs / peak, 3)})
+        del sets, rsets
+    torch.cuda.empty_cache()
+    return out
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -167,6 +272,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-configs", action="store_true", help="skip the other BASELINE configs (N=1 only)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     if args.impl == "reference":
@@ -285,6 +391,10 @@ def main():
             "smem_bank_conflicts": smem_conflicts(),
             "clocks": clk.summary(),
         }
+        if world == 1 and not args.no_configs:
+            del src, dst
+            torch.cuda.empty_cache()
+            line["configs"] = other_configs(ll, W, torch, peak)
         if not args.no_cpu_baseline:
             line["cpu_baseline"] = cpu_baseline_oracle(A_spec, B_spec, w)
         print(json.dumps(line), flush=True)

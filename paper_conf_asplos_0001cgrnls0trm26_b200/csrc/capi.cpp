@@ -52,6 +52,28 @@ void check_cuda(cudaError_t e, const char* what) {
   if (e != cudaSuccess) fail(LL_ERR_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
 }
 
+// Launch of a specialised kernel with programmatic dependent launch (the kernels
+// start with griddepcontrol.wait; ll_kernels.cuh ll_pdl_begin).  LL_PDL=0 disables.
+void launch_kernel(void* kernel, unsigned grid, unsigned block, void** args, size_t smem, cudaStream_t st,
+                   const char* what) {
+  static const bool pdl = [] {
+    const char* e = getenv("LL_PDL");
+    return !(e && std::string(e) == "0");
+  }();
+  cudaLaunchConfig_t cfg;
+  std::memset(&cfg, 0, sizeof cfg);
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(block);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = pdl ? 1 : 0;
+  check_cuda(cudaLaunchKernelExC(&cfg, kernel, args), what);
+}
+
 }  // namespace ll
 
 namespace ll {
@@ -149,8 +171,8 @@ ll_status convert_impl(const void* src, void* dst, void* ws, ConvPlan& P, cudaSt
     u64 ntiles = u64(1) << P.tile.grid_dst_bit.size();
     unsigned long long nt = ntiles;
     void* args[] = {const_cast<void**>(&src), &dst, &nt};
-    check_cuda(cudaLaunchKernel(P.kernel, dim3(grid_for(ntiles)), dim3(P.tile.threads()), args, size_t(P.smem_bytes), st),
-               "cudaLaunchKernel(ll_tile_kernel)");
+    launch_kernel(P.kernel, grid_for(ntiles), P.tile.threads(), args, size_t(P.smem_bytes), st,
+                  "cudaLaunchKernelEx(ll_tile_kernel)");
     return LL_OK;
   }
   if (P.exec == EXEC_GENERIC) {
@@ -563,8 +585,8 @@ ll_status ll_convert_host(const void* src_host, void* dst_host, void* dev_buf, s
       ensure_tile_kernel(P);
       unsigned long long n = nt;
       void* args[] = {&dsrc, &ddst, &n};
-      check_cuda(cudaLaunchKernel(P.kernel, dim3(grid_for(nt)), dim3(T.threads()), args, size_t(P.smem_bytes), st),
-                 "cudaLaunchKernel(ll_tile_kernel)");
+      launch_kernel(P.kernel, grid_for(nt), T.threads(), args, size_t(P.smem_bytes), st,
+                    "cudaLaunchKernelEx(ll_tile_kernel)");
     }
     check_cuda(cudaMemcpyAsync(static_cast<char*>(dst_host) + t0 * tile_dst, ddst, nt * tile_dst,
                                cudaMemcpyDeviceToHost, st), "cudaMemcpyAsync(D2H)");
@@ -599,9 +621,8 @@ ll_status ll_gather(const void* src, const int32_t* idx, void* dst, const ll_pla
     u64 per_sm = std::max<u64>(1, std::min<u64>(8, (228u * 1024u) / u64(G.smem_bytes + 1024)));
     grid = unsigned(std::min<u64>(nt, per_sm * u64(num_sms())));
   }
-  check_cuda(cudaLaunchKernel(G.kernel, dim3(grid), dim3(32u << G.Wb), args, size_t(G.smem_bytes),
-                              static_cast<cudaStream_t>(stream)),
-             "cudaLaunchKernel(ll_gather_kernel)");
+  launch_kernel(G.kernel, grid, 32u << G.Wb, args, size_t(G.smem_bytes), static_cast<cudaStream_t>(stream),
+                "cudaLaunchKernelEx(ll_gather_kernel)");
   LL_CATCH
 }
 
@@ -634,9 +655,8 @@ ll_status ll_reduce(const float* src, float* dst, const ll_plan* p, void* stream
   void* args[] = {const_cast<float**>(&src), &dst, &nt};
   // the TMA pipeline is persistent: one CTA per SM streams its tiles through the stages
   unsigned grid = Rp.tma ? unsigned(std::min<u64>(nt, u64(num_sms()))) : grid_for(nt);
-  check_cuda(cudaLaunchKernel(Rp.kernel, dim3(grid), dim3(32u << Rp.Wb), args, size_t(Rp.smem_bytes),
-                              static_cast<cudaStream_t>(stream)),
-             "cudaLaunchKernel(ll_reduce_kernel)");
+  launch_kernel(Rp.kernel, grid, 32u << Rp.Wb, args, size_t(Rp.smem_bytes), static_cast<cudaStream_t>(stream),
+                "cudaLaunchKernelEx(ll_reduce_kernel)");
   LL_CATCH
 }
 

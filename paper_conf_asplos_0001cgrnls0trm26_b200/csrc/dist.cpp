@@ -268,9 +268,8 @@ namespace {
 void launch_peer_tiles(ConvPlan& F, const void* src, const LLPeersHost& tab, u64 ntiles, u64 tile0, cudaStream_t st) {
   unsigned long long nt = ntiles, t0 = tile0;
   void* args[] = {const_cast<void**>(&src), const_cast<LLPeersHost*>(&tab), &nt, &t0};
-  check_cuda(cudaLaunchKernel(F.kernel, dim3(grid_for_tiles(ntiles)), dim3(F.tile.threads()), args,
-                              size_t(F.smem_bytes), st),
-             "cudaLaunchKernel(ll_tile_peer_kernel)");
+  launch_kernel(F.kernel, grid_for_tiles(ntiles), F.tile.threads(), args, size_t(F.smem_bytes), st,
+                "cudaLaunchKernelEx(ll_tile_peer_kernel)");
 }
 }  // namespace
 

@@ -216,6 +216,8 @@ std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, 
 Layout atomize(const Layout& L);   // 8-byte elements as pairs of 4-byte atoms (capi.cpp)
 int num_sms();
 void check_cuda(cudaError_t e, const char* what);
+void launch_kernel(void* kernel, unsigned grid, unsigned block, void** args, size_t smem, cudaStream_t st,
+                   const char* what);
 // host mirror of LLPeers (ll_kernels.cuh): kernel parameter of the peer tile kernel
 struct LLPeersHost { void* dst[64]; };
 std::string describe(const ConvPlan& P);

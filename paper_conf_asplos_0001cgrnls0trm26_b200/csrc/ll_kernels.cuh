@@ -370,6 +370,16 @@ __device__ __forceinline__ void xchg_smem(const u32 (&r)[P::NW], u32 (&o)[P::NW]
 }
 
 // ------------------------------------------------------------------ tile kernel
+// Programmatic dependent launch (sm_90+): the host launches every kernel with the
+// programmatic-stream-serialization attribute, so a kernel's CTAs may be scheduled
+// while the previous kernel in the stream drains.  Each CTA waits for the previous
+// grid's memory to be visible before touching global memory, then lets the next
+// grid launch (its CTAs in turn wait here), hiding launch latency and ramp.
+__device__ __forceinline__ void ll_pdl_begin() {
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+
 // Destination addressing of the tile kernel.  DstLocal: one buffer.  DstPeers (row
 // a9 DEVICE plans executed as peer stores, §8(f) N4): the dst offset is an offset in
 // the GLOBAL packed index space (local bits, then the dev bits on top); its top bits
@@ -399,6 +409,7 @@ struct DstPeers {
 template <class P, class Dst, bool PEER_REG = false>
 __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, Dst D, u64 ntiles, u64 tile0 = 0) {
   extern __shared__ __align__(16) u8 ll_smem[];
+  ll_pdl_begin();
   const u32 lane = threadIdx.x & 31u;
   const u32 warp = threadIdx.x >> 5;
   const u64 ld_thr = thread_base<P, true>(lane, warp);
@@ -527,6 +538,7 @@ template <class P>
 __device__ __forceinline__ void ll_gather_body(const u8* __restrict__ src, const u8* __restrict__ idx,
                                                u8* __restrict__ dst, u64 ntiles) {
   extern __shared__ __align__(16) u8 ll_smem[];
+  ll_pdl_begin();
   typedef typename std::conditional<P::W == 4, u32, typename std::conditional<P::W == 2, u16, u8>::type>::type ET;
   const u32 lane = threadIdx.x & 31u;
   const u32 warp = threadIdx.x >> 5;
@@ -728,6 +740,7 @@ __device__ __forceinline__ void ll_reduce_tile(u32 (&r)[1 << P::R], float* sm, u
 template <class P>
 __device__ __forceinline__ void ll_reduce_body(const float* __restrict__ src, float* __restrict__ dst, u64 ntiles) {
   extern __shared__ __align__(16) u8 ll_smem[];
+  ll_pdl_begin();
   const u32 lane = threadIdx.x & 31u;
   const u32 warp = threadIdx.x >> 5;
   u64 othr = 0;
