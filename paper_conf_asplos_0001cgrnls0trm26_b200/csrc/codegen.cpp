@@ -150,6 +150,11 @@ std::string codegen_gather(const GatherPlan& G) {
   o << "  static constexpr bool GATHER_SMEM = " << (G.smem ? "true" : "false") << ";\n";
   o << "  static constexpr bool TMA = " << (G.tma ? "true" : "false") << ";\n";
   o << "  static constexpr unsigned STAGES = " << std::max(1, G.stages) << "u;\n";
+  // staging stores as 2^v-element vectors when the thread's vector registers are
+  // consecutive in the logical tile order (line σ: the lowest logical bits)
+  int smv = 0;
+  while (smv < G.v && smv < int(G.smoff.size()) && G.smoff[smv] == (1u << smv)) ++smv;
+  o << icon("SMV", smv);
   o << arr("u32", "SMOFF", G.smoff) << "  static constexpr u32 AXMASK = " << G.axmask << "u;\n"
     << arr("int", "AXPOS", G.axpos);
   o << "  template <int E> static constexpr u32 smoff_of_slot() { u32 s = 0;"

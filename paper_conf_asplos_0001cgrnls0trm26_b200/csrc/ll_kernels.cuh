@@ -612,11 +612,28 @@ __device__ __forceinline__ void ll_gather_body(const u8* __restrict__ src, const
     u32 o[P::NW];
     static_for<P::NW>([&](auto q) { o[decltype(q)::value] = 0; });
     if constexpr (P::GATHER_SMEM) {
-      // stage the tile in logical order, then every output reads its source element
-      static_for<(1 << P::R)>([&](auto e) {
-        constexpr int E = decltype(e)::value;
-        sm[sthr ^ P::template smoff_of_slot<E>()] = ET(get_e<P::W, E>(r));
-      });
+      // stage the tile in logical order (16-byte vectors where the thread's vector
+      // registers are logically consecutive: whole 128 B lines per 8 lanes, no bank
+      // conflicts), then every output reads its source element
+      if constexpr (P::SMV > 0) {
+        constexpr int VE = 1 << P::SMV, VW = (P::W * VE + 3) / 4;
+        const u32 smb = u32(__cvta_generic_to_shared(sm));
+        static_for<(1 << (P::R - P::SMV))>([&](auto k) {
+          constexpr int E0 = decltype(k)::value << P::SMV;
+          u32 v[VW];
+          static_for<VW>([&](auto q) { v[decltype(q)::value] = 0; });
+          static_for<VE>([&](auto ii) {
+            constexpr int I = decltype(ii)::value;
+            set_e<P::W, I>(v, get_e<P::W, E0 + I>(r));
+          });
+          sts_vec<P::W, P::SMV>(smb + (sthr ^ P::template smoff_of_slot<E0>()) * P::W, v);
+        });
+      } else {
+        static_for<(1 << P::R)>([&](auto e) {
+          constexpr int E = decltype(e)::value;
+          sm[sthr ^ P::template smoff_of_slot<E>()] = ET(get_e<P::W, E>(r));
+        });
+      }
       __syncthreads();
       static_for<(1 << P::R)>([&](auto e) {
         constexpr int E = decltype(e)::value;

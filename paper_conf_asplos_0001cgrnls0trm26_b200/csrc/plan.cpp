@@ -910,17 +910,31 @@ std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const 
   // candidates per element remain (force_class selects either)
   int force = opts ? opts->force_class : -1;
   G->smem = force == LL_CLASS_SMEM || (force != LL_CLASS_SHUFFLE && G->cand_bits > 2);
-  // smem layout: the tile's logical bits in ascending order (logical row-major tile)
-  std::vector<u64> tl(G->lcol.begin(), G->lcol.end());
-  std::sort(tl.begin(), tl.end());
-  auto rank_of = [&](u64 c) { return int(std::lower_bound(tl.begin(), tl.end(), c) - tl.begin()); };
+  // smem layout of the staged tile: vector registers, then lanes, then the other
+  // registers, then warps (offset order kreg[0,v), klane, kreg[v,R), kwarp), so the
+  // staging stores are whole 16-byte vectors with consecutive lanes on consecutive
+  // vectors — 4 wavefronts per 512 B, no bank conflicts.  Any linear bijection works
+  // for the reads: an output's source is its own logical coordinate with the axis bits
+  // replaced, i.e. its own offset with the offset bits holding axis bits (AXPOS)
+  // replaced by idx.
   G->smoff.resize(G->lcol.size());
-  for (size_t b = 0; b < G->lcol.size(); ++b) G->smoff[b] = 1u << rank_of(G->lcol[b]);
+  {
+    const int vv = std::min(G->v, R);
+    int o = 0;
+    for (int b = 0; b < vv; ++b) G->smoff[b] = 1u << o++;
+    for (int l = 0; l < 5; ++l) G->smoff[R + l] = 1u << o++;
+    for (int b = vv; b < R; ++b) G->smoff[b] = 1u << o++;
+    for (size_t b = R + 5; b < G->lcol.size(); ++b) G->smoff[b] = 1u << o++;
+  }
   G->axpos.assign(G->K_bits, 0);
   G->axmask = 0;
   for (int t = 0; t < G->K_bits; ++t) {
-    G->axpos[t] = rank_of(u64(1) << (sh + t));
-    G->axmask |= 1u << G->axpos[t];
+    int pos = -1;
+    for (size_t b = 0; b < G->lcol.size(); ++b)
+      if (G->lcol[b] == (u64(1) << (sh + t))) pos = __builtin_ctz(G->smoff[b]);
+    if (pos < 0) fail(LL_ERR_UNSUPPORTED, "gather: an in-tile axis bit has no kernel bit (internal)");
+    G->axpos[t] = pos;
+    G->axmask |= 1u << pos;
   }
   const u64 ne = u64(1) << G->lcol.size();
   const u64 gbytes = G->smem ? ne * u64(w) : 0;
@@ -936,10 +950,11 @@ std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const 
   }
   G->stages = 2;
   const u64 stage_bytes = ne * u64(w + 4);
-  // measured (profiles/r01_sweep_gather_tma.jsonl): the bulk-copy pipeline wins from
-  // 64 KiB stages (K = 64: +10-15%), direct LDG wins below (K = 16: +5-8%)
+  // measured (profiles/r01_sweep_gather_tma.jsonl, r01_sweep_gather_smem_vec.jsonl):
+  // the bulk-copy pipeline wins from 32 KiB stages (K = 32 smem gather: +4%; K = 64:
+  // +10-15%), direct LDG wins below (K = 16: +5-8%)
   G->tma = G->sigma == SIGMA_COALESCED && contiguous && force != LL_CLASS_CTA &&
-           (stage_bytes >= 65536 || force == LL_CLASS_SHUFFLE || force == LL_CLASS_SMEM) &&
+           (stage_bytes >= 32768 || force == LL_CLASS_SHUFFLE || force == LL_CLASS_SMEM) &&
            u64(G->stages) * stage_bytes + gbytes + 16 <= 200 * 1024 && (G->v + ilog2(u64(w))) >= 2;
   G->smem_bytes = int(gbytes + (G->tma ? u64(G->stages) * stage_bytes + 8 * G->stages : 0));
   return G;

@@ -1,5 +1,6 @@
 """Run one hot-path kernel a few times (for ncu captures): --case c2 | c2smem | c3 |
-c3b | c1b | c1bsmem | gather_mma | gather_blocked | reduce_mma | reduce_blocked."""
+c3b | c1b | c1bsmem | c5T | n1 | n2 | c5peer | gather_mma | gather_blocked | reduce_mma |
+reduce_blocked."""
 import argparse
 import os
 import sys
@@ -25,7 +26,16 @@ conv = {"c2": (W.c2(16), 2, {}), "c2smem": (W.c2(16), 2, {"force_class": "SMEM"}
         "c3_small": (W.c3(3), 2, {}), "c2_small": (W.c2(3), 2, {}),
         "c5T": (W.c5T(0, n=15), 2, {}), "n1": (W.n1_preshuffle(14, 14), 2, {}),
         "n2": (W.n2_tmem_epilogue(13), 4, {})}
-if a.case in conv:
+if a.case == "c5peer":
+    # config 5 at P = 8 on one GPU (loopback): one peer-store tile kernel per virtual rank
+    sa, sb = W.c5(3)
+    p = ll.ll_plan_convert(ll.Layout.from_spec(sa), ll.Layout.from_spec(sb), 2, comm=ll.Comm.loopback(8),
+                           exchange="peer")
+    src = torch.randint(-2 ** 15, 2 ** 15, (1 << 30,), dtype=torch.int16, device="cuda")
+    dst = torch.empty_like(src)
+    for _ in range(a.iters):
+        ll.ll_convert(src, dst, p)
+elif a.case in conv:
     (sa, sb), w, opts = conv[a.case]
     A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
     p = ll.ll_plan_convert(A, B, w, **opts)
