@@ -362,6 +362,25 @@ def main():
     torch.cuda.synchronize()
     pick = torch.randint(0, n, (1 << 16,))
     ok_e2e = bool(torch.equal(h_dst[pick].cuda(), dst[pick.cuda()]))
+    # the host link's own limit for the same traffic: concurrent H2D + D2H of the same
+    # bytes with plain pinned copies on two streams (torch), timed the same way
+    d_tmp = torch.empty_like(src)
+    l0, l1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    l0.record(streams[0])
+    streams[1].wait_event(l0)
+    for _ in range(args.e2e_steps):
+        with torch.cuda.stream(streams[0]):
+            d_tmp.copy_(h_src, non_blocking=True)
+        with torch.cuda.stream(streams[1]):
+            h_dst.copy_(dst, non_blocking=True)
+    evl = torch.cuda.Event()
+    evl.record(streams[1])
+    streams[0].wait_event(evl)
+    l1.record(streams[0])
+    torch.cuda.synchronize()
+    link_ms = l0.elapsed_time(l1) / args.e2e_steps
+    del d_tmp
     del dev_buf
 
     if rank == 0:
@@ -386,7 +405,10 @@ def main():
             "e2e": {"value": round(world * bytes_per_step / (e2e_ms / 1e3) / 1e9, 2), "unit": "GB/s",
                     "h2d_bytes_per_step": n * w, "d2h_bytes_per_step": n * w, "ms_per_step": round(e2e_ms, 3),
                     "api": "ll_convert_host (chunked H2D -> kernel -> D2H over 2 streams)",
-                    "matches_device_run": ok_e2e},
+                    "matches_device_run": ok_e2e,
+                    "host_link_GBps": round(2 * n * w / (link_ms / 1e3) / 1e9, 2),
+                    "frac_of_host_link": round(link_ms / e2e_ms, 3),
+                    "host_link": "plain pinned H2D + D2H of the same bytes, concurrent on two streams"},
             "gpu_launches": args.steps,
             "smem_bank_conflicts": smem_conflicts(),
             "clocks": clk.summary(),

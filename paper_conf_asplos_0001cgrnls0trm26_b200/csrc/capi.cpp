@@ -568,7 +568,8 @@ ll_status ll_convert_host(const void* src_host, void* dst_host, void* dev_buf, s
     tile_dst >>= g;
     (void)lw;
   }
-  const u64 slot_bytes = dev_buf_bytes / u64(n_streams);
+  if (reinterpret_cast<uintptr_t>(dev_buf) & 15) fail(LL_ERR_MISALIGNED, "ll_convert_host: dev_buf must be 16-byte aligned");
+  const u64 slot_bytes = (dev_buf_bytes / u64(n_streams)) & ~u64(255);   // 256-byte aligned slots
   u64 chunk = slot_bytes / (tile_src + tile_dst);
   if (chunk == 0) fail(LL_ERR_INVALID_ARG, "ll_convert_host: dev_buf too small for one tile per stream");
   chunk = std::min<u64>(chunk, std::max<u64>(1, ntiles / (2 * u64(n_streams))));   // >= 2 chunks per stream

@@ -392,9 +392,11 @@ def test_broadcast_tile_kernels_gpu():
     assert tiles >= 8
 
 
-def test_convert_host_pipeline():
-    """ll_convert_host: pinned host src -> chunked H2D / kernel / D2H over two streams
-    -> pinned host dst, equal to the oracle."""
+@pytest.mark.parametrize("n_streams,dev_bytes", [(2, 1 << 20), (3, (1 << 20) + 48), (4, 3 << 20)])
+def test_convert_host_pipeline(n_streams, dev_bytes):
+    """ll_convert_host: pinned host src -> chunked H2D / kernel / D2H over 2-4 streams
+    (device scratch split into aligned slots, also for sizes not divisible by the
+    stream count) -> pinned host dst, equal to the oracle."""
     import torch
     sa, sb = W.c2(6)
     A, OA = both(sa)
@@ -404,8 +406,8 @@ def test_convert_host_pipeline():
     src = O.pack(OA, gen.random_bits(rng, 1 << OA.d_out, 2))
     h_src = torch.from_numpy(src.view(np.int16).copy()).pin_memory()
     h_dst = torch.zeros_like(h_src).pin_memory()
-    dev = torch.empty(1 << 20, dtype=torch.uint8, device="cuda")    # forces several chunks
-    streams = [torch.cuda.Stream(), torch.cuda.Stream()]
+    dev = torch.empty(dev_bytes, dtype=torch.uint8, device="cuda")    # forces several chunks
+    streams = [torch.cuda.Stream() for _ in range(n_streams)]
     ll.ll_convert_host(h_src, h_dst, dev, plan, streams)
     torch.cuda.synchronize()
     assert np.array_equal(h_dst.numpy().view(np.uint16), O.convert(OA, OB, src))
