@@ -248,6 +248,18 @@ ll_status ll_convert(const void* src, void* dst, void* workspace, const ll_plan*
 ll_status ll_convert_host(const void* src_host, void* dst_host, void* dev_buf, size_t dev_buf_bytes,
                           const ll_plan* plan, int n_streams, void* const* streams);
 
+/* ll_plan_autotune: measured plan selection for (A, B).  Plans the conversion under
+ * each candidate kernel decomposition — `base` (NULL = defaults), thread_bytes 64 /
+ * 128 / 256 when base leaves it 0, each also with a forced smem exchange when base
+ * does not force a class — compiles every distinct kernel, runs it `iters` times
+ * (default 10) on the caller's src / dst (device buffers as for ll_convert; dst is
+ * overwritten) on `stream`, and returns the fastest plan; describe lists the
+ * candidates and their times ("autotune").  Synchronises `stream`.  Plans without a
+ * tile kernel (NOOP, generic, DEVICE) are returned untuned.  Errors as
+ * ll_plan_convert, plus LL_ERR_CUDA. */
+ll_status ll_plan_autotune(const ll_layout* A, const ll_layout* B, int elem_bytes, const ll_plan_opts* base,
+                           const void* src, void* dst, void* stream, int iters, ll_plan** plan);
+
 /* ---------------------------------------------------------------- gather --
  * ll_plan_gather (row a11; §5.5).  src, idx and dst share layout L
  * (P:430).  Along logical dim `axis`, K = 2^(non-block axis bits of L); these

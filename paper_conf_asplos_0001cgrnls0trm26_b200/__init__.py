@@ -93,6 +93,7 @@ _sig = {
     "ll_comm_create_loopback": [C.c_int, _PP],
     "ll_plan_device_stages": [_P, _PP, _PP, C.POINTER(C.c_size_t), C.POINTER(C.c_int)],
     "ll_comm_create_peers": [C.c_int, C.c_int, _PP, _PP, C.c_size_t, _PP],
+    "ll_plan_autotune": [_P, _P, C.c_int, C.POINTER(_Opts), _P, _P, _P, C.c_int, _PP],
     "ll_ipc_export": [_P, _P],
     "ll_ipc_import": [_P, _PP],
     "ll_ipc_close": [_P],
@@ -528,6 +529,17 @@ def ll_plan_convert(A: Layout, B: Layout, elem_bytes: int, **opts) -> Plan:
     _check(_lib.ll_plan_convert(A.handle, B.handle, int(elem_bytes), C.byref(o), C.byref(h)))
     p = Plan(h, "convert")
     p.comm = opts.get("comm")   # keep the communicator alive as long as the plan
+    return p
+
+
+def ll_plan_autotune(A: Layout, B: Layout, elem_bytes: int, src, dst, stream=None, iters: int = 10, **opts) -> Plan:
+    """Fastest plan among the candidate kernel decompositions, timed on src/dst."""
+    h = C.c_void_p()
+    o = _opts(**opts)
+    _check(_lib.ll_plan_autotune(A.handle, B.handle, int(elem_bytes), C.byref(o), _ptr(src), _ptr(dst),
+                                 _stream_ptr(stream), int(iters), C.byref(h)))
+    p = Plan(h, "convert")
+    p.comm = opts.get("comm")
     return p
 
 

@@ -544,6 +544,75 @@ ll_status ll_convert(const void* src, void* dst, void* ws, const ll_plan* p, voi
   LL_CATCH
 }
 
+// Measured plan selection: every candidate kernel decomposition (thread_bytes 64 / 128
+// / 256 and the default, with and without a forced smem exchange) is planned,
+// compiled and timed on the caller's buffers; the fastest plan is returned.
+ll_status ll_plan_autotune(const ll_layout* A, const ll_layout* B, int w, const ll_plan_opts* base,
+                           const void* src, void* dst, void* stream, int iters, ll_plan** out) {
+  LL_TRY
+  if (!A || !B || !out || !src || !dst) fail(LL_ERR_INVALID_ARG, "null argument");
+  if (iters < 1) iters = 10;
+  ll_plan_opts o0;
+  if (base) o0 = *base; else ll_plan_opts_default(&o0);
+  std::vector<ll_plan_opts> cand{o0};
+  for (int tb : {64, 128, 256})
+    if (o0.thread_bytes == 0) { ll_plan_opts c = o0; c.thread_bytes = tb; cand.push_back(c); }
+  if (o0.force_class < 0) {
+    const size_t nc = cand.size();
+    for (size_t i = 0; i < nc; ++i) { ll_plan_opts c = cand[i]; c.force_class = LL_CLASS_SMEM; cand.push_back(c); }
+  }
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  cudaEvent_t e0, e1;
+  check_cuda(cudaEventCreate(&e0), "cudaEventCreate");
+  check_cuda(cudaEventCreate(&e1), "cudaEventCreate");
+  std::unique_ptr<ll_plan> best;
+  float best_ms = 0;
+  std::vector<std::string> seen;
+  std::ostringstream log;
+  log << "[";
+  bool first = true;
+  try {
+    for (const ll_plan_opts& c : cand) {
+      ll_plan* raw = nullptr;
+      if (ll_plan_convert(A, B, w, &c, &raw) != LL_OK) continue;
+      std::unique_ptr<ll_plan> p(raw);
+      ConvPlan& P = p->cp();
+      if (P.exec != EXEC_TILE) {          // nothing to tune: NOOP / generic / DEVICE
+        if (!best) best = std::move(p);
+        break;
+      }
+      if (std::find(seen.begin(), seen.end(), P.source) != seen.end()) continue;
+      seen.push_back(P.source);
+      convert_impl(src, dst, nullptr, P, st);   // compile, load, warm up
+      convert_impl(src, dst, nullptr, P, st);
+      check_cuda(cudaEventRecord(e0, st), "cudaEventRecord");
+      for (int i = 0; i < iters; ++i) convert_impl(src, dst, nullptr, P, st);
+      check_cuda(cudaEventRecord(e1, st), "cudaEventRecord");
+      check_cuda(cudaEventSynchronize(e1), "cudaEventSynchronize");
+      float ms = 0;
+      check_cuda(cudaEventElapsedTime(&ms, e0, e1), "cudaEventElapsedTime");
+      ms /= float(iters);
+      static const char* xc[] = {"copy", "regperm", "shuffle", "smem"};
+      log << (first ? "" : ",") << "{\"thread_bytes\":" << c.thread_bytes << ",\"force_smem\":"
+          << (c.force_class == LL_CLASS_SMEM ? "true" : "false") << ",\"xchg\":\"" << xc[P.tile.xchg]
+          << "\",\"R\":" << P.tile.R << ",\"threads\":" << P.tile.threads() << ",\"ms\":" << ms << "}";
+      first = false;
+      if (!best || ms < best_ms) { best = std::move(p); best_ms = ms; }
+    }
+  } catch (...) {
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    throw;
+  }
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  if (!best) fail(LL_ERR_UNSUPPORTED, "autotune: no candidate plan");
+  log << "]";
+  if (!first) best->cp().tune_json = log.str();
+  *out = best.release();
+  LL_CATCH
+}
+
 ll_status ll_convert_host(const void* src_host, void* dst_host, void* dev_buf, size_t dev_buf_bytes,
                           const ll_plan* p, int n_streams, void* const* streams) {
   LL_TRY

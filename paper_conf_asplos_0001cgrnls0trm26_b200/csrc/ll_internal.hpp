@@ -204,6 +204,7 @@ struct ConvPlan {
   u64 rank_tiles = 0;
   int peer_shift = -1;    // >= 0: this tile plan is a peer kernel; log2 local elements
   bool peer_reg = false;  // a dst register / replica bit crosses ranks
+  std::string tune_json;   // ll_plan_autotune: the candidates and their times (describe)
   std::string source;   // specialised kernel source (EXEC_TILE)
   std::string kernel_key;
   void* kernel = nullptr;   // cudaKernel_t once loaded

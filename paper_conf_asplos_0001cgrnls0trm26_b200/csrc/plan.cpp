@@ -802,6 +802,7 @@ std::string describe(const ConvPlan& P) {
         << ",\"ideal_wavefronts\":" << T.ideal_wavefronts;
     o << "}";
   }
+  if (!P.tune_json.empty()) o << ",\"autotune\":" << P.tune_json;
   if (P.exec == EXEC_DEVICE) {
     o << ",\"dev_bits\":" << P.dev_bits << ",\"workspace_bytes\":" << P.workspace_bytes
       << ",\"exchange\":\"" << (P.exchange == LL_EXCHANGE_PEER ? "peer" : "collective") << "\"";

@@ -519,3 +519,21 @@ def test_e1_exhaustive_generic_gpu():
     got = d_dst.cpu().numpy().view(np.uint32)
     bad = np.nonzero(~np.all(got == want, axis=1))[0]
     assert bad.size == 0, [perms[i] for i in bad[:5]]
+
+
+@pytest.mark.parametrize("which", ["n2", "c1b", "c3"])
+def test_autotune_bitexact(which):
+    """ll_plan_autotune: every candidate decomposition is timed on the caller's buffers;
+    the returned (fastest) plan converts bit-exactly, and describe lists the candidates."""
+    sa, sb, w = {"n2": (*W.n2_tmem_epilogue(5), 4), "c1b": (*W.c1_batched(8), 4), "c3": (*W.c3(3), 2)}[which]
+    A, OA = both(sa)
+    B, OB = both(sb)
+    T = gen.random_bits(np.random.default_rng(12), 1 << OA.d_out, w)
+    src = O.pack(OA, T)
+    d_src, d_dst = to_device(src), empty_device(1 << OB.d_in, w)
+    plan = ll.ll_plan_autotune(A, B, w, d_src, d_dst, iters=3)
+    cands = plan.describe()["autotune"]
+    assert len(cands) >= 2 and all(c["ms"] > 0 for c in cands)
+    d_dst.zero_()
+    ll.ll_convert(d_src, d_dst, plan)
+    assert np.array_equal(from_device(d_dst, w), O.pack(OB, T))

@@ -255,6 +255,8 @@ def test_device_entry_fails_loudly_without_gpu():
     p = ll.ll_plan_convert(A, B, 4)
     with pytest.raises(ll.LLError, match="CUDA"):
         ll.ll_convert(1 << 20, 2 << 20, p, stream=0)
+    with pytest.raises(ll.LLError, match="CUDA"):
+        ll.ll_plan_autotune(A, B, 4, 1 << 20, 2 << 20, stream=0)
 
 
 # ---------------------------------------------------------------- layout families

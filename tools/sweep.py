@@ -53,7 +53,8 @@ def conv_case(name, sa, sb, w, **opts):
     gbs = 2 * n * w / ms / 1e6
     d = p.describe()
     t = d.get("tile", {})
-    print(json.dumps({"case": name, "opts": opts, "class": d["class"], "xchg": t.get("xchg"), "ms": round(ms, 4),
+    print(json.dumps({"case": name, "opts": opts, "class": d["class"], "xchg": t.get("xchg"), "threads": t.get("threads"),
+                      "R": t.get("R"), "ms": round(ms, 4),
                       "GBps": round(gbs, 1), "frac_6539": round(gbs / 6539.5, 3)}), flush=True)
     del src, dst
     torch.cuda.empty_cache()
@@ -71,6 +72,12 @@ def main():
         return next_rows()
     if "lat" in only:
         return latency_and_ksweep()
+    if "n2" in only:
+        return n2_options()
+    if "tb" in only:
+        return thread_bytes_sweep()
+    if "tune" in only:
+        return autotune_sweep()
     if "all" not in only and "conv" not in only:
         return gather_reduce()
     # raw copy roofline reference
@@ -126,6 +133,57 @@ def next_rows():
         conv_case("c5T P=1 transpose", sa, sb, 2, **opts)
     for opts in [dict(), dict(tile_bytes=65536), dict(thread_bytes=128)]:
         conv_case("N1 preshuffle", *W.n1_preshuffle(14, 14), 2, **opts)
+
+
+def n2_options():
+    """N2 (TMEM 32x32b fragment -> blocked) under the plan options."""
+    sa, sb = W.n2_tmem_epilogue(13)
+    for opts in [dict(), dict(force_class="SMEM"), dict(thread_bytes=32), dict(thread_bytes=128),
+                 dict(tile_bytes=32768), dict(tile_bytes=65536), dict(force_class="SMEM", thread_bytes=128),
+                 dict(force_class="SMEM", thread_bytes=32)]:
+        conv_case("N2 tmem 32x32b -> blocked", sa, sb, 4, **opts)
+    sa, sb = W.n1_preshuffle(14, 14)
+    for opts in [dict(thread_bytes=32), dict(tile_bytes=32768), dict(force_class="SMEM", thread_bytes=128)]:
+        conv_case("N1 preshuffle", sa, sb, 2, **opts)
+
+
+def thread_bytes_sweep():
+    """Every tile-kernel config under thread_bytes 64 / 128 / 256 (default = None)."""
+    cases = [("c1b", W.c1_batched(20), 4), ("c2", W.c2(16), 2), ("c3", W.c3(14), 2), ("c3b", W.c3b(14), 2),
+             ("n2", W.n2_tmem_epilogue(13), 4), ("c5T", W.c5T(0), 2), ("n1", W.n1_preshuffle(14, 14), 2)]
+    for name, (sa, sb), w in cases:
+        for tb in (None, 64, 128, 256):
+            opts = {} if tb is None else {"thread_bytes": tb}
+            try:
+                conv_case(name, sa, sb, w, **opts)
+            except Exception as e:  # noqa: BLE001
+                print(json.dumps({"case": name, "opts": opts, "error": str(e)[:120]}), flush=True)
+
+
+def autotune_sweep():
+    """ll_plan_autotune vs the default plan on every tile-kernel config."""
+    cases = [("c1b", W.c1_batched(20), 4), ("c2", W.c2(16), 2), ("c3", W.c3(14), 2), ("c3b", W.c3b(14), 2),
+             ("n2", W.n2_tmem_epilogue(13), 4), ("c5T", W.c5T(0), 2), ("n1", W.n1_preshuffle(14, 14), 2)]
+    for name, (sa, sb), w in cases:
+        A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
+        n = 1 << A.d_in
+        src = torch.randint(-2 ** 15, 2 ** 15, (n * w // 2,), dtype=torch.int16, device="cuda")
+        dst = torch.empty_like(src)
+        t0 = time.time()
+        p = ll.ll_plan_autotune(A, B, w, src, dst, iters=5)
+        tune_s = time.time() - t0
+        pd = ll.ll_plan_convert(A, B, w)
+        pd.prepare()
+        ms_d = time_fn(lambda: ll.ll_convert(src, dst, pd))
+        ms_t = time_fn(lambda: ll.ll_convert(src, dst, p))
+        d = p.describe()
+        print(json.dumps({"case": name, "default_GBps": round(2 * n * w / ms_d / 1e6, 1),
+                          "tuned_GBps": round(2 * n * w / ms_t / 1e6, 1),
+                          "tuned_frac_6539": round(2 * n * w / ms_t / 1e6 / 6539.5, 3),
+                          "tune_seconds": round(tune_s, 1), "chosen": {k: d["tile"][k] for k in ("xchg", "R", "threads")},
+                          "candidates": d.get("autotune")}), flush=True)
+        del src, dst
+        torch.cuda.empty_cache()
 
 
 def latency_and_ksweep():
