@@ -66,6 +66,7 @@ std::string codegen_tile(const ConvPlan& Pl) {
     << icon("VLD", T.vld) << icon("VST", T.vst) << icon("XCHG", T.xchg) << icon("THREADS", T.threads());
   o << "  static constexpr bool ISOLATE_SMEM = " << (std::getenv("LL_ISOLATE_SMEM") ? "true" : "false") << ";\n";
   o << icon("ST_HINT", st_hint());
+  o << "  static constexpr bool PIPE = " << (T.pipe ? "true" : "false") << ";\n";
   // per-thread-contiguous loads (faithful σ) re-use sectors across instructions
   o << "  static constexpr bool LD_L1 = " << (T.sigma == SIGMA_FAITHFUL ? "true" : "false") << ";\n";
   std::vector<u64> ldc, stc;

@@ -152,6 +152,7 @@ struct TilePlan {
   std::vector<u64> ld_xcol, grid_src_xcol;
   int sigma = SIGMA_COALESCED;
   int xchg = X_COPY;
+  bool pipe = false;    // X_SMEM: next tile's loads issued before this tile's stores
 
   // --- REGPERM: out slot e <- in slot perm[e]
   std::vector<int> perm;

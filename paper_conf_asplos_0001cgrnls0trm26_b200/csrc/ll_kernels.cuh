@@ -338,7 +338,7 @@ __device__ __forceinline__ u32 smem_thread_base(u32 lane, u32 warp) {
 // a8 SMEM: st.shared through M^{-1}∘L_ld, barrier,
 // ld.shared through M^{-1}∘L_st; M is the optimal swizzle (conflict-free).
 template <class P>
-__device__ __forceinline__ void xchg_smem(const u32 (&r)[P::NW], u32 (&o)[P::NW], u32 lane, u32 warp, u32 sbase) {
+__device__ __forceinline__ void smem_write(const u32 (&r)[P::NW], u32 lane, u32 warp, u32 sbase) {
   constexpr int VE = 1 << P::SV;
   constexpr int VW = (P::W * VE + 3) / 4;
   const u32 tst = smem_thread_base<P, true>(lane, warp);
@@ -354,7 +354,11 @@ __device__ __forceinline__ void xchg_smem(const u32 (&r)[P::NW], u32 (&o)[P::NW]
     constexpr u32 off = u32(SmVec<P, K, true>::off());
     sts_vec<P::W, P::SV>(sbase + (tst ^ off) * P::W, v);
   });
-  __syncthreads();
+}
+template <class P>
+__device__ __forceinline__ void smem_read(u32 (&o)[P::NW], u32 lane, u32 warp, u32 sbase) {
+  constexpr int VE = 1 << P::SV;
+  constexpr int VW = (P::W * VE + 3) / 4;
   const u32 tld = smem_thread_base<P, false>(lane, warp);
   static_for<(1 << (P::R - P::SV))>([&](auto k) {
     constexpr int K = decltype(k)::value;
@@ -367,6 +371,12 @@ __device__ __forceinline__ void xchg_smem(const u32 (&r)[P::NW], u32 (&o)[P::NW]
       set_e<P::W, S>(o, get_e<P::W, I>(v));
     });
   });
+}
+template <class P>
+__device__ __forceinline__ void xchg_smem(const u32 (&r)[P::NW], u32 (&o)[P::NW], u32 lane, u32 warp, u32 sbase) {
+  smem_write<P>(r, lane, warp, sbase);
+  __syncthreads();
+  smem_read<P>(o, lane, warp, sbase);
 }
 
 // ------------------------------------------------------------------ tile kernel
@@ -429,13 +439,10 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, Dst D, 
     if (r[0] == 0x9e3779b9u) *D.at(threadIdx.x) = u8(r[P::NW - 1]);
     return;
   }
-  for (u64 t = blockIdx.x; t < ntiles; t += gridDim.x) {
+  // a5: HBM load of a src tile (16-byte vectors; coalesced under σ_ld)
+  auto load_tile = [&](u32 (&r)[P::NW], u64 t) {
     const u64 sofs = tile_base<P, true>(t) ^ ld_thr;
     const u8* s = src + sofs;
-    const u64 doff = tile_base<P, false>(t | tile0) ^ st_thr;
-    u8* d = D.at(doff);
-    u32 r[P::NW];
-    // a5: HBM load of the src tile (16-byte vectors; coalesced under σ_ld)
     static_for<(1 << (P::R - P::VLD))>([&](auto k) {
       constexpr int K = decltype(k)::value;
       // XOR-copy plans (non-permutation Q): register and thread offsets share bits,
@@ -445,6 +452,45 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, Dst D, 
       else
         load_vec<P::W, P::VLD, K, P::NW, P::LD_L1>(r, s + LdOff<P, K>::value());
     });
+  };
+  // a10: HBM store of a dst tile (and of its broadcast replicas)
+  auto store_tile = [&](const u32 (&o)[P::NW], u64 t) {
+    const u64 doff = tile_base<P, false>(t | tile0) ^ st_thr;
+    u8* d = D.at(doff);
+    static_for<P::NREP>([&](auto rp) {
+      constexpr u64 RO = P::REP_OFF[decltype(rp)::value];
+      static_for<(1 << (P::R - P::VST))>([&](auto k) {
+        constexpr int K = decltype(k)::value;
+        if constexpr (PEER_REG)
+          store_vec<P::W, P::VST, K, P::NW, P::ST_HINT>(o, D.at(doff + (StOff<P, K>::value() ^ RO)));
+        else
+          store_vec<P::W, P::VST, K, P::NW, P::ST_HINT>(o, d + (StOff<P, K>::value() ^ RO));
+      });
+    });
+  };
+  if constexpr (P::XCHG == 3 && P::PIPE) {
+    // Software-pipelined smem exchange: once tile t sits in shared memory its
+    // registers are free, so tile t + grid's loads are issued before t's smem reads
+    // and HBM stores — the CTA keeps loads in flight through its store phase.
+    u64 t = blockIdx.x;
+    if (t >= ntiles) return;
+    u32 r[P::NW];
+    load_tile(r, t);
+    for (; t < ntiles; t += gridDim.x) {
+      smem_write<P>(r, lane, warp, sbase);
+      __syncthreads();
+      if (t + gridDim.x < ntiles) load_tile(r, t + gridDim.x);
+      u32 o[P::NW];
+      static_for<P::NW>([&](auto q) { o[decltype(q)::value] = 0; });
+      smem_read<P>(o, lane, warp, sbase);
+      store_tile(o, t);
+      __syncthreads();   // smem reuse by the next tile
+    }
+    return;
+  }
+  for (u64 t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    u32 r[P::NW];
+    load_tile(r, t);
     u32 o[P::NW];
     if constexpr (P::XCHG == 0) {
       static_for<P::NW>([&](auto q) { o[decltype(q)::value] = r[decltype(q)::value]; });
@@ -457,17 +503,7 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, Dst D, 
       static_for<P::NW>([&](auto q) { o[decltype(q)::value] = 0; });
       xchg_smem<P>(r, o, lane, warp, sbase);
     }
-    // a10: HBM store of the dst tile (and of its broadcast replicas)
-    static_for<P::NREP>([&](auto rp) {
-      constexpr u64 RO = P::REP_OFF[decltype(rp)::value];
-      static_for<(1 << (P::R - P::VST))>([&](auto k) {
-        constexpr int K = decltype(k)::value;
-        if constexpr (PEER_REG)
-          store_vec<P::W, P::VST, K, P::NW, P::ST_HINT>(o, D.at(doff + (StOff<P, K>::value() ^ RO)));
-        else
-          store_vec<P::W, P::VST, K, P::NW, P::ST_HINT>(o, d + (StOff<P, K>::value() ^ RO));
-      });
-    });
+    store_tile(o, t);
     if constexpr (P::XCHG == 3) __syncthreads();   // smem reuse by the next tile
   }
 }

@@ -1,6 +1,7 @@
 // Conversion planner (rows a3, a4, a6-a9) plus gather (a11) and
 // reduce (a12) plans.
 #include <algorithm>
+#include <cstdlib>
 #include <functional>
 #include <cstring>
 #include <sstream>
@@ -551,6 +552,13 @@ static void build_tile(ConvPlan& P, const std::vector<int>& S0, const std::vecto
   }
   if (T.xchg == X_REGPERM) plan_regperm(T);
   if (T.xchg == X_SMEM) plan_smem(T, maxvec);
+  if (T.xchg == X_SMEM) {
+    // software-pipelined smem exchange (next tile's loads before this tile's stores):
+    // measured slower on every default-sized config — the second register buffer costs
+    // occupancy (profiles/r01_sweep_smem_pipeline.jsonl) — so only on request
+    const char* e = std::getenv("LL_PIPE");
+    T.pipe = e && std::string(e) == "1";
+  }
   if (T.xchg == X_SMEM && (T.smem_elems * u64(T.w)) > 200 * 1024)
     fail(LL_ERR_UNSUPPORTED, "smem tile too large");
   P.smem_bytes = T.xchg == X_SMEM ? int(T.smem_elems * T.w) : 0;
