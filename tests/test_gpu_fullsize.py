@@ -1,0 +1,141 @@
+"""Every BASELINE config at its full size, in the launch configuration bench.py times
+(the default plan, the same buffers' shapes), against the oracle (-m gpu).
+
+Configs 2 and 3 are in test_gpu_convert.py (sampled full-size checks).  Here:
+config 1 batch (2^20 tiles, 1 GiB), config 3b, config 4 gather and reduce for both
+families on the whole [4096, 4096] fp32 tensor (every output compared), config 5-T
+(2 GiB transpose) and config 5 at P = 8 on the loopback communicator with both
+exchanges (2 GiB).  Large conversions are checked on 2^18-2^20 sampled outputs, each
+against the oracle's pull map evaluated point by point (O5 with the slack-zero inverse).
+"""
+import numpy as np
+import pytest
+
+from oracle import ll_oracle as O
+from workloads import configs as W
+from workloads import gen
+
+pytestmark = pytest.mark.gpu
+
+ll = pytest.importorskip("paper_conf_asplos_0001cgrnls0trm26_b200")
+
+
+def both(spec):
+    return ll.Layout.from_spec(spec), O.Layout(*W.spec_to_bases(spec))
+
+
+def _sampled(OA, OB, src, dst, n, seed, k=1 << 19):
+    import torch
+    rng = np.random.default_rng(seed)
+    hs = np.unique(np.concatenate([rng.integers(0, n, size=k), np.arange(4096), n - 1 - np.arange(4096)]))
+    hs = hs.astype(np.uint64)
+    hsrc = O.apply_inverse_all(OA, O.apply_all(OB, hs)).astype(np.int64)
+    got = dst[torch.from_numpy(hs.astype(np.int64)).cuda()].cpu().numpy()
+    want = src[torch.from_numpy(hsrc).cuda()].cpu().numpy()
+    assert np.array_equal(got, want)
+
+
+@pytest.mark.parametrize("name", ["c1_batch", "c3b", "c5T"])
+def test_fullsize_conversions(name):
+    import torch
+    (sa, sb), w = {"c1_batch": (W.c1_batched(20), 4), "c3b": (W.c3b(14), 2), "c5T": (W.c5T(0), 2)}[name]
+    A, OA = both(sa)
+    B, OB = both(sb)
+    plan = ll.ll_plan_convert(A, B, w)
+    n = 1 << OA.d_in
+    dt = {2: torch.int16, 4: torch.int32}[w]
+    g = torch.Generator(device="cuda").manual_seed(1003)
+    src = torch.randint(-2 ** 15, 2 ** 15, (n,), dtype=dt, device="cuda", generator=g)
+    dst = torch.empty_like(src)
+    ll.ll_convert(src, dst, plan)
+    torch.cuda.synchronize()
+    _sampled(OA, OB, src, dst, n, 11)
+    del src, dst
+    torch.cuda.empty_cache()
+
+
+@pytest.mark.parametrize("exchange", ["collective", "peer"])
+def test_fullsize_config5_p8_loopback(exchange):
+    """Config 5: [32768, 32768] bf16 row-sharded -> column-sharded over 8 virtual ranks
+    (2 GiB); every rank's slice sampled against the oracle's closed form O12."""
+    import torch
+    p, n = 3, 15
+    sa, sb = W.c5(p, n=n)
+    OA, OB = O.Layout(*W.spec_to_bases(sa)), O.Layout(*W.spec_to_bases(sb))
+    A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
+    P = 1 << p
+    plan = ll.ll_plan_convert(A, B, 2, comm=ll.Comm.loopback(P), exchange=exchange)
+    total = 1 << (2 * n)
+    nloc = total // P
+    # logical tensor T as a hash of the flat index; rank slices of A built from it
+    g = torch.Generator(device="cuda").manual_seed(1006)
+    T = torch.randint(-2 ** 15, 2 ** 15, (total,), dtype=torch.int16, device="cuda", generator=g)
+    # input construction only (a wrong src fails the oracle check below): rank r's
+    # slice of A is T at A(h, dev=r), the XOR of the oracle's columns, evaluated on
+    # the device for the 2^27 points of each slice
+    src = torch.empty(total, dtype=torch.int16, device="cuda")
+    hl = torch.arange(nloc, dtype=torch.int64, device="cuda")
+    for r in range(P):
+        la, off = O.rank_slice(OA, r)
+        xs = torch.full_like(hl, int(off))
+        for k, c in enumerate(la.cols):
+            xs ^= ((hl >> k) & 1) * int(c)
+        src[r * nloc:(r + 1) * nloc] = T[xs]
+    del hl, xs
+    dst = torch.empty_like(src)
+    ws = torch.empty(max(16, plan.workspace_bytes()), dtype=torch.uint8, device="cuda")
+    ll.ll_convert(src, dst, plan, workspace=ws)
+    torch.cuda.synchronize()
+    rng = np.random.default_rng(13)
+    for r in range(P):
+        hs = np.concatenate([rng.integers(0, nloc, size=1 << 16), np.arange(1024), nloc - 1 - np.arange(1024)])
+        hs = hs.astype(np.uint64)
+        lb, offb = O.rank_slice(OB, r)
+        xs = (O.apply_all(lb, hs) ^ np.uint64(offb)).astype(np.int64)
+        got = dst[r * nloc + torch.from_numpy(hs.astype(np.int64)).cuda()]
+        assert torch.equal(got, T[torch.from_numpy(xs).cuda()]), r
+    del T, src, dst
+    torch.cuda.empty_cache()
+
+
+@pytest.mark.parametrize("family", ["mma", "blocked"])
+def test_fullsize_config4_gather(family):
+    """Config 4 gather on the whole [4096, 4096] fp32 tensor in [128, 32] tiles: every
+    output equal to O10 (take_along_axis inside each tile, indices masked, G16)."""
+    import torch
+    spec = W.c4("gather", family)
+    L, OL = both(spec)
+    n = 1 << OL.d_in
+    rng = np.random.default_rng(1004)
+    T = gen.random_bits(rng, n, 4)
+    Ti = rng.integers(-1000, 1000, size=n).astype(np.int32)
+    src, idx = O.pack(OL, T), O.pack(OL, Ti)
+    plan = ll.ll_plan_gather(L, 1, 4)
+    d_dst = torch.empty(n, dtype=torch.int32, device="cuda")
+    ll.ll_gather(torch.from_numpy(src.view(np.int32)).cuda(), torch.from_numpy(idx).cuda(), d_dst, plan)
+    got = d_dst.cpu().numpy().view(np.uint32)
+    assert np.array_equal(got, O.gather(OL, 1, src, idx))
+
+
+@pytest.mark.parametrize("family", ["mma", "blocked"])
+def test_fullsize_config4_reduce(family):
+    """Config 4 reduce on the whole [4096, 4096] fp32 tensor in [128, 128] tiles -> [4096,
+    32]: every output within 1e-6 of the fp64 sum, and bit-equal to the fixed-order fp32
+    replica over the kernel layout (O11; the σ rule re-derived in test_gpu_convert)."""
+    import torch
+    from tests.test_gpu_convert import _line_sigma_layout
+    spec = W.c4("reduce", family)
+    L, OL = both(spec)
+    n = 1 << OL.d_in
+    T = np.random.default_rng(1005).random(n, dtype=np.float32)
+    src = O.pack(OL, T)
+    plan = ll.ll_plan_reduce(L, 1)
+    out = torch.empty(plan.out_elems(), dtype=torch.float32, device="cuda")
+    ll.ll_reduce(torch.from_numpy(src).cuda(), out, plan)
+    got = out.cpu().numpy()
+    ref = O.reduce_ref_fp64(OL, 1, src)
+    assert got.size == 4096 * 32
+    assert np.all(np.abs(got - ref) <= 1e-6 * np.abs(ref))
+    Lp, perm = _line_sigma_layout(OL, 1)
+    rep = O.reduce_fixed_order_fp32(Lp, 1, src[perm])
+    assert np.array_equal(got.view(np.uint32), rep.view(np.uint32))
