@@ -264,6 +264,57 @@ def other_configs(ll, W, torch, peak):
     return out
 
 
+def config5_exchange(ll, W, torch, world, rank, steps=10, warmup=3):
+    """Config 5 across the GPUs of this job (N > 1, N a power of two): a [32768, 32768]
+    bf16 tensor row-sharded over N ranks, redistributed to column-sharded — the DEVICE
+    class over NVLink, with both exchanges: the collective decomposition (pack ->
+    grouped ncclSend/ncclRecv -> unpack) and the fused peer-store kernel writing into
+    the receivers' windows (CUDA IPC).  Time = max over ranks of CUDA-event time per
+    conversion; errors are reported, not raised, so the main line still prints."""
+    import torch.distributed as dist
+    p = world.bit_length() - 1
+    total = 1 << 30
+    nloc = total // world
+    sa, sb = W.c5(p)
+    A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
+    src = torch.randint(-2 ** 15, 2 ** 15, (nloc,), dtype=torch.int16, device="cuda")
+    dst = torch.empty_like(src)
+    flags = torch.zeros(ll.PEER_FLAG_BYTES // 4, dtype=torch.int32, device="cuda")
+    out = {"workload": f"config 5: [32768,32768] bf16 row-sharded -> column-sharded over {world} GPUs",
+           "bytes_per_gpu_each_way_nvlink": int((world - 1) * nloc * 2 // world)}
+    for exchange in ("collective", "peer"):
+        try:
+            comm = ll.Comm.from_process_group() if exchange == "collective" else ll.Comm.peers(dst, flags)
+            plan = ll.ll_plan_convert(A, B, 2, comm=comm, exchange=exchange)
+            plan.prepare()
+            ws = torch.empty(max(16, plan.workspace_bytes()), dtype=torch.uint8, device="cuda")
+            for _ in range(warmup):
+                ll.ll_convert(src, dst, plan, workspace=ws)
+            torch.cuda.synchronize()
+            dist.barrier()
+            torch.cuda.synchronize()
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record()
+            for _ in range(steps):
+                ll.ll_convert(src, dst, plan, workspace=ws)
+            b.record()
+            torch.cuda.synchronize()
+            t = torch.tensor([a.elapsed_time(b) / steps], device="cuda", dtype=torch.float64)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ms = float(t.item())
+            nvl = out["bytes_per_gpu_each_way_nvlink"]
+            out[exchange] = {"ms": round(ms, 4), "aggregate_GBps": round(2 * total * 2 / (ms / 1e3) / 1e9, 1),
+                             "nvlink_GBps_per_gpu_each_way": round(nvl / (ms / 1e3) / 1e9, 1),
+                             "frac_of_900": round(nvl / (ms / 1e3) / 1e9 / 900, 3),
+                             "class": plan.cls, "exchange": plan.describe().get("exchange")}
+            del plan, comm, ws
+        except Exception as e:  # noqa: BLE001 - reported in the JSON line
+            out[exchange] = {"error": f"{type(e).__name__}: {str(e)[:200]}"}
+    del src, dst
+    torch.cuda.empty_cache()
+    return out
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -273,6 +324,7 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-configs", action="store_true", help="skip the other BASELINE configs (N=1 only)")
+    ap.add_argument("--no-config5", action="store_true", help="skip the cross-GPU config-5 exchange (N>1 only)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     if args.impl == "reference":
@@ -382,6 +434,9 @@ def main():
     link_ms = l0.elapsed_time(l1) / args.e2e_steps
     del d_tmp
     del dev_buf
+    c5 = None
+    if world > 1 and (world & (world - 1)) == 0 and not args.no_config5:
+        c5 = config5_exchange(ll, W, torch, world, rank)
 
     if rank == 0:
         peak, peak_kind = hbm_peak()
@@ -413,6 +468,8 @@ def main():
             "smem_bank_conflicts": smem_conflicts(),
             "clocks": clk.summary(),
         }
+        if c5 is not None:
+            line["config5_nvlink"] = c5
         if world == 1 and not args.no_configs:
             del src, dst
             torch.cuda.empty_cache()
