@@ -492,3 +492,26 @@ def test_random_memory_layouts_xor_copy_simulated(w):
                 s = O.pack(OA_, T)
                 assert np.array_equal(p.simulate(s, 1 << d), O.convert(OA_, OB_, s)), (d, seed)
     assert tiles >= 40
+
+
+def test_planner_faithful_reproduces_gv6_gv8():
+    """Under faithful σ (the kernel holds the data exactly as the paper's layouts do) the
+    planner's swizzle and shuffle sets equal the hand derivations GV6-GV8 of the paper's
+    constructions (tests/golden/derived_gv6_gv8.json; P:375-387, P:406-426)."""
+    import json
+    import os
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "derived_gv6_gv8.json")))
+
+    def flat(e, jb):
+        v = 0
+        for t in e.split("^"):
+            v ^= 1 << (int(t[1:]) if t[0] == "j" else int(t[1:]) + jb)
+        return v
+    for key, (sa, sb), w, fields in [("GV6_config1", (W.C1_A, W.C1_B), 4, ("Vec", "Bank", "Seg")),
+                                     ("GV8_config3", W.c3(0), 2, ("Vec", "Bank", "Seg")),
+                                     ("GV7_config2", W.c2(0), 2, ("V", "I", "E", "F", "G"))]:
+        p = ll.ll_plan_convert(ll.Layout.from_spec(sa), ll.Layout.from_spec(sb), w, sigma="faithful")
+        t = p.describe()["tile"]
+        for f in fields:
+            assert t[f] == [flat(e, g[key]["j_bits"]) for e in g[key][f]], (key, f)
+    assert t["rounds"] == g["GV7_config2"]["rounds"]

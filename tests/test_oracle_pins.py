@@ -585,3 +585,50 @@ def test_oracle_mma_operand_matches_ptx(bits):
         i, lane = h & ((1 << len(B.dim_bits("reg"))) - 1), h >> len(B.dim_bits("reg"))
         g, t = lane // 4, lane % 4
         assert O.logical_coords(B.out_dims, O.apply(B, h)) == (e * t + i % e + 4 * e * (i // e), g)
+
+
+# ----------------------------------------------------------------------------- GV6-GV8
+def _flat(expr, j_bits):
+    """'j3^i3' -> flat logical value (j_k = 2^k, i_k = 2^(k + j_bits))."""
+    v = 0
+    for term in expr.split("^"):
+        k = int(term[1:])
+        v ^= 1 << (k if term[0] == "j" else k + j_bits)
+    return v
+
+
+def test_gv6_config1_swizzle_columns():
+    """GV6 (hand derivation of P:406-426 on Fig. 1 A -> B, tests/golden/derived_gv6_gv8.json):
+    Vec = [j0, i0], Bank = [j1, j2, j3], Seg = H = [j1^i1, j2^i2, j3^i3], C empty."""
+    g = load("derived_gv6_gv8.json")["GV6_config1"]
+    sw = O.optimal_swizzle(L_of(W.C1_A), L_of(W.C1_B), 4)
+    for key in ("Vec", "Bank", "Seg"):
+        assert sw[key] == [_flat(e, g["j_bits"]) for e in g[key]], key
+    assert sw["C"] == []
+
+
+def test_gv7_config2_shuffle_sets():
+    """GV7 (hand derivation of P:375-387 on config 2): V = [j0], I empty, E, F ascending,
+    G = {e_i ^ f_i}, |R| = 6 -> 64 rounds."""
+    g = load("derived_gv6_gv8.json")["GV7_config2"]
+    sa, sb = W.c2(0)
+    s = O.shuffle_sets(L_of(sa), L_of(sb), 2)
+    for key in ("V", "I", "E", "F", "G"):
+        assert s[key] == [_flat(e, g["j_bits"]) for e in g[key]], key
+    assert len(s["R"]) == g["R_size"] and s["rounds"] == g["rounds"]
+
+
+def test_gv8_config3_swizzle_and_offsets():
+    """GV8 (hand derivation of P:406-426 on config 3): the swizzle columns, and the
+    element offsets of eight logical points under the smem layout (offset bits Vec,
+    Bank, Seg in that order) — S^{-1}(i, j)."""
+    g = load("derived_gv6_gv8.json")["GV8_config3"]
+    sa, sb = W.c3(0)
+    A3, B3 = L_of(sa), L_of(sb)
+    sw = O.optimal_swizzle(A3, B3, 2)
+    for key in ("Vec", "Bank", "Seg"):
+        assert sw[key] == [_flat(e, g["j_bits"]) for e in g[key]], key
+    S = O.smem_layout_from_swizzle(sw, A3.out_dims)
+    for (i, j), off in g["offsets"]:
+        x = np.array([(i << g["j_bits"]) | j], dtype=np.uint64)
+        assert int(O.apply_inverse_all(S, x)[0]) == off, (i, j)
