@@ -60,8 +60,7 @@ void launch_kernel(void* kernel, unsigned grid, unsigned block, void** args, siz
     const char* e = getenv("LL_PDL");
     return !(e && std::string(e) == "0");
   }();
-  cudaLaunchConfig_t cfg;
-  std::memset(&cfg, 0, sizeof cfg);
+  cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(grid);
   cfg.blockDim = dim3(block);
   cfg.dynamicSmemBytes = smem;
@@ -624,7 +623,6 @@ ll_status ll_convert_host(const void* src_host, void* dst_host, void* dev_buf, s
   const TilePlan& T = P.tile;
   // chunks are runs of whole CTA tiles, contiguous in both buffers: the grid bits must be
   // the top bits of src and dst, in the same order
-  const int lw = P.w == 1 ? 0 : P.w == 2 ? 1 : P.w == 4 ? 2 : 3;
   u64 ntiles = 1, tile_src = P.src_elems * P.w, tile_dst = P.dst_elems * P.w;
   if (P.exec == EXEC_TILE) {
     const size_t g = T.grid_dst_bit.size();
@@ -635,7 +633,6 @@ ll_status ll_convert_host(const void* src_host, void* dst_host, void* dev_buf, s
     ntiles = u64(1) << g;
     tile_src >>= g;
     tile_dst >>= g;
-    (void)lw;
   }
   if (reinterpret_cast<uintptr_t>(dev_buf) & 15) fail(LL_ERR_MISALIGNED, "ll_convert_host: dev_buf must be 16-byte aligned");
   const u64 slot_bytes = (dev_buf_bytes / u64(n_streams)) & ~u64(255);   // 256-byte aligned slots
