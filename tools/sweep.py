@@ -78,6 +78,8 @@ def main():
         return thread_bytes_sweep()
     if "tune" in only:
         return autotune_sweep()
+    if "big" in only:
+        return big_configs()
     if "all" not in only and "conv" not in only:
         return gather_reduce()
     # raw copy roofline reference
@@ -184,6 +186,14 @@ def autotune_sweep():
                           "candidates": d.get("autotune")}), flush=True)
         del src, dst
         torch.cuda.empty_cache()
+
+
+def big_configs():
+    """The 1-2 GiB conversions only (for A/B tests of code-generation knobs)."""
+    for name, (sa, sb), w in [("c2", W.c2(16), 2), ("c3", W.c3(14), 2), ("c1b", W.c1_batched(20), 4),
+                              ("c5T", W.c5T(0), 2), ("n1", W.n1_preshuffle(14, 14), 2),
+                              ("n2", W.n2_tmem_epilogue(13), 4)]:
+        conv_case(name, sa, sb, w)
 
 
 def latency_and_ksweep():
