@@ -243,9 +243,20 @@ def other_configs(ll, W, torch, peak):
         ms = _time_stream(g1, torch)
         d = p.describe()
         gbs = 12 * n / ms / 1e6
+        # context: PyTorch's own gather on the logical [4096*128, 32] view, same bytes,
+        # same 4-set rotation (a library kernel for the op, not the roofline)
+        tsets = [(s[0].view(-1, 32), s[1].view(-1, 32).to(torch.int64) & 31, s[2].view(-1, 32)) for s in sets]
+
+        def tg():
+            s = tsets[it[0] % 4]
+            it[0] += 1
+            torch.gather(s[0], 1, s[1], out=s[2])
+        ms_t = _time_stream(tg, torch)
         out.append({"workload": f"config 4 gather: [4096,4096] fp32, {fam} [128,32] tiles", "class": "gather",
                     "executed": d["exchange"] + (" (TMA stages)" if d.get("tma") else ""), "ms": round(ms, 4),
-                    "GBps": round(gbs, 1), "frac": round(gbs / peak, 3)})
+                    "GBps": round(gbs, 1), "frac": round(gbs / peak, 3),
+                    "torch_gather_same_bytes_GBps": round(12 * n / ms_t / 1e6, 1)})
+        del tsets
         L = ll.Layout.from_spec(W.c4("reduce", fam))
         p = ll.ll_plan_reduce(L, 1)
         rsets = [(torch.rand(n, device="cuda"), torch.empty(p.out_elems(), device="cuda")) for _ in range(4)]
@@ -256,9 +267,17 @@ def other_configs(ll, W, torch, peak):
             ll.ll_reduce(s[0], s[1], p)
         ms = _time_stream(r1, torch)
         gbs = (4 * n + 4 * p.out_elems()) / ms / 1e6
+
+        # context: PyTorch's own sum over the logical [4096, 32, 128] view (same bytes)
+        def tr():
+            s = rsets[it[0] % 4]
+            it[0] += 1
+            torch.sum(s[0].view(4096, 32, 128), dim=2, out=s[1].view(4096, 32))
+        ms_t = _time_stream(tr, torch)
         out.append({"workload": f"config 4 reduce: [4096,4096] fp32 -> [4096,32], {fam} [128,128] tiles",
                     "class": "reduce", "executed": "tree + shfl.bfly" + (" (TMA stages)" if p.describe().get("tma") else ""),
-                    "ms": round(ms, 4), "GBps": round(gbs, 1), "frac": round(gbs / peak, 3)})
+                    "ms": round(ms, 4), "GBps": round(gbs, 1), "frac": round(gbs / peak, 3),
+                    "torch_sum_same_bytes_GBps": round((4 * n + 4 * p.out_elems()) / ms_t / 1e6, 1)})
         del sets, rsets
     torch.cuda.empty_cache()
     return out
