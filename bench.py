@@ -178,6 +178,45 @@ def _time_stream(fn, torch, samples=10, batch=20, warmup=3):
     return ts[len(ts) // 2]
 
 
+def torch_permute_baseline(torch, A_spec, B_spec, src, steps=5):
+    """Context for the headline: the same conversion done the way a PyTorch user would —
+    the packed buffer viewed as a tensor of 2-sized dims, permuted and made contiguous
+    (torch's generic strided copy).  For bijective layouts the dst packed bit k holds the
+    logical bit B[k], found at src packed bit A.index(B[k]) (spec bookkeeping only);
+    runs of bits that stay adjacent are merged into one dim."""
+    a_bits = [b for _, bits in A_spec["in"] for b in bits]
+    b_bits = [b for _, bits in B_spec["in"] for b in bits]
+    perm = [a_bits.index(x) for x in b_bits]          # dst packed bit -> src packed bit
+    n = len(perm)
+    runs = []                                           # (src lo bit, length) in dst bit order
+    k = 0
+    while k < n:
+        j = k
+        while j + 1 < n and perm[j + 1] == perm[j] + 1:
+            j += 1
+        runs.append((perm[k], j - k + 1))
+        k = j + 1
+    src_runs = sorted(runs)                             # src dims, least significant first
+    shape = [1 << ln for _, ln in reversed(src_runs)]
+    dim_of = {lo: len(src_runs) - 1 - i for i, (lo, _) in enumerate(src_runs)}
+    order = [dim_of[lo] for lo, _ in reversed(runs)]   # dst dims, most significant first
+    x = src.view(*shape)
+
+    def run():
+        return x.permute(*order).contiguous()
+    y = run()
+    torch.cuda.synchronize()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record()
+    for _ in range(steps):
+        y = run()
+    b.record()
+    torch.cuda.synchronize()
+    ms = a.elapsed_time(b) / steps
+    return {"impl": "torch: packed src viewed as %d dims, permute(...).contiguous()" % len(shape),
+            "GBps": round(2 * src.numel() * src.element_size() / (ms / 1e3) / 1e9, 1), "ms": round(ms, 4)}, y
+
+
 def other_configs(ll, W, torch, peak):
     """The other BASELINE configs (1, 3, 4, 5) measured live on this GPU, each against
     the same copy roofline: GB/s = algorithmic bytes / median time per call.  Inputs
@@ -200,8 +239,14 @@ def other_configs(ll, W, torch, peak):
             ex = "peer stores: one %s tile kernel per rank" % d["fused"]["tile"]["xchg"]
         else:
             ex = d["exec"]
-        out.append({"workload": name, "class": d["class"], "executed": ex, "ms": round(ms, 4),
-                    "GBps": round(gbs, 1), "frac": round(gbs / peak, 3)})
+        entry = {"workload": name, "class": d["class"], "executed": ex, "ms": round(ms, 4),
+                 "GBps": round(gbs, 1), "frac": round(gbs / peak, 3)}
+        if comm is None:
+            tb, y = torch_permute_baseline(torch, sa, sb, src)
+            entry["torch_permute_GBps"] = tb["GBps"]
+            entry["torch_permute_matches"] = bool(torch.equal(y.reshape(-1), dst))
+            del y
+        out.append(entry)
         del src, dst
 
     # config 1 single tile: latency of one conversion in a CUDA graph of 1000
@@ -490,6 +535,11 @@ def main():
         if c5 is not None:
             line["config5_nvlink"] = c5
         if world == 1 and not args.no_configs:
+            # the library baseline must produce the same bytes as our kernel
+            tb, y = torch_permute_baseline(torch, A_spec, B_spec, src)
+            tb["matches"] = bool(torch.equal(y.reshape(-1), dst))
+            line["torch_baseline"] = tb
+            del y
             del src, dst
             torch.cuda.empty_cache()
             line["configs"] = other_configs(ll, W, torch, peak)
