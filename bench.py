@@ -178,7 +178,7 @@ def _time_stream(fn, torch, samples=10, batch=20, warmup=3):
     return ts[len(ts) // 2]
 
 
-def torch_permute_baseline(torch, A_spec, B_spec, src, steps=5):
+def torch_permute_baseline(torch, A_spec, B_spec, src, w, steps=5):
     """Context for the headline: the same conversion done the way a PyTorch user would —
     the packed buffer viewed as a tensor of 2-sized dims, permuted and made contiguous
     (torch's generic strided copy).  For bijective layouts the dst packed bit k holds the
@@ -200,7 +200,8 @@ def torch_permute_baseline(torch, A_spec, B_spec, src, steps=5):
     shape = [1 << ln for _, ln in reversed(src_runs)]
     dim_of = {lo: len(src_runs) - 1 - i for i, (lo, _) in enumerate(src_runs)}
     order = [dim_of[lo] for lo, _ in reversed(runs)]   # dst dims, most significant first
-    x = src.view(*shape)
+    et = {1: torch.uint8, 2: torch.int16, 4: torch.int32, 8: torch.int64}[w]
+    x = src.view(et).view(*shape)
 
     def run():
         return x.permute(*order).contiguous()
@@ -214,7 +215,8 @@ def torch_permute_baseline(torch, A_spec, B_spec, src, steps=5):
     torch.cuda.synchronize()
     ms = a.elapsed_time(b) / steps
     return {"impl": "torch: packed src viewed as %d dims, permute(...).contiguous()" % len(shape),
-            "GBps": round(2 * src.numel() * src.element_size() / (ms / 1e3) / 1e9, 1), "ms": round(ms, 4)}, y
+            "GBps": round(2 * src.numel() * src.element_size() / (ms / 1e3) / 1e9, 1), "ms": round(ms, 4)}, \
+        y.reshape(-1).view(src.dtype)
 
 
 def other_configs(ll, W, torch, peak):
@@ -242,9 +244,9 @@ def other_configs(ll, W, torch, peak):
         entry = {"workload": name, "class": d["class"], "executed": ex, "ms": round(ms, 4),
                  "GBps": round(gbs, 1), "frac": round(gbs / peak, 3)}
         if comm is None:
-            tb, y = torch_permute_baseline(torch, sa, sb, src)
+            tb, y = torch_permute_baseline(torch, sa, sb, src, w)
             entry["torch_permute_GBps"] = tb["GBps"]
-            entry["torch_permute_matches"] = bool(torch.equal(y.reshape(-1), dst))
+            entry["torch_permute_matches"] = bool(torch.equal(y, dst))
             del y
         out.append(entry)
         del src, dst
@@ -536,8 +538,8 @@ def main():
             line["config5_nvlink"] = c5
         if world == 1 and not args.no_configs:
             # the library baseline must produce the same bytes as our kernel
-            tb, y = torch_permute_baseline(torch, A_spec, B_spec, src)
-            tb["matches"] = bool(torch.equal(y.reshape(-1), dst))
+            tb, y = torch_permute_baseline(torch, A_spec, B_spec, src, w)
+            tb["matches"] = bool(torch.equal(y, dst))
             line["torch_baseline"] = tb
             del y
             del src, dst
