@@ -889,6 +889,60 @@ def reduce_fixed_order_fp32(L: Layout, axis: int, src: np.ndarray) -> np.ndarray
 
 
 # --------------------------------------------------------------------------------------
+# O13  Scan (inclusive prefix sum) along an axis inside each tile ("reduction and
+#      scan operations").  The paper fixes no scan algorithm; reading
+#      R-scan: the in-tile axis is the low K bits of the axis coordinate
+#      (as for gather / reduce), and the fp32 order is the bit-doubling recurrence below,
+#      written in logical coordinates so that it does not depend on any hardware mapping.
+# --------------------------------------------------------------------------------------
+
+def _scan_setup(L: Layout, axis: int, src: np.ndarray, dtype):
+    shape = [1 << b for _, b in L.out_dims]
+    x_of_h = image_table(L).astype(np.int64)
+    T = np.empty(int(np.prod(shape)), dtype=dtype)
+    T[x_of_h] = np.asarray(src, dtype=dtype).reshape(-1)
+    axis_shift = sum(b for _, b in L.out_dims[axis + 1:])
+    axis_mask = ((1 << L.out_dims[axis][1]) - 1) << axis_shift
+    nonblock = [k for n, _ in L.in_dims if n not in ("block", "dev") for k in L.dim_bits(n)]
+    kbits = len([k for k in nonblock if L.cols[k] & axis_mask])
+    T = T.reshape(shape[:axis] + [shape[axis] >> kbits, 1 << kbits] + shape[axis + 1:])
+    return T, kbits, x_of_h, shape
+
+
+def scan_ref_fp64(L: Layout, axis: int, src: np.ndarray) -> np.ndarray:
+    """out[x] = sum of T[x with axis coordinate a'] over the a' of x's tile with a' <= a(x)
+    (inclusive), in fp64, returned packed in L like the input (library cumsum)."""
+    T, kbits, x_of_h, shape = _scan_setup(L, axis, src, np.float64)
+    out = np.cumsum(T, axis=axis + 1).reshape(-1)
+    return out[x_of_h]
+
+
+def scan_bitdoubling_fp32(L: Layout, axis: int, src: np.ndarray) -> np.ndarray:
+    """The fixed-order fp32 scan (reading R-scan), in logical coordinates, step by step:
+    for t = 0 .. K_bits-1, every element whose in-tile axis coordinate a has bit t set
+    adds the value, before this step, of the last element of the lower half of its
+    aligned 2^(t+1)-block, a' = (a with bit t cleared) | (2^t - 1):
+        v[a] <- v[a] + v[a']   (fp32, round to nearest; simultaneous update).
+    After step t every element holds the inclusive sum of its aligned 2^(t+1)-block
+    prefix; after the last step, the in-tile inclusive prefix sum."""
+    T, kbits, x_of_h, shape = _scan_setup(L, axis, src, np.float32)
+    ax = axis + 1
+    K = 1 << kbits
+    v = T.copy()
+    a = np.arange(K)
+    for t in range(kbits):
+        upper = (a >> t) & 1 == 1
+        partner = (a & ~((2 << t) - 1)) | ((1 << t) - 1)
+        src_vals = np.take(v, partner[upper], axis=ax)
+        cur = np.take(v, a[upper], axis=ax)
+        new = (cur + src_vals).astype(np.float32)
+        idx = [slice(None)] * v.ndim
+        idx[ax] = a[upper]
+        v[tuple(idx)] = new
+    return v.reshape(-1)[x_of_h]
+
+
+# --------------------------------------------------------------------------------------
 # O12  Distributed view (dev input dimension declared last, SURVEY §8(b), G21)
 # --------------------------------------------------------------------------------------
 

@@ -632,3 +632,46 @@ def test_gv8_config3_swizzle_and_offsets():
     for (i, j), off in g["offsets"]:
         x = np.array([(i << g["j_bits"]) | j], dtype=np.uint64)
         assert int(O.apply_inverse_all(S, x)[0]) == off, (i, j)
+
+
+# ----------------------------------------------------------------------------- O13 scan
+@pytest.mark.parametrize("family", ["mma", "blocked"])
+def test_scan_fp64_is_cumsum_per_tile(family):
+    """O13 fp64 reference against a hand loop: every output is the sum of its tile's
+    axis prefix (brute force over a few points), computed without numpy.cumsum."""
+    OL = L_of(W.c4("reduce", family, n_i=8, n_j=8))
+    rng = np.random.default_rng(21)
+    T = rng.random(1 << OL.d_out)
+    src = O.pack(OL, T)
+    out = O.scan_ref_fp64(OL, 1, src)
+    x_of_h = O.image_table(OL).astype(np.int64)
+    for h in rng.integers(0, src.size, size=64):
+        x = int(x_of_h[h])
+        i, j = x >> 8, x & 255
+        j0 = j & ~127
+        want = sum(T[(i << 8) | jj] for jj in range(j0, j + 1))
+        assert abs(out[h] - want) <= 1e-12 * max(1.0, want)
+
+
+@pytest.mark.parametrize("family", ["mma", "blocked"])
+def test_scan_fp32_recurrence_exact_on_integers(family):
+    """O13 fp32 bit-doubling recurrence: on integer-valued inputs every partial sum is
+    exact in fp32 (< 2^24), so it must equal the integer cumulative sum exactly — any
+    wrong partner index, step order or tile boundary fails."""
+    OL = L_of(W.c4("reduce", family, n_i=8, n_j=8))
+    rng = np.random.default_rng(22)
+    T = rng.integers(0, 1000, size=1 << OL.d_out).astype(np.float32)
+    src = O.pack(OL, T)
+    got = O.scan_bitdoubling_fp32(OL, 1, src)
+    want = O.scan_ref_fp64(OL, 1, src)
+    assert np.array_equal(got.astype(np.float64), want)
+
+
+def test_scan_fp32_recurrence_within_bound():
+    """On U[0,1) inputs the recurrence (depth K_bits = 7 additions per element at most)
+    stays within 7 * 2^-24 relative of the fp64 prefix sums."""
+    OL = L_of(W.c4("reduce", "mma", n_i=8, n_j=8))
+    src = O.pack(OL, np.random.default_rng(23).random(1 << OL.d_out, dtype=np.float32))
+    got = O.scan_bitdoubling_fp32(OL, 1, src).astype(np.float64)
+    ref = O.scan_ref_fp64(OL, 1, src)
+    assert np.all(np.abs(got - ref) <= 7 * 2.0 ** -24 * np.abs(ref) + 1e-30)
