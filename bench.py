@@ -329,7 +329,28 @@ def other_configs(ll, W, torch, peak):
                     "class": "reduce", "executed": "tree + shfl.bfly" + (" (TMA stages)" if p.describe().get("tma") else ""),
                     "ms": round(ms, 4), "GBps": round(gbs, 1), "frac": round(gbs / peak, 3),
                     "torch_sum_same_bytes_GBps": round((4 * n + 4 * p.out_elems()) / ms_t / 1e6, 1)})
-        del sets, rsets
+        # scan (N3): inclusive prefix sum along the axis inside each [128, 128] tile
+        p = ll.ll_plan_scan(L, 1)
+        ssets = [(rs[0], torch.empty_like(rs[0])) for rs in rsets]
+
+        def s1():
+            s = ssets[it[0] % 4]
+            it[0] += 1
+            ll.ll_scan(s[0], s[1], p)
+        ms = _time_stream(s1, torch)
+        gbs = 8 * n / ms / 1e6
+
+        def ts():
+            s = ssets[it[0] % 4]
+            it[0] += 1
+            torch.cumsum(s[0].view(4096, 32, 128), dim=2, out=s[1].view(4096, 32, 128))
+        ms_t = _time_stream(ts, torch)
+        d = p.describe()
+        out.append({"workload": f"config 4 scan (N3): [4096,4096] fp32 inclusive prefix sum inside {fam} [128,128] tiles",
+                    "class": "scan", "executed": f"{d['steps']} bit-doubling steps, {d['shuffles_per_elem']} shuffles/elem",
+                    "ms": round(ms, 4), "GBps": round(gbs, 1), "frac": round(gbs / peak, 3),
+                    "torch_cumsum_same_bytes_GBps": round(8 * n / ms_t / 1e6, 1)})
+        del sets, rsets, ssets
     torch.cuda.empty_cache()
     return out
 

@@ -286,6 +286,19 @@ ll_status ll_plan_reduce_out_elems(const ll_plan* plan, size_t* n);
  * its block part (one write per element). */
 ll_status ll_reduce(const float* src, float* dst, const ll_plan* plan, void* stream);
 
+/* ---------------------------------------------------------------- scan --
+ * ll_plan_scan ("reduction and scan operations").  Inclusive
+ * prefix sum (fp32) along `axis` inside each CTA tile of L (the in-tile axis bits are
+ * the low bits of the axis coordinate, as for gather / reduce; each tile's scan starts
+ * from zero).  The fp32 order is fixed (reading R-scan): for axis bit t =
+ * 0, 1, ..., an element whose axis bit t is set adds the value of the last element of
+ * the lower half of its aligned 2^(t+1)-block.  L: a distributed layout (duplicated
+ * positions, zero columns, each get the same value); the in-tile axis bits must be
+ * register or lane bits (LL_ERR_UNSUPPORTED for warp bits). */
+ll_status ll_plan_scan(const ll_layout* L, int axis, const ll_plan_opts* opts, ll_plan** plan);
+/* src, dst: fp32 packed in L (same positions); must not overlap partially. */
+ll_status ll_scan(const float* src, float* dst, const ll_plan* plan, void* stream);
+
 /* ---------------------------------------------------------------- comm --
  * NCCL communicator for DEVICE plans: nccl_unique_id is the 128-byte
  * ncclUniqueId produced by rank 0 and broadcast by the caller (e.g. over a torch

@@ -87,6 +87,8 @@ _sig = {
     "ll_plan_reduce": [_P, C.c_int, C.POINTER(_Opts), _PP],
     "ll_plan_reduce_out_elems": [_P, C.POINTER(C.c_size_t)],
     "ll_reduce": [_P, _P, _P, _P],
+    "ll_plan_scan": [_P, C.c_int, C.POINTER(_Opts), _PP],
+    "ll_scan": [_P, _P, _P, _P],
     "ll_plan_simulate": [_P, _P, _P],
     "ll_comm_create": [_P, C.c_int, C.c_int, _PP],
     "ll_comm_get_unique_id": [_P],
@@ -573,6 +575,17 @@ def ll_plan_reduce(L: Layout, axis: int, **opts) -> Plan:
     o = _opts(**opts)
     _check(_lib.ll_plan_reduce(L.handle, int(axis), C.byref(o), C.byref(h)))
     return Plan(h, "reduce")
+
+
+def ll_plan_scan(L: Layout, axis: int, **opts) -> Plan:
+    h = C.c_void_p()
+    o = _opts(**opts)
+    _check(_lib.ll_plan_scan(L.handle, int(axis), C.byref(o), C.byref(h)))
+    return Plan(h, "scan")
+
+
+def ll_scan(src, dst, plan: Plan, stream=None):
+    _check(_lib.ll_scan(_ptr(src), _ptr(dst), plan.handle, _stream_ptr(stream)))
 
 
 def ll_reduce(src, dst, plan: Plan, stream=None):

@@ -460,6 +460,16 @@ ll_status ll_plan_describe(const ll_plan* p, char* json, size_t cap) {
       << ",\"exchange\":\"" << (G.smem ? "smem" : "shuffle") << "\",\"tma\":" << (G.tma ? "true" : "false") << ",\"shuffles_per_elem\":" << (G.smem ? 0 : (1 << G.cand_bits))
       << ",\"ctas\":" << (u64(1) << G.grid_bit.size()) << "}";
     s = o.str();
+  } else if (p->kind == 3) {
+    const ScanPlan& S = *p->scan;
+    std::ostringstream o;
+    o << "{\"kind\":\"scan\",\"sigma\":\"" << (S.sigma ? "faithful" : "coalesced") << "\",\"R\":" << S.R
+      << ",\"warp_bits\":" << S.Wb << ",\"K_bits\":" << S.K_bits << ",\"steps\":" << S.K_bits
+      << ",\"axis_hw\":" << "[";
+    for (size_t t = 0; t < S.axis_hw.size(); ++t) o << (t ? "," : "") << S.axis_hw[t];
+    o << "],\"shuffles_per_elem\":" << double(S.shfl_per_thread) / double(1 << S.R)
+      << ",\"ctas\":" << (u64(1) << S.grid_bit.size()) << "}";
+    s = o.str();
   } else {
     const ReducePlan& Rp = *p->reduce;
     std::ostringstream o;
@@ -484,6 +494,7 @@ ll_status ll_plan_source(const ll_plan* p, char* buf, size_t cap, size_t* needed
   if (p->kind == 0 && p->cp().fused) s = p->cp().fused->source;
   if (p->kind == 1) s = codegen_gather(*p->gather);
   if (p->kind == 2) s = codegen_reduce(*p->reduce);
+  if (p->kind == 3) s = codegen_scan(*p->scan);
   if (needed) *needed = s.size() + 1;
   if (buf && cap) {
     std::strncpy(buf, s.c_str(), cap - 1);
@@ -503,6 +514,10 @@ ll_status ll_plan_prepare(ll_plan* p) {
   }
   if (p->kind == 1) {
     ensure_gather_kernel(*p->gather);
+  }
+  if (p->kind == 3) {
+    std::lock_guard<std::mutex> g(p->scan->mu);
+    if (!p->scan->kernel) p->scan->kernel = jit_kernel(codegen_scan(*p->scan), "ll_scan_kernel");
   }
   if (p->kind == 2) {
     std::lock_guard<std::mutex> g(p->reduce->mu);
@@ -528,6 +543,7 @@ ll_status ll_jit_precompile(const ll_plan* p) {
   }
   if (p->kind == 1) jit_precompile(codegen_gather(*p->gather), "ll_gather_kernel");
   if (p->kind == 2) jit_precompile(codegen_reduce(*p->reduce), "ll_reduce_kernel");
+  if (p->kind == 3) jit_precompile(codegen_scan(*p->scan), "ll_scan_kernel");
   LL_CATCH
 }
 
@@ -690,6 +706,32 @@ ll_status ll_gather(const void* src, const int32_t* idx, void* dst, const ll_pla
   }
   launch_kernel(G.kernel, grid, 32u << G.Wb, args, size_t(G.smem_bytes), static_cast<cudaStream_t>(stream),
                 "cudaLaunchKernelEx(ll_gather_kernel)");
+  LL_CATCH
+}
+
+ll_status ll_plan_scan(const ll_layout* L, int axis, const ll_plan_opts* opts, ll_plan** plan) {
+  LL_TRY
+  if (!L || !plan) fail(LL_ERR_INVALID_ARG, "null argument");
+  auto h = std::make_unique<ll_plan>();
+  h->kind = 3;
+  h->scan = plan_scan(L->L, axis, opts);
+  *plan = h.release();
+  LL_CATCH
+}
+
+ll_status ll_scan(const float* src, float* dst, const ll_plan* p, void* stream) {
+  LL_TRY
+  if (!p || p->kind != 3) fail(LL_ERR_INVALID_ARG, "not a scan plan");
+  if (!src || !dst) fail(LL_ERR_INVALID_ARG, "null buffer");
+  if ((reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst)) & 15)
+    fail(LL_ERR_MISALIGNED, "buffers must be 16-byte aligned");
+  ll_status st = ll_plan_prepare(const_cast<ll_plan*>(p));
+  if (st != LL_OK) return st;
+  ScanPlan& S = *p->scan;
+  unsigned long long nt = u64(1) << S.grid_bit.size();
+  void* args[] = {const_cast<float**>(&src), &dst, &nt};
+  launch_kernel(S.kernel, grid_for(nt), 32u << S.Wb, args, 0, static_cast<cudaStream_t>(stream),
+                "cudaLaunchKernelEx(ll_scan_kernel)");
   LL_CATCH
 }
 

@@ -169,6 +169,24 @@ std::string codegen_gather(const GatherPlan& G) {
   return o.str();
 }
 
+std::string codegen_scan(const ScanPlan& S) {
+  std::ostringstream o;
+  o << "struct P {\n";
+  o << icon("W", 4) << icon("R", S.R) << icon("WB", S.Wb) << icon("VLD", S.v) << icon("NW", 1 << S.R);
+  o << "  static constexpr bool LD_L1 = " << (S.sigma == SIGMA_FAITHFUL ? "true" : "false") << ";\n";
+  o << icon("ST_HINT", st_hint());
+  std::vector<u64> ldc;
+  for (int b : S.hw_bit) ldc.push_back(u64(4) << b);
+  o << arr("u64", "LD_COL", ldc);
+  emit_grid(o, S.grid_bit, S.grid_bit, 2);
+  o << icon("KB", S.K_bits) << arr("int", "AXIS_HW", S.axis_hw);
+  o << "};\n";
+  o << "extern \"C\" __global__ void __launch_bounds__(" << (32 << S.Wb)
+    << ") ll_scan_kernel(const u8* __restrict__ src, u8* __restrict__ dst, u64 ntiles) {\n"
+    << "  ll_scan_body<P>(src, dst, ntiles);\n}\n";
+  return o.str();
+}
+
 std::string codegen_reduce(const ReducePlan& Rp) {
   std::ostringstream o;
   o << "struct P {\n";

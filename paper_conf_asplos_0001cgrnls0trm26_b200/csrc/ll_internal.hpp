@@ -278,6 +278,24 @@ std::unique_ptr<ReducePlan> plan_reduce(const Layout& L, int axis, const ll_plan
 
 // ------------------------------------------------------------------ codegen / jit
 std::string codegen_tile(const ConvPlan& P);
+// In-tile inclusive scan along an axis ("reduction and scan operations"; §8(f)
+// N3), fixed fp32 order = the bit-doubling recurrence of reading R-scan.
+struct ScanPlan {
+  Layout L;
+  int axis = 0;
+  int sigma = SIGMA_COALESCED;
+  int R = 0, Wb = 0, v = 0;
+  int K_bits = 0;
+  std::vector<int> hw_bit;     // kernel bit -> packed bit (src and dst)
+  std::vector<int> grid_bit;   // CTA index bit -> packed bit
+  std::vector<int> axis_hw;    // logical axis bit t -> kernel bit (reg < R or lane)
+  int shfl_per_thread = 0;     // shuffles per thread per tile
+  std::string source;
+  void* kernel = nullptr;
+  std::mutex mu;
+};
+std::unique_ptr<ScanPlan> plan_scan(const Layout& L, int axis, const ll_plan_opts* opts);
+std::string codegen_scan(const ScanPlan& P);
 std::string codegen_gather(const GatherPlan& P);
 std::string codegen_reduce(const ReducePlan& P);
 // Compile (or fetch from cache) and return a cudaKernel_t for `source`.
@@ -291,12 +309,13 @@ void simulate_tile(const ConvPlan& P, const uint8_t* src, uint8_t* dst);
 
 struct ll_layout { ll::Layout L; };
 struct ll_plan {
-  int kind;   // 0 conv, 1 gather, 2 reduce
+  int kind;   // 0 conv, 1 gather, 2 reduce, 3 scan
   std::unique_ptr<ll::ConvPlan> conv;
   ll::ConvPlan* borrowed = nullptr;          // sub-plan handles (DEVICE stages)
   std::unique_ptr<ll_plan> stage[2];         // pack / unpack views of a DEVICE plan
   std::unique_ptr<ll::GatherPlan> gather;
   std::unique_ptr<ll::ReducePlan> reduce;
+  std::unique_ptr<ll::ScanPlan> scan;
   ll::ConvPlan& cp() const { return borrowed ? *borrowed : *conv; }
 };
 struct ll_comm {

@@ -875,3 +875,75 @@ __device__ __forceinline__ void ll_reduce_body(const float* __restrict__ src, fl
     }
   }
 }
+
+// ------------------------------------------------------------------ scan (N3)
+// P:308 / SURVEY §8(f) N3: inclusive fp32 prefix sum along the axis inside each tile,
+// in the fixed order of reading R-scan: for logical axis bit S = 0, 1,
+// ..., an element whose bit S is set adds the value (before this step) of the last
+// element of the lower half of its aligned 2^(S+1)-block — the position with the
+// hardware bit of S cleared and the hardware bits of the lower axis bits set.  Those
+// partner positions have bit S clear, so no step overwrites a value it still reads.
+template <class P, int S> struct ScanStep {
+  static constexpr int HB = P::AXIS_HW[S];
+  static constexpr bool HREG = HB < P::R;
+  static constexpr u32 low_reg() { u32 m = 0; for (int q = 0; q < S; ++q) if (P::AXIS_HW[q] < P::R) m |= 1u << P::AXIS_HW[q]; return m; }
+  static constexpr u32 low_lane() { u32 m = 0; for (int q = 0; q < S; ++q) if (P::AXIS_HW[q] >= P::R) m |= 1u << (P::AXIS_HW[q] - P::R); return m; }
+  static constexpr bool SHFL = !HREG || low_lane() != 0;
+};
+
+template <class P>
+__device__ __forceinline__ void ll_scan_body(const u8* __restrict__ src, u8* __restrict__ dst, u64 ntiles) {
+  ll_pdl_begin();
+  const u32 lane = threadIdx.x & 31u;
+  const u32 warp = threadIdx.x >> 5;
+  const u64 thr = thread_base<P, true>(lane, warp);
+  for (u64 t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    const u64 base = tile_base<P, true>(t) ^ thr;
+    u32 r[P::NW];
+    static_for<(1 << (P::R - P::VLD))>([&](auto k) {
+      constexpr int K = decltype(k)::value;
+      load_vec<4, P::VLD, K, P::NW, P::LD_L1>(r, src + base + LdOff<P, K>::value());
+    });
+    static_for<P::KB>([&](auto s) {
+      using St = ScanStep<P, decltype(s)::value>;
+      constexpr int HB = St::HB;
+      constexpr u32 LR = St::low_reg(), LL = St::low_lane();
+      if constexpr (!St::SHFL) {
+        // bit S and every lower axis bit live in this thread's registers
+        static_for<P::NW>([&](auto e) {
+          constexpr int E = decltype(e)::value;
+          if constexpr ((E >> HB) & 1) {
+            constexpr int E2 = (E & ~(1 << HB)) | int(LR);
+            r[E] = __float_as_uint(__fadd_rn(__uint_as_float(r[E]), __uint_as_float(r[E2])));
+          }
+        });
+      } else if constexpr (St::HREG) {
+        // bit S in registers, some lower axis bit in lanes: shuffle from lane | LL
+        const int sl = int(lane | LL);
+        static_for<P::NW>([&](auto e) {
+          constexpr int E = decltype(e)::value;
+          if constexpr ((E >> HB) & 1) {
+            constexpr int E2 = (E & ~(1 << HB)) | int(LR);
+            const float x = __shfl_sync(0xffffffffu, __uint_as_float(r[E2]), sl);
+            r[E] = __float_as_uint(__fadd_rn(__uint_as_float(r[E]), x));
+          }
+        });
+      } else {
+        // bit S is a lane bit: every slot shuffles; the upper lanes add
+        constexpr int LB = HB - P::R;
+        const int sl = int((lane & ~(1u << LB)) | LL);
+        const bool upper = (lane >> LB) & 1u;
+        static_for<P::NW>([&](auto e) {
+          constexpr int E = decltype(e)::value;
+          constexpr int E2 = E | int(LR);
+          const float x = __shfl_sync(0xffffffffu, __uint_as_float(r[E2]), sl);
+          if (upper) r[E] = __float_as_uint(__fadd_rn(__uint_as_float(r[E]), x));
+        });
+      }
+    });
+    static_for<(1 << (P::R - P::VLD))>([&](auto k) {
+      constexpr int K = decltype(k)::value;
+      store_vec<4, P::VLD, K, P::NW, P::ST_HINT>(r, dst + base + LdOff<P, K>::value());
+    });
+  }
+}

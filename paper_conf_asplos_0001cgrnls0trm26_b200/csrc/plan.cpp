@@ -1059,4 +1059,58 @@ std::unique_ptr<ReducePlan> plan_reduce(const Layout& L, int axis, const ll_plan
   return Rp;
 }
 
+// ---------------------------------------------------------------------------
+// Scan: inclusive prefix sum along `axis` inside each CTA
+// tile, fp32, in the order of reading R-scan: for logical axis bit t = 0, 1, ...,
+// every element with bit t set adds the value of the last element of the lower half
+// of its aligned 2^(t+1)-block.  In the kernel layout L∘σ that partner differs in the
+// hardware bit of t (cleared) and the hardware bits of the lower axis bits (set): a
+// register read when they are all registers, else a warp shuffle from the partner lane.
+// Duplicated (zero-column) positions compute identical values from identical
+// inputs and store their own copies.
+// ---------------------------------------------------------------------------
+std::unique_ptr<ScanPlan> plan_scan(const Layout& L, int axis, const ll_plan_opts* opts) {
+  if (axis < 0 || axis >= int(L.out.size())) fail(LL_ERR_INVALID_ARG, "axis out of range");
+  if (!L.distributed()) fail(LL_ERR_UNSUPPORTED, "scan: L must be a distributed layout (Def 4.10)");
+  if (L.in_bits("lane") != 5) fail(LL_ERR_UNSUPPORTED, "scan: 5 lane bits required");
+  if (L.in.size() < 1 || L.in[0].name != "reg") fail(LL_ERR_UNSUPPORTED, "scan: dims must be reg, lane, warp[, block]");
+  auto S = std::make_unique<ScanPlan>();
+  S->L = L; S->axis = axis;
+  const int sh = L.out_shift(axis), ab = L.out[axis].bits;
+  const u64 amask = ((u64(1) << ab) - 1) << sh;
+  const int R = L.in_bits("reg");
+  S->R = R;
+  S->Wb = L.in_bits("warp");
+  int K = 0;
+  for (int k : bits_at_level(L, 0, 2)) if (L.cols[k] & amask) ++K;
+  S->K_bits = K;
+  S->v = std::min(2, R);
+  const int sigma = opts ? opts->sigma : 0;
+  if (sigma == SIGMA_FAITHFUL) {
+    S->sigma = SIGMA_FAITHFUL;
+    for (int k : bits_at_level(L, 0, 2)) S->hw_bit.push_back(k);
+  } else {
+    // axis bits stay in registers where possible (register steps need no shuffle)
+    S->hw_bit = sigma_line(L, S->v, [&](int k) { return L.cols[k] != 0 && !(L.cols[k] & amask); });
+  }
+  const int n = int(S->hw_bit.size());
+  for (int t = 0; t < K; ++t) {
+    int b = -1;
+    for (int q = 0; q < n; ++q) if (L.cols[S->hw_bit[q]] == (u64(1) << (sh + t))) b = q;
+    if (b < 0) fail(LL_ERR_UNSUPPORTED, "scan: in-tile axis bits must be the low axis bits");
+    if (b >= R + 5) fail(LL_ERR_UNSUPPORTED, "scan: an axis bit on the warps is not supported (registers and lanes only)");
+    S->axis_hw.push_back(b);
+  }
+  S->grid_bit = bits_at_level(L, 3, 3);
+  // shuffles per thread per tile: a step needs them when its bit or a lower axis bit is
+  // a lane (all slots when its own bit is a lane, else the slots with the bit set)
+  bool lane_below = false;
+  for (int t = 0; t < K; ++t) {
+    const bool hreg = S->axis_hw[t] < R;
+    if (!hreg || lane_below) S->shfl_per_thread += hreg ? (1 << (R - 1)) : (1 << R);
+    if (!hreg) lane_below = true;
+  }
+  return S;
+}
+
 }  // namespace ll

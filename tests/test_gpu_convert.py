@@ -537,3 +537,50 @@ def test_autotune_bitexact(which):
     d_dst.zero_()
     ll.ll_convert(d_src, d_dst, plan)
     assert np.array_equal(from_device(d_dst, w), O.pack(OB, T))
+
+
+# ---------------------------------------------------------------- N3: scans
+@pytest.mark.parametrize("family", ["mma", "blocked"])
+@pytest.mark.parametrize("sigma", ["coalesced", "faithful"])
+def test_scan_bitexact(family, sigma):
+    """O13: in-tile inclusive scan along the axis (§8(f) N3) on config-4 tiles —
+    bit-equal to the oracle's fixed-order fp32 recurrence (defined in logical
+    coordinates, so independent of σ) and within 7·2^-24 of the fp64 prefix sums."""
+    import torch
+    spec = W.c4("reduce", family, n_i=9, n_j=9)
+    L, OL = both(spec)
+    T = np.random.default_rng(1007).random(1 << OL.d_out, dtype=np.float32)
+    src = O.pack(OL, T)
+    plan = ll.ll_plan_scan(L, 1, sigma=sigma)
+    out = torch.empty(src.size, dtype=torch.float32, device="cuda")
+    ll.ll_scan(torch.from_numpy(src).cuda(), out, plan)
+    got = out.cpu().numpy()
+    rep = O.scan_bitdoubling_fp32(OL, 1, src)
+    assert np.array_equal(got.view(np.uint32), rep.view(np.uint32))
+    ref = O.scan_ref_fp64(OL, 1, src)
+    assert np.all(np.abs(got - ref) <= 7 * 2.0 ** -24 * np.abs(ref) + 1e-30)
+
+
+@pytest.mark.parametrize("family", ["blocked", "mma", "mma_input", "sliced_blocked", "sliced_mma",
+                                    "sliced_mma_input", "custom"])
+def test_table4_scan_families(family):
+    """§8(f) N3: scans along the last dim over every Table 4 family and shape,
+    including broadcast layouts whose duplicated positions must all hold the same value
+    (P:308): bit-exact against the fixed-order replica, packed like the input."""
+    import torch
+    rng = np.random.default_rng(4848)
+    for shape in TABLE4_SHAPES:
+        OL, L = _table4_layout(family, shape, rng)
+        try:
+            plan = ll.ll_plan_scan(L, 1)
+        except ll.LLError as e:
+            # the only refusal: an in-tile axis bit on the warps
+            assert "warps" in str(e), (family, shape, e)
+            continue
+        T = rng.random(1 << OL.d_out, dtype=np.float32)
+        src = O.pack(OL, T)
+        out = torch.empty(src.size, dtype=torch.float32, device="cuda")
+        ll.ll_scan(torch.from_numpy(src).cuda(), out, plan)
+        got = out.cpu().numpy()
+        rep = O.scan_bitdoubling_fp32(OL, 1, src)
+        assert np.array_equal(got.view(np.uint32), rep.view(np.uint32)), (family, shape)

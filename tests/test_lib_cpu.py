@@ -515,3 +515,18 @@ def test_planner_faithful_reproduces_gv6_gv8():
         for f in fields:
             assert t[f] == [flat(e, g[key]["j_bits"]) for e in g[key][f]], (key, f)
     assert t["rounds"] == g["GV7_config2"]["rounds"]
+
+
+def test_scan_plans():
+    """Scan plans (§8(f) N3): one step per in-tile axis bit, each axis bit on a register
+    or a lane of the kernel layout; warp axis bits are refused."""
+    for fam in ("mma", "blocked"):
+        d = ll.ll_plan_scan(ll.Layout.from_spec(W.c4("reduce", fam)), 1).describe()
+        assert d["kind"] == "scan" and d["steps"] == 7 and len(d["axis_hw"]) == 7
+        assert all(b < d["R"] + 5 for b in d["axis_hw"])
+        assert d["ctas"] == 1024
+    # a layout whose axis runs over the warps
+    spec = {"out": [("i", 5), ("j", 7)],
+            "in": [("reg", ["j0", "j1", "j2"]), ("lane", ["i0", "i1", "i2", "i3", "i4"]), ("warp", ["j3", "j4", "j5", "j6"])]}
+    with pytest.raises(ll.LLError, match="warps"):
+        ll.ll_plan_scan(ll.Layout.from_spec(spec), 1)
