@@ -1103,12 +1103,15 @@ std::unique_ptr<ScanPlan> plan_scan(const Layout& L, int axis, const ll_plan_opt
   }
   S->grid_bit = bits_at_level(L, 3, 3);
   // shuffles per thread per tile: a step needs them when its bit or a lower axis bit is
-  // a lane (all slots when its own bit is a lane, else the slots with the bit set)
+  // a lane; one per distinct partner register (slots whose partners coincide share it:
+  // the partner has every lower register axis bit set)
   bool lane_below = false;
+  int low_reg_bits = 0;
   for (int t = 0; t < K; ++t) {
     const bool hreg = S->axis_hw[t] < R;
-    if (!hreg || lane_below) S->shfl_per_thread += hreg ? (1 << (R - 1)) : (1 << R);
+    if (!hreg || lane_below) S->shfl_per_thread += 1 << (R - low_reg_bits - (hreg ? 1 : 0));
     if (!hreg) lane_below = true;
+    else ++low_reg_bits;
   }
   return S;
 }
