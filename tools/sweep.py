@@ -80,6 +80,8 @@ def main():
         return autotune_sweep()
     if "big" in only:
         return big_configs()
+    if "small" in only:
+        return small_kernels()
     if "all" not in only and "conv" not in only:
         return gather_reduce()
     # raw copy roofline reference
@@ -194,6 +196,31 @@ def big_configs():
                               ("c5T", W.c5T(0), 2), ("n1", W.n1_preshuffle(14, 14), 2),
                               ("n2", W.n2_tmem_epilogue(13), 4)]:
         conv_case(name, sa, sb, w)
+
+
+def small_kernels():
+    """Config-4 reduce (TMA vs LDG staging) and scan, 4 rotated buffer sets."""
+    n = 1 << 24
+    for fam in ("mma", "blocked"):
+        L = ll.Layout.from_spec(W.c4("reduce", fam))
+        for name, mk in [("reduce tma", lambda: ll.ll_plan_reduce(L, 1)),
+                         ("reduce ldg", lambda: ll.ll_plan_reduce(L, 1, force_class="SHUFFLE")),
+                         ("scan", lambda: ll.ll_plan_scan(L, 1))]:
+            p = mk()
+            p.prepare()
+            is_scan = name == "scan"
+            sets = [(torch.rand(n, device="cuda"),
+                     torch.empty(n if is_scan else p.out_elems(), device="cuda")) for _ in range(4)]
+            it = [0]
+
+            def f():
+                st = sets[it[0] % 4]
+                it[0] += 1
+                (ll.ll_scan if is_scan else ll.ll_reduce)(st[0], st[1], p)
+            ms = time_fn(f)
+            b = 8 * n if is_scan else 4 * n + 4 * p.out_elems()
+            print(json.dumps({"case": f"{name} {fam}", "ms": round(ms, 4), "GBps": round(b / ms / 1e6, 1)}), flush=True)
+            del sets
 
 
 def latency_and_ksweep():
