@@ -468,6 +468,7 @@ ll_status ll_plan_describe(const ll_plan* p, char* json, size_t cap) {
       << ",\"axis_hw\":" << "[";
     for (size_t t = 0; t < S.axis_hw.size(); ++t) o << (t ? "," : "") << S.axis_hw[t];
     o << "],\"shuffles_per_elem\":" << double(S.shfl_per_thread) / double(1 << S.R)
+      << ",\"tma\":" << (S.tma ? "true" : "false") << ",\"stages\":" << S.stages
       << ",\"ctas\":" << (u64(1) << S.grid_bit.size()) << "}";
     s = o.str();
   } else {
@@ -517,7 +518,12 @@ ll_status ll_plan_prepare(ll_plan* p) {
   }
   if (p->kind == 3) {
     std::lock_guard<std::mutex> g(p->scan->mu);
-    if (!p->scan->kernel) p->scan->kernel = jit_kernel(codegen_scan(*p->scan), "ll_scan_kernel");
+    if (!p->scan->kernel) {
+      p->scan->kernel = jit_kernel(codegen_scan(*p->scan), "ll_scan_kernel");
+      if (p->scan->smem_bytes > 48 * 1024)
+        check_cuda(cudaFuncSetAttribute(p->scan->kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                        p->scan->smem_bytes), "cudaFuncSetAttribute");
+    }
   }
   if (p->kind == 2) {
     std::lock_guard<std::mutex> g(p->reduce->mu);
@@ -730,7 +736,9 @@ ll_status ll_scan(const float* src, float* dst, const ll_plan* p, void* stream) 
   ScanPlan& S = *p->scan;
   unsigned long long nt = u64(1) << S.grid_bit.size();
   void* args[] = {const_cast<float**>(&src), &dst, &nt};
-  launch_kernel(S.kernel, grid_for(nt), 32u << S.Wb, args, 0, static_cast<cudaStream_t>(stream),
+  // the TMA pipeline is persistent: one CTA per SM streams its tiles through the stages
+  unsigned grid = S.tma ? unsigned(std::min<u64>(nt, u64(num_sms()))) : grid_for(nt);
+  launch_kernel(S.kernel, grid, 32u << S.Wb, args, size_t(S.smem_bytes), static_cast<cudaStream_t>(stream),
                 "cudaLaunchKernelEx(ll_scan_kernel)");
   LL_CATCH
 }

@@ -290,6 +290,9 @@ struct ScanPlan {
   std::vector<int> grid_bit;   // CTA index bit -> packed bit
   std::vector<int> axis_hw;    // logical axis bit t -> kernel bit (reg < R or lane)
   int shfl_per_thread = 0;     // shuffles per thread per tile
+  bool tma = false;            // cp.async.bulk staging of the contiguous CTA tiles
+  int stages = 0;
+  int smem_bytes = 0;
   std::string source;
   void* kernel = nullptr;
   std::mutex mu;

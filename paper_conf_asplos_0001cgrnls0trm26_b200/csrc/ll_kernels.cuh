@@ -892,18 +892,7 @@ template <class P, int S> struct ScanStep {
 };
 
 template <class P>
-__device__ __forceinline__ void ll_scan_body(const u8* __restrict__ src, u8* __restrict__ dst, u64 ntiles) {
-  ll_pdl_begin();
-  const u32 lane = threadIdx.x & 31u;
-  const u32 warp = threadIdx.x >> 5;
-  const u64 thr = thread_base<P, true>(lane, warp);
-  for (u64 t = blockIdx.x; t < ntiles; t += gridDim.x) {
-    const u64 base = tile_base<P, true>(t) ^ thr;
-    u32 r[P::NW];
-    static_for<(1 << (P::R - P::VLD))>([&](auto k) {
-      constexpr int K = decltype(k)::value;
-      load_vec<4, P::VLD, K, P::NW, P::LD_L1>(r, src + base + LdOff<P, K>::value());
-    });
+__device__ __forceinline__ void ll_scan_steps(u32 (&r)[P::NW], u32 lane) {
     static_for<P::KB>([&](auto s) {
       using St = ScanStep<P, decltype(s)::value>;
       constexpr int HB = St::HB;
@@ -941,9 +930,71 @@ __device__ __forceinline__ void ll_scan_body(const u8* __restrict__ src, u8* __r
         });
       }
     });
+}
+
+template <class P>
+__device__ __forceinline__ void ll_scan_body(const u8* __restrict__ src, u8* __restrict__ dst, u64 ntiles) {
+  extern __shared__ __align__(16) u8 ll_smem[];
+  ll_pdl_begin();
+  const u32 lane = threadIdx.x & 31u;
+  const u32 warp = threadIdx.x >> 5;
+  const u64 thr = thread_base<P, true>(lane, warp);
+  auto store_tile = [&](const u32 (&r)[P::NW], u64 base) {
     static_for<(1 << (P::R - P::VLD))>([&](auto k) {
       constexpr int K = decltype(k)::value;
       store_vec<4, P::VLD, K, P::NW, P::ST_HINT>(r, dst + base + LdOff<P, K>::value());
     });
+  };
+  if constexpr (P::TMA) {
+    // the CTA tile is contiguous in HBM: cp.async.bulk into NS stages (mbarrier
+    // completion, the next tiles in flight while this one is scanned), 16-byte stage
+    // reads through the line σ, results stored from registers
+    constexpr u32 TB = u32(4) << (P::R + 5 + P::WB);
+    constexpr u32 NS = P::STAGES;
+    const u32 sbase = u32(__cvta_generic_to_shared(ll_smem));
+    const u32 bar0 = sbase + NS * TB;
+    if (threadIdx.x == 0) {
+      for (u32 q = 0; q < NS; ++q) mbar_init(bar0 + 8 * q, 1);
+      mbar_fence_init();
+    }
+    __syncthreads();
+    auto issue = [&](u64 tq, u32 q) {
+      mbar_expect_tx(bar0 + 8 * q, TB);
+      bulk_g2s(sbase + q * TB, src + tile_base<P, true>(tq), TB, bar0 + 8 * q);
+    };
+    if (threadIdx.x == 0)
+      for (u32 q = 0; q + 1 < NS; ++q)
+        if (blockIdx.x + u64(q) * gridDim.x < ntiles) issue(blockIdx.x + u64(q) * gridDim.x, q);
+    u32 i = 0;
+    for (u64 t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
+      const u32 st = i % NS;
+      const u64 tn = t + u64(NS - 1) * gridDim.x;
+      if (threadIdx.x == 0 && tn < ntiles) {
+        fence_proxy_async();
+        issue(tn, (i + NS - 1) % NS);
+      }
+      mbar_wait(bar0 + 8 * st, (i / NS) & 1u);
+      u32 r[P::NW];
+      const u32 tb = sbase + st * TB + u32(thr);
+      static_for<(1 << (P::R - P::VLD))>([&](auto k) {
+        constexpr int K = decltype(k)::value;
+        constexpr int E0 = K << P::VLD;
+        lds_v4(tb + u32(LdOff<P, K>::value()), r[E0], r[E0 + 1], r[E0 + 2], r[E0 + 3]);
+      });
+      __syncthreads();   // stage st is read by every thread before it is refilled
+      ll_scan_steps<P>(r, lane);
+      store_tile(r, tile_base<P, true>(t) ^ thr);
+    }
+  } else {
+    for (u64 t = blockIdx.x; t < ntiles; t += gridDim.x) {
+      const u64 base = tile_base<P, true>(t) ^ thr;
+      u32 r[P::NW];
+      static_for<(1 << (P::R - P::VLD))>([&](auto k) {
+        constexpr int K = decltype(k)::value;
+        load_vec<4, P::VLD, K, P::NW, P::LD_L1>(r, src + base + LdOff<P, K>::value());
+      });
+      ll_scan_steps<P>(r, lane);
+      store_tile(r, base);
+    }
   }
 }

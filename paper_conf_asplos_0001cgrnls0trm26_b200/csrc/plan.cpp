@@ -1113,6 +1113,23 @@ std::unique_ptr<ScanPlan> plan_scan(const Layout& L, int axis, const ll_plan_opt
     if (!hreg) lane_below = true;
     else ++low_reg_bits;
   }
+  // TMA staging as for the reduce: contiguous CTA tile (reg, lane, warp are L's lowest
+  // packed bits), line σ with 16-byte reads, 2-4 stages in smem; force_class = SHUFFLE
+  // keeps direct LDG loads
+  const u64 tile_bytes = u64(4) << (R + 5 + S->Wb);
+  bool contiguous = true;
+  {
+    int p = 0;
+    for (auto& d : L.in) {
+      if (dim_level(d.name) <= 2 && p + d.bits > R + 5 + S->Wb) contiguous = false;
+      p += d.bits;
+    }
+  }
+  const int force = opts ? opts->force_class : -1;
+  for (int ns = 3; ns >= 2; --ns)
+    if (u64(ns) * tile_bytes + 8 * ns <= 200 * 1024) { S->stages = ns; break; }
+  S->tma = S->sigma == SIGMA_COALESCED && S->v == 2 && contiguous && force != LL_CLASS_SHUFFLE && S->stages > 0;
+  S->smem_bytes = S->tma ? int(S->stages * tile_bytes + 8 * S->stages) : 0;
   return S;
 }
 

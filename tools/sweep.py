@@ -205,10 +205,11 @@ def small_kernels():
         L = ll.Layout.from_spec(W.c4("reduce", fam))
         for name, mk in [("reduce tma", lambda: ll.ll_plan_reduce(L, 1)),
                          ("reduce ldg", lambda: ll.ll_plan_reduce(L, 1, force_class="SHUFFLE")),
-                         ("scan", lambda: ll.ll_plan_scan(L, 1))]:
+                         ("scan", lambda: ll.ll_plan_scan(L, 1)),
+                         ("scan ldg", lambda: ll.ll_plan_scan(L, 1, force_class="SHUFFLE"))]:
             p = mk()
             p.prepare()
-            is_scan = name == "scan"
+            is_scan = name.startswith("scan")
             sets = [(torch.rand(n, device="cuda"),
                      torch.empty(n if is_scan else p.out_elems(), device="cuda")) for _ in range(4)]
             it = [0]
