@@ -168,3 +168,63 @@ def test_nccl_comm_bootstrap_single_rank():
     ll._check(ll._lib.ll_comm_create(uid, 1, 0, ctypes.byref(h)))
     assert h.value
     ll._lib.ll_comm_destroy(h)
+
+
+def _with_dev(spec, p):
+    """The top p block bits of a batched spec become `dev` bits."""
+    ins, dev = [], []
+    for n, bits in spec["in"]:
+        if n == "block":
+            ins.append(("block", bits[:-p]))
+            dev = bits[-p:]
+        else:
+            ins.append((n, bits))
+    ins.append(("dev", dev))
+    return {"out": spec["out"], "in": ins}
+
+
+def _weak_worker(rank, world, port, q):
+    import torch
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        p = world.bit_length() - 1
+        for make, w in ((lambda: W.c2(4), 2), (lambda: W.c3(3), 2), (lambda: W.c1_batched(4), 4)):
+            sa, sb = (_with_dev(s, p) for s in make())
+            OA, OB = O.Layout(*W.spec_to_bases(sa)), O.Layout(*W.spec_to_bases(sb))
+            plan = ll.ll_plan_convert(ll.Layout.from_spec(sa), ll.Layout.from_spec(sb), w)
+            # Q is the identity on the dev bits: a local class, no communicator needed
+            assert plan.cls == O.classify(OA, OB) and plan.cls != "DEVICE"
+            T = gen.random_bits(np.random.default_rng(1002), 1 << OA.d_out, w)
+            src = _rank_src(OA, T, rank)
+            got = plan.simulate(src, src.size)
+            ok = np.array_equal(got, O.convert_distributed_rank(OA, OB, T, rank))
+            # the bench's max-over-ranks reduction, on a per-rank figure
+            t = torch.tensor([float(rank + 1)], dtype=torch.float64)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            assert ok and t.item() == world
+        q.put((rank, "ok"))
+    except Exception as e:  # pragma: no cover
+        q.put((rank, repr(e)))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 4])
+def test_weak_sharding_independent_tiles_gloo(world):
+    """Row e(1): configs 1-batch, 2 and 3 sharded over ranks by declaring the top block
+    bits `dev` in both layouts — each rank plans and converts its own slice with no
+    communication (host schedule emulation), equal to the oracle's rank slice (O12)."""
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_weak_worker, args=(r, world, port, q)) for r in range(world)]
+    for pr in procs:
+        pr.start()
+    res = dict(q.get(timeout=300) for _ in procs)
+    for pr in procs:
+        pr.join(timeout=60)
+    assert all(v == "ok" for v in res.values()), res
