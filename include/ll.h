@@ -293,8 +293,9 @@ ll_status ll_reduce(const float* src, float* dst, const ll_plan* plan, void* str
  * from zero).  The fp32 order is fixed (reading R-scan): for axis bit t =
  * 0, 1, ..., an element whose axis bit t is set adds the value of the last element of
  * the lower half of its aligned 2^(t+1)-block.  L: a distributed layout (duplicated
- * positions, zero columns, each get the same value); the in-tile axis bits must be
- * register or lane bits (LL_ERR_UNSUPPORTED for warp bits). */
+ * positions, zero columns, each get the same value).  Steps over register bits are
+ * register adds, over lane bits warp shuffles, over warp bits a shared-memory
+ * exchange (LL_ERR_UNSUPPORTED when it exceeds shared memory). */
 ll_status ll_plan_scan(const ll_layout* L, int axis, const ll_plan_opts* opts, ll_plan** plan);
 /* src, dst: fp32 packed in L (same positions); must not overlap partially. */
 ll_status ll_scan(const float* src, float* dst, const ll_plan* plan, void* stream);

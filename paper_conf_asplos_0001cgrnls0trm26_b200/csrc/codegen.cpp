@@ -182,6 +182,7 @@ std::string codegen_scan(const ScanPlan& S) {
   o << icon("KB", S.K_bits) << arr("int", "AXIS_HW", S.axis_hw);
   o << "  static constexpr bool TMA = " << (S.tma ? "true" : "false") << ";\n";
   o << "  static constexpr unsigned STAGES = " << std::max(1, S.stages) << "u;\n";
+  o << "  static constexpr unsigned XS_BYTES = " << S.xs_bytes << "u;\n";
   o << "};\n";
   o << "extern \"C\" __global__ void __launch_bounds__(" << (32 << S.Wb)
     << ") ll_scan_kernel(const u8* __restrict__ src, u8* __restrict__ dst, u64 ntiles) {\n"

@@ -292,6 +292,7 @@ struct ScanPlan {
   int shfl_per_thread = 0;     // shuffles per thread per tile
   bool tma = false;            // cp.async.bulk staging of the contiguous CTA tiles
   int stages = 0;
+  int xs_bytes = 0;            // exchange buffer of the warp-crossing steps
   int smem_bytes = 0;
   std::string source;
   void* kernel = nullptr;

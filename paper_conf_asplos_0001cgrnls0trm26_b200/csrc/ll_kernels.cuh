@@ -886,18 +886,59 @@ __device__ __forceinline__ void ll_reduce_body(const float* __restrict__ src, fl
 template <class P, int S> struct ScanStep {
   static constexpr int HB = P::AXIS_HW[S];
   static constexpr bool HREG = HB < P::R;
+  static constexpr bool HWARP = HB >= P::R + 5;
   static constexpr u32 low_reg() { u32 m = 0; for (int q = 0; q < S; ++q) if (P::AXIS_HW[q] < P::R) m |= 1u << P::AXIS_HW[q]; return m; }
-  static constexpr u32 low_lane() { u32 m = 0; for (int q = 0; q < S; ++q) if (P::AXIS_HW[q] >= P::R) m |= 1u << (P::AXIS_HW[q] - P::R); return m; }
-  static constexpr bool SHFL = !HREG || low_lane() != 0;
+  static constexpr u32 low_lane() {
+    u32 m = 0;
+    for (int q = 0; q < S; ++q)
+      if (P::AXIS_HW[q] >= P::R && P::AXIS_HW[q] < P::R + 5) m |= 1u << (P::AXIS_HW[q] - P::R);
+    return m;
+  }
+  static constexpr u32 low_warp() { u32 m = 0; for (int q = 0; q < S; ++q) if (P::AXIS_HW[q] >= P::R + 5) m |= 1u << (P::AXIS_HW[q] - P::R - 5); return m; }
+  static constexpr bool SMEM = HWARP || low_warp() != 0;
+  static constexpr bool SHFL = !SMEM && (!HREG || low_lane() != 0);
 };
 
+// sm: NW x threads floats (the warp-crossing steps' exchange buffer)
 template <class P>
-__device__ __forceinline__ void ll_scan_steps(u32 (&r)[P::NW], u32 lane) {
+__device__ __forceinline__ void ll_scan_steps(u32 (&r)[P::NW], u32 lane, float* sm) {
     static_for<P::KB>([&](auto s) {
       using St = ScanStep<P, decltype(s)::value>;
       constexpr int HB = St::HB;
       constexpr u32 LR = St::low_reg(), LL = St::low_lane();
-      if constexpr (!St::SHFL) {
+      if constexpr (St::SMEM) {
+        // bit S or a lower axis bit on the warps: every value goes through shared memory
+        // ([slot][thread]); the partner is (slot, lane, warp) with the bit of S cleared
+        // and the lower axis bits set
+        constexpr u32 NT = 32u << P::WB;
+        constexpr u32 LW = St::low_warp();
+        const u32 warp = threadIdx.x >> 5;
+        static_for<P::NW>([&](auto e) {
+          constexpr int E = decltype(e)::value;
+          sm[E * NT + threadIdx.x] = __uint_as_float(r[E]);
+        });
+        __syncthreads();
+        u32 pl = lane | LL, pw = warp | LW;
+        bool upper = true;
+        if constexpr (St::HWARP) {
+          constexpr int WBIT = HB - P::R - 5;
+          pw &= ~(1u << WBIT);
+          upper = (warp >> WBIT) & 1u;
+        } else if constexpr (!St::HREG) {
+          constexpr int LBIT = HB - P::R;
+          pl &= ~(1u << LBIT);
+          upper = (lane >> LBIT) & 1u;
+        }
+        const u32 pt = pw * 32u + pl;
+        static_for<P::NW>([&](auto e) {
+          constexpr int E = decltype(e)::value;
+          if constexpr (!St::HREG || ((E >> HB) & 1)) {
+            constexpr int E2 = (St::HREG ? (E & ~(1 << HB)) : E) | int(LR);
+            if (upper) r[E] = __float_as_uint(__fadd_rn(__uint_as_float(r[E]), sm[E2 * NT + pt]));
+          }
+        });
+        __syncthreads();
+      } else if constexpr (!St::SHFL) {
         // bit S and every lower axis bit live in this thread's registers
         static_for<P::NW>([&](auto e) {
           constexpr int E = decltype(e)::value;
@@ -952,7 +993,8 @@ __device__ __forceinline__ void ll_scan_body(const u8* __restrict__ src, u8* __r
     constexpr u32 TB = u32(4) << (P::R + 5 + P::WB);
     constexpr u32 NS = P::STAGES;
     const u32 sbase = u32(__cvta_generic_to_shared(ll_smem));
-    const u32 bar0 = sbase + NS * TB;
+    const u32 bar0 = sbase + NS * TB + P::XS_BYTES;
+    float* xs = reinterpret_cast<float*>(ll_smem + NS * TB);
     if (threadIdx.x == 0) {
       for (u32 q = 0; q < NS; ++q) mbar_init(bar0 + 8 * q, 1);
       mbar_fence_init();
@@ -982,10 +1024,11 @@ __device__ __forceinline__ void ll_scan_body(const u8* __restrict__ src, u8* __r
         lds_v4(tb + u32(LdOff<P, K>::value()), r[E0], r[E0 + 1], r[E0 + 2], r[E0 + 3]);
       });
       __syncthreads();   // stage st is read by every thread before it is refilled
-      ll_scan_steps<P>(r, lane);
+      ll_scan_steps<P>(r, lane, xs);
       store_tile(r, tile_base<P, true>(t) ^ thr);
     }
   } else {
+    float* xs = reinterpret_cast<float*>(ll_smem);
     for (u64 t = blockIdx.x; t < ntiles; t += gridDim.x) {
       const u64 base = tile_base<P, true>(t) ^ thr;
       u32 r[P::NW];
@@ -993,7 +1036,7 @@ __device__ __forceinline__ void ll_scan_body(const u8* __restrict__ src, u8* __r
         constexpr int K = decltype(k)::value;
         load_vec<4, P::VLD, K, P::NW, P::LD_L1>(r, src + base + LdOff<P, K>::value());
       });
-      ll_scan_steps<P>(r, lane);
+      ll_scan_steps<P>(r, lane, xs);
       store_tile(r, base);
     }
   }

@@ -1098,19 +1098,20 @@ std::unique_ptr<ScanPlan> plan_scan(const Layout& L, int axis, const ll_plan_opt
     int b = -1;
     for (int q = 0; q < n; ++q) if (L.cols[S->hw_bit[q]] == (u64(1) << (sh + t))) b = q;
     if (b < 0) fail(LL_ERR_UNSUPPORTED, "scan: in-tile axis bits must be the low axis bits");
-    if (b >= R + 5) fail(LL_ERR_UNSUPPORTED, "scan: an axis bit on the warps is not supported (registers and lanes only)");
     S->axis_hw.push_back(b);
   }
   S->grid_bit = bits_at_level(L, 3, 3);
   // shuffles per thread per tile: a step needs them when its bit or a lower axis bit is
   // a lane; one per distinct partner register (slots whose partners coincide share it:
   // the partner has every lower register axis bit set)
-  bool lane_below = false;
+  bool lane_below = false, warp_below = false;
   int low_reg_bits = 0;
   for (int t = 0; t < K; ++t) {
-    const bool hreg = S->axis_hw[t] < R;
-    if (!hreg || lane_below) S->shfl_per_thread += 1 << (R - low_reg_bits - (hreg ? 1 : 0));
-    if (!hreg) lane_below = true;
+    const bool hreg = S->axis_hw[t] < R, hwarp = S->axis_hw[t] >= R + 5;
+    if (hwarp || warp_below) S->xs_bytes = (4 << R) * (32 << S->Wb);   // smem step
+    else if (!hreg || lane_below) S->shfl_per_thread += 1 << (R - low_reg_bits - (hreg ? 1 : 0));
+    if (hwarp) warp_below = true;
+    else if (!hreg) lane_below = true;
     else ++low_reg_bits;
   }
   // TMA staging as for the reduce: contiguous CTA tile (reg, lane, warp are L's lowest
@@ -1127,9 +1128,10 @@ std::unique_ptr<ScanPlan> plan_scan(const Layout& L, int axis, const ll_plan_opt
   }
   const int force = opts ? opts->force_class : -1;
   for (int ns = 3; ns >= 2; --ns)
-    if (u64(ns) * tile_bytes + 8 * ns <= 200 * 1024) { S->stages = ns; break; }
+    if (u64(ns) * tile_bytes + u64(S->xs_bytes) + 8 * ns <= 200 * 1024) { S->stages = ns; break; }
   S->tma = S->sigma == SIGMA_COALESCED && S->v == 2 && contiguous && force != LL_CLASS_SHUFFLE && S->stages > 0;
-  S->smem_bytes = S->tma ? int(S->stages * tile_bytes + 8 * S->stages) : 0;
+  S->smem_bytes = S->tma ? int(S->stages * tile_bytes + S->xs_bytes + 8 * S->stages) : S->xs_bytes;
+  if (S->smem_bytes > 200 * 1024) fail(LL_ERR_UNSUPPORTED, "scan: tile too large for the shared-memory exchange");
   return S;
 }
 

@@ -451,26 +451,27 @@ def _table4_layout(family, shape, rng):
 @pytest.mark.parametrize("family", ["blocked", "mma", "mma_input", "sliced_blocked", "sliced_mma",
                                     "sliced_mma_input", "custom"])
 def test_table4_reduce_families(family):
-    """§8(f) N3: reductions (tl.sum along the last dim) over every Table 4 layout family
-    on the Table 4 shapes: ≤ 1e-6 relative vs fp64 and bit-exact vs the
-    fixed-order replica on the kernel layout; broadcast copies counted once."""
+    """§8(f) N3: reductions (tl.sum) along either dim over every Table 4 layout family on
+    the Table 4 shapes (5 shapes x 2 axes per family): ≤ 1e-6 relative vs
+    fp64 and bit-exact vs the fixed-order replica on the kernel layout; broadcast copies
+    counted once."""
     import torch
     rng = np.random.default_rng(4747)
     for shape in TABLE4_SHAPES:
         OL, L = _table4_layout(family, shape, rng)
         assert L.cols() == OL.cols
-        n = 1 << OL.d_in
         T = rng.random(1 << OL.d_out, dtype=np.float32)
         src = O.pack(OL, T)
-        plan = ll.ll_plan_reduce(L, 1)
-        out = torch.full((plan.out_elems(),), -1.0, dtype=torch.float32, device="cuda")
-        ll.ll_reduce(torch.from_numpy(src).cuda(), out, plan)
-        got = out.cpu().numpy()
-        ref = T.astype(np.float64).reshape(shape).sum(axis=1)
-        assert np.all(np.abs(got - ref) <= 1e-6 * np.abs(ref)), (family, shape)
-        Lp, perm = _line_sigma_layout(OL, 1)
-        rep = O.reduce_fixed_order_fp32(Lp, 1, src[perm])
-        assert np.array_equal(got.view(np.uint32), rep.view(np.uint32)), (family, shape)
+        for axis in (1, 0):
+            plan = ll.ll_plan_reduce(L, axis)
+            out = torch.full((plan.out_elems(),), -1.0, dtype=torch.float32, device="cuda")
+            ll.ll_reduce(torch.from_numpy(src).cuda(), out, plan)
+            got = out.cpu().numpy()
+            ref = T.astype(np.float64).reshape(shape).sum(axis=axis)
+            assert np.all(np.abs(got - ref) <= 1e-6 * np.abs(ref)), (family, shape, axis)
+            Lp, perm = _line_sigma_layout(OL, axis)
+            rep = O.reduce_fixed_order_fp32(Lp, axis, src[perm])
+            assert np.array_equal(got.view(np.uint32), rep.view(np.uint32)), (family, shape, axis)
 
 
 def test_swizzled_memory_layout_gpu():
@@ -564,23 +565,47 @@ def test_scan_bitexact(family, sigma):
 @pytest.mark.parametrize("family", ["blocked", "mma", "mma_input", "sliced_blocked", "sliced_mma",
                                     "sliced_mma_input", "custom"])
 def test_table4_scan_families(family):
-    """§8(f) N3: scans along the last dim over every Table 4 family and shape,
-    including broadcast layouts whose duplicated positions must all hold the same value
-    (P:308): bit-exact against the fixed-order replica, packed like the input."""
+    """§8(f) N3: scans along either dim over every Table 4 family and shape —
+    steps over registers, lanes and (through shared memory) warps — including broadcast
+    layouts whose duplicated positions must all hold the same value: bit-exact
+    against the fixed-order replica, packed like the input."""
     import torch
     rng = np.random.default_rng(4848)
+    ran = 0
     for shape in TABLE4_SHAPES:
         OL, L = _table4_layout(family, shape, rng)
-        try:
-            plan = ll.ll_plan_scan(L, 1)
-        except ll.LLError as e:
-            # the only refusal: an in-tile axis bit on the warps
-            assert "warps" in str(e), (family, shape, e)
-            continue
         T = rng.random(1 << OL.d_out, dtype=np.float32)
         src = O.pack(OL, T)
+        for axis in (1, 0):
+            try:
+                plan = ll.ll_plan_scan(L, axis)
+            except ll.LLError as e:
+                # the only refusal: a warp-crossing step whose exchange buffer (one value
+                # per thread and register) exceeds shared memory (the 512-register custom tile)
+                assert "too large" in str(e), (family, shape, axis, e)
+                continue
+            out = torch.empty(src.size, dtype=torch.float32, device="cuda")
+            ll.ll_scan(torch.from_numpy(src).cuda(), out, plan)
+            got = out.cpu().numpy()
+            rep = O.scan_bitdoubling_fp32(OL, axis, src)
+            assert np.array_equal(got.view(np.uint32), rep.view(np.uint32)), (family, shape, axis)
+            ran += 1
+    assert ran >= 8
+
+
+def test_scan_axis_over_warps():
+    """Scan steps over warp bits (shared-memory exchange) and over lanes and registers in
+    one tile: axis j = (reg j0..j2, warp j3..j6) on a 512-thread CTA."""
+    import torch
+    spec = {"out": [("b", 3), ("i", 5), ("j", 7)],
+            "in": [("reg", ["j0", "j1", "j2"]), ("lane", ["i0", "i1", "i2", "i3", "i4"]),
+                   ("warp", ["j3", "j4", "j5", "j6"]), ("block", ["b0", "b1", "b2"])]}
+    L, OL = both(spec)
+    T = np.random.default_rng(1010).random(1 << OL.d_out, dtype=np.float32)
+    src = O.pack(OL, T)
+    for sigma in ("coalesced", "faithful"):
+        plan = ll.ll_plan_scan(L, 2, sigma=sigma)
         out = torch.empty(src.size, dtype=torch.float32, device="cuda")
         ll.ll_scan(torch.from_numpy(src).cuda(), out, plan)
-        got = out.cpu().numpy()
-        rep = O.scan_bitdoubling_fp32(OL, 1, src)
-        assert np.array_equal(got.view(np.uint32), rep.view(np.uint32)), (family, shape)
+        rep = O.scan_bitdoubling_fp32(OL, 2, src)
+        assert np.array_equal(out.cpu().numpy().view(np.uint32), rep.view(np.uint32)), sigma
