@@ -265,8 +265,11 @@ ll_status ll_plan_autotune(const ll_layout* A, const ll_layout* B, int elem_byte
  * (P:430).  Along logical dim `axis`, K = 2^(non-block axis bits of L); these
  * must be the low bits of the axis coordinate.  out[x] = src[x with the axis
  * coordinate's low bits replaced by idx[x] & (K-1)] (take_along_axis inside each
- * tile; out-of-range indices are masked).  Warp shuffles are used
- * when L_Wrp^axis = 0. */
+ * tile; out-of-range indices are masked).  Warp shuffles when
+ * L_Wrp^axis = 0 and at most 4 candidate registers remain, else a
+ * shared-memory gather over the staged CTA tile (any axis placement; the P:519
+ * crossover); opts->force_class SHUFFLE / SMEM selects one (SHUFFLE with warp axis
+ * bits: LL_ERR_UNSUPPORTED). */
 ll_status ll_plan_gather(const ll_layout* L, int axis, int elem_bytes,
                          const ll_plan_opts* opts, ll_plan** plan);
 /* src, dst: packed in L; idx: int32 packed in L. */

@@ -876,8 +876,11 @@ std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const 
     for (int k : axis_bits) if (L.cols[k] == (u64(1) << (sh + t))) found = true;
     if (!found) fail(LL_ERR_UNSUPPORTED, "gather: in-tile axis bits must be the low axis bits");
   }
+  // the paper's shuffle gather needs L_Wrp^axis = 0; the shared-memory gather
+  // stages the whole CTA tile and serves axis bits on any level
+  bool warp_axis = false;
   for (int k : bits_at_level(L, 2, 2))
-    if (L.cols[k] & amask) fail(LL_ERR_UNSUPPORTED, "gather: L_Wrp^axis != 0 (P:430)");
+    if (L.cols[k] & amask) warp_axis = true;
   // kernel decomposition: faithful (L itself) or coalesced σ; pick the one with
   // fewer shuffle candidates 2^{|L_Reg^axis|}, coalesced on ties.
   const int ev = std::max(w, 4);   // idx is int32: one σ for both
@@ -918,7 +921,9 @@ std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const 
   // the gathered dimension grows; the planner switches when more than 4
   // candidates per element remain (force_class selects either)
   int force = opts ? opts->force_class : -1;
-  G->smem = force == LL_CLASS_SMEM || (force != LL_CLASS_SHUFFLE && G->cand_bits > 2);
+  if (warp_axis && force == LL_CLASS_SHUFFLE)
+    fail(LL_ERR_UNSUPPORTED, "gather: L_Wrp^axis != 0 (P:430): the shuffle gather needs the axis off the warps");
+  G->smem = warp_axis || force == LL_CLASS_SMEM || (force != LL_CLASS_SHUFFLE && G->cand_bits > 2);
   // smem layout of the staged tile: vector registers, then lanes, then the other
   // registers, then warps (offset order kreg[0,v), klane, kreg[v,R), kwarp), so the
   // staging stores are whole 16-byte vectors with consecutive lanes on consecutive

@@ -609,3 +609,24 @@ def test_scan_axis_over_warps():
         ll.ll_scan(torch.from_numpy(src).cuda(), out, plan)
         rep = O.scan_bitdoubling_fp32(OL, 2, src)
         assert np.array_equal(out.cpu().numpy().view(np.uint32), rep.view(np.uint32)), sigma
+
+
+def test_gather_axis_over_warps_smem():
+    """Gather with in-tile axis bits on the warps (L_Wrp^axis != 0, outside the paper's
+    shuffle gather): the shared-memory gather over the staged tile, bit-exact."""
+    import torch
+    spec = {"out": [("b", 3), ("i", 5), ("j", 7)],
+            "in": [("reg", ["j0", "j1", "j2"]), ("lane", ["i0", "i1", "i2", "i3", "i4"]),
+                   ("warp", ["j3", "j4", "j5", "j6"]), ("block", ["b0", "b1", "b2"])]}
+    L, OL = both(spec)
+    rng = np.random.default_rng(1011)
+    n = 1 << OL.d_in
+    src = O.pack(OL, gen.random_bits(rng, n, 4))
+    idx = O.pack(OL, rng.integers(-500, 500, size=n).astype(np.int32))
+    with pytest.raises(ll.LLError, match="warps"):
+        ll.ll_plan_gather(L, 2, 4, force_class="SHUFFLE")
+    plan = ll.ll_plan_gather(L, 2, 4)
+    assert plan.describe()["exchange"] == "smem"
+    d_dst = empty_device(n, 4)
+    ll.ll_gather(to_device(src), to_device(idx.view(np.uint32)), d_dst, plan)
+    assert np.array_equal(from_device(d_dst, 4), O.gather(OL, 2, src, idx))
