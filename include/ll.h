@@ -101,6 +101,10 @@ typedef struct {
   int generic;          /* 1 = force the runtime-generic kernel                   */
   ll_comm* comm;        /* required for DEVICE plans                              */
   int exchange;         /* DEVICE plans: an ll_exchange (default AUTO)            */
+  int smem_instr;       /* smem round trips (Thm 5.1): 0 = auto — stmatrix /
+                         * ldmatrix where M^{-1}∘L is divisible by their tile and that
+                         * widens the swizzle's vector; 1 = vectorised ld/st.shared only;
+                         * 2 = prefer stmatrix / ldmatrix wherever their tile divides   */
 } ll_plan_opts;
 
 /* Fill *opts with defaults (force_class = -1, max_vec_bytes = 16, ...). */

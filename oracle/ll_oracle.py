@@ -623,6 +623,74 @@ def smem_wavefronts(S: Layout, L: Layout, w: int, vec_cols: Sequence[int],
     return total, ideal
 
 
+def smem_matrix_wavefronts(S: Layout, L: Layout, w: int, word_cols: Sequence[int],
+                           trans: bool = False, bank_bytes: int = 4,
+                           n_banks: int = 32) -> Tuple[int, int]:
+    """The same bank model for the ldmatrix / stmatrix instructions ("each
+    thread ... handle[s] 4 contiguous bytes, with 8 groups of 4 threads collaborating
+    to store a row each"; the fragment is PTX's m8n8 b16 matrix [HW]).
+
+    Every thread holds one 32-bit word per matrix, made of the elements over the
+    logical vectors ``word_cols`` (the log2(4/w) register columns of L whose elements
+    form the word, lowest first).  Non-transposed: lane l's word is bytes 4·(l mod 4)
+    .. +3 of row l div 4 of the matrix; transposed (.trans, w = 2): the two halves h
+    of lane l's word are column l div 4 of rows 2·(l mod 4) + h.  The matrices are
+    enumerated by L's remaining register bits and its warp bits.  Every matrix must
+    really be 8 rows of 16 contiguous, 16-byte aligned bytes in S (the instruction
+    can lower L, Thm 5.1) — otherwise ValueError.  A matrix takes one
+    128-byte wavefront per distinct row in its most loaded 16-byte bank group
+    (rows are whole 16-byte pieces of the 128-byte segment).  Returns
+    (wavefronts, ideal); ideal = 1 per matrix."""
+    if trans and w != 2:
+        raise ValueError(".trans moves b16 elements")
+    k = (4 // w).bit_length() - 1
+    if len(word_cols) != k:
+        raise ValueError("a 32-bit word holds 4/w elements")
+    lane_bits = L.dim_bits("lane")
+    reg_bits = L.dim_bits("reg")
+    warp_bits = L.dim_bits("warp")
+    word_bits = []
+    for c in word_cols:
+        ks = [b for b in reg_bits if L.cols[b] == c]
+        assert len(ks) == 1, "word columns must be register columns of L"
+        word_bits.append(ks[0])
+    other = [b for b in reg_bits if b not in word_bits] + list(warp_bits)
+    S_inv = preimage_min(S)
+    group_bytes = n_banks * bank_bytes // 8        # 16-byte bank groups of a segment
+    total = ideal = 0
+    for m in range(1 << len(other)):
+        base = 0
+        for t, b in enumerate(other):
+            if (m >> t) & 1:
+                base |= 1 << b
+        rows: Dict[int, int] = {}                  # row index -> byte address of byte 0
+        for l in range(32):
+            h0 = base
+            for t, b in enumerate(lane_bits):
+                if (l >> t) & 1:
+                    h0 |= 1 << b
+            for e in range(1 << k):                # element e of the word (byte e·w)
+                h = h0
+                for t, b in enumerate(word_bits):
+                    if (e >> t) & 1:
+                        h |= 1 << b
+                addr = int(S_inv[apply(L, h)]) * w
+                if trans:
+                    row, col_byte = 2 * (l % 4) + e, 2 * (l // 4)
+                else:
+                    row, col_byte = l // 4, 4 * (l % 4) + e * w
+                start = addr - col_byte
+                if start % 16 or rows.setdefault(row, start) != start:
+                    raise ValueError("the instruction's tile does not divide M^-1∘L (Thm 5.1)")
+        per_group: Dict[int, int] = {}
+        for start in set(rows.values()):
+            g = (start // group_bytes) % 8
+            per_group[g] = per_group.get(g, 0) + 1
+        total += max(per_group.values())
+        ideal += 1
+    return total, ideal
+
+
 # --------------------------------------------------------------------------------------
 # F2 helpers over sets of logical vectors (spans, completion) — used by the paper's
 # shuffle and swizzle constructions (P:375-387, P:406-426, P:732-756)

@@ -107,6 +107,12 @@ std::string codegen_tile(const ConvPlan& Pl) {
   // SMEM
   o << icon("SV", T.sm_v) << arr("int", "VSLOT_LD", T.vec_slot_ld) << arr("int", "VSLOT_ST", T.vec_slot_st)
     << arr("u64", "SMOFF_LD", T.smoff_ld) << arr("u64", "SMOFF_ST", T.smoff_st);
+  // stmatrix / ldmatrix sides (Thm 5.1)
+  o << icon("SMI_LD", T.smi_ld) << icon("SMI_ST", T.smi_st)
+    << icon("NMW", T.w <= 4 ? ilog2i(u64(4 / T.w)) : 0)
+    << arr("int", "MWORD_LD", T.mat_word_ld) << arr("int", "MWORD_ST", T.mat_word_st)
+    << icon("NMSEL_LD", T.mat_sel_ld.size()) << icon("NMSEL_ST", T.mat_sel_st.size())
+    << arr("int", "MSEL_LD", T.mat_sel_ld) << arr("int", "MSEL_ST", T.mat_sel_st);
   o << "};\n";
   if (Pl.peer_shift >= 0) {
     // DEVICE plan executed as peer stores (N4): global dst offsets, window per rank

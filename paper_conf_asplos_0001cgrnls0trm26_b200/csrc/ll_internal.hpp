@@ -130,6 +130,7 @@ Layout make_tmem_32x32b(int M, int N);                                          
 enum ExecKind { EXEC_NOOP = 0, EXEC_TILE = 1, EXEC_GENERIC = 2, EXEC_DEVICE = 3 };
 enum TileXchg { X_COPY = 0, X_REGPERM = 1, X_SHUFFLE = 2, X_SMEM = 3 };
 enum SigmaMode { SIGMA_COALESCED = 0, SIGMA_FAITHFUL = 1 };
+enum SmemInstr { SMI_VEC = 0, SMI_MAT = 1, SMI_MATT = 2 };
 
 // Kernel decomposition of a conversion whose pull map is a bit permutation:
 // a CTA owns `n` tile bits; kernel hardware inside the CTA is (R reg bits,
@@ -176,6 +177,19 @@ struct TilePlan {
   std::vector<u64> smoff_ld, smoff_st;
   u64 smem_elems = 0;
   long predicted_wavefronts_st = -1, predicted_wavefronts_ld = -1, ideal_wavefronts = -1;
+  // Shared-memory instruction of each side (Thm 5.1), chosen by left
+  // division of M^{-1}∘L by the instruction's tile:
+  //   SMI_VEC  vectorised st/ld.shared (tile id_n^{Reg,Off}),
+  //   SMI_MAT  stmatrix / ldmatrix m8n8 b16 (tile id_k^{Reg,Off} × id_2^{Thr,Off},
+  //            k = log2(4/w)): reg word bits + lanes 0,1 form a 16-byte row,
+  //            lanes 2-4 address the 8 rows of a matrix,
+  //   SMI_MATT the .trans forms (w = 2): lanes 2-4 form the row, (word bit, lane 0,
+  //            lane 1) address the rows.
+  // ld = the smem store through L_ld, st = the smem load through L_st.
+  int smi_ld = 0, smi_st = 0;
+  std::vector<int> mat_word_ld, mat_word_st;   // reg bits forming a matrix word (k of them)
+  std::vector<int> mat_sel_ld, mat_sel_st;     // reg bits selecting the matrix (.x1/.x2/.x4)
+  long smem_instr_st = 0, smem_instr_ld = 0;   // shared instructions per thread per tile
 
   int threads() const { return 32 << Wb; }
   int elems_per_thread() const { return 1 << R; }

@@ -372,11 +372,178 @@ __device__ __forceinline__ void smem_read(u32 (&o)[P::NW], u32 lane, u32 warp, u
     });
   });
 }
+// stmatrix / ldmatrix sides (Thm 5.1): M^{-1}∘L is divisible by the tile
+// id_k^{Reg,Off} × id_2^{Thr,Off} (k = log2(4/W)): a 32-bit word of k register bits
+// and lanes 0, 1 make one 16-byte row of an 8x8 b16 matrix, lanes 2-4 its 8 rows
+// (SMI 1); or, transposed (SMI 2, W = 2), lanes 2-4 make the row and (word bit,
+// lane 0, lane 1) its rows.  Up to two further register bits select the matrix
+// (.x1/.x2/.x4); lane 8m + r supplies the address of row r of matrix m.
+// ST = true: the store side (L_ld data, stmatrix); false: the load side (ldmatrix).
+template <class P, bool ST> struct Mx {
+  static constexpr int KIND = ST ? P::SMI_LD : P::SMI_ST;
+  static constexpr int NWB = P::NMW;
+  static constexpr int NSEL = ST ? P::NMSEL_LD : P::NMSEL_ST;
+  static constexpr int NOTHER = P::R - NWB - NSEL;
+  static constexpr int wordbit(int i) { return ST ? P::MWORD_LD[i] : P::MWORD_ST[i]; }
+  static constexpr int selbit(int j) { return ST ? P::MSEL_LD[j] : P::MSEL_ST[j]; }
+  static constexpr u64 smoff(int b) { return ST ? P::SMOFF_LD[b] : P::SMOFF_ST[b]; }
+  static constexpr bool special(int b) {
+    for (int i = 0; i < NWB; ++i) if (wordbit(i) == b) return true;
+    for (int j = 0; j < NSEL; ++j) if (selbit(j) == b) return true;
+    return false;
+  }
+  // register slot of element i of matrix m in instruction k
+  static constexpr int slot(int k, int m, int i) {
+    int s = 0, t = 0;
+    for (int b = 0; b < P::R; ++b) {
+      if (special(b)) continue;
+      if ((k >> t) & 1) s |= 1 << b;
+      ++t;
+    }
+    for (int j = 0; j < NSEL; ++j) if ((m >> j) & 1) s |= 1 << selbit(j);
+    for (int q = 0; q < NWB; ++q) if ((i >> q) & 1) s |= 1 << wordbit(q);
+    return s;
+  }
+  // smem element offset of instruction k (its non-special register bits)
+  static constexpr u64 off(int k) {
+    u64 o = 0;
+    int t = 0;
+    for (int b = 0; b < P::R; ++b) {
+      if (special(b)) continue;
+      if ((k >> t) & 1) o ^= smoff(b);
+      ++t;
+    }
+    return o;
+  }
+  // the three bits addressing the rows of a matrix
+  static constexpr u64 rowoff(int t) {
+    return KIND == 1 ? smoff(P::R + 2 + t) : (t == 0 ? smoff(wordbit(0)) : smoff(P::R + t - 1));
+  }
+};
+
+// Row address supplied by this lane: row (lane & 7) of matrix (lane >> 3).
+template <class P, bool ST>
+__device__ __forceinline__ u32 mat_thread_base(u32 lane, u32 warp) {
+  typedef Mx<P, ST> X;
+  u32 o = 0;
+  static_for<3>([&](auto t) {
+    constexpr int T = decltype(t)::value;
+    if ((lane >> T) & 1) o ^= u32(X::rowoff(T));
+  });
+  static_for<X::NSEL>([&](auto j) {
+    constexpr int J = decltype(j)::value;
+    if ((lane >> (3 + J)) & 1) o ^= u32(X::smoff(X::selbit(J)));
+  });
+  static_for<P::WB>([&](auto t) {
+    constexpr int T = decltype(t)::value;
+    if ((warp >> T) & 1) o ^= u32(X::smoff(P::R + 5 + T));
+  });
+  return o;
+}
+
+template <int NSEL, bool TRANS>
+__device__ __forceinline__ void stsm(u32 addr, const u32* v) {
+  if constexpr (NSEL == 2) {
+    if constexpr (TRANS)
+      asm volatile("stmatrix.sync.aligned.m8n8.x4.trans.shared.b16 [%0], {%1,%2,%3,%4};"
+                   ::"r"(addr), "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]) : "memory");
+    else
+      asm volatile("stmatrix.sync.aligned.m8n8.x4.shared.b16 [%0], {%1,%2,%3,%4};"
+                   ::"r"(addr), "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]) : "memory");
+  } else if constexpr (NSEL == 1) {
+    if constexpr (TRANS)
+      asm volatile("stmatrix.sync.aligned.m8n8.x2.trans.shared.b16 [%0], {%1,%2};" ::"r"(addr), "r"(v[0]), "r"(v[1]) : "memory");
+    else
+      asm volatile("stmatrix.sync.aligned.m8n8.x2.shared.b16 [%0], {%1,%2};" ::"r"(addr), "r"(v[0]), "r"(v[1]) : "memory");
+  } else {
+    if constexpr (TRANS)
+      asm volatile("stmatrix.sync.aligned.m8n8.x1.trans.shared.b16 [%0], {%1};" ::"r"(addr), "r"(v[0]) : "memory");
+    else
+      asm volatile("stmatrix.sync.aligned.m8n8.x1.shared.b16 [%0], {%1};" ::"r"(addr), "r"(v[0]) : "memory");
+  }
+}
+template <int NSEL, bool TRANS>
+__device__ __forceinline__ void ldsm(u32 addr, u32* v) {
+  if constexpr (NSEL == 2) {
+    if constexpr (TRANS)
+      asm volatile("ldmatrix.sync.aligned.m8n8.x4.trans.shared.b16 {%0,%1,%2,%3}, [%4];"
+                   : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]) : "r"(addr) : "memory");
+    else
+      asm volatile("ldmatrix.sync.aligned.m8n8.x4.shared.b16 {%0,%1,%2,%3}, [%4];"
+                   : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]) : "r"(addr) : "memory");
+  } else if constexpr (NSEL == 1) {
+    if constexpr (TRANS)
+      asm volatile("ldmatrix.sync.aligned.m8n8.x2.trans.shared.b16 {%0,%1}, [%2];" : "=r"(v[0]), "=r"(v[1]) : "r"(addr) : "memory");
+    else
+      asm volatile("ldmatrix.sync.aligned.m8n8.x2.shared.b16 {%0,%1}, [%2];" : "=r"(v[0]), "=r"(v[1]) : "r"(addr) : "memory");
+  } else {
+    if constexpr (TRANS)
+      asm volatile("ldmatrix.sync.aligned.m8n8.x1.trans.shared.b16 {%0}, [%1];" : "=r"(v[0]) : "r"(addr) : "memory");
+    else
+      asm volatile("ldmatrix.sync.aligned.m8n8.x1.shared.b16 {%0}, [%1];" : "=r"(v[0]) : "r"(addr) : "memory");
+  }
+}
+
+template <class P>
+__device__ __forceinline__ void smem_write_mat(const u32 (&r)[P::NW], u32 lane, u32 warp, u32 sbase) {
+  typedef Mx<P, true> X;
+  const u32 tb = mat_thread_base<P, true>(lane, warp);
+  static_for<(1 << X::NOTHER)>([&](auto k) {
+    constexpr int K = decltype(k)::value;
+    u32 v[1 << X::NSEL];
+    static_for<(1 << X::NSEL)>([&](auto m) {
+      constexpr int M = decltype(m)::value;
+      if constexpr (P::W == 4) {
+        v[M] = r[X::slot(K, M, 0)];
+      } else {
+        u32 word = 0;
+        static_for<(1 << X::NWB)>([&](auto i) {
+          constexpr int I = decltype(i)::value;
+          word |= get_e<P::W, X::slot(K, M, I)>(r) << (8 * P::W * I);
+        });
+        v[M] = word;
+      }
+    });
+    stsm<X::NSEL, X::KIND == 2>(sbase + (tb ^ u32(X::off(K))) * P::W, v);
+  });
+}
+template <class P>
+__device__ __forceinline__ void smem_read_mat(u32 (&o)[P::NW], u32 lane, u32 warp, u32 sbase) {
+  typedef Mx<P, false> X;
+  const u32 tb = mat_thread_base<P, false>(lane, warp);
+  static_for<(1 << X::NOTHER)>([&](auto k) {
+    constexpr int K = decltype(k)::value;
+    u32 v[1 << X::NSEL];
+    ldsm<X::NSEL, X::KIND == 2>(sbase + (tb ^ u32(X::off(K))) * P::W, v);
+    static_for<(1 << X::NSEL)>([&](auto m) {
+      constexpr int M = decltype(m)::value;
+      if constexpr (P::W == 4) {
+        o[X::slot(K, M, 0)] = v[M];
+      } else {
+        static_for<(1 << X::NWB)>([&](auto i) {
+          constexpr int I = decltype(i)::value;
+          set_e<P::W, X::slot(K, M, I)>(o, (v[M] >> (8 * P::W * I)) & (P::W == 2 ? 0xffffu : 0xffu));
+        });
+      }
+    });
+  });
+}
+
+template <class P>
+__device__ __forceinline__ void smem_store(const u32 (&r)[P::NW], u32 lane, u32 warp, u32 sbase) {
+  if constexpr (P::SMI_LD != 0) smem_write_mat<P>(r, lane, warp, sbase);
+  else smem_write<P>(r, lane, warp, sbase);
+}
+template <class P>
+__device__ __forceinline__ void smem_load(u32 (&o)[P::NW], u32 lane, u32 warp, u32 sbase) {
+  if constexpr (P::SMI_ST != 0) smem_read_mat<P>(o, lane, warp, sbase);
+  else smem_read<P>(o, lane, warp, sbase);
+}
 template <class P>
 __device__ __forceinline__ void xchg_smem(const u32 (&r)[P::NW], u32 (&o)[P::NW], u32 lane, u32 warp, u32 sbase) {
-  smem_write<P>(r, lane, warp, sbase);
+  smem_store<P>(r, lane, warp, sbase);
   __syncthreads();
-  smem_read<P>(o, lane, warp, sbase);
+  smem_load<P>(o, lane, warp, sbase);
 }
 
 // ------------------------------------------------------------------ tile kernel
@@ -477,12 +644,12 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, Dst D, 
     u32 r[P::NW];
     load_tile(r, t);
     for (; t < ntiles; t += gridDim.x) {
-      smem_write<P>(r, lane, warp, sbase);
+      smem_store<P>(r, lane, warp, sbase);
       __syncthreads();
       if (t + gridDim.x < ntiles) load_tile(r, t + gridDim.x);
       u32 o[P::NW];
       static_for<P::NW>([&](auto q) { o[decltype(q)::value] = 0; });
-      smem_read<P>(o, lane, warp, sbase);
+      smem_load<P>(o, lane, warp, sbase);
       store_tile(o, t);
       __syncthreads();   // smem reuse by the next tile
     }

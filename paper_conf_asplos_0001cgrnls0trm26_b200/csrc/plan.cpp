@@ -406,20 +406,131 @@ static long sim_wavefronts(const TilePlan& T, const std::vector<u64>& smoff,
   return total;
 }
 
-static void plan_smem(TilePlan& T, int maxvec) {
+// Simulated wavefronts (same model) of a side executed with stmatrix /
+// ldmatrix (kind SMI_MAT / SMI_MATT): every 8x8 b16 matrix is 8 rows of 16 bytes
+// addressed by 8 lanes, one 128-byte wavefront when the rows fall in distinct
+// 16-byte bank groups ("8 groups of 4 threads collaborating to store a row").
+static long sim_mat_wavefronts(const TilePlan& T, const std::vector<u64>& smoff, int kind,
+                               const std::vector<int>& word, long* ideal) {
+  const int R = T.R, w = T.w;
+  u64 rows[3];
+  for (int t = 0; t < 3; ++t)
+    rows[t] = kind == SMI_MAT ? smoff[R + 2 + t] : (t == 0 ? smoff[word[0]] : smoff[R + t - 1]);
+  std::vector<u64> other;   // bits enumerating the matrices: non-word registers, warps
+  for (int b = 0; b < R; ++b)
+    if (std::find(word.begin(), word.end(), b) == word.end()) other.push_back(smoff[b]);
+  for (int t = 0; t < T.Wb; ++t) other.push_back(smoff[R + 5 + t]);
+  long total = 0, id = 0;
+  for (u64 m = 0; m < (u64(1) << other.size()); ++m) {
+    u64 base = 0;
+    for (size_t t = 0; t < other.size(); ++t) if ((m >> t) & 1) base ^= other[t];
+    int cnt[8] = {0};
+    for (int r = 0; r < 8; ++r) {
+      u64 o = base;
+      for (int t = 0; t < 3; ++t) if ((r >> t) & 1) o ^= rows[t];
+      ++cnt[(o * u64(w) / 16) % 8];
+    }
+    total += *std::max_element(cnt, cnt + 8);
+    id += 1;
+  }
+  if (ideal) *ideal = id;
+  return total;
+}
+
+static void plan_smem(TilePlan& T, int maxvec, int smem_instr) {
   // Optimal swizzling (appendix) on the kernel layouts.
   const int R = T.R, w = T.w, n = T.n;
-  // 1. Vec: common register vectors, in L_ld register order, within max_vec_bytes.
+  auto reg_of = [&](const std::vector<u64>& lc, u64 c) {
+    for (int q = 0; q < R; ++q) if (lc[q] == c) return q;
+    return -1;
+  };
+  // 1. Vec: common register vectors, in L_ld register order, within max_vec_bytes
+  //    (vectorised ld/st.shared on both sides, tile id_n^{Reg,Off}).
   T.sw_vec.clear(); T.vec_slot_ld.clear(); T.vec_slot_st.clear();
+  T.smi_ld = T.smi_st = SMI_VEC;
+  T.mat_word_ld.clear(); T.mat_word_st.clear(); T.mat_sel_ld.clear(); T.mat_sel_st.clear();
   for (int b = 0; b < R; ++b) {
     u64 c = T.lcol_ld[b];
-    int bs = -1;
-    for (int q = 0; q < R; ++q) if (T.lcol_st[q] == c) bs = q;
+    int bs = reg_of(T.lcol_st, c);
     if (bs < 0) continue;
     if ((int(1) << (T.sw_vec.size() + 1)) * w > maxvec) break;
     T.sw_vec.push_back(c);
     T.vec_slot_ld.push_back(b);
     T.vec_slot_st.push_back(bs);
+  }
+  // 1b. stmatrix / ldmatrix (Thm 5.1).  Their tile makes a 16-byte row of
+  //     k = log2(4/w) register bits and lanes 0, 1 (or, transposed, of lanes 2-4), so a
+  //     side whose registers share too few vectors with the other side still moves
+  //     whole 16-byte rows.  The row is the Vec of the swizzle; M is built with it as
+  //     the lowest offset bits, so M^{-1}∘L is divisible by the tile by construction
+  //     (the planner asserts it below).  Tried when the common registers give less than
+  //     16 bytes (auto) or always (smem_instr = 2); the first divisible choice wins, in
+  //     the order: one side matrix, the other vectorised; then both sides matrix.
+  const int full = w <= 4 ? ilog2(u64(16 / w)) : 0;
+  const int k = w <= 4 ? ilog2(u64(4 / w)) : 0;
+  if (smem_instr != 1 && w <= 4 && maxvec >= 16 && R >= k &&
+      (int(T.sw_vec.size()) < full || smem_instr == 2)) {
+    struct Side { int kind; std::vector<int> word; std::vector<u64> row; };
+    auto options = [&](const std::vector<u64>& lc) {
+      std::vector<Side> out;
+      std::vector<std::vector<int>> words;
+      if (k == 0) words.push_back({});
+      for (int a = 0; a < R && k >= 1; ++a) {
+        if (k == 1) { words.push_back({a}); continue; }
+        for (int b2 = 0; b2 < R; ++b2) if (b2 != a) words.push_back({a, b2});
+      }
+      for (auto& wd : words) {
+        Side s{SMI_MAT, wd, {}};
+        for (int q : wd) s.row.push_back(lc[q]);
+        s.row.push_back(lc[R]);
+        s.row.push_back(lc[R + 1]);
+        out.push_back(s);
+      }
+      if (w == 2)
+        for (auto& wd : words) out.push_back(Side{SMI_MATT, wd, {lc[R + 2], lc[R + 3], lc[R + 4]}});
+      return out;
+    };
+    auto optL = options(T.lcol_ld), optS = options(T.lcol_st);
+    auto vec_slots = [&](const std::vector<u64>& lc, const std::vector<u64>& row, std::vector<int>& sl) {
+      sl.clear();
+      for (u64 c : row) { int q = reg_of(lc, c); if (q < 0) return false; sl.push_back(q); }
+      return true;
+    };
+    bool found = false;
+    std::vector<int> sl;
+    for (int pass = 0; pass < 3 && !found; ++pass) {
+      if (pass == 0)        // matrix stores, vectorised loads
+        for (auto& o : optL) {
+          if (vec_slots(T.lcol_st, o.row, sl)) {
+            T.smi_ld = o.kind; T.mat_word_ld = o.word; T.sw_vec = o.row;
+            T.vec_slot_st = sl; T.vec_slot_ld.clear(); found = true; break;
+          }
+        }
+      else if (pass == 1)   // vectorised stores, matrix loads
+        for (auto& o : optS) {
+          if (vec_slots(T.lcol_ld, o.row, sl)) {
+            T.smi_st = o.kind; T.mat_word_st = o.word; T.sw_vec = o.row;
+            T.vec_slot_ld = sl; T.vec_slot_st.clear(); found = true; break;
+          }
+        }
+      else
+        for (auto& a : optL) {
+          for (auto& b : optS)
+            if (a.row == b.row) {
+              T.smi_ld = a.kind; T.mat_word_ld = a.word; T.smi_st = b.kind; T.mat_word_st = b.word;
+              T.sw_vec = a.row; T.vec_slot_ld.clear(); T.vec_slot_st.clear(); found = true; break;
+            }
+          if (found) break;
+        }
+    }
+    // matrix-select bits: up to two of the remaining registers (.x4)
+    auto sel = [&](const std::vector<int>& word, std::vector<int>& s) {
+      s.clear();
+      for (int b = 0; b < R && s.size() < 2; ++b)
+        if (std::find(word.begin(), word.end(), b) == word.end()) s.push_back(b);
+    };
+    if (T.smi_ld != SMI_VEC) sel(T.mat_word_ld, T.mat_sel_ld);
+    if (T.smi_st != SMI_VEC) sel(T.mat_word_st, T.mat_sel_st);
   }
   const int v = int(T.sw_vec.size());
   T.sm_v = v;
@@ -427,11 +538,21 @@ static void plan_smem(TilePlan& T, int maxvec) {
   // 2. b = log2(128 / (2^v w))
   int b = std::max(0, ilog2(u64(std::max(1, 128 / vec_bytes))));
   if (b > n - v) b = n - v;
-  // 3. A_Bank, B_Bank: drop the last log2 max(1, 2^v w / 4) thread vectors
+  // 3. A_Bank, B_Bank: the vectors enumerating one 128-byte wavefront.  Vectorised
+  //    side: its lanes without the last log2 max(1, 2^v w / 4).  Matrix side:
+  //    the vectors addressing the 8 rows of one matrix (lanes 2-4; transposed: word
+  //    bit, lanes 0, 1).
   int drop = ilog2(u64(std::max(1, vec_bytes / 4)));
   std::vector<u64> aThr(T.lcol_ld.begin() + R, T.lcol_ld.begin() + R + 5);
   std::vector<u64> bThr(T.lcol_st.begin() + R, T.lcol_st.begin() + R + 5);
-  std::vector<u64> aBank(aThr.begin(), aThr.end() - drop), bBank(bThr.begin(), bThr.end() - drop);
+  auto bank_of = [&](int kind, const std::vector<u64>& lc, const std::vector<int>& word,
+                     const std::vector<u64>& thr) {
+    if (kind == SMI_MAT) return std::vector<u64>{lc[R + 2], lc[R + 3], lc[R + 4]};
+    if (kind == SMI_MATT) return std::vector<u64>{lc[word[0]], lc[R], lc[R + 1]};
+    return std::vector<u64>(thr.begin(), thr.end() - drop);
+  };
+  std::vector<u64> aBank = bank_of(T.smi_ld, T.lcol_ld, T.mat_word_ld, aThr);
+  std::vector<u64> bBank = bank_of(T.smi_st, T.lcol_st, T.mat_word_st, bThr);
   // 4. E, F, H
   std::vector<u64> E, F;
   for (u64 c : aBank) if (std::find(bBank.begin(), bBank.end(), c) == bBank.end()) E.push_back(c);
@@ -477,15 +598,40 @@ static void plan_smem(TilePlan& T, int maxvec) {
   auto minv = [&](u64 x) { u64 c = 0; if (em.reduce(x, &c)) fail(LL_ERR_UNSUPPORTED, "swizzle: not invertible"); return c; };
   T.smoff_ld.resize(n);
   T.smoff_st.resize(n);
-  for (int k = 0; k < n; ++k) { T.smoff_ld[k] = minv(T.lcol_ld[k]); T.smoff_st[k] = minv(T.lcol_st[k]); }
-  for (int i = 0; i < v; ++i)
-    if (T.smoff_ld[T.vec_slot_ld[i]] != (u64(1) << i) || T.smoff_st[T.vec_slot_st[i]] != (u64(1) << i))
-      fail(LL_ERR_UNSUPPORTED, "swizzle: vector bits not lowest (internal)");
+  for (int q = 0; q < n; ++q) { T.smoff_ld[q] = minv(T.lcol_ld[q]); T.smoff_st[q] = minv(T.lcol_st[q]); }
+  // Thm 5.1: each side's M^{-1}∘L must be divisible by its instruction's tile — the
+  // tile's hardware bits are offset bits 0..v-1 in order, and (Def 4.4) no other
+  // hardware bit reaches them.
+  auto check_tile = [&](int kind, const std::vector<u64>& so, const std::vector<int>& vslot,
+                        const std::vector<int>& word) {
+    std::vector<int> tile;
+    if (kind == SMI_VEC) tile = vslot;
+    else if (kind == SMI_MAT) { tile = word; tile.push_back(R); tile.push_back(R + 1); }
+    else tile = {R + 2, R + 3, R + 4};
+    if (int(tile.size()) != v) fail(LL_ERR_UNSUPPORTED, "swizzle: tile size (internal)");
+    const u64 low = (u64(1) << v) - 1;
+    for (int q = 0; q < n; ++q) {
+      auto it = std::find(tile.begin(), tile.end(), q);
+      if (it != tile.end() ? so[q] != (u64(1) << (it - tile.begin())) : (so[q] & low) != 0)
+        fail(LL_ERR_UNSUPPORTED, "swizzle: M^-1∘L not divisible by the instruction tile (internal)");
+    }
+  };
+  check_tile(T.smi_ld, T.smoff_ld, T.vec_slot_ld, T.mat_word_ld);
+  check_tile(T.smi_st, T.smoff_st, T.vec_slot_st, T.mat_word_st);
   T.smem_elems = u64(1) << n;
   long id1 = 0, id2 = 0;
-  T.predicted_wavefronts_st = sim_wavefronts(T, T.smoff_ld, T.vec_slot_ld, &id1);
-  T.predicted_wavefronts_ld = sim_wavefronts(T, T.smoff_st, T.vec_slot_st, &id2);
+  T.predicted_wavefronts_st = T.smi_ld == SMI_VEC ? sim_wavefronts(T, T.smoff_ld, T.vec_slot_ld, &id1)
+                                                  : sim_mat_wavefronts(T, T.smoff_ld, T.smi_ld, T.mat_word_ld, &id1);
+  T.predicted_wavefronts_ld = T.smi_st == SMI_VEC ? sim_wavefronts(T, T.smoff_st, T.vec_slot_st, &id2)
+                                                  : sim_mat_wavefronts(T, T.smoff_st, T.smi_st, T.mat_word_st, &id2);
   T.ideal_wavefronts = id1 + id2;
+  // shared instructions per thread per tile
+  auto ninstr = [&](int kind, const std::vector<int>& word, const std::vector<int>& s) {
+    if (kind == SMI_VEC) return long(1) << (R - v);
+    return long(1) << (R - int(word.size()) - int(s.size()));
+  };
+  T.smem_instr_st = ninstr(T.smi_ld, T.mat_word_ld, T.mat_sel_ld);
+  T.smem_instr_ld = ninstr(T.smi_st, T.mat_word_st, T.mat_sel_st);
 }
 
 // ---------------------------------------------------------------------------
@@ -502,7 +648,9 @@ static void build_tile(ConvPlan& P, const std::vector<int>& S0, const std::vecto
   std::vector<int> S = S0, D = D0;
   // fold low grid bits into the tile while it is small (common vectors)
   std::vector<int> foldS, foldD;
-  while ((u64(1) << S.size()) * u64(P.w) < u64(tile_bytes) && S.size() < 20) {
+  // faithful σ: folded bits become kernel warps beside the layout's own (≤ 32 warps)
+  const size_t max_fold = (sigma == SIGMA_FAITHFUL && in_cta) ? size_t(std::max(0, 5 - A.in_bits("warp"))) : 64;
+  while ((u64(1) << S.size()) * u64(P.w) < u64(tile_bytes) && S.size() < 20 && foldS.size() < max_fold) {
     size_t g = 0;
     while (g < gridS.size() && ((grid_only_src >> gridS[g]) & 1)) ++g;
     if (g == gridS.size()) break;
@@ -551,7 +699,7 @@ static void build_tile(ConvPlan& P, const std::vector<int>& S0, const std::vecto
     T.xchg = X_SMEM;
   }
   if (T.xchg == X_REGPERM) plan_regperm(T);
-  if (T.xchg == X_SMEM) plan_smem(T, maxvec);
+  if (T.xchg == X_SMEM) plan_smem(T, maxvec, opts ? opts->smem_instr : 0);
   if (T.xchg == X_SMEM) {
     // software-pipelined smem exchange (next tile's loads before this tile's stores):
     // measured slower on every default-sized config — the second register buffer costs
@@ -781,6 +929,19 @@ static std::string ivec_json(const std::vector<T>& v) {
   return o.str();
 }
 
+static std::string smem_instr_name(int kind, bool store, size_t nsel, int v, int w) {
+  std::ostringstream o;
+  if (kind == SMI_VEC) {
+    const int bytes = (1 << v) * w;
+    o << (store ? "st" : "ld") << ".shared";
+    if (bytes > 4) o << ".v" << bytes / 4 << ".b32";
+    else o << ".b" << bytes * 8;
+  } else {
+    o << (store ? "stmatrix" : "ldmatrix") << ".m8n8.x" << (1 << nsel) << (kind == SMI_MATT ? ".trans" : "") << ".b16";
+  }
+  return o.str();
+}
+
 std::string describe(const ConvPlan& P) {
   static const char* cls[] = {"NOOP", "REGPERM", "SHUFFLE", "SMEM", "CTA", "DEVICE"};
   static const char* ex[] = {"noop", "tile", "generic", "device"};
@@ -807,7 +968,13 @@ std::string describe(const ConvPlan& P) {
         << ",\"H\":" << vec_json(T.sw_H) << ",\"C\":" << vec_json(T.sw_C)
         << ",\"smem_bytes\":" << T.smem_elems * T.w
         << ",\"wavefronts_st\":" << T.predicted_wavefronts_st << ",\"wavefronts_ld\":" << T.predicted_wavefronts_ld
-        << ",\"ideal_wavefronts\":" << T.ideal_wavefronts;
+        << ",\"ideal_wavefronts\":" << T.ideal_wavefronts
+        << ",\"smem_store\":\"" << smem_instr_name(T.smi_ld, true, T.mat_sel_ld.size(), T.sm_v, T.w) << "\""
+        << ",\"smem_load\":\"" << smem_instr_name(T.smi_st, false, T.mat_sel_st.size(), T.sm_v, T.w) << "\""
+        << ",\"smem_store_instrs\":" << T.smem_instr_st << ",\"smem_load_instrs\":" << T.smem_instr_ld
+        << ",\"mat_word_ld\":" << ivec_json(T.mat_word_ld) << ",\"mat_sel_ld\":" << ivec_json(T.mat_sel_ld)
+        << ",\"mat_word_st\":" << ivec_json(T.mat_word_st) << ",\"mat_sel_st\":" << ivec_json(T.mat_sel_st)
+        << ",\"smoff_ld\":" << vec_json(T.smoff_ld) << ",\"smoff_st\":" << vec_json(T.smoff_st);
     o << "}";
   }
   if (!P.tune_json.empty()) o << ",\"autotune\":" << P.tune_json;

@@ -212,8 +212,11 @@ def test_swizzle_plans_conflict_free_under_oracle_model():
         Lld, Lst = mk(t["L_ld"]), mk(t["L_st"])
         S = O.layout_from_cols([("offset", t["n"])], out, t["Vec"] + t["Bank"] + t["Seg"])
         assert O.is_memory(S) or O.is_surjective(S)
-        for L in (Lld, Lst):
-            wf, ideal = O.smem_wavefronts(S, L, w, t["Vec"])
+        for L, instr, word in ((Lld, t["smem_store"], t["mat_word_ld"]), (Lst, t["smem_load"], t["mat_word_st"])):
+            if "matrix" in instr:
+                wf, ideal = O.smem_matrix_wavefronts(S, L, w, [L.cols[b] for b in word], trans=".trans" in instr)
+            else:
+                wf, ideal = O.smem_wavefronts(S, L, w, t["Vec"])
             assert wf == ideal
         assert t["wavefronts_st"] + t["wavefronts_ld"] == t["ideal_wavefronts"]
 
@@ -497,7 +500,9 @@ def test_random_memory_layouts_xor_copy_simulated(w):
 def test_planner_faithful_reproduces_gv6_gv8():
     """Under faithful σ (the kernel holds the data exactly as the paper's layouts do) the
     planner's swizzle and shuffle sets equal the hand derivations GV6-GV8 of the paper's
-    constructions (tests/golden/derived_gv6_gv8.json; P:375-387, P:406-426)."""
+    constructions (tests/golden/derived_gv6_gv8.json; P:375-387, P:406-426).  The
+    swizzle derivations use the vectorised ld/st.shared tile, so stmatrix /
+    ldmatrix selection is switched off here (smem_instr="vec")."""
     import json
     import os
     g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "derived_gv6_gv8.json")))
@@ -510,7 +515,8 @@ def test_planner_faithful_reproduces_gv6_gv8():
     for key, (sa, sb), w, fields in [("GV6_config1", (W.C1_A, W.C1_B), 4, ("Vec", "Bank", "Seg")),
                                      ("GV8_config3", W.c3(0), 2, ("Vec", "Bank", "Seg")),
                                      ("GV7_config2", W.c2(0), 2, ("V", "I", "E", "F", "G"))]:
-        p = ll.ll_plan_convert(ll.Layout.from_spec(sa), ll.Layout.from_spec(sb), w, sigma="faithful")
+        p = ll.ll_plan_convert(ll.Layout.from_spec(sa), ll.Layout.from_spec(sb), w, sigma="faithful",
+                               smem_instr="vec")
         t = p.describe()["tile"]
         for f in fields:
             assert t[f] == [flat(e, g[key]["j_bits"]) for e in g[key][f]], (key, f)
@@ -530,3 +536,117 @@ def test_scan_plans():
             "in": [("reg", ["j0", "j1", "j2"]), ("lane", ["i0", "i1", "i2", "i3", "i4"]), ("warp", ["j3", "j4", "j5", "j6"])]}
     d = ll.ll_plan_scan(ll.Layout.from_spec(spec), 1).describe()
     assert d["smem_exchange_bytes"] == 4 * 8 * 512
+
+
+# ----------------------------------------------------------------------------- Thm 5.1
+from tests._matrix_cases import MATRIX_CASES  # noqa: E402
+
+
+def _check_matrix_plan(t, OA, w):
+    """Oracle-side checks of an SMEM tile plan whose sides may use stmatrix / ldmatrix:
+    the oracle's bank model (P:344 fragment semantics; raises unless every matrix row is
+    16 contiguous bytes) counts the wavefronts the planner predicts for each side, and a
+    non-transposed matrix side satisfies Thm 5.1 by the paper's left division (Def 4.4)
+    after renaming the word registers first (P_Reg)."""
+    out = OA.out_dims
+    hw = [("reg", t["R"]), ("lane", 5), ("warp", t["warp_bits"])]
+    S = O.layout_from_cols([("offset", t["n"])], out, t["Vec"] + t["Bank"] + t["Seg"])
+    S_inv = O.right_inverse(S)
+    k = (4 // w).bit_length() - 1
+    for cols, instr, word, pred in ((t["L_ld"], t["smem_store"], t["mat_word_ld"], t["wavefronts_st"]),
+                                    (t["L_st"], t["smem_load"], t["mat_word_st"], t["wavefronts_ld"])):
+        L = O.layout_from_cols(hw, out, cols)
+        if "matrix" not in instr:
+            wf, ideal = O.smem_wavefronts(S, L, w, t["Vec"])
+            assert wf == pred, instr
+            continue
+        wf, ideal = O.smem_matrix_wavefronts(S, L, w, [cols[b] for b in word], trans=".trans" in instr)
+        assert wf == pred, instr
+        if ".trans" in instr:
+            continue
+        # P_Reg: word registers first, then the rest in order
+        regs = list(word) + [b for b in range(t["R"]) if b not in word]
+        cols2 = [cols[b] for b in regs] + cols[t["R"]:]
+        Moff = O.compose(S_inv, O.layout_from_cols(hw, out, cols2))       # hw -> offset
+        T = O.Layout([("reg", k), ("lane", 2)], [("offset", k + 2)],
+                     {"reg": [(1 << i,) for i in range(k)], "lane": [(1 << (k + i),) for i in range(2)]})
+        O.left_divide(Moff, T)     # raises if the tile does not divide
+
+
+@pytest.mark.parametrize("case", MATRIX_CASES, ids=[c[0] for c in MATRIX_CASES])
+def test_matrix_tiles_literal_cases(case):
+    """stmatrix / ldmatrix (.x1/.x2/.x4, .trans) selection on literal layout pairs:
+    the expected instructions, the plan's schedule reproduces the oracle conversion,
+    and the oracle's bank model / Thm 5.1 checks hold."""
+    name, sa, sb, w, (want_st, want_ld) = case
+    d = _sim_check(sa, sb, w, 3, sigma="faithful", force_class="SMEM")
+    t = d["tile"]
+    assert (t["smem_store"], t["smem_load"]) == (want_st, want_ld)
+    assert t["wavefronts_st"] + t["wavefronts_ld"] == t["ideal_wavefronts"]
+    _check_matrix_plan(t, both(sa)[1], w)
+
+
+def test_matrix_tiles_on_paper_configs():
+    """Thm 5.1 selection on the paper's layouts (faithful σ): the wgmma accumulator of
+    config 2 (each thread 4 contiguous bytes, lanes 0,1 along j) is stored with
+    stmatrix.x4 and the blocked side loaded with ld.shared.v4 — 16 instructions per
+    thread per side instead of 32 with the common 8-byte register vector; config 3's
+    blocked [1,8] side also goes through stmatrix (32 instead of 128: -75%, the Table 4
+    kind of smem-instruction reduction).  Coalesced σ on config 3b widens the
+    swizzle vector from 8 to 16 bytes with stmatrix."""
+    cases = [(W.c2(0), 2, "faithful", 16, 32), (W.c3(0), 2, "faithful", 32, 128), (W.c3b(0), 2, "coalesced", None, None)]
+    for (sa, sb), w, sigma, n_mat, n_vec in cases:
+        d = _sim_check(sa, sb, w, 4, sigma=sigma, force_class="SMEM")
+        t = d["tile"]
+        assert t["smem_store"] == "stmatrix.m8n8.x4.b16" and t["smem_load"] == "ld.shared.v4.b32", t
+        assert (1 << len(t["Vec"])) * w == 16
+        _check_matrix_plan(t, both(sa)[1], w)
+        if n_mat:
+            A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
+            tv = ll.ll_plan_convert(A, B, w, sigma=sigma, force_class="SMEM", smem_instr="vec").describe()["tile"]
+            assert t["smem_store_instrs"] == n_mat and tv["smem_store_instrs"] == n_vec
+
+
+def test_matrix_tiles_random_layouts_simulated():
+    """Random distributed pairs (R1) planned with smem_instr = "matrix": every matrix
+    side is bit-exact in the host schedule emulation and passes the oracle checks."""
+    rng = np.random.default_rng(344)
+    out = [("i", 5), ("j", 5)]
+    seen = set()
+    for R in (1, 2, 3):
+        hw = [("reg", R), ("lane", 5), ("warp", 5 - R)]
+        for case in range(24):
+            sa = gen.random_distributed(rng, out, hw)
+            sb = gen.random_distributed(rng, out, hw)
+            w = [1, 2, 4][case % 3]
+            sigma = ("faithful", "coalesced")[case % 2]
+            d = _sim_check(sa, sb, w, case, sigma=sigma, force_class="SMEM", smem_instr="matrix")
+            t = d["tile"]
+            _check_matrix_plan(t, both(sa)[1], w)
+            seen.add(t["smem_store"].split(".")[0] + "/" + t["smem_load"].split(".")[0])
+    assert {"stmatrix/ld", "st/ldmatrix"} <= seen, seen
+
+
+def test_matrix_kernels_emit_stsm_ldsm_sass(tmp_path, monkeypatch):
+    """The specialised sm_100a kernels really use the matrix instructions: SASS of the
+    NVRTC cubins (cuobjdump, no GPU needed) holds STSM / LDSM (.MT88 = transposed)."""
+    import shutil
+    import subprocess
+    cuobjdump = shutil.which("cuobjdump") or "/usr/local/cuda/bin/cuobjdump"
+    if not os.path.exists(cuobjdump):
+        pytest.skip("cuobjdump not available")
+    want = {"x1_mat_to_trans_b16": ("STSM.16.M88 ", "LDSM.16.MT88 "),
+            "x2_mat_mat_b32": ("STSM.16.M88.2", "LDSM.16.M88.2"),
+            "x4_mat_to_vec_b8": ("STSM.16.M88.4", "LDS.128"),
+            "x4_trans_to_vec_b16": ("STSM.16.MT88.4", "LDS.128")}
+    for name, sa, sb, w, _ in MATRIX_CASES:
+        d = tmp_path / name
+        d.mkdir()
+        monkeypatch.setenv("LL_JIT_CACHE", str(d))
+        ll.ll_plan_convert(ll.Layout.from_spec(sa), ll.Layout.from_spec(sb), w, sigma="faithful",
+                           force_class="SMEM").precompile()
+        (cubin,) = list(d.glob("*.cubin"))
+        sass = subprocess.run([cuobjdump, "-sass", str(cubin)], capture_output=True, text=True, check=True).stdout
+        sass = sass.replace(" ;", " ")
+        for mnem in want[name]:
+            assert mnem in sass, (name, mnem)

@@ -445,6 +445,86 @@ def test_unswizzled_config3_conflicts():
     assert wfB == 32 * idB     # lanes run along i (256 B apart): all in one bank
 
 
+def _mat_layouts(rows_log2_cols=3, trans=False):
+    """One 8x8 b16 matrix held as the ldmatrix fragment (PTX m8n8 [HW]):
+    non-transposed, reg bit -> j0, lanes 0,1 -> j1,j2, lanes 2-4 -> i0..i2; transposed,
+    reg bit -> i0, lanes 0,1 -> i1,i2, lanes 2-4 -> j0..j2.  The smem buffer S is the
+    row-major [8, 2^c] tensor (identity memory layout)."""
+    out = [("i", 3), ("j", rows_log2_cols)]
+    if trans:
+        bases = {"reg": [(1, 0)], "lane": [(2, 0), (4, 0), (0, 1), (0, 2), (0, 4)]}
+    else:
+        bases = {"reg": [(0, 1)], "lane": [(0, 2), (0, 4), (1, 0), (2, 0), (4, 0)]}
+    L = O.Layout([("reg", 1), ("lane", 5)], out, bases)
+    return L, O.identity_memory(out)
+
+
+def test_matrix_model_closed_forms():
+    """Bank model of ldmatrix/stmatrix, pinned to textbook bank arithmetic
+    (bank = byte address / 4 mod 32): an 8x8 b16 matrix stored densely (rows 16 B
+    apart) covers one 128-byte segment — 1 wavefront; the same fragment in an [8, 64]
+    b16 row-major tensor has its 8 rows 128 B apart, all in banks 0-3 — 8 wavefronts
+    (8-way conflict); rows 32 B apart ([8, 16]) — 4 rows per group pair: 2-way."""
+    for c, want in [(3, 1), (6, 8), (4, 2)]:
+        L, S = _mat_layouts(c)
+        # widen L with zero-free extra columns: the remaining j bits of the row as regs
+        extra = [(0, 8 << t) for t in range(c - 3)]
+        L = O.Layout([("reg", 1 + len(extra)), ("lane", 5)], L.out_dims,
+                     {"reg": [(0, 1)] + extra, "lane": L.bases["lane"]})
+        wf, ideal = O.smem_matrix_wavefronts(S, L, 2, [1])
+        assert ideal == 1 << len(extra)
+        assert wf == want * ideal, (c, wf, ideal)
+    L, S = _mat_layouts(3, trans=True)
+    assert O.smem_matrix_wavefronts(S, L, 2, [8], trans=True) == (1, 1)   # word: i0
+    # the non-transposed fragment read with .trans is not a valid access
+    L, S = _mat_layouts(3)
+    with pytest.raises(ValueError):
+        O.smem_matrix_wavefronts(S, L, 2, [1], trans=True)
+
+
+def test_matrix_model_agrees_with_thm51_left_division():
+    """Thm 5.1: the instruction lowers M^{-1}∘L iff M^{-1}∘L /_l T exists for
+    T = id_k^{Reg,Off} × id_2^{Thr,Off}, k = log2(4/w).  Two independent
+    formulations — the PTX fragment semantics of the bank model (raises when the
+    rows are not 16 contiguous bytes) and the paper's left division (Def 4.4) — must
+    agree on random bijective (reg, lane) -> smem-offset maps."""
+    rng = np.random.default_rng(51)
+    agree = {True: 0, False: 0}
+    for w in (1, 2, 4):
+        k = (4 // w).bit_length() - 1
+        nreg = k + 2
+        d = nreg + 5
+        out = [("x", d)]
+        T = O.Layout([("reg", k), ("lane", 2)], [("x", k + 2)],
+                     {"reg": [(1 << i,) for i in range(k)], "lane": [(1 << (k + t),) for t in range(2)]})
+        for case in range(150):
+            perm = list(rng.permutation(d))
+            if case % 3 == 0:                      # force the tile bits into place
+                rest = [p for p in perm if p >= k + 2]
+                pos = list(range(k)) + [nreg, nreg + 1]
+                perm = [None] * d
+                for b, p in zip(pos, range(k + 2)):
+                    perm[b] = p
+                it = iter(rest)
+                perm = [p if p is not None else next(it) for p in perm]
+            cols = [1 << int(p) for p in perm]
+            L = O.layout_from_cols([("reg", nreg), ("lane", 5)], out, cols)
+            S = O.identity_memory(out)
+            try:
+                O.smem_matrix_wavefronts(S, L, w, cols[:k])
+                ok_model = True
+            except ValueError:
+                ok_model = False
+            try:
+                O.left_divide(L, T)
+                ok_div = True
+            except ValueError:
+                ok_div = False
+            assert ok_model == ok_div, (w, perm)
+            agree[ok_div] += 1
+    assert agree[True] >= 50 and agree[False] >= 50
+
+
 def _all_subspaces(d, k):
     """All k-dim subspaces of F2^d as sorted tuples of their reduced bases."""
     seen = set()

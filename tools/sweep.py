@@ -82,6 +82,8 @@ def main():
         return big_configs()
     if "small" in only:
         return small_kernels()
+    if "matrix" in only:
+        return matrix_tiles()
     if "all" not in only and "conv" not in only:
         return gather_reduce()
     # raw copy roofline reference
@@ -108,6 +110,19 @@ def main():
     for opts in [dict(), dict(force_class="SMEM"), dict(tile_bytes=65536), dict(thread_bytes=16)]:
         conv_case("c1batch", sa, sb, 4, **opts)
     gather_reduce()
+
+
+def matrix_tiles():
+    """Thm 5.1 instruction selection: stmatrix / ldmatrix vs vectorised
+    ld/st.shared only, same layouts, same bytes."""
+    cases = [("c2 faithful smem", W.c2(16), dict(sigma="faithful", force_class="SMEM")),
+             ("c3 faithful", W.c3(14), dict(sigma="faithful")),
+             ("c3 faithful smem", W.c3(14), dict(sigma="faithful", force_class="SMEM")),
+             ("c3b", W.c3b(14), dict()),
+             ("c3b tb128", W.c3b(14), dict(thread_bytes=128))]
+    for name, (sa, sb), opts in cases:
+        for mode in ("auto", "vec"):
+            conv_case(f"{name} smem_instr={mode}", sa, sb, 2, smem_instr=mode, **opts)
 
 
 def swizzle_case():
