@@ -255,7 +255,8 @@ ll_status ll_convert_host(const void* src_host, void* dst_host, void* dev_buf, s
 /* ll_plan_autotune: measured plan selection for (A, B).  Plans the conversion under
  * each candidate kernel decomposition — `base` (NULL = defaults), thread_bytes 64 /
  * 128 / 256 when base leaves it 0, each also with a forced smem exchange when base
- * does not force a class — compiles every distinct kernel, runs it `iters` times
+ * does not force a class, and each also with smem_instr = 1 (vectorised ld/st.shared
+ * only) when base leaves it 0 (automatic stmatrix / ldmatrix) — compiles every distinct kernel, runs it `iters` times
  * (default 10) on the caller's src / dst (device buffers as for ll_convert; dst is
  * overwritten) on `stream`, and returns the fastest plan; describe lists the
  * candidates and their times ("autotune").  Synchronises `stream`.  Plans without a

@@ -567,7 +567,8 @@ ll_status ll_convert(const void* src, void* dst, void* ws, const ll_plan* p, voi
 }
 
 // Measured plan selection: every candidate kernel decomposition (thread_bytes 64 / 128
-// / 256 and the default, with and without a forced smem exchange) is planned,
+// / 256 and the default, with and without a forced smem exchange, with and without
+// stmatrix / ldmatrix) is planned,
 // compiled and timed on the caller's buffers; the fastest plan is returned.
 ll_status ll_plan_autotune(const ll_layout* A, const ll_layout* B, int w, const ll_plan_opts* base,
                            const void* src, void* dst, void* stream, int iters, ll_plan** out) {
@@ -582,6 +583,12 @@ ll_status ll_plan_autotune(const ll_layout* A, const ll_layout* B, int w, const 
   if (o0.force_class < 0) {
     const size_t nc = cand.size();
     for (size_t i = 0; i < nc; ++i) { ll_plan_opts c = cand[i]; c.force_class = LL_CLASS_SMEM; cand.push_back(c); }
+  }
+  // smem instructions (Thm 5.1): the automatic stmatrix / ldmatrix choice against
+  // vectorised ld/st.shared only (identical plans are timed once)
+  if (o0.smem_instr == 0) {
+    const size_t nc = cand.size();
+    for (size_t i = 0; i < nc; ++i) { ll_plan_opts c = cand[i]; c.smem_instr = 1; cand.push_back(c); }
   }
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   cudaEvent_t e0, e1;
@@ -616,7 +623,8 @@ ll_status ll_plan_autotune(const ll_layout* A, const ll_layout* B, int w, const 
       ms /= float(iters);
       static const char* xc[] = {"copy", "regperm", "shuffle", "smem"};
       log << (first ? "" : ",") << "{\"thread_bytes\":" << c.thread_bytes << ",\"force_smem\":"
-          << (c.force_class == LL_CLASS_SMEM ? "true" : "false") << ",\"xchg\":\"" << xc[P.tile.xchg]
+          << (c.force_class == LL_CLASS_SMEM ? "true" : "false") << ",\"smem_instr\":" << c.smem_instr
+          << ",\"xchg\":\"" << xc[P.tile.xchg]
           << "\",\"R\":" << P.tile.R << ",\"threads\":" << P.tile.threads() << ",\"ms\":" << ms << "}";
       first = false;
       if (!best || ms < best_ms) { best = std::move(p); best_ms = ms; }
