@@ -36,6 +36,15 @@
  *    allocate device memory and never synchronise; asynchronous faults surface
  *    at the caller's synchronisation as CUDA errors.  There is no CPU fallback:
  *    the device entry points return LL_ERR_CUDA when no usable GPU is present.
+ *
+ * ENVIRONMENT (debugging / test hooks, read at planning time)
+ *  - LL_FORCE_CLASS=shuffle|smem: the executed exchange of conversion plans whose
+ *    opts leave force_class automatic (-1).
+ *  - LL_LOG=1: every conversion plan is printed (ll_plan_describe JSON) to stderr.
+ *  - LL_JIT_CACHE=<dir>: the NVRTC cubin cache (default: in-tree .ll_jit_cache/).
+ *  - LL_PDL=0: launch without programmatic dependent launch.
+ *  Host entry points (planning, launches) are wrapped in NVTX ranges named after
+ *  the call (ll_plan_convert, ll_convert, ll_gather, ll_reduce, ll_scan).
  */
 #ifndef LL_H_
 #define LL_H_

@@ -2,7 +2,12 @@
 // ll_status and a thread-local message (nothing throws across the ABI).
 #include <cuda_runtime.h>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include <algorithm>
+#include <cctype>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <sstream>
 
@@ -18,6 +23,35 @@ void plan_device(ConvPlan& P, const ll_plan_opts* opts);
 }  // namespace ll
 
 using namespace ll;
+
+namespace {
+// NVTX range around a host entry point (planning, launches): shows up in Nsight
+// timelines; header-only NVTX v3, a no-op without a tool attached.
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
+
+// Test / debugging hooks read at planning time:
+//   LL_FORCE_CLASS=shuffle|smem  force the executed exchange when the caller's opts
+//                                leave force_class automatic;
+//   LL_LOG=1                     print every conversion plan (describe JSON) to stderr.
+const ll_plan_opts* env_opts(const ll_plan_opts* opts, ll_plan_opts& tmp) {
+  const char* e = std::getenv("LL_FORCE_CLASS");
+  if (!e || !*e || (opts && opts->force_class >= 0)) return opts;
+  if (opts) tmp = *opts; else ll_plan_opts_default(&tmp);
+  std::string v(e);
+  for (auto& c : v) c = char(std::tolower(static_cast<unsigned char>(c)));
+  if (v == "shuffle") tmp.force_class = LL_CLASS_SHUFFLE;
+  else if (v == "smem") tmp.force_class = LL_CLASS_SMEM;
+  else return opts;
+  return &tmp;
+}
+bool env_log() {
+  const char* e = std::getenv("LL_LOG");
+  return e && *e && std::string(e) != "0";
+}
+}  // namespace
 
 #define LL_TRY try {
 #define LL_CATCH                                                  \
@@ -398,9 +432,12 @@ ll_status ll_layout_slice(const ll_layout* L, int dim, ll_layout** out) {
   LL_CATCH
 }
 
-ll_status ll_plan_convert(const ll_layout* A, const ll_layout* B, int w, const ll_plan_opts* opts, ll_plan** plan) {
+ll_status ll_plan_convert(const ll_layout* A, const ll_layout* B, int w, const ll_plan_opts* opts_in, ll_plan** plan) {
   LL_TRY
+  NvtxRange nvtx("ll_plan_convert");
   if (!A || !B || !plan) fail(LL_ERR_INVALID_ARG, "null argument");
+  ll_plan_opts opts_env;
+  const ll_plan_opts* opts = env_opts(opts_in, opts_env);
   auto h = std::make_unique<ll_plan>();
   h->kind = 0;
   if (w == 8) {
@@ -429,6 +466,7 @@ ll_status ll_plan_convert(const ll_layout* A, const ll_layout* B, int w, const l
       }
   }
   if (h->conv->exec == EXEC_TILE) h->conv->source = codegen_tile(*h->conv);
+  if (env_log()) std::fprintf(stderr, "[ll] plan %s\n", describe(*h->conv).c_str());
   *plan = h.release();
   LL_CATCH
 }
@@ -560,6 +598,7 @@ void ll_plan_destroy(ll_plan* p) {
 
 ll_status ll_convert(const void* src, void* dst, void* ws, const ll_plan* p, void* stream) {
   LL_TRY
+  NvtxRange nvtx("ll_convert");
   if (!p || p->kind != 0) fail(LL_ERR_INVALID_ARG, "not a conversion plan");
   if (!src || !dst) fail(LL_ERR_INVALID_ARG, "null buffer");
   return convert_impl(src, dst, ws, p->cp(), static_cast<cudaStream_t>(stream));
@@ -705,6 +744,7 @@ ll_status ll_plan_gather(const ll_layout* L, int axis, int w, const ll_plan_opts
 
 ll_status ll_gather(const void* src, const int32_t* idx, void* dst, const ll_plan* p, void* stream) {
   LL_TRY
+  NvtxRange nvtx("ll_gather");
   if (!p || p->kind != 1) fail(LL_ERR_INVALID_ARG, "not a gather plan");
   if (!src || !idx || !dst) fail(LL_ERR_INVALID_ARG, "null buffer");
   if ((reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(idx) | reinterpret_cast<uintptr_t>(dst)) & 15)
@@ -736,6 +776,7 @@ ll_status ll_plan_scan(const ll_layout* L, int axis, const ll_plan_opts* opts, l
 
 ll_status ll_scan(const float* src, float* dst, const ll_plan* p, void* stream) {
   LL_TRY
+  NvtxRange nvtx("ll_scan");
   if (!p || p->kind != 3) fail(LL_ERR_INVALID_ARG, "not a scan plan");
   if (!src || !dst) fail(LL_ERR_INVALID_ARG, "null buffer");
   if ((reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst)) & 15)
@@ -771,6 +812,7 @@ ll_status ll_plan_reduce_out_elems(const ll_plan* p, size_t* n) {
 
 ll_status ll_reduce(const float* src, float* dst, const ll_plan* p, void* stream) {
   LL_TRY
+  NvtxRange nvtx("ll_reduce");
   if (!p || p->kind != 2) fail(LL_ERR_INVALID_ARG, "not a reduce plan");
   if (!src || !dst) fail(LL_ERR_INVALID_ARG, "null buffer");
   if (reinterpret_cast<uintptr_t>(src) & 15) fail(LL_ERR_MISALIGNED, "src must be 16-byte aligned");

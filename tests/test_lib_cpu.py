@@ -650,3 +650,22 @@ def test_matrix_kernels_emit_stsm_ldsm_sass(tmp_path, monkeypatch):
         sass = sass.replace(" ;", " ")
         for mnem in want[name]:
             assert mnem in sass, (name, mnem)
+
+
+def test_env_hooks_force_class_and_log():
+    """LL_FORCE_CLASS / LL_LOG (include/ll.h ENVIRONMENT) in a fresh process."""
+    import subprocess
+    import sys
+    code = ("import sys; sys.path.insert(0, %r)\n"
+            "import paper_conf_asplos_0001cgrnls0trm26_b200 as ll\n"
+            "from workloads import configs as W\n"
+            "sa, sb = W.c2(0)\n"
+            "p = ll.ll_plan_convert(ll.Layout.from_spec(sa), ll.Layout.from_spec(sb), 2)\n"
+            "print(p.describe()['tile']['xchg'])\n") % os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, LL_FORCE_CLASS="smem", LL_LOG="1")
+    r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, check=True)
+    assert r.stdout.strip() == "smem"
+    assert r.stderr.startswith("[ll] plan {") and '"xchg":"smem"' in r.stderr
+    env = {k: v for k, v in os.environ.items() if k not in ("LL_FORCE_CLASS", "LL_LOG")}
+    r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, check=True)
+    assert r.stdout.strip() == "shuffle" and "[ll] plan" not in r.stderr
