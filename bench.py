@@ -223,6 +223,25 @@ def torch_permute_baseline(torch, A_spec, B_spec, src, w, steps=5):
         y.reshape(-1).view(src.dtype)
 
 
+def size_matched_copy(torch, nbytes, nsets=4):
+    """The copy roofline at a small problem size: torch copy_ moving `nbytes` in total
+    (nbytes/2 read + nbytes/2 written), rotated over `nsets` buffer sets and timed as a
+    stream like the config-4 kernels — launch ramp and tail included, as they are for
+    any kernel of that size.  Context for the config-4 fractions, not the roofline."""
+    n = nbytes // 8
+    bufs = [(torch.empty(n, dtype=torch.int32, device="cuda"), torch.empty(n, dtype=torch.int32, device="cuda"))
+            for _ in range(nsets)]
+    it = [0]
+
+    def f():
+        s = bufs[it[0] % nsets]
+        it[0] += 1
+        s[1].copy_(s[0])
+    ms = _time_stream(f, torch)
+    del bufs
+    return round(8 * n / ms / 1e6, 1)
+
+
 def other_configs(ll, W, torch, peak):
     """The other BASELINE configs (1, 3, 4, 5) measured live on this GPU, each against
     the same copy roofline: GB/s = algorithmic bytes / median time per call.  Inputs
@@ -247,6 +266,8 @@ def other_configs(ll, W, torch, peak):
             ex = d["exec"]
         entry = {"workload": name, "class": d["class"], "executed": ex, "ms": round(ms, 4),
                  "GBps": round(gbs, 1), "frac": round(gbs / peak, 3)}
+        if "tile" in d and d["tile"]["xchg"] == "smem":     # Thm 5.1 instruction choice
+            entry["smem_instructions"] = [d["tile"]["smem_store"], d["tile"]["smem_load"]]
         if comm is None:
             tb, y = torch_permute_baseline(torch, sa, sb, src, w)
             entry["torch_permute_GBps"] = tb["GBps"]
@@ -274,6 +295,8 @@ def other_configs(ll, W, torch, peak):
                 "class": p1.cls, "us_per_conversion": round(ms, 4)})
     conv("config 1 batch: 2^20 Fig.-1 tiles (16x16 fp32, A -> B = A^T), 1+1 GiB", *W.c1_batched(20), 4)
     conv("config 3: 16384 tiles 256x128 fp16 blocked -> transposed blocked (optimal swizzle), 1+1 GiB", *W.c3(14), 2)
+    conv("config 3b: 16384 tiles 256x128 fp16, [8,8] per thread row- -> column-order (16-byte rows via stmatrix), 1+1 GiB",
+         *W.c3b(14), 2)
     conv("config 5-T, P=1: 32768^2 bf16 row-major -> column-major, 2+2 GiB", *W.c5T(0), 2)
     conv("config 5, P=8 loopback on one GPU: row- -> column-sharded, peer-store kernels, 2+2 GiB",
          *W.c5(3), 2, comm=ll.Comm.loopback(8), exchange="peer")
@@ -306,7 +329,8 @@ def other_configs(ll, W, torch, peak):
         out.append({"workload": f"config 4 gather: [4096,4096] fp32, {fam} [128,32] tiles", "class": "gather",
                     "executed": d["exchange"] + (" (TMA stages)" if d.get("tma") else ""), "ms": round(ms, 4),
                     "GBps": round(gbs, 1), "frac": round(gbs / peak, 3),
-                    "torch_gather_same_bytes_GBps": round(12 * n / ms_t / 1e6, 1)})
+                    "torch_gather_same_bytes_GBps": round(12 * n / ms_t / 1e6, 1),
+                    "size_matched_copy_GBps": size_matched_copy(torch, 12 * n)})
         del tsets
         L = ll.Layout.from_spec(W.c4("reduce", fam))
         p = ll.ll_plan_reduce(L, 1)
@@ -328,7 +352,8 @@ def other_configs(ll, W, torch, peak):
         out.append({"workload": f"config 4 reduce: [4096,4096] fp32 -> [4096,32], {fam} [128,128] tiles",
                     "class": "reduce", "executed": "tree + shfl.bfly" + (" (TMA stages)" if p.describe().get("tma") else ""),
                     "ms": round(ms, 4), "GBps": round(gbs, 1), "frac": round(gbs / peak, 3),
-                    "torch_sum_same_bytes_GBps": round((4 * n + 4 * p.out_elems()) / ms_t / 1e6, 1)})
+                    "torch_sum_same_bytes_GBps": round((4 * n + 4 * p.out_elems()) / ms_t / 1e6, 1),
+                    "size_matched_copy_GBps": size_matched_copy(torch, 4 * n + 4 * p.out_elems())})
         # scan (N3): inclusive prefix sum along the axis inside each [128, 128] tile
         p = ll.ll_plan_scan(L, 1)
         ssets = [(rs[0], torch.empty_like(rs[0])) for rs in rsets]
@@ -349,7 +374,8 @@ def other_configs(ll, W, torch, peak):
         out.append({"workload": f"config 4 scan (N3): [4096,4096] fp32 inclusive prefix sum inside {fam} [128,128] tiles",
                     "class": "scan", "executed": f"{d['steps']} bit-doubling steps, {d['shuffles_per_elem']} shuffles/elem",
                     "ms": round(ms, 4), "GBps": round(gbs, 1), "frac": round(gbs / peak, 3),
-                    "torch_cumsum_same_bytes_GBps": round(8 * n / ms_t / 1e6, 1)})
+                    "torch_cumsum_same_bytes_GBps": round(8 * n / ms_t / 1e6, 1),
+                    "size_matched_copy_GBps": size_matched_copy(torch, 8 * n)})
         del sets, rsets, ssets
     torch.cuda.empty_cache()
     return out
