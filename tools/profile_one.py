@@ -16,6 +16,7 @@ from workloads import configs as W  # noqa: E402
 ap = argparse.ArgumentParser()
 ap.add_argument("--case", default="c2")
 ap.add_argument("--iters", type=int, default=3)
+ap.add_argument("--opts", default="{}", help="extra ll_plan_convert options as JSON")
 a = ap.parse_args()
 
 conv = {"c2": (W.c2(16), 2, {}), "c2smem": (W.c2(16), 2, {"force_class": "SMEM"}),
@@ -46,6 +47,8 @@ if a.case == "c5peer":
         ll.ll_convert(src, dst, p)
 elif a.case in conv:
     (sa, sb), w, opts = conv[a.case]
+    import json
+    opts = dict(opts, **json.loads(a.opts))
     A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
     p = ll.ll_plan_convert(A, B, w, **opts)
     n = (1 << A.d_in) * w // 2
