@@ -233,7 +233,9 @@ ll_status ll_plan_class(const ll_plan* plan, ll_class* cls);
 /* Workspace needed by ll_convert (> 0 only for DEVICE plans). */
 ll_status ll_plan_workspace_bytes(const ll_plan* plan, size_t* bytes);
 /* JSON description: class, executed exchange, V/I/E/F/G/R, swizzle columns,
- * rounds, predicted wavefronts, launch geometry.  Truncates to cap bytes. */
+ * rounds, predicted wavefronts, the smem instruction of each side (Thm 5.1:
+ * "smem_store" / "smem_load", e.g. "stmatrix.m8n8.x4.b16", "ld.shared.v4.b32") and
+ * their counts per thread per tile, launch geometry.  Truncates to cap bytes. */
 ll_status ll_plan_describe(const ll_plan* plan, char* json, size_t cap);
 /* Specialised CUDA source of the plan's kernel (empty if none). */
 ll_status ll_plan_source(const ll_plan* plan, char* buf, size_t cap, size_t* needed);
