@@ -69,20 +69,34 @@ std::string codegen_tile(const ConvPlan& Pl) {
   o << "  static constexpr bool PIPE = " << (T.pipe ? "true" : "false") << ";\n";
   // per-thread-contiguous loads (faithful σ) re-use sectors across instructions
   o << "  static constexpr bool LD_L1 = " << (T.sigma == SIGMA_FAITHFUL ? "true" : "false") << ";\n";
+  // XOR-copy plans: a src column may reach below the vector (bits [0, VLD)): that part is
+  // an element XOR inside the aligned src vector (in-vector XOR, LD_LO / GRID_LD_LO),
+  // the rest a byte offset
+  const u64 lowm = (u64(1) << T.vld) - 1;
+  bool invec = false;
+  for (size_t b = size_t(T.vld); b < T.ld_xcol.size(); ++b) invec |= (T.ld_xcol[b] & lowm) != 0;
+  for (u64 c : T.grid_src_xcol) invec |= (c & lowm) != 0;
   std::vector<u64> ldc, stc;
+  std::vector<uint32_t> ldlo, gridlo;
   for (int b = 0; b < T.n; ++b) {
-    ldc.push_back(T.ld_xcol.empty() ? (u64(1) << (T.ld_bit[b] + lw)) : (T.ld_xcol[b] << lw));
+    const bool vecbit = b < T.vld;
+    ldc.push_back(T.ld_xcol.empty() ? (u64(1) << (T.ld_bit[b] + lw))
+                                    : ((vecbit ? T.ld_xcol[b] : (T.ld_xcol[b] & ~lowm)) << lw));
+    ldlo.push_back(T.ld_xcol.empty() || vecbit ? 0u : uint32_t(T.ld_xcol[b] & lowm));
     stc.push_back(u64(1) << (T.st_bit[b] + lw));
   }
+  for (u64 c : T.grid_src_xcol) gridlo.push_back(uint32_t(c & lowm));
   o << arr("u64", "LD_COL", ldc) << arr("u64", "ST_COL", stc);
   o << "  static constexpr bool LD_XOR = " << (T.ld_xcol.empty() ? "false" : "true") << ";\n";
+  o << "  static constexpr bool LD_INVEC = " << (invec ? "true" : "false") << ";\n";
+  o << arr("u32", "LD_LO", ldlo) << arr("u32", "GRID_LD_LO", gridlo);
   if (T.grid_src_xcol.empty()) {
     emit_grid(o, T.grid_src_bit, T.grid_dst_bit, lw);
   } else {
     // XOR grid: per-bit src / dst offsets (never contiguous shifts)
     std::vector<u64> ld, st;
     for (size_t g = 0; g < T.grid_dst_bit.size(); ++g) {
-      ld.push_back(T.grid_src_xcol[g] << lw);
+      ld.push_back((T.grid_src_xcol[g] & ~lowm) << lw);
       st.push_back(u64(1) << (T.grid_dst_bit[g] + lw));
     }
     o << icon("G", T.grid_dst_bit.size()) << "  static constexpr bool GRID_CONTIG = false;\n"

@@ -159,6 +159,53 @@ template <class P, int K> struct StOff {
   }
 };
 
+// In-vector XOR of thread-local vector K (XOR-copy plans, LD_INVEC): the element XOR
+// its register bits contribute inside the aligned src vector (compile time).
+template <class P, int K> struct LdLo {
+  static constexpr u32 value() {
+    u32 c = 0;
+    for (int b = P::VLD; b < P::R; ++b) if (((K << P::VLD) >> b) & 1) c ^= P::LD_LO[b];
+    return c;
+  }
+};
+
+// Permute the 2^VL elements of W bytes of vector K by element index XOR c (runtime):
+// out element e = in element e ^ c.  Word-index bits by conditional swaps (selp),
+// sub-word bits by one byte permute (prmt) per word.  Vectors of >= 4 bytes.
+template <int W, int VL, int K, int NW>
+__device__ __forceinline__ void xor_perm_vec(u32 (&r)[NW], u32 c) {
+  constexpr int VB = W << VL;
+  static_assert(VB >= 4, "in-vector XOR needs vectors of >= 4 bytes");
+  constexpr int NWV = VB / 4;                  // words in the vector
+  constexpr int EPW = W < 4 ? 4 / W : 1;       // elements per word
+  constexpr int SH = EPW == 4 ? 2 : (EPW == 2 ? 1 : 0);
+  constexpr int W0 = (K << VL) * W / 4;        // first word of the vector
+  if constexpr (SH > 0) {
+    const u32 ce = c & (EPW - 1);
+    u32 sel;
+    if constexpr (W == 2) sel = ce ? 0x1032u : 0x3210u;
+    else sel = (0u ^ ce) | ((1u ^ ce) << 4) | ((2u ^ ce) << 8) | ((3u ^ ce) << 12);
+    static_for<NWV>([&](auto q) {
+      constexpr int Q = decltype(q)::value;
+      r[W0 + Q] = __byte_perm(r[W0 + Q], 0u, sel);
+    });
+  }
+  const u32 cw = c >> SH;
+  static_for<(NWV > 1 ? (NWV == 2 ? 1 : 2) : 0)>([&](auto t) {
+    constexpr int T = decltype(t)::value;
+    const bool p = (cw >> T) & 1u;
+    static_for<NWV>([&](auto j) {
+      constexpr int J = decltype(j)::value;
+      constexpr int JX = J ^ (1 << T);
+      if constexpr (JX > J) {
+        const u32 a = r[W0 + J], b = r[W0 + JX];
+        r[W0 + J] = p ? b : a;
+        r[W0 + JX] = p ? a : b;
+      }
+    });
+  });
+}
+
 // Per-thread base from the lane / warp columns (runtime lane, warp).
 template <class P, bool LD>
 __device__ __forceinline__ u64 thread_base(u32 lane, u32 warp) {
@@ -607,17 +654,38 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, Dst D, 
     return;
   }
   // a5: HBM load of a src tile (16-byte vectors; coalesced under σ_ld)
+  // in-vector XOR of this thread (lane / warp columns), XOR-copy plans only
+  u32 lo_thr = 0;
+  if constexpr (P::LD_INVEC) {
+    static_for<5>([&](auto q) {
+      constexpr int T = decltype(q)::value;
+      if ((lane >> T) & 1) lo_thr ^= P::LD_LO[P::R + T];
+    });
+    static_for<P::WB>([&](auto q) {
+      constexpr int T = decltype(q)::value;
+      if ((warp >> T) & 1) lo_thr ^= P::LD_LO[P::R + 5 + T];
+    });
+  }
   auto load_tile = [&](u32 (&r)[P::NW], u64 t) {
     const u64 sofs = tile_base<P, true>(t) ^ ld_thr;
     const u8* s = src + sofs;
+    u32 lo = lo_thr;
+    if constexpr (P::LD_INVEC) {
+      static_for<P::G>([&](auto g) {
+        constexpr int Gi = decltype(g)::value;
+        if ((t >> Gi) & 1) lo ^= P::GRID_LD_LO[Gi];
+      });
+    }
     static_for<(1 << (P::R - P::VLD))>([&](auto k) {
       constexpr int K = decltype(k)::value;
       // XOR-copy plans (non-permutation Q): register and thread offsets share bits,
       // so they combine by XOR; permutation plans' bits are disjoint (immediate add)
-      if constexpr (P::LD_XOR)
+      if constexpr (P::LD_XOR) {
         load_vec<P::W, P::VLD, K, P::NW, P::LD_L1>(r, src + (sofs ^ LdOff<P, K>::value()));
-      else
+        if constexpr (P::LD_INVEC) xor_perm_vec<P::W, P::VLD, K, P::NW>(r, lo ^ LdLo<P, K>::value());
+      } else {
         load_vec<P::W, P::VLD, K, P::NW, P::LD_L1>(r, s + LdOff<P, K>::value());
+      }
     });
   };
   // a10: HBM store of a dst tile (and of its broadcast replicas)

@@ -855,16 +855,24 @@ std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, 
     // below bit v, so each vector's 2^v elements are contiguous and aligned in src
     int v = 0;
     while (v < vmax && v < nB && P->Q[v] == (u64(1) << v)) ++v;
+    // Other columns may reach below bit v (a swizzle that XORs inside the vector, e.g.
+    // Def 4.11 with vec < 16 bytes): each dst vector's elements are then one aligned src
+    // vector, permuted by an element XOR — loaded whole and permuted in registers
+    // (in-vector XOR, vectors of >= 4 bytes; LL_XOR_INVEC=0 disables).  Otherwise the
+    // vector shrinks until no column reaches below it.
+    const char* ie = std::getenv("LL_XOR_INVEC");
+    const bool invec = !(ie && std::string(ie) == "0") && (w << v) >= 4;
     for (;;) {
       bool clean = true;
       for (int k = v; k < nB; ++k) if (P->Q[k] & ((u64(1) << v) - 1)) clean = false;
-      if (clean || v == 0) break;
+      if (clean || v == 0 || invec) break;
       --v;
     }
+    const u64 lowm = (u64(1) << v) - 1;
     // the low lane bits must keep whole 32-byte sectors together: Q maps dst bits [v, v+2)
-    // to src bits of single weight
+    // to src bits of single weight above the vector
     bool rowlocal = true;
-    for (int k = v; k < std::min(nB, v + 2); ++k) if (popc(P->Q[k]) != 1) rowlocal = false;
+    for (int k = v; k < std::min(nB, v + 2); ++k) if (popc(P->Q[k] & ~lowm) != 1) rowlocal = false;
     if (rowlocal) {
       TilePlan& T = P->tile;
       T = TilePlan();

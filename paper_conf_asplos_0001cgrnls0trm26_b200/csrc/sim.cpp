@@ -46,7 +46,12 @@ void simulate_tile(const ConvPlan& P, const uint8_t* src, uint8_t* dst) {
         u64 hw = u64(e) | (u64(th) << R);
         struct_off a = ld_off(hw);
         u64 base = sb ^ a.thr;
-        u64 idx = (ld_xor ? (base ^ a.reg) : (base + a.reg)) + a.elem;
+        // XOR-copy plans: as the kernel does it — an aligned vector load at the high part
+        // of the XOR, element e taken from position e ^ (low part) (in-vector XOR, when a
+        // swizzle reaches below the vector)
+        const u64 vmask = (u64(1) << T.vld) - 1;
+        const u64 x = base ^ a.reg;
+        u64 idx = ld_xor ? ((x & ~vmask) + (a.elem ^ (x & vmask))) : (base + a.reg + a.elem);
         in[size_t(th) * E + e] = getv(src + idx * w);
       }
     if (T.xchg == X_COPY) {

@@ -495,6 +495,40 @@ def test_swizzled_memory_layout_gpu():
     assert np.array_equal(got[off.reshape(-1)], T)
 
 
+@pytest.mark.parametrize("w", [1, 2, 4, 8])
+def test_swizzled_memory_layouts_in_vector_xor_gpu(w):
+    """Def 4.11 swizzles whose XOR reaches below the 16-byte vector (vec * w < 16):
+    the XOR-copy kernel loads whole aligned src vectors and permutes the elements in
+    registers (in-vector XOR).  Both directions, every parameter set, 256 x 256, each
+    element (i, j) found at i*2^8 + the Def 4.11 offset (oracle formula)."""
+    m = n = 8
+    R = ll.Layout([("offset", m + n)], [("d0", m), ("d1", n)],
+                  {"offset": [((1 << (k - n)) if k >= n else 0, (1 << k) if k < n else 0) for k in range(m + n)]})
+    rng = np.random.default_rng(40 + w)
+    i = np.arange(1 << m)[:, None]
+    j = np.arange(1 << n)[None, :]
+    for vec, pp, mp in [(1, 1, 8), (2, 1, 8), (4, 2, 4), (1, 2, 8), (1, 1, 4), (8, 1, 8), (16, 1, 8)]:
+        S = ll.ll_layout_mma_swizzle(m, n, vec, pp, mp)
+        off = ((i << n) + np.vectorize(lambda a, b: O.mma_swizzle_offset(int(a), int(b), vec, pp, mp))(i, j)).reshape(-1)
+        T = gen.random_bits(rng, 1 << (m + n), w)
+        for A, B in ((R, S), (S, R)):
+            plan = ll.ll_plan_convert(A, B, w)
+            d = plan.describe()
+            assert d["exec"] == "tile" and (1 << d["tile"]["vld"]) * min(w, 4) == 16, d["tile"]["vld"]
+            src = T if A is R else _scatter(T, off)
+            d_dst = empty_device(1 << (m + n), w)
+            ll.ll_convert(to_device(src), d_dst, plan)
+            got = from_device(d_dst, w)
+            want = _scatter(T, off) if A is R else T
+            assert np.array_equal(got, want), (vec, pp, mp, A is R)
+
+
+def _scatter(T, off):
+    out = np.empty_like(T)
+    out[off] = T
+    return out
+
+
 @pytest.mark.gpu
 def test_e1_exhaustive_generic_gpu():
     """E1 on the GPU, exhaustive: all 8! = 40320 bijective relabelings B

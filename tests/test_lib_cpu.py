@@ -444,7 +444,7 @@ def test_exhaustive_fig1_all_40320():
     assert counts.get("NOOP") == 1
 
 
-@pytest.mark.parametrize("vec,pp,mp", [(8, 1, 8), (4, 2, 4), (8, 2, 4), (2, 1, 8)])
+@pytest.mark.parametrize("vec,pp,mp", [(8, 1, 8), (4, 2, 4), (8, 2, 4), (2, 1, 8), (1, 1, 8), (1, 2, 4)])
 def test_swizzled_memory_layout_xor_copy(vec, pp, mp):
     """Row-major -> Def 4.11 mma-swizzled memory layout and back: the pull
     map has 2-bit columns; the planner runs it as a vectorised XOR-column copy kernel
@@ -458,6 +458,7 @@ def test_swizzled_memory_layout_xor_copy(vec, pp, mp):
     for A, B in ((R, S), (S, R)):
         p = ll.ll_plan_convert(A, B, 2)
         assert p.describe()["exec"] == "tile"
+        assert p.describe()["tile"]["vld"] == 3      # whole 16-byte vectors (in-vector XOR below)
         OA = O.layout_from_cols([("offset", m + n)], [("d0", m), ("d1", n)], A.cols())
         OB = O.layout_from_cols([("offset", m + n)], [("d0", m), ("d1", n)], B.cols())
         src = O.pack(OA, T)
@@ -669,3 +670,23 @@ def test_env_hooks_force_class_and_log():
     env = {k: v for k, v in os.environ.items() if k not in ("LL_FORCE_CLASS", "LL_LOG")}
     r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, check=True)
     assert r.stdout.strip() == "shuffle" and "[ll] plan" not in r.stderr
+
+
+@pytest.mark.parametrize("w", [1, 4, 8])
+def test_swizzled_memory_layout_in_vector_xor_other_widths(w):
+    """In-vector XOR copies for 1-, 4- and 8-byte elements (the bf16 case is above):
+    16-byte vectors for every Def 4.11 parameter set, emulated schedule == oracle."""
+    m = n = 6
+    row = O.identity_memory([("i", m), ("j", n)])
+    R = ll.Layout(row.in_dims, [("d0", m), ("d1", n)], {"offset": [((c >> n), c & ((1 << n) - 1)) for c in row.cols]})
+    rng = np.random.default_rng(w)
+    for vec, pp, mp in [(1, 1, 8), (2, 1, 8), (4, 2, 4), (8, 1, 8), (1, 2, 4)]:
+        S = ll.ll_layout_mma_swizzle(m, n, vec, pp, mp)
+        for A, B in ((R, S), (S, R)):
+            p = ll.ll_plan_convert(A, B, w)
+            t = p.describe()["tile"]
+            assert (1 << t["vld"]) * min(w, 4) == 16
+            OA = O.layout_from_cols([("offset", m + n)], [("d0", m), ("d1", n)], A.cols())
+            OB = O.layout_from_cols([("offset", m + n)], [("d0", m), ("d1", n)], B.cols())
+            src = O.pack(OA, gen.random_bits(rng, 1 << (m + n), w))
+            assert np.array_equal(p.simulate(src, 1 << (m + n)), O.convert(OA, OB, src)), (vec, pp, mp)

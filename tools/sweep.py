@@ -84,6 +84,8 @@ def main():
         return small_kernels()
     if "matrix" in only:
         return matrix_tiles()
+    if "invec" in only:
+        return invec_swizzles()
     if "all" not in only and "conv" not in only:
         return gather_reduce()
     # raw copy roofline reference
@@ -123,6 +125,31 @@ def matrix_tiles():
     for name, (sa, sb), opts in cases:
         for mode in ("auto", "vec"):
             conv_case(f"{name} smem_instr={mode}", sa, sb, 2, smem_instr=mode, **opts)
+
+
+def invec_swizzles():
+    """Def 4.11 swizzles whose XOR reaches below the 16-byte vector: in-vector XOR copy
+    (default) vs shrinking the vector (LL_XOR_INVEC=0), 16384^2 elements, both directions."""
+    m = n = 14
+    R = ll.Layout([("offset", m + n)], [("d0", m), ("d1", n)],
+                  {"offset": [((1 << (k - n)) if k >= n else 0, (1 << k) if k < n else 0) for k in range(m + n)]})
+    for w in (1, 2, 4):
+        for vec, pp, mp in [(1, 1, 8), (2, 1, 8), (4, 2, 4), (8, 1, 8)]:
+            S = ll.ll_layout_mma_swizzle(m, n, vec, pp, mp)
+            for mode in ("1", "0"):
+                os.environ["LL_XOR_INVEC"] = mode
+                p = ll.ll_plan_convert(R, S, w)
+                p.prepare()
+                nbytes = (1 << (m + n)) * w
+                src = torch.randint(-2 ** 15, 2 ** 15, (nbytes // 2,), dtype=torch.int16, device="cuda")
+                dst = torch.empty_like(src)
+                ms = time_fn(lambda: ll.ll_convert(src, dst, p))
+                gbs = 2 * nbytes / ms / 1e6
+                print(json.dumps({"case": f"row-major -> mma swizzle vec={vec} pp={pp} mp={mp}, 16384^2 x {w} B",
+                                  "in_vector_xor": mode == "1", "vld": p.describe()["tile"]["vld"],
+                                  "ms": round(ms, 4), "GBps": round(gbs, 1), "frac_6539": round(gbs / 6539.5, 3)}), flush=True)
+                del src, dst
+    os.environ.pop("LL_XOR_INVEC", None)
 
 
 def swizzle_case():
