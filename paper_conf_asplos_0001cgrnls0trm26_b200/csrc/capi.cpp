@@ -700,6 +700,11 @@ ll_status ll_convert_host(const void* src_host, void* dst_host, void* dev_buf, s
     for (size_t k = 0; k < g; ++k)
       if (T.grid_src_bit[k] != ns - int(g) + int(k) || T.grid_dst_bit[k] != nd - int(g) + int(k))
         fail(LL_ERR_UNSUPPORTED, "ll_convert_host: the CTA grid is not the top bits of both buffers");
+    // XOR (linear) grids: a chunk's tiles index their src by the global tile number, so
+    // every grid column must be exactly its top src bit
+    for (size_t k = 0; k < T.grid_src_xcol.size(); ++k)
+      if (T.grid_src_xcol[k] != (u64(1) << T.grid_src_bit[k]))
+        fail(LL_ERR_UNSUPPORTED, "ll_convert_host: the CTA grid's src columns are not plain top bits");
     ntiles = u64(1) << g;
     tile_src >>= g;
     tile_dst >>= g;

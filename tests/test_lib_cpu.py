@@ -690,3 +690,24 @@ def test_swizzled_memory_layout_in_vector_xor_other_widths(w):
             OB = O.layout_from_cols([("offset", m + n)], [("d0", m), ("d1", n)], B.cols())
             src = O.pack(OA, gen.random_bits(rng, 1 << (m + n), w))
             assert np.array_equal(p.simulate(src, 1 << (m + n)), O.convert(OA, OB, src)), (vec, pp, mp)
+
+
+def test_convert_host_refuses_xor_grids():
+    """ll_convert_host chunks the batch by CTA tiles; a Def 4.11 swizzle's XOR grid
+    (row bits XOR into column bits) indexes src by the global tile number, so the call
+    is refused up front (LL_ERR_UNSUPPORTED) rather than computed per chunk."""
+    import ctypes as C
+    m = n = 10
+    row = O.identity_memory([("i", m), ("j", n)])
+    R = ll.Layout(row.in_dims, [("d0", m), ("d1", n)], {"offset": [((c >> n), c & ((1 << n) - 1)) for c in row.cols]})
+    S = ll.ll_layout_mma_swizzle(m, n, 8, 16, 8)       # row bits 4-6 XOR into the columns
+    p = ll.ll_plan_convert(R, S, 2)
+    t = p.describe()["tile"]
+    assert t["grid_dst_bit"] and t["n"] < n + 4     # row bit 4 is a grid bit
+    h = np.zeros(1 << (m + n), dtype=np.uint16)
+    dev = np.zeros(1 << 16, dtype=np.uint8)
+    streams = (C.c_void_p * 1)(None)
+    st = ll._lib.ll_convert_host(h.ctypes.data, h.ctypes.data, (dev.ctypes.data + 15) // 16 * 16, 1 << 15,
+                                 p.handle, 1, streams)
+    assert ll.STATUS[st] == "UNSUPPORTED"
+    assert b"grid" in ll._lib.ll_last_error()

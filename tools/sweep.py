@@ -86,6 +86,8 @@ def main():
         return matrix_tiles()
     if "invec" in only:
         return invec_swizzles()
+    if "generic" in only:
+        return generic_maps()
     if "all" not in only and "conv" not in only:
         return gather_reduce()
     # raw copy roofline reference
@@ -150,6 +152,30 @@ def invec_swizzles():
                                   "ms": round(ms, 4), "GBps": round(gbs, 1), "frac_6539": round(gbs / 6539.5, 3)}), flush=True)
                 del src, dst
     os.environ.pop("LL_XOR_INVEC", None)
+
+
+def generic_maps():
+    """Linear maps outside the specialised decompositions (random Def 4.14 memory
+    layouts, R2; a transpose into a swizzled layout): the runtime-generic kernel."""
+    import numpy as np
+    from workloads import gen
+    rng = np.random.default_rng(5)
+    d = 28
+    for w in (2, 4):
+        for case in range(3):
+            ca, cb = gen.random_memory_cols(rng, d), gen.random_memory_cols(rng, d)
+            A = ll.Layout([("offset", d)], [("x", d)], {"offset": [(c,) for c in ca]})
+            B = ll.Layout([("offset", d)], [("x", d)], {"offset": [(c,) for c in cb]})
+            p = ll.ll_plan_convert(A, B, w)
+            p.prepare()
+            nbytes = (1 << d) * w
+            src = torch.randint(-2 ** 15, 2 ** 15, (nbytes // 2,), dtype=torch.int16, device="cuda")
+            dst = torch.empty_like(src)
+            ms = time_fn(lambda: ll.ll_convert(src, dst, p))
+            gbs = 2 * nbytes / ms / 1e6
+            print(json.dumps({"case": f"random R2 memory layouts 2^{d} x {w} B #{case}", "exec": p.describe()["exec"],
+                              "ms": round(ms, 4), "GBps": round(gbs, 1), "frac_6539": round(gbs / 6539.5, 3)}), flush=True)
+            del src, dst
 
 
 def swizzle_case():
