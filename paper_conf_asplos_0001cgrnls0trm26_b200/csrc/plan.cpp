@@ -634,6 +634,8 @@ static void plan_smem(TilePlan& T, int maxvec, int smem_instr) {
   T.smem_instr_ld = ninstr(T.smi_st, T.mat_word_st, T.mat_sel_st);
 }
 
+static void plan_exchange(ConvPlan& P, const ll_plan_opts* opts);
+
 // ---------------------------------------------------------------------------
 static void build_tile(ConvPlan& P, const std::vector<int>& S0, const std::vector<int>& D0,
                        std::vector<int> gridS, std::vector<int> gridD, const ll_plan_opts* opts,
@@ -682,6 +684,14 @@ static void build_tile(ConvPlan& P, const std::vector<int>& S0, const std::vecto
   T.lcol_ld.resize(T.n);
   T.lcol_st.resize(T.n);
   for (int b = 0; b < T.n; ++b) { T.lcol_ld[b] = A.cols[T.ld_bit[b]]; T.lcol_st[b] = B.cols[T.st_bit[b]]; }
+  plan_exchange(P, opts);
+}
+
+// The exchange L_ld -> L_st of a tile plan whose kernel layouts (lcol_ld / lcol_st) are
+// set: its class (copy, register permutation, shuffle, smem) and that class's plan.
+static void plan_exchange(ConvPlan& P, const ll_plan_opts* opts) {
+  TilePlan& T = P.tile;
+  const int maxvec = default_int(opts, &ll_plan_opts::max_vec_bytes, 16);
   // exchange class of L_ld -> L_st
   bool same_lane = true, same_warp = true, same_reg = true;
   for (int t = 0; t < 5; ++t) same_lane &= T.lcol_ld[T.R + t] == T.lcol_st[T.R + t];
@@ -699,7 +709,20 @@ static void build_tile(ConvPlan& P, const std::vector<int>& S0, const std::vecto
     T.xchg = X_SMEM;
   }
   if (T.xchg == X_REGPERM) plan_regperm(T);
-  if (T.xchg == X_SMEM) plan_smem(T, maxvec, opts ? opts->smem_instr : 0);
+  if (T.xchg == X_SMEM) {
+    // Tiles of general linear maps (build_linear_tile): the kernel layouts' columns need
+    // not be unit vectors, and a wide Vec may leave no complement that every other bit of
+    // both sides lies in (M^{-1}∘L not divisible by the instruction tile, Thm 5.1): the
+    // vector then narrows until the tile divides (at one element it always does).
+    for (int mv = maxvec;; mv /= 2) {
+      try {
+        plan_smem(T, mv, opts ? opts->smem_instr : 0);
+        break;
+      } catch (const Error& e) {
+        if (mv <= T.w) throw;
+      }
+    }
+  }
   if (T.xchg == X_SMEM) {
     // software-pipelined smem exchange (next tile's loads before this tile's stores):
     // measured slower on every default-sized config — the second register buffer costs
@@ -735,6 +758,111 @@ static void choose_cta_tile(const std::vector<int>& pi, int nloc, int c_bits,
     if (inT[k]) { D.push_back(k); S.push_back(pi[k]); }
     else { gD.push_back(k); gS.push_back(pi[k]); }
   }
+}
+
+// General invertible pull maps (memory layouts whose Q scatters the low bits: any Def
+// 4.14 layout, Thm 4.13; products of swizzles and transposes).  A CTA tile is
+// the dst subspace spanned by a set D of dst bits chosen so that Q(span D) contains the
+// low src bits [0, c): loads (XOR-addressed src vectors, LD_XOR) and stores both run
+// over contiguous 2^c-element runs, and the exchange between the two kernel layouts is
+// planned as for any tile (shuffle / smem with the optimal swizzle).  The logical
+// column of a loaded src vector s is A(s).  Returns false when no tile of <= 64 KiB
+// exists (the generic kernel then runs).
+static bool build_linear_tile(ConvPlan& P, const ll_plan_opts* opts) {
+  const Layout &A = P.A, &B = P.B;
+  const int w = P.w;
+  const int nd = B.d_in();
+  if (A.d_in() != nd || !A.injective() || !B.injective() || nd > 40) return false;
+  Echelon eq;   // Q's columns, to invert Q
+  for (int k = 0; k < nd; ++k)
+    if (!eq.insert(P.Q[k], u64(1) << k)) return false;
+  auto qinv = [&](u64 x) { u64 c = 0; eq.reduce(x, &c); return c; };
+  auto alog = [&](u64 s) { u64 x = 0; for (int k = 0; k < nd; ++k) if ((s >> k) & 1) x ^= A.cols[k]; return x; };
+  const int maxvec = default_int(opts, &ll_plan_opts::max_vec_bytes, 16);
+  const int v = std::max(0, ilog2(u64(std::max(1, maxvec / w))));
+  if (v + 5 > nd) return false;
+  const int max_bits = ilog2(u64(65536 / w));
+  std::vector<char> inD(nd, 0);
+  int cnt = 0;
+  bool ok = false;
+  for (int c = v + 5; c >= v + 3 && !ok; --c) {
+    std::fill(inD.begin(), inD.end(), 0);
+    for (int k = 0; k < c; ++k) {
+      inD[k] = 1;
+      const u64 y = qinv(u64(1) << k);   // the dst vector whose image is src bit k
+      for (int d = 0; d < nd; ++d) if ((y >> d) & 1) inD[d] = 1;
+    }
+    cnt = int(std::count(inD.begin(), inD.end(), 1));
+    ok = cnt <= max_bits;
+  }
+  if (!ok) return false;
+  const int target = std::max(v + 5, ilog2(u64(std::max(1, default_int(opts, &ll_plan_opts::tile_bytes, 16384) / w))));
+  for (int k = 0; k < nd && cnt < target; ++k) if (!inD[k]) { inD[k] = 1; ++cnt; }
+  TilePlan& T = P.tile;
+  T = TilePlan();
+  T.w = w;
+  T.n = cnt;
+  int R = std::max(v, ilog2(u64(std::max(1, default_int(opts, &ll_plan_opts::thread_bytes, 256) / w))));
+  T.Wb = std::min(5, std::max(0, T.n - 5 - R));
+  T.R = T.n - 5 - T.Wb;
+  if (T.R < v) return false;
+  T.vld = T.vst = v;
+  // store side: the 16-byte vector, then 5 lanes over the next dst bits (512 contiguous
+  // bytes per warp instruction), then the rest of D: registers low, warps high
+  std::vector<int> rest;
+  for (int k = v + 5; k < nd; ++k) if (inD[k]) rest.push_back(k);
+  T.st_bit.assign(T.n, -1);
+  for (int b = 0; b < v; ++b) T.st_bit[b] = b;
+  for (int t = 0; t < 5; ++t) T.st_bit[T.R + t] = v + t;
+  size_t ri = 0;
+  for (int b = v; b < T.R; ++b) T.st_bit[b] = rest[ri++];
+  for (int t = 0; t < T.Wb; ++t) T.st_bit[T.R + 5 + t] = rest[ri++];
+  // load side: the src vector and lanes over the low src bits (when in the tile's image),
+  // then for every other kernel bit the src vector of the same logical element as the
+  // store side (common vectors keep the exchange cheap), else any completing vector
+  Echelon es;
+  T.ld_xcol.assign(T.n, 0);
+  std::vector<char> done(T.n, 0);
+  u64 dspan = 0;
+  for (int k = 0; k < nd; ++k) if (inD[k]) dspan |= u64(1) << k;
+  auto in_image = [&](u64 s) { return (qinv(s) & ~dspan) == 0; };
+  for (int b = 0; b < v; ++b) { T.ld_xcol[b] = u64(1) << b; es.insert(T.ld_xcol[b]); done[b] = 1; }
+  for (int t = 0; t < 5; ++t) {
+    const u64 s = u64(1) << (v + t);
+    if (in_image(s) && es.insert(s)) { T.ld_xcol[T.R + t] = s; done[T.R + t] = 1; }
+  }
+  std::vector<u64> pool;
+  for (int k = 0; k < nd; ++k) if (inD[k]) pool.push_back(P.Q[k]);
+  std::vector<int> order;
+  for (int b = v; b < T.R; ++b) order.push_back(b);
+  for (int t = 0; t < 5; ++t) order.push_back(T.R + t);
+  for (int t = 0; t < T.Wb; ++t) order.push_back(T.R + 5 + t);
+  for (int b : order) {
+    if (done[b]) continue;
+    u64 s = P.Q[T.st_bit[b]];
+    if (!es.insert(s)) {
+      s = 0;
+      for (u64 q : pool) if (es.insert(q)) { s = q; break; }
+      if (!s) return false;
+    }
+    T.ld_xcol[b] = s;
+    done[b] = 1;
+  }
+  if (es.rank != T.n) return false;
+  T.ld_bit = T.st_bit;   // (unused for the load side: ld_xcol)
+  for (int k = 0; k < nd; ++k)
+    if (!inD[k]) {
+      T.grid_dst_bit.push_back(k);
+      T.grid_src_bit.push_back(k);
+      T.grid_src_xcol.push_back(P.Q[k]);
+    }
+  T.lcol_ld.resize(T.n);
+  T.lcol_st.resize(T.n);
+  for (int b = 0; b < T.n; ++b) { T.lcol_ld[b] = alog(T.ld_xcol[b]); T.lcol_st[b] = B.cols[T.st_bit[b]]; }
+  T.sigma = SIGMA_COALESCED;
+  plan_exchange(P, opts);
+  P.exec = EXEC_TILE;
+  return true;
 }
 
 std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, const ll_plan_opts* opts,
@@ -916,6 +1044,14 @@ std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, 
       }
     }
   }
+  if (!generic && lev <= 3) {
+    try {
+      if (build_linear_tile(*P, opts)) return P;
+    } catch (const Error& e) {
+      if (opts && opts->force_class >= 0) throw;
+    }
+  }
+  P->tile = TilePlan();
   P->exec = EXEC_GENERIC;
   return P;
 }

@@ -529,6 +529,35 @@ def _scatter(T, off):
     return out
 
 
+@pytest.mark.parametrize("w", [1, 2, 4, 8])
+def test_linear_tiles_random_memory_layouts_gpu(w):
+    """General invertible pull maps (random Def 4.14 memory layouts, R2, whose Q
+    scatters the low bits; and a transpose into a Def 4.11 swizzle): planned as linear
+    CTA tiles (XOR-addressed src vectors, coalesced runs on both sides, smem / shuffle
+    exchange), never the generic kernel; bit-exact against the oracle."""
+    import torch
+    rng = np.random.default_rng(300 + w)
+    cases = []
+    for d in (14, 17, 20):
+        cases.append(([("offset", d)], [("x", d)], gen.random_memory_cols(rng, d), gen.random_memory_cols(rng, d)))
+    m = n = 9
+    S = ll.ll_layout_mma_swizzle(m, n, 1, 1, 8)             # Def 4.11, vec 1
+    tcols = [(1 << (k + n)) if k < m else (1 << (k - m)) for k in range(m + n)]   # column-major
+    cases.append(([("offset", m + n)], [tuple(x) for x in S.out_dims], tcols, S.cols()))
+    for in_dims, out, ca, cb in cases:
+        d = in_dims[0][1]
+        OA, OB = O.layout_from_cols(in_dims, out, ca), O.layout_from_cols(in_dims, out, cb)
+        A = ll.Layout(in_dims, out, {"offset": [O.logical_coords(out, c) for c in ca]})
+        B = ll.Layout(in_dims, out, {"offset": [O.logical_coords(out, c) for c in cb]})
+        plan = ll.ll_plan_convert(A, B, w)
+        assert plan.describe()["exec"] == "tile", plan.describe()["exec"]
+        src = gen.random_bits(rng, 1 << d, w)
+        d_dst = empty_device(1 << d, w)
+        ll.ll_convert(to_device(src), d_dst, plan)
+        torch.cuda.synchronize()
+        assert np.array_equal(from_device(d_dst, w), O.convert(OA, OB, src)), d
+
+
 @pytest.mark.gpu
 def test_e1_exhaustive_generic_gpu():
     """E1 on the GPU, exhaustive: all 8! = 40320 bijective relabelings B
