@@ -588,7 +588,9 @@ static void plan_smem(TilePlan& T, int maxvec, int smem_instr) {
   T.sw_bank.clear();
   for (u64 c : space) if (es.insert(c)) T.sw_bank.push_back(c);
   if (int(T.sw_vec.size() + T.sw_bank.size() + T.sw_seg.size()) != n)
-    fail(LL_ERR_UNSUPPORTED, "swizzle: basis incomplete (internal)");
+    fail(LL_ERR_UNSUPPORTED, "swizzle: basis incomplete (internal): |Vec| " + std::to_string(T.sw_vec.size()) +
+                                 " |Bank| " + std::to_string(T.sw_bank.size()) + " |Seg| " + std::to_string(T.sw_seg.size()) +
+                                 " n " + std::to_string(n));
   // M: offset bit -> logical (Vec, Bank, Seg); invert to get smem offsets.
   std::vector<u64> M = T.sw_vec;
   M.insert(M.end(), T.sw_bank.begin(), T.sw_bank.end());
@@ -785,10 +787,12 @@ static bool build_linear_tile(ConvPlan& P, const ll_plan_opts* opts) {
   std::vector<char> inD(nd, 0);
   int cnt = 0;
   bool ok = false;
-  for (int c = v + 5; c >= v + 3 && !ok; --c) {
+  // c = v + 1 still fills whole 32-byte sectors on the load side (two 16-byte lane vectors
+  // per sector), so DRAM traffic stays algorithmic; longer runs cut L2 requests
+  for (int c = v + 5; c >= v + 1 && !ok; --c) {
     std::fill(inD.begin(), inD.end(), 0);
+    for (int k = 0; k < v + 5; ++k) inD[k] = 1;   // the store side's vector and lanes
     for (int k = 0; k < c; ++k) {
-      inD[k] = 1;
       const u64 y = qinv(u64(1) << k);   // the dst vector whose image is src bit k
       for (int d = 0; d < nd; ++d) if ((y >> d) & 1) inD[d] = 1;
     }
