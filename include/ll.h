@@ -114,6 +114,7 @@ typedef struct {
                          * ldmatrix where M^{-1}∘L is divisible by their tile and that
                          * widens the swizzle's vector; 1 = vectorised ld/st.shared only;
                          * 2 = prefer stmatrix / ldmatrix wherever their tile divides   */
+  int reduce_op;        /* ll_plan_reduce: 0 = sum (default), 1 = max, 2 = min (fp32)   */
 } ll_plan_opts;
 
 /* Fill *opts with defaults (force_class = -1, max_vec_bytes = 16, ...). */
@@ -293,11 +294,12 @@ ll_status ll_gather(const void* src, const int32_t* idx, void* dst, const ll_pla
                     void* stream);
 
 /* ---------------------------------------------------------------- reduce --
- * ll_plan_reduce (row a12; Table 4).  Sum (fp32) along
- * logical dim `axis` over the non-block axis bits of L (within each CTA tile):
- * an in-register tree over Reg axis bits, shfl.bfly over Lane axis bits and smem
- * over Warp axis bits, in that fixed order (reg, lane, warp ascending);
- * broadcast (zero-column) bits are skipped, each output is written once. */
+ * ll_plan_reduce (row a12; Table 4).  Sum (fp32; or max / min
+ * with opts->reduce_op = 1 / 2) along logical dim `axis` over the non-block axis
+ * bits of L (within each CTA tile): an in-register tree over Reg axis bits,
+ * shfl.bfly over Lane axis bits and smem over Warp axis bits, in that fixed order
+ * (reg, lane, warp ascending); broadcast (zero-column) bits are skipped, each
+ * output is written once.  LL_ERR_INVALID_ARG for another reduce_op. */
 ll_status ll_plan_reduce(const ll_layout* L, int axis, const ll_plan_opts* opts, ll_plan** plan);
 /* Number of output elements. */
 ll_status ll_plan_reduce_out_elems(const ll_plan* plan, size_t* n);

@@ -889,10 +889,12 @@ def gather(L: Layout, axis: int, src: np.ndarray, idx: np.ndarray) -> np.ndarray
 # O11  Reduction (sum) with broadcast de-duplication (Table 4)
 # --------------------------------------------------------------------------------------
 
-def reduce_ref_fp64(L: Layout, axis: int, src: np.ndarray) -> np.ndarray:
-    """out[y] = Σ over logical x whose non-(in-tile)-axis part is y of T[x], in fp64.
+def reduce_ref_fp64(L: Layout, axis: int, src: np.ndarray, op: str = "sum") -> np.ndarray:
+    """out[y] = Σ (op = "sum"; or max / min) over logical x whose non-(in-tile)-axis part
+    is y of T[x], in fp64 (max / min are exact: the result is one of the fp32 inputs).
     The in-tile axis bits are the non-block axis bits of L; the output is the logical
-    tensor with the axis replaced by its block part (row-major)."""
+    tensor with the axis replaced by its block part (row-major).  Table 4
+    benchmarks `tl.sum`-style reductions; max and min are the other common ones."""
     shape = [1 << b for _, b in L.out_dims]
     x_of_h = image_table(L).astype(np.int64)
     T = np.empty(int(np.prod(shape)), dtype=np.float64)
@@ -905,7 +907,7 @@ def reduce_ref_fp64(L: Layout, axis: int, src: np.ndarray) -> np.ndarray:
     new_shape = shape.copy()
     new_shape[axis] = shape[axis] // K
     T = T.reshape(shape[:axis] + [shape[axis] // K, K] + shape[axis + 1:])
-    return T.sum(axis=axis + 1).reshape(-1)
+    return {"sum": T.sum, "max": T.max, "min": T.min}[op](axis=axis + 1).reshape(-1)
 
 
 def reduce_fixed_order_fp32(L: Layout, axis: int, src: np.ndarray) -> np.ndarray:

@@ -57,7 +57,7 @@ class _Dim(C.Structure):
 class _Opts(C.Structure):
     _fields_ = [("force_class", C.c_int), ("max_vec_bytes", C.c_int), ("sigma", C.c_int),
                 ("tile_bytes", C.c_int), ("thread_bytes", C.c_int), ("generic", C.c_int),
-                ("comm", C.c_void_p), ("exchange", C.c_int), ("smem_instr", C.c_int)]
+                ("comm", C.c_void_p), ("exchange", C.c_int), ("smem_instr", C.c_int), ("reduce_op", C.c_int)]
 
 
 _P = C.c_void_p
@@ -145,12 +145,14 @@ EXCHANGES = ("auto", "collective", "peer")
 # ll_plan_opts.smem_instr: auto (Thm 5.1 selection), vectorised ld/st.shared only, or
 # prefer stmatrix / ldmatrix wherever their tile divides
 SMEM_INSTRS = ["auto", "vec", "matrix"]
+# ll_plan_opts.reduce_op (ll_plan_reduce)
+REDUCE_OPS = ["sum", "max", "min"]
 PEER_FLAG_BYTES = 512
 IPC_HANDLE_BYTES = 72
 
 
 def _opts(force_class=None, max_vec_bytes=16, sigma=0, tile_bytes=0, thread_bytes=0, generic=False, comm=None,
-          exchange="auto", smem_instr="auto"):
+          exchange="auto", smem_instr="auto", reduce_op="sum"):
     o = _Opts()
     _lib.ll_plan_opts_default(C.byref(o))
     if force_class is not None:
@@ -163,6 +165,7 @@ def _opts(force_class=None, max_vec_bytes=16, sigma=0, tile_bytes=0, thread_byte
     o.comm = comm.handle if comm is not None else None
     o.exchange = EXCHANGES.index(exchange) if isinstance(exchange, str) else int(exchange)
     o.smem_instr = SMEM_INSTRS.index(smem_instr) if isinstance(smem_instr, str) else int(smem_instr)
+    o.reduce_op = REDUCE_OPS.index(reduce_op) if isinstance(reduce_op, str) else int(reduce_op)
     return o
 
 

@@ -513,7 +513,8 @@ ll_status ll_plan_describe(const ll_plan* p, char* json, size_t cap) {
   } else {
     const ReducePlan& Rp = *p->reduce;
     std::ostringstream o;
-    o << "{\"kind\":\"reduce\",\"R\":" << Rp.R << ",\"warp_bits\":" << Rp.Wb << ",\"tree_levels\":" << Rp.red_reg.size()
+    static const char* opn[] = {"sum", "max", "min"};
+    o << "{\"kind\":\"reduce\",\"op\":\"" << opn[Rp.op] << "\",\"R\":" << Rp.R << ",\"warp_bits\":" << Rp.Wb << ",\"tree_levels\":" << Rp.red_reg.size()
       << ",\"bfly_stages\":" << Rp.red_lane.size() << ",\"warp_stages\":" << Rp.red_warp.size()
       << ",\"dup_bits\":" << Rp.dup_bits.size() << ",\"out_elems\":" << Rp.out_elems
       << ",\"tma\":" << (Rp.tma ? "true" : "false") << ",\"stages\":" << Rp.stages << ",\"sigma\":\"" << (Rp.sigma ? "faithful" : "coalesced") << "\""

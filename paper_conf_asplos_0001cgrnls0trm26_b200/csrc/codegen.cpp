@@ -214,7 +214,7 @@ std::string codegen_reduce(const ReducePlan& Rp) {
   std::ostringstream o;
   o << "struct P {\n";
   const int R = Rp.R, n = int(Rp.hw_bit.size());
-  o << icon("W", 4) << icon("R", R) << icon("WB", Rp.Wb) << icon("VLD", Rp.v);
+  o << icon("W", 4) << icon("R", R) << icon("WB", Rp.Wb) << icon("VLD", Rp.v) << icon("OP", Rp.op);
   o << "  static constexpr bool LD_L1 = " << (Rp.sigma == SIGMA_FAITHFUL ? "true" : "false") << ";\n";
   o << "  static constexpr bool TMA = " << (Rp.tma ? "true" : "false") << ";\n";
   o << "  static constexpr unsigned WRED_BYTES = " << Rp.wred_bytes << "u;\n";

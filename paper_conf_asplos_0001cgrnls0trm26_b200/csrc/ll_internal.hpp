@@ -271,6 +271,7 @@ struct ReducePlan {
   int axis = 0;
   int exec = EXEC_TILE;
   int sigma = SIGMA_COALESCED;
+  int op = 0;                     // 0 sum, 1 max, 2 min (ll_plan_opts.reduce_op)
   int R = 0, Wb = 0, v = 0;
   std::vector<int> hw_bit;        // kernel bit -> packed bit of L (σ)
   std::vector<int> grid_bit;      // CTA index bit -> packed bit (non-duplicate block bits)

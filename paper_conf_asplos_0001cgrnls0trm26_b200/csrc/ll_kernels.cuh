@@ -953,6 +953,14 @@ __device__ __forceinline__ void ll_gather_body(const u8* __restrict__ src, const
 // in-register tree over the Reg axis bits, shfl.bfly over the Lane axis
 // bits, smem over the Warp axis bits — in the layout's bit order (reg, lane, warp
 // ascending); zero-column (broadcast) bits are skipped and de-duplicated at store.
+// The reduction operator (ll_plan_opts.reduce_op): fp32 round-to-nearest add (no FMA
+// contraction), max or min (exact: the result is one of the operands).
+template <int OP> __device__ __forceinline__ float red_op(float a, float b) {
+  if constexpr (OP == 1) return fmaxf(a, b);
+  else if constexpr (OP == 2) return fminf(a, b);
+  else return __fadd_rn(a, b);
+}
+
 template <class P>
 __device__ __forceinline__ void ll_reduce_tile(u32 (&r)[1 << P::R], float* sm, u32 lane, u32 warp, u64 oblk,
                                                u64 othr, bool do_store, float* __restrict__ dst) {
@@ -963,7 +971,7 @@ __device__ __forceinline__ void ll_reduce_tile(u32 (&r)[1 << P::R], float* sm, u
       constexpr int E = decltype(e)::value;
       if constexpr (((E >> B) & 1) == 0 && (E & P::template done_mask<decltype(i)::value>()) == 0 &&
                     (E & P::DUP_REG_MASK) == 0) {
-        r[E] = __float_as_uint(__fadd_rn(__uint_as_float(r[E]), __uint_as_float(r[E | (1 << B)])));
+        r[E] = __float_as_uint(red_op<P::OP>(__uint_as_float(r[E]), __uint_as_float(r[E | (1 << B)])));
       }
     });
   });
@@ -974,7 +982,7 @@ __device__ __forceinline__ void ll_reduce_tile(u32 (&r)[1 << P::R], float* sm, u
       constexpr int E = decltype(e)::value;
       if constexpr ((E & (P::RED_REG_MASK | P::DUP_REG_MASK)) == 0) {
         const float x = __uint_as_float(r[E]);
-        r[E] = __float_as_uint(__fadd_rn(x, __shfl_xor_sync(0xffffffffu, x, 1 << L)));
+        r[E] = __float_as_uint(red_op<P::OP>(x, __shfl_xor_sync(0xffffffffu, x, 1 << L)));
       }
     });
   });
@@ -1005,7 +1013,7 @@ __device__ __forceinline__ void ll_reduce_tile(u32 (&r)[1 << P::R], float* sm, u
             static_for<(1 << P::NRED_WARP)>([&](auto m) {
               constexpr int M = decltype(m)::value;
               if constexpr (((M >> Q) & 1) == 0 && (M & ((1 << Q) - 1)) == 0)
-                v[M] = __fadd_rn(v[M], v[M | (1 << Q)]);
+                v[M] = red_op<P::OP>(v[M], v[M | (1 << Q)]);
             });
           });
           r[E] = __float_as_uint(v[0]);

@@ -1300,6 +1300,8 @@ std::unique_ptr<ReducePlan> plan_reduce(const Layout& L, int axis, const ll_plan
   if (L.in.size() < 1 || L.in[0].name != "reg") fail(LL_ERR_UNSUPPORTED, "reduce: dims must be reg, lane, warp[, block]");
   auto Rp = std::make_unique<ReducePlan>();
   Rp->L = L; Rp->axis = axis;
+  Rp->op = opts ? opts->reduce_op : 0;
+  if (Rp->op < 0 || Rp->op > 2) fail(LL_ERR_INVALID_ARG, "reduce_op must be 0 (sum), 1 (max) or 2 (min)");
   const int sh = L.out_shift(axis), ab = L.out[axis].bits;
   const u64 amask = ((u64(1) << ab) - 1) << sh;
   const int R = L.in_bits("reg");

@@ -270,6 +270,26 @@ def test_reduce_tolerance_and_fixed_order(family, sigma):
     assert np.array_equal(got.view(np.uint32), rep.view(np.uint32))
 
 
+@pytest.mark.parametrize("family", ["mma", "blocked"])
+@pytest.mark.parametrize("sigma", ["coalesced", "faithful"])
+@pytest.mark.parametrize("op", ["max", "min"])
+def test_reduce_max_min_bitexact(family, sigma, op):
+    """max / min reductions (ll_plan_opts.reduce_op) along axis 1 inside [128,128]
+    tiles: exact, so bit-equal to the oracle's fp64 reference."""
+    import torch
+    rng = np.random.default_rng(1006)
+    L, OL = both(W.c4("reduce", family, n_i=9, n_j=9))
+    n = 1 << OL.d_in
+    T = (rng.random(n, dtype=np.float32) - 0.5).astype(np.float32)
+    src = O.pack(OL, T)
+    plan = ll.ll_plan_reduce(L, 1, sigma=sigma, reduce_op=op)
+    assert plan.describe()["op"] == op
+    out = torch.empty(plan.out_elems(), dtype=torch.float32, device="cuda")
+    ll.ll_reduce(torch.from_numpy(src).cuda(), out, plan)
+    ref = O.reduce_ref_fp64(OL, 1, src, op).astype(np.float32)
+    assert np.array_equal(out.cpu().numpy().view(np.uint32), ref.view(np.uint32))
+
+
 def test_reduce_broadcast_dedup_gpu():
     """a layout with zero columns (duplicated lanes and registers) reduces each
     logical element once; one write per output."""

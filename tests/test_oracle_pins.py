@@ -755,3 +755,17 @@ def test_scan_fp32_recurrence_within_bound():
     got = O.scan_bitdoubling_fp32(OL, 1, src).astype(np.float64)
     ref = O.scan_ref_fp64(OL, 1, src)
     assert np.all(np.abs(got - ref) <= 7 * 2.0 ** -24 * np.abs(ref) + 1e-30)
+
+
+@pytest.mark.parametrize("family", ["mma", "blocked"])
+def test_reduce_max_min_closed_form(family):
+    """max / min reductions (O11 with another op): on T[x] = x (the logical flat index,
+    exact in fp64) the max over a [.., K] in-tile row is its last index and the min its
+    first — a closed form independent of any layout arithmetic."""
+    L = L_of(W.c4("reduce", family, n_i=8, n_j=8))     # [256, 256] in [128, 128] tiles
+    n = 1 << L.d_in
+    T = np.arange(n, dtype=np.float64)
+    src = O.pack(L, T)
+    rows = np.arange(256)[:, None] * 256 + np.arange(2)[None, :] * 128
+    assert np.array_equal(O.reduce_ref_fp64(L, 1, src, "max"), (rows + 127).reshape(-1))
+    assert np.array_equal(O.reduce_ref_fp64(L, 1, src, "min"), rows.reshape(-1))
