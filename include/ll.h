@@ -316,7 +316,8 @@ ll_status ll_reduce(const float* src, float* dst, const ll_plan* plan, void* str
  * the lower half of its aligned 2^(t+1)-block.  L: a distributed layout (duplicated
  * positions, zero columns, each get the same value).  Steps over register bits are
  * register adds, over lane bits warp shuffles, over warp bits a shared-memory
- * exchange (LL_ERR_UNSUPPORTED when it exceeds shared memory). */
+ * exchange (LL_ERR_UNSUPPORTED when it exceeds shared memory).  opts->reduce_op = 1 / 2
+ * gives the running max / min instead of the sum (same steps, exact). */
 ll_status ll_plan_scan(const ll_layout* L, int axis, const ll_plan_opts* opts, ll_plan** plan);
 /* src, dst: fp32 packed in L (same positions); must not overlap partially. */
 ll_status ll_scan(const float* src, float* dst, const ll_plan* plan, void* stream);

@@ -979,11 +979,13 @@ def _scan_setup(L: Layout, axis: int, src: np.ndarray, dtype):
     return T, kbits, x_of_h, shape
 
 
-def scan_ref_fp64(L: Layout, axis: int, src: np.ndarray) -> np.ndarray:
-    """out[x] = sum of T[x with axis coordinate a'] over the a' of x's tile with a' <= a(x)
-    (inclusive), in fp64, returned packed in L like the input (library cumsum)."""
+def scan_ref_fp64(L: Layout, axis: int, src: np.ndarray, op: str = "sum") -> np.ndarray:
+    """out[x] = sum (op = "sum"; or max / min) of T[x with axis coordinate a'] over the a'
+    of x's tile with a' <= a(x) (inclusive), in fp64, returned packed in L like the input
+    (library cumsum / running maximum / running minimum; max and min are exact)."""
     T, kbits, x_of_h, shape = _scan_setup(L, axis, src, np.float64)
-    out = np.cumsum(T, axis=axis + 1).reshape(-1)
+    acc = {"sum": np.cumsum, "max": np.maximum.accumulate, "min": np.minimum.accumulate}[op]
+    out = acc(T, axis=axis + 1).reshape(-1)
     return out[x_of_h]
 
 

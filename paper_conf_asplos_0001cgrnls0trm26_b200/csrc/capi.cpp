@@ -501,7 +501,8 @@ ll_status ll_plan_describe(const ll_plan* p, char* json, size_t cap) {
   } else if (p->kind == 3) {
     const ScanPlan& S = *p->scan;
     std::ostringstream o;
-    o << "{\"kind\":\"scan\",\"sigma\":\"" << (S.sigma ? "faithful" : "coalesced") << "\",\"R\":" << S.R
+    static const char* sopn[] = {"sum", "max", "min"};
+    o << "{\"kind\":\"scan\",\"op\":\"" << sopn[S.op] << "\",\"sigma\":\"" << (S.sigma ? "faithful" : "coalesced") << "\",\"R\":" << S.R
       << ",\"warp_bits\":" << S.Wb << ",\"K_bits\":" << S.K_bits << ",\"steps\":" << S.K_bits
       << ",\"axis_hw\":" << "[";
     for (size_t t = 0; t < S.axis_hw.size(); ++t) o << (t ? "," : "") << S.axis_hw[t];

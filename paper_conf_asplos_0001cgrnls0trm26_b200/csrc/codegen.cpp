@@ -192,7 +192,8 @@ std::string codegen_gather(const GatherPlan& G) {
 std::string codegen_scan(const ScanPlan& S) {
   std::ostringstream o;
   o << "struct P {\n";
-  o << icon("W", 4) << icon("R", S.R) << icon("WB", S.Wb) << icon("VLD", S.v) << icon("NW", 1 << S.R);
+  o << icon("W", 4) << icon("R", S.R) << icon("WB", S.Wb) << icon("VLD", S.v) << icon("NW", 1 << S.R)
+    << icon("OP", S.op);
   o << "  static constexpr bool LD_L1 = " << (S.sigma == SIGMA_FAITHFUL ? "true" : "false") << ";\n";
   o << icon("ST_HINT", st_hint());
   std::vector<u64> ldc;

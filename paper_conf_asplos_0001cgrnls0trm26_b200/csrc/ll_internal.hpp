@@ -299,6 +299,7 @@ struct ScanPlan {
   Layout L;
   int axis = 0;
   int sigma = SIGMA_COALESCED;
+  int op = 0;                  // 0 sum, 1 max, 2 min (ll_plan_opts.reduce_op)
   int R = 0, Wb = 0, v = 0;
   int K_bits = 0;
   std::vector<int> hw_bit;     // kernel bit -> packed bit (src and dst)

@@ -1177,7 +1177,7 @@ __device__ __forceinline__ void ll_scan_steps(u32 (&r)[P::NW], u32 lane, float* 
           constexpr int E = decltype(e)::value;
           if constexpr (!St::HREG || ((E >> HB) & 1)) {
             constexpr int E2 = (St::HREG ? (E & ~(1 << HB)) : E) | int(LR);
-            if (upper) r[E] = __float_as_uint(__fadd_rn(__uint_as_float(r[E]), sm[E2 * NT + pt]));
+            if (upper) r[E] = __float_as_uint(red_op<P::OP>(__uint_as_float(r[E]), sm[E2 * NT + pt]));
           }
         });
         __syncthreads();
@@ -1187,7 +1187,7 @@ __device__ __forceinline__ void ll_scan_steps(u32 (&r)[P::NW], u32 lane, float* 
           constexpr int E = decltype(e)::value;
           if constexpr ((E >> HB) & 1) {
             constexpr int E2 = (E & ~(1 << HB)) | int(LR);
-            r[E] = __float_as_uint(__fadd_rn(__uint_as_float(r[E]), __uint_as_float(r[E2])));
+            r[E] = __float_as_uint(red_op<P::OP>(__uint_as_float(r[E]), __uint_as_float(r[E2])));
           }
         });
       } else if constexpr (St::HREG) {
@@ -1198,7 +1198,7 @@ __device__ __forceinline__ void ll_scan_steps(u32 (&r)[P::NW], u32 lane, float* 
           if constexpr ((E >> HB) & 1) {
             constexpr int E2 = (E & ~(1 << HB)) | int(LR);
             const float x = __shfl_sync(0xffffffffu, __uint_as_float(r[E2]), sl);
-            r[E] = __float_as_uint(__fadd_rn(__uint_as_float(r[E]), x));
+            r[E] = __float_as_uint(red_op<P::OP>(__uint_as_float(r[E]), x));
           }
         });
       } else {
@@ -1210,7 +1210,7 @@ __device__ __forceinline__ void ll_scan_steps(u32 (&r)[P::NW], u32 lane, float* 
           constexpr int E = decltype(e)::value;
           constexpr int E2 = E | int(LR);
           const float x = __shfl_sync(0xffffffffu, __uint_as_float(r[E2]), sl);
-          if (upper) r[E] = __float_as_uint(__fadd_rn(__uint_as_float(r[E]), x));
+          if (upper) r[E] = __float_as_uint(red_op<P::OP>(__uint_as_float(r[E]), x));
         });
       }
     });

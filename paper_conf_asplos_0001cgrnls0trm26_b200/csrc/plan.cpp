@@ -1398,6 +1398,8 @@ std::unique_ptr<ScanPlan> plan_scan(const Layout& L, int axis, const ll_plan_opt
   if (L.in.size() < 1 || L.in[0].name != "reg") fail(LL_ERR_UNSUPPORTED, "scan: dims must be reg, lane, warp[, block]");
   auto S = std::make_unique<ScanPlan>();
   S->L = L; S->axis = axis;
+  S->op = opts ? opts->reduce_op : 0;
+  if (S->op < 0 || S->op > 2) fail(LL_ERR_INVALID_ARG, "reduce_op must be 0 (sum), 1 (max) or 2 (min)");
   const int sh = L.out_shift(axis), ab = L.out[axis].bits;
   const u64 amask = ((u64(1) << ab) - 1) << sh;
   const int R = L.in_bits("reg");

@@ -645,6 +645,30 @@ def test_scan_bitexact(family, sigma):
     assert np.all(np.abs(got - ref) <= 7 * 2.0 ** -24 * np.abs(ref) + 1e-30)
 
 
+@pytest.mark.parametrize("family", ["mma", "blocked"])
+@pytest.mark.parametrize("op", ["max", "min"])
+def test_scan_max_min_bitexact(family, op):
+    """Running max / min (ll_plan_opts.reduce_op) along the axis inside [128,128] tiles,
+    plus the warp-crossing (smem) steps of a layout with axis bits on the warps: exact,
+    so bit-equal to the oracle's fp64 running max / min."""
+    import torch
+    rng = np.random.default_rng(1011)
+    warp_axis = {"out": [("b", 3), ("i", 5), ("j", 7)],
+                 "in": [("reg", ["j0", "j1", "j2"]), ("lane", ["i0", "i1", "i2", "i3", "i4"]),
+                        ("warp", ["j3", "j4", "j5", "j6"]), ("block", ["b0", "b1", "b2"])]}
+    for spec, axis in ((W.c4("reduce", family, n_i=9, n_j=9), 1), (warp_axis, 2)):
+        L, OL = both(spec)
+        T = (rng.random(1 << OL.d_out, dtype=np.float32) - 0.5).astype(np.float32)
+        src = O.pack(OL, T)
+        for sigma in ("coalesced", "faithful"):
+            plan = ll.ll_plan_scan(L, axis, sigma=sigma, reduce_op=op)
+            assert plan.describe()["op"] == op
+            out = torch.empty(src.size, dtype=torch.float32, device="cuda")
+            ll.ll_scan(torch.from_numpy(src).cuda(), out, plan)
+            ref = O.scan_ref_fp64(OL, axis, src, op).astype(np.float32)
+            assert np.array_equal(out.cpu().numpy().view(np.uint32), ref.view(np.uint32)), (sigma, axis)
+
+
 @pytest.mark.parametrize("family", ["blocked", "mma", "mma_input", "sliced_blocked", "sliced_mma",
                                     "sliced_mma_input", "custom"])
 def test_table4_scan_families(family):

@@ -769,3 +769,18 @@ def test_reduce_max_min_closed_form(family):
     rows = np.arange(256)[:, None] * 256 + np.arange(2)[None, :] * 128
     assert np.array_equal(O.reduce_ref_fp64(L, 1, src, "max"), (rows + 127).reshape(-1))
     assert np.array_equal(O.reduce_ref_fp64(L, 1, src, "min"), rows.reshape(-1))
+
+
+@pytest.mark.parametrize("family", ["mma", "blocked"])
+def test_scan_max_min_closed_form(family):
+    """Running max / min scans: on T[x] = -x (decreasing along every row) the running
+    max of a [.., K] in-tile row is its first element and the running min the element
+    itself; on T[x] = x the other way round."""
+    L = L_of(W.c4("reduce", family, n_i=8, n_j=8))     # [256, 256] in [128, 128] tiles
+    n = 1 << L.d_in
+    x = np.arange(n, dtype=np.float64)
+    first = (x // 128) * 128                            # first index of x's in-tile row
+    for T, mx, mn in ((-x, -first, -x), (x, x, first)):
+        src = O.pack(L, T)
+        assert np.array_equal(O.scan_ref_fp64(L, 1, src, "max"), O.pack(L, mx))
+        assert np.array_equal(O.scan_ref_fp64(L, 1, src, "min"), O.pack(L, mn))
