@@ -151,6 +151,7 @@ struct TilePlan {
   // F2 combination Q(dst bit) (swizzled memory layouts, Def 4.14; broadcast).  When
   // non-empty these replace 1 << ld_bit / 1 << grid_src_bit.
   std::vector<u64> ld_xcol, grid_src_xcol;
+  int ld_run = -1;      // linear tiles: low src bits loaded as contiguous runs (c)
   int sigma = SIGMA_COALESCED;
   int xchg = X_COPY;
   bool pipe = false;    // X_SMEM: next tile's loads issued before this tile's stores

@@ -853,6 +853,8 @@ static bool build_linear_tile(ConvPlan& P, const ll_plan_opts* opts) {
     done[b] = 1;
   }
   if (es.rank != T.n) return false;
+  T.ld_run = v;
+  while (T.ld_run < v + 5 && T.ld_xcol[T.R + (T.ld_run - v)] == (u64(1) << T.ld_run)) ++T.ld_run;
   T.ld_bit = T.st_bit;   // (unused for the load side: ld_xcol)
   for (int k = 0; k < nd; ++k)
     if (!inD[k]) {
@@ -1106,6 +1108,9 @@ std::string describe(const ConvPlan& P) {
       << ",\"ld_bit\":" << ivec_json(T.ld_bit) << ",\"st_bit\":" << ivec_json(T.st_bit)
       << ",\"L_ld\":" << vec_json(T.lcol_ld) << ",\"L_st\":" << vec_json(T.lcol_st)
       << ",\"grid_src_bit\":" << ivec_json(T.grid_src_bit) << ",\"grid_dst_bit\":" << ivec_json(T.grid_dst_bit);
+    if (!T.ld_xcol.empty())
+      o << ",\"ld_xcol\":" << vec_json(T.ld_xcol) << ",\"linear_tile\":" << (T.ld_run >= 0 ? "true" : "false")
+        << ",\"ld_run_bits\":" << (T.ld_run >= 0 ? T.ld_run : T.vld + 5);
     if (T.xchg == X_SHUFFLE)
       o << ",\"V\":" << vec_json(T.V) << ",\"I\":" << vec_json(T.I) << ",\"E\":" << vec_json(T.E)
         << ",\"F\":" << vec_json(T.F) << ",\"G\":" << vec_json(T.G) << ",\"R_basis\":" << vec_json(T.Rb)
