@@ -127,6 +127,8 @@ def matrix_tiles():
     for name, (sa, sb), opts in cases:
         for mode in ("auto", "vec"):
             conv_case(f"{name} smem_instr={mode}", sa, sb, 2, smem_instr=mode, **opts)
+    for mode in ("auto", "matrix"):
+        conv_case(f"N1 preshuffle smem_instr={mode}", *W.n1_preshuffle(14, 14), 2, smem_instr=mode)
 
 
 def invec_swizzles():
