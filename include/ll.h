@@ -334,6 +334,11 @@ ll_status ll_comm_get_unique_id(void* nccl_unique_id /* 128 bytes */);
  * back, and the exchange is a set of device memcpys.  For tests of the DEVICE
  * decomposition on one GPU. */
 ll_status ll_comm_create_loopback(int nranks, ll_comm** comm);
+/* Failure detection: LL_ERR_NCCL (with ncclGetErrorString's text in ll_last_error)
+ * when an NCCL communicator has recorded an asynchronous error
+ * (ncclCommGetAsyncError); LL_OK otherwise and for loopback / peer communicators,
+ * whose failures surface as CUDA errors.  ll_convert checks it after each exchange. */
+ll_status ll_comm_check(const ll_comm* comm);
 void ll_comm_destroy(ll_comm* comm);
 
 /* Peer-window communicator (§8(f) N4, LL_EXCHANGE_PEER).  Every rank owns a dst

@@ -93,6 +93,7 @@ _sig = {
     "ll_comm_create": [_P, C.c_int, C.c_int, _PP],
     "ll_comm_get_unique_id": [_P],
     "ll_comm_create_loopback": [C.c_int, _PP],
+    "ll_comm_check": [_P],
     "ll_plan_device_stages": [_P, _PP, _PP, C.POINTER(C.c_size_t), C.POINTER(C.c_int)],
     "ll_comm_create_peers": [C.c_int, C.c_int, _PP, _PP, C.c_size_t, _PP],
     "ll_plan_autotune": [_P, _P, C.c_int, C.POINTER(_Opts), _P, _P, _P, C.c_int, _PP],
@@ -452,6 +453,11 @@ class Comm:
 
     def __init__(self, handle, nranks):
         self.handle, self.nranks = handle, nranks
+
+    def check(self):
+        """ll_comm_check: raise LLError(NCCL) if the communicator recorded an
+        asynchronous NCCL error (failure detection)."""
+        _check(_lib.ll_comm_check(self.handle))
 
     @classmethod
     def loopback(cls, nranks: int) -> "Comm":

@@ -34,6 +34,7 @@ struct Nccl {
   int (*send)(const void*, size_t, int, int, void*, cudaStream_t) = nullptr;
   int (*recv)(void*, size_t, int, int, void*, cudaStream_t) = nullptr;
   const char* (*errstr)(int) = nullptr;
+  int (*asyncError)(void*, int*) = nullptr;
 };
 
 Nccl& nccl() {
@@ -55,6 +56,7 @@ Nccl& nccl() {
     n.send = reinterpret_cast<decltype(n.send)>(dlsym(n.h, "ncclSend"));
     n.recv = reinterpret_cast<decltype(n.recv)>(dlsym(n.h, "ncclRecv"));
     n.errstr = reinterpret_cast<decltype(n.errstr)>(dlsym(n.h, "ncclGetErrorString"));
+    n.asyncError = reinterpret_cast<decltype(n.asyncError)>(dlsym(n.h, "ncclCommGetAsyncError"));
   });
   if (!n.h || !n.send || !n.recv || !n.commInitRank) fail(LL_ERR_NCCL, "libnccl.so.2 not available");
   return n;
@@ -335,6 +337,10 @@ ll_status device_convert(const ConvPlan& Pc, const void* src, void* dst, void* w
       check_nccl(n.recv(recvbuf(0) + q * cb, cb, 0, q, comm->nccl, st), "ncclRecv");
     }
     check_nccl(n.groupEnd(), "ncclGroupEnd");
+    // an earlier asynchronous NCCL failure on this communicator surfaces here
+    int aerr = 0;
+    if (n.asyncError) check_nccl(n.asyncError(comm->nccl, &aerr), "ncclCommGetAsyncError");
+    check_nccl(aerr, "NCCL asynchronous error");
   }
   // 3. unpack
   if (P.unpack)
@@ -479,6 +485,22 @@ ll_status ll_comm_create_loopback(int nranks, ll_comm** out) {
   c->rank = -1;
   c->loopback = true;
   *out = c.release();
+  return LL_OK;
+}
+
+ll_status ll_comm_check(const ll_comm* c) {
+  try {
+    if (!c) ll::fail(LL_ERR_INVALID_ARG, "null communicator");
+    if (!c->nccl) return LL_OK;   // loopback / peer windows: errors surface as CUDA errors
+    ll::Nccl& n = ll::nccl();
+    if (!n.asyncError) ll::fail(LL_ERR_NCCL, "ncclCommGetAsyncError not available");
+    int aerr = 0;
+    ll::check_nccl(n.asyncError(c->nccl, &aerr), "ncclCommGetAsyncError");
+    ll::check_nccl(aerr, "NCCL asynchronous error");
+  } catch (const ll::Error& e) {
+    ll::set_last_error(e.what());
+    return e.st;
+  }
   return LL_OK;
 }
 

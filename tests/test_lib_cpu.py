@@ -711,3 +711,11 @@ def test_convert_host_refuses_xor_grids():
                                  p.handle, 1, streams)
     assert ll.STATUS[st] == "UNSUPPORTED"
     assert b"grid" in ll._lib.ll_last_error()
+
+
+def test_comm_check_loopback_ok_and_null_invalid():
+    """ll_comm_check (failure detection): loopback communicators have no NCCL state
+    (LL_OK); a null handle is an invalid argument."""
+    c = ll.Comm.loopback(4)
+    c.check()
+    assert ll.STATUS[ll._lib.ll_comm_check(None)] == "INVALID_ARG"
