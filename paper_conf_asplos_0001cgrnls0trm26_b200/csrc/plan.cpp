@@ -468,8 +468,13 @@ static void plan_smem(TilePlan& T, int maxvec, int smem_instr) {
   //     the order: one side matrix, the other vectorised; then both sides matrix.
   const int full = w <= 4 ? ilog2(u64(16 / w)) : 0;
   const int k = w <= 4 ? ilog2(u64(4 / w)) : 0;
+  // auto: the matrix tiles are tried when the common registers give less than 16 bytes
+  // — under faithful σ less than 8 (measured: its L1-allocating per-thread loads make
+  // STSM a net loss when the vectorised path already moves 8 bytes, config 2: 3237 vs
+  // 2822 GB/s; a gain from 4 bytes, config 3: 3276 -> 3342; profiles/r01_thm51_*)
+  const int want = T.sigma == SIGMA_FAITHFUL ? full - 1 : full;
   if (smem_instr != 1 && w <= 4 && maxvec >= 16 && R >= k &&
-      (int(T.sw_vec.size()) < full || smem_instr == 2)) {
+      (int(T.sw_vec.size()) < want || smem_instr == 2)) {
     struct Side { int kind; std::vector<int> word; std::vector<u64> row; };
     auto options = [&](const std::vector<u64>& lc) {
       std::vector<Side> out;

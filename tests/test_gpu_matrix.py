@@ -43,7 +43,7 @@ def test_matrix_cases_bitexact(case, nb):
 
 
 @pytest.mark.parametrize("cfg", ["c2", "c3", "c3b"])
-@pytest.mark.parametrize("smem_instr", ["auto", "vec"])
+@pytest.mark.parametrize("smem_instr", ["matrix", "vec"])
 def test_paper_configs_matrix_vs_vec_bitexact(cfg, smem_instr):
     """Config 2 / 3 under faithful σ (stmatrix for the accumulator / [1,8] side) and
     config 3b under coalesced σ (stmatrix widens the vector to 16 B), each against the
@@ -52,7 +52,7 @@ def test_paper_configs_matrix_vs_vec_bitexact(cfg, smem_instr):
     sigma = "coalesced" if cfg == "c3b" else "faithful"
     got, ref, d = _run(sa, sb, 2, 1002, sigma=sigma, force_class="SMEM", smem_instr=smem_instr)
     t = d["tile"]
-    assert ("stmatrix" in t["smem_store"]) == (smem_instr == "auto")
+    assert ("stmatrix" in t["smem_store"]) == (smem_instr == "matrix")
     assert np.array_equal(got, ref)
 
 

@@ -597,7 +597,12 @@ def test_matrix_tiles_on_paper_configs():
     swizzle vector from 8 to 16 bytes with stmatrix."""
     cases = [(W.c2(0), 2, "faithful", 16, 32), (W.c3(0), 2, "faithful", 32, 128), (W.c3b(0), 2, "coalesced", None, None)]
     for (sa, sb), w, sigma, n_mat, n_vec in cases:
-        d = _sim_check(sa, sb, w, 4, sigma=sigma, force_class="SMEM")
+        # the automatic choice takes stmatrix for config 3 (4-byte common vector) and 3b;
+        # config 2 (8-byte common vector under faithful σ) keeps the vectorised path
+        # by the measured default and gets the matrix tiles on request
+        auto = _sim_check(sa, sb, w, 4, sigma=sigma, force_class="SMEM")["tile"]
+        assert ("stmatrix" in auto["smem_store"]) == (n_mat != 16)
+        d = _sim_check(sa, sb, w, 4, sigma=sigma, force_class="SMEM", smem_instr="matrix")
         t = d["tile"]
         assert t["smem_store"] == "stmatrix.m8n8.x4.b16" and t["smem_load"] == "ld.shared.v4.b32", t
         assert (1 << len(t["Vec"])) * w == 16

@@ -26,13 +26,13 @@ conv = {"c2": (W.c2(16), 2, {}), "c2smem": (W.c2(16), 2, {"force_class": "SMEM"}
         "c1bsmem_small": (W.c1_batched(6), 4, {"force_class": "SMEM"}),
         "c3_small": (W.c3(3), 2, {}), "c2_small": (W.c2(3), 2, {}),
         "c3b_small": (W.c3b(3), 2, {}),
-        "c2fsmem_small": (W.c2(3), 2, {"sigma": "faithful", "force_class": "SMEM"}),
+        "c2fsmem_small": (W.c2(3), 2, {"sigma": "faithful", "force_class": "SMEM", "smem_instr": "matrix"}),
         "c3f_small": (W.c3(3), 2, {"sigma": "faithful"}),
         "c5T": (W.c5T(0, n=15), 2, {}), "n1": (W.n1_preshuffle(14, 14), 2, {}),
         "n2": (W.n2_tmem_epilogue(13), 4, {}),
         # Thm 5.1: stmatrix / ldmatrix vs vectorised ld/st.shared only
         "c3bvec": (W.c3b(14), 2, {"smem_instr": "vec"}),
-        "c2fsmem": (W.c2(16), 2, {"sigma": "faithful", "force_class": "SMEM"}),
+        "c2fsmem": (W.c2(16), 2, {"sigma": "faithful", "force_class": "SMEM", "smem_instr": "matrix"}),
         "c2fsmemvec": (W.c2(16), 2, {"sigma": "faithful", "force_class": "SMEM", "smem_instr": "vec"}),
         "c3f": (W.c3(14), 2, {"sigma": "faithful"}),
         "c3fvec": (W.c3(14), 2, {"sigma": "faithful", "smem_instr": "vec"})}

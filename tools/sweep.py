@@ -120,6 +120,7 @@ def matrix_tiles():
     """Thm 5.1 instruction selection: stmatrix / ldmatrix vs vectorised
     ld/st.shared only, same layouts, same bytes."""
     cases = [("c2 faithful smem", W.c2(16), dict(sigma="faithful", force_class="SMEM")),
+             ("c2 faithful smem (matrix)", W.c2(16), dict(sigma="faithful", force_class="SMEM", smem_instr="matrix")),
              ("c3 faithful", W.c3(14), dict(sigma="faithful")),
              ("c3 faithful smem", W.c3(14), dict(sigma="faithful", force_class="SMEM")),
              ("c3b", W.c3b(14), dict()),
