@@ -778,8 +778,9 @@ static void choose_cta_tile(const std::vector<int>& pi, int nloc, int c_bits,
 static bool build_linear_tile(ConvPlan& P, const ll_plan_opts* opts) {
   const Layout &A = P.A, &B = P.B;
   const int w = P.w;
-  const int nd = B.d_in();
-  if (A.d_in() != nd || !A.injective() || !B.injective() || nd > 40) return false;
+  const int nd = B.d_in() - dev_bits(B);   // local bits (the class is below DEVICE)
+  if (A.d_in() - dev_bits(A) != nd || int(P.Q.size()) < nd || !A.injective() || !B.injective() || nd > 40)
+    return false;
   Echelon eq;   // Q's columns, to invert Q
   for (int k = 0; k < nd; ++k)
     if (!eq.insert(P.Q[k], u64(1) << k)) return false;

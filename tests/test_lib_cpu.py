@@ -724,3 +724,27 @@ def test_comm_check_loopback_ok_and_null_invalid():
     c = ll.Comm.loopback(4)
     c.check()
     assert ll.STATUS[ll._lib.ll_comm_check(None)] == "INVALID_ARG"
+
+
+def test_linear_tiles_with_identical_dev_bits():
+    """General memory layouts (R2) with the same `dev` bits in A and B: the class stays
+    local (CTA), each rank's slice is planned as a linear tile over its local bits, and
+    the emulated schedule equals the oracle on the slice."""
+    rng = np.random.default_rng(9)
+    d = 12
+    linear = 0
+    for trial in range(8):
+        ca, cb = gen.random_memory_cols(rng, d), gen.random_memory_cols(rng, d)
+        out = [("x", d + 2)]
+        ins = [("offset", d), ("dev", 2)]
+        A = ll.Layout(ins, out, {"offset": [(c,) for c in ca], "dev": [(1 << d,), (2 << d,)]})
+        B = ll.Layout(ins, out, {"offset": [(c,) for c in cb], "dev": [(1 << d,), (2 << d,)]})
+        p = ll.ll_plan_convert(A, B, 4)
+        t = p.describe()
+        assert t["class"] == "CTA" and t["exec"] == "tile"
+        linear += bool(t["tile"].get("linear_tile"))
+        OA = O.layout_from_cols([("offset", d)], [("x", d)], ca)
+        OB = O.layout_from_cols([("offset", d)], [("x", d)], cb)
+        src = gen.random_bits(rng, 1 << d, 4)
+        assert np.array_equal(p.simulate(src, 1 << d), O.convert(OA, OB, src))
+    assert linear >= 4
