@@ -152,6 +152,7 @@ struct TilePlan {
   // non-empty these replace 1 << ld_bit / 1 << grid_src_bit.
   std::vector<u64> ld_xcol, grid_src_xcol;
   int ld_run = -1;      // linear tiles: low src bits loaded as contiguous runs (c)
+  int st_run = -1;      // linear tiles: low dst bits stored as contiguous runs (cs)
   int sigma = SIGMA_COALESCED;
   int xchg = X_COPY;
   bool pipe = false;    // X_SMEM: next tile's loads issued before this tile's stores

@@ -790,22 +790,43 @@ static bool build_linear_tile(ConvPlan& P, const ll_plan_opts* opts) {
   const int v = std::max(0, ilog2(u64(std::max(1, maxvec / w))));
   if (v + 5 > nd) return false;
   const int max_bits = ilog2(u64(65536 / w));
+  // The tile must hold dst bits [0, cs) (store runs of 2^cs elements) and the preimages of
+  // src bits [0, cl) (load runs of 2^cl).  cl = v + 1 still fills whole 32-byte sectors on
+  // the load side (two 16-byte lane vectors per sector), so L2 traffic stays algorithmic.
+  // Default: the widest store runs (cs = v + 5, 512 B per warp instruction) and the longest
+  // load runs that then fit.  Balanced (LL_LINEAR_BALANCE=1): maximise the shorter of the
+  // two runs first — a closure that only fits at cl = v + 1 with cs = v + 5 may fit 128-byte
+  // runs on both sides.
+  const char* bal_env = std::getenv("LL_LINEAR_BALANCE");
+  const bool balance = bal_env && std::string(bal_env) == "1";
   std::vector<char> inD(nd, 0);
-  int cnt = 0;
-  bool ok = false;
-  // c = v + 1 still fills whole 32-byte sectors on the load side (two 16-byte lane vectors
-  // per sector), so DRAM traffic stays algorithmic; longer runs cut L2 requests
-  for (int c = v + 5; c >= v + 1 && !ok; --c) {
-    std::fill(inD.begin(), inD.end(), 0);
-    for (int k = 0; k < v + 5; ++k) inD[k] = 1;   // the store side's vector and lanes
-    for (int k = 0; k < c; ++k) {
+  int cnt = 0, cs_best = -1, cl_best = -1;
+  auto closure = [&](int cs, int cl, std::vector<char>& in) {
+    std::fill(in.begin(), in.end(), 0);
+    for (int k = 0; k < cs; ++k) in[k] = 1;
+    for (int k = 0; k < cl; ++k) {
       const u64 y = qinv(u64(1) << k);   // the dst vector whose image is src bit k
-      for (int d = 0; d < nd; ++d) if ((y >> d) & 1) inD[d] = 1;
+      for (int d = 0; d < nd; ++d) if ((y >> d) & 1) in[d] = 1;
     }
-    cnt = int(std::count(inD.begin(), inD.end(), 1));
-    ok = cnt <= max_bits;
+    return int(std::count(in.begin(), in.end(), 1));
+  };
+  {
+    std::vector<char> tmp(nd, 0);
+    auto better = [&](int cs, int cl) {
+      if (cs_best < 0) return true;
+      if (!balance) return cs > cs_best || (cs == cs_best && cl > cl_best);
+      const int m = std::min(cs, cl), mb = std::min(cs_best, cl_best);
+      return m > mb || (m == mb && cs + cl > cs_best + cl_best) || (m == mb && cs + cl == cs_best + cl_best && cs > cs_best);
+    };
+    for (int cs = v + 5; cs >= (balance ? v + 2 : v + 5); --cs)
+      for (int cl = v + 5; cl >= v + 1; --cl) {
+        if (!better(cs, cl)) continue;
+        const int c = closure(cs, cl, tmp);
+        if (c <= max_bits) { cs_best = cs; cl_best = cl; cnt = c; inD = tmp; }
+      }
   }
-  if (!ok) return false;
+  if (cs_best < 0) return false;
+  const int cs = cs_best;
   const int target = std::max(v + 5, ilog2(u64(std::max(1, default_int(opts, &ll_plan_opts::tile_bytes, 16384) / w))));
   for (int k = 0; k < nd && cnt < target; ++k) if (!inD[k]) { inD[k] = 1; ++cnt; }
   TilePlan& T = P.tile;
@@ -817,14 +838,15 @@ static bool build_linear_tile(ConvPlan& P, const ll_plan_opts* opts) {
   T.R = T.n - 5 - T.Wb;
   if (T.R < v) return false;
   T.vld = T.vst = v;
-  // store side: the 16-byte vector, then 5 lanes over the next dst bits (512 contiguous
-  // bytes per warp instruction), then the rest of D: registers low, warps high
+  // store side: the 16-byte vector, then lanes over the next cs - v dst bits (2^cs
+  // contiguous elements per warp instruction; 512 bytes at cs = v + 5), the remaining
+  // lanes over the lowest other bits of D, then the rest of D: registers low, warps high
   std::vector<int> rest;
-  for (int k = v + 5; k < nd; ++k) if (inD[k]) rest.push_back(k);
+  for (int k = cs; k < nd; ++k) if (inD[k]) rest.push_back(k);
   T.st_bit.assign(T.n, -1);
   for (int b = 0; b < v; ++b) T.st_bit[b] = b;
-  for (int t = 0; t < 5; ++t) T.st_bit[T.R + t] = v + t;
   size_t ri = 0;
+  for (int t = 0; t < 5; ++t) T.st_bit[T.R + t] = v + t < cs ? v + t : rest[ri++];
   for (int b = v; b < T.R; ++b) T.st_bit[b] = rest[ri++];
   for (int t = 0; t < T.Wb; ++t) T.st_bit[T.R + 5 + t] = rest[ri++];
   // load side: the src vector and lanes over the low src bits (when in the tile's image),
@@ -860,6 +882,7 @@ static bool build_linear_tile(ConvPlan& P, const ll_plan_opts* opts) {
   }
   if (es.rank != T.n) return false;
   T.ld_run = v;
+  T.st_run = cs;
   while (T.ld_run < v + 5 && T.ld_xcol[T.R + (T.ld_run - v)] == (u64(1) << T.ld_run)) ++T.ld_run;
   T.ld_bit = T.st_bit;   // (unused for the load side: ld_xcol)
   for (int k = 0; k < nd; ++k)
@@ -1116,7 +1139,8 @@ std::string describe(const ConvPlan& P) {
       << ",\"grid_src_bit\":" << ivec_json(T.grid_src_bit) << ",\"grid_dst_bit\":" << ivec_json(T.grid_dst_bit);
     if (!T.ld_xcol.empty())
       o << ",\"ld_xcol\":" << vec_json(T.ld_xcol) << ",\"linear_tile\":" << (T.ld_run >= 0 ? "true" : "false")
-        << ",\"ld_run_bits\":" << (T.ld_run >= 0 ? T.ld_run : T.vld + 5);
+        << ",\"ld_run_bits\":" << (T.ld_run >= 0 ? T.ld_run : T.vld + 5)
+        << ",\"st_run_bits\":" << (T.st_run >= 0 ? T.st_run : T.vst + 5);
     if (T.xchg == X_SHUFFLE)
       o << ",\"V\":" << vec_json(T.V) << ",\"I\":" << vec_json(T.I) << ",\"E\":" << vec_json(T.E)
         << ",\"F\":" << vec_json(T.F) << ",\"G\":" << vec_json(T.G) << ",\"R_basis\":" << vec_json(T.Rb)

@@ -748,3 +748,40 @@ def test_linear_tiles_with_identical_dev_bits():
         src = gen.random_bits(rng, 1 << d, 4)
         assert np.array_equal(p.simulate(src, 1 << d), O.convert(OA, OB, src))
     assert linear >= 4
+
+
+@pytest.mark.parametrize("balance", ["0", "1"])
+def test_linear_tile_run_choice_simulated(monkeypatch, balance):
+    """Linear tiles under both run choices (LL_LINEAR_BALANCE): widest store runs, or the
+    longest shorter run of the two sides.  The tile holds dst bits [0, cs) and the
+    preimages of src bits [0, cl); the first cs - v lanes store consecutive dst bits.
+    Emulated schedules of random R2 memory layouts equal the oracle."""
+    monkeypatch.setenv("LL_LINEAR_BALANCE", balance)
+    shorter = 0
+    tiles = 0
+    for w in (1, 2, 4, 8):
+        rng = np.random.default_rng(700 + w)
+        for d in (12, 14, 16):
+            for _ in range(3):
+                ca, cb = gen.random_memory_cols(rng, d), gen.random_memory_cols(rng, d)
+                ins, out = [("offset", d)], [("x", d)]
+                OA, OB = O.layout_from_cols(ins, out, ca), O.layout_from_cols(ins, out, cb)
+                A = ll.Layout(ins, out, {"offset": [(c,) for c in ca]})
+                B = ll.Layout(ins, out, {"offset": [(c,) for c in cb]})
+                p = ll.ll_plan_convert(A, B, w)
+                t = p.describe()
+                if t["exec"] != "tile" or not t["tile"].get("linear_tile"):
+                    continue
+                tiles += 1
+                T = t["tile"]
+                v = T["vst"]
+                cs = T["st_run_bits"]
+                assert v + 2 <= cs <= v + 5
+                lanes = T["st_bit"][T["R"]:T["R"] + 5]
+                assert lanes[:cs - v] == list(range(v, cs))
+                shorter += cs < v + 5
+                src = gen.random_bits(rng, 1 << d, w)
+                assert np.array_equal(p.simulate(src, 1 << d), O.convert(OA, OB, src)), (w, d)
+    assert tiles >= 20
+    if balance == "0":
+        assert shorter == 0

@@ -169,16 +169,27 @@ def generic_maps():
             ca, cb = gen.random_memory_cols(rng, d), gen.random_memory_cols(rng, d)
             A = ll.Layout([("offset", d)], [("x", d)], {"offset": [(c,) for c in ca]})
             B = ll.Layout([("offset", d)], [("x", d)], {"offset": [(c,) for c in cb]})
-            p = ll.ll_plan_convert(A, B, w)
-            p.prepare()
             nbytes = (1 << d) * w
             src = torch.randint(-2 ** 15, 2 ** 15, (nbytes // 2,), dtype=torch.int16, device="cuda")
             dst = torch.empty_like(src)
-            ms = time_fn(lambda: ll.ll_convert(src, dst, p))
-            gbs = 2 * nbytes / ms / 1e6
-            print(json.dumps({"case": f"random R2 memory layouts 2^{d} x {w} B #{case}", "exec": p.describe()["exec"],
-                              "ms": round(ms, 4), "GBps": round(gbs, 1), "frac_6539": round(gbs / 6539.5, 3)}), flush=True)
-            del src, dst
+            ref = None
+            for bal in ("0", "1"):          # linear-tile run choice: widest stores vs balanced runs
+                os.environ["LL_LINEAR_BALANCE"] = bal
+                p = ll.ll_plan_convert(A, B, w)
+                p.prepare()
+                ms = time_fn(lambda: ll.ll_convert(src, dst, p))
+                out = dst.clone()
+                same = ref is None or bool(torch.equal(ref, out))
+                ref = out if ref is None else ref
+                gbs = 2 * nbytes / ms / 1e6
+                t = p.describe().get("tile", {})
+                print(json.dumps({"case": f"random R2 memory layouts 2^{d} x {w} B #{case}", "balance": bal,
+                                  "exec": p.describe()["exec"], "st_run_bits": t.get("st_run_bits"),
+                                  "ld_run_bits": t.get("ld_run_bits"), "smem_bytes": t.get("smem_bytes"),
+                                  "same_bytes": same, "ms": round(ms, 4), "GBps": round(gbs, 1),
+                                  "frac_6539": round(gbs / 6539.5, 3)}), flush=True)
+            os.environ.pop("LL_LINEAR_BALANCE", None)
+            del src, dst, ref, out
 
 
 def swizzle_case():
