@@ -43,6 +43,8 @@
  *  - LL_LOG=1: every conversion plan is printed (ll_plan_describe JSON) to stderr.
  *  - LL_JIT_CACHE=<dir>: the NVRTC cubin cache (default: in-tree .ll_jit_cache/).
  *  - LL_PDL=0: launch without programmatic dependent launch.
+ *  - LL_LINEAR_BALANCE=0: linear CTA tiles (general invertible pull maps) take the
+ *    widest store runs instead of the default balanced load/store run lengths.
  *  Host entry points (planning, launches) are wrapped in NVTX ranges named after
  *  the call (ll_plan_convert, ll_convert, ll_gather, ll_reduce, ll_scan).
  */

@@ -785,3 +785,5 @@ def test_linear_tile_run_choice_simulated(monkeypatch, balance):
     assert tiles >= 20
     if balance == "0":
         assert shorter == 0
+    else:
+        assert shorter > 0
