@@ -733,9 +733,12 @@ static void plan_exchange(ConvPlan& P, const ll_plan_opts* opts) {
   if (T.xchg == X_SMEM) {
     // software-pipelined smem exchange (next tile's loads before this tile's stores):
     // measured slower on every default-sized config — the second register buffer costs
-    // occupancy (profiles/r01_sweep_smem_pipeline.jsonl) — so only on request
+    // occupancy (profiles/r01_sweep_smem_pipeline.jsonl) — so only on request (LL_PIPE=1),
+    // except for linear tiles (ld_run set): their XOR-addressed 64 KiB tiles run one CTA
+    // per SM, whose load and store phases otherwise serialise; pipelined they measured
+    // 1.0-1.29x on random R2 maps (profiles/r01_sweep_linear_pipe.jsonl; LL_PIPE=0 off)
     const char* e = std::getenv("LL_PIPE");
-    T.pipe = e && std::string(e) == "1";
+    T.pipe = e ? std::string(e) == "1" : T.ld_run >= 0;
   }
   if (T.xchg == X_SMEM && (T.smem_elems * u64(T.w)) > 200 * 1024)
     fail(LL_ERR_UNSUPPORTED, "smem tile too large");
@@ -888,6 +891,8 @@ static bool build_linear_tile(ConvPlan& P, const ll_plan_opts* opts) {
   T.st_run = cs;
   while (T.ld_run < v + 5 && T.ld_xcol[T.R + (T.ld_run - v)] == (u64(1) << T.ld_run)) ++T.ld_run;
   T.ld_bit = T.st_bit;   // (unused for the load side: ld_xcol)
+  // CTA grid: the dst bits outside D, ascending (concurrent CTAs store neighbouring dst
+  // runs; ordering by the src side's bits measured no better, r01_sweep_linear_tiles2.jsonl)
   for (int k = 0; k < nd; ++k)
     if (!inD[k]) {
       T.grid_dst_bit.push_back(k);
@@ -1152,7 +1157,7 @@ std::string describe(const ConvPlan& P) {
     if (T.xchg == X_SMEM)
       o << ",\"Vec\":" << vec_json(T.sw_vec) << ",\"Bank\":" << vec_json(T.sw_bank) << ",\"Seg\":" << vec_json(T.sw_seg)
         << ",\"H\":" << vec_json(T.sw_H) << ",\"C\":" << vec_json(T.sw_C)
-        << ",\"smem_bytes\":" << T.smem_elems * T.w
+        << ",\"smem_bytes\":" << T.smem_elems * T.w << ",\"pipe\":" << (T.pipe ? "true" : "false")
         << ",\"wavefronts_st\":" << T.predicted_wavefronts_st << ",\"wavefronts_ld\":" << T.predicted_wavefronts_ld
         << ",\"ideal_wavefronts\":" << T.ideal_wavefronts
         << ",\"smem_store\":\"" << smem_instr_name(T.smi_ld, true, T.mat_sel_ld.size(), T.sm_v, T.w) << "\""

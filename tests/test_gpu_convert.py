@@ -737,3 +737,53 @@ def test_gather_axis_over_warps_smem():
     d_dst = empty_device(n, 4)
     ll.ll_gather(to_device(src), to_device(idx.view(np.uint32)), d_dst, plan)
     assert np.array_equal(from_device(d_dst, 4), O.gather(OL, 2, src, idx))
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("grid_per_sm", [None, "1"])
+@pytest.mark.parametrize("pipe", ["0", "1"])
+def test_smem_pipeline_both_ways_gpu(monkeypatch, pipe, grid_per_sm):
+    """The software-pipelined smem exchange (next tile's loads before this tile's smem
+    reads and stores; default for linear tiles, LL_PIPE=1 elsewhere) and the plain one
+    are both bit-exact against the oracle: config 3, config 1-batch (smem forced) and
+    random R2 memory layouts planned as linear tiles.  LL_GRID_PER_SM=1 caps the grid at
+    one CTA per SM, so every CTA loops over several tiles (the pipelined path's
+    steady state)."""
+    import torch
+    monkeypatch.setenv("LL_PIPE", pipe)
+    if grid_per_sm:
+        monkeypatch.setenv("LL_GRID_PER_SM", grid_per_sm)
+    else:
+        monkeypatch.delenv("LL_GRID_PER_SM", raising=False)
+    for (sa, sb), w, opts in [(W.c3(9), 2, {}), (W.c1_batched(12), 4, {"force_class": "SMEM"})]:
+        A, OA = both(sa)
+        B, OB = both(sb)
+        plan = ll.ll_plan_convert(A, B, w, **opts)
+        assert plan.describe()["tile"]["pipe"] == (pipe == "1")
+        src = O.pack(OA, gen.random_bits(np.random.default_rng(1003), 1 << OA.d_out, w))
+        d_dst = empty_device(src.size, w)
+        ll.ll_convert(to_device(src), d_dst, plan)
+        torch.cuda.synchronize()
+        assert np.array_equal(from_device(d_dst, w), O.convert(OA, OB, src))
+    rng = np.random.default_rng(800)
+    linear = 0
+    for w in (2, 4):
+        for d in (16, 20):
+            ca, cb = gen.random_memory_cols(rng, d), gen.random_memory_cols(rng, d)
+            ins, out = [("offset", d)], [("x", d)]
+            OA, OB = O.layout_from_cols(ins, out, ca), O.layout_from_cols(ins, out, cb)
+            A = ll.Layout(ins, out, {"offset": [(c,) for c in ca]})
+            B = ll.Layout(ins, out, {"offset": [(c,) for c in cb]})
+            plan = ll.ll_plan_convert(A, B, w)
+            t = plan.describe()
+            if t["exec"] != "tile" or t["tile"]["xchg"] != "smem":
+                continue
+            linear += 1
+            assert t["tile"]["pipe"] == (pipe == "1")
+            src = gen.random_bits(rng, 1 << d, w)
+            d_dst = empty_device(1 << d, w)
+            ll.ll_convert(to_device(src), d_dst, plan)
+            torch.cuda.synchronize()
+            assert np.array_equal(from_device(d_dst, w), O.convert(OA, OB, src)), (w, d)
+    assert linear >= 2
+

@@ -787,3 +787,23 @@ def test_linear_tile_run_choice_simulated(monkeypatch, balance):
         assert shorter == 0
     else:
         assert shorter > 0
+
+
+def test_linear_tiles_pipelined_by_default(monkeypatch):
+    """Without LL_PIPE, linear-tile plans (random R2 memory layouts) take the pipelined
+    smem exchange and other smem plans (config 3) do not."""
+    monkeypatch.delenv("LL_PIPE", raising=False)
+    A, B = (ll.Layout.from_spec(x) for x in W.c3(9))
+    assert ll.ll_plan_convert(A, B, 2).describe()["tile"]["pipe"] is False
+    rng = np.random.default_rng(801)
+    seen = 0
+    for _ in range(6):
+        d = 18
+        ca, cb = gen.random_memory_cols(rng, d), gen.random_memory_cols(rng, d)
+        ins, out = [("offset", d)], [("x", d)]
+        t = ll.ll_plan_convert(ll.Layout(ins, out, {"offset": [(c,) for c in ca]}),
+                               ll.Layout(ins, out, {"offset": [(c,) for c in cb]}), 4).describe()
+        if t["exec"] == "tile" and t["tile"].get("linear_tile") and t["tile"]["xchg"] == "smem":
+            assert t["tile"]["pipe"] is True
+            seen += 1
+    assert seen >= 1

@@ -56,6 +56,24 @@ elif a.case in conv:
     dst = torch.empty_like(src)
     for _ in range(a.iters):
         ll.ll_convert(src, dst, p)
+elif a.case.startswith("r2_"):
+    # random R2 memory layouts of 2^28 elements, as tools/sweep.py --only generic: r2_<w>_<i>
+    import numpy as np
+    from workloads import gen
+    _, wq, iq = a.case.split("_")
+    rng = np.random.default_rng(5)
+    d = 28
+    for w in (2, 4):
+        for i in range(3):
+            ca, cb = gen.random_memory_cols(rng, d), gen.random_memory_cols(rng, d)
+            if w == int(wq) and i == int(iq):
+                A = ll.Layout([("offset", d)], [("x", d)], {"offset": [(c,) for c in ca]})
+                B = ll.Layout([("offset", d)], [("x", d)], {"offset": [(c,) for c in cb]})
+                p = ll.ll_plan_convert(A, B, w)
+                src = torch.randint(-2 ** 15, 2 ** 15, ((1 << d) * w // 2,), dtype=torch.int16, device="cuda")
+                dst = torch.empty_like(src)
+                for _ in range(a.iters):
+                    ll.ll_convert(src, dst, p)
 elif a.case.startswith("gather"):
     parts = a.case.split("_")
     fam = parts[1]

@@ -86,6 +86,8 @@ def main():
         return matrix_tiles()
     if "invec" in only:
         return invec_swizzles()
+    if "lintb" in only:
+        return linear_thread_bytes()
     if "generic" in only:
         return generic_maps()
     if "all" not in only and "conv" not in only:
@@ -190,6 +192,42 @@ def generic_maps():
                                   "frac_6539": round(gbs / 6539.5, 3)}), flush=True)
             os.environ.pop("LL_LINEAR_BALANCE", None)
             del src, dst, ref, out
+
+
+def linear_thread_bytes():
+    """Linear tiles on the random R2 maps of generic_maps(): bytes per thread (registers
+    and occupancy against in-flight bytes), balanced runs."""
+    import numpy as np
+    from workloads import gen
+    rng = np.random.default_rng(5)
+    d = 28
+    for w in (2, 4):
+        for case in range(3):
+            ca, cb = gen.random_memory_cols(rng, d), gen.random_memory_cols(rng, d)
+            A = ll.Layout([("offset", d)], [("x", d)], {"offset": [(c,) for c in ca]})
+            B = ll.Layout([("offset", d)], [("x", d)], {"offset": [(c,) for c in cb]})
+            nbytes = (1 << d) * w
+            src = torch.randint(-2 ** 15, 2 ** 15, (nbytes // 2,), dtype=torch.int16, device="cuda")
+            dst = torch.empty_like(src)
+            ref = None
+            for tb, pipe in ((0, "0"), (0, "1"), (64, "1"), (128, "1")):
+                os.environ["LL_PIPE"] = pipe      # software-pipelined smem exchange
+                p = ll.ll_plan_convert(A, B, w, thread_bytes=tb)
+                p.prepare()
+                ms = time_fn(lambda: ll.ll_convert(src, dst, p))
+                same = ref is None or bool(torch.equal(ref, dst))
+                if ref is None:
+                    ref = dst.clone()
+                gbs = 2 * nbytes / ms / 1e6
+                t = p.describe().get("tile", {})
+                print(json.dumps({"case": f"random R2 memory layouts 2^{d} x {w} B #{case}", "thread_bytes": tb,
+                                  "pipe": pipe,
+                                  "exec": p.describe()["exec"], "threads": t.get("threads"), "R": t.get("R"),
+                                  "st_run_bits": t.get("st_run_bits"), "ld_run_bits": t.get("ld_run_bits"),
+                                  "smem_store": t.get("smem_store"), "same_bytes": same, "ms": round(ms, 4),
+                                  "GBps": round(gbs, 1), "frac_6539": round(gbs / 6539.5, 3)}), flush=True)
+            os.environ.pop("LL_PIPE", None)
+            del src, dst, ref
 
 
 def swizzle_case():
