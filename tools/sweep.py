@@ -210,8 +210,9 @@ def linear_thread_bytes():
             src = torch.randint(-2 ** 15, 2 ** 15, (nbytes // 2,), dtype=torch.int16, device="cuda")
             dst = torch.empty_like(src)
             ref = None
-            for tb, pipe in ((0, "0"), (0, "1"), (64, "1"), (128, "1")):
+            for tb, pipe, mb in ((0, "1", "0"), (0, "0", "2"), (0, "1", "2"), (0, "0", "3"), (128, "0", "2")):
                 os.environ["LL_PIPE"] = pipe      # software-pipelined smem exchange
+                os.environ["LL_MIN_BLOCKS"] = mb  # __launch_bounds__ min CTAs per SM
                 p = ll.ll_plan_convert(A, B, w, thread_bytes=tb)
                 p.prepare()
                 ms = time_fn(lambda: ll.ll_convert(src, dst, p))
@@ -221,12 +222,13 @@ def linear_thread_bytes():
                 gbs = 2 * nbytes / ms / 1e6
                 t = p.describe().get("tile", {})
                 print(json.dumps({"case": f"random R2 memory layouts 2^{d} x {w} B #{case}", "thread_bytes": tb,
-                                  "pipe": pipe,
+                                  "pipe": pipe, "min_blocks": mb,
                                   "exec": p.describe()["exec"], "threads": t.get("threads"), "R": t.get("R"),
                                   "st_run_bits": t.get("st_run_bits"), "ld_run_bits": t.get("ld_run_bits"),
                                   "smem_store": t.get("smem_store"), "same_bytes": same, "ms": round(ms, 4),
                                   "GBps": round(gbs, 1), "frac_6539": round(gbs / 6539.5, 3)}), flush=True)
             os.environ.pop("LL_PIPE", None)
+            os.environ.pop("LL_MIN_BLOCKS", None)
             del src, dst, ref
 
 
