@@ -57,7 +57,8 @@ class _Dim(C.Structure):
 class _Opts(C.Structure):
     _fields_ = [("force_class", C.c_int), ("max_vec_bytes", C.c_int), ("sigma", C.c_int),
                 ("tile_bytes", C.c_int), ("thread_bytes", C.c_int), ("generic", C.c_int),
-                ("comm", C.c_void_p), ("exchange", C.c_int), ("smem_instr", C.c_int), ("reduce_op", C.c_int)]
+                ("comm", C.c_void_p), ("exchange", C.c_int), ("smem_instr", C.c_int), ("reduce_op", C.c_int),
+                ("pipe", C.c_int), ("min_blocks", C.c_int)]
 
 
 _P = C.c_void_p
@@ -153,7 +154,7 @@ IPC_HANDLE_BYTES = 72
 
 
 def _opts(force_class=None, max_vec_bytes=16, sigma=0, tile_bytes=0, thread_bytes=0, generic=False, comm=None,
-          exchange="auto", smem_instr="auto", reduce_op="sum"):
+          exchange="auto", smem_instr="auto", reduce_op="sum", pipe="auto", min_blocks=0):
     o = _Opts()
     _lib.ll_plan_opts_default(C.byref(o))
     if force_class is not None:
@@ -167,6 +168,8 @@ def _opts(force_class=None, max_vec_bytes=16, sigma=0, tile_bytes=0, thread_byte
     o.exchange = EXCHANGES.index(exchange) if isinstance(exchange, str) else int(exchange)
     o.smem_instr = SMEM_INSTRS.index(smem_instr) if isinstance(smem_instr, str) else int(smem_instr)
     o.reduce_op = REDUCE_OPS.index(reduce_op) if isinstance(reduce_op, str) else int(reduce_op)
+    o.pipe = {"auto": 0, "off": 1, "on": 2}[pipe] if isinstance(pipe, str) else int(pipe)
+    o.min_blocks = int(min_blocks)
     return o
 
 

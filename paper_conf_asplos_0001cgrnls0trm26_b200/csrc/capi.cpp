@@ -609,7 +609,8 @@ ll_status ll_convert(const void* src, void* dst, void* ws, const ll_plan* p, voi
 
 // Measured plan selection: every candidate kernel decomposition (thread_bytes 64 / 128
 // / 256 and the default, with and without a forced smem exchange, with and without
-// stmatrix / ldmatrix) is planned,
+// stmatrix / ldmatrix; for linear tiles also with and without the pipelined exchange
+// and the two-CTAs-per-SM register cap) is planned,
 // compiled and timed on the caller's buffers; the fastest plan is returned.
 ll_status ll_plan_autotune(const ll_layout* A, const ll_layout* B, int w, const ll_plan_opts* base,
                            const void* src, void* dst, void* stream, int iters, ll_plan** out) {
@@ -630,6 +631,18 @@ ll_status ll_plan_autotune(const ll_layout* A, const ll_layout* B, int w, const 
   if (o0.smem_instr == 0) {
     const size_t nc = cand.size();
     for (size_t i = 0; i < nc; ++i) { ll_plan_opts c = cand[i]; c.smem_instr = 1; cand.push_back(c); }
+  }
+  // linear tiles (general invertible pull maps): the pipelined exchange and the ptxas
+  // register cap (two CTAs per SM) both help some maps and hurt others — time them
+  {
+    ll_plan* raw = nullptr;
+    if (ll_plan_convert(A, B, w, &o0, &raw) == LL_OK) {
+      std::unique_ptr<ll_plan> p0(raw);
+      const ConvPlan& P0 = p0->cp();
+      if (P0.exec == EXEC_TILE && P0.tile.ld_run >= 0 && o0.pipe == 0 && o0.min_blocks == 0)
+        for (int pp : {1, 2})
+          for (int mb : {-1, 2}) { ll_plan_opts c = o0; c.pipe = pp; c.min_blocks = mb; cand.push_back(c); }
+    }
   }
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   cudaEvent_t e0, e1;
@@ -665,6 +678,7 @@ ll_status ll_plan_autotune(const ll_layout* A, const ll_layout* B, int w, const 
       static const char* xc[] = {"copy", "regperm", "shuffle", "smem"};
       log << (first ? "" : ",") << "{\"thread_bytes\":" << c.thread_bytes << ",\"force_smem\":"
           << (c.force_class == LL_CLASS_SMEM ? "true" : "false") << ",\"smem_instr\":" << c.smem_instr
+          << ",\"pipe\":" << (P.tile.pipe ? "true" : "false") << ",\"min_blocks\":" << P.tile.min_blocks
           << ",\"xchg\":\"" << xc[P.tile.xchg]
           << "\",\"R\":" << P.tile.R << ",\"threads\":" << P.tile.threads() << ",\"ms\":" << ms << "}";
       first = false;

@@ -137,11 +137,8 @@ std::string codegen_tile(const ConvPlan& Pl) {
       << "  ll_tile_body<P, DstPeers<" << sh << ">, " << (Pl.peer_reg ? "true" : "false") << ">(src, DstPeers<" << sh
       << ">(&peers), ntiles, tile0);\n}\n";
   } else {
-    // LL_MIN_BLOCKS=k (experiment hook): ask ptxas for k resident CTAs per SM
-    const char* mb = std::getenv("LL_MIN_BLOCKS");
-    const int minb = mb ? std::atoi(mb) : 0;
     o << "extern \"C\" __global__ void __launch_bounds__(" << T.threads();
-    if (minb > 0) o << ", " << minb;
+    if (T.min_blocks > 0) o << ", " << T.min_blocks;   // ptxas register cap (plan_exchange)
     o << ") ll_tile_kernel(const u8* __restrict__ src, u8* __restrict__ dst, u64 ntiles) {\n"
       << "  ll_tile_body<P>(src, DstLocal(dst), ntiles);\n}\n";
   }

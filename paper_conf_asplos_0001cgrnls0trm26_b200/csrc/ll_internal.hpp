@@ -156,6 +156,7 @@ struct TilePlan {
   int sigma = SIGMA_COALESCED;
   int xchg = X_COPY;
   bool pipe = false;    // X_SMEM: next tile's loads issued before this tile's stores
+  int min_blocks = 0;   // __launch_bounds__ minimum resident CTAs per SM (0 = none)
 
   // --- REGPERM: out slot e <- in slot perm[e]
   std::vector<int> perm;

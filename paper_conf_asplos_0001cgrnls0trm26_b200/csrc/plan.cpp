@@ -738,7 +738,21 @@ static void plan_exchange(ConvPlan& P, const ll_plan_opts* opts) {
     // per SM, whose load and store phases otherwise serialise; pipelined they measured
     // 1.0-1.29x on random R2 maps (profiles/r01_sweep_linear_pipe.jsonl; LL_PIPE=0 off)
     const char* e = std::getenv("LL_PIPE");
-    T.pipe = e ? std::string(e) == "1" : T.ld_run >= 0;
+    const int op = opts ? opts->pipe : 0;
+    T.pipe = e ? std::string(e) == "1" : (op == 2 || (op == 0 && T.ld_run >= 0));
+  }
+  // Resident CTAs per SM (ptxas register cap).  Linear tiles compile to 170-255
+  // registers (XOR addresses that cannot fold into immediates), i.e. one CTA per SM;
+  // asking for 2 trades registers for a few spills.  Measured on random R2 maps: 4-byte
+  // elements 1.0-1.21x (two of three maps), 2-byte elements slower (b16 smem traffic
+  // spills more), profiles/r01_sweep_linear_minblocks.jsonl; ll_plan_autotune times both.
+  {
+    const char* e = std::getenv("LL_MIN_BLOCKS");
+    const int om = opts ? opts->min_blocks : 0;
+    if (e) T.min_blocks = std::max(0, std::atoi(e));
+    else if (om > 0) T.min_blocks = om;
+    else if (om == 0 && T.ld_run >= 0 && T.xchg == X_SMEM && T.w >= 4) T.min_blocks = 2;
+    else T.min_blocks = 0;
   }
   if (T.xchg == X_SMEM && (T.smem_elems * u64(T.w)) > 200 * 1024)
     fail(LL_ERR_UNSUPPORTED, "smem tile too large");
@@ -1157,7 +1171,7 @@ std::string describe(const ConvPlan& P) {
     if (T.xchg == X_SMEM)
       o << ",\"Vec\":" << vec_json(T.sw_vec) << ",\"Bank\":" << vec_json(T.sw_bank) << ",\"Seg\":" << vec_json(T.sw_seg)
         << ",\"H\":" << vec_json(T.sw_H) << ",\"C\":" << vec_json(T.sw_C)
-        << ",\"smem_bytes\":" << T.smem_elems * T.w << ",\"pipe\":" << (T.pipe ? "true" : "false")
+        << ",\"smem_bytes\":" << T.smem_elems * T.w << ",\"pipe\":" << (T.pipe ? "true" : "false") << ",\"min_blocks\":" << T.min_blocks
         << ",\"wavefronts_st\":" << T.predicted_wavefronts_st << ",\"wavefronts_ld\":" << T.predicted_wavefronts_ld
         << ",\"ideal_wavefronts\":" << T.ideal_wavefronts
         << ",\"smem_store\":\"" << smem_instr_name(T.smi_ld, true, T.mat_sel_ld.size(), T.sm_v, T.w) << "\""

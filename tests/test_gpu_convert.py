@@ -787,3 +787,37 @@ def test_smem_pipeline_both_ways_gpu(monkeypatch, pipe, grid_per_sm):
             assert np.array_equal(from_device(d_dst, w), O.convert(OA, OB, src)), (w, d)
     assert linear >= 2
 
+
+
+@pytest.mark.parametrize("w", [2, 4])
+def test_linear_tile_register_cap_and_autotune_gpu(w):
+    """Linear tiles under every pipe x min_blocks variant (the ptxas register cap makes
+    the kernel spill) and the plan ll_plan_autotune picks among them: bit-exact against
+    the oracle on random R2 memory layouts."""
+    import torch
+    rng = np.random.default_rng(900 + w)
+    d = 20
+    ca, cb = gen.random_memory_cols(rng, d), gen.random_memory_cols(rng, d)
+    ins, out = [("offset", d)], [("x", d)]
+    OA, OB = O.layout_from_cols(ins, out, ca), O.layout_from_cols(ins, out, cb)
+    A = ll.Layout(ins, out, {"offset": [(c,) for c in ca]})
+    B = ll.Layout(ins, out, {"offset": [(c,) for c in cb]})
+    src = gen.random_bits(rng, 1 << d, w)
+    ref = O.convert(OA, OB, src)
+    d_src = to_device(src)
+    for pipe in ("off", "on"):
+        for mb in (-1, 2, 3):
+            plan = ll.ll_plan_convert(A, B, w, pipe=pipe, min_blocks=mb)
+            assert plan.describe()["tile"]["linear_tile"]
+            d_dst = empty_device(1 << d, w)
+            ll.ll_convert(d_src, d_dst, plan)
+            torch.cuda.synchronize()
+            assert np.array_equal(from_device(d_dst, w), ref), (pipe, mb)
+    d_dst = empty_device(1 << d, w)
+    plan = ll.ll_plan_autotune(A, B, w, d_src, d_dst, iters=2)
+    tune = plan.describe().get("autotune", [])
+    assert any(c.get("min_blocks") == 2 for c in tune) and any(c.get("pipe") is False for c in tune)
+    d_dst.zero_()
+    ll.ll_convert(d_src, d_dst, plan)
+    torch.cuda.synchronize()
+    assert np.array_equal(from_device(d_dst, w), ref)

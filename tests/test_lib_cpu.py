@@ -807,3 +807,28 @@ def test_linear_tiles_pipelined_by_default(monkeypatch):
             assert t["tile"]["pipe"] is True
             seen += 1
     assert seen >= 1
+
+
+def test_plan_opts_pipe_and_min_blocks():
+    """ll_plan_opts.pipe / min_blocks reach the plan (describe) and the generated kernel
+    (__launch_bounds__ minimum): auto = pipelined linear tiles, with two CTAs per SM for
+    >= 4-byte elements; explicit values override; other smem plans stay unpipelined."""
+    rng = np.random.default_rng(9)
+    d = 16
+    ca, cb = gen.random_memory_cols(rng, d), gen.random_memory_cols(rng, d)
+    ins, out = [("offset", d)], [("x", d)]
+    A = ll.Layout(ins, out, {"offset": [(c,) for c in ca]})
+    B = ll.Layout(ins, out, {"offset": [(c,) for c in cb]})
+    for w, mb_auto in ((2, 0), (4, 2)):
+        p = ll.ll_plan_convert(A, B, w)
+        t = p.describe()["tile"]
+        assert t["linear_tile"] and t["pipe"] is True and t["min_blocks"] == mb_auto
+        assert (", 2)" in p.source()) == (mb_auto == 2)
+        t = ll.ll_plan_convert(A, B, w, pipe="off", min_blocks=-1).describe()["tile"]
+        assert t["pipe"] is False and t["min_blocks"] == 0
+        p = ll.ll_plan_convert(A, B, w, min_blocks=3)
+        assert p.describe()["tile"]["min_blocks"] == 3 and ", 3) ll_tile_kernel" in p.source()
+    Ac, Bc = (ll.Layout.from_spec(x) for x in W.c3(9))
+    t = ll.ll_plan_convert(Ac, Bc, 2).describe()["tile"]
+    assert t["pipe"] is False and t["min_blocks"] == 0
+    assert ll.ll_plan_convert(Ac, Bc, 2, pipe="on").describe()["tile"]["pipe"] is True

@@ -195,8 +195,9 @@ def generic_maps():
 
 
 def linear_thread_bytes():
-    """Linear tiles on the random R2 maps of generic_maps(): bytes per thread (registers
-    and occupancy against in-flight bytes), balanced runs."""
+    """Linear tiles on the random R2 maps of generic_maps(): the automatic plan, the
+    pipelined exchange with and without the two-CTAs-per-SM register cap, and the
+    plan ll_plan_autotune picks."""
     import numpy as np
     from workloads import gen
     rng = np.random.default_rng(5)
@@ -210,10 +211,14 @@ def linear_thread_bytes():
             src = torch.randint(-2 ** 15, 2 ** 15, (nbytes // 2,), dtype=torch.int16, device="cuda")
             dst = torch.empty_like(src)
             ref = None
-            for tb, pipe, mb in ((0, "1", "0"), (0, "0", "2"), (0, "1", "2"), (0, "0", "3"), (128, "0", "2")):
-                os.environ["LL_PIPE"] = pipe      # software-pipelined smem exchange
-                os.environ["LL_MIN_BLOCKS"] = mb  # __launch_bounds__ min CTAs per SM
-                p = ll.ll_plan_convert(A, B, w, thread_bytes=tb)
+            variants = [("auto", {}), ("pipe, no cap", {"pipe": "on", "min_blocks": -1}),
+                        ("pipe, 2 CTAs/SM", {"pipe": "on", "min_blocks": 2}),
+                        ("no pipe, 2 CTAs/SM", {"pipe": "off", "min_blocks": 2}), ("autotune", None)]
+            for name, opts in variants:
+                if opts is None:
+                    p = ll.ll_plan_autotune(A, B, w, src, dst, iters=5)
+                else:
+                    p = ll.ll_plan_convert(A, B, w, **opts)
                 p.prepare()
                 ms = time_fn(lambda: ll.ll_convert(src, dst, p))
                 same = ref is None or bool(torch.equal(ref, dst))
@@ -221,11 +226,11 @@ def linear_thread_bytes():
                     ref = dst.clone()
                 gbs = 2 * nbytes / ms / 1e6
                 t = p.describe().get("tile", {})
-                print(json.dumps({"case": f"random R2 memory layouts 2^{d} x {w} B #{case}", "thread_bytes": tb,
-                                  "pipe": pipe, "min_blocks": mb,
-                                  "exec": p.describe()["exec"], "threads": t.get("threads"), "R": t.get("R"),
+                print(json.dumps({"case": f"random R2 memory layouts 2^{d} x {w} B #{case}", "variant": name,
+                                  "exec": p.describe()["exec"], "threads": t.get("threads"),
+                                  "pipe": t.get("pipe"), "min_blocks": t.get("min_blocks"),
                                   "st_run_bits": t.get("st_run_bits"), "ld_run_bits": t.get("ld_run_bits"),
-                                  "smem_store": t.get("smem_store"), "same_bytes": same, "ms": round(ms, 4),
+                                  "same_bytes": same, "ms": round(ms, 4),
                                   "GBps": round(gbs, 1), "frac_6539": round(gbs / 6539.5, 3)}), flush=True)
             os.environ.pop("LL_PIPE", None)
             os.environ.pop("LL_MIN_BLOCKS", None)
