@@ -832,3 +832,15 @@ def test_plan_opts_pipe_and_min_blocks():
     t = ll.ll_plan_convert(Ac, Bc, 2).describe()["tile"]
     assert t["pipe"] is False and t["min_blocks"] == 0
     assert ll.ll_plan_convert(Ac, Bc, 2, pipe="on").describe()["tile"]["pipe"] is True
+
+
+def test_opts_struct_matches_the_c_abi():
+    """The Python mirror of ll_plan_opts has the C struct's size: ll_plan_opts_default
+    (memset + defaults) writes exactly sizeof(ll_plan_opts) bytes of a guarded buffer."""
+    n = ctypes.sizeof(ll._Opts)
+    buf = (ctypes.c_ubyte * (n + 64))(*([0xAB] * (n + 64)))
+    ll._lib.ll_plan_opts_default(ctypes.cast(buf, ctypes.POINTER(ll._Opts)))
+    assert all(b == 0xAB for b in buf[n:])
+    assert any(b != 0xAB for b in buf[n - 8:n])        # the last fields were written
+    o = ll._Opts.from_buffer(buf)
+    assert o.force_class == -1 and o.max_vec_bytes == 16 and o.pipe == 0 and o.min_blocks == 0
