@@ -56,6 +56,24 @@ elif a.case in conv:
     dst = torch.empty_like(src)
     for _ in range(a.iters):
         ll.ll_convert(src, dst, p)
+elif a.case.startswith("r2small_"):
+    # a 2^16-element random R2 map (linear tile, pipelined; compute-sanitizer size)
+    import numpy as np
+    from workloads import gen
+    w = int(a.case.split("_")[1])
+    rng = np.random.default_rng(77)
+    d = 16
+    ca, cb = gen.random_memory_cols(rng, d), gen.random_memory_cols(rng, d)
+    A = ll.Layout([("offset", d)], [("x", d)], {"offset": [(c,) for c in ca]})
+    B = ll.Layout([("offset", d)], [("x", d)], {"offset": [(c,) for c in cb]})
+    import json
+    p = ll.ll_plan_convert(A, B, w, **json.loads(a.opts))
+    print(json.dumps({k: p.describe()["tile"].get(k) for k in ("linear_tile", "pipe", "min_blocks", "ctas")}))
+    src = torch.randint(-2 ** 15, 2 ** 15, ((1 << d) * w // 2,), dtype=torch.int16, device="cuda")
+    dst = torch.empty_like(src)
+    for _ in range(a.iters):
+        ll.ll_convert(src, dst, p)
+    torch.cuda.synchronize()
 elif a.case.startswith("r2_"):
     # random R2 memory layouts of 2^28 elements, as tools/sweep.py --only generic: r2_<w>_<i>
     import numpy as np
