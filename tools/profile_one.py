@@ -24,7 +24,7 @@ conv = {"c2": (W.c2(16), 2, {}), "c2smem": (W.c2(16), 2, {"force_class": "SMEM"}
         "c1bsmem": (W.c1_batched(20), 4, {"force_class": "SMEM"}),
         # small variants for compute-sanitizer
         "c1bsmem_small": (W.c1_batched(6), 4, {"force_class": "SMEM"}),
-        "c3_small": (W.c3(3), 2, {}), "c2_small": (W.c2(3), 2, {}),
+        "c3_small": (W.c3(3), 2, {}), "c3_mid_pipe": (W.c3(9), 2, {"pipe": "on"}), "c2_small": (W.c2(3), 2, {}),
         "c3b_small": (W.c3b(3), 2, {}),
         "c2fsmem_small": (W.c2(3), 2, {"sigma": "faithful", "force_class": "SMEM", "smem_instr": "matrix"}),
         "c3f_small": (W.c3(3), 2, {"sigma": "faithful"}),
@@ -56,13 +56,13 @@ elif a.case in conv:
     dst = torch.empty_like(src)
     for _ in range(a.iters):
         ll.ll_convert(src, dst, p)
-elif a.case.startswith("r2small_"):
-    # a 2^16-element random R2 map (linear tile, pipelined; compute-sanitizer size)
+elif a.case.startswith("r2small_") or a.case.startswith("r2mid_"):
+    # a 2^16 (2^21) element random R2 map (linear tile, pipelined; compute-sanitizer size)
     import numpy as np
     from workloads import gen
     w = int(a.case.split("_")[1])
     rng = np.random.default_rng(77)
-    d = 16
+    d = 16 if a.case.startswith("r2small_") else 21
     ca, cb = gen.random_memory_cols(rng, d), gen.random_memory_cols(rng, d)
     A = ll.Layout([("offset", d)], [("x", d)], {"offset": [(c,) for c in ca]})
     B = ll.Layout([("offset", d)], [("x", d)], {"offset": [(c,) for c in cb]})
