@@ -640,8 +640,12 @@ ll_status ll_plan_autotune(const ll_layout* A, const ll_layout* B, int w, const 
       std::unique_ptr<ll_plan> p0(raw);
       const ConvPlan& P0 = p0->cp();
       if (P0.exec == EXEC_TILE && P0.tile.ld_run >= 0 && o0.pipe == 0 && o0.min_blocks == 0)
+      {
         for (int pp : {1, 2})
           for (int mb : {-1, 2}) { ll_plan_opts c = o0; c.pipe = pp; c.min_blocks = mb; cand.push_back(c); }
+        if (o0.tile_bytes == 0)   // 32 KiB tiles: shorter runs, lighter CTAs
+          for (int mb : {0, -1}) { ll_plan_opts c = o0; c.tile_bytes = 32768; c.min_blocks = mb; cand.push_back(c); }
+      }
     }
   }
   cudaStream_t st = static_cast<cudaStream_t>(stream);
@@ -676,7 +680,8 @@ ll_status ll_plan_autotune(const ll_layout* A, const ll_layout* B, int w, const 
       check_cuda(cudaEventElapsedTime(&ms, e0, e1), "cudaEventElapsedTime");
       ms /= float(iters);
       static const char* xc[] = {"copy", "regperm", "shuffle", "smem"};
-      log << (first ? "" : ",") << "{\"thread_bytes\":" << c.thread_bytes << ",\"force_smem\":"
+      log << (first ? "" : ",") << "{\"thread_bytes\":" << c.thread_bytes << ",\"tile_bytes\":" << c.tile_bytes
+          << ",\"force_smem\":"
           << (c.force_class == LL_CLASS_SMEM ? "true" : "false") << ",\"smem_instr\":" << c.smem_instr
           << ",\"pipe\":" << (P.tile.pipe ? "true" : "false") << ",\"min_blocks\":" << P.tile.min_blocks
           << ",\"xchg\":\"" << xc[P.tile.xchg]

@@ -806,8 +806,11 @@ static bool build_linear_tile(ConvPlan& P, const ll_plan_opts* opts) {
   const int maxvec = default_int(opts, &ll_plan_opts::max_vec_bytes, 16);
   const int v = std::max(0, ilog2(u64(std::max(1, maxvec / w))));
   if (v + 5 > nd) return false;
-  const char* mt_env = std::getenv("LL_LINEAR_MAX_TILE");   // experiment hook: tile byte cap
-  const int max_bits = ilog2(u64((mt_env ? std::max(1024, std::atoi(mt_env)) : 65536) / w));
+  // tile byte cap: 64 KiB, or ll_plan_opts.tile_bytes when given (32 KiB measured 0.61-1.10x
+  // of the 64 KiB tiles on random R2 maps, 128 KiB 0.15-0.96x: an autotune candidate,
+  // profiles/r01_sweep_linear_maxtile.jsonl)
+  const int tb_cap = opts && opts->tile_bytes > 0 ? std::max(opts->tile_bytes, w << (v + 5)) : 65536;
+  const int max_bits = ilog2(u64(tb_cap / w));
   // The tile must hold dst bits [0, cs) (store runs of 2^cs elements) and the preimages of
   // src bits [0, cl) (load runs of 2^cl).  cl = v + 1 still fills whole 32-byte sectors on
   // the load side (two 16-byte lane vectors per sector), so L2 traffic stays algorithmic.

@@ -215,12 +215,9 @@ def linear_thread_bytes():
                         ("pipe, 2 CTAs/SM", {"pipe": "on", "min_blocks": 2}),
                         ("no pipe, 2 CTAs/SM", {"pipe": "off", "min_blocks": 2}), ("autotune", None)]
             if os.environ.get("LL_SWEEP_MAXTILE"):
-                variants = [(f"max tile {mt}, {n}", dict(o, _mt=mt)) for mt in ("65536", "32768", "131072")
+                variants = [(f"max tile {mt}, {n}", dict(o, tile_bytes=mt)) for mt in (65536, 32768, 131072)
                             for n, o in (("auto", {}), ("2 CTAs/SM", {"min_blocks": 2}), ("no cap", {"min_blocks": -1}))]
             for name, opts in variants:
-                opts = dict(opts) if opts is not None else None
-                if opts is not None and "_mt" in opts:
-                    os.environ["LL_LINEAR_MAX_TILE"] = opts.pop("_mt")
                 if opts is None:
                     p = ll.ll_plan_autotune(A, B, w, src, dst, iters=5)
                 else:
@@ -240,7 +237,6 @@ def linear_thread_bytes():
                                   "GBps": round(gbs, 1), "frac_6539": round(gbs / 6539.5, 3)}), flush=True)
             os.environ.pop("LL_PIPE", None)
             os.environ.pop("LL_MIN_BLOCKS", None)
-            os.environ.pop("LL_LINEAR_MAX_TILE", None)
             del src, dst, ref
 
 
