@@ -43,7 +43,7 @@
  *  - LL_LOG=1: every conversion plan is printed (ll_plan_describe JSON) to stderr.
  *  - LL_JIT_CACHE=<dir>: the NVRTC cubin cache (default: in-tree .ll_jit_cache/).
  *  - LL_PDL=0: launch without programmatic dependent launch.
- *  - LL_PIPE=0|1, LL_MIN_BLOCKS=k: override ll_plan_opts.pipe / min_blocks.
+ *  - LL_PIPE=0|1|staged, LL_MIN_BLOCKS=k: override ll_plan_opts.pipe / min_blocks.
  *  - LL_LINEAR_BALANCE=0: linear CTA tiles (general invertible pull maps) take the
  *    widest store runs instead of the default balanced load/store run lengths.
  *  Host entry points (planning, launches) are wrapped in NVTX ranges named after
@@ -121,7 +121,10 @@ typedef struct {
   int reduce_op;        /* ll_plan_reduce: 0 = sum (default), 1 = max, 2 = min (fp32)   */
   int pipe;             /* smem-exchange tiles: 0 = auto (pipelined for linear tiles
                          * only), 1 = off, 2 = software-pipelined (next tile's loads
-                         * before this tile's smem reads and HBM stores)             */
+                         * before this tile's smem reads and HBM stores), 3 = staged
+                         * (the next two tiles' 16-byte src vectors streamed by
+                         * cp.async into two raw smem stages; persistent grid; needs
+                         * 16-byte load vectors and exchange + 2 tiles <= 227 KiB)   */
   int min_blocks;       /* tile kernels: resident CTAs per SM requested from ptxas
                          * (__launch_bounds__ minimum): 0 = auto (2 for linear tiles of
                          * >= 4-byte elements, else none), -1 = none, k >= 1 = k      */

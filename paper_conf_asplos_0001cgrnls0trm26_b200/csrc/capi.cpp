@@ -204,7 +204,9 @@ ll_status convert_impl(const void* src, void* dst, void* ws, ConvPlan& P, cudaSt
     u64 ntiles = u64(1) << P.tile.grid_dst_bit.size();
     unsigned long long nt = ntiles;
     void* args[] = {const_cast<void**>(&src), &dst, &nt};
-    launch_kernel(P.kernel, grid_for(ntiles), P.tile.threads(), args, size_t(P.smem_bytes), st,
+    // staged tiles loop over their tiles with two stages in flight: a persistent grid
+    const unsigned grid = P.tile.staged ? unsigned(std::min<u64>(ntiles, u64(num_sms()))) : grid_for(ntiles);
+    launch_kernel(P.kernel, grid, P.tile.threads(), args, size_t(P.smem_bytes), st,
                   "cudaLaunchKernelEx(ll_tile_kernel)");
     return LL_OK;
   }
@@ -643,6 +645,7 @@ ll_status ll_plan_autotune(const ll_layout* A, const ll_layout* B, int w, const 
       {
         for (int pp : {1, 2})
           for (int mb : {-1, 2}) { ll_plan_opts c = o0; c.pipe = pp; c.min_blocks = mb; cand.push_back(c); }
+        { ll_plan_opts c = o0; c.pipe = 3; c.min_blocks = -1; cand.push_back(c); }   // cp.async stages
         if (o0.tile_bytes == 0)   // 32 KiB tiles: shorter runs, lighter CTAs
           for (int mb : {0, -1}) { ll_plan_opts c = o0; c.tile_bytes = 32768; c.min_blocks = mb; cand.push_back(c); }
       }
@@ -683,7 +686,8 @@ ll_status ll_plan_autotune(const ll_layout* A, const ll_layout* B, int w, const 
       log << (first ? "" : ",") << "{\"thread_bytes\":" << c.thread_bytes << ",\"tile_bytes\":" << c.tile_bytes
           << ",\"force_smem\":"
           << (c.force_class == LL_CLASS_SMEM ? "true" : "false") << ",\"smem_instr\":" << c.smem_instr
-          << ",\"pipe\":" << (P.tile.pipe ? "true" : "false") << ",\"min_blocks\":" << P.tile.min_blocks
+          << ",\"pipe\":" << (P.tile.pipe ? "true" : "false") << ",\"staged\":" << (P.tile.staged ? "true" : "false")
+          << ",\"min_blocks\":" << P.tile.min_blocks
           << ",\"xchg\":\"" << xc[P.tile.xchg]
           << "\",\"R\":" << P.tile.R << ",\"threads\":" << P.tile.threads() << ",\"ms\":" << ms << "}";
       first = false;

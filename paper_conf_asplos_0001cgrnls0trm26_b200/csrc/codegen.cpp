@@ -67,6 +67,8 @@ std::string codegen_tile(const ConvPlan& Pl) {
   o << "  static constexpr bool ISOLATE_SMEM = " << (std::getenv("LL_ISOLATE_SMEM") ? "true" : "false") << ";\n";
   o << icon("ST_HINT", st_hint());
   o << "  static constexpr bool PIPE = " << (T.pipe ? "true" : "false") << ";\n";
+  o << "  static constexpr bool STAGED = " << (T.staged ? "true" : "false") << ";\n";
+  o << icon("XBYTES", (long long)(T.smem_elems * u64(T.w)));
   // per-thread-contiguous loads (faithful σ) re-use sectors across instructions
   o << "  static constexpr bool LD_L1 = " << (T.sigma == SIGMA_FAITHFUL ? "true" : "false") << ";\n";
   // XOR-copy plans: a src column may reach below the vector (bits [0, VLD)): that part is

@@ -157,6 +157,7 @@ struct TilePlan {
   int xchg = X_COPY;
   bool pipe = false;    // X_SMEM: next tile's loads issued before this tile's stores
   int min_blocks = 0;   // __launch_bounds__ minimum resident CTAs per SM (0 = none)
+  bool staged = false;  // X_SMEM: src tiles streamed by cp.async into two raw smem stages
 
   // --- REGPERM: out slot e <- in slot perm[e]
   std::vector<int> perm;

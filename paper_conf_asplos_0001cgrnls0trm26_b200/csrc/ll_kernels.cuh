@@ -108,6 +108,18 @@ __device__ __forceinline__ void stg_b32(u8* p, u32 a) {
     asm volatile("st.global.u32 [%0], %1;" ::"l"(p), "r"(a) : "memory");
 }
 
+__device__ __forceinline__ void lds_v4(u32 addr, u32& a, u32& b, u32& c, u32& d) {
+  asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(a), "=r"(b), "=r"(c), "=r"(d) : "r"(addr) : "memory");
+}
+// cp.async (LDGSTS): 16 bytes global -> shared, bypassing L1 and registers; groups
+// complete in order (cp.async.wait_group N: all but the newest N groups have landed).
+__device__ __forceinline__ void cp_async16(u32 dst, const void* src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait1() { asm volatile("cp.async.wait_group 1;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait0() { asm volatile("cp.async.wait_group 0;" ::: "memory"); }
+
 // Load vector K of the thread (2^VL elements of W bytes starting at slot K<<VL).
 template <int W, int VL, int K, int NW, bool L1A = false>
 __device__ __forceinline__ void load_vec(u32 (&r)[NW], const u8* p) {
@@ -703,6 +715,64 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, Dst D, 
       });
     });
   };
+  if constexpr (P::XCHG == 3 && P::STAGED) {
+    // Staged smem exchange (ll_plan_opts.pipe = 3): the src vectors of the next two
+    // tiles stream into two raw stages by cp.async (16 bytes each, thread-slot order
+    // [vector][thread]: 512 contiguous bytes per warp instruction, conflict-free), so a
+    // CTA keeps two tiles of loads in flight without holding them in registers.  Each
+    // thread reads back only its own slots (cp.async.wait_group is per thread), then
+    // the tile takes the usual swizzled round trip.  Persistent grid (one CTA per SM).
+    constexpr int NV = 1 << (P::R - P::VLD);
+    constexpr u32 TB = u32(P::THREADS) * NV * 16u;
+    const u32 stage0 = sbase + P::XBYTES;
+    auto issue = [&](u64 t, u32 st) {
+      if (t < ntiles) {
+        const u64 sofs = tile_base<P, true>(t) ^ ld_thr;
+        static_for<NV>([&](auto k) {
+          constexpr int K = decltype(k)::value;
+          const u8* g;
+          if constexpr (P::LD_XOR) g = src + (sofs ^ LdOff<P, K>::value());
+          else g = src + sofs + LdOff<P, K>::value();
+          cp_async16(stage0 + st * TB + (u32(K) * P::THREADS + threadIdx.x) * 16u, g);
+        });
+      }
+      cp_async_commit();   // empty groups past the end keep the group count uniform
+    };
+    u64 t = blockIdx.x;
+    issue(t, 0);
+    issue(t + gridDim.x, 1);
+    for (u32 i = 0; t < ntiles; t += gridDim.x, ++i) {
+      const u32 st = i & 1u;
+      cp_async_wait1();    // every group but the newest: tile t's vectors have landed
+      u32 r[P::NW];
+      static_for<NV>([&](auto k) {
+        constexpr int K = decltype(k)::value;
+        lds_v4(stage0 + st * TB + (u32(K) * P::THREADS + threadIdx.x) * 16u, r[4 * K], r[4 * K + 1], r[4 * K + 2],
+               r[4 * K + 3]);
+      });
+      if constexpr (P::LD_INVEC) {
+        u32 lo = lo_thr;
+        static_for<P::G>([&](auto g) {
+          constexpr int Gi = decltype(g)::value;
+          if ((t >> Gi) & 1) lo ^= P::GRID_LD_LO[Gi];
+        });
+        static_for<NV>([&](auto k) {
+          constexpr int K = decltype(k)::value;
+          xor_perm_vec<P::W, P::VLD, K, P::NW>(r, lo ^ LdLo<P, K>::value());
+        });
+      }
+      smem_store<P>(r, lane, warp, sbase);   // r consumed: this thread's stage reads are done
+      issue(t + 2 * u64(gridDim.x), st);
+      __syncthreads();
+      u32 o[P::NW];
+      static_for<P::NW>([&](auto q) { o[decltype(q)::value] = 0; });
+      smem_load<P>(o, lane, warp, sbase);
+      store_tile(o, t);
+      __syncthreads();   // exchange buffer reuse by the next tile
+    }
+    cp_async_wait0();
+    return;
+  }
   if constexpr (P::XCHG == 3 && P::PIPE) {
     // Software-pipelined smem exchange: once tile t sits in shared memory its
     // registers are free, so tile t + grid's loads are issued before t's smem reads
@@ -773,9 +843,7 @@ __device__ __forceinline__ void mbar_wait(u32 bar, u32 parity) {
                  "selp.u32 %0, 1, 0, p;\n\t}" : "=r"(ok) : "r"(bar), "r"(parity) : "memory");
   } while (!ok);
 }
-__device__ __forceinline__ void lds_v4(u32 addr, u32& a, u32& b, u32& c, u32& d) {
-  asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(a), "=r"(b), "=r"(c), "=r"(d) : "r"(addr) : "memory");
-}
+
 
 // Shared-memory vector load of thread-local vector K (2^VL elements of W bytes).
 template <int W, int VL, int K, int NW>

@@ -740,6 +740,14 @@ static void plan_exchange(ConvPlan& P, const ll_plan_opts* opts) {
     const char* e = std::getenv("LL_PIPE");
     const int op = opts ? opts->pipe : 0;
     T.pipe = e ? std::string(e) == "1" : (op == 2 || (op == 0 && T.ld_run >= 0));
+    // staged (pipe = 3 / LL_PIPE=staged): cp.async double-buffered src stages; needs
+    // 16-byte load vectors and room for the exchange buffer plus two raw tiles
+    const bool want_staged = e ? std::string(e) == "staged" : op == 3;
+    const u64 tile_b = (u64(1) << T.n) * u64(T.w);
+    if (want_staged && (T.w << T.vld) == 16 && T.smem_elems * u64(T.w) + 2 * tile_b <= 227 * 1024) {
+      T.staged = true;
+      T.pipe = false;
+    }
   }
   // Resident CTAs per SM (ptxas register cap).  Linear tiles compile to 170-255
   // registers (XOR addresses that cannot fold into immediates), i.e. one CTA per SM;
@@ -751,12 +759,13 @@ static void plan_exchange(ConvPlan& P, const ll_plan_opts* opts) {
     const int om = opts ? opts->min_blocks : 0;
     if (e) T.min_blocks = std::max(0, std::atoi(e));
     else if (om > 0) T.min_blocks = om;
-    else if (om == 0 && T.ld_run >= 0 && T.xchg == X_SMEM && T.w >= 4) T.min_blocks = 2;
+    else if (om == 0 && T.ld_run >= 0 && T.xchg == X_SMEM && T.w >= 4 && !T.staged) T.min_blocks = 2;
     else T.min_blocks = 0;
   }
   if (T.xchg == X_SMEM && (T.smem_elems * u64(T.w)) > 200 * 1024)
     fail(LL_ERR_UNSUPPORTED, "smem tile too large");
   P.smem_bytes = T.xchg == X_SMEM ? int(T.smem_elems * T.w) : 0;
+  if (T.staged) P.smem_bytes += int(2 * (u64(1) << T.n) * u64(T.w));
 }
 
 // CTA class (Q mixes block/offset bits): choose the dst bits a CTA owns so that both
@@ -1175,7 +1184,7 @@ std::string describe(const ConvPlan& P) {
     if (T.xchg == X_SMEM)
       o << ",\"Vec\":" << vec_json(T.sw_vec) << ",\"Bank\":" << vec_json(T.sw_bank) << ",\"Seg\":" << vec_json(T.sw_seg)
         << ",\"H\":" << vec_json(T.sw_H) << ",\"C\":" << vec_json(T.sw_C)
-        << ",\"smem_bytes\":" << T.smem_elems * T.w << ",\"pipe\":" << (T.pipe ? "true" : "false") << ",\"min_blocks\":" << T.min_blocks
+        << ",\"smem_bytes\":" << T.smem_elems * T.w << ",\"pipe\":" << (T.pipe ? "true" : "false") << ",\"staged\":" << (T.staged ? "true" : "false") << ",\"min_blocks\":" << T.min_blocks
         << ",\"wavefronts_st\":" << T.predicted_wavefronts_st << ",\"wavefronts_ld\":" << T.predicted_wavefronts_ld
         << ",\"ideal_wavefronts\":" << T.ideal_wavefronts
         << ",\"smem_store\":\"" << smem_instr_name(T.smi_ld, true, T.mat_sel_ld.size(), T.sm_v, T.w) << "\""

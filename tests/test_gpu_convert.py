@@ -821,3 +821,48 @@ def test_linear_tile_register_cap_and_autotune_gpu(w):
     ll.ll_convert(d_src, d_dst, plan)
     torch.cuda.synchronize()
     assert np.array_equal(from_device(d_dst, w), ref)
+
+
+def test_staged_exchange_gpu():
+    """The staged smem exchange (ll_plan_opts.pipe = "staged": the next two tiles' src
+    vectors streamed by cp.async into two raw smem stages, persistent grid, so every CTA
+    loops over several tiles) is bit-exact against the oracle on config 3, config
+    1-batch (smem forced) and random R2 memory layouts (linear tiles), and autotune
+    times it for linear tiles."""
+    import torch
+    for (sa, sb), w, opts in [(W.c3(9), 2, {}), (W.c1_batched(14), 4, {"force_class": "SMEM"})]:
+        A, OA = both(sa)
+        B, OB = both(sb)
+        plan = ll.ll_plan_convert(A, B, w, pipe="staged", **opts)
+        assert plan.describe()["tile"]["staged"] is True
+        src = O.pack(OA, gen.random_bits(np.random.default_rng(1007), 1 << OA.d_out, w))
+        d_dst = empty_device(src.size, w)
+        ll.ll_convert(to_device(src), d_dst, plan)
+        torch.cuda.synchronize()
+        assert np.array_equal(from_device(d_dst, w), O.convert(OA, OB, src))
+    rng = np.random.default_rng(810)
+    for w in (1, 2, 4, 8):
+        for d in (18, 22):
+            ca, cb = gen.random_memory_cols(rng, d), gen.random_memory_cols(rng, d)
+            ins, out = [("offset", d)], [("x", d)]
+            OA, OB = O.layout_from_cols(ins, out, ca), O.layout_from_cols(ins, out, cb)
+            A = ll.Layout(ins, out, {"offset": [(c,) for c in ca]})
+            B = ll.Layout(ins, out, {"offset": [(c,) for c in cb]})
+            plan = ll.ll_plan_convert(A, B, w, pipe="staged")
+            t = plan.describe()
+            if t["exec"] != "tile" or t["tile"]["xchg"] != "smem":
+                continue
+            src = gen.random_bits(rng, 1 << d, w)
+            d_src = to_device(src)
+            d_dst = empty_device(1 << d, w)
+            ll.ll_convert(d_src, d_dst, plan)
+            torch.cuda.synchronize()
+            ref = O.convert(OA, OB, src)
+            assert np.array_equal(from_device(d_dst, w), ref), (w, d, t["tile"]["staged"])
+            if w == 4 and d == 22:
+                tuned = ll.ll_plan_autotune(A, B, w, d_src, d_dst, iters=2)
+                assert any(c.get("staged") for c in tuned.describe().get("autotune", []))
+                d_dst.zero_()
+                ll.ll_convert(d_src, d_dst, tuned)
+                torch.cuda.synchronize()
+                assert np.array_equal(from_device(d_dst, w), ref)

@@ -88,6 +88,8 @@ def main():
         return invec_swizzles()
     if "lintb" in only:
         return linear_thread_bytes()
+    if "staged" in only:
+        return staged_configs()
     if "generic" in only:
         return generic_maps()
     if "all" not in only and "conv" not in only:
@@ -213,7 +215,8 @@ def linear_thread_bytes():
             ref = None
             variants = [("auto", {}), ("pipe, no cap", {"pipe": "on", "min_blocks": -1}),
                         ("pipe, 2 CTAs/SM", {"pipe": "on", "min_blocks": 2}),
-                        ("no pipe, 2 CTAs/SM", {"pipe": "off", "min_blocks": 2}), ("autotune", None)]
+                        ("no pipe, 2 CTAs/SM", {"pipe": "off", "min_blocks": 2}),
+                        ("staged (cp.async)", {"pipe": "staged", "min_blocks": -1}), ("autotune", None)]
             if os.environ.get("LL_SWEEP_MAXTILE"):
                 variants = [(f"max tile {mt}, {n}", dict(o, tile_bytes=mt)) for mt in (65536, 32768, 131072)
                             for n, o in (("auto", {}), ("2 CTAs/SM", {"min_blocks": 2}), ("no cap", {"min_blocks": -1}))]
@@ -231,13 +234,38 @@ def linear_thread_bytes():
                 t = p.describe().get("tile", {})
                 print(json.dumps({"case": f"random R2 memory layouts 2^{d} x {w} B #{case}", "variant": name,
                                   "exec": p.describe()["exec"], "threads": t.get("threads"),
-                                  "pipe": t.get("pipe"), "min_blocks": t.get("min_blocks"),
+                                  "pipe": t.get("pipe"), "staged": t.get("staged"), "min_blocks": t.get("min_blocks"),
                                   "st_run_bits": t.get("st_run_bits"), "ld_run_bits": t.get("ld_run_bits"),
                                   "same_bytes": same, "ms": round(ms, 4),
                                   "GBps": round(gbs, 1), "frac_6539": round(gbs / 6539.5, 3)}), flush=True)
             os.environ.pop("LL_PIPE", None)
             os.environ.pop("LL_MIN_BLOCKS", None)
             del src, dst, ref
+
+
+def staged_configs():
+    """The staged (cp.async) smem exchange against the default plan on the smem-class
+    BASELINE conversions (config 3, 3b, 5-T, config 1-batch with smem forced)."""
+    cases = [("c3", W.c3(14), 2, {}), ("c3b", W.c3b(14), 2, {}), ("c5T", W.c5T(0), 2, {}),
+             ("c1b smem", W.c1_batched(20), 4, {"force_class": "SMEM"})]
+    for name, (sa, sb), w, o in cases:
+        A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
+        n = (1 << A.d_in) * w // 2
+        src = torch.randint(-2 ** 15, 2 ** 15, (n,), dtype=torch.int16, device="cuda")
+        dst = torch.empty_like(src)
+        ref = None
+        for var, extra in (("default", {}), ("staged", {"pipe": "staged"})):
+            p = ll.ll_plan_convert(A, B, w, **o, **extra)
+            p.prepare()
+            ms = time_fn(lambda: ll.ll_convert(src, dst, p))
+            same = ref is None or bool(torch.equal(ref, dst))
+            if ref is None:
+                ref = dst.clone()
+            gbs = 4 * n / ms / 1e6
+            print(json.dumps({"case": name, "variant": var, "staged": p.describe()["tile"].get("staged"),
+                              "same_bytes": same, "ms": round(ms, 4), "GBps": round(gbs, 1),
+                              "frac_6539": round(gbs / 6539.5, 3)}), flush=True)
+        del src, dst, ref
 
 
 def swizzle_case():
