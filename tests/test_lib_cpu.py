@@ -844,3 +844,24 @@ def test_opts_struct_matches_the_c_abi():
     assert any(b != 0xAB for b in buf[n - 8:n])        # the last fields were written
     o = ll._Opts.from_buffer(buf)
     assert o.force_class == -1 and o.max_vec_bytes == 16 and o.pipe == 0 and o.min_blocks == 0
+
+
+def test_planned_wavefronts_equal_ncu_sass_counts():
+    """the planner's predicted shared-memory wavefronts per tile (Lemma 9.4
+    model) times the tiles of the launch equal the SASS-attributed wavefronts
+    ncu counted on the B200 for the same plans (committed capture
+    profiles/r01_smem_sass_wavefronts.json, tools/jobs/job59.sh), for every smem-exchange
+    kernel captured — and both equal the conflict-free ideal (bytes / 128)."""
+    import json
+    path = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles",
+                        "r01_smem_sass_wavefronts.json")
+    m = json.load(open(path))["cases"]
+    cases = {"c3": (W.c3(14), 2, {}), "c3b": (W.c3b(14), 2, {}), "c5T": (W.c5T(0, n=15), 2, {}),
+             "n1": (W.n1_preshuffle(14, 14), 2, {}), "c1bsmem": (W.c1_batched(20), 4, {"force_class": "SMEM"}),
+             "c2smem": (W.c2(16), 2, {"force_class": "SMEM"}), "c3f": (W.c3(14), 2, {"sigma": "faithful"})}
+    assert sorted(cases) == sorted(m)
+    for k, ((sa, sb), w, o) in cases.items():
+        t = ll.ll_plan_convert(ll.Layout.from_spec(sa), ll.Layout.from_spec(sb), w, **o).describe()["tile"]
+        nt = t["ctas"]
+        assert t["wavefronts_st"] * nt == m[k]["st"]["sass_wavefronts"] == m[k]["st"]["ideal_wavefronts"], k
+        assert t["wavefronts_ld"] * nt == m[k]["ld"]["sass_wavefronts"] == m[k]["ld"]["ideal_wavefronts"], k
