@@ -865,3 +865,20 @@ def test_planned_wavefronts_equal_ncu_sass_counts():
         nt = t["ctas"]
         assert t["wavefronts_st"] * nt == m[k]["st"]["sass_wavefronts"] == m[k]["st"]["ideal_wavefronts"], k
         assert t["wavefronts_ld"] * nt == m[k]["ld"]["sass_wavefronts"] == m[k]["ld"]["ideal_wavefronts"], k
+
+
+def test_ncu_dram_traffic_within_algorithmic_bytes():
+    """DRAM read + write bytes per launch that ncu measured for every bench
+    kernel (profiles/ncu_traffic.json, the `roofline.traffic` source) stay within 1.05x of
+    the algorithmic bytes (each element read once and written once; gather: src + idx +
+    dst; reduce: src + dst) — no wasted re-reads."""
+    import json
+    path = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles", "ncu_traffic.json")
+    t = json.load(open(path))
+    GiB, MiB = 1 << 30, 1 << 20
+    algo = {"c2_shuffle": 4 * GiB, "c3": 2 * GiB, "c3b": 2 * GiB, "c1b": 2 * GiB, "c5T": 4 * GiB,
+            "n1": GiB, "n2": GiB, "c5_peer_one_rank": 512 * MiB,   # P = 8: one rank moves 256 MiB in + out
+            "gather_mma": 192 * MiB, "gather_blocked": 192 * MiB,
+            "reduce_mma": 64 * MiB + MiB // 2, "reduce_blocked": 64 * MiB + MiB // 2}
+    for k, a in algo.items():
+        assert t[k] <= 1.05 * a, (k, t[k], a)
