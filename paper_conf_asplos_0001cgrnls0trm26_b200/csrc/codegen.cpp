@@ -68,6 +68,11 @@ std::string codegen_tile(const ConvPlan& Pl) {
   o << icon("ST_HINT", st_hint());
   o << "  static constexpr bool PIPE = " << (T.pipe ? "true" : "false") << ";\n";
   o << "  static constexpr bool STAGED = " << (T.staged ? "true" : "false") << ";\n";
+  {
+    const char* nh = std::getenv("LL_NOHOIST");   // experiment hook: 0 / 1 override
+    const bool nohoist = nh ? std::string(nh) == "1" : T.ld_run >= 0;
+    o << "  static constexpr bool NOHOIST = " << (nohoist ? "true" : "false") << ";\n";
+  }
   o << icon("XBYTES", (long long)(T.smem_elems * u64(T.w)));
   // per-thread-contiguous loads (faithful σ) re-use sectors across instructions
   o << "  static constexpr bool LD_L1 = " << (T.sigma == SIGMA_FAITHFUL ? "true" : "false") << ";\n";

@@ -400,7 +400,11 @@ template <class P>
 __device__ __forceinline__ void smem_write(const u32 (&r)[P::NW], u32 lane, u32 warp, u32 sbase) {
   constexpr int VE = 1 << P::SV;
   constexpr int VW = (P::W * VE + 3) / 4;
-  const u32 tst = smem_thread_base<P, true>(lane, warp);
+  u32 tst = smem_thread_base<P, true>(lane, warp);
+  // NOHOIST (linear tiles): an opaque copy per call keeps the 2^R XOR-combined smem
+  // addresses out of the tile loop — hoisted as loop invariants they outgrow the register
+  // file and spill (measured: 255 registers + local-memory stack)
+  if constexpr (P::NOHOIST) asm volatile("" : "+r"(tst));
   static_for<(1 << (P::R - P::SV))>([&](auto k) {
     constexpr int K = decltype(k)::value;
     u32 v[VW > 0 ? VW : 1];
@@ -418,7 +422,8 @@ template <class P>
 __device__ __forceinline__ void smem_read(u32 (&o)[P::NW], u32 lane, u32 warp, u32 sbase) {
   constexpr int VE = 1 << P::SV;
   constexpr int VW = (P::W * VE + 3) / 4;
-  const u32 tld = smem_thread_base<P, false>(lane, warp);
+  u32 tld = smem_thread_base<P, false>(lane, warp);
+  if constexpr (P::NOHOIST) asm volatile("" : "+r"(tld));
   static_for<(1 << (P::R - P::SV))>([&](auto k) {
     constexpr int K = decltype(k)::value;
     u32 v[VW > 0 ? VW : 1];
@@ -679,7 +684,9 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, Dst D, 
     });
   }
   auto load_tile = [&](u32 (&r)[P::NW], u64 t) {
-    const u64 sofs = tile_base<P, true>(t) ^ ld_thr;
+    u64 thr = ld_thr;
+    if constexpr (P::NOHOIST) asm volatile("" : "+l"(thr));   // keep per-vector addresses in the loop
+    const u64 sofs = tile_base<P, true>(t) ^ thr;
     const u8* s = src + sofs;
     u32 lo = lo_thr;
     if constexpr (P::LD_INVEC) {
@@ -702,7 +709,9 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, Dst D, 
   };
   // a10: HBM store of a dst tile (and of its broadcast replicas)
   auto store_tile = [&](const u32 (&o)[P::NW], u64 t) {
-    const u64 doff = tile_base<P, false>(t | tile0) ^ st_thr;
+    u64 thr = st_thr;
+    if constexpr (P::NOHOIST) asm volatile("" : "+l"(thr));
+    const u64 doff = tile_base<P, false>(t | tile0) ^ thr;
     u8* d = D.at(doff);
     static_for<P::NREP>([&](auto rp) {
       constexpr u64 RO = P::REP_OFF[decltype(rp)::value];
