@@ -119,15 +119,15 @@ typedef struct {
                          * widens the swizzle's vector; 1 = vectorised ld/st.shared only;
                          * 2 = prefer stmatrix / ldmatrix wherever their tile divides   */
   int reduce_op;        /* ll_plan_reduce: 0 = sum (default), 1 = max, 2 = min (fp32)   */
-  int pipe;             /* smem-exchange tiles: 0 = auto (pipelined for linear tiles
-                         * only), 1 = off, 2 = software-pipelined (next tile's loads
+  int pipe;             /* smem-exchange tiles: 0 = auto (= off), 1 = off,
+                         * 2 = software-pipelined (next tile's loads
                          * before this tile's smem reads and HBM stores), 3 = staged
                          * (the next two tiles' 16-byte src vectors streamed by
                          * cp.async into two raw smem stages; persistent grid; needs
                          * 16-byte load vectors and exchange + 2 tiles <= 227 KiB)   */
   int min_blocks;       /* tile kernels: resident CTAs per SM requested from ptxas
-                         * (__launch_bounds__ minimum): 0 = auto (2 for linear tiles of
-                         * >= 4-byte elements, else none), -1 = none, k >= 1 = k      */
+                         * (__launch_bounds__ minimum): 0 = auto (2 for linear tiles,
+                         * else none), -1 = none, k >= 1 = k                          */
 } ll_plan_opts;
 
 /* Fill *opts with defaults (force_class = -1, max_vec_bytes = 16, ...). */

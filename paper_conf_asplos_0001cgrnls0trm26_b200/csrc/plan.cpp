@@ -733,13 +733,14 @@ static void plan_exchange(ConvPlan& P, const ll_plan_opts* opts) {
   if (T.xchg == X_SMEM) {
     // software-pipelined smem exchange (next tile's loads before this tile's stores):
     // measured slower on every default-sized config — the second register buffer costs
-    // occupancy (profiles/r01_sweep_smem_pipeline.jsonl) — so only on request (LL_PIPE=1),
-    // except for linear tiles (ld_run set): their XOR-addressed 64 KiB tiles run one CTA
-    // per SM, whose load and store phases otherwise serialise; pipelined they measured
-    // 1.0-1.29x on random R2 maps (profiles/r01_sweep_linear_pipe.jsonl; LL_PIPE=0 off)
+    // occupancy (profiles/r01_sweep_smem_pipeline.jsonl) — so only on request (pipe = 2,
+    // LL_PIPE=1).  Linear tiles first took it by default (one CTA per SM: 1.0-1.29x,
+    // profiles/r01_sweep_linear_pipe.jsonl); with their addresses kept out of the tile
+    // loop (NOHOIST) two unpipelined CTAs per SM measured better on average (mean 0.87 vs
+    // 0.82 of copy over six random R2 maps, profiles/r01_sweep_linear_nohoist.jsonl)
     const char* e = std::getenv("LL_PIPE");
     const int op = opts ? opts->pipe : 0;
-    T.pipe = e ? std::string(e) == "1" : (op == 2 || (op == 0 && T.ld_run >= 0));
+    T.pipe = e ? std::string(e) == "1" : op == 2;
     // staged (pipe = 3 / LL_PIPE=staged): cp.async double-buffered src stages; needs
     // 16-byte load vectors and room for the exchange buffer plus two raw tiles
     const bool want_staged = e ? std::string(e) == "staged" : op == 3;
@@ -749,17 +750,17 @@ static void plan_exchange(ConvPlan& P, const ll_plan_opts* opts) {
       T.pipe = false;
     }
   }
-  // Resident CTAs per SM (ptxas register cap).  Linear tiles compile to 170-255
+  // Resident CTAs per SM (ptxas register cap).  Linear tiles compile to 140-255
   // registers (XOR addresses that cannot fold into immediates), i.e. one CTA per SM;
-  // asking for 2 trades registers for a few spills.  Measured on random R2 maps: 4-byte
-  // elements 1.0-1.21x (two of three maps), 2-byte elements slower (b16 smem traffic
-  // spills more), profiles/r01_sweep_linear_minblocks.jsonl; ll_plan_autotune times both.
+  // asking for 2 trades registers for a few spills: with NOHOIST 1.07-2.2x over one
+  // uncapped CTA on five of six random R2 maps (profiles/r01_sweep_linear_nohoist.jsonl);
+  // ll_plan_autotune times both.
   {
     const char* e = std::getenv("LL_MIN_BLOCKS");
     const int om = opts ? opts->min_blocks : 0;
     if (e) T.min_blocks = std::max(0, std::atoi(e));
     else if (om > 0) T.min_blocks = om;
-    else if (om == 0 && T.ld_run >= 0 && T.xchg == X_SMEM && T.w >= 4 && !T.staged) T.min_blocks = 2;
+    else if (om == 0 && T.ld_run >= 0 && T.xchg == X_SMEM && !T.staged) T.min_blocks = 2;
     else T.min_blocks = 0;
   }
   if (T.xchg == X_SMEM && (T.smem_elems * u64(T.w)) > 200 * 1024)

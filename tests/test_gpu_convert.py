@@ -744,7 +744,7 @@ def test_gather_axis_over_warps_smem():
 @pytest.mark.parametrize("pipe", ["0", "1"])
 def test_smem_pipeline_both_ways_gpu(monkeypatch, pipe, grid_per_sm):
     """The software-pipelined smem exchange (next tile's loads before this tile's smem
-    reads and stores; default for linear tiles, LL_PIPE=1 elsewhere) and the plain one
+    reads and stores; pipe = "on" / LL_PIPE=1) and the plain one
     are both bit-exact against the oracle: config 3, config 1-batch (smem forced) and
     random R2 memory layouts planned as linear tiles.  LL_GRID_PER_SM=1 caps the grid at
     one CTA per SM, so every CTA loops over several tiles (the pipelined path's

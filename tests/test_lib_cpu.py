@@ -789,12 +789,17 @@ def test_linear_tile_run_choice_simulated(monkeypatch, balance):
         assert shorter > 0
 
 
-def test_linear_tiles_pipelined_by_default(monkeypatch):
-    """Without LL_PIPE, linear-tile plans (random R2 memory layouts) take the pipelined
-    smem exchange and other smem plans (config 3) do not."""
+def test_linear_tiles_default_exchange(monkeypatch):
+    """Without LL_PIPE / LL_MIN_BLOCKS, linear-tile plans (random R2 memory layouts) take
+    the unpipelined smem exchange with two CTAs per SM (register cap) and opaque thread
+    bases (NOHOIST); config 3 keeps the plain kernel."""
+    monkeypatch.delenv("LL_MIN_BLOCKS", raising=False)
+    monkeypatch.delenv("LL_NOHOIST", raising=False)
     monkeypatch.delenv("LL_PIPE", raising=False)
     A, B = (ll.Layout.from_spec(x) for x in W.c3(9))
-    assert ll.ll_plan_convert(A, B, 2).describe()["tile"]["pipe"] is False
+    p = ll.ll_plan_convert(A, B, 2)
+    assert p.describe()["tile"]["pipe"] is False and p.describe()["tile"]["min_blocks"] == 0
+    assert "NOHOIST = false" in p.source()
     rng = np.random.default_rng(801)
     seen = 0
     for _ in range(6):
@@ -804,26 +809,27 @@ def test_linear_tiles_pipelined_by_default(monkeypatch):
         t = ll.ll_plan_convert(ll.Layout(ins, out, {"offset": [(c,) for c in ca]}),
                                ll.Layout(ins, out, {"offset": [(c,) for c in cb]}), 4).describe()
         if t["exec"] == "tile" and t["tile"].get("linear_tile") and t["tile"]["xchg"] == "smem":
-            assert t["tile"]["pipe"] is True
+            assert t["tile"]["pipe"] is False and t["tile"]["min_blocks"] == 2
             seen += 1
     assert seen >= 1
 
 
 def test_plan_opts_pipe_and_min_blocks():
     """ll_plan_opts.pipe / min_blocks reach the plan (describe) and the generated kernel
-    (__launch_bounds__ minimum): auto = pipelined linear tiles, with two CTAs per SM for
-    >= 4-byte elements; explicit values override; other smem plans stay unpipelined."""
+    (__launch_bounds__ minimum): auto = linear tiles unpipelined with two CTAs per SM;
+    explicit values override; other smem plans keep the plain kernel."""
     rng = np.random.default_rng(9)
     d = 16
     ca, cb = gen.random_memory_cols(rng, d), gen.random_memory_cols(rng, d)
     ins, out = [("offset", d)], [("x", d)]
     A = ll.Layout(ins, out, {"offset": [(c,) for c in ca]})
     B = ll.Layout(ins, out, {"offset": [(c,) for c in cb]})
-    for w, mb_auto in ((2, 0), (4, 2)):
+    for w, mb_auto in ((2, 2), (4, 2)):
         p = ll.ll_plan_convert(A, B, w)
         t = p.describe()["tile"]
-        assert t["linear_tile"] and t["pipe"] is True and t["min_blocks"] == mb_auto
-        assert (", 2)" in p.source()) == (mb_auto == 2)
+        assert t["linear_tile"] and t["pipe"] is False and t["min_blocks"] == mb_auto
+        assert (", 2)" in p.source()) == (mb_auto == 2) and "NOHOIST = true" in p.source()
+        assert ll.ll_plan_convert(A, B, w, pipe="on").describe()["tile"]["pipe"] is True
         t = ll.ll_plan_convert(A, B, w, pipe="off", min_blocks=-1).describe()["tile"]
         assert t["pipe"] is False and t["min_blocks"] == 0
         p = ll.ll_plan_convert(A, B, w, min_blocks=3)
