@@ -44,6 +44,8 @@
  *  - LL_JIT_CACHE=<dir>: the NVRTC cubin cache (default: in-tree .ll_jit_cache/).
  *  - LL_PDL=0: launch without programmatic dependent launch.
  *  - LL_PIPE=0|1|staged, LL_MIN_BLOCKS=k: override ll_plan_opts.pipe / min_blocks.
+ *  - LL_NOHOIST=0|1: opaque thread bases in tile kernels (keeps XOR-combined addresses
+ *    inside the tile loop; default on for linear tiles only).
  *  - LL_LINEAR_BALANCE=0: linear CTA tiles (general invertible pull maps) take the
  *    widest store runs instead of the default balanced load/store run lengths.
  *  Host entry points (planning, launches) are wrapped in NVTX ranges named after
