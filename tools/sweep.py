@@ -217,6 +217,8 @@ def linear_thread_bytes():
                         ("pipe, 2 CTAs/SM", {"pipe": "on", "min_blocks": 2}),
                         ("no pipe, 2 CTAs/SM", {"pipe": "off", "min_blocks": 2}),
                         ("staged (cp.async)", {"pipe": "staged", "min_blocks": -1}), ("autotune", None)]
+            if os.environ.get("LL_SWEEP_TB"):
+                variants = [(f"thread_bytes {tb}", {"thread_bytes": tb}) for tb in (0, 64, 128, 512)]
             if os.environ.get("LL_SWEEP_MAXTILE"):
                 variants = [(f"max tile {mt}, {n}", dict(o, tile_bytes=mt)) for mt in (65536, 32768, 131072)
                             for n, o in (("auto", {}), ("2 CTAs/SM", {"min_blocks": 2}), ("no cap", {"min_blocks": -1}))]
