@@ -248,6 +248,14 @@ ll_status ll_plan_convert(const ll_layout* A, const ll_layout* B, int elem_bytes
 ll_status ll_plan_class(const ll_plan* plan, ll_class* cls);
 /* Workspace needed by ll_convert (> 0 only for DEVICE plans). */
 ll_status ll_plan_workspace_bytes(const ll_plan* plan, size_t* bytes);
+/* Bytes of each caller buffer the plan's execution call reads or writes (this rank's
+ * slice for DEVICE plans): src and dst of ll_convert / ll_gather / ll_reduce / ll_scan
+ * (2^{d_in} elements of the layout, §8(b) storage convention; ll_reduce's dst is
+ * ll_plan_reduce_out_elems floats) and the int32 idx of ll_gather (0 for other kinds).
+ * The execution calls take bare pointers: callers (the Python binding) check their
+ * buffers against these sizes before launching.  Any out pointer may be NULL.
+ * Errors: INVALID_ARG (null plan). */
+ll_status ll_plan_buffer_bytes(const ll_plan* plan, size_t* src_bytes, size_t* dst_bytes, size_t* idx_bytes);
 /* JSON description: class, executed exchange, V/I/E/F/G/R, swizzle columns,
  * rounds, predicted wavefronts, the smem instruction of each side (Thm 5.1:
  * "smem_store" / "smem_load", e.g. "stmatrix.m8n8.x4.b16", "ld.shared.v4.b32") and

@@ -911,51 +911,33 @@ def reduce_ref_fp64(L: Layout, axis: int, src: np.ndarray, op: str = "sum") -> n
 
 
 def reduce_fixed_order_fp32(L: Layout, axis: int, src: np.ndarray) -> np.ndarray:
-    """The fixed-order fp32 replica: over the axis hardware bits of
-    L whose column is non-zero and lies on the axis, ordered reg, lane, warp
-    (ascending within each), do v ← v(b=0) + v(b=1) in fp32 round-to-nearest;
-    zero-column (broadcast) bits are dropped, not summed."""
-    order = []
-    zero_bits = []
+    """The fixed-order fp32 replica (the paper fixes no order, so the
+    order is reading R-reduce), in LOGICAL coordinates: with the in-tile
+    axis coordinate a in [0, K) (the low K bits of the axis, as for O10), for
+    t = 0, 1, ..., log2 K - 1 in ascending order combine the pairs that differ only in
+    bit t of a,  v <- v(t = 0) + v(t = 1)  (fp32, round to nearest, no FMA) — i.e. the
+    recursive halving (pairwise) sum  S(x) = S(x[:K/2]) + S(x[K/2:]).  The result is a
+    function of the logical tensor alone: it does not depend on how L places the bits
+    on registers, lanes or warps, and broadcast (zero-column) copies of L
+    contribute once.  Output: the logical tensor with the axis replaced by its block
+    part, row-major (as reduce_ref_fp64)."""
+    shape = [1 << b for _, b in L.out_dims]
+    x_of_h = image_table(L).astype(np.int64)
+    T = np.empty(int(np.prod(shape)), dtype=np.float32)
+    T[x_of_h] = np.asarray(src, dtype=np.float32).reshape(-1)
     axis_shift = sum(b for _, b in L.out_dims[axis + 1:])
     axis_mask = ((1 << L.out_dims[axis][1]) - 1) << axis_shift
-    for name in ("reg", "lane", "warp"):
-        for k in L.dim_bits(name):
-            if L.cols[k] == 0:
-                zero_bits.append(k)
-            elif L.cols[k] & axis_mask:
-                order.append(k)
-    for name in ("block", "dev"):
-        for k in L.dim_bits(name):
-            if L.cols[k] == 0:
-                zero_bits.append(k)
-    vals = np.asarray(src, dtype=np.float32).reshape(-1).copy()
-    hs = np.arange(vals.size, dtype=np.int64)
-    alive = np.ones(vals.size, dtype=bool)
-    for k in zero_bits:                       # keep only the copy with bit k = 0
-        alive &= ((hs >> k) & 1) == 0
-    acc = vals
-    for k in order:
-        lo = alive & (((hs >> k) & 1) == 0)
-        partner = hs ^ (1 << k)
-        new = acc.copy()
-        new[lo] = (acc[lo] + acc[partner[lo]]).astype(np.float32)
-        acc = new
-        alive = lo
-    # surviving h: all reduced bits 0; map to the output coordinate
-    x_of_h = apply_all(L, hs.astype(np.uint64)).astype(np.int64)
-    shape = [1 << b for _, b in L.out_dims]
     nonblock = [k for n, _ in L.in_dims if n not in ("block", "dev") for k in L.dim_bits(n)]
-    K = 1 << len([k for k in nonblock if L.cols[k] & axis_mask])
-    out = np.empty(int(np.prod(shape)) // K, dtype=np.float32)
-    xs = x_of_h[alive]
-    a = (xs & axis_mask) >> axis_shift
-    lower = xs & ((1 << axis_shift) - 1)
-    upper = xs >> (axis_shift + L.out_dims[axis][1])
-    na = shape[axis] // K
-    yo = (upper * na + (a // K)) * (1 << axis_shift) + lower
-    out[yo] = acc[alive]
-    return out
+    kbits = len([k for k in nonblock if L.cols[k] & axis_mask])
+    K = 1 << kbits
+    # [outer, tiles along the axis, K, inner]: the in-tile axis coordinate is axis 2
+    v = T.reshape(int(np.prod(shape[:axis], dtype=np.int64)), shape[axis] // K, K,
+                  int(np.prod(shape[axis + 1:], dtype=np.int64)))
+    for t in range(kbits):
+        # after t steps, position q of axis 2 holds the sum over the aligned block of
+        # 2^t original positions q*2^t ...; bit t of a is now the lowest bit of q
+        v = (v[:, :, 0::2, :] + v[:, :, 1::2, :]).astype(np.float32)
+    return v.reshape(-1)
 
 
 # --------------------------------------------------------------------------------------

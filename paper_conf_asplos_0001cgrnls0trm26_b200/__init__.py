@@ -78,6 +78,7 @@ _sig = {
     "ll_plan_convert": [_P, _P, C.c_int, C.POINTER(_Opts), _PP],
     "ll_plan_class": [_P, C.POINTER(C.c_int)],
     "ll_plan_workspace_bytes": [_P, C.POINTER(C.c_size_t)],
+    "ll_plan_buffer_bytes": [_P] + [C.POINTER(C.c_size_t)] * 3,
     "ll_plan_describe": [_P, C.c_char_p, C.c_size_t],
     "ll_plan_source": [_P, C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t)],
     "ll_plan_prepare": [_P],
@@ -405,6 +406,28 @@ class Plan:
         _check(_lib.ll_plan_source(self.handle, buf, len(buf), C.byref(n)))
         return buf.value.decode()
 
+    def buffer_bytes(self):
+        """(src, dst, idx) bytes the execution call touches (ll_plan_buffer_bytes)."""
+        a, b, c = C.c_size_t(), C.c_size_t(), C.c_size_t()
+        _check(_lib.ll_plan_buffer_bytes(self.handle, C.byref(a), C.byref(b), C.byref(c)))
+        return a.value, b.value, c.value
+
+    def check_buffers(self, src=None, dst=None, idx=None, workspace=None):
+        """Raise LLError when a torch tensor is smaller than the plan's buffer (raw
+        pointers cannot be checked and pass through)."""
+        need = dict(zip(("src", "dst", "idx"), self.buffer_bytes()))
+        need["workspace"] = self.workspace_bytes() if self.kind == "convert" else 0
+        for name, t in (("src", src), ("dst", dst), ("idx", idx), ("workspace", workspace)):
+            if t is None or isinstance(t, int) or not hasattr(t, "numel"):
+                if name == "workspace" and t is None and need[name] > 0:
+                    raise LLError(1, f"{name}: the plan needs {need[name]} bytes of workspace")
+                continue
+            have = t.numel() * t.element_size()
+            if have < need[name]:
+                raise LLError(1, f"{name}: {have} bytes < the plan's {need[name]} bytes")
+            if not t.is_contiguous():
+                raise LLError(1, f"{name}: tensor must be contiguous")
+
     def workspace_bytes(self) -> int:
         n = C.c_size_t()
         _check(_lib.ll_plan_workspace_bytes(self.handle, C.byref(n)))
@@ -563,6 +586,7 @@ def ll_plan_autotune(A: Layout, B: Layout, elem_bytes: int, src, dst, stream=Non
 
 def ll_convert(src, dst, plan: Plan, stream=None, workspace=None):
     """dst <- convert(src) on `stream` (torch CUDA tensors or raw device pointers)."""
+    plan.check_buffers(src, dst, workspace=workspace)
     _check(_lib.ll_convert(_ptr(src), _ptr(dst), _ptr(workspace), plan.handle, _stream_ptr(stream)))
 
 
@@ -583,6 +607,7 @@ def ll_plan_gather(L: Layout, axis: int, elem_bytes: int, **opts) -> Plan:
 
 
 def ll_gather(src, idx, dst, plan: Plan, stream=None):
+    plan.check_buffers(src, dst, idx)
     _check(_lib.ll_gather(_ptr(src), _ptr(idx), _ptr(dst), plan.handle, _stream_ptr(stream)))
 
 
@@ -601,8 +626,10 @@ def ll_plan_scan(L: Layout, axis: int, **opts) -> Plan:
 
 
 def ll_scan(src, dst, plan: Plan, stream=None):
+    plan.check_buffers(src, dst)
     _check(_lib.ll_scan(_ptr(src), _ptr(dst), plan.handle, _stream_ptr(stream)))
 
 
 def ll_reduce(src, dst, plan: Plan, stream=None):
+    plan.check_buffers(src, dst)
     _check(_lib.ll_reduce(_ptr(src), _ptr(dst), plan.handle, _stream_ptr(stream)))

@@ -434,12 +434,24 @@ ll_status ll_layout_slice(const ll_layout* L, int dim, ll_layout** out) {
   LL_CATCH
 }
 
+namespace {
+// Plan options shared by every planner: the vector bound must be a power of two in
+// [1, 16] bytes (0 = default 16) — wider vectors have no ld/st instruction.
+void validate_opts(const ll_plan_opts* o) {
+  if (!o) return;
+  const int v = o->max_vec_bytes;
+  if (v < 0 || v > 16 || (v & (v - 1)) != 0)
+    ll::fail(LL_ERR_INVALID_ARG, "max_vec_bytes must be 0 (default 16) or a power of two in [1, 16]");
+}
+}  // namespace
+
 ll_status ll_plan_convert(const ll_layout* A, const ll_layout* B, int w, const ll_plan_opts* opts_in, ll_plan** plan) {
   LL_TRY
   NvtxRange nvtx("ll_plan_convert");
   if (!A || !B || !plan) fail(LL_ERR_INVALID_ARG, "null argument");
   ll_plan_opts opts_env;
   const ll_plan_opts* opts = env_opts(opts_in, opts_env);
+  validate_opts(opts);
   auto h = std::make_unique<ll_plan>();
   h->kind = 0;
   if (w == 8) {
@@ -487,6 +499,35 @@ ll_status ll_plan_workspace_bytes(const ll_plan* p, size_t* bytes) {
   LL_CATCH
 }
 
+ll_status ll_plan_buffer_bytes(const ll_plan* p, size_t* src_bytes, size_t* dst_bytes, size_t* idx_bytes) {
+  LL_TRY
+  if (!p) fail(LL_ERR_INVALID_ARG, "null argument");
+  auto local_bits = [](const Layout& L) {
+    int n = 0;
+    for (auto& d : L.in) if (d.name != "dev") n += d.bits;
+    return n;
+  };
+  size_t s = 0, d = 0, i = 0;
+  if (p->kind == 0) {
+    const ConvPlan& P = p->cp();
+    s = (size_t(1) << local_bits(P.A)) * size_t(P.w);
+    d = (size_t(1) << local_bits(P.B)) * size_t(P.w);
+  } else if (p->kind == 1) {
+    const GatherPlan& G = *p->gather;
+    s = d = (size_t(1) << local_bits(G.L)) * size_t(G.w);
+    i = (size_t(1) << local_bits(G.L)) * 4;
+  } else if (p->kind == 2) {
+    s = (size_t(1) << local_bits(p->reduce->L)) * 4;
+    d = size_t(p->reduce->out_elems) * 4;
+  } else {
+    s = d = (size_t(1) << local_bits(p->scan->L)) * 4;
+  }
+  if (src_bytes) *src_bytes = s;
+  if (dst_bytes) *dst_bytes = d;
+  if (idx_bytes) *idx_bytes = i;
+  LL_CATCH
+}
+
 ll_status ll_plan_describe(const ll_plan* p, char* json, size_t cap) {
   LL_TRY
   if (!p || !json || !cap) fail(LL_ERR_INVALID_ARG, "null argument");
@@ -520,6 +561,9 @@ ll_status ll_plan_describe(const ll_plan* p, char* json, size_t cap) {
     o << "{\"kind\":\"reduce\",\"op\":\"" << opn[Rp.op] << "\",\"R\":" << Rp.R << ",\"warp_bits\":" << Rp.Wb << ",\"tree_levels\":" << Rp.red_reg.size()
       << ",\"bfly_stages\":" << Rp.red_lane.size() << ",\"warp_stages\":" << Rp.red_warp.size()
       << ",\"dup_bits\":" << Rp.dup_bits.size() << ",\"out_elems\":" << Rp.out_elems
+      << ",\"axis_hw\":[";
+    for (size_t t = 0; t < Rp.axis_hw.size(); ++t) o << (t ? "," : "") << Rp.axis_hw[t];
+    o << "],\"shuffles_per_thread\":" << Rp.shfl_per_thread
       << ",\"tma\":" << (Rp.tma ? "true" : "false") << ",\"stages\":" << Rp.stages << ",\"sigma\":\"" << (Rp.sigma ? "faithful" : "coalesced") << "\""
       << ",\"ctas\":" << (u64(1) << Rp.grid_bit.size()) << "}";
     s = o.str();
@@ -765,6 +809,7 @@ ll_status ll_plan_gather(const ll_layout* L, int axis, int w, const ll_plan_opts
   LL_TRY
   if (!L || !plan) fail(LL_ERR_INVALID_ARG, "null argument");
   if (w == 8) fail(LL_ERR_UNSUPPORTED, "gather: elem_bytes 8 not supported");
+  validate_opts(opts);
   auto h = std::make_unique<ll_plan>();
   h->kind = 1;
   h->gather = plan_gather(L->L, axis, w, opts);
@@ -797,6 +842,7 @@ ll_status ll_gather(const void* src, const int32_t* idx, void* dst, const ll_pla
 ll_status ll_plan_scan(const ll_layout* L, int axis, const ll_plan_opts* opts, ll_plan** plan) {
   LL_TRY
   if (!L || !plan) fail(LL_ERR_INVALID_ARG, "null argument");
+  validate_opts(opts);
   auto h = std::make_unique<ll_plan>();
   h->kind = 3;
   h->scan = plan_scan(L->L, axis, opts);
@@ -826,6 +872,7 @@ ll_status ll_scan(const float* src, float* dst, const ll_plan* p, void* stream) 
 ll_status ll_plan_reduce(const ll_layout* L, int axis, const ll_plan_opts* opts, ll_plan** plan) {
   LL_TRY
   if (!L || !plan) fail(LL_ERR_INVALID_ARG, "null argument");
+  validate_opts(opts);
   auto h = std::make_unique<ll_plan>();
   h->kind = 2;
   h->reduce = plan_reduce(L->L, axis, opts);

@@ -234,25 +234,20 @@ std::string codegen_reduce(const ReducePlan& Rp) {
   emit_grid(o, Rp.grid_bit, Rp.grid_bit, 2);
   o << arr("u64", "GRID_OUT", Rp.grid_out) << arr("u64", "OUT_COL", Rp.out_col);
   int regmask = 0, dupreg = 0;
-  uint32_t nolane = 0, nowarp = 0, rwmask = 0;
+  uint32_t nolane = 0, nowarp = 0;
   for (int b : Rp.red_reg) regmask |= 1 << b;
   for (int b : Rp.red_lane) nolane |= 1u << b;
-  for (int b : Rp.red_warp) { nowarp |= 1u << b; rwmask |= 1u << b; }
+  for (int b : Rp.red_warp) nowarp |= 1u << b;
   for (int k : Rp.dup_bits) {
     if (k < R) dupreg |= 1 << k;
     else if (k < R + 5) nolane |= 1u << (k - R);
     else nowarp |= 1u << (k - R - 5);
   }
-  o << icon("NRED_REG", Rp.red_reg.size()) << arr("int", "RED_REG", Rp.red_reg) << icon("RED_REG_MASK", regmask)
-    << icon("DUP_REG_MASK", dupreg) << icon("NRED_LANE", Rp.red_lane.size()) << arr("int", "RED_LANE", Rp.red_lane)
-    << icon("NRED_WARP", Rp.red_warp.size()) << arr("int", "RED_WARP", Rp.red_warp);
+  o << icon("RED_REG_MASK", regmask) << icon("DUP_REG_MASK", dupreg)
+    << icon("KB", Rp.axis_hw.size()) << arr("int", "AXIS_HW", Rp.axis_hw);
   o << "  static constexpr u32 NOSTORE_LANE_MASK = " << nolane << "u;\n"
-    << "  static constexpr u32 NOSTORE_WARP_MASK = " << nowarp << "u;\n"
-    << "  static constexpr u32 RED_WARP_MASK = " << rwmask << "u;\n";
-  o << "  template <int I> static constexpr int done_mask() { int m = 0; for (int j = 0; j < I; ++j) m |= 1 << RED_REG[j]; return m; }\n";
+    << "  static constexpr u32 NOSTORE_WARP_MASK = " << nowarp << "u;\n";
   o << "  template <int E> static constexpr u64 out_of_slot() { u64 c = 0; for (int b = 0; b < R; ++b) if ((E >> b) & 1) c ^= OUT_COL[b]; return c; }\n";
-  o << "  template <int E> static constexpr int live_index() { int k = 0, t = 0;"
-       " for (int b = 0; b < R; ++b) { if ((RED_REG_MASK | DUP_REG_MASK) & (1 << b)) continue; if ((E >> b) & 1) k |= 1 << t; ++t; } return k; }\n";
   o << "};\n";
   o << "extern \"C\" __global__ void __launch_bounds__(" << (32 << Rp.Wb)
     << ") ll_reduce_kernel(const float* __restrict__ src, float* __restrict__ dst, u64 ntiles) {\n"

@@ -10,6 +10,8 @@
 #include <cstdlib>
 #include <fstream>
 #include <sstream>
+#include <mutex>
+#include <thread>
 #include <unordered_map>
 
 #include "ll_internal.hpp"
@@ -106,12 +108,20 @@ std::string cubin_for(const std::string& full, const char* name, std::string* ke
     if (!s.empty()) return s;
   }
   std::string cubin = compile(full, name);
-  std::string tmp = path + ".tmp" + std::to_string(getpid());
+  // unique temp name per process and thread; a failed write (full disk) is not renamed
+  // into the cache, the cubin in memory is still used
+  std::ostringstream tn;
+  tn << path << ".tmp" << getpid() << "." << std::this_thread::get_id();
+  const std::string tmp = tn.str();
+  bool ok;
   {
     std::ofstream f(tmp, std::ios::binary);
     f.write(cubin.data(), std::streamsize(cubin.size()));
+    f.flush();
+    ok = f.good();
   }
-  rename(tmp.c_str(), path.c_str());
+  if (ok) rename(tmp.c_str(), path.c_str());
+  else std::remove(tmp.c_str());
   // keep the source beside it (ncu source view / inspection)
   std::ofstream(cache_dir() + "/" + key + ".cu") << full;
   return cubin;
@@ -121,6 +131,7 @@ std::string cubin_for(const std::string& full, const char* name, std::string* ke
 const char* kernel_template() { return kTemplate; }
 
 std::string jit_precompile(const std::string& plan_src, const char* name) {
+  std::lock_guard<std::mutex> g(g_mu);
   std::string key;
   cubin_for(full_source(plan_src), name, &key);
   return key;

@@ -279,8 +279,11 @@ struct ReducePlan {
   int R = 0, Wb = 0, v = 0;
   std::vector<int> hw_bit;        // kernel bit -> packed bit of L (σ)
   std::vector<int> grid_bit;      // CTA index bit -> packed bit (non-duplicate block bits)
-  // reduced kernel bits, each list ascending: the fixed order is reg, lane, warp
+  // reduced kernel bits per level (ascending); the steps run in logical axis bit order:
+  // axis_hw[t] = the kernel bit holding in-tile axis bit t
   std::vector<int> red_reg, red_lane, red_warp;
+  std::vector<int> axis_hw;
+  int shfl_per_thread = 0;
   std::vector<int> dup_bits;      // zero-column kernel bits (de-dup)
   std::vector<u64> out_col;       // per kernel bit: output flat offset (0 for reduced/dup)
   std::vector<u64> grid_out;      // per grid bit: output flat offset

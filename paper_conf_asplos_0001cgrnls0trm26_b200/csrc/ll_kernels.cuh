@@ -134,6 +134,7 @@ __device__ __forceinline__ void load_vec(u32 (&r)[NW], const u8* p) {
   } else if constexpr (VB == 2) {
     set_e<2, E0 * W / 2>(r, u32(*reinterpret_cast<const u16*>(p)));
   } else {
+    static_assert(VB == 1, "global vector width must be 1, 2, 4, 8 or 16 bytes");
     set_e<1, E0>(r, u32(*p));
   }
 }
@@ -150,6 +151,7 @@ __device__ __forceinline__ void store_vec(const u32 (&r)[NW], u8* p) {
   } else if constexpr (VB == 2) {
     *reinterpret_cast<u16*>(p) = u16(get_e<2, E0 * W / 2>(r));
   } else {
+    static_assert(VB == 1, "global vector width must be 1, 2, 4, 8 or 16 bytes");
     *p = u8(get_e<1, E0>(r));
   }
 }
@@ -328,8 +330,10 @@ __device__ __forceinline__ void sts_vec(u32 addr, const u32* v) {
     asm volatile("st.shared.u32 [%0], %1;" ::"r"(addr), "r"(v[0]) : "memory");
   else if constexpr (VB == 2)
     asm volatile("st.shared.u16 [%0], %1;" ::"r"(addr), "h"(u16(v[0])) : "memory");
-  else
+  else {
+    static_assert(VB == 1, "shared vector width must be 1, 2, 4, 8 or 16 bytes");
     asm volatile("st.shared.u8 [%0], %1;" ::"r"(addr), "r"(v[0]) : "memory");
+  }
 }
 template <int W, int SV>
 __device__ __forceinline__ void lds_vec(u32 addr, u32* v) {
@@ -345,6 +349,7 @@ __device__ __forceinline__ void lds_vec(u32 addr, u32* v) {
     asm volatile("ld.shared.u16 %0, [%1];" : "=h"(h) : "r"(addr) : "memory");
     v[0] = h;
   } else {
+    static_assert(VB == 1, "shared vector width must be 1, 2, 4, 8 or 16 bytes");
     u32 b;
     asm volatile("ld.shared.u8 %0, [%1];" : "=r"(b) : "r"(addr) : "memory");
     v[0] = b & 0xffu;
@@ -870,6 +875,7 @@ __device__ __forceinline__ void load_vec_s(u32 (&r)[NW], u32 addr) {
     asm volatile("ld.shared.u16 %0, [%1];" : "=h"(h) : "r"(addr) : "memory");
     set_e<2, E0 * W / 2>(r, u32(h));
   } else {
+    static_assert(VB == 1, "shared vector width must be 1, 2, 4, 8 or 16 bytes");
     u32 b;
     asm volatile("ld.shared.u8 %0, [%1];" : "=r"(b) : "r"(addr) : "memory");
     set_e<1, E0>(r, b & 0xffu);
@@ -1027,9 +1033,11 @@ __device__ __forceinline__ void ll_gather_body(const u8* __restrict__ src, const
 }
 
 // ------------------------------------------------------------------ reduce (a12)
-// in-register tree over the Reg axis bits, shfl.bfly over the Lane axis
-// bits, smem over the Warp axis bits — in the layout's bit order (reg, lane, warp
-// ascending); zero-column (broadcast) bits are skipped and de-duplicated at store.
+// the reduction over the axis bits of the tile — register adds, shfl.bfly
+// over lanes, shared memory over warps — run in the fixed order of reading R-reduce
+// (DESIGN.md §3): one step per in-tile logical axis bit t = 0, 1, ..., K-1, each
+// v <- v(t = 0) (op) v(t = 1) at whichever level of the kernel layout holds bit t.
+// Zero-column (broadcast) bits are skipped and de-duplicated at store.
 // The reduction operator (ll_plan_opts.reduce_op): fp32 round-to-nearest add (no FMA
 // contraction), max or min (exact: the result is one of the operands).
 template <int OP> __device__ __forceinline__ float red_op(float a, float b) {
@@ -1038,67 +1046,69 @@ template <int OP> __device__ __forceinline__ float red_op(float a, float b) {
   else return __fadd_rn(a, b);
 }
 
+template <class P, int S> struct RedStep {
+  static constexpr int HB = P::AXIS_HW[S];
+  static constexpr bool HREG = HB < P::R;
+  static constexpr bool HWARP = HB >= P::R + 5;
+  // registers no longer live at step S: reduced by an earlier register step, or duplicate
+  static constexpr int dead() {
+    int m = P::DUP_REG_MASK;
+    for (int q = 0; q < S; ++q) if (P::AXIS_HW[q] < P::R) m |= 1 << P::AXIS_HW[q];
+    return m;
+  }
+  // index of live register E among the live ones (the warp step's smem slot)
+  template <int E> static constexpr int live_index() {
+    int k = 0, t = 0;
+    for (int b = 0; b < P::R; ++b) { if ((dead() >> b) & 1) continue; if ((E >> b) & 1) k |= 1 << t; ++t; }
+    return k;
+  }
+};
+
 template <class P>
 __device__ __forceinline__ void ll_reduce_tile(u32 (&r)[1 << P::R], float* sm, u32 lane, u32 warp, u64 oblk,
                                                u64 othr, bool do_store, float* __restrict__ dst) {
-  // register tree, in the kernel layout's register-bit order
-  static_for<P::NRED_REG>([&](auto i) {
-    constexpr int B = P::RED_REG[decltype(i)::value];
-    static_for<(1 << P::R)>([&](auto e) {
-      constexpr int E = decltype(e)::value;
-      if constexpr (((E >> B) & 1) == 0 && (E & P::template done_mask<decltype(i)::value>()) == 0 &&
-                    (E & P::DUP_REG_MASK) == 0) {
-        r[E] = __float_as_uint(red_op<P::OP>(__uint_as_float(r[E]), __uint_as_float(r[E | (1 << B)])));
-      }
-    });
-  });
-  // butterfly over the lane axis bits
-  static_for<P::NRED_LANE>([&](auto i) {
-    constexpr int L = P::RED_LANE[decltype(i)::value];
-    static_for<(1 << P::R)>([&](auto e) {
-      constexpr int E = decltype(e)::value;
-      if constexpr ((E & (P::RED_REG_MASK | P::DUP_REG_MASK)) == 0) {
-        const float x = __uint_as_float(r[E]);
-        r[E] = __float_as_uint(red_op<P::OP>(x, __shfl_xor_sync(0xffffffffu, x, 1 << L)));
-      }
-    });
-  });
-  // warps through smem
-  if constexpr (P::NRED_WARP > 0) {
-    static_for<(1 << P::R)>([&](auto e) {
-      constexpr int E = decltype(e)::value;
-      if constexpr ((E & (P::RED_REG_MASK | P::DUP_REG_MASK)) == 0)
-        sm[(P::template live_index<E>() * (32 << P::WB)) + threadIdx.x] = __uint_as_float(r[E]);
-    });
-    __syncthreads();
-    if ((warp & P::RED_WARP_MASK) == 0) {
+  static_for<P::KB>([&](auto s) {
+    using St = RedStep<P, decltype(s)::value>;
+    constexpr int HB = St::HB;
+    constexpr int DEAD = St::dead();
+    if constexpr (St::HREG) {
+      // register step: slot E (bit HB clear) takes r[E] (op) r[E | bit HB]
       static_for<(1 << P::R)>([&](auto e) {
         constexpr int E = decltype(e)::value;
-        if constexpr ((E & (P::RED_REG_MASK | P::DUP_REG_MASK)) == 0) {
-          float v[1 << P::NRED_WARP];
-          static_for<(1 << P::NRED_WARP)>([&](auto m) {
-            constexpr int M = decltype(m)::value;
-            u32 wsel = warp;
-            static_for<P::NRED_WARP>([&](auto q) {
-              constexpr int Q = decltype(q)::value;
-              if ((M >> Q) & 1) wsel |= 1u << P::RED_WARP[Q];
-            });
-            v[M] = sm[(P::template live_index<E>() * (32 << P::WB)) + wsel * 32 + lane];
-          });
-          static_for<P::NRED_WARP>([&](auto q) {
-            constexpr int Q = decltype(q)::value;
-            static_for<(1 << P::NRED_WARP)>([&](auto m) {
-              constexpr int M = decltype(m)::value;
-              if constexpr (((M >> Q) & 1) == 0 && (M & ((1 << Q) - 1)) == 0)
-                v[M] = red_op<P::OP>(v[M], v[M | (1 << Q)]);
-            });
-          });
-          r[E] = __float_as_uint(v[0]);
+        if constexpr (((E >> HB) & 1) == 0 && (E & DEAD) == 0)
+          r[E] = __float_as_uint(red_op<P::OP>(__uint_as_float(r[E]), __uint_as_float(r[E | (1 << HB)])));
+      });
+    } else if constexpr (!St::HWARP) {
+      // lane step: butterfly partner lane ^ bit; the lane with the bit clear computes
+      // v(t = 0) (op) v(t = 1) — it is the copy later steps and the store use
+      constexpr int LB = HB - P::R;
+      static_for<(1 << P::R)>([&](auto e) {
+        constexpr int E = decltype(e)::value;
+        if constexpr ((E & DEAD) == 0) {
+          const float x = __uint_as_float(r[E]);
+          r[E] = __float_as_uint(red_op<P::OP>(x, __shfl_xor_sync(0xffffffffu, x, 1 << LB)));
         }
       });
+    } else {
+      // warp step through shared memory: [live slot][thread], partner warp ^ bit
+      constexpr int WBIT = HB - P::R - 5;
+      constexpr u32 NT = 32u << P::WB;
+      static_for<(1 << P::R)>([&](auto e) {
+        constexpr int E = decltype(e)::value;
+        if constexpr ((E & DEAD) == 0)
+          sm[St::template live_index<E>() * NT + threadIdx.x] = __uint_as_float(r[E]);
+      });
+      __syncthreads();
+      const u32 pt = threadIdx.x ^ (32u << WBIT);
+      static_for<(1 << P::R)>([&](auto e) {
+        constexpr int E = decltype(e)::value;
+        if constexpr ((E & DEAD) == 0)
+          r[E] = __float_as_uint(red_op<P::OP>(__uint_as_float(r[E]), sm[St::template live_index<E>() * NT + pt]));
+      });
+      __syncthreads();
     }
-    __syncthreads();
-  }
+    (void)warp;
+  });
   if (do_store) {
     static_for<(1 << P::R)>([&](auto e) {
       constexpr int E = decltype(e)::value;

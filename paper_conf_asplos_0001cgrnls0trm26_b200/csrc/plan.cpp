@@ -927,6 +927,13 @@ static bool build_linear_tile(ConvPlan& P, const ll_plan_opts* opts) {
       T.grid_src_bit.push_back(k);
       T.grid_src_xcol.push_back(P.Q[k]);
     }
+  // a column reaching below the vector needs the in-vector XOR permute, which works on
+  // vectors of >= 4 bytes (xor_perm_vec); narrower vectors: not a linear tile
+  if ((w << v) < 4) {
+    const u64 lowm = (u64(1) << v) - 1;
+    for (int b = v; b < T.n; ++b) if (T.ld_xcol[b] & lowm) return false;
+    for (u64 c : T.grid_src_xcol) if (c & lowm) return false;
+  }
   T.lcol_ld.resize(T.n);
   T.lcol_st.resize(T.n);
   for (int b = 0; b < T.n; ++b) { T.lcol_ld[b] = alog(T.ld_xcol[b]); T.lcol_st[b] = B.cols[T.st_bit[b]]; }
@@ -1361,8 +1368,11 @@ std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const 
 }
 
 // ---------------------------------------------------------------------------
-// Reduce: faithful kernel layout so the fixed order (reg, lane, warp
-// ascending) is exactly the layout's.
+// Reduce in the fixed fp32 order of reading R-reduce:
+// for each in-tile logical axis bit t = 0, 1, ..., K-1 (ascending),
+// v <- v(t = 0) + v(t = 1) — a register add, a shfl.bfly or a shared-memory step,
+// whichever level of the kernel layout L∘σ holds bit t.  The order is a property of the
+// logical tensor alone, so the fp32 bits do not depend on L, on σ or on any plan option.
 // ---------------------------------------------------------------------------
 std::unique_ptr<ReducePlan> plan_reduce(const Layout& L, int axis, const ll_plan_opts* opts) {
   if (axis < 0 || axis >= int(L.out.size())) fail(LL_ERR_INVALID_ARG, "axis out of range");
@@ -1398,8 +1408,8 @@ std::unique_ptr<ReducePlan> plan_reduce(const Layout& L, int axis, const ll_plan
     Rp->hw_bit = sigma_line(L, Rp->v, [&](int k) { return L.cols[k] != 0 && !(L.cols[k] & amask); });
   }
   const int n = int(Rp->hw_bit.size());
-  // classify kernel bits; the fixed order is kernel reg, lane, warp bits
-  // ascending — equal to L's own order for the faithful decomposition
+  // classify kernel bits (reduced per level, duplicate) and map each logical axis bit t
+  // to the kernel bit that holds it: the steps run in t order
   for (int b = 0; b < n; ++b) {
     u64 c = L.cols[Rp->hw_bit[b]];
     if (c == 0) { Rp->dup_bits.push_back(b); continue; }
@@ -1408,6 +1418,10 @@ std::unique_ptr<ReducePlan> plan_reduce(const Layout& L, int axis, const ll_plan
     else if (b < R + 5) Rp->red_lane.push_back(b - R);
     else Rp->red_warp.push_back(b - R - 5);
   }
+  for (int t = 0; t < K; ++t)
+    for (int b = 0; b < n; ++b)
+      if (L.cols[Rp->hw_bit[b]] == (u64(1) << (sh + t))) Rp->axis_hw.push_back(b);
+  if (int(Rp->axis_hw.size()) != K) fail(LL_ERR_UNSUPPORTED, "reduce: axis bit without a kernel bit (internal)");
   auto out_of = [&](u64 c) {
     u64 lower = c & ((u64(1) << sh) - 1);
     u64 a = (c & amask) >> sh;
@@ -1428,9 +1442,21 @@ std::unique_ptr<ReducePlan> plan_reduce(const Layout& L, int axis, const ll_plan
     Rp->grid_out.push_back(out_of(L.cols[k]));
   }
   Rp->out_elems = u64(1) << (L.d_out() - K);
-  int live = R - int(Rp->red_reg.size());
-  for (int b : Rp->dup_bits) if (b < R) --live;
-  Rp->wred_bytes = Rp->red_warp.empty() ? 0 : int((u64(4) << (std::max(0, live) + 5 + Rp->Wb)));
+  // shared memory of the warp steps: the registers still live at the step (not yet
+  // reduced, not duplicate) of every thread; shuffles: every live register per lane step
+  {
+    int dead = 0;
+    for (int b : Rp->dup_bits) if (b < R) ++dead;
+    Rp->wred_bytes = 0;
+    Rp->shfl_per_thread = 0;
+    for (int t = 0; t < K; ++t) {
+      const int b = Rp->axis_hw[t];
+      const int live = R - dead;
+      if (b >= R + 5) Rp->wred_bytes = std::max(Rp->wred_bytes, int(u64(4) << (live + 5 + Rp->Wb)));
+      else if (b >= R) Rp->shfl_per_thread += 1 << live;
+      else ++dead;
+    }
+  }
   // TMA staging (cp.async.bulk) when the CTA tile is contiguous in HBM (reg, lane, warp
   // are L's lowest packed bits), the stage reads are 16-byte line-coalesced (σ), and two
   // stages fit in smem; force_class = SHUFFLE keeps direct LDG loads

@@ -216,36 +216,12 @@ def test_gather_narrow_elements(w, exchange):
     assert np.array_equal(from_device(d_dst, w), O.gather(OL, 1, src, idx))
 
 
-def _line_sigma_layout(OL, axis):
-    """The reduce kernel's layout L' = L∘σ, re-derived from the rule written in
-    DESIGN.md §5.7 (line-coalesced σ: 16-byte vector bits, 3 forced lanes, 2 free lanes
-    preferring non-axis columns, the rest registers; warps and blocks unchanged).
-    Returns (L', perm) with src'[h'] = src[perm[h']]."""
-    R = OL.dim_bits("reg").__len__()
-    sh = sum(b for _, b in OL.out_dims[axis + 1:])
-    amask = ((1 << OL.out_dims[axis][1]) - 1) << sh
-    nw = sorted(OL.dim_bits("reg") + OL.dim_bits("lane"))
-    v = min(2, R)
-    rest = nw[v + 3:]
-    pref = lambda k: OL.cols[k] != 0 and not (OL.cols[k] & amask)
-    rest_sorted = [k for k in rest if pref(k)] + [k for k in rest if not pref(k)]
-    lanes = nw[v:v + 3] + rest_sorted[:2]
-    regs = nw[:v] + sorted(rest_sorted[2:])
-    hw = regs + lanes + OL.dim_bits("warp") + OL.dim_bits("block")
-    Lp = O.layout_from_cols(OL.in_dims, OL.out_dims, [OL.cols[k] for k in hw])
-    hs = np.arange(1 << OL.d_in, dtype=np.int64)
-    perm = np.zeros_like(hs)
-    for b, k in enumerate(hw):
-        perm |= ((hs >> b) & 1) << k
-    return Lp, perm
-
-
 @pytest.mark.parametrize("family", ["mma", "blocked"])
 @pytest.mark.parametrize("sigma", ["coalesced", "coalesced-ldg", "faithful"])
 def test_reduce_tolerance_and_fixed_order(family, sigma):
-    """O11: ≤ 1e-6 relative vs fp64, and bit-exact vs the fixed-order fp32 replica
-    taken over the kernel's layout (L itself for faithful σ; L∘σ for the coalesced
-    one, the order being reg, lane, warp bits ascending in both cases)."""
+    """O11: ≤ 1e-6 relative vs fp64, and bit-exact vs the fixed-order fp32 replica on
+    L itself (reading R-reduce: logical axis-bit order), for every kernel layout σ and
+    load path — the bits do not depend on plan options."""
     import torch
     rng = np.random.default_rng(1005)
     spec = W.c4("reduce", family, n_i=9, n_j=9)
@@ -262,11 +238,7 @@ def test_reduce_tolerance_and_fixed_order(family, sigma):
     got = out.cpu().numpy()
     ref = O.reduce_ref_fp64(OL, 1, src)
     assert np.all(np.abs(got - ref) <= 1e-6 * np.abs(ref))
-    if sigma == "faithful":
-        rep = O.reduce_fixed_order_fp32(OL, 1, src)
-    else:
-        Lp, perm = _line_sigma_layout(OL, 1)
-        rep = O.reduce_fixed_order_fp32(Lp, 1, src[perm])
+    rep = O.reduce_fixed_order_fp32(OL, 1, src)
     assert np.array_equal(got.view(np.uint32), rep.view(np.uint32))
 
 
@@ -473,8 +445,8 @@ def _table4_layout(family, shape, rng):
 def test_table4_reduce_families(family):
     """§8(f) N3: reductions (tl.sum) along either dim over every Table 4 layout family on
     the Table 4 shapes (5 shapes x 2 axes per family): ≤ 1e-6 relative vs
-    fp64 and bit-exact vs the fixed-order replica on the kernel layout; broadcast copies
-    counted once."""
+    fp64 and bit-exact vs the fixed-order replica (on L; no knowledge of the kernel's
+    layout); broadcast copies counted once."""
     import torch
     rng = np.random.default_rng(4747)
     for shape in TABLE4_SHAPES:
@@ -489,9 +461,14 @@ def test_table4_reduce_families(family):
             got = out.cpu().numpy()
             ref = T.astype(np.float64).reshape(shape).sum(axis=axis)
             assert np.all(np.abs(got - ref) <= 1e-6 * np.abs(ref)), (family, shape, axis)
-            Lp, perm = _line_sigma_layout(OL, axis)
-            rep = O.reduce_fixed_order_fp32(Lp, axis, src[perm])
-            assert np.array_equal(got.view(np.uint32), rep.view(np.uint32)), (family, shape, axis)
+            for sigma in ("coalesced", "faithful"):
+                if sigma == "faithful":
+                    plan = ll.ll_plan_reduce(L, axis, sigma="faithful")
+                    out.fill_(-1.0)
+                    ll.ll_reduce(torch.from_numpy(src).cuda(), out, plan)
+                    got = out.cpu().numpy()
+                rep = O.reduce_fixed_order_fp32(OL, axis, src)
+                assert np.array_equal(got.view(np.uint32), rep.view(np.uint32)), (family, shape, axis, sigma)
 
 
 def test_swizzled_memory_layout_gpu():

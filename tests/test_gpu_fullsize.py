@@ -121,9 +121,8 @@ def test_fullsize_config4_gather(family):
 def test_fullsize_config4_reduce(family):
     """Config 4 reduce on the whole [4096, 4096] fp32 tensor in [128, 128] tiles -> [4096,
     32]: every output within 1e-6 of the fp64 sum, and bit-equal to the fixed-order fp32
-    replica over the kernel layout (O11; the σ rule re-derived in test_gpu_convert)."""
+    replica on L (O11, reading R-reduce), for both kernel layouts σ."""
     import torch
-    from tests.test_gpu_convert import _line_sigma_layout
     spec = W.c4("reduce", family)
     L, OL = both(spec)
     n = 1 << OL.d_in
@@ -136,6 +135,9 @@ def test_fullsize_config4_reduce(family):
     ref = O.reduce_ref_fp64(OL, 1, src)
     assert got.size == 4096 * 32
     assert np.all(np.abs(got - ref) <= 1e-6 * np.abs(ref))
-    Lp, perm = _line_sigma_layout(OL, 1)
-    rep = O.reduce_fixed_order_fp32(Lp, 1, src[perm])
+    rep = O.reduce_fixed_order_fp32(OL, 1, src)
     assert np.array_equal(got.view(np.uint32), rep.view(np.uint32))
+    plan_f = ll.ll_plan_reduce(L, 1, sigma="faithful")
+    out.fill_(-1.0)
+    ll.ll_reduce(torch.from_numpy(src).cuda(), out, plan_f)
+    assert np.array_equal(out.cpu().numpy().view(np.uint32), rep.view(np.uint32))

@@ -95,6 +95,58 @@ def test_errors():
         ll.Layout([("reg", 1)], [("x", 1)], {"reg": [(2,)]})
 
 
+@pytest.mark.parametrize("mvb", [3, 24, 32, 64, -4])
+def test_max_vec_bytes_validated(mvb):
+    """max_vec_bytes outside {0, 1, 2, 4, 8, 16} is rejected at plan time by every
+    planner (no ld/st instruction is wider than 16 B): no plan silently
+    falls back to byte loads."""
+    A, _ = both(W.C1_A)
+    B, _ = both(W.C1_B)
+    L = ll.Layout.from_spec(W.c4("reduce", "mma", n_i=7, n_j=7))
+    with pytest.raises(ll.LLError, match="INVALID_ARG"):
+        ll.ll_plan_convert(A, B, 4, max_vec_bytes=mvb)
+    with pytest.raises(ll.LLError, match="INVALID_ARG"):
+        ll.ll_plan_gather(ll.Layout.from_spec(W.c4("gather", "mma", n_i=7, n_j=5)), 1, 4, max_vec_bytes=mvb)
+    with pytest.raises(ll.LLError, match="INVALID_ARG"):
+        ll.ll_plan_reduce(L, 1, max_vec_bytes=mvb)
+    with pytest.raises(ll.LLError, match="INVALID_ARG"):
+        ll.ll_plan_scan(L, 1, max_vec_bytes=mvb)
+
+
+@pytest.mark.parametrize("mvb", [1, 2, 4, 8, 16])
+def test_max_vec_bytes_accepted(mvb):
+    A, _ = both(W.C1_A)
+    B, _ = both(W.C1_B)
+    p = ll.ll_plan_convert(A, B, 4, max_vec_bytes=mvb)
+    assert p.buffer_bytes() == (1024, 1024, 0)
+
+
+def test_buffer_sizes_checked_before_launch():
+    """The execution wrappers compare tensor sizes with ll_plan_buffer_bytes and raise
+    before any pointer reaches the library (CPU tensors: nothing is launched)."""
+    import torch
+    A, _ = both(W.C1_A)
+    B, _ = both(W.C1_B)
+    p = ll.ll_plan_convert(A, B, 4)
+    ok = torch.empty(256, dtype=torch.int32)
+    small = torch.empty(255, dtype=torch.int32)
+    with pytest.raises(ll.LLError, match="src"):
+        ll.ll_convert(small, ok, p)
+    with pytest.raises(ll.LLError, match="dst"):
+        ll.ll_convert(ok, torch.empty(128, dtype=torch.int16), p)
+    L = ll.Layout.from_spec(W.c4("gather", "mma", n_i=7, n_j=5))
+    g = ll.ll_plan_gather(L, 1, 4)
+    n = 1 << 12
+    assert g.buffer_bytes() == (4 * n, 4 * n, 4 * n)
+    with pytest.raises(ll.LLError, match="idx"):
+        ll.ll_gather(torch.empty(n, dtype=torch.float32), torch.empty(n // 2, dtype=torch.int32),
+                     torch.empty(n, dtype=torch.float32), g)
+    R = ll.ll_plan_reduce(ll.Layout.from_spec(W.c4("reduce", "mma", n_i=7, n_j=7)), 1)
+    assert R.buffer_bytes() == (4 << 14, 4 * R.out_elems(), 0)
+    with pytest.raises(ll.LLError, match="dst"):
+        ll.ll_reduce(torch.empty(1 << 14), torch.empty(R.out_elems() - 1), R)
+
+
 @pytest.mark.parametrize("cfg", ["c1", "c2", "c3"])
 def test_planner_class_matches_oracle_configs(cfg):
     sa, sb = {"c1": (W.C1_A, W.C1_B), "c2": W.c2(0), "c3": W.c3(0)}[cfg]

@@ -632,6 +632,70 @@ def test_reduce_broadcast_dedup():
     assert np.allclose(rep, ref, rtol=1e-6)
 
 
+def _reduce_rows(L, rows):
+    """O11 replica applied to the logical [n_rows, K] tensor `rows` packed under L."""
+    T = np.asarray(rows, dtype=np.float32).reshape(-1)
+    return O.reduce_fixed_order_fp32(L, 1, O.pack(L, T))
+
+
+@pytest.mark.parametrize("which", ["blocked_row", "blocked_col"])
+def test_reduce_order_golden(which):
+    """Pin (tests/golden/reduce_order.json, hand-derived under IEEE binary32 RN-even):
+    the fixed order of reading R-reduce gives the expected fp32 bits on rows whose sum
+    depends on the order, under two layouts that place the axis bits on different
+    hardware levels (registers first vs lanes first)."""
+    g = load("reduce_order.json")
+    u = np.float32(2.0 ** -24)
+    rows = [np.array(c["x_in_u"], dtype=np.float64) * float(u) for c in g["cases"]]
+    L = {"blocked_row": O.blocked([4, 8], [1, 2], [4, 8], [1, 1], [1, 0]),
+         "blocked_col": O.blocked([4, 8], [2, 1], [2, 16], [1, 1], [0, 1])}[which]
+    out = _reduce_rows(L, rows)
+    for c, got in zip(g["cases"], out):
+        assert "%08x" % int(np.float32(got).view(np.uint32)) == c["expected_hex"], c["name"]
+        for other in c["other_orders_hex"].values():
+            assert other != c["expected_hex"]          # the case really separates orders
+
+
+def _pairwise(x):
+    """Textbook recursive pairwise summation in fp32 (Higham, Accuracy and Stability
+    of Numerical Algorithms, §4.2): S(x) = S(x[:n/2]) + S(x[n/2:])."""
+    if len(x) == 1:
+        return np.float32(x[0])
+    h = len(x) // 2
+    return np.float32(_pairwise(x[:h]) + _pairwise(x[h:]))
+
+
+@pytest.mark.parametrize("family", ["mma", "blocked"])
+def test_reduce_order_is_recursive_pairwise(family):
+    """Pin: the replica equals the recursive pairwise sum of each in-tile row segment
+    (a top-down formulation of the same order), on [128, 128]-tile layouts of config 4
+    with adversarial magnitudes (1 followed by tiny values, so that the order matters)."""
+    rng = np.random.default_rng(11)
+    L = L_of(W.c4("reduce", family, n_i=7, n_j=8))      # [128, 256], K = 128
+    T = rng.random((128, 256), dtype=np.float32) * np.float32(2.0 ** -22)
+    T[:, ::128] = 1.0
+    got = O.reduce_fixed_order_fp32(L, 1, O.pack(L, T.reshape(-1))).reshape(128, 2)
+    for r in range(0, 128, 7):
+        for q in range(2):
+            ref = _pairwise(list(T[r, q * 128:(q + 1) * 128]))
+            assert got[r, q].view(np.uint32) == ref.view(np.uint32), (r, q)
+    # the order matters on these rows: a sequential fp32 sum differs somewhere
+    seq = np.array([np.float32(sum(np.float32(v) for v in T[r, :128])) for r in range(0, 128, 7)])
+    assert np.any(seq.view(np.uint32) != got[::7, 0].view(np.uint32))
+
+
+def test_reduce_order_layout_independent():
+    """Invariant of reading R-reduce: the replica's bits depend on the logical tensor
+    only — the MMA-accumulator and blocked layouts of config 4 give identical bits."""
+    rng = np.random.default_rng(12)
+    La = L_of(W.c4("reduce", "mma", n_i=8, n_j=8))
+    Lb = L_of(W.c4("reduce", "blocked", n_i=8, n_j=8))
+    T = (rng.random(1 << 16, dtype=np.float32) * np.float32(3.0)).astype(np.float32)
+    ra = O.reduce_fixed_order_fp32(La, 1, O.pack(La, T))
+    rb = O.reduce_fixed_order_fp32(Lb, 1, O.pack(Lb, T))
+    assert np.array_equal(ra.view(np.uint32), rb.view(np.uint32))
+
+
 def test_distributed_rank_slices_concatenate():
     """O12: the per-rank slices of B, for config-5 layouts at small size, are the
     column shards of the logical tensor (an all_to_all of row shards)."""
