@@ -146,55 +146,71 @@ def relaunch_if_needed(args):
     os.execv(sys.executable, cmd)
 
 
-def cpu_baseline_oracle(A_spec, B_spec, w, budget_s=12.0):
-    """The CPU oracle (oracle/ll_oracle.py, as it stands) on a bounded sample: dst[h]
-    for a contiguous run of whole tiles via the oracle's pull map (B(h), then the
-    slack-zero right inverse of A, then the element copy).  Single numpy thread."""
+def _oracle_sample(threads, budget_s, tiles=256):
+    """The C++17/OpenMP oracle (oracle/ll_oracle.cpp, as it stands) on a bounded sample
+    of the config-2 workload: `tiles` 128x128 bf16 tiles of the same A -> B (the block
+    bits are a batch index: every tile is the same conversion), repeated until
+    `budget_s`.  Per element: B(h) bit by bit, then the slack-zero right inverse of A
+    applied linearly, then the 2-byte copy (O5).  Returns (GB/s, elements, seconds)."""
     import numpy as np
+    from oracle import cpp as OC
     from oracle import ll_oracle as O
     from workloads import configs as W
-    OA = O.Layout(*W.spec_to_bases(A_spec))
-    OB = O.Layout(*W.spec_to_bases(B_spec))
-    tile = 1 << 14
-    rng = np.random.default_rng(0)
-    src = rng.integers(0, 1 << 16, size=1 << 22, dtype=np.uint16)   # 64 tiles of source data
+    nb = tiles.bit_length() - 1
+    sa, sb = W.c2(nb)
+    OA, OB = O.Layout(*W.spec_to_bases(sa)), O.Layout(*W.spec_to_bases(sb))
+    src = np.random.default_rng(0).integers(0, 1 << 16, size=1 << OA.d_in, dtype=np.uint16)
+    out = np.empty(src.size * 2, dtype=np.uint8)
     done, t0 = 0, time.perf_counter()
-    while time.perf_counter() - t0 < budget_s:
-        hs = np.arange(done * tile, (done + 8) * tile, dtype=np.uint64) % np.uint64(1 << OB.d_in)
-        xs = O.apply_all(OB, hs)
-        h_src = O.apply_inverse_all(OA, xs).astype(np.int64) & ((1 << 22) - 1)
-        _ = src[h_src]
-        done += 8
-    dt = time.perf_counter() - t0
-    elems = done * tile
-    return {"value": round(2 * w * elems / dt / 1e9, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
-            "sample": f"{done} tiles ({elems} elements) of the config-2 batch, oracle pull map + copy, {dt:.1f}s"}
+    while True:
+        OC.convert(OA.cols, OB.cols, OA.d_out, 2, src, threads=threads, out=out)
+        done += src.size
+        dt = time.perf_counter() - t0
+        if dt >= budget_s:
+            break
+    return 2 * 2 * done / dt / 1e9, done, dt
+
+
+def cpu_baseline_oracle(budget_s=10.0):
+    """cpu_baseline: the C++ oracle on all host cores (os.cpu_count() OpenMP threads)
+    and on one core, with the CPU model; a baseline only."""
+    from oracle import cpp as OC
+    ncores = os.cpu_count() or 1
+    v_all, n_all, t_all = _oracle_sample(ncores, budget_s * 0.7)
+    v_one, n_one, t_one = _oracle_sample(1, budget_s * 0.3)
+    return {"value": round(v_all, 4), "unit": "GB/s", "cores": ncores, "kind": "oracle",
+            "impl": "oracle/ll_oracle.cpp (C++17, OpenMP, g++ -O2)", "cpu_model": OC.cpu_model(),
+            "sample": f"{n_all} elements ({n_all >> 14} tiles) of the config-2 batch in {t_all:.1f}s, "
+                      f"pull map B(h) -> A^+ -> copy, {ncores} threads",
+            "single_core": {"value": round(v_one, 4), "cores": 1,
+                            "sample": f"{n_one} elements in {t_one:.1f}s, 1 thread"}}
 
 
 def run_reference(args):
-    """--impl reference: the oracle timed on host cores on the same config/metric."""
+    """--impl reference: the oracle (C++17/OpenMP, all host cores) timed on the same
+    config / metric; each step is one bounded sample of the workload (256 tiles =
+    8 MiB in + 8 MiB out), and ms_per_step is that step's actual duration."""
     rank, world, _ = dist_env()
     if world > 1 and rank != 0:
         return
-    from workloads import configs as W
-    A_spec, B_spec = W.c2(16)
-    per = []
-    budget = min(1.0, max(0.05, 60.0 / max(1, args.steps)))
+    from oracle import cpp as OC
+    ncores = os.cpu_count() or 1
     for _ in range(args.warmup):
-        cpu_baseline_oracle(A_spec, B_spec, 2, budget_s=0.05)
-    for _ in range(args.steps):
-        per.append(cpu_baseline_oracle(A_spec, B_spec, 2, budget_s=budget))
-    value = statistics.median(p["value"] for p in per)
-    step_bytes = 2 * (1 << 30) * 2          # one step: the whole config-2 batch, read + write
-    line = {"metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": args.gpus, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": round(step_bytes / (value * 1e9) * 1e3, 1),
-            "ms_per_step_note": "projected: one full step's bytes at the sampled rate (each timed step is a "
-                                "bounded sample of the workload)",
+        _oracle_sample(ncores, 0.0)
+    per = [_oracle_sample(ncores, 0.0) for _ in range(args.steps)]
+    total_bytes = sum(4 * n for _, n, _ in per)
+    total_s = sum(t for _, _, t in per)
+    value = total_bytes / total_s / 1e9
+    ms = total_s / len(per) * 1e3
+    sample = f"{per[0][1]} elements (256 tiles) of the config-2 batch per step, {ncores} threads"
+    line = {"metric": METRIC, "value": round(value, 4), "unit": "GB/s", "n_gpus": args.gpus, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": round(ms, 3),
             "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "bf16", "data": "synthetic", "impl": "reference",
-            "config": {"workload": WORKLOAD, "elem_bytes": 2},
-            "cpu_baseline": {"value": value, "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": per[0]["sample"]},
-            "e2e": {"value": value, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+            "config": {"workload": WORKLOAD, "elem_bytes": 2, "step": "one bounded sample: 256 of the 65536 tiles"},
+            "cpu_baseline": {"value": round(value, 4), "unit": "GB/s", "cores": ncores, "kind": "oracle",
+                             "cpu_model": OC.cpu_model(), "sample": sample},
+            "e2e": {"value": round(value, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
 
@@ -646,7 +662,7 @@ def main():
             torch.cuda.empty_cache()
             line["configs"] = other_configs(ll, W, torch, peak)
         if world == 1 and not args.no_cpu_baseline:   # the oracle baseline: rank 0 at N=1 only
-            line["cpu_baseline"] = cpu_baseline_oracle(A_spec, B_spec, w)
+            line["cpu_baseline"] = cpu_baseline_oracle()
         print(json.dumps(line), flush=True)
     if world > 1:
         torch.distributed.destroy_process_group()
