@@ -125,22 +125,23 @@ def test_noop_memcpy():
     assert np.array_equal(from_device(d_dst, 4), src)
 
 
-def test_config2_full_size_sampled():
-    """BASELINE config 2 at full size (65536 tiles, 2 GiB in) in the launch
-    configuration bench.py times; 2^20 sampled outputs checked against the oracle's
-    pull map one by one."""
+def _full_size_every_element(sa, sb, w, nsample_seed):
+    """Full-size conversion in bench.py's launch configuration (the default plan):
+    src hash-filled (src[h] = H(A(h)), workloads/hashfill.py), then EVERY dst element
+    compared on the device with the closed form H(B(h)) (O5), and 2^20 sampled outputs
+    additionally against the oracle's pull map A^+(B(h)) one by one."""
     import torch
-    sa, sb = W.c2(16)
+    from workloads import hashfill as H
     A, OA = both(sa)
     B, OB = both(sb)
-    plan = ll.ll_plan_convert(A, B, 2)
-    n = 1 << 30
-    g = torch.Generator(device="cuda").manual_seed(1002)
-    src = torch.randint(-2 ** 15, 2 ** 15, (n,), dtype=torch.int16, device="cuda", generator=g)
+    plan = ll.ll_plan_convert(A, B, w)
+    src = H.fill(sa, w, nsample_seed)
+    n = src.numel()
     dst = torch.empty_like(src)
     ll.ll_convert(src, dst, plan)
     torch.cuda.synchronize()
-    rng = np.random.default_rng(3)
+    assert H.check(sb, w, nsample_seed, dst) == 0
+    rng = np.random.default_rng(nsample_seed)
     hs = np.concatenate([rng.integers(0, n, size=1 << 20), np.arange(4096), n - 1 - np.arange(4096)]).astype(np.uint64)
     hsrc = O.apply_inverse_all(OA, O.apply_all(OB, hs)).astype(np.int64)
     got = dst[torch.from_numpy(hs.astype(np.int64)).cuda()].cpu().numpy()
@@ -150,24 +151,14 @@ def test_config2_full_size_sampled():
     torch.cuda.empty_cache()
 
 
-def test_config3_full_size_sampled():
-    import torch
-    sa, sb = W.c3(14)
-    A, OA = both(sa)
-    B, OB = both(sb)
-    plan = ll.ll_plan_convert(A, B, 2)
-    n = 1 << 29
-    g = torch.Generator(device="cuda").manual_seed(1003)
-    src = torch.randint(-2 ** 15, 2 ** 15, (n,), dtype=torch.int16, device="cuda", generator=g)
-    dst = torch.empty_like(src)
-    ll.ll_convert(src, dst, plan)
-    torch.cuda.synchronize()
-    rng = np.random.default_rng(4)
-    hs = np.concatenate([rng.integers(0, n, size=1 << 20), np.arange(4096)]).astype(np.uint64)
-    hsrc = O.apply_inverse_all(OA, O.apply_all(OB, hs)).astype(np.int64)
-    got = dst[torch.from_numpy(hs.astype(np.int64)).cuda()].cpu().numpy()
-    want = src[torch.from_numpy(hsrc).cuda()].cpu().numpy()
-    assert np.array_equal(got, want)
+def test_config2_full_size():
+    """BASELINE config 2 at full size (65536 tiles, 2^30 bf16 elements)."""
+    _full_size_every_element(*W.c2(16), 2, 1002)
+
+
+def test_config3_full_size():
+    """BASELINE config 3 at full size (16384 tiles, 2^29 fp16 elements)."""
+    _full_size_every_element(*W.c3(14), 2, 1003)
 
 
 @pytest.mark.parametrize("family", ["mma", "blocked"])

@@ -78,12 +78,13 @@ def test_max_size_convert_8gib():
     A, OA = both(sa)
     B, OB = both(sb)
     plan = ll.ll_plan_convert(A, B, 2)
+    from workloads import hashfill as H
     n = 1 << 32
-    g = torch.Generator(device="cuda").manual_seed(1002)
-    src = torch.randint(-2 ** 15, 2 ** 15, (n,), dtype=torch.int16, device="cuda", generator=g)
+    src = H.fill(sa, 2, 1002)
     dst = torch.empty_like(src)
     ll.ll_convert(src, dst, plan)
     torch.cuda.synchronize()
+    assert H.check(sb, 2, 1002, dst) == 0          # every one of the 2^32 elements
     hs = _sample(n, np.random.default_rng(5))
     hsrc = O.apply_inverse_all(OA, O.apply_all(OB, hs)).astype(np.int64)
     got = dst[torch.from_numpy(hs.astype(np.int64)).cuda()].cpu().numpy()

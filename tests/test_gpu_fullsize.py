@@ -1,12 +1,13 @@
 """Every BASELINE config at its full size, in the launch configuration bench.py times
 (the default plan, the same buffers' shapes), against the oracle (-m gpu).
 
-Configs 2 and 3 are in test_gpu_convert.py (sampled full-size checks).  Here:
-config 1 batch (2^20 tiles, 1 GiB), config 3b, config 4 gather and reduce for both
-families on the whole [4096, 4096] fp32 tensor (every output compared), config 5-T
-(2 GiB transpose) and config 5 at P = 8 on the loopback communicator with both
-exchanges (2 GiB).  Large conversions are checked on 2^18-2^20 sampled outputs, each
-against the oracle's pull map evaluated point by point (O5 with the slack-zero inverse).
+Configs 2 and 3 are in test_gpu_convert.py.  Here: config 1 batch (2^20 tiles,
+1 GiB), config 3b, config 4 gather and reduce for both families on the whole
+[4096, 4096] fp32 tensor (every output compared with the oracle), config 5-T (2 GiB
+transpose) and config 5 at P = 8 on the loopback communicator with both exchanges
+(2 GiB).  Every element of every large conversion is compared on the device with the
+closed form H(B(h)) of hash-filled src (O5 at scale, workloads/hashfill.py); 2^18-2^20
+sampled outputs are additionally checked against the oracle's pull map point by point.
 """
 import numpy as np
 import pytest
@@ -42,13 +43,13 @@ def test_fullsize_conversions(name):
     A, OA = both(sa)
     B, OB = both(sb)
     plan = ll.ll_plan_convert(A, B, w)
+    from workloads import hashfill as H
     n = 1 << OA.d_in
-    dt = {2: torch.int16, 4: torch.int32}[w]
-    g = torch.Generator(device="cuda").manual_seed(1003)
-    src = torch.randint(-2 ** 15, 2 ** 15, (n,), dtype=dt, device="cuda", generator=g)
+    src = H.fill(sa, w, 1003)
     dst = torch.empty_like(src)
     ll.ll_convert(src, dst, plan)
     torch.cuda.synchronize()
+    assert H.check(sb, w, 1003, dst) == 0
     _sampled(OA, OB, src, dst, n, 11)
     del src, dst
     torch.cuda.empty_cache()
@@ -57,7 +58,7 @@ def test_fullsize_conversions(name):
 @pytest.mark.parametrize("exchange", ["collective", "peer"])
 def test_fullsize_config5_p8_loopback(exchange):
     """Config 5: [32768, 32768] bf16 row-sharded -> column-sharded over 8 virtual ranks
-    (2 GiB); every rank's slice sampled against the oracle's closed form O12."""
+    (2 GiB); every element of every rank's slice against the closed form of O12."""
     import torch
     p, n = 3, 15
     sa, sb = W.c5(p, n=n)
@@ -67,34 +68,29 @@ def test_fullsize_config5_p8_loopback(exchange):
     plan = ll.ll_plan_convert(A, B, 2, comm=ll.Comm.loopback(P), exchange=exchange)
     total = 1 << (2 * n)
     nloc = total // P
-    # logical tensor T as a hash of the flat index; rank slices of A built from it
-    g = torch.Generator(device="cuda").manual_seed(1006)
-    T = torch.randint(-2 ** 15, 2 ** 15, (total,), dtype=torch.int16, device="cuda", generator=g)
-    # input construction only (a wrong src fails the oracle check below): rank r's
-    # slice of A is T at A(h, dev=r), the XOR of the oracle's columns, evaluated on
-    # the device for the 2^27 points of each slice
-    src = torch.empty(total, dtype=torch.int16, device="cuda")
-    hl = torch.arange(nloc, dtype=torch.int64, device="cuda")
-    for r in range(P):
-        la, off = O.rank_slice(OA, r)
-        xs = torch.full_like(hl, int(off))
-        for k, c in enumerate(la.cols):
-            xs ^= ((hl >> k) & 1) * int(c)
-        src[r * nloc:(r + 1) * nloc] = T[xs]
-    del hl, xs
+    # src hash-filled: rank r's slice holds H(A(h, dev = r)); the closed form of O12 is
+    # dst_r[h] = H(B(h, dev = r)), checked at every element of every rank's slice
+    from workloads import hashfill as H
+    seed = 1006
+    src = H.fill(sa, 2, seed)
     dst = torch.empty_like(src)
     ws = torch.empty(max(16, plan.workspace_bytes()), dtype=torch.uint8, device="cuda")
     ll.ll_convert(src, dst, plan, workspace=ws)
     torch.cuda.synchronize()
+    assert H.check(sb, 2, seed, dst) == 0
+    # and sampled outputs of every rank against the oracle's O12 slice pull map
     rng = np.random.default_rng(13)
     for r in range(P):
         hs = np.concatenate([rng.integers(0, nloc, size=1 << 16), np.arange(1024), nloc - 1 - np.arange(1024)])
         hs = hs.astype(np.uint64)
         lb, offb = O.rank_slice(OB, r)
-        xs = (O.apply_all(lb, hs) ^ np.uint64(offb)).astype(np.int64)
+        xs = (O.apply_all(lb, hs) ^ np.uint64(offb))
+        # the loopback src holds all ranks' slices back to back: A^+(x) is the global index
+        hsrc = O.apply_inverse_all(OA, xs).astype(np.int64)
         got = dst[r * nloc + torch.from_numpy(hs.astype(np.int64)).cuda()]
-        assert torch.equal(got, T[torch.from_numpy(xs).cuda()]), r
-    del T, src, dst
+        want = src[torch.from_numpy(hsrc).cuda()]
+        assert torch.equal(got, want), r
+    del src, dst
     torch.cuda.empty_cache()
 
 
