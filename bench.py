@@ -294,21 +294,23 @@ def size_matched_copy(torch, nbytes, nsets=4):
 
 
 def other_configs(ll, W, torch, peak):
+    from workloads import hashfill
     """The other BASELINE configs (1, 3, 4, 5) measured live on this GPU, each against
     the same copy roofline: GB/s = algorithmic bytes / median time per call.  Inputs
     larger than L2, or 4 rotated buffer sets for config 4 (192 / 64.5 MiB per set)."""
     out = []
 
-    def conv(name, sa, sb, w, comm=None, batch=5, **opts):
+    def conv(name, sa, sb, w, comm=None, batch=5, torch_ref=True, **opts):
         A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
         p = ll.ll_plan_convert(A, B, w, comm=comm, **opts) if comm else ll.ll_plan_convert(A, B, w, **opts)
         p.prepare()
         n = 1 << A.d_in        # all ranks' slices for the loopback communicator (dev bits included)
-        src = torch.randint(-2 ** 15, 2 ** 15, (n * w // 2,), dtype=torch.int16, device="cuda")
-        dst = torch.empty_like(src)
+        nb = 1 << B.d_in       # > n for broadcasting B (replicas written)
+        src = hashfill.fill(sa, w, 11)
+        dst = torch.empty(nb * w, dtype=torch.uint8, device="cuda")
         ms = _time_stream(lambda: ll.ll_convert(src, dst, p), torch, batch=batch)
         d = p.describe()
-        gbs = 2 * n * w / ms / 1e6
+        gbs = (n + nb) * w / ms / 1e6   # algorithmic: src read once + every dst element written
         if "tile" in d:
             ex = d["tile"]["xchg"]
         elif d.get("exchange") == "peer":
@@ -316,13 +318,14 @@ def other_configs(ll, W, torch, peak):
         else:
             ex = d["exec"]
         entry = {"workload": name, "class": d["class"], "executed": ex, "ms": round(ms, 4),
-                 "GBps": round(gbs, 1), "frac": round(gbs / peak, 3)}
+                 "GBps": round(gbs, 1), "frac": round(gbs / peak, 3),
+                 "verified": hashfill.check(sb, w, 11, dst) == 0}
         if "tile" in d and d["tile"]["xchg"] == "smem":     # Thm 5.1 instruction choice
             entry["smem_instructions"] = [d["tile"]["smem_store"], d["tile"]["smem_load"]]
-        if comm is None:
+        if comm is None and torch_ref:
             tb, y = torch_permute_baseline(torch, sa, sb, src, w)
             entry["torch_permute_GBps"] = tb["GBps"]
-            entry["torch_permute_matches"] = bool(torch.equal(y, dst))
+            entry["torch_permute_matches"] = bool(torch.equal(y.view(torch.uint8), dst))
             del y
         out.append(entry)
         del src, dst
@@ -351,6 +354,22 @@ def other_configs(ll, W, torch, peak):
     conv("config 5-T, P=1: 32768^2 bf16 row-major -> column-major, 2+2 GiB", *W.c5T(0), 2)
     conv("config 5, P=8 loopback on one GPU: row- -> column-sharded, peer-store kernels, 2+2 GiB",
          *W.c5(3), 2, comm=ll.Comm.loopback(8), exchange="peer")
+    # §8(f) next rows: N1 (HBM operand pre-shuffle), N2 (Blackwell TMEM fragments ->
+    # coalesced epilogue; chained-GEMM accumulator -> register-A operand), broadcast
+    conv("N1: [32768,32768] bf16 row-major -> mma m16n8k16 rhs fragment order (HBM pre-shuffle), 2+2 GiB",
+         *W.n1_preshuffle(15, 15), 2)
+    for shape in ("32x32b", "16x64b", "16x128b", "16x256b"):
+        conv(f"N2: 16384 tiles 128x128 fp32 tcgen05.ld.{shape} fragment -> blocked epilogue layout, 1+1 GiB",
+             *W.n2_tmem(shape, 14), 4)
+    conv("N2: 2^18 tiles 64x64 wgmma accumulator -> fp8 register-A operand of the next wgmma, 1+1 GiB",
+         *W.n2_acc_to_lhs(8, 18), 1)
+    conv("N2: 2^17 tiles 64x64 wgmma accumulator -> bf16 register-A operand (equal layouts), 1+1 GiB",
+         *W.n2_acc_to_lhs(16, 17), 2)
+    import numpy as np
+    from workloads import gen
+    sa_b, sb_b = gen.random_broadcast_pair(np.random.default_rng(908), 8, ki=5, kj=5, batch_bits=11)
+    conv("broadcast: bijective A -> B with 8 zero columns (256 replicas), 8 MiB in + 2 GiB out, fp32",
+         sa_b, sb_b, 4, torch_ref=False)
     # config 4: gather and reduce, [4096, 4096] fp32 in [128, K=32] / [128, 128] tiles
     for fam in ("mma", "blocked"):
         L = ll.Layout.from_spec(W.c4("gather", fam))

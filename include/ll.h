@@ -222,6 +222,19 @@ ll_status ll_layout_mma_operand(int is_rhs, int rows, int cols, int bitwidth, in
  * 128 x N fp32 TMEM accumulator (Blackwell tensor memory): thread t of warp w
  * holds row 32w + t, register r holds column r. */
 ll_status ll_layout_tmem_32x32b(int M, int N, ll_layout** L);
+/* ll_layout_tmem: the registers of a warpgroup after loading a 128 x N fp32 TMEM
+ * accumulator with tcgen05.ld.sync.aligned.<shape>.x<num>.b32,
+ * shape = "32x32b", "16x64b", "16x128b" or "16x256b" (TMEM lane = row d0, 32-bit TMEM
+ * column = column d1; warp w owns lanes [32w, 32w+32)).  Per warp and x1 load:
+ *   32x32b : thread -> row bits 0-4
+ *   16x64b : thread bits -> (row 3, col 0, row 0, row 1, row 2)
+ *   16x128b: thread bits -> (col 0, col 1, row 0-2); register -> row 3
+ *   16x256b: thread bits -> (col 1, col 2, row 0-2); registers -> (col 0, row 3)
+ * .x<num> repetitions along the columns are the next register bits; the 16-lane shapes
+ * take a second load 16 lanes down (next register bit -> row 4); warps -> rows 5, 6.
+ * Matches the CUTLASS SM100 TMEM_LOAD copy traits.  Errors: INVALID_ARG (M != 128,
+ * unknown shape, N below one x1 load).  *L is owned by the caller (ll_layout_destroy). */
+ll_status ll_layout_tmem(const char* shape, int M, int N, ll_layout** L);
 /* ll_layout_contiguity (§5.1 "Contiguous elements"): the number of
  * elements each thread can move with one vector instruction — the largest u with
  * L^{-1}_Reg(i) = i for all i < u (leading register bits mapping in order to the

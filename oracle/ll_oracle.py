@@ -520,6 +520,49 @@ def mma_operand(is_rhs: bool, shape, bitwidth: int, warps_m: int = 1, warps_n: i
     return Layout(in_dims, [("d0", rb), ("d1", cb)], {"reg": reg, "lane": lane, "warp": warp})
 
 
+TMEM_SHAPES = ("32x32b", "16x64b", "16x128b", "16x256b")
+
+
+def tmem_ld(shape: str, M: int, N: int) -> Layout:
+    """Registers of a warpgroup after loading a 128 x N fp32 accumulator from Blackwell
+    tensor memory (P:53 names tensor memory) with
+    tcgen05.ld.sync.aligned.<shape>.x<num>.b32 — TMEM lane (data path) = row i, TMEM
+    column (32-bit) = column j [HW]; warp w of the warpgroup reads lanes [32w, 32w+32).
+    Per warp and x1 repetition (PTX "matrix fragments for tcgen05.ld"):
+      32x32b : thread t <- lane t; 1 register: column 0.
+      16x64b : 16 lanes x 2 columns; thread t <- row 8*t0 + (t >> 2), column t1
+               (t0, t1 = bits 0, 1 of t); 1 register.
+      16x128b: 16 lanes x 4 columns; thread t <- row (t >> 2), column t & 3;
+               register r <- row + 8r; 2 registers.
+      16x256b: 16 lanes x 8 columns; thread t <- row (t >> 2), column 2*(t & 3) + r0;
+               register r = r0 + 2 r1 <- row + 8 r1 (the mma m16n8 C fragment); 4 registers.
+    Repetitions .x<num> step along the columns (register bits above the x1 ones, column
+    bits above the x1 width, ascending); 16-lane shapes then take a second load 16 lanes
+    down (one more register bit -> row bit 4); warps -> rows 5, 6.  Pinned to the CUTLASS
+    SM100 TMEM_LOAD copy traits (tests/test_oracle_pins.py)."""
+    assert M == 128, "a warpgroup reads 128 TMEM lanes"
+    nb = int(N).bit_length() - 1
+    I = lambda k: (1 << k, 0)
+    J = lambda k: (0, 1 << k) if k < nb else (0, 0)
+    if shape == "32x32b":
+        reg0, lane, w_cols, rows16 = [], [I(0), I(1), I(2), I(3), I(4)], 0, False
+    elif shape == "16x64b":
+        reg0, lane, w_cols, rows16 = [], [I(3), J(0), I(0), I(1), I(2)], 1, True
+    elif shape == "16x128b":
+        reg0, lane, w_cols, rows16 = [I(3)], [J(0), J(1), I(0), I(1), I(2)], 2, True
+    elif shape == "16x256b":
+        reg0, lane, w_cols, rows16 = [J(0), I(3)], [J(1), J(2), I(0), I(1), I(2)], 3, True
+    else:
+        raise ValueError(shape)
+    assert nb >= w_cols, "N smaller than one x1 load"
+    reg = list(reg0) + [J(k) for k in range(w_cols, nb)]
+    if rows16:
+        reg.append(I(4))
+    warp = [I(5), I(6)]
+    in_dims = [("reg", len(reg)), ("lane", 5), ("warp", 2)]
+    return Layout(in_dims, [("d0", 7), ("d1", nb)], {"reg": reg, "lane": lane, "warp": warp})
+
+
 def sliced(L: Layout, dim: int) -> Layout:
     """Slice: remove logical dim ``dim`` (Prop 4.8).  The result may be
     non-injective (zero columns) but stays surjective (Remark P:224)."""

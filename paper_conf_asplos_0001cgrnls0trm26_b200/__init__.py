@@ -109,6 +109,7 @@ _sig = {
     "ll_layout_contiguity": [_P, C.c_int, C.c_int, C.POINTER(C.c_int)],
     "ll_layout_mma_operand": [C.c_int] * 6 + [_PP],
     "ll_layout_tmem_32x32b": [C.c_int, C.c_int, _PP],
+    "ll_layout_tmem": [C.c_char_p, C.c_int, C.c_int, _PP],
     "ll_convert_host": [_P, _P, _P, C.c_size_t, _P, C.c_int, C.POINTER(C.c_void_p)],
 }
 for _name, _args in _sig.items():
@@ -334,6 +335,13 @@ def ll_layout_mma_operand(is_rhs, rows, cols, bitwidth, warps_m=1, warps_n=1) ->
 def ll_layout_tmem_32x32b(M, N) -> Layout:
     h = C.c_void_p()
     _check(_lib.ll_layout_tmem_32x32b(M, N, C.byref(h)))
+    return Layout(None, None, _handle=h)
+
+
+def ll_layout_tmem(shape: str, M: int, N: int) -> Layout:
+    """tcgen05.ld.<shape> fragment of a 128 x N fp32 TMEM accumulator (ll.h)."""
+    h = C.c_void_p()
+    _check(_lib.ll_layout_tmem(shape.encode(), M, N, C.byref(h)))
     return Layout(None, None, _handle=h)
 
 

@@ -427,6 +427,13 @@ ll_status ll_layout_tmem_32x32b(int M, int N, ll_layout** out) {
   LL_CATCH
 }
 
+ll_status ll_layout_tmem(const char* shape, int M, int N, ll_layout** out) {
+  LL_TRY
+  if (!out || !shape) fail(LL_ERR_INVALID_ARG, "null argument");
+  *out = new ll_layout{make_tmem(shape, M, N)};
+  LL_CATCH
+}
+
 ll_status ll_layout_slice(const ll_layout* L, int dim, ll_layout** out) {
   LL_TRY
   if (!L || !out) fail(LL_ERR_INVALID_ARG, "null argument");

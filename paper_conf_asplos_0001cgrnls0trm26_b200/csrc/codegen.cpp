@@ -1,3 +1,4 @@
+#include <algorithm>
 // Specialisation of the sm_100a kernel templates (ll_kernels.cuh): emits the plan
 // constants as a `struct P` of compile-time tables and instantiates the entry point.
 #include <cstdlib>
@@ -109,12 +110,21 @@ std::string codegen_tile(const ConvPlan& Pl) {
     o << icon("G", T.grid_dst_bit.size()) << "  static constexpr bool GRID_CONTIG = false;\n"
       << icon("GRID_LD_SHIFT", 0) << icon("GRID_ST_SHIFT", 0) << arr("u64", "GRID_LD", ld) << arr("u64", "GRID_ST", st);
   }
-  // broadcast destinations: every value is stored at 2^|rep| replica offsets (bytes)
-  std::vector<u64> rep(size_t(1) << T.rep_bits.size(), 0);
+  // broadcast destinations: every value is stored at 2^|rep| replica offsets (bytes).
+  // The lowest (up to) 4 replica bits are unrolled (16 stores to neighbouring offsets
+  // per vector); the remaining ones run as a loop around them (REP_HI: one offset per
+  // bit, XOR-combined by the loop counter), so any number of zero columns stays on the
+  // specialised kernel.
+  std::vector<int> rb = T.rep_bits;
+  std::sort(rb.begin(), rb.end());
+  const size_t nlo = std::min<size_t>(4, rb.size());
+  std::vector<u64> rep(size_t(1) << nlo, 0), rep_hi;
   for (size_t r = 0; r < rep.size(); ++r)
-    for (size_t t = 0; t < T.rep_bits.size(); ++t)
-      if ((r >> t) & 1) rep[r] |= u64(1) << (T.rep_bits[t] + lw);
-  o << icon("NREP", rep.size()) << arr("u64", "REP_OFF", rep);
+    for (size_t t = 0; t < nlo; ++t)
+      if ((r >> t) & 1) rep[r] |= u64(1) << (rb[t] + lw);
+  for (size_t t = nlo; t < rb.size(); ++t) rep_hi.push_back(u64(1) << (rb[t] + lw));
+  o << icon("NREP", rep.size()) << arr("u64", "REP_OFF", rep)
+    << icon("NREP_HI_BITS", rep_hi.size()) << arr("u64", "REP_HI", rep_hi);
   // REGPERM
   o << arr("int", "PERM", T.perm);
   // SHUFFLE

@@ -401,4 +401,52 @@ Layout make_tmem_32x32b(int M, int N) {
   return L;
 }
 
+// tcgen05.ld fragment families: a warpgroup loads the 128 x N fp32
+// accumulator (TMEM lane = row, 32-bit TMEM column = column); warp w owns lanes
+// [32w, 32w + 32).  One x1 load per warp covers (lanes x columns):
+//   32x32b  32 x 1   thread -> row (5 bits)
+//   16x64b  16 x 2   thread bits (row 3, col 0, row 0, row 1, row 2)
+//   16x128b 16 x 4   thread bits (col 0, col 1, row 0-2); register -> row 3
+//   16x256b 16 x 8   thread bits (col 1, col 2, row 0-2); registers (col 0, row 3)
+// then .x<num> repetitions along the columns (register bits), the second 16-lane load
+// of the 16-row shapes (register bit -> row 4), and the warps (rows 5, 6).
+Layout make_tmem(const std::string& shape, int M, int N) {
+  const int mb = lg2(M), nb = lg2(N);
+  if (mb != 7) fail(LL_ERR_INVALID_ARG, "tmem fragment: M must be 128 (a warpgroup's 128 TMEM lanes)");
+  auto row = [&](int k) { return u64(1) << (nb + k); };
+  auto col = [&](int k) { return k < nb ? u64(1) << k : u64(0); };
+  std::vector<u64> reg, lane;
+  int x1_cols;   // log2 of the columns one x1 load covers
+  bool half = true;
+  if (shape == "32x32b") {
+    for (int k = 0; k < 5; ++k) lane.push_back(row(k));
+    x1_cols = 0;
+    half = false;
+  } else if (shape == "16x64b") {
+    lane = {row(3), col(0), row(0), row(1), row(2)};
+    x1_cols = 1;
+  } else if (shape == "16x128b") {
+    reg = {row(3)};
+    lane = {col(0), col(1), row(0), row(1), row(2)};
+    x1_cols = 2;
+  } else if (shape == "16x256b") {
+    reg = {col(0), row(3)};
+    lane = {col(1), col(2), row(0), row(1), row(2)};
+    x1_cols = 3;
+  } else {
+    fail(LL_ERR_INVALID_ARG, "tmem fragment shape must be 32x32b, 16x64b, 16x128b or 16x256b");
+  }
+  if (nb < x1_cols) fail(LL_ERR_INVALID_ARG, "tmem fragment: N smaller than one x1 load");
+  for (int k = x1_cols; k < nb; ++k) reg.push_back(col(k));
+  if (half) reg.push_back(row(4));
+  Layout L;
+  L.out = {{"d0", mb}, {"d1", nb}};
+  L.in = {{"reg", int(reg.size())}, {"lane", 5}, {"warp", 2}};
+  L.cols = reg;
+  L.cols.insert(L.cols.end(), lane.begin(), lane.end());
+  L.cols.push_back(row(5));
+  L.cols.push_back(row(6));
+  return L;
+}
+
 }  // namespace ll

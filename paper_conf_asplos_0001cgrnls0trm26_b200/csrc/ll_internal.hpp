@@ -125,6 +125,7 @@ Layout make_mma_swizzle(int m, int n, int vec, int per_phase, int max_phase);   
 Layout make_slice(const Layout& L, int dim);                                     // Prop 4.8
 Layout make_mma_operand(int is_rhs, int rows, int cols, int bitwidth, int warps_m, int warps_n);  // Prop 9.2
 Layout make_tmem_32x32b(int M, int N);                                           // tcgen05.ld
+Layout make_tmem(const std::string& shape, int M, int N);                        // tcgen05.ld families
 
 // ------------------------------------------------------------------ plans
 enum ExecKind { EXEC_NOOP = 0, EXEC_TILE = 1, EXEC_GENERIC = 2, EXEC_DEVICE = 3 };

@@ -717,17 +717,32 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, Dst D, 
     u64 thr = st_thr;
     if constexpr (P::NOHOIST) asm volatile("" : "+l"(thr));
     const u64 doff = tile_base<P, false>(t | tile0) ^ thr;
-    u8* d = D.at(doff);
-    static_for<P::NREP>([&](auto rp) {
-      constexpr u64 RO = P::REP_OFF[decltype(rp)::value];
-      static_for<(1 << (P::R - P::VST))>([&](auto k) {
-        constexpr int K = decltype(k)::value;
-        if constexpr (PEER_REG)
-          store_vec<P::W, P::VST, K, P::NW, P::ST_HINT>(o, D.at(doff + (StOff<P, K>::value() ^ RO)));
-        else
-          store_vec<P::W, P::VST, K, P::NW, P::ST_HINT>(o, d + (StOff<P, K>::value() ^ RO));
+    auto store_reps = [&](u64 ho) {
+      u8* d = D.at(doff ^ ho);
+      static_for<P::NREP>([&](auto rp) {
+        constexpr u64 RO = P::REP_OFF[decltype(rp)::value];
+        static_for<(1 << (P::R - P::VST))>([&](auto k) {
+          constexpr int K = decltype(k)::value;
+          if constexpr (PEER_REG)
+            store_vec<P::W, P::VST, K, P::NW, P::ST_HINT>(o, D.at((doff ^ ho) + (StOff<P, K>::value() ^ RO)));
+          else
+            store_vec<P::W, P::VST, K, P::NW, P::ST_HINT>(o, d + (StOff<P, K>::value() ^ RO));
+        });
       });
-    });
+    };
+    if constexpr (P::NREP_HI_BITS == 0) {
+      store_reps(0);
+    } else {
+      // replica bits above the unrolled 4: a loop over their 2^k combinations
+      for (u32 rh = 0; rh < (1u << P::NREP_HI_BITS); ++rh) {
+        u64 ho = 0;
+        static_for<P::NREP_HI_BITS>([&](auto j) {
+          constexpr int J = decltype(j)::value;
+          if ((rh >> J) & 1u) ho ^= P::REP_HI[J];
+        });
+        store_reps(ho);
+      }
+    }
   };
   if constexpr (P::XCHG == 3 && P::STAGED) {
     // Staged smem exchange (ll_plan_opts.pipe = 3): the src vectors of the next two

@@ -1039,12 +1039,10 @@ std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, 
           if (B.cols[k]) { gD.push_back(k); gS.push_back(srcbit_of(B.cols[k])); }
           else rep.push_back(k);
         }
-        if (rep.size() <= 4) {
-          build_tile(*P, S, D, gS, gD, opts, true);
-          P->tile.rep_bits = rep;
-          P->exec = EXEC_TILE;
-          return P;
-        }
+        build_tile(*P, S, D, gS, gD, opts, true);
+        P->tile.rep_bits = rep;
+        P->exec = EXEC_TILE;
+        return P;
       } catch (const Error& e) {
         if (opts && opts->force_class >= 0) throw;
       }
@@ -1179,7 +1177,8 @@ std::string describe(const ConvPlan& P) {
       << ",\"vld\":" << T.vld << ",\"vst\":" << T.vst << ",\"ctas\":" << (u64(1) << T.grid_dst_bit.size())
       << ",\"ld_bit\":" << ivec_json(T.ld_bit) << ",\"st_bit\":" << ivec_json(T.st_bit)
       << ",\"L_ld\":" << vec_json(T.lcol_ld) << ",\"L_st\":" << vec_json(T.lcol_st)
-      << ",\"grid_src_bit\":" << ivec_json(T.grid_src_bit) << ",\"grid_dst_bit\":" << ivec_json(T.grid_dst_bit);
+      << ",\"grid_src_bit\":" << ivec_json(T.grid_src_bit) << ",\"grid_dst_bit\":" << ivec_json(T.grid_dst_bit)
+      << ",\"rep_bits\":" << ivec_json(T.rep_bits);
     if (!T.ld_xcol.empty())
       o << ",\"ld_xcol\":" << vec_json(T.ld_xcol) << ",\"linear_tile\":" << (T.ld_run >= 0 ? "true" : "false")
         << ",\"ld_run_bits\":" << (T.ld_run >= 0 ? T.ld_run : T.vld + 5)

@@ -358,6 +358,36 @@ def test_next_rows_n1_n2_bitexact(which):
     assert np.array_equal(got, ref)
 
 
+@pytest.mark.parametrize("which", ["tmem_32x32b", "tmem_16x64b", "tmem_16x128b", "tmem_16x256b",
+                                   "acc_lhs_bf16", "acc_lhs_fp8"])
+@pytest.mark.parametrize("sigma", ["coalesced", "faithful"])
+def test_n2_families_bitexact(which, sigma):
+    """§8(f) N2: every tcgen05.ld fragment shape (ll_layout_tmem; CUTLASS-pinned oracle
+    tables) -> coalesced blocked epilogue layout, and the chained-GEMM wgmma accumulator
+    -> register-A operand conversions (bf16: NOOP; fp8: SHUFFLE class) — small batches
+    against the oracle's conversion."""
+    if which.startswith("tmem"):
+        (sa, sb), w = W.n2_tmem(which[5:], 3), 4
+    else:
+        bits = 16 if which.endswith("bf16") else 8
+        (sa, sb), w = W.n2_acc_to_lhs(bits, 4), bits // 8
+    got, ref, plan = run_convert(sa, sb, w, 78, sigma=sigma)
+    assert plan.describe()["exec"] in ("tile", "noop")
+    assert np.array_equal(got, ref)
+
+
+@pytest.mark.parametrize("which", ["n1", "tmem_16x64b", "tmem_16x128b", "tmem_16x256b", "acc_lhs_fp8"])
+def test_next_rows_full_size_every_element(which):
+    """N1 / N2 at the bench's sizes (1-2 GiB): every element against H(B(h))."""
+    if which == "n1":
+        (sa, sb), w = W.n1_preshuffle(15, 15), 2
+    elif which.startswith("tmem"):
+        (sa, sb), w = W.n2_tmem(which[5:], 14), 4
+    else:
+        (sa, sb), w = W.n2_acc_to_lhs(8, 18), 1
+    _full_size_every_element(sa, sb, w, 4242)
+
+
 def test_broadcast_tile_kernels_gpu():
     """Broadcast (zero-column) layouts through the specialised kernels (rule (2),
     P:362): bit-exact, and at least some plans execute as tile kernels."""

@@ -940,3 +940,73 @@ def test_ncu_dram_traffic_within_algorithmic_bytes():
             "reduce_mma": 64 * MiB + MiB // 2, "reduce_blocked": 64 * MiB + MiB // 2}
     for k, a in algo.items():
         assert t[k] <= 1.05 * a, (k, t[k], a)
+
+
+@pytest.mark.parametrize("n_zero", [1, 3, 5, 6, 7, 8])
+def test_broadcast_sweep_specialised_and_simulated(n_zero):
+    """Broadcast targets with up to 8 zero columns stay on the specialised
+    tile kernel (replica stores: 16 unrolled, the rest looped) — never the generic
+    kernel — and the simulated schedule equals the oracle's conversion."""
+    rng = np.random.default_rng(500 + n_zero)
+    for case in range(12):
+        sa, sb = gen.random_broadcast_pair(rng, n_zero, batch_bits=2)
+        w = [1, 2, 4, 8][case % 4]
+        d = _sim_check(sa, sb, w, case)
+        assert d["exec"] == "tile", d
+        assert len(d["tile"]["rep_bits"]) == n_zero
+
+
+def test_broadcast_probe_never_generic():
+    """300 random distributed -> broadcast pairs (5-8 zero columns, batched): the
+    planner picks the generic kernel for none of them."""
+    rng = np.random.default_rng(300)
+    for _ in range(300):
+        sa, sb = gen.random_broadcast_pair(rng, int(rng.integers(5, 9)), ki=7, kj=7, batch_bits=10)
+        p = ll.ll_plan_convert(ll.Layout.from_spec(sa), ll.Layout.from_spec(sb), 4)
+        assert p.describe()["exec"] == "tile"
+
+
+@pytest.mark.parametrize("shape", ["32x32b", "16x64b", "16x128b", "16x256b"])
+@pytest.mark.parametrize("N", [8, 64, 256])
+def test_tmem_family_matches_oracle(shape, N):
+    """ll_layout_tmem (product) == O.tmem_ld (oracle, pinned to the CUTLASS SM100
+    TMEM_LOAD traits) column by column."""
+    L = ll.ll_layout_tmem(shape, 128, N)
+    assert L.cols() == O.tmem_ld(shape, 128, N).cols
+
+
+def test_tmem_family_errors():
+    with pytest.raises(ll.LLError, match="INVALID_ARG"):
+        ll.ll_layout_tmem("16x32b", 128, 64)
+    with pytest.raises(ll.LLError, match="INVALID_ARG"):
+        ll.ll_layout_tmem("16x256b", 64, 64)
+    with pytest.raises(ll.LLError, match="INVALID_ARG"):
+        ll.ll_layout_tmem("16x256b", 128, 4)
+
+
+@pytest.mark.parametrize("shape", ["32x32b", "16x64b", "16x128b", "16x256b"])
+def test_n2_tmem_epilogue_simulated(shape):
+    """TMEM fragment -> coalesced blocked epilogue layout: the planner's class equals
+    the oracle's and the simulated schedule equals the oracle's conversion."""
+    sa, sb = W.n2_tmem(shape, nb=1)
+    A, OA = both(sa)
+    B, OB = both(sb)
+    assert ll.ll_plan_convert(A, B, 4).cls == O.classify(OA, OB)
+    d = _sim_check(sa, sb, 4, 3)
+    assert d["exec"] == "tile"
+
+
+@pytest.mark.parametrize("bits", [8, 16])
+def test_n2_acc_to_lhs_simulated(bits):
+    sa, sb = W.n2_acc_to_lhs(bits, nb=2)
+    A, OA = both(sa)
+    B, OB = both(sb)
+    p = ll.ll_plan_convert(A, B, bits // 8)
+    assert p.cls == ("NOOP" if bits == 16 else "SHUFFLE")
+    if bits == 8:
+        # default (coalesced HBM vectors of 16 fp8) and the layouts' own registers
+        # (faithful σ).  The executed exchange is smem in both: a 32-bit shuffle unit
+        # holds (j0, i3) in A but (j0, j1) in B (reading R-V, DESIGN.md §3)
+        for seed, opts in ((4, {}), (5, {"sigma": "faithful"})):
+            d = _sim_check(sa, sb, 1, seed, **opts)
+            assert d["exec"] == "tile"

@@ -848,3 +848,75 @@ def test_scan_max_min_closed_form(family):
         src = O.pack(L, T)
         assert np.array_equal(O.scan_ref_fp64(L, 1, src, "max"), O.pack(L, mx))
         assert np.array_equal(O.scan_ref_fp64(L, 1, src, "min"), O.pack(L, mn))
+
+
+# ----------------------------------------------------------------------------- N2 TMEM
+
+# CUTLASS SM100 TMEM_LOAD copy traits (flashinfer/data/cutlass/include/cute/atom/
+# copy_traits_sm100.hpp, Copy_Traits<SM100_TMEM_LOAD_<dp>dp<bits>b<num>x>): the vendor's
+# own description of each tcgen05.ld fragment as a CuTe layout
+#   DstLayout: (thread, value bit) -> i,   ValID: i -> (bit = i % BITS, data path = i // BITS)
+# written here as (thread shape, thread stride, value shape, value stride, BITS).
+CUTE_TMEM_LOAD = {
+    ("32x32b", 1): ((32,), (32,), (32,), (1,), 32),
+    ("32x32b", 2): ((32,), (64,), (64,), (1,), 64),
+    ("16x64b", 1): ((2, 2, 8), (512, 32, 64), (32,), (1,), 64),
+    ("16x64b", 2): ((2, 2, 8), (1024, 32, 128), (32, 2), (1, 64), 128),
+    ("16x128b", 1): ((4, 8), (32, 128), (32, 2), (1, 1024), 128),
+    ("16x128b", 2): ((4, 8), (32, 256), (32, 2, 2), (1, 2048, 128), 256),
+    ("16x256b", 1): ((4, 8), (64, 256), (64, 2), (1, 2048), 256),
+    ("16x256b", 2): ((4, 8), (64, 512), (64, 2, 2), (1, 4096, 256), 512),
+}
+
+
+def _cute(shape, stride, lin):
+    """CuTe layout function: colexicographic coordinates of `lin` dotted with stride."""
+    out = 0
+    for sz, st in zip(shape, stride):
+        out += (lin % sz) * st
+        lin //= sz
+    return out
+
+
+@pytest.mark.parametrize("key", sorted(CUTE_TMEM_LOAD))
+def test_tmem_ld_matches_cutlass_traits(key):
+    """N2: the oracle's tcgen05.ld fragment layouts (one warp, one load) equal the
+    CUTLASS SM100 TMEM_LOAD traits at every (thread, register): register r holds value
+    bits [32r, 32r + 32) of the thread, i.e. TMEM row dp and 32-bit column bit // 32."""
+    shape, num = key
+    tsh, tst, vsh, vst, BITS = CUTE_TMEM_LOAD[key]
+    N = BITS // 32
+    L = O.tmem_ld(shape, 128, N)
+    nregs = int(np.prod(vsh)) // 32
+    for t in range(32):
+        for r in range(nregs):
+            i = _cute(tsh, tst, t) + _cute(vsh, vst, 32 * r)
+            dp, col = i // BITS, (i % BITS) // 32
+            h = r | (t << L.dim_bits("lane")[0])
+            assert O.apply(L, h) == (dp << (N.bit_length() - 1)) | col, (key, t, r)
+
+
+@pytest.mark.parametrize("shape", ["32x32b", "16x64b", "16x128b", "16x256b"])
+def test_n2_tmem_config_tables_are_the_fragments(shape):
+    """The literal workload tables of N2 (workloads/configs.py) are the oracle's
+    tcgen05.ld fragment layouts (pinned to CUTLASS above) on every tile."""
+    sa, _ = W.n2_tmem(shape, nb=1)
+    L = L_of(sa)
+    F = O.tmem_ld(shape, 128, 128)
+    assert [c & ((1 << 14) - 1) for c in L.cols[:F.d_in]] == F.cols
+
+
+@pytest.mark.parametrize("bits", [8, 16])
+def test_n2_acc_to_lhs_tables(bits):
+    """The chained-GEMM tables are the oracle's Prop 9.2 accumulator (m64n64, 4 warps
+    along M) and lhs operand (m64 x k64, `bits`-bit elements) layouts."""
+    sa, sb = W.n2_acc_to_lhs(bits, nb=1)
+    A, B = L_of(sa), L_of(sb)
+    acc = O.mma_acc((64, 64), 4)
+    lhs = O.mma_operand(False, (64, 64), bits, warps_m=4)
+    m = (1 << 12) - 1
+    assert [c & m for c in A.cols[:acc.d_in]] == acc.cols
+    assert [c & m for c in B.cols[:lhs.d_in]] == lhs.cols
+    assert O.classify(O.Layout(*W.spec_to_bases(W.n2_acc_to_lhs(bits, nb=0)[0])),
+                      O.Layout(*W.spec_to_bases(W.n2_acc_to_lhs(bits, nb=0)[1]))) == \
+        ("NOOP" if bits == 16 else "SHUFFLE")

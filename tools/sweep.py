@@ -92,6 +92,8 @@ def main():
         return staged_configs()
     if "generic" in only:
         return generic_maps()
+    if "broadcast" in only:
+        return broadcast_sweep()
     if "all" not in only and "conv" not in only:
         return gather_reduce()
     # raw copy roofline reference
@@ -118,6 +120,36 @@ def main():
     for opts in [dict(), dict(force_class="SMEM"), dict(tile_bytes=65536), dict(thread_bytes=16)]:
         conv_case("c1batch", sa, sb, 4, **opts)
     gather_reduce()
+
+
+def broadcast_sweep():
+    """Broadcast targets: random bijective A -> B with 5-8 zero columns,
+    batched to ~2 GiB of dst, fp32.  GB/s on algorithmic bytes (src read once + every
+    dst replica written: (2^dA + 2^dB) * w), the specialised replica-store tile kernel
+    vs the generic kernel on the same pair, and the copy roofline."""
+    import numpy as np
+    from workloads import gen, hashfill
+    w = 4
+    for nz in (5, 6, 7, 8):
+        rng = np.random.default_rng(900 + nz)
+        for case in range(6):
+            sa, sb = gen.random_broadcast_pair(rng, nz, ki=5, kj=5, batch_bits=19 - nz)
+            A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
+            src = hashfill.fill(sa, w, case)
+            dst = torch.empty(1 << B.d_in, dtype=torch.int32, device="cuda")
+            alg = (src.numel() + dst.numel()) * w
+            row = {"case": f"bcast nz={nz} #{case}", "src_MiB": src.numel() * w >> 20, "dst_MiB": dst.numel() * w >> 20}
+            for tag, opts in (("tile", {}), ("generic", {"generic": True})):
+                p = ll.ll_plan_convert(A, B, w, **opts)
+                p.prepare()
+                d = p.describe()
+                ms = time_fn(lambda: ll.ll_convert(src, dst, p), iters=10, warmup=3)
+                ok = hashfill.check(sb, w, case, dst) == 0
+                row[tag] = {"exec": d["exec"], "xchg": d.get("tile", {}).get("xchg"), "vst": d.get("tile", {}).get("vst"),
+                            "ms": round(ms, 4), "GBps": round(alg / ms / 1e6, 1), "ok": ok}
+            print(json.dumps(row), flush=True)
+            del src, dst
+            torch.cuda.empty_cache()
 
 
 def matrix_tiles():

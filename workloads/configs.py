@@ -183,3 +183,42 @@ def n2_tmem_epilogue(nb: int = 13):
     B = _spec(out, ["j0", "j1", "j6", "i3", "i4", "i5", "i6"], ["j2", "j3", "j4", "j5", "i0"], ["i1", "i2"],
               _b("b", 0, nb))
     return A, B
+
+
+# ---- §8(f) N2: the other tcgen05.ld fragment shapes (CUTLASS SM100 TMEM_LOAD traits) ----
+N2_TMEM_FRAGMENTS = {
+    # shape: (reg, lane, warp) logical bits of a 128 x 128 fp32 accumulator tile
+    "32x32b": (_b("j", 0, 7), _b("i", 0, 5), ["i5", "i6"]),
+    "16x64b": (_b("j", 1, 7) + ["i4"], ["i3", "j0", "i0", "i1", "i2"], ["i5", "i6"]),
+    "16x128b": (["i3"] + _b("j", 2, 7) + ["i4"], ["j0", "j1", "i0", "i1", "i2"], ["i5", "i6"]),
+    "16x256b": (["j0", "i3"] + _b("j", 3, 7) + ["i4"], ["j1", "j2", "i0", "i1", "i2"], ["i5", "i6"]),
+}
+
+
+def n2_tmem(shape: str, nb: int = 13):
+    """A batch of 2^nb 128 x 128 fp32 accumulator tiles as loaded from TMEM by
+    tcgen05.ld.<shape> (N2_TMEM_FRAGMENTS) converted to the coalesced blocked
+    [1,4]/[2,16]/[4,1] row-major epilogue layout (as n2_tmem_epilogue)."""
+    reg, lane, warp = N2_TMEM_FRAGMENTS[shape]
+    out = [("b", nb), ("i", 7), ("j", 7)]
+    A = _spec(out, reg, lane, warp, _b("b", 0, nb))
+    B = n2_tmem_epilogue(nb)[1]
+    return A, B
+
+
+def n2_acc_to_lhs(bits: int, nb: int = 14):
+    """Chained GEMM (P:28 FlashAttention's register reuse; Prop 9.2): a batch
+    of 2^nb 64 x 64 wgmma m64n64 accumulator tiles (4 warps along M; G17), downcast to
+    `bits`-bit elements, converted into the register-A (lhs) operand of the next wgmma
+    (m64nNk{32/bits*8}).  bf16 (16): the two layouts coincide (NOOP).  fp8 (8): the lhs
+    holds 4 consecutive k per register, so k bits 1 and 3 swap between a register and
+    a lane — an intra-warp shuffle."""
+    out = [("b", nb), ("i", 6), ("j", 6)]
+    A = _spec(out, ["j0", "i3", "j3", "j4", "j5"], ["j1", "j2", "i0", "i1", "i2"], ["i4", "i5"], _b("b", 0, nb))
+    if bits == 16:
+        B = _spec(out, ["j0", "i3", "j3", "j4", "j5"], ["j1", "j2", "i0", "i1", "i2"], ["i4", "i5"], _b("b", 0, nb))
+    elif bits == 8:
+        B = _spec(out, ["j0", "j1", "i3", "j4", "j5"], ["j2", "j3", "i0", "i1", "i2"], ["i4", "i5"], _b("b", 0, nb))
+    else:
+        raise ValueError(bits)
+    return A, B

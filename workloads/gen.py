@@ -90,3 +90,29 @@ def splitmix64(x: np.ndarray, seed: int) -> np.ndarray:
     z = (z ^ (z >> np.uint64(30))) * np.uint64(0xBF58476D1CE4E5B9)
     z = (z ^ (z >> np.uint64(27))) * np.uint64(0x94D049BB133111EB)
     return z ^ (z >> np.uint64(31))
+
+
+def random_broadcast_pair(rng: np.random.Generator, n_zero: int, ki: int = 5, kj: int = 5,
+                          batch_bits: int = 0, w_bits_a: Optional[Tuple[int, int]] = None):
+    """Broadcast sweep (P:306-308 zero columns; rule (2) P:358-362): a random bijective
+    distributed A and a random distributed B with `n_zero` zero (broadcast) columns over
+    reg / lane / warp, on the logical [2^ki, 2^kj] tile, plus `batch_bits` batch bits
+    that are the block bits of both (independent tiles).  Returns (spec_A, spec_B)."""
+    d = ki + kj
+    out = [("i", ki), ("j", kj)]
+    ra = int(rng.integers(1, 4)) if w_bits_a is None else w_bits_a[0]
+    wa = d - 5 - ra
+    assert wa >= 0
+    tot_b = d + n_zero
+    rb = int(rng.integers(1, min(6, tot_b - 5) + 1))
+    wb = tot_b - 5 - rb
+    if wb > 5:
+        rb += wb - 5
+        wb = 5
+    sa = random_distributed(rng, out, [("reg", ra), ("lane", 5), ("warp", wa)])
+    sb = random_distributed(rng, out, [("reg", rb), ("lane", 5), ("warp", wb)])
+    if batch_bits:
+        for s in (sa, sb):
+            s["out"] = [("b", batch_bits)] + list(s["out"])
+            s["in"] = list(s["in"]) + [("block", [f"b{k}" for k in range(batch_bits)])]
+    return sa, sb
