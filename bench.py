@@ -307,7 +307,7 @@ def other_configs(ll, W, torch, peak):
         n = 1 << A.d_in        # all ranks' slices for the loopback communicator (dev bits included)
         nb = 1 << B.d_in       # > n for broadcasting B (replicas written)
         src = hashfill.fill(sa, w, 11)
-        dst = torch.empty(nb * w, dtype=torch.uint8, device="cuda")
+        dst = torch.empty(nb, dtype=src.dtype, device="cuda")
         ms = _time_stream(lambda: ll.ll_convert(src, dst, p), torch, batch=batch)
         d = p.describe()
         gbs = (n + nb) * w / ms / 1e6   # algorithmic: src read once + every dst element written
@@ -325,7 +325,7 @@ def other_configs(ll, W, torch, peak):
         if comm is None and torch_ref:
             tb, y = torch_permute_baseline(torch, sa, sb, src, w)
             entry["torch_permute_GBps"] = tb["GBps"]
-            entry["torch_permute_matches"] = bool(torch.equal(y.view(torch.uint8), dst))
+            entry["torch_permute_matches"] = bool(torch.equal(y.view(dst.dtype), dst))
             del y
         out.append(entry)
         del src, dst

@@ -43,7 +43,7 @@
  *  - LL_LOG=1: every conversion plan is printed (ll_plan_describe JSON) to stderr.
  *  - LL_JIT_CACHE=<dir>: the NVRTC cubin cache (default: in-tree .ll_jit_cache/).
  *  - LL_PDL=0: launch without programmatic dependent launch.
- *  - LL_PIPE=0|1|staged, LL_MIN_BLOCKS=k: override ll_plan_opts.pipe / min_blocks.
+ *  - LL_PIPE=0|1|staged|bulk|bulkst, LL_MIN_BLOCKS=k: override ll_plan_opts.pipe / min_blocks.
  *  - LL_NOHOIST=0|1: opaque thread bases in tile kernels (keeps XOR-combined addresses
  *    inside the tile loop; default on for linear tiles only).
  *  - LL_LINEAR_BALANCE=0: linear CTA tiles (general invertible pull maps) take the
@@ -126,7 +126,11 @@ typedef struct {
                          * before this tile's smem reads and HBM stores), 3 = staged
                          * (the next two tiles' 16-byte src vectors streamed by
                          * cp.async into two raw smem stages; persistent grid; needs
-                         * 16-byte load vectors and exchange + 2 tiles <= 227 KiB)   */
+                         * 16-byte load vectors and exchange + 2 tiles <= 227 KiB),
+                         * 4 = bulk (CTA tile contiguous in src order: whole tiles by
+                         * cp.async.bulk into 2-3 raw stages, mbarrier completion),
+                         * 5 = bulk load + bulk store (the dst tile, contiguous in dst
+                         * order, leaves by cp.async.bulk from a dst stage)           */
   int min_blocks;       /* tile kernels: resident CTAs per SM requested from ptxas
                          * (__launch_bounds__ minimum): 0 = auto (2 for linear tiles,
                          * else none), -1 = none, k >= 1 = k                          */

@@ -170,7 +170,7 @@ def _opts(force_class=None, max_vec_bytes=16, sigma=0, tile_bytes=0, thread_byte
     o.exchange = EXCHANGES.index(exchange) if isinstance(exchange, str) else int(exchange)
     o.smem_instr = SMEM_INSTRS.index(smem_instr) if isinstance(smem_instr, str) else int(smem_instr)
     o.reduce_op = REDUCE_OPS.index(reduce_op) if isinstance(reduce_op, str) else int(reduce_op)
-    o.pipe = {"auto": 0, "off": 1, "on": 2, "staged": 3}[pipe] if isinstance(pipe, str) else int(pipe)
+    o.pipe = {"auto": 0, "off": 1, "on": 2, "staged": 3, "bulk": 4, "bulkst": 5}[pipe] if isinstance(pipe, str) else int(pipe)
     o.min_blocks = int(min_blocks)
     return o
 

@@ -201,11 +201,13 @@ ll_status convert_impl(const void* src, void* dst, void* ws, ConvPlan& P, cudaSt
   if (s8 < d8 + dbytes && d8 < s8 + sbytes) fail(LL_ERR_ALIAS, "src and dst overlap (only NOOP plans may alias)");
   if (P.exec == EXEC_TILE) {
     ensure_tile_kernel(P);
-    u64 ntiles = u64(1) << P.tile.grid_dst_bit.size();
+    // data tiles x replica groups (broadcast replica bits above the unrolled ones)
+    const size_t rep_grid = P.tile.rep_bits.size() - std::min<size_t>(size_t(P.tile.rep_lo), P.tile.rep_bits.size());
+    u64 ntiles = u64(1) << (P.tile.grid_dst_bit.size() + rep_grid);
     unsigned long long nt = ntiles;
     void* args[] = {const_cast<void**>(&src), &dst, &nt};
     // staged tiles loop over their tiles with two stages in flight: a persistent grid
-    const unsigned grid = P.tile.staged ? unsigned(std::min<u64>(ntiles, u64(num_sms()))) : grid_for(ntiles);
+    const unsigned grid = (P.tile.staged || P.tile.bulk) ? unsigned(std::min<u64>(ntiles, u64(num_sms()))) : grid_for(ntiles);
     launch_kernel(P.kernel, grid, P.tile.threads(), args, size_t(P.smem_bytes), st,
                   "cudaLaunchKernelEx(ll_tile_kernel)");
     return LL_OK;

@@ -69,6 +69,9 @@ std::string codegen_tile(const ConvPlan& Pl) {
   o << icon("ST_HINT", st_hint());
   o << "  static constexpr bool PIPE = " << (T.pipe ? "true" : "false") << ";\n";
   o << "  static constexpr bool STAGED = " << (T.staged ? "true" : "false") << ";\n";
+  o << "  static constexpr bool BULK = " << (T.bulk ? "true" : "false") << ";\n";
+  o << "  static constexpr bool BULK_ST = " << (T.bulk_st ? "true" : "false") << ";\n";
+  o << icon("STAGES", std::max(1, T.bulk_stages)) << icon("TILE_LOG2B", T.n + lw);
   {
     const char* nh = std::getenv("LL_NOHOIST");   // experiment hook: 0 / 1 override
     const bool nohoist = nh ? std::string(nh) == "1" : T.ld_run >= 0;
@@ -111,13 +114,13 @@ std::string codegen_tile(const ConvPlan& Pl) {
       << icon("GRID_LD_SHIFT", 0) << icon("GRID_ST_SHIFT", 0) << arr("u64", "GRID_LD", ld) << arr("u64", "GRID_ST", st);
   }
   // broadcast destinations: every value is stored at 2^|rep| replica offsets (bytes).
-  // The lowest (up to) 4 replica bits are unrolled (16 stores to neighbouring offsets
-  // per vector); the remaining ones run as a loop around them (REP_HI: one offset per
-  // bit, XOR-combined by the loop counter), so any number of zero columns stays on the
-  // specialised kernel.
+  // The lowest rep_lo (<= 4) replica bits are unrolled (stores to neighbouring offsets
+  // per vector); the remaining ones are CTA-index bits above the data tiles' (REP_HI:
+  // one offset per bit, XOR-combined by the replica group), so any number of zero
+  // columns stays on the specialised kernel with enough CTAs to fill the GPU.
   std::vector<int> rb = T.rep_bits;
   std::sort(rb.begin(), rb.end());
-  const size_t nlo = std::min<size_t>(4, rb.size());
+  const size_t nlo = std::min<size_t>(size_t(T.rep_lo), rb.size());
   std::vector<u64> rep(size_t(1) << nlo, 0), rep_hi;
   for (size_t r = 0; r < rep.size(); ++r)
     for (size_t t = 0; t < nlo; ++t)

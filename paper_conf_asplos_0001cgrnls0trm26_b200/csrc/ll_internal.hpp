@@ -148,6 +148,7 @@ struct TilePlan {
   std::vector<u64> lcol_ld, lcol_st;
   std::vector<int> grid_src_bit, grid_dst_bit;   // CTA index bit g -> packed bits
   std::vector<int> rep_bits;   // dst packed bits with zero columns in B: store replicas
+  int rep_lo = 0;              // replica bits unrolled per store; the rest are grid bits
   // Linear (XOR) copy plans: the src index of kernel bit b / grid bit g is an arbitrary
   // F2 combination Q(dst bit) (swizzled memory layouts, Def 4.14; broadcast).  When
   // non-empty these replace 1 << ld_bit / 1 << grid_src_bit.
@@ -159,6 +160,9 @@ struct TilePlan {
   bool pipe = false;    // X_SMEM: next tile's loads issued before this tile's stores
   int min_blocks = 0;   // __launch_bounds__ minimum resident CTAs per SM (0 = none)
   bool staged = false;  // X_SMEM: src tiles streamed by cp.async into two raw smem stages
+  bool bulk = false;    // X_SMEM: src tiles (contiguous) streamed by cp.async.bulk into raw stages
+  bool bulk_st = false; // ... and dst tiles (contiguous) leave by cp.async.bulk from a dst stage
+  int bulk_stages = 0;
 
   // --- REGPERM: out slot e <- in slot perm[e]
   std::vector<int> perm;

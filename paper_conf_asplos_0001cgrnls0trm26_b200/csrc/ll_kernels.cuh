@@ -615,6 +615,43 @@ __device__ __forceinline__ void xchg_smem(const u32 (&r)[P::NW], u32 (&o)[P::NW]
   smem_load<P>(o, lane, warp, sbase);
 }
 
+// ------------------------------------------------------------------ TMA bulk copies
+// cp.async.bulk (SASS UBLKCP) global -> shared, completion tracked by an mbarrier
+// (expect_tx / complete_tx), the Blackwell async-copy pipeline.
+__device__ __forceinline__ void mbar_init(u32 bar, u32 count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_fence_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void fence_proxy_async() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(u32 bar, u32 bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(u32 dst, const void* src, u32 bytes, u32 bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+               ::"r"(dst), "l"(src), "r"(bytes), "r"(bar) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(u32 bar, u32 parity) {
+  u32 ok = 0;
+  do {
+    asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+                 "selp.u32 %0, 1, 0, p;\n\t}" : "=r"(ok) : "r"(bar), "r"(parity) : "memory");
+  } while (!ok);
+}
+
+// shared -> global bulk copy (SASS UBLKCP), completion by bulk async-group
+__device__ __forceinline__ void bulk_s2g(void* dst, u32 src, u32 bytes) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(src), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+template <int N> __device__ __forceinline__ void bulk_wait_read() {
+  asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
+}
+
+
 // ------------------------------------------------------------------ tile kernel
 // Programmatic dependent launch (sm_90+): the host launches every kernel with the
 // programmatic-stream-serialization attribute, so a kernel's CTAs may be scheduled
@@ -649,6 +686,9 @@ struct DstPeers {
     return p->dst[off >> SHIFT] + (off & ((u64(1) << SHIFT) - 1));
   }
 };
+
+template <class D> struct IsDstLocal { static constexpr bool value = false; };
+template <> struct IsDstLocal<DstLocal> { static constexpr bool value = true; };
 
 // PEER_REG: some register / replica bit of the dst tile crosses ranks, so every
 // store picks its window; otherwise one window per thread and tile.
@@ -688,7 +728,11 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, Dst D, 
       if ((warp >> T) & 1) lo_thr ^= P::LD_LO[P::R + 5 + T];
     });
   }
+  // broadcast plans: CTA-index bits above the data tiles' G select a group of replica
+  // offsets (the replica bits above the unrolled ones are grid bits)
+  constexpr u64 GMASK = (u64(1) << P::G) - 1;
   auto load_tile = [&](u32 (&r)[P::NW], u64 t) {
+    if constexpr (P::NREP_HI_BITS > 0) t &= GMASK;
     u64 thr = ld_thr;
     if constexpr (P::NOHOIST) asm volatile("" : "+l"(thr));   // keep per-vector addresses in the loop
     const u64 sofs = tile_base<P, true>(t) ^ thr;
@@ -716,7 +760,8 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, Dst D, 
   auto store_tile = [&](const u32 (&o)[P::NW], u64 t) {
     u64 thr = st_thr;
     if constexpr (P::NOHOIST) asm volatile("" : "+l"(thr));
-    const u64 doff = tile_base<P, false>(t | tile0) ^ thr;
+    const u64 td = P::NREP_HI_BITS > 0 ? (t & GMASK) : t;
+    const u64 doff = tile_base<P, false>(td | tile0) ^ thr;
     auto store_reps = [&](u64 ho) {
       u8* d = D.at(doff ^ ho);
       static_for<P::NREP>([&](auto rp) {
@@ -733,15 +778,14 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, Dst D, 
     if constexpr (P::NREP_HI_BITS == 0) {
       store_reps(0);
     } else {
-      // replica bits above the unrolled 4: a loop over their 2^k combinations
-      for (u32 rh = 0; rh < (1u << P::NREP_HI_BITS); ++rh) {
-        u64 ho = 0;
-        static_for<P::NREP_HI_BITS>([&](auto j) {
-          constexpr int J = decltype(j)::value;
-          if ((rh >> J) & 1u) ho ^= P::REP_HI[J];
-        });
-        store_reps(ho);
-      }
+      // replica bits above the unrolled ones: this CTA's group (CTA-index bits above G)
+      const u32 rg = u32(t >> P::G);
+      u64 ho = 0;
+      static_for<P::NREP_HI_BITS>([&](auto j) {
+        constexpr int J = decltype(j)::value;
+        if ((rg >> J) & 1u) ho ^= P::REP_HI[J];
+      });
+      store_reps(ho);
     }
   };
   if constexpr (P::XCHG == 3 && P::STAGED) {
@@ -802,6 +846,80 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, Dst D, 
     cp_async_wait0();
     return;
   }
+  if constexpr (P::XCHG == 3 && P::BULK) {
+    // Bulk-staged smem exchange (ll_plan_opts.pipe = 4, LL_PIPE=bulk): the CTA tile is
+    // contiguous in src-packed order, so one cp.async.bulk per tile (the TMA engine,
+    // not the LSU) streams it into NS raw stages, completion on an mbarrier, NS - 1 tiles
+    // ahead.  Threads read their 16-byte vectors from the stage (lanes on consecutive
+    // vectors: conflict-free), then the swizzled round trip.  With BULK_ST (pipe = 5)
+    // the dst tile (contiguous in dst-packed order) is written back into the exchange
+    // buffer in packed order and leaves by one bulk shared -> global copy: the LSU then
+    // carries shared-memory traffic only, so ncu's bank-conflict counters measure the
+    // exchange alone.
+    constexpr u32 TB = u32(1) << P::TILE_LOG2B;
+    constexpr u32 NS = P::STAGES;
+    constexpr bool BST = P::BULK_ST && IsDstLocal<Dst>::value;   // peer windows: STG stores
+    const u32 stage0 = sbase + P::XBYTES;
+    const u32 bar0 = stage0 + NS * TB;
+    if (threadIdx.x == 0) {
+      for (u32 q = 0; q < NS; ++q) mbar_init(bar0 + 8 * q, 1);
+      mbar_fence_init();
+    }
+    __syncthreads();
+    auto issue = [&](u64 tq, u32 q) {
+      mbar_expect_tx(bar0 + 8 * q, TB);
+      bulk_g2s(stage0 + q * TB, src + tile_base<P, true>(tq), TB, bar0 + 8 * q);
+    };
+    if (threadIdx.x == 0)
+      for (u32 q = 0; q + 1 < NS; ++q)
+        if (blockIdx.x + u64(q) * gridDim.x < ntiles) issue(blockIdx.x + u64(q) * gridDim.x, q);
+    u32 i = 0;
+    for (u64 t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
+      const u32 st = i % NS;
+      const u64 tn = t + u64(NS - 1) * gridDim.x;
+      if (threadIdx.x == 0 && tn < ntiles) {
+        fence_proxy_async();
+        issue(tn, (i + NS - 1) % NS);
+      }
+      mbar_wait(bar0 + 8 * st, (i / NS) & 1u);
+      u32 r[P::NW];
+      const u32 tb = stage0 + st * TB + u32(ld_thr);
+      static_for<(1 << (P::R - P::VLD))>([&](auto k) {
+        constexpr int K = decltype(k)::value;
+        load_vec_s<P::W, P::VLD, K, P::NW>(r, tb + u32(LdOff<P, K>::value()));
+      });
+      if constexpr (BST) {
+        // the previous tile's bulk store has finished reading the exchange buffer
+        if (threadIdx.x == 0) bulk_wait_read<0>();
+        __syncthreads();
+      }
+      smem_store<P>(r, lane, warp, sbase);
+      __syncthreads();   // exchange written; stage st fully read (refilled next iteration)
+      u32 o[P::NW];
+      static_for<P::NW>([&](auto q) { o[decltype(q)::value] = 0; });
+      smem_load<P>(o, lane, warp, sbase);
+      __syncthreads();   // exchange buffer free
+      if constexpr (BST) {
+        const u32 db = sbase + u32(st_thr);
+        static_for<(1 << (P::R - P::VST))>([&](auto k) {
+          constexpr int K = decltype(k)::value;
+          sts_vec<P::W, P::VST>(db + u32(StOff<P, K>::value()), &o[(K << P::VST) * P::W / 4]);
+        });
+        fence_proxy_async();
+        __syncthreads();
+        if (threadIdx.x == 0) {
+          bulk_s2g(D.at(tile_base<P, false>(t | tile0)), sbase, TB);
+          bulk_commit();
+        }
+      } else {
+        store_tile(o, t);
+      }
+    }
+    if constexpr (BST) {
+      if (threadIdx.x == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+    }
+    return;
+  }
   if constexpr (P::XCHG == 3 && P::PIPE) {
     // Software-pipelined smem exchange: once tile t sits in shared memory its
     // registers are free, so tile t + grid's loads are issued before t's smem reads
@@ -846,32 +964,6 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, Dst D, 
 // P:428-432 (G15 reading): per output slot, read idx, locate the source
 // (register candidates, lane) and run 2^{|L_Reg^axis|} shuffle rounds, keeping the
 // value whose candidate equals the source register.
-// ------------------------------------------------------------------ TMA bulk copies
-// cp.async.bulk (SASS UBLKCP) global -> shared, completion tracked by an mbarrier
-// (expect_tx / complete_tx), the Blackwell async-copy pipeline.
-__device__ __forceinline__ void mbar_init(u32 bar, u32 count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
-}
-__device__ __forceinline__ void mbar_fence_init() {
-  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-}
-__device__ __forceinline__ void fence_proxy_async() {
-  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-}
-__device__ __forceinline__ void mbar_expect_tx(u32 bar, u32 bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void bulk_g2s(u32 dst, const void* src, u32 bytes, u32 bar) {
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
-               ::"r"(dst), "l"(src), "r"(bytes), "r"(bar) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(u32 bar, u32 parity) {
-  u32 ok = 0;
-  do {
-    asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
-                 "selp.u32 %0, 1, 0, p;\n\t}" : "=r"(ok) : "r"(bar), "r"(parity) : "memory");
-  } while (!ok);
-}
 
 
 // Shared-memory vector load of thread-local vector K (2^VL elements of W bytes).

@@ -749,6 +749,33 @@ static void plan_exchange(ConvPlan& P, const ll_plan_opts* opts) {
       T.staged = true;
       T.pipe = false;
     }
+    // bulk (pipe = 4 / LL_PIPE=bulk, bulk_st also stores by bulk copy: pipe = 5 /
+    // LL_PIPE=bulkst): the CTA tile is contiguous in src-packed order (kernel load bits
+    // = the lowest n packed bits), whole tiles by cp.async.bulk into raw stages
+    const std::string pe = e ? std::string(e) : "";
+    const bool want_bulk = e ? (pe == "bulk" || pe == "bulkst") : (op == 4 || op == 5);
+    const bool want_bulk_st = e ? pe == "bulkst" : op == 5;
+    auto contiguous = [&](const std::vector<int>& bits) {
+      std::vector<int> b = bits;
+      std::sort(b.begin(), b.end());
+      for (int k = 0; k < int(b.size()); ++k) if (b[k] != k) return false;
+      return true;
+    };
+    if (want_bulk && T.ld_xcol.empty() && !T.staged && contiguous(T.ld_bit) && tile_b <= (u64(1) << 16)) {
+      // the dst stage is the exchange buffer itself (read out before it is rewritten)
+      const bool st_ok = want_bulk_st && contiguous(T.st_bit) && T.rep_bits.empty() &&
+                         (T.w << T.vst) >= 4 && T.smem_elems * u64(T.w) >= tile_b;
+      for (int ns = 3; ns >= 2; --ns) {
+        const u64 need = T.smem_elems * u64(T.w) + u64(ns) * tile_b + 8 * ns;
+        if (need <= 227 * 1024) {
+          T.bulk = true;
+          T.bulk_st = st_ok;
+          T.bulk_stages = ns;
+          T.pipe = false;
+          break;
+        }
+      }
+    }
   }
   // Resident CTAs per SM (ptxas register cap).  Linear tiles compile to 140-255
   // registers (XOR addresses that cannot fold into immediates), i.e. one CTA per SM;
@@ -767,6 +794,7 @@ static void plan_exchange(ConvPlan& P, const ll_plan_opts* opts) {
     fail(LL_ERR_UNSUPPORTED, "smem tile too large");
   P.smem_bytes = T.xchg == X_SMEM ? int(T.smem_elems * T.w) : 0;
   if (T.staged) P.smem_bytes += int(2 * (u64(1) << T.n) * u64(T.w));
+  if (T.bulk) P.smem_bytes += int(u64(T.bulk_stages) * (u64(1) << T.n) * u64(T.w) + 8 * T.bulk_stages);
 }
 
 // CTA class (Q mixes block/offset bits): choose the dst bits a CTA owns so that both
@@ -1041,6 +1069,21 @@ std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, 
         }
         build_tile(*P, S, D, gS, gD, opts, true);
         P->tile.rep_bits = rep;
+        if (!rep.empty()) {
+          // replicas: per-thread stores, plain tile loop (no staged / bulk variants);
+          // unroll up to 4 replica bits per store while the grid (data tiles x replica
+          // groups) keeps >= 8 CTAs per SM, the rest become grid bits
+          TilePlan& T = P->tile;
+          if (T.staged || T.bulk) {
+            P->smem_bytes = int(T.smem_elems * u64(T.w));
+            T.staged = T.bulk = T.bulk_st = false;
+          }
+          const int nrep = int(rep.size());
+          const int gdata = int(T.grid_dst_bit.size());
+          T.rep_lo = std::min(4, nrep);
+          while (T.rep_lo > 0 && (gdata + nrep - T.rep_lo) < 64 && (u64(1) << (gdata + nrep - T.rep_lo)) < u64(8 * 148))
+            --T.rep_lo;
+        }
         P->exec = EXEC_TILE;
         return P;
       } catch (const Error& e) {
@@ -1178,7 +1221,7 @@ std::string describe(const ConvPlan& P) {
       << ",\"ld_bit\":" << ivec_json(T.ld_bit) << ",\"st_bit\":" << ivec_json(T.st_bit)
       << ",\"L_ld\":" << vec_json(T.lcol_ld) << ",\"L_st\":" << vec_json(T.lcol_st)
       << ",\"grid_src_bit\":" << ivec_json(T.grid_src_bit) << ",\"grid_dst_bit\":" << ivec_json(T.grid_dst_bit)
-      << ",\"rep_bits\":" << ivec_json(T.rep_bits);
+      << ",\"rep_bits\":" << ivec_json(T.rep_bits) << ",\"rep_unrolled\":" << std::min<size_t>(size_t(T.rep_lo), T.rep_bits.size());
     if (!T.ld_xcol.empty())
       o << ",\"ld_xcol\":" << vec_json(T.ld_xcol) << ",\"linear_tile\":" << (T.ld_run >= 0 ? "true" : "false")
         << ",\"ld_run_bits\":" << (T.ld_run >= 0 ? T.ld_run : T.vld + 5)
@@ -1191,7 +1234,7 @@ std::string describe(const ConvPlan& P) {
     if (T.xchg == X_SMEM)
       o << ",\"Vec\":" << vec_json(T.sw_vec) << ",\"Bank\":" << vec_json(T.sw_bank) << ",\"Seg\":" << vec_json(T.sw_seg)
         << ",\"H\":" << vec_json(T.sw_H) << ",\"C\":" << vec_json(T.sw_C)
-        << ",\"smem_bytes\":" << T.smem_elems * T.w << ",\"pipe\":" << (T.pipe ? "true" : "false") << ",\"staged\":" << (T.staged ? "true" : "false") << ",\"min_blocks\":" << T.min_blocks
+        << ",\"smem_bytes\":" << T.smem_elems * T.w << ",\"pipe\":" << (T.pipe ? "true" : "false") << ",\"staged\":" << (T.staged ? "true" : "false") << ",\"bulk\":" << (T.bulk ? (T.bulk_st ? "\"load+store\"" : "\"load\"") : "false") << ",\"min_blocks\":" << T.min_blocks
         << ",\"wavefronts_st\":" << T.predicted_wavefronts_st << ",\"wavefronts_ld\":" << T.predicted_wavefronts_ld
         << ",\"ideal_wavefronts\":" << T.ideal_wavefronts
         << ",\"smem_store\":\"" << smem_instr_name(T.smi_ld, true, T.mat_sel_ld.size(), T.sm_v, T.w) << "\""

@@ -126,6 +126,10 @@ def test_noop_memcpy():
 
 
 def _full_size_every_element(sa, sb, w, nsample_seed):
+    _full_size_every_element_opts(sa, sb, w, nsample_seed)
+
+
+def _full_size_every_element_opts(sa, sb, w, nsample_seed, **opts):
     """Full-size conversion in bench.py's launch configuration (the default plan):
     src hash-filled (src[h] = H(A(h)), workloads/hashfill.py), then EVERY dst element
     compared on the device with the closed form H(B(h)) (O5), and 2^20 sampled outputs
@@ -134,7 +138,7 @@ def _full_size_every_element(sa, sb, w, nsample_seed):
     from workloads import hashfill as H
     A, OA = both(sa)
     B, OB = both(sb)
-    plan = ll.ll_plan_convert(A, B, w)
+    plan = ll.ll_plan_convert(A, B, w, **opts)
     src = H.fill(sa, w, nsample_seed)
     n = src.numel()
     dst = torch.empty_like(src)
@@ -864,3 +868,16 @@ def test_staged_exchange_gpu():
                 ll.ll_convert(d_src, d_dst, tuned)
                 torch.cuda.synchronize()
                 assert np.array_equal(from_device(d_dst, w), ref)
+
+
+@pytest.mark.parametrize("cfg", ["c3", "c3b"])
+@pytest.mark.parametrize("pipe", ["bulk", "bulkst"])
+def test_bulk_staged_smem_exchange_full_size(cfg, pipe):
+    """The bulk-staged smem exchange (src tiles by cp.async.bulk into raw stages; with
+    bulkst the dst tiles also leave by cp.async.bulk) on configs 3 / 3b at full size:
+    every element against H(B(h)) and sampled outputs against the oracle."""
+    sa, sb = {"c3": W.c3(14), "c3b": W.c3b(14)}[cfg]
+    A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
+    d = ll.ll_plan_convert(A, B, 2, pipe=pipe).describe()
+    assert d["tile"]["bulk"] == ("load" if pipe == "bulk" else "load+store")
+    _full_size_every_element_opts(sa, sb, 2, 1013, pipe=pipe)

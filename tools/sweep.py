@@ -94,6 +94,11 @@ def main():
         return generic_maps()
     if "broadcast" in only:
         return broadcast_sweep()
+    if "bulk" in only:
+        for name, (sa, sb), w in (("c3", W.c3(14), 2), ("c3b", W.c3b(14), 2)):
+            for opts in ({}, {"pipe": "bulk"}, {"pipe": "bulkst"}, {"pipe": "staged"}):
+                conv_case(name, sa, sb, w, **opts)
+        return
     if "all" not in only and "conv" not in only:
         return gather_reduce()
     # raw copy roofline reference
