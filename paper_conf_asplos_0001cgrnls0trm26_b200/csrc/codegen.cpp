@@ -70,6 +70,14 @@ std::string codegen_tile(const ConvPlan& Pl) {
   o << "  static constexpr bool PIPE = " << (T.pipe ? "true" : "false") << ";\n";
   o << "  static constexpr bool STAGED = " << (T.staged ? "true" : "false") << ";\n";
   o << "  static constexpr bool BULK = " << (T.bulk ? "true" : "false") << ";\n";
+  o << "  static constexpr bool BCAST = " << (T.bcast ? "true" : "false") << ";\n";
+  {
+    std::vector<u64> bst;
+    for (int u : T.bc_U) bst.push_back(u64(1) << (u + lw));
+    const int nk = T.bcast ? int(T.bc_U.size()) - T.bc_v - 5 - T.Wb : 0;
+    o << icon("BC_V", T.bc_v) << icon("BC_NK", nk) << arr("u64", "BC_SMW", T.bc_smw) << arr("u64", "BC_SMR", T.bc_smr)
+      << arr("u64", "BC_ST", bst);
+  }
   o << "  static constexpr bool BULK_ST = " << (T.bulk_st ? "true" : "false") << ";\n";
   o << icon("STAGES", std::max(1, T.bulk_stages)) << icon("TILE_LOG2B", T.n + lw);
   {

@@ -163,6 +163,18 @@ struct TilePlan {
   bool bulk = false;    // X_SMEM: src tiles (contiguous) streamed by cp.async.bulk into raw stages
   bool bulk_st = false; // ... and dst tiles (contiguous) leave by cp.async.bulk from a dst stage
   int bulk_stages = 0;
+  // Broadcast stores in dst order (bcast): when B has zero columns among its lowest
+  // v + 5 dst bits (inside the 16-byte store vector or the lanes), the data tile goes
+  // through shared memory in dst-data order and is read back in full dst order — the
+  // replica (zero-column) bits address the same smem element — so every thread stores
+  // whole 16-byte vectors and every warp 512 contiguous bytes.  bc_U = the store tile's
+  // dst bits (data bits of the tile ∪ low replica bits, ascending: vector, lanes, warps,
+  // then per-thread vectors); bc_smr[u] = smem element offset of U bit u (0 for a
+  // replica bit); bc_smw[b] = smem element offset written by kernel load bit b.
+  bool bcast = false;
+  int bc_v = 0;
+  std::vector<int> bc_U;
+  std::vector<u64> bc_smr, bc_smw;
 
   // --- REGPERM: out slot e <- in slot perm[e]
   std::vector<int> perm;

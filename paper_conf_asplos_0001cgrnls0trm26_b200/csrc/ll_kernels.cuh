@@ -652,6 +652,32 @@ template <int N> __device__ __forceinline__ void bulk_wait_read() {
 }
 
 
+// One w-byte element to / from shared memory (broadcast dst-order stores).
+template <int W> __device__ __forceinline__ void sts_elem(u32 addr, u32 v) {
+  if constexpr (W == 4) asm volatile("st.shared.u32 [%0], %1;" ::"r"(addr), "r"(v) : "memory");
+  else if constexpr (W == 2) asm volatile("st.shared.u16 [%0], %1;" ::"r"(addr), "h"(u16(v)) : "memory");
+  else { static_assert(W == 1, "element width"); asm volatile("st.shared.u8 [%0], %1;" ::"r"(addr), "r"(v) : "memory"); }
+}
+template <int W> __device__ __forceinline__ u32 lds_elem(u32 addr) {
+  u32 v;
+  if constexpr (W == 4) asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(addr) : "memory");
+  else if constexpr (W == 2) { u16 h; asm volatile("ld.shared.u16 %0, [%1];" : "=h"(h) : "r"(addr) : "memory"); v = h; }
+  else { static_assert(W == 1, "element width"); asm volatile("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"(addr) : "memory"); v &= 0xffu; }
+  return v;
+}
+// compile-time XOR of a column table over the set bits of an index
+template <class P, int E> struct BcW {   // smem element offset of load register slot E
+  static constexpr u32 value() { u32 o = 0; for (int b = 0; b < P::R; ++b) if ((E >> b) & 1) o ^= u32(P::BC_SMW[b]); return o; }
+};
+template <class P, int E> struct BcR {   // smem element offset of store-vector element E
+  static constexpr u32 value() { u32 o = 0; for (int b = 0; b < P::BC_V; ++b) if ((E >> b) & 1) o ^= u32(P::BC_SMR[b]); return o; }
+  // the element E' < E that reads the same smem element (a replica bit of the vector)
+  static constexpr int same() {
+    for (int b = 0; b < P::BC_V; ++b) if (((E >> b) & 1) && P::BC_SMR[b] == 0) return E & ~(1 << b);
+    return -1;
+  }
+};
+
 // ------------------------------------------------------------------ tile kernel
 // Programmatic dependent launch (sm_90+): the host launches every kernel with the
 // programmatic-stream-serialization attribute, so a kernel's CTAs may be scheduled
@@ -844,6 +870,66 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, Dst D, 
       __syncthreads();   // exchange buffer reuse by the next tile
     }
     cp_async_wait0();
+    return;
+  }
+  if constexpr (P::BCAST) {
+    // Broadcast stores in dst order (TilePlan::bcast): the data tile goes to
+    // smem in dst-data order; every thread then reads whole 16-byte dst vectors along
+    // the store tile U (replica bits add 0 to the smem offset: broadcast reads of the same
+    // element) and stores them with 512 contiguous bytes per warp instruction; replica
+    // bits above U are unrolled offsets / grid groups as in store_tile.
+    u32 thr_w = 0, thr_r = 0;
+    u64 thr_s = 0;
+    static_for<5>([&](auto q) {
+      constexpr int T = decltype(q)::value;
+      if ((lane >> T) & 1) { thr_w ^= u32(P::BC_SMW[P::R + T]); thr_r ^= u32(P::BC_SMR[P::BC_V + T]); thr_s ^= P::BC_ST[P::BC_V + T]; }
+    });
+    static_for<P::WB>([&](auto q) {
+      constexpr int T = decltype(q)::value;
+      if ((warp >> T) & 1) { thr_w ^= u32(P::BC_SMW[P::R + 5 + T]); thr_r ^= u32(P::BC_SMR[P::BC_V + 5 + T]); thr_s ^= P::BC_ST[P::BC_V + 5 + T]; }
+    });
+    constexpr int KB0 = P::BC_V + 5 + P::WB;   // first U bit of the per-thread vector index
+    for (u64 t = blockIdx.x; t < ntiles; t += gridDim.x) {
+      u32 r[P::NW];
+      load_tile(r, t);
+      static_for<(1 << P::R)>([&](auto e) {
+        constexpr int E = decltype(e)::value;
+        sts_elem<P::W>(sbase + (thr_w ^ BcW<P, E>::value()) * u32(P::W), get_e<P::W, E>(r));
+      });
+      __syncthreads();
+      const u64 td = P::NREP_HI_BITS > 0 ? (t & GMASK) : t;
+      u64 ho = 0;
+      if constexpr (P::NREP_HI_BITS > 0) {
+        const u32 rg = u32(t >> P::G);
+        static_for<P::NREP_HI_BITS>([&](auto j) {
+          constexpr int J = decltype(j)::value;
+          if ((rg >> J) & 1u) ho ^= P::REP_HI[J];
+        });
+      }
+      const u64 dbase = (tile_base<P, false>(td | tile0) ^ thr_s) ^ ho;
+#pragma unroll 4
+      for (u32 k = 0; k < (1u << P::BC_NK); ++k) {
+        u32 kr = 0;
+        u64 ks = 0;
+        static_for<P::BC_NK>([&](auto j) {
+          constexpr int J = decltype(j)::value;
+          if ((k >> J) & 1u) { kr ^= u32(P::BC_SMR[KB0 + J]); ks ^= P::BC_ST[KB0 + J]; }
+        });
+        u32 v[4] = {0u, 0u, 0u, 0u};
+        u32 ev[1 << P::BC_V];
+        static_for<(1 << P::BC_V)>([&](auto e) {
+          constexpr int E = decltype(e)::value;
+          if constexpr (BcR<P, E>::same() >= 0) ev[E] = ev[BcR<P, E>::same()];
+          else ev[E] = lds_elem<P::W>(sbase + (thr_r ^ kr ^ BcR<P, E>::value()) * u32(P::W));
+          set_e<P::W, E>(v, ev[E]);
+        });
+        static_for<P::NREP>([&](auto rp) {
+          constexpr u64 RO = P::REP_OFF[decltype(rp)::value];
+          store_vec<P::W, P::BC_V, 0, 4, P::ST_HINT>(v, D.at((dbase ^ ks) ^ RO));
+        });
+      }
+      __syncthreads();   // smem reuse by the next tile
+    }
     return;
   }
   if constexpr (P::XCHG == 3 && P::BULK) {

@@ -971,6 +971,52 @@ static bool build_linear_tile(ConvPlan& P, const ll_plan_opts* opts) {
   return true;
 }
 
+// Broadcast stores in dst order (TilePlan::bcast): used when a zero column of B lies
+// among the lowest v + 5 dst bits, where per-thread replica stores would leave holes in
+// every vector / warp instruction.  The data tile is written to smem in dst-data order
+// (bc_smw) and read back along the store tile U = data bits ∪ those low replica bits,
+// replica bits contributing 0 to the smem offset (the broadcast copies are
+// the same element).  Higher replica bits stay replica offsets (unrolled / grid).
+static void plan_bcast_store(ConvPlan& P, const ll_plan_opts* opts) {
+  TilePlan& T = P.tile;
+  const Layout& B = P.B;
+  const int w = T.w;
+  if (T.rep_bits.empty() || w > 4 || !T.ld_xcol.empty()) return;
+  const char* e = std::getenv("LL_BCAST");
+  if (e && std::string(e) == "0") return;
+  const int maxvec = default_int(opts, &ll_plan_opts::max_vec_bytes, 16);
+  const int v = std::max(0, ilog2(u64(std::max(1, maxvec / w))));
+  std::vector<int> low, high;
+  for (int r : T.rep_bits) (r < v + 5 ? low : high).push_back(r);
+  if (low.empty()) return;
+  std::vector<int> Dt(T.st_bit.begin(), T.st_bit.end());
+  std::sort(Dt.begin(), Dt.end());
+  std::vector<int> U = Dt;
+  U.insert(U.end(), low.begin(), low.end());
+  std::sort(U.begin(), U.end());
+  const int nU = int(U.size());
+  if (nU < v + 5 + T.Wb) return;
+  for (int i = 0; i < v + 5; ++i) if (U[i] != i) return;   // whole vectors and 512-byte warp runs
+  if (nU - v - 5 - T.Wb > 10) return;                       // per-thread vectors (code size)
+  auto posD = [&](int k) { return int(std::lower_bound(Dt.begin(), Dt.end(), k) - Dt.begin()); };
+  T.bc_smw.assign(T.n, 0);
+  for (int b = 0; b < T.n; ++b) {
+    int k = -1;
+    for (int d : Dt) if (B.cols[d] == T.lcol_ld[b]) k = d;
+    if (k < 0) return;                                       // not a data bit of this tile
+    T.bc_smw[b] = u64(1) << posD(k);
+  }
+  T.bc_smr.assign(nU, 0);
+  for (int u = 0; u < nU; ++u)
+    if (std::binary_search(Dt.begin(), Dt.end(), U[u])) T.bc_smr[u] = u64(1) << posD(U[u]);
+  T.bc_U = U;
+  T.bc_v = v;
+  T.bcast = true;
+  T.rep_bits = high;
+  T.staged = T.bulk = T.bulk_st = T.pipe = false;
+  P.smem_bytes = int((u64(1) << T.n) * u64(w));
+}
+
 std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, const ll_plan_opts* opts,
                                        u64 grid_only_src) {
   if (w != 1 && w != 2 && w != 4 && w != 8) fail(LL_ERR_INVALID_ARG, "elem_bytes must be 1, 2, 4 or 8");
@@ -1078,9 +1124,11 @@ std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, 
             P->smem_bytes = int(T.smem_elems * u64(T.w));
             T.staged = T.bulk = T.bulk_st = false;
           }
-          const int nrep = int(rep.size());
+          plan_bcast_store(*P, opts);
+          const int nrep = int(T.rep_bits.size());
           const int gdata = int(T.grid_dst_bit.size());
           T.rep_lo = std::min(4, nrep);
+          if (nrep == 0) T.rep_lo = 0;
           while (T.rep_lo > 0 && (gdata + nrep - T.rep_lo) < 64 && (u64(1) << (gdata + nrep - T.rep_lo)) < u64(8 * 148))
             --T.rep_lo;
         }
@@ -1221,7 +1269,9 @@ std::string describe(const ConvPlan& P) {
       << ",\"ld_bit\":" << ivec_json(T.ld_bit) << ",\"st_bit\":" << ivec_json(T.st_bit)
       << ",\"L_ld\":" << vec_json(T.lcol_ld) << ",\"L_st\":" << vec_json(T.lcol_st)
       << ",\"grid_src_bit\":" << ivec_json(T.grid_src_bit) << ",\"grid_dst_bit\":" << ivec_json(T.grid_dst_bit)
-      << ",\"rep_bits\":" << ivec_json(T.rep_bits) << ",\"rep_unrolled\":" << std::min<size_t>(size_t(T.rep_lo), T.rep_bits.size());
+      << ",\"rep_bits\":" << ivec_json(T.rep_bits) << ",\"rep_unrolled\":" << std::min<size_t>(size_t(T.rep_lo), T.rep_bits.size())
+      << ",\"bcast_store\":" << (T.bcast ? "true" : "false");
+    if (T.bcast) o << ",\"bcast_U\":" << ivec_json(T.bc_U) << ",\"bcast_v\":" << T.bc_v;
     if (!T.ld_xcol.empty())
       o << ",\"ld_xcol\":" << vec_json(T.ld_xcol) << ",\"linear_tile\":" << (T.ld_run >= 0 ? "true" : "false")
         << ",\"ld_run_bits\":" << (T.ld_run >= 0 ? T.ld_run : T.vld + 5)

@@ -54,6 +54,31 @@ void simulate_tile(const ConvPlan& P, const uint8_t* src, uint8_t* dst) {
         u64 idx = ld_xor ? ((x & ~vmask) + (a.elem ^ (x & vmask))) : (base + a.reg + a.elem);
         in[size_t(th) * E + e] = getv(src + idx * w);
       }
+    if (T.bcast) {
+      // broadcast stores in dst order: data to smem in dst-data order, then read along
+      // the store tile U (vector, lanes, warps, per-thread vectors) and stored at every
+      // remaining replica offset
+      std::vector<uint8_t> sm((u64(1) << n) * w);
+      for (int th = 0; th < NT; ++th)
+        for (int e = 0; e < E; ++e) {
+          u64 hw = u64(e) | (u64(th) << R);
+          u64 so = 0;
+          for (int b = 0; b < n; ++b) if ((hw >> b) & 1) so ^= T.bc_smw[b];
+          std::memcpy(&sm[so * w], &in[size_t(th) * E + e], w);
+        }
+      const int nU = int(T.bc_U.size());
+      for (u64 pos = 0; pos < (u64(1) << nU); ++pos) {
+        u64 so = 0, d = db;
+        for (int u = 0; u < nU; ++u)
+          if ((pos >> u) & 1) { so ^= T.bc_smr[u]; d ^= u64(1) << T.bc_U[u]; }
+        for (u64 rp = 0; rp < (u64(1) << T.rep_bits.size()); ++rp) {
+          u64 ro = 0;
+          for (size_t q = 0; q < T.rep_bits.size(); ++q) if ((rp >> q) & 1) ro |= u64(1) << T.rep_bits[q];
+          std::memcpy(dst + (d ^ ro) * w, &sm[so * w], w);
+        }
+      }
+      continue;
+    }
     if (T.xchg == X_COPY) {
       out = in;
     } else if (T.xchg == X_REGPERM) {

@@ -953,7 +953,9 @@ def test_broadcast_sweep_specialised_and_simulated(n_zero):
         w = [1, 2, 4, 8][case % 4]
         d = _sim_check(sa, sb, w, case)
         assert d["exec"] == "tile", d
-        assert len(d["tile"]["rep_bits"]) == n_zero
+        t = d["tile"]
+        low = len(t["bcast_U"]) - t["n"] if t["bcast_store"] else 0
+        assert len(t["rep_bits"]) + low == n_zero
 
 
 def test_broadcast_probe_never_generic():
