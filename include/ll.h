@@ -413,6 +413,14 @@ ll_status ll_ipc_close(void* dev_ptr);
  * every peer.  The stage handles are owned by `plan` (do not destroy them). */
 ll_status ll_plan_device_stages(const ll_plan* plan, ll_plan** pack, ll_plan** unpack,
                                 size_t* chunk_elems, int* nranks);
+/* ll_plan_device_peers: the chunk routing of a collective DEVICE plan for `rank`
+ * (SURVEY §8(e)(2)).  The pack stage leaves *nchunks (= 2^xk <= nranks) equal chunks of
+ * ll_plan_device_stages' chunk_elems; send chunk j goes to rank send_peers[j], and recv
+ * chunk i (the unpack stage's input) comes from rank recv_peers[i].  A full exchange has
+ * nchunks = nranks; a partial one (dev bits shared by A and B) talks to fewer ranks.
+ * send_peers / recv_peers: caller arrays of >= nranks ints, or NULL.
+ * Errors: INVALID_ARG (not a collective DEVICE plan, rank out of range). */
+ll_status ll_plan_device_peers(const ll_plan* plan, int rank, int* send_peers, int* recv_peers, int* nchunks);
 
 /* ---------------------------------------------------------------- test hooks --
  * ll_plan_simulate: host emulation of a specialised tile plan's schedule (the

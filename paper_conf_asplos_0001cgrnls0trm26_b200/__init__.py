@@ -97,6 +97,7 @@ _sig = {
     "ll_comm_create_loopback": [C.c_int, _PP],
     "ll_comm_check": [_P],
     "ll_plan_device_stages": [_P, _PP, _PP, C.POINTER(C.c_size_t), C.POINTER(C.c_int)],
+    "ll_plan_device_peers": [_P, C.c_int, C.POINTER(C.c_int), C.POINTER(C.c_int), C.POINTER(C.c_int)],
     "ll_comm_create_peers": [C.c_int, C.c_int, _PP, _PP, C.c_size_t, _PP],
     "ll_plan_autotune": [_P, _P, C.c_int, C.POINTER(_Opts), _P, _P, _P, C.c_int, _PP],
     "ll_ipc_export": [_P, _P],
@@ -453,6 +454,14 @@ class Plan:
         n = C.c_size_t()
         _check(_lib.ll_plan_reduce_out_elems(self.handle, C.byref(n)))
         return n.value
+
+    def device_peers(self, rank: int):
+        """(send_peers, recv_peers) of a collective DEVICE plan for `rank`: send chunk j
+        goes to send_peers[j], recv chunk i comes from recv_peers[i] (ll.h)."""
+        n = C.c_int()
+        sp, rp = (C.c_int * 64)(), (C.c_int * 64)()
+        _check(_lib.ll_plan_device_peers(self.handle, int(rank), sp, rp, C.byref(n)))
+        return list(sp[:n.value]), list(rp[:n.value])
 
     def device_stages(self):
         """(pack, unpack, chunk_elems, nranks) of a DEVICE plan; stages are None when

@@ -927,6 +927,21 @@ ll_status ll_plan_device_stages(const ll_plan* p, ll_plan** pack, ll_plan** unpa
   LL_CATCH
 }
 
+ll_status ll_plan_device_peers(const ll_plan* p, int rank, int* send_peers, int* recv_peers, int* nchunks) {
+  LL_TRY
+  if (!p || p->kind != 0 || !nchunks) fail(LL_ERR_INVALID_ARG, "bad argument");
+  const ConvPlan& P = p->cp();
+  if (P.exec != EXEC_DEVICE || P.exchange == LL_EXCHANGE_PEER) fail(LL_ERR_INVALID_ARG, "not a collective DEVICE plan");
+  if (rank < 0 || rank >= P.nranks) fail(LL_ERR_INVALID_ARG, "rank out of range");
+  const int n = 1 << P.xk;
+  *nchunks = n;
+  for (int j = 0; j < n; ++j) {
+    if (send_peers) send_peers[j] = P.send_peer(u64(j), rank);
+    if (recv_peers) recv_peers[j] = P.recv_peer(u64(j), rank);
+  }
+  LL_CATCH
+}
+
 ll_status ll_plan_simulate(const ll_plan* p, const void* src, void* dst) {
   LL_TRY
   if (!p || p->kind != 0 || !src || !dst) fail(LL_ERR_INVALID_ARG, "bad argument");

@@ -226,16 +226,42 @@ void plan_device(ConvPlan& P, const ll_plan_opts* opts) {
   std::vector<u64> a(p), b(p);
   for (int t = 0; t < p; ++t) { a[t] = A.cols[pa + t]; b[t] = B.cols[pb + t]; }
   auto in = [](const std::vector<u64>& v, u64 c) { return std::find(v.begin(), v.end(), c) != v.end(); };
-  for (int t = 0; t < p; ++t) {
-    if (!in(Bl.cols, a[t]) || !in(Al.cols, b[t]))
-      fail(LL_ERR_UNSUPPORTED, "DEVICE: partial device exchanges (dev bits shared by A and B) are not supported");
+  // Logical bits by where they live: LL (local in both), LD (A-local, B-dev: they pick
+  // the receiver), DL (A-dev, B-local: they pick the sender), DD (a dev bit of both: the
+  // rank bit is fixed or relabelled, SURVEY §8(e)(2) partial exchange).  Rank r sends
+  // 2^xk chunks (xk = |LD| = |DL|) to the ranks whose B-dev coordinates agree with r on
+  // the DD columns, and receives 2^xk chunks from the ranks whose A-dev coordinates agree
+  // with r's B-dev coordinates there; all chunks are equal (bijective layouts).
+  std::vector<u64> LD, DL;
+  for (int t = 0; t < p; ++t) if (in(Al.cols, b[t])) LD.push_back(b[t]);   // B-dev order
+  for (int t = 0; t < p; ++t) if (in(Bl.cols, a[t])) DL.push_back(a[t]);   // A-dev order
+  if (LD.size() != DL.size()) fail(LL_ERR_UNSUPPORTED, "DEVICE: unequal send / receive bits (internal)");
+  const int xk = int(LD.size());
+  P.xk = xk;
+  P.send_jcol.assign(xk, 0);
+  P.send_rcol.assign(p, 0);
+  P.recv_icol.assign(xk, 0);
+  P.recv_rcol.assign(p, 0);
+  {
+    int j = 0;
+    for (int t = 0; t < p; ++t) {
+      if (in(Al.cols, b[t])) { P.send_jcol[j++] = 1u << t; continue; }
+      // DD: receiver's B-dev bit t = sender's A-dev bit t' with the same column
+      for (int t2 = 0; t2 < p; ++t2) if (a[t2] == b[t]) P.send_rcol[t2] ^= 1u << t;
+    }
+    int i = 0;
+    for (int t = 0; t < p; ++t) {
+      if (in(Bl.cols, a[t])) { P.recv_icol[i++] = 1u << t; continue; }
+      // DD: sender's A-dev bit t = receiver's B-dev bit t' with the same column
+      for (int t2 = 0; t2 < p; ++t2) if (b[t2] == a[t]) P.recv_rcol[t2] ^= 1u << t;
+    }
   }
-  // C_B: B-local vectors that are A-local too, in B's order
+  // C: B-local vectors that are A-local too (LL), in B's order
   std::vector<u64> C;
   for (u64 c : Bl.cols) if (!in(a, c)) C.push_back(c);
   std::vector<u64> scols = C, rcols = C;
-  scols.insert(scols.end(), b.begin(), b.end());   // send: receiver rank bits on top
-  rcols.insert(rcols.end(), a.begin(), a.end());   // recv: source rank bits on top
+  scols.insert(scols.end(), LD.begin(), LD.end());   // send: chunk (receiver) bits on top
+  rcols.insert(rcols.end(), DL.begin(), DL.end());   // recv: chunk (sender) bits on top
   Layout S = memory_layout(scols, A.out), R = memory_layout(rcols, A.out);
   ll_plan_opts lo;
   std::memset(&lo, 0, sizeof lo);
@@ -255,7 +281,7 @@ void plan_device(ConvPlan& P, const ll_plan_opts* opts) {
   P.nranks = comm->nranks;
   P.comm = comm;
   P.local_elems = u64(1) << nloc;
-  P.chunk_elems = u64(1) << (nloc - p);
+  P.chunk_elems = u64(1) << (nloc - xk);
   const size_t lb = size_t(P.local_elems) * P.w;
   const size_t per_rank = (P.pack ? lb : 0) + (P.unpack ? lb : 0);
   P.workspace_bytes = comm->loopback ? per_rank * comm->nranks : per_rank;
@@ -322,20 +348,27 @@ ll_status device_convert(const ConvPlan& Pc, const void* src, void* dst, void* w
   if (P.pack)
     for (int r = 0; r < nloc_ranks; ++r)
       convert_impl(static_cast<const char*>(src) + r * lb, const_cast<char*>(sendbuf(r)), nullptr, *P.pack, st);
-  // 2. exchange: chunk q of rank s's send buffer -> chunk s of rank q's recv buffer
+  // 2. exchange: send chunk j of rank s -> rank q = send_peer(j, s), which files it as
+  // its recv chunk i with recv_peer(i, q) = s (all 2^xk chunks equal; grouped point-to-
+  // point, so partial exchanges only talk to the ranks they share data with)
+  const u64 nch = u64(1) << P.xk;
   if (comm->loopback) {
     for (int s = 0; s < N; ++s)
-      for (int q = 0; q < N; ++q) {
-        cudaError_t e = cudaMemcpyAsync(recvbuf(q) + s * cb, sendbuf(s) + q * cb, cb, cudaMemcpyDeviceToDevice, st);
+      for (u64 j = 0; j < nch; ++j) {
+        const int q = P.send_peer(j, s);
+        u64 i = 0;
+        while (i < nch && P.recv_peer(i, q) != s) ++i;
+        if (i == nch) fail(LL_ERR_UNSUPPORTED, "DEVICE: inconsistent chunk routing (internal)");
+        cudaError_t e = cudaMemcpyAsync(recvbuf(q) + i * cb, sendbuf(s) + j * cb, cb, cudaMemcpyDeviceToDevice, st);
         if (e != cudaSuccess) fail(LL_ERR_CUDA, std::string("loopback exchange: ") + cudaGetErrorString(e));
       }
   } else {
     Nccl& n = nccl();
     check_nccl(n.groupStart(), "ncclGroupStart");
-    for (int q = 0; q < N; ++q) {
-      check_nccl(n.send(sendbuf(0) + q * cb, cb, /*ncclInt8*/ 0, q, comm->nccl, st), "ncclSend");
-      check_nccl(n.recv(recvbuf(0) + q * cb, cb, 0, q, comm->nccl, st), "ncclRecv");
-    }
+    for (u64 j = 0; j < nch; ++j)
+      check_nccl(n.send(sendbuf(0) + j * cb, cb, /*ncclInt8*/ 0, P.send_peer(j, comm->rank), comm->nccl, st), "ncclSend");
+    for (u64 i = 0; i < nch; ++i)
+      check_nccl(n.recv(recvbuf(0) + i * cb, cb, 0, P.recv_peer(i, comm->rank), comm->nccl, st), "ncclRecv");
     check_nccl(n.groupEnd(), "ncclGroupEnd");
     // an earlier asynchronous NCCL failure on this communicator surfaces here
     int aerr = 0;

@@ -230,6 +230,23 @@ struct ConvPlan {
   ll_comm* comm = nullptr;
   std::unique_ptr<ConvPlan> pack, unpack;   // local stages of a DEVICE plan (null = identity)
   u64 chunk_elems = 0;                      // elements exchanged with every peer
+  // Partial exchanges (dev bits shared by A and B): 2^xk chunks per
+  // rank.  Send chunk j of rank r goes to rank (XOR of send_jcol over j's bits) ^ (XOR
+  // of send_rcol over r's bits); recv chunk i of rank r comes from the analogous rank.
+  int xk = 0;
+  std::vector<uint32_t> send_jcol, send_rcol, recv_icol, recv_rcol;
+  int send_peer(u64 j, int r) const {
+    uint32_t q = 0;
+    for (size_t b = 0; b < send_jcol.size(); ++b) if ((j >> b) & 1) q ^= send_jcol[b];
+    for (size_t b = 0; b < send_rcol.size(); ++b) if ((r >> b) & 1) q ^= send_rcol[b];
+    return int(q);
+  }
+  int recv_peer(u64 i, int r) const {
+    uint32_t q = 0;
+    for (size_t b = 0; b < recv_icol.size(); ++b) if ((i >> b) & 1) q ^= recv_icol[b];
+    for (size_t b = 0; b < recv_rcol.size(); ++b) if ((r >> b) & 1) q ^= recv_rcol[b];
+    return int(q);
+  }
   int nranks = 1;
   u64 local_elems = 0;
   // DEVICE plans executed as peer stores (§8(f) N4): `fused` is one tile plan over the

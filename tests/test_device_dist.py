@@ -32,6 +32,10 @@ def _rank_src(OA, T, r):
     return T[xs.astype(np.int64)]
 
 
+def src_elems(OA):
+    return 1 << (OA.d_in - len(OA.dim_bits("dev")))
+
+
 def _worker(rank, world, port, n, q):
     import torch
     import torch.distributed as dist
@@ -40,8 +44,10 @@ def _worker(rank, world, port, n, q):
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
         p = world.bit_length() - 1
-        for make in (W.c5, W.c5T):
-            sa, sb = make(p, n=n)
+        cases = [W.c5(p, n=n), W.c5T(p, n=n)]
+        if p >= 2:
+            cases += [W.c5_partial(p, n=n), W.c5_partial(p, n=n, swap=True)]
+        for sa, sb in cases:
             OA, OB = O.Layout(*W.spec_to_bases(sa)), O.Layout(*W.spec_to_bases(sb))
             A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
             # the communicator handle is only consulted for its size at plan time
@@ -49,17 +55,27 @@ def _worker(rank, world, port, n, q):
             assert plan.cls == "DEVICE"
             pack, unpack, chunk, nr = plan.device_stages()
             assert nr == world
+            sp, rp = plan.device_peers(rank)
+            assert len(sp) * chunk == len(rp) * chunk == src_elems(OA)
             T = gen.random_bits(np.random.default_rng(1006), 1 << (2 * n), 2)
             src = _rank_src(OA, T, rank)
             send = pack.simulate(src, src.size) if pack else src
+            # all_to_all_single takes chunks in rank order: send chunk j to sp[j], file
+            # the chunk from rp[i] as recv chunk i (ranks outside the routing get 0);
             # gloo has no 16-bit all_to_all: move the bf16 bits as int32 pairs
-            recv = torch.empty(src.size // 2, dtype=torch.int32)
-            dist.all_to_all_single(recv, torch.from_numpy(send.view(np.int32).copy()),
-                                   [chunk // 2] * world, [chunk // 2] * world)
-            recv = recv.numpy().view(np.uint16)
+            c2 = chunk // 2
+            sv = send.view(np.int32).reshape(len(sp), c2)
+            order = sorted(range(len(sp)), key=lambda j: sp[j])
+            insz = [c2 if q in sp else 0 for q in range(world)]
+            outsz = [c2 if q in rp else 0 for q in range(world)]
+            recv_t = torch.empty(len(rp) * c2, dtype=torch.int32)
+            dist.all_to_all_single(recv_t, torch.from_numpy(np.ascontiguousarray(sv[order]).reshape(-1)),
+                                   outsz, insz)
+            by_src = dict(zip(sorted(rp), recv_t.numpy().reshape(len(rp), c2)))
+            recv = np.concatenate([by_src[rp[i]] for i in range(len(rp))]).view(np.uint16)
             got = unpack.simulate(recv, recv.size) if unpack else recv
             want = O.convert_distributed_rank(OA, OB, T, rank)
-            assert np.array_equal(got, want), (make.__name__, rank)
+            assert np.array_equal(got, want), (sa, rank)
         q.put((rank, "ok"))
     except Exception as e:  # pragma: no cover - reported to the parent
         q.put((rank, repr(e)))
@@ -82,6 +98,32 @@ def test_device_decomposition_gloo(world):
     assert all(v == "ok" for v in res.values()), res
 
 
+def test_partial_exchange_routing():
+    """Partial exchanges: with the top row bit a dev bit of both A and
+    B, each rank sends to and receives from 2^(p-1) ranks — exactly those that agree with
+    it on the shared bit (at the same rank position, or moved to rank bit 0 by swap) —
+    and every (sender, receiver) pair is routed once."""
+    for p in (2, 3):
+        for swap in (False, True):
+            sa, sb = W.c5_partial(p, n=6, swap=swap)
+            plan = ll.ll_plan_convert(ll.Layout.from_spec(sa), ll.Layout.from_spec(sb), 2,
+                                      comm=ll.Comm.loopback(1 << p))
+            assert plan.cls == "DEVICE"
+            _, _, chunk, nr = plan.device_stages()
+            assert chunk == 1 << (12 - p - (p - 1))
+            pairs = set()
+            for r in range(nr):
+                sp, rp = plan.device_peers(r)
+                assert len(sp) == len(rp) == 1 << (p - 1)
+                top = (r >> (p - 1)) & 1
+                for q in sp:
+                    assert ((q >> (0 if swap else p - 1)) & 1) == top
+                    pairs.add((r, q))
+            for r in range(nr):
+                for s in plan.device_peers(r)[1]:
+                    assert (s, r) in pairs
+
+
 def test_device_plan_errors():
     sa, sb = W.c5(1, n=4)
     A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
@@ -101,12 +143,17 @@ def test_device_p1_is_noop_and_5T_is_cta():
 
 @pytest.mark.gpu
 @pytest.mark.parametrize("p", [1, 2, 3])
-@pytest.mark.parametrize("make", ["c5", "c5T"])
+@pytest.mark.parametrize("make", ["c5", "c5T", "c5_partial", "c5_partial_swap"])
 def test_device_loopback_gpu(p, make):
     import torch
     from tests._util import empty_device, from_device, to_device
     n = 9
-    sa, sb = getattr(W, make)(p, n=n)
+    if make.startswith("c5_partial"):
+        if p < 2:
+            pytest.skip("partial exchanges need >= 2 dev bits")
+        sa, sb = W.c5_partial(p, n=n, swap=make.endswith("swap"))
+    else:
+        sa, sb = getattr(W, make)(p, n=n)
     OA, OB = O.Layout(*W.spec_to_bases(sa)), O.Layout(*W.spec_to_bases(sb))
     A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
     P = 1 << p

@@ -222,3 +222,19 @@ def n2_acc_to_lhs(bits: int, nb: int = 14):
     else:
         raise ValueError(bits)
     return A, B
+
+
+# ---- §8(e)(2): partial device exchanges (a dev bit shared by A and B) ----
+def c5_partial(p: int, n: int = 15, swap: bool = False):
+    """Config 5 with the top row bit i_{n-1} a device bit of BOTH layouts (p >= 2): A is
+    row-sharded over (i_{n-p} .. i_{n-1}); B moves the low p-1 of those rows into its
+    offset and shards its columns j_{n-p+1} .. j_{n-1} instead, keeping i_{n-1} as a dev
+    bit — at the same position (rank bit p-1) or, with swap, as rank bit 0.  Each rank
+    then exchanges with 2^(p-1) ranks, not 2^p: a partial exchange."""
+    assert p >= 2
+    out = [("i", n), ("j", n)]
+    A = {"out": out, "in": [("offset", _b("j", 0, n) + _b("i", 0, n - p)), ("dev", _b("i", n - p, n))]}
+    jdev = _b("j", n - p + 1, n)
+    bdev = (["i" + str(n - 1)] + jdev) if swap else (jdev + ["i" + str(n - 1)])
+    B = {"out": out, "in": [("offset", _b("j", 0, n - p + 1) + _b("i", 0, n - 1)), ("dev", bdev)]}
+    return A, B
