@@ -448,6 +448,34 @@ def other_configs(ll, W, torch, peak):
                     "size_matched_copy_GBps": size_matched_copy(torch, 8 * n)})
         del sets, rsets, ssets
     torch.cuda.empty_cache()
+    # the same gather / reduce / scan kernels at 1 GiB of input (2^28 fp32, [32768, 8192]
+    # in the same tiles): their own ceiling, free of the small problem's launch / ramp
+    for fam in ("mma", "blocked"):
+        L = ll.Layout.from_spec(W.c4("gather", fam, n_i=15, n_j=13))
+        p = ll.ll_plan_gather(L, 1, 4)
+        n = 1 << L.d_in
+        s0 = torch.randint(-2 ** 31, 2 ** 31 - 1, (n,), dtype=torch.int32, device="cuda")
+        i0 = torch.randint(0, 32, (n,), dtype=torch.int32, device="cuda")
+        o0 = torch.empty(n, dtype=torch.int32, device="cuda")
+        ms = _time_stream(lambda: ll.ll_gather(s0, i0, o0, p), torch, batch=3)
+        out.append({"workload": f"config 4 gather at 1 GiB: [32768,8192] fp32, {fam} [128,32] tiles", "class": "gather",
+                    "ms": round(ms, 4), "GBps": round(12 * n / ms / 1e6, 1), "frac": round(12 * n / ms / 1e6 / peak, 3)})
+        del s0, i0, o0
+        L = ll.Layout.from_spec(W.c4("reduce", fam, n_i=15, n_j=13))
+        p = ll.ll_plan_reduce(L, 1)
+        s0 = torch.rand(n, device="cuda")
+        o0 = torch.empty(p.out_elems(), device="cuda")
+        ms = _time_stream(lambda: ll.ll_reduce(s0, o0, p), torch, batch=3)
+        gbs = (4 * n + 4 * p.out_elems()) / ms / 1e6
+        out.append({"workload": f"config 4 reduce at 1 GiB: [32768,8192] fp32 -> [32768,64], {fam} [128,128] tiles",
+                    "class": "reduce", "ms": round(ms, 4), "GBps": round(gbs, 1), "frac": round(gbs / peak, 3)})
+        p = ll.ll_plan_scan(L, 1)
+        o1 = torch.empty_like(s0)
+        ms = _time_stream(lambda: ll.ll_scan(s0, o1, p), torch, batch=3)
+        out.append({"workload": f"config 4 scan at 1 GiB: [32768,8192] fp32, {fam} [128,128] tiles", "class": "scan",
+                    "ms": round(ms, 4), "GBps": round(8 * n / ms / 1e6, 1), "frac": round(8 * n / ms / 1e6 / peak, 3)})
+        del s0, o0, o1
+        torch.cuda.empty_cache()
     return out
 
 
