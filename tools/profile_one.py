@@ -36,7 +36,20 @@ conv = {"c2": (W.c2(16), 2, {}), "c2smem": (W.c2(16), 2, {"force_class": "SMEM"}
         "c2fsmemvec": (W.c2(16), 2, {"sigma": "faithful", "force_class": "SMEM", "smem_instr": "vec"}),
         "c3f": (W.c3(14), 2, {"sigma": "faithful"}),
         "c3fvec": (W.c3(14), 2, {"sigma": "faithful", "smem_instr": "vec"})}
-if a.case == "c5peer":
+if a.case.startswith("bcast"):
+    # the bench's broadcast row: random bijective A -> B with 8 zero columns (seed 908)
+    import numpy as np
+    from workloads import gen
+    sa, sb = gen.random_broadcast_pair(np.random.default_rng(int(a.case[5:] or 908)), 8, ki=5, kj=5, batch_bits=11)
+    import json
+    p = ll.ll_plan_convert(ll.Layout.from_spec(sa), ll.Layout.from_spec(sb), 4, **json.loads(a.opts))
+    A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
+    src = torch.randint(-2 ** 31, 2 ** 31 - 1, (1 << A.d_in,), dtype=torch.int32, device="cuda")
+    dst = torch.empty(1 << B.d_in, dtype=torch.int32, device="cuda")
+    for _ in range(a.iters):
+        ll.ll_convert(src, dst, p)
+    torch.cuda.synchronize()
+elif a.case == "c5peer":
     # config 5 at P = 8 on one GPU (loopback): one peer-store tile kernel per virtual rank
     sa, sb = W.c5(3)
     p = ll.ll_plan_convert(ll.Layout.from_spec(sa), ll.Layout.from_spec(sb), 2, comm=ll.Comm.loopback(8),
