@@ -40,7 +40,11 @@ if a.case.startswith("bcast"):
     # the bench's broadcast row: random bijective A -> B with 8 zero columns (seed 908)
     import numpy as np
     from workloads import gen
-    sa, sb = gen.random_broadcast_pair(np.random.default_rng(int(a.case[5:] or 908)), 8, ki=5, kj=5, batch_bits=11)
+    # bcast<seed>: the bench size (8 MiB -> 2 GiB); bcastS<seed>: 2 batch bits (sanitizer size)
+    small = a.case.startswith("bcastS")
+    seed = int(a.case[6:] if small else a.case[5:] or 908)
+    sa, sb = gen.random_broadcast_pair(np.random.default_rng(seed), 8 if not small else 5, ki=5, kj=5,
+                                       batch_bits=2 if small else 11)
     import json
     p = ll.ll_plan_convert(ll.Layout.from_spec(sa), ll.Layout.from_spec(sb), 4, **json.loads(a.opts))
     A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
