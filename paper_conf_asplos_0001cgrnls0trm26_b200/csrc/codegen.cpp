@@ -136,6 +136,9 @@ std::string codegen_tile(const ConvPlan& Pl) {
   for (size_t t = nlo; t < rb.size(); ++t) rep_hi.push_back(u64(1) << (rb[t] + lw));
   o << icon("NREP", rep.size()) << arr("u64", "REP_OFF", rep)
     << icon("NREP_HI_BITS", rep_hi.size()) << arr("u64", "REP_HI", rep_hi);
+  // element permutations around a sub-word shuffle (plan_shuffle_eperm)
+  o << "  static constexpr bool EPERM = " << (T.pre_eperm.empty() ? "false" : "true") << ";\n"
+    << arr("int", "PRE_EPERM", T.pre_eperm) << arr("int", "POST_EPERM", T.post_eperm);
   // REGPERM
   o << arr("int", "PERM", T.perm);
   // SHUFFLE

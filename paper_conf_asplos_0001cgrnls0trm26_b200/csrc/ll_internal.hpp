@@ -189,6 +189,12 @@ struct TilePlan {
   uint32_t src_lane_col[5] = {0, 0, 0, 0, 0};  // linear part: lane bit t -> XOR
   std::vector<uint32_t> pre_lmask, post_lmask; // per stage: lane mask (parity predicate)
   std::vector<int> pre_x, post_x;              // per stage: slot XOR constant
+  // Sub-word elements (w < 4) whose common 32-bit unit V is not the lowest register
+  // bits of a side: thread-local element permutations (byte permutes) around the
+  // shuffle.  pre_eperm[e'] = the loaded register element that becomes element e' of
+  // the shuffle's input; post_eperm[e] = the shuffle-output element stored as e.
+  // Empty = identity.
+  std::vector<int> pre_eperm, post_eperm;
 
   // --- SMEM: smem layout M: offset bits (Vec, Bank, Seg)
   std::vector<u64> sw_vec, sw_bank, sw_seg, sw_H, sw_C;

@@ -923,9 +923,13 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, Dst D, 
           else ev[E] = lds_elem<P::W>(sbase + (thr_r ^ kr ^ BcR<P, E>::value()) * u32(P::W));
           set_e<P::W, E>(v, ev[E]);
         });
+        // replica offsets are disjoint from the tile / thread / vector bits: one base
+        // pointer plus compile-time offsets (immediates, no per-store address registers
+        // held by in-flight stores)
+        u8* const pv = D.at(dbase ^ ks);
         static_for<P::NREP>([&](auto rp) {
           constexpr u64 RO = P::REP_OFF[decltype(rp)::value];
-          store_vec<P::W, P::BC_V, 0, 4, P::ST_HINT>(v, D.at((dbase ^ ks) ^ RO));
+          store_vec<P::W, P::BC_V, 0, 4, P::ST_HINT>(v, pv + RO);
         });
       }
       __syncthreads();   // smem reuse by the next tile
@@ -1036,7 +1040,23 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, Dst D, 
       static_for<P::NW>([&](auto q) { o[decltype(q)::value] = 0; });
       xchg_regperm<P>(r, o);
     } else if constexpr (P::XCHG == 2) {
-      xchg_shuffle<P>(r, o, lane);
+      if constexpr (P::EPERM) {
+        // thread-local element permutations: the common 32-bit unit to the lowest
+        // register bits before the shuffle, the store order after it
+        u32 r2[P::NW], o2[P::NW];
+        static_for<P::NW>([&](auto q) { r2[decltype(q)::value] = 0; o[decltype(q)::value] = 0; });
+        static_for<(1 << P::R)>([&](auto e) {
+          constexpr int E = decltype(e)::value;
+          set_e<P::W, E>(r2, get_e<P::W, P::PRE_EPERM[E]>(r));
+        });
+        xchg_shuffle<P>(r2, o2, lane);
+        static_for<(1 << P::R)>([&](auto e) {
+          constexpr int E = decltype(e)::value;
+          set_e<P::W, E>(o, get_e<P::W, P::POST_EPERM[E]>(o2));
+        });
+      } else {
+        xchg_shuffle<P>(r, o, lane);
+      }
     } else {
       static_for<P::NW>([&](auto q) { o[decltype(q)::value] = 0; });
       xchg_smem<P>(r, o, lane, warp, sbase);

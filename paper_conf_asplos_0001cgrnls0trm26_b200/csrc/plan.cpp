@@ -364,6 +364,77 @@ static bool plan_shuffle(TilePlan& T) {
   return true;
 }
 
+// Shuffles of sub-word elements (w < 4) whose 32-bit unit is not common at the lowest
+// register bits (reading R-V): choose the unit V among the logical vectors common to
+// both sides' registers (in L_ld's register order), move it to the lowest
+// register bits of each side by a thread-local element permutation (prmt / bit-field
+// moves — the "prmt.b32 when sub-32-bit elements change position" of row a6), and plan
+// the paper's shuffle between the permuted layouts.
+static bool plan_shuffle_eperm(TilePlan& T) {
+  const int R = T.R, w = T.w;
+  if (w >= 4) return false;
+  const int u = ilog2(u64(4 / w));
+  if (u > R) return false;
+  std::vector<int> common;   // L_ld register positions whose column is a register of L_st
+  for (int b = 0; b < R; ++b)
+    for (int c = 0; c < R; ++c) if (T.lcol_ld[b] == T.lcol_st[c]) common.push_back(b);
+  if (int(common.size()) < u) return false;
+  const std::vector<u64> ld0 = T.lcol_ld, st0 = T.lcol_st;
+  auto reorder = [&](const std::vector<u64>& lc, const std::vector<u64>& V, std::vector<int>& perm_bits) {
+    // new register order: V first (in V's order), then the other registers ascending
+    std::vector<int> order;
+    for (u64 c : V) for (int b = 0; b < R; ++b) if (lc[b] == c) order.push_back(b);
+    for (int b = 0; b < R; ++b) if (std::find(order.begin(), order.end(), b) == order.end()) order.push_back(b);
+    perm_bits = order;   // new register bit k = old register bit order[k]
+    std::vector<u64> out = lc;
+    for (int k = 0; k < R; ++k) out[k] = lc[order[k]];
+    return out;
+  };
+  // element e' of the new order = element e of the old order with bit order[k] = bit k of e'
+  auto eperm = [&](const std::vector<int>& order) {
+    std::vector<int> src(size_t(1) << R);
+    for (int e2 = 0; e2 < (1 << R); ++e2) {
+      int e = 0;
+      for (int k = 0; k < R; ++k) if ((e2 >> k) & 1) e |= 1 << order[k];
+      src[e2] = e;
+    }
+    return src;
+  };
+  // candidate units: u-subsets of the common vectors, in L_ld's register order
+  std::vector<int> pick(u);
+  std::function<bool(int, int)> rec = [&](int start, int k) -> bool {
+    if (k == u) {
+      std::vector<u64> V;
+      for (int b : pick) V.push_back(ld0[b]);
+      std::vector<int> oa, ob;
+      T.lcol_ld = reorder(ld0, V, oa);
+      T.lcol_st = reorder(st0, V, ob);
+      if (plan_shuffle(T)) {
+        T.pre_eperm = eperm(oa);
+        // shuffle output (new st order) element e2 holds old-st element eperm(ob)[e2]:
+        // the stored element e takes the e2 with eperm(ob)[e2] = e
+        const std::vector<int> fwd = eperm(ob);
+        T.post_eperm.assign(fwd.size(), 0);
+        for (size_t e2 = 0; e2 < fwd.size(); ++e2) T.post_eperm[fwd[e2]] = int(e2);
+        T.lcol_ld = ld0;
+        T.lcol_st = st0;
+        return true;
+      }
+      return false;
+    }
+    for (size_t i = start; i < common.size(); ++i) {
+      pick[k] = common[i];
+      if (rec(int(i) + 1, k + 1)) return true;
+    }
+    return false;
+  };
+  const bool ok = rec(0, 0);
+  T.lcol_ld = ld0;
+  T.lcol_st = st0;
+  if (!ok) { T.pre_eperm.clear(); T.post_eperm.clear(); }
+  return ok;
+}
+
 // Simulated wavefront count (Lemma 9.4 model) of a kernel layout
 // accessing smem through offsets `smoff` (per kernel bit) with `v` vector bits.
 static long sim_wavefronts(const TilePlan& T, const std::vector<u64>& smoff,
@@ -710,6 +781,8 @@ static void plan_exchange(ConvPlan& P, const ll_plan_opts* opts) {
   } else if (same_lane && same_warp) {
     T.xchg = same_reg ? X_COPY : X_REGPERM;
   } else if (same_warp && plan_shuffle(T)) {
+    T.xchg = X_SHUFFLE;
+  } else if (same_warp && plan_shuffle_eperm(T)) {
     T.xchg = X_SHUFFLE;
   } else {
     if (force == LL_CLASS_SHUFFLE) fail(LL_ERR_UNSUPPORTED, "SHUFFLE forced but the kernel layouts need smem");

@@ -86,6 +86,12 @@ void simulate_tile(const ConvPlan& P, const uint8_t* src, uint8_t* dst) {
         for (int e = 0; e < E; ++e) out[size_t(th) * E + e] = in[size_t(th) * E + T.perm[e]];
     } else if (T.xchg == X_SHUFFLE) {
       const int U = T.unit_elems;
+      if (!T.pre_eperm.empty()) {
+        std::vector<uint64_t> tmp(in.size());
+        for (int th = 0; th < NT; ++th)
+          for (int e = 0; e < E; ++e) tmp[size_t(th) * E + e] = in[size_t(th) * E + T.pre_eperm[e]];
+        in.swap(tmp);
+      }
       for (int wp = 0; wp < (1 << T.Wb); ++wp) {
         // pre network: slot j <-> j ^ X when parity(lane & mask)
         auto net = [&](std::vector<uint64_t>& buf, const std::vector<uint32_t>& mk, const std::vector<int>& xs) {
@@ -117,6 +123,12 @@ void simulate_tile(const ConvPlan& P, const uint8_t* src, uint8_t* dst) {
             for (int q = 0; q < U; ++q)
               out[size_t(wp * 32 + l) * E + T.recv_slot[rr] * U + q] = in[size_t(wp * 32 + l) * E + T.send_slot[rr] * U + q];
         net(out, T.post_lmask, T.post_x);
+      }
+      if (!T.post_eperm.empty()) {
+        std::vector<uint64_t> tmp(out.size());
+        for (int th = 0; th < NT; ++th)
+          for (int e = 0; e < E; ++e) tmp[size_t(th) * E + e] = out[size_t(th) * E + T.post_eperm[e]];
+        out.swap(tmp);
       }
     } else {
       for (int th = 0; th < NT; ++th)

@@ -914,7 +914,7 @@ def test_planned_wavefronts_equal_ncu_sass_counts():
     path = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles",
                         "r01_smem_sass_wavefronts.json")
     m = json.load(open(path))["cases"]
-    cases = {"c3": (W.c3(14), 2, {}), "c3b": (W.c3b(14), 2, {}), "c5T": (W.c5T(0, n=15), 2, {}),
+    cases = {"c3": (W.c3(14), 2, {}), "c3b": (W.c3b(14), 2, {"force_class": "SMEM"}), "c5T": (W.c5T(0, n=15), 2, {}),
              "n1": (W.n1_preshuffle(14, 14), 2, {}), "c1bsmem": (W.c1_batched(20), 4, {"force_class": "SMEM"}),
              "c2smem": (W.c2(16), 2, {"force_class": "SMEM"}), "c3f": (W.c3(14), 2, {"sigma": "faithful"})}
     assert sorted(cases) == sorted(m)

@@ -94,6 +94,12 @@ def main():
         return generic_maps()
     if "broadcast" in only:
         return broadcast_sweep()
+    if "eperm" in only:
+        # sub-word shuffles with element permutations (plan_shuffle_eperm) vs the smem exchange
+        for name, (sa, sb), w in (("c3b", W.c3b(14), 2), ("acc_fp8", W.n2_acc_to_lhs(8, 18), 1)):
+            for opts in ({}, {"force_class": "SMEM"}, {"sigma": "faithful"}):
+                conv_case(name, sa, sb, w, **opts)
+        return
     if "bulk" in only:
         for name, (sa, sb), w in (("c3", W.c3(14), 2), ("c3b", W.c3b(14), 2)):
             for opts in ({}, {"pipe": "bulk"}, {"pipe": "bulkst"}, {"pipe": "staged"}):
