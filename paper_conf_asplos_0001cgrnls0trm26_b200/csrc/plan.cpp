@@ -782,7 +782,10 @@ static void plan_exchange(ConvPlan& P, const ll_plan_opts* opts) {
     T.xchg = same_reg ? X_COPY : X_REGPERM;
   } else if (same_warp && plan_shuffle(T)) {
     T.xchg = X_SHUFFLE;
-  } else if (same_warp && plan_shuffle_eperm(T)) {
+  } else if (same_warp && P.cls <= LL_CLASS_SHUFFLE && plan_shuffle_eperm(T)) {
+    // only where the paper's class is SHUFFLE: measured against the smem exchange, the
+    // permuted shuffle wins on the fp8 operand conversion (6365 vs 6099 GB/s) and loses
+    // where the class is SMEM (config 3b: 5968 vs 6338; profiles/r02_sweep_eperm.jsonl)
     T.xchg = X_SHUFFLE;
   } else {
     if (force == LL_CLASS_SHUFFLE) fail(LL_ERR_UNSUPPORTED, "SHUFFLE forced but the kernel layouts need smem");
