@@ -681,6 +681,10 @@ ll_status ll_plan_autotune(const ll_layout* A, const ll_layout* B, int w, const 
     const size_t nc = cand.size();
     for (size_t i = 0; i < nc; ++i) { ll_plan_opts c = cand[i]; c.force_class = LL_CLASS_SMEM; cand.push_back(c); }
   }
+  // the layouts' own registers (faithful σ) against the coalesced decomposition: the
+  // permuted fp8 operand shuffle measured 6656 vs 6365 GB/s faithful vs coalesced
+  // (profiles/r02_sweep_eperm.jsonl); identical plans are timed once
+  if (o0.sigma == SIGMA_COALESCED) { ll_plan_opts c = o0; c.sigma = SIGMA_FAITHFUL; cand.push_back(c); }
   // smem instructions (Thm 5.1): the automatic stmatrix / ldmatrix choice against
   // vectorised ld/st.shared only (identical plans are timed once)
   if (o0.smem_instr == 0) {

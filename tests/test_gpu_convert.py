@@ -607,11 +607,13 @@ def test_e1_exhaustive_generic_gpu():
     assert bad.size == 0, [perms[i] for i in bad[:5]]
 
 
-@pytest.mark.parametrize("which", ["n2", "c1b", "c3"])
+@pytest.mark.parametrize("which", ["n2", "c1b", "c3", "acc_fp8"])
 def test_autotune_bitexact(which):
-    """ll_plan_autotune: every candidate decomposition is timed on the caller's buffers;
-    the returned (fastest) plan converts bit-exactly, and describe lists the candidates."""
-    sa, sb, w = {"n2": (*W.n2_tmem_epilogue(5), 4), "c1b": (*W.c1_batched(8), 4), "c3": (*W.c3(3), 2)}[which]
+    """ll_plan_autotune: every candidate decomposition (incl. faithful σ and the permuted
+    sub-word shuffle) is timed on the caller's buffers; the returned (fastest) plan
+    converts bit-exactly, and describe lists the candidates."""
+    sa, sb, w = {"n2": (*W.n2_tmem_epilogue(5), 4), "c1b": (*W.c1_batched(8), 4), "c3": (*W.c3(3), 2),
+                 "acc_fp8": (*W.n2_acc_to_lhs(8, 6), 1)}[which]
     A, OA = both(sa)
     B, OB = both(sb)
     T = gen.random_bits(np.random.default_rng(12), 1 << OA.d_out, w)
