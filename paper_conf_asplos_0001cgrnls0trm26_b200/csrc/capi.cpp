@@ -559,8 +559,8 @@ ll_status ll_plan_describe(const ll_plan* p, char* json, size_t cap) {
       << ",\"axis_hw\":" << "[";
     for (size_t t = 0; t < S.axis_hw.size(); ++t) o << (t ? "," : "") << S.axis_hw[t];
     o << "],\"shuffles_per_elem\":" << double(S.shfl_per_thread) / double(1 << S.R)
-      << ",\"tma\":" << (S.tma ? "true" : "false") << ",\"stages\":" << S.stages
-      << ",\"smem_exchange_bytes\":" << S.xs_bytes
+      << ",\"tma\":" << (S.tma ? "true" : "false") << ",\"tma_store\":" << (S.tma_store ? "true" : "false")
+      << ",\"stages\":" << S.stages << ",\"smem_exchange_bytes\":" << S.xs_bytes
       << ",\"ctas\":" << (u64(1) << S.grid_bit.size()) << "}";
     s = o.str();
   } else {

@@ -234,6 +234,7 @@ std::string codegen_scan(const ScanPlan& S) {
   emit_grid(o, S.grid_bit, S.grid_bit, 2);
   o << icon("KB", S.K_bits) << arr("int", "AXIS_HW", S.axis_hw);
   o << "  static constexpr bool TMA = " << (S.tma ? "true" : "false") << ";\n";
+  o << "  static constexpr bool TMA_STORE = " << (S.tma_store ? "true" : "false") << ";\n";
   o << "  static constexpr unsigned STAGES = " << std::max(1, S.stages) << "u;\n";
   o << "  static constexpr unsigned XS_BYTES = " << S.xs_bytes << "u;\n";
   o << "};\n";

@@ -354,6 +354,7 @@ struct ScanPlan {
   std::vector<int> axis_hw;    // logical axis bit t -> kernel bit (reg < R or lane)
   int shfl_per_thread = 0;     // shuffles per thread per tile
   bool tma = false;            // cp.async.bulk staging of the contiguous CTA tiles
+  bool tma_store = false;      // results written back into the stage, stored by cp.async.bulk
   int stages = 0;
   int xs_bytes = 0;            // exchange buffer of the warp-crossing steps
   int smem_bytes = 0;

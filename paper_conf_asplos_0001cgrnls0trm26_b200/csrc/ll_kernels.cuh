@@ -1555,6 +1555,8 @@ __device__ __forceinline__ void ll_scan_body(const u8* __restrict__ src, u8* __r
       const u32 st = i % NS;
       const u64 tn = t + u64(NS - 1) * gridDim.x;
       if (threadIdx.x == 0 && tn < ntiles) {
+        // TMA_STORE: the previous tile's bulk store read out the stage being refilled
+        if constexpr (P::TMA_STORE) bulk_wait_read<0>();
         fence_proxy_async();
         issue(tn, (i + NS - 1) % NS);
       }
@@ -1566,9 +1568,28 @@ __device__ __forceinline__ void ll_scan_body(const u8* __restrict__ src, u8* __r
         constexpr int E0 = K << P::VLD;
         lds_v4(tb + u32(LdOff<P, K>::value()), r[E0], r[E0 + 1], r[E0 + 2], r[E0 + 3]);
       });
-      __syncthreads();   // stage st is read by every thread before it is refilled
+      if constexpr (!P::TMA_STORE) __syncthreads();   // stage st read by every thread before it is refilled
       ll_scan_steps<P>(r, lane, xs);
-      store_tile(r, tile_base<P, true>(t) ^ thr);
+      if constexpr (P::TMA_STORE) {
+        // results back into this thread's own 16-byte slots of the stage, then one
+        // cp.async.bulk shared -> global of the whole (contiguous) dst tile
+        static_for<(1 << (P::R - P::VLD))>([&](auto k) {
+          constexpr int K = decltype(k)::value;
+          constexpr int E0 = K << P::VLD;
+          sts_vec<4, 2>(tb + u32(LdOff<P, K>::value()), &r[E0]);
+        });
+        fence_proxy_async();
+        __syncthreads();
+        if (threadIdx.x == 0) {
+          bulk_s2g(dst + tile_base<P, true>(t), sbase + st * TB, TB);
+          bulk_commit();
+        }
+      } else {
+        store_tile(r, tile_base<P, true>(t) ^ thr);
+      }
+    }
+    if constexpr (P::TMA_STORE) {
+      if (threadIdx.x == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
     }
   } else {
     float* xs = reinterpret_cast<float*>(ll_smem);

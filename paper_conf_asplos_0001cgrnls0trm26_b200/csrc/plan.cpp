@@ -1719,6 +1719,14 @@ std::unique_ptr<ScanPlan> plan_scan(const Layout& L, int axis, const ll_plan_opt
   for (int ns = 3; ns >= 2; --ns)
     if (u64(ns) * tile_bytes + u64(S->xs_bytes) + 8 * ns <= 200 * 1024) { S->stages = ns; break; }
   S->tma = S->sigma == SIGMA_COALESCED && S->v == 2 && contiguous && force != LL_CLASS_SHUFFLE && S->stages > 0;
+  // the results go back into the stage they were read from (each thread rewrites the
+  // 16-byte vectors it read) and leave by one cp.async.bulk shared -> global per tile
+  // (the dst tile is contiguous like the src tile): the LSU carries no global stores.
+  // LL_SCAN_TMA_STORE=0 keeps per-thread STG stores.
+  {
+    const char* e = std::getenv("LL_SCAN_TMA_STORE");
+    S->tma_store = S->tma && !(e && std::string(e) == "0");
+  }
   S->smem_bytes = S->tma ? int(S->stages * tile_bytes + S->xs_bytes + 8 * S->stages) : S->xs_bytes;
   if (S->smem_bytes > 200 * 1024) fail(LL_ERR_UNSUPPORTED, "scan: tile too large for the shared-memory exchange");
   return S;

@@ -650,6 +650,25 @@ def test_scan_bitexact(family, sigma):
 
 
 @pytest.mark.parametrize("family", ["mma", "blocked"])
+def test_scan_fullsize_tma_store(family):
+    """Config-4 scan on the whole [4096, 4096] fp32 tensor in [128, 128] tiles, in the
+    bench's launch configuration (TMA stages in, results back through the stage and out by
+    cp.async.bulk): every element bit-equal to the oracle's fixed-order recurrence."""
+    import torch
+    spec = W.c4("reduce", family)
+    L, OL = both(spec)
+    plan = ll.ll_plan_scan(L, 1)
+    d = plan.describe()
+    assert d["tma"] and d["tma_store"]
+    T = np.random.default_rng(1008).random(1 << OL.d_out, dtype=np.float32)
+    src = O.pack(OL, T)
+    out = torch.empty(src.size, dtype=torch.float32, device="cuda")
+    ll.ll_scan(torch.from_numpy(src).cuda(), out, plan)
+    rep = O.scan_bitdoubling_fp32(OL, 1, src)
+    assert np.array_equal(out.cpu().numpy().view(np.uint32), rep.view(np.uint32))
+
+
+@pytest.mark.parametrize("family", ["mma", "blocked"])
 @pytest.mark.parametrize("op", ["max", "min"])
 def test_scan_max_min_bitexact(family, op):
     """Running max / min (ll_plan_opts.reduce_op) along the axis inside [128,128] tiles,

@@ -94,6 +94,28 @@ def main():
         return generic_maps()
     if "broadcast" in only:
         return broadcast_sweep()
+    if "scan" in only:
+        # scan output by TMA bulk store (default) vs per-thread STG (LL_SCAN_TMA_STORE=0),
+        # config size and 1 GiB; env is read at plan time
+        for env in ("1", "0"):
+            os.environ["LL_SCAN_TMA_STORE"] = env
+            for fam in ("mma", "blocked"):
+                for ni, nj in ((12, 12), (15, 13)):
+                    L = ll.Layout.from_spec(W.c4("reduce", fam, n_i=ni, n_j=nj))
+                    p = ll.ll_plan_scan(L, 1)
+                    n = 1 << L.d_in
+                    sets = [(torch.rand(n, device="cuda"), torch.empty(n, device="cuda")) for _ in range(4 if ni == 12 else 1)]
+                    it = [0]
+
+                    def f():
+                        a = sets[it[0] % len(sets)]
+                        it[0] += 1
+                        ll.ll_scan(a[0], a[1], p)
+                    ms = time_fn(f, batch=20 if ni == 12 else 3)
+                    print(json.dumps({"case": f"scan {fam} [{1 << ni},{1 << nj}]", "tma_store": p.describe()["tma_store"],
+                                      "ms": round(ms, 4), "GBps": round(8 * n / ms / 1e6, 1)}), flush=True)
+                    del sets
+        return
     if "eperm" in only:
         # sub-word shuffles with element permutations (plan_shuffle_eperm) vs the smem exchange
         for name, (sa, sb), w in (("c3b", W.c3b(14), 2), ("acc_fp8", W.n2_acc_to_lhs(8, 18), 1)):
