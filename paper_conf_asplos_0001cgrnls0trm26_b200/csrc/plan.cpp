@@ -1719,13 +1719,17 @@ std::unique_ptr<ScanPlan> plan_scan(const Layout& L, int axis, const ll_plan_opt
   for (int ns = 3; ns >= 2; --ns)
     if (u64(ns) * tile_bytes + u64(S->xs_bytes) + 8 * ns <= 200 * 1024) { S->stages = ns; break; }
   S->tma = S->sigma == SIGMA_COALESCED && S->v == 2 && contiguous && force != LL_CLASS_SHUFFLE && S->stages > 0;
-  // the results go back into the stage they were read from (each thread rewrites the
+  // The results can go back into the stage they were read from (each thread rewrites the
   // 16-byte vectors it read) and leave by one cp.async.bulk shared -> global per tile
-  // (the dst tile is contiguous like the src tile): the LSU carries no global stores.
-  // LL_SCAN_TMA_STORE=0 keeps per-thread STG stores.
+  // (the dst tile is contiguous like the src tile): the LSU then carries no global
+  // stores.  Measured (profiles/r02_sweep_scan.jsonl): +4.5% on the config-4 size (1024
+  // tiles, ramp-bound), -4% at 1 GiB (16384 tiles), where the stage held by the in-flight
+  // store shortens the load pipeline — so only for launches of <= 4096 tiles.
+  // LL_SCAN_TMA_STORE=0 / 1 forces either.
   {
     const char* e = std::getenv("LL_SCAN_TMA_STORE");
-    S->tma_store = S->tma && !(e && std::string(e) == "0");
+    const bool small = S->grid_bit.size() <= 12;
+    S->tma_store = S->tma && (e ? std::string(e) == "1" : small);
   }
   S->smem_bytes = S->tma ? int(S->stages * tile_bytes + S->xs_bytes + 8 * S->stages) : S->xs_bytes;
   if (S->smem_bytes > 200 * 1024) fail(LL_ERR_UNSUPPORTED, "scan: tile too large for the shared-memory exchange");

@@ -659,7 +659,7 @@ def test_scan_fullsize_tma_store(family):
     L, OL = both(spec)
     plan = ll.ll_plan_scan(L, 1)
     d = plan.describe()
-    assert d["tma"] and d["tma_store"]
+    assert d["tma"] and d["tma_store"]        # 1024 tiles: the bulk-store path
     T = np.random.default_rng(1008).random(1 << OL.d_out, dtype=np.float32)
     src = O.pack(OL, T)
     out = torch.empty(src.size, dtype=torch.float32, device="cuda")

@@ -97,8 +97,11 @@ def main():
     if "scan" in only:
         # scan output by TMA bulk store (default) vs per-thread STG (LL_SCAN_TMA_STORE=0),
         # config size and 1 GiB; env is read at plan time
-        for env in ("1", "0"):
-            os.environ["LL_SCAN_TMA_STORE"] = env
+        for env in ("1", "0", None):
+            if env is None:
+                os.environ.pop("LL_SCAN_TMA_STORE", None)
+            else:
+                os.environ["LL_SCAN_TMA_STORE"] = env
             for fam in ("mma", "blocked"):
                 for ni, nj in ((12, 12), (15, 13)):
                     L = ll.Layout.from_spec(W.c4("reduce", fam, n_i=ni, n_j=nj))
