@@ -547,7 +547,7 @@ ll_status ll_plan_describe(const ll_plan* p, char* json, size_t cap) {
     std::ostringstream o;
     o << "{\"kind\":\"gather\",\"sigma\":\"" << (G.sigma ? "faithful" : "coalesced") << "\",\"R\":" << G.R
       << ",\"warp_bits\":" << G.Wb << ",\"K_bits\":" << G.K_bits
-      << ",\"exchange\":\"" << (G.smem ? "smem" : "shuffle") << "\",\"tma\":" << (G.tma ? "true" : "false") << ",\"shuffles_per_elem\":" << (G.smem ? 0 : (1 << G.cand_bits))
+      << ",\"exchange\":\"" << (G.smem ? "smem" : "shuffle") << "\",\"tma\":" << (G.tma ? "true" : "false") << ",\"tma_store\":" << (G.tma_store ? "true" : "false") << ",\"shuffles_per_elem\":" << (G.smem ? 0 : (1 << G.cand_bits))
       << ",\"ctas\":" << (u64(1) << G.grid_bit.size()) << "}";
     s = o.str();
   } else if (p->kind == 3) {

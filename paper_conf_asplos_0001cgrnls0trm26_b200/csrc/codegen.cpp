@@ -202,6 +202,7 @@ std::string codegen_gather(const GatherPlan& G) {
        " for (int i = 0; i < CBITS; ++i) if ((E >> CAND_REG[i]) & 1) c |= 1u << i; return c; }\n";
   o << "  static constexpr bool GATHER_SMEM = " << (G.smem ? "true" : "false") << ";\n";
   o << "  static constexpr bool TMA = " << (G.tma ? "true" : "false") << ";\n";
+  o << "  static constexpr bool TMA_STORE = " << (G.tma_store ? "true" : "false") << ";\n";
   o << "  static constexpr unsigned STAGES = " << std::max(1, G.stages) << "u;\n";
   // staging stores as 2^v-element vectors when the thread's vector registers are
   // consecutive in the logical tile order (line σ: the lowest logical bits)

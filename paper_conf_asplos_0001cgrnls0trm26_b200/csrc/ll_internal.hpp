@@ -302,6 +302,7 @@ struct GatherPlan {
   uint32_t axmask = 0;           // smem offset bits of the in-tile axis bits
   std::vector<int> axpos;        // axis bit t -> smem offset bit
   int smem_bytes = 0;
+  bool tma_store = false;  // outputs back into the stage, stored by cp.async.bulk
   bool tma = false;        // stream the contiguous src / idx tiles with cp.async.bulk
   int stages = 0;
   std::string source;

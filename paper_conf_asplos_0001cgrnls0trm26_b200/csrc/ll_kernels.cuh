@@ -1159,6 +1159,8 @@ __device__ __forceinline__ void ll_gather_body(const u8* __restrict__ src, const
       const u32 st = i % NS;
       const u64 tn = t + u64(NS - 1) * gridDim.x;
       if (threadIdx.x == 0 && tn < ntiles) {
+        // TMA_STORE: the previous tile's bulk store read out the stage being refilled
+        if constexpr (P::TMA_STORE) bulk_wait_read<0>();
         fence_proxy_async();
         issue(tn, (i + NS - 1) % NS);
       }
@@ -1237,11 +1239,31 @@ __device__ __forceinline__ void ll_gather_body(const u8* __restrict__ src, const
         set_e<P::W, E>(o, res);
       });
     }
-    static_for<(1 << (P::R - P::VLD))>([&](auto k) {
-      constexpr int K = decltype(k)::value;
-      store_vec<P::W, P::VLD, K, P::NW, P::ST_HINT>(o, dst + (eoff ^ LdOff<P, K>::value()) * P::W);
-    });
+    if constexpr (P::TMA_STORE) {
+      // outputs into this thread's own slots of the stage's src tile (read only by this
+      // thread: the shuffle gather keeps sources in registers, the smem gather reads
+      // its own staging area), then one cp.async.bulk of the contiguous dst tile
+      const u32 ts = sbase + (i % NS) * TBST;
+      static_for<(1 << (P::R - P::VLD))>([&](auto k) {
+        constexpr int K = decltype(k)::value;
+        sts_vec<P::W, P::VLD>(ts + u32((thr ^ LdOff<P, K>::value()) * P::W), &o[((K << P::VLD) * P::W) / 4]);
+      });
+      fence_proxy_async();
+      __syncthreads();
+      if (threadIdx.x == 0) {
+        bulk_s2g(dst + tile_base<P, true>(t) * P::W, ts, TBS);
+        bulk_commit();
+      }
+    } else {
+      static_for<(1 << (P::R - P::VLD))>([&](auto k) {
+        constexpr int K = decltype(k)::value;
+        store_vec<P::W, P::VLD, K, P::NW, P::ST_HINT>(o, dst + (eoff ^ LdOff<P, K>::value()) * P::W);
+      });
+    }
     if constexpr (P::TMA || P::GATHER_SMEM) __syncthreads();
+  }
+  if constexpr (P::TMA_STORE) {
+    if (threadIdx.x == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
   }
 }
 

@@ -1532,6 +1532,14 @@ std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const 
            (stage_bytes >= 32768 || force == LL_CLASS_SHUFFLE || force == LL_CLASS_SMEM) &&
            u64(G->stages) * stage_bytes + gbytes + 16 <= 200 * 1024 && (G->v + ilog2(u64(w))) >= 2;
   G->smem_bytes = int(gbytes + (G->tma ? u64(G->stages) * stage_bytes + 8 * G->stages : 0));
+  // outputs through the stage and one cp.async.bulk per tile, as for the scan: for
+  // launches of <= 4096 tiles (ramp-bound; measured in profiles/r02_sweep_gather_tma_store.jsonl);
+  // LL_GATHER_TMA_STORE=0 / 1 forces either
+  {
+    const char* e = std::getenv("LL_GATHER_TMA_STORE");
+    const bool small = G->grid_bit.size() <= 12;
+    G->tma_store = G->tma && (G->w << G->v) >= 4 && (e ? std::string(e) == "1" : small);
+  }
   return G;
 }
 

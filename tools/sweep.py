@@ -119,6 +119,32 @@ def main():
                                       "ms": round(ms, 4), "GBps": round(8 * n / ms / 1e6, 1)}), flush=True)
                     del sets
         return
+    if "gtma" in only:
+        # gather output by TMA bulk store vs per-thread STG, config size and 1 GiB
+        for env in ("1", "0", None):
+            if env is None:
+                os.environ.pop("LL_GATHER_TMA_STORE", None)
+            else:
+                os.environ["LL_GATHER_TMA_STORE"] = env
+            for fam in ("mma", "blocked"):
+                for ni, nj in ((12, 12), (15, 13)):
+                    L = ll.Layout.from_spec(W.c4("gather", fam, n_i=ni, n_j=nj))
+                    p = ll.ll_plan_gather(L, 1, 4)
+                    n = 1 << L.d_in
+                    sets = [(torch.randint(0, 1 << 30, (n,), dtype=torch.int32, device="cuda"),
+                             torch.randint(0, 32, (n,), dtype=torch.int32, device="cuda"),
+                             torch.empty(n, dtype=torch.int32, device="cuda")) for _ in range(4 if ni == 12 else 1)]
+                    it = [0]
+
+                    def f():
+                        a = sets[it[0] % len(sets)]
+                        it[0] += 1
+                        ll.ll_gather(a[0], a[1], a[2], p)
+                    ms = time_fn(f, batch=20 if ni == 12 else 3)
+                    print(json.dumps({"case": f"gather {fam} [{1 << ni},{1 << nj}]", "tma_store": p.describe()["tma_store"],
+                                      "ms": round(ms, 4), "GBps": round(12 * n / ms / 1e6, 1)}), flush=True)
+                    del sets
+        return
     if "eperm" in only:
         # sub-word shuffles with element permutations (plan_shuffle_eperm) vs the smem exchange
         for name, (sa, sb), w in (("c3b", W.c3b(14), 2), ("acc_fp8", W.n2_acc_to_lhs(8, 18), 1)):
