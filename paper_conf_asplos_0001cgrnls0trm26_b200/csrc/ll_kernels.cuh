@@ -754,11 +754,13 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, Dst D, 
       if ((warp >> T) & 1) lo_thr ^= P::LD_LO[P::R + 5 + T];
     });
   }
-  // broadcast plans: CTA-index bits above the data tiles' G select a group of replica
-  // offsets (the replica bits above the unrolled ones are grid bits)
-  constexpr u64 GMASK = (u64(1) << P::G) - 1;
+  // broadcast plans: the lowest NREP_HI_BITS CTA-index bits select a group of replica
+  // offsets (the replica bits above the unrolled ones are grid bits), the
+  // bits above them the data tile — CTAs that load the same src tile run together, so
+  // its re-reads hit L2
+  constexpr u64 RGMASK = (u64(1) << P::NREP_HI_BITS) - 1;
   auto load_tile = [&](u32 (&r)[P::NW], u64 t) {
-    if constexpr (P::NREP_HI_BITS > 0) t &= GMASK;
+    if constexpr (P::NREP_HI_BITS > 0) t >>= P::NREP_HI_BITS;
     u64 thr = ld_thr;
     if constexpr (P::NOHOIST) asm volatile("" : "+l"(thr));   // keep per-vector addresses in the loop
     const u64 sofs = tile_base<P, true>(t) ^ thr;
@@ -786,7 +788,7 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, Dst D, 
   auto store_tile = [&](const u32 (&o)[P::NW], u64 t) {
     u64 thr = st_thr;
     if constexpr (P::NOHOIST) asm volatile("" : "+l"(thr));
-    const u64 td = P::NREP_HI_BITS > 0 ? (t & GMASK) : t;
+    const u64 td = P::NREP_HI_BITS > 0 ? (t >> P::NREP_HI_BITS) : t;
     const u64 doff = tile_base<P, false>(td | tile0) ^ thr;
     auto store_reps = [&](u64 ho) {
       u8* d = D.at(doff ^ ho);
@@ -805,7 +807,7 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, Dst D, 
       store_reps(0);
     } else {
       // replica bits above the unrolled ones: this CTA's group (CTA-index bits above G)
-      const u32 rg = u32(t >> P::G);
+      const u32 rg = u32(t & RGMASK);
       u64 ho = 0;
       static_for<P::NREP_HI_BITS>([&](auto j) {
         constexpr int J = decltype(j)::value;
@@ -897,10 +899,10 @@ __device__ __forceinline__ void ll_tile_body(const u8* __restrict__ src, Dst D, 
         sts_elem<P::W>(sbase + (thr_w ^ BcW<P, E>::value()) * u32(P::W), get_e<P::W, E>(r));
       });
       __syncthreads();
-      const u64 td = P::NREP_HI_BITS > 0 ? (t & GMASK) : t;
+      const u64 td = P::NREP_HI_BITS > 0 ? (t >> P::NREP_HI_BITS) : t;
       u64 ho = 0;
       if constexpr (P::NREP_HI_BITS > 0) {
-        const u32 rg = u32(t >> P::G);
+        const u32 rg = u32(t & RGMASK);
         static_for<P::NREP_HI_BITS>([&](auto j) {
           constexpr int J = decltype(j)::value;
           if ((rg >> J) & 1u) ho ^= P::REP_HI[J];
