@@ -109,6 +109,28 @@ elif a.case.startswith("r2_"):
                 dst = torch.empty_like(src)
                 for _ in range(a.iters):
                     ll.ll_convert(src, dst, p)
+elif a.case.startswith("scan"):
+    # scan_<fam>[_1g]: config-4 scan, or at 1 GiB ([32768, 8192])
+    parts = a.case.split("_")
+    fam = parts[1]
+    big = len(parts) > 2 and parts[2] == "1g"
+    spec = W.c4("reduce", fam, n_i=15, n_j=13) if big else W.c4("reduce", fam)
+    L = ll.Layout.from_spec(spec)
+    p = ll.ll_plan_scan(L, 1)
+    s = torch.rand(1 << L.d_in, device="cuda")
+    d = torch.empty_like(s)
+    for _ in range(a.iters):
+        ll.ll_scan(s, d, p)
+elif a.case.startswith("gather") and a.case.endswith("_1g"):
+    fam = a.case.split("_")[1]
+    L = ll.Layout.from_spec(W.c4("gather", fam, n_i=15, n_j=13))
+    p = ll.ll_plan_gather(L, 1, 4)
+    n = 1 << L.d_in
+    s = torch.randint(0, 1 << 30, (n,), dtype=torch.int32, device="cuda")
+    i = torch.randint(0, 32, (n,), dtype=torch.int32, device="cuda")
+    d = torch.empty_like(s)
+    for _ in range(a.iters):
+        ll.ll_gather(s, i, d, p)
 elif a.case.startswith("gather"):
     parts = a.case.split("_")
     fam = parts[1]
