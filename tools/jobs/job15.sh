@@ -1,0 +1,4 @@
+cd $GRAFT_REPO_ROOT
+timeout 900 python -m pytest tests -m gpu -q -x > gpurun_out/pytest_gpu15.txt 2>&1
+tail -3 gpurun_out/pytest_gpu15.txt
+timeout 600 python tools/sweep.py --only next > gpurun_out/sweep15.txt 2>&1

@@ -1,0 +1,10 @@
+cd $GRAFT_REPO_ROOT
+# several tiles per CTA (LL_GRID_PER_SM=1: 148 CTAs over 256-512 tiles): the pipelined loop's steady state
+for c in r2mid_2 r2mid_4 c3_mid_pipe; do
+  for tool in racecheck memcheck; do
+    echo "== $c tool=$tool"
+    LL_GRID_PER_SM=1 timeout 900 compute-sanitizer --tool $tool --error-exitcode 9 python tools/profile_one.py --case $c --iters 1 2>&1 | grep -E "ERROR SUMMARY|RACECHECK SUMMARY|linear_tile|rror" | head -4
+    echo "rc=${PIPESTATUS[0]}"
+  done
+done > gpurun_out/sanitizer66.txt 2>&1
+cat gpurun_out/sanitizer66.txt
