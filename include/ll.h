@@ -236,7 +236,10 @@ ll_status ll_layout_tmem_32x32b(int M, int N, ll_layout** L);
  *   16x256b: thread bits -> (col 1, col 2, row 0-2); registers -> (col 0, row 3)
  * .x<num> repetitions along the columns are the next register bits; the 16-lane shapes
  * take a second load 16 lanes down (next register bit -> row 4); warps -> rows 5, 6.
- * Matches the CUTLASS SM100 TMEM_LOAD copy traits.  Errors: INVALID_ARG (M != 128,
+ * Matches the CUTLASS SM100 TMEM_LOAD copy traits; tcgen05.st.<shape> takes its
+ * registers in the same fragment (the TMEM_STORE traits reuse the load's thread and
+ * value layouts), so the same layout describes an epilogue's TMEM store.
+ * Errors: INVALID_ARG (M != 128,
  * unknown shape, N below one x1 load).  *L is owned by the caller (ll_layout_destroy). */
 ll_status ll_layout_tmem(const char* shape, int M, int N, ll_layout** L);
 /* ll_layout_contiguity (§5.1 "Contiguous elements"): the number of
