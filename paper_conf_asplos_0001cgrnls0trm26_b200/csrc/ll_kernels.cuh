@@ -1578,11 +1578,11 @@ __device__ __forceinline__ void ll_scan_body(const u8* __restrict__ src, u8* __r
     for (u64 t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
       const u32 st = i % NS;
       const u64 tn = t + u64(NS - 1) * gridDim.x;
-      if (threadIdx.x == 0 && tn < ntiles) {
-        // TMA_STORE: the previous tile's bulk store read out the stage being refilled
-        if constexpr (P::TMA_STORE) bulk_wait_read<0>();
-        fence_proxy_async();
-        issue(tn, (i + NS - 1) % NS);
+      if constexpr (!P::TMA_STORE) {
+        if (threadIdx.x == 0 && tn < ntiles) {
+          fence_proxy_async();
+          issue(tn, (i + NS - 1) % NS);
+        }
       }
       mbar_wait(bar0 + 8 * st, (i / NS) & 1u);
       u32 r[P::NW];
@@ -1607,6 +1607,15 @@ __device__ __forceinline__ void ll_scan_body(const u8* __restrict__ src, u8* __r
         if (threadIdx.x == 0) {
           bulk_s2g(dst + tile_base<P, true>(t), sbase + st * TB, TB);
           bulk_commit();
+          // refill the stage of the PREVIOUS tile (its bulk store has had this whole
+          // iteration to read it out: allow only this tile's store to be pending) with
+          // tile i + NS - 1 — the loads stay NS - 1 tiles ahead without waiting on the
+          // store just issued
+          if (tn < ntiles) {
+            bulk_wait_read<1>();
+            fence_proxy_async();
+            issue(tn, (i + NS - 1) % NS);
+          }
         }
       } else {
         store_tile(r, tile_base<P, true>(t) ^ thr);
