@@ -309,10 +309,12 @@ ll_status peer_convert(ConvPlan& P, const void* src, void* dst, cudaStream_t st)
   LLPeersHost tab;
   std::memset(&tab, 0, sizeof tab);
   if (comm->loopback) {
-    // virtual ranks in one buffer: the windows are the slices; one launch per rank
+    // virtual ranks in one buffer: the windows are the slices.  Rank r's tiles are the
+    // CTA indices [r * rank_tiles, (r + 1) * rank_tiles) of the global plan and its src
+    // slice starts at r * lb, i.e. all ranks together are exactly one launch over every
+    // tile with src = the whole buffer (no per-rank ramp and tail)
     for (int q = 0; q < P.nranks; ++q) tab.dst[q] = static_cast<char*>(dst) + q * lb;
-    for (int r = 0; r < P.nranks; ++r)
-      launch_peer_tiles(F, static_cast<const char*>(src) + r * lb, tab, P.rank_tiles, u64(r) * P.rank_tiles, st);
+    launch_peer_tiles(F, src, tab, P.rank_tiles * u64(P.nranks), 0, st);
     return LL_OK;
   }
   if (dst != comm->peer_dst[comm->rank])
