@@ -902,3 +902,27 @@ def test_bulk_staged_smem_exchange_full_size(cfg, pipe):
     d = ll.ll_plan_convert(A, B, 2, pipe=pipe).describe()
     assert d["tile"]["bulk"] == ("load" if pipe == "bulk" else "load+store")
     _full_size_every_element_opts(sa, sb, 2, 1013, pipe=pipe)
+
+
+def test_permuted_subword_shuffles_gpu():
+    """The element-permuted sub-word shuffles (reading R-V) on random SHUFFLE-class pairs
+    with 1- and 2-byte elements, batched over 8 tiles: bit-exact against the oracle."""
+    rng = np.random.default_rng(31)
+    out = [("i", 5), ("j", 5)]
+    done = 0
+    for case in range(400):
+        r = int(rng.integers(3, 6))
+        hw = [("reg", r), ("lane", 5), ("warp", 10 - r - 5)]
+        sa = gen.random_distributed(rng, out, hw)
+        sb = gen.random_distributed(rng, out, hw)
+        for w in (1, 2):
+            d = ll.ll_plan_convert(ll.Layout.from_spec(sa), ll.Layout.from_spec(sb), w).describe()
+            if not d.get("tile", {}).get("element_permutes"):
+                continue
+            ba = {"out": [("b", 3)] + list(sa["out"]), "in": list(sa["in"]) + [("block", ["b0", "b1", "b2"])]}
+            bb = {"out": [("b", 3)] + list(sb["out"]), "in": list(sb["in"]) + [("block", ["b0", "b1", "b2"])]}
+            got, ref, plan = run_convert(ba, bb, w, case)
+            assert plan.describe()["tile"]["element_permutes"]
+            assert np.array_equal(got, ref), (case, w)
+            done += 1
+    assert done >= 5

@@ -1012,3 +1012,26 @@ def test_n2_acc_to_lhs_simulated(bits):
         for seed, opts in ((4, {}), (5, {"sigma": "faithful"})):
             d = _sim_check(sa, sb, 1, seed, **opts)
             assert d["exec"] == "tile"
+
+
+def test_permuted_subword_shuffles_simulated():
+    """Sub-word shuffles whose 32-bit unit is not common at the lowest registers (reading
+    R-V): random SHUFFLE-class pairs with 1- and 2-byte elements; the plans that take the
+    element-permuted shuffle (plan_shuffle_eperm) reproduce the oracle's conversion in
+    the host emulation, and some do."""
+    rng = np.random.default_rng(31)
+    out = [("i", 5), ("j", 5)]
+    seen = 0
+    for case in range(400):
+        r = int(rng.integers(3, 6))
+        hw = [("reg", r), ("lane", 5), ("warp", 10 - r - 5)]
+        sa = gen.random_distributed(rng, out, hw)
+        sb = gen.random_distributed(rng, out, hw)
+        for w in (1, 2):
+            A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
+            d = ll.ll_plan_convert(A, B, w).describe()
+            if d.get("tile", {}).get("element_permutes"):
+                seen += 1
+                dd = _sim_check(sa, sb, w, case)
+                assert dd["class"] == "SHUFFLE"
+    assert seen >= 5, seen
