@@ -925,4 +925,6 @@ def test_permuted_subword_shuffles_gpu():
             assert plan.describe()["tile"]["element_permutes"]
             assert np.array_equal(got, ref), (case, w)
             done += 1
+        if done >= 24:
+            break
     assert done >= 5
