@@ -145,6 +145,30 @@ def main():
                                       "ms": round(ms, 4), "GBps": round(12 * n / ms / 1e6, 1)}), flush=True)
                     del sets
         return
+    if "epermfuzz" in only:
+        # random SHUFFLE-class pairs that take the element-permuted shuffle, batched to
+        # 2^30 bytes: default (permuted shuffle) vs the smem exchange vs faithful σ
+        import numpy as np
+        from workloads import gen
+        rng = np.random.default_rng(31)
+        out = [("i", 5), ("j", 5)]
+        done = 0
+        for case in range(400):
+            r = int(rng.integers(3, 6))
+            hw = [("reg", r), ("lane", 5), ("warp", 10 - r - 5)]
+            sa = gen.random_distributed(rng, out, hw)
+            sb = gen.random_distributed(rng, out, hw)
+            for w in (1, 2):
+                d = ll.ll_plan_convert(ll.Layout.from_spec(sa), ll.Layout.from_spec(sb), w).describe()
+                if not d.get("tile", {}).get("element_permutes") or done >= 12:
+                    continue
+                nb = 20 - (w - 1)
+                ba = {"out": [("b", nb)] + list(sa["out"]), "in": list(sa["in"]) + [("block", [f"b{k}" for k in range(nb)])]}
+                bb = {"out": [("b", nb)] + list(sb["out"]), "in": list(sb["in"]) + [("block", [f"b{k}" for k in range(nb)])]}
+                for opts in ({}, {"force_class": "SMEM"}, {"sigma": "faithful"}):
+                    conv_case(f"eperm#{case} w{w}", ba, bb, w, **opts)
+                done += 1
+        return
     if "eperm" in only:
         # sub-word shuffles with element permutations (plan_shuffle_eperm) vs the smem exchange
         for name, (sa, sb), w in (("c3b", W.c3b(14), 2), ("acc_fp8", W.n2_acc_to_lhs(8, 18), 1)):
