@@ -1164,7 +1164,7 @@ std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, 
   // non-zero columns of A and of B are each a permutation of the logical unit vectors.
   // The kernel moves the distinct elements only: src bits with zero columns are never
   // read (slack = 0), dst bits with zero columns become store replicas.
-  if (!generic && lev <= 2 && !(opts && opts->sigma == SIGMA_FAITHFUL)) {
+  if (!generic && lev <= 3 && !(opts && opts->sigma == SIGMA_FAITHFUL)) {
     auto nz_unit = [](const Layout& L) {
       u64 seen = 0;
       for (u64 c : L.cols) {
@@ -1181,20 +1181,53 @@ std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, 
           for (int k = 0; k < nA; ++k) if (A.cols[k] == c) return k;
           fail(LL_ERR_UNSUPPORTED, "broadcast: column missing in A (internal)");
         };
-        for (int k : bits_at_level(B, 0, 2)) {
-          if (B.cols[k]) { D.push_back(k); S.push_back(srcbit_of(B.cols[k])); }
-          else rep.push_back(k);
+        if (lev <= 2) {
+          for (int k : bits_at_level(B, 0, 2)) {
+            if (B.cols[k]) { D.push_back(k); S.push_back(srcbit_of(B.cols[k])); }
+            else rep.push_back(k);
+          }
+          for (int k : bits_at_level(B, 3, 3)) {
+            if (B.cols[k]) { gD.push_back(k); gS.push_back(srcbit_of(B.cols[k])); }
+            else rep.push_back(k);
+          }
+          build_tile(*P, S, D, gS, gD, opts, true);
+        } else {
+          // CTA class (the map mixes block / offset bits): the data bits of B and the
+          // non-zero bits of A form a bit permutation; the CTA tile is chosen on it as in
+          // the permutation path (choose_cta_tile), over the data bits
+          // compressed to consecutive indices, then mapped back to packed bits
+          std::vector<int> Dall, Sall;
+          for (int k = 0; k < nB; ++k) (B.cols[k] ? Dall : rep).push_back(k);
+          for (int k = 0; k < nA; ++k) if (A.cols[k]) Sall.push_back(k);
+          if (Dall.size() != Sall.size()) fail(LL_ERR_UNSUPPORTED, "broadcast: data bits differ (internal)");
+          const int nd = int(Dall.size());
+          std::vector<int> pi(nd);
+          for (int c = 0; c < nd; ++c) {
+            const int sb = srcbit_of(B.cols[Dall[c]]);
+            pi[c] = int(std::lower_bound(Sall.begin(), Sall.end(), sb) - Sall.begin());
+          }
+          const int maxvec = default_int(opts, &ll_plan_opts::max_vec_bytes, 16);
+          const int v = std::max(0, ilog2(u64(std::max(1, maxvec / w))));
+          const int tbytes = default_int(opts, &ll_plan_opts::tile_bytes, 16384);
+          const int target = std::max(v + 5, ilog2(u64(std::max(1, tbytes / w))));
+          const int max_bits = ilog2(u64(65536 / w));
+          std::vector<int> Sc, Dc, gSc, gDc;
+          for (int c_bits = v + 5; c_bits >= v + 3; --c_bits) {
+            choose_cta_tile(pi, nd, c_bits, target, Sc, Dc, gSc, gDc);
+            if (int(Sc.size()) <= max_bits) break;
+          }
+          for (int c : Sc) S.push_back(Sall[c]);
+          for (int c : Dc) D.push_back(Dall[c]);
+          for (int c : gSc) gS.push_back(Sall[c]);
+          for (int c : gDc) gD.push_back(Dall[c]);
+          build_tile(*P, S, D, gS, gD, opts, false);
         }
-        for (int k : bits_at_level(B, 3, 3)) {
-          if (B.cols[k]) { gD.push_back(k); gS.push_back(srcbit_of(B.cols[k])); }
-          else rep.push_back(k);
-        }
-        build_tile(*P, S, D, gS, gD, opts, true);
         P->tile.rep_bits = rep;
         if (!rep.empty()) {
           // replicas: per-thread stores, plain tile loop (no staged / bulk variants);
-          // unroll up to 4 replica bits per store while the grid (data tiles x replica
-          // groups) keeps >= 8 CTAs per SM, the rest become grid bits
+          // dst-order broadcast stores when a replica bit is low (plan_bcast_store); at
+          // most 2 unrolled replica bits, the rest CTA-grid bits below the data tiles'
+          // while the grid keeps >= 8 CTAs per SM
           TilePlan& T = P->tile;
           if (T.staged || T.bulk) {
             P->smem_bytes = int(T.smem_elems * u64(T.w));

@@ -51,3 +51,29 @@ def test_broadcast_large_every_element(n_zero):
     ll.ll_convert(src, dst, p)
     torch.cuda.synchronize()
     assert H.check(sb, 4, 5, dst) == 0
+
+
+@pytest.mark.parametrize("n_zero", [2, 5, 8])
+def test_broadcast_cta_class_bitexact(n_zero):
+    """Broadcast targets with permuted block bits (CTA class), batched: bit-exact against
+    the oracle, and at ~1 GiB every element against H(B(h))."""
+    import torch
+    from tests._util import to_device
+    rng = np.random.default_rng(7100 + n_zero)
+    for case in range(3):
+        sa, sb = gen.random_broadcast_pair(rng, n_zero, batch_bits=4, permute_batch=True)
+        OA, OB = O.Layout(*W.spec_to_bases(sa)), O.Layout(*W.spec_to_bases(sb))
+        p = ll.ll_plan_convert(ll.Layout.from_spec(sa), ll.Layout.from_spec(sb), 4)
+        assert p.cls == "CTA" and p.describe()["exec"] == "tile"
+        src = O.pack(OA, gen.random_bits(rng, 1 << OA.d_out, 4))
+        d_dst = torch.zeros(1 << OB.d_in, dtype=torch.int32, device="cuda")
+        ll.ll_convert(to_device(src), d_dst, p)
+        assert np.array_equal(d_dst.cpu().numpy().view(np.uint32), O.convert(OA, OB, src)), case
+    sa, sb = gen.random_broadcast_pair(rng, n_zero, ki=5, kj=5, batch_bits=18 - n_zero, permute_batch=True)
+    A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
+    p = ll.ll_plan_convert(A, B, 4)
+    src = H.fill(sa, 4, 9)
+    dst = torch.zeros(1 << B.d_in, dtype=torch.int32, device="cuda")
+    ll.ll_convert(src, dst, p)
+    torch.cuda.synchronize()
+    assert H.check(sb, 4, 9, dst) == 0

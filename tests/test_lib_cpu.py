@@ -1035,3 +1035,16 @@ def test_permuted_subword_shuffles_simulated():
                 dd = _sim_check(sa, sb, w, case)
                 assert dd["class"] == "SHUFFLE"
     assert seen >= 5, seen
+
+
+@pytest.mark.parametrize("n_zero", [1, 3, 6])
+def test_broadcast_cta_class_simulated(n_zero):
+    """Broadcast targets whose block bits are permuted (CTA class): the data bits run as a
+    CTA-tiled permutation with replica stores — no XOR-copy or generic kernel — and the
+    simulated schedule equals the oracle's conversion."""
+    rng = np.random.default_rng(700 + n_zero)
+    for case in range(10):
+        sa, sb = gen.random_broadcast_pair(rng, n_zero, batch_bits=4, permute_batch=True)
+        w = [1, 2, 4, 8][case % 4]
+        d = _sim_check(sa, sb, w, case)
+        assert d["exec"] == "tile" and "ld_xcol" not in d["tile"], d

@@ -94,6 +94,8 @@ def main():
         return generic_maps()
     if "broadcast" in only:
         return broadcast_sweep()
+    if "bcastcta" in only:
+        return broadcast_sweep(permute_batch=True)
     if "scan" in only:
         # scan output by TMA bulk store (default) vs per-thread STG (LL_SCAN_TMA_STORE=0),
         # config size and 1 GiB; env is read at plan time
@@ -208,7 +210,7 @@ def main():
     gather_reduce()
 
 
-def broadcast_sweep():
+def broadcast_sweep(permute_batch=False):
     """Broadcast targets: random bijective A -> B with 5-8 zero columns,
     batched to ~2 GiB of dst, fp32.  GB/s on algorithmic bytes (src read once + every
     dst replica written: (2^dA + 2^dB) * w), the specialised replica-store tile kernel
@@ -219,12 +221,12 @@ def broadcast_sweep():
     for nz in (5, 6, 7, 8):
         rng = np.random.default_rng(900 + nz)
         for case in range(6):
-            sa, sb = gen.random_broadcast_pair(rng, nz, ki=5, kj=5, batch_bits=19 - nz)
+            sa, sb = gen.random_broadcast_pair(rng, nz, ki=5, kj=5, batch_bits=19 - nz, permute_batch=permute_batch)
             A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
             src = hashfill.fill(sa, w, case)
             dst = torch.empty(1 << B.d_in, dtype=torch.int32, device="cuda")
             alg = (src.numel() + dst.numel()) * w
-            row = {"case": f"bcast nz={nz} #{case}", "src_MiB": src.numel() * w >> 20, "dst_MiB": dst.numel() * w >> 20}
+            row = {"case": f"bcast{'-cta' if permute_batch else ''} nz={nz} #{case}", "src_MiB": src.numel() * w >> 20, "dst_MiB": dst.numel() * w >> 20}
             for tag, opts in (("tile", {}), ("generic", {"generic": True})):
                 p = ll.ll_plan_convert(A, B, w, **opts)
                 p.prepare()

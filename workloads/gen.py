@@ -93,11 +93,13 @@ def splitmix64(x: np.ndarray, seed: int) -> np.ndarray:
 
 
 def random_broadcast_pair(rng: np.random.Generator, n_zero: int, ki: int = 5, kj: int = 5,
-                          batch_bits: int = 0, w_bits_a: Optional[Tuple[int, int]] = None):
+                          batch_bits: int = 0, w_bits_a: Optional[Tuple[int, int]] = None,
+                          permute_batch: bool = False):
     """Broadcast sweep (P:306-308 zero columns; rule (2) P:358-362): a random bijective
     distributed A and a random distributed B with `n_zero` zero (broadcast) columns over
     reg / lane / warp, on the logical [2^ki, 2^kj] tile, plus `batch_bits` batch bits
-    that are the block bits of both (independent tiles).  Returns (spec_A, spec_B)."""
+    that are the block bits of both (independent tiles) — or, with permute_batch, B's
+    block bits a random permutation of A's (a CTA-class map).  Returns (spec_A, spec_B)."""
     d = ki + kj
     out = [("i", ki), ("j", kj)]
     ra = int(rng.integers(1, 4)) if w_bits_a is None else w_bits_a[0]
@@ -112,7 +114,8 @@ def random_broadcast_pair(rng: np.random.Generator, n_zero: int, ki: int = 5, kj
     sa = random_distributed(rng, out, [("reg", ra), ("lane", 5), ("warp", wa)])
     sb = random_distributed(rng, out, [("reg", rb), ("lane", 5), ("warp", wb)])
     if batch_bits:
-        for s in (sa, sb):
+        perm = rng.permutation(batch_bits) if permute_batch else np.arange(batch_bits)
+        for s, order in ((sa, np.arange(batch_bits)), (sb, perm)):
             s["out"] = [("b", batch_bits)] + list(s["out"])
-            s["in"] = list(s["in"]) + [("block", [f"b{k}" for k in range(batch_bits)])]
+            s["in"] = list(s["in"]) + [("block", [f"b{int(k)}" for k in order])]
     return sa, sb
