@@ -1164,7 +1164,8 @@ std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, 
   // non-zero columns of A and of B are each a permutation of the logical unit vectors.
   // The kernel moves the distinct elements only: src bits with zero columns are never
   // read (slack = 0), dst bits with zero columns become store replicas.
-  if (!generic && lev <= 3 && !(opts && opts->sigma == SIGMA_FAITHFUL)) {
+  auto try_bcast = [&]() -> bool {
+    if (generic || lev > 3 || (opts && opts->sigma == SIGMA_FAITHFUL)) return false;
     auto nz_unit = [](const Layout& L) {
       u64 seen = 0;
       for (u64 c : L.cols) {
@@ -1244,12 +1245,21 @@ std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, 
             --T.rep_lo;
         }
         P->exec = EXEC_TILE;
-        return P;
+        return true;
       } catch (const Error& e) {
         if (opts && opts->force_class >= 0) throw;
+        P->tile = TilePlan();
       }
     }
-  }
+    return false;
+  };
+  // lev <= 2: inside one CTA.  CTA class (lev 3): after the XOR-copy tiles below, which
+  // keep the widest global vectors on the small memory <-> distributed maps of Table 3
+  // (LL_BCAST_CTA=1 tries the CTA-tiled broadcast first, =0 never)
+  const char* bce = std::getenv("LL_BCAST_CTA");
+  const bool bcast_cta_first = bce && std::string(bce) == "1";
+  const bool bcast_cta_never = bce && std::string(bce) == "0";
+  if ((lev <= 2 || bcast_cta_first) && try_bcast()) return P;
   // Any other linear pull map (2-bit columns of swizzled memory layouts, Def 4.14 /
   // P:240-276; broadcast across CTAs): a copy kernel in dst order — coalesced 16-byte
   // stores, loads at src = Q(dst) (XOR of columns), vectorised over the low dst bits Q
@@ -1322,6 +1332,7 @@ std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, 
       }
     }
   }
+  if (lev == 3 && !bcast_cta_first && !bcast_cta_never && try_bcast()) return P;
   if (!generic && lev <= 3) {
     try {
       if (build_linear_tile(*P, opts)) return P;

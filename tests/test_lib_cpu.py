@@ -1042,9 +1042,24 @@ def test_broadcast_cta_class_simulated(n_zero):
     """Broadcast targets whose block bits are permuted (CTA class): the data bits run as a
     CTA-tiled permutation with replica stores — no XOR-copy or generic kernel — and the
     simulated schedule equals the oracle's conversion."""
+    import os
     rng = np.random.default_rng(700 + n_zero)
-    for case in range(10):
-        sa, sb = gen.random_broadcast_pair(rng, n_zero, batch_bits=4, permute_batch=True)
-        w = [1, 2, 4, 8][case % 4]
-        d = _sim_check(sa, sb, w, case)
-        assert d["exec"] == "tile" and "ld_xcol" not in d["tile"], d
+    old = os.environ.get("LL_BCAST_CTA")
+    try:
+        for mode in ("1", None):      # CTA-tiled broadcast first; the default order
+            if mode:
+                os.environ["LL_BCAST_CTA"] = mode
+            else:
+                os.environ.pop("LL_BCAST_CTA", None)
+            for case in range(10):
+                sa, sb = gen.random_broadcast_pair(rng, n_zero, batch_bits=4, permute_batch=True)
+                w = [1, 2, 4, 8][case % 4]
+                d = _sim_check(sa, sb, w, case)
+                assert d["exec"] == "tile", d
+                if mode == "1":
+                    assert "ld_xcol" not in d["tile"], d
+    finally:
+        if old is None:
+            os.environ.pop("LL_BCAST_CTA", None)
+        else:
+            os.environ["LL_BCAST_CTA"] = old

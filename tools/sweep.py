@@ -96,6 +96,16 @@ def main():
         return broadcast_sweep()
     if "bcastcta" in only:
         return broadcast_sweep(permute_batch=True)
+    if "bcastctacmp" in only:
+        # CTA-class broadcast: XOR-copy tiles first (default) vs the CTA-tiled broadcast
+        for env in ("1", None):
+            if env:
+                os.environ["LL_BCAST_CTA"] = env
+            else:
+                os.environ.pop("LL_BCAST_CTA", None)
+            print(json.dumps({"LL_BCAST_CTA": env}), flush=True)
+            broadcast_sweep(permute_batch=True)
+        return
     if "scan" in only:
         # scan output by TMA bulk store (default) vs per-thread STG (LL_SCAN_TMA_STORE=0),
         # config size and 1 GiB; env is read at plan time
