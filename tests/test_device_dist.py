@@ -275,3 +275,15 @@ def test_weak_sharding_independent_tiles_gloo(world):
     for pr in procs:
         pr.join(timeout=60)
     assert all(v == "ok" for v in res.values()), res
+
+
+def test_device_peers_errors():
+    """ll_plan_device_peers: only collective DEVICE plans, rank in range."""
+    A, B = ll.Layout.from_spec(W.C1_A), ll.Layout.from_spec(W.C1_B)
+    with pytest.raises(ll.LLError, match="INVALID_ARG"):
+        ll.ll_plan_convert(A, B, 4).device_peers(0)
+    sa, sb = W.c5(1, n=4)
+    plan = ll.ll_plan_convert(ll.Layout.from_spec(sa), ll.Layout.from_spec(sb), 2, comm=ll.Comm.loopback(2))
+    assert plan.device_peers(0) == ([0, 1], [0, 1])
+    with pytest.raises(ll.LLError, match="INVALID_ARG"):
+        plan.device_peers(2)
