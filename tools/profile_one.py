@@ -26,6 +26,7 @@ conv = {"c2": (W.c2(16), 2, {}), "c2smem": (W.c2(16), 2, {"force_class": "SMEM"}
         "c1bsmem_small": (W.c1_batched(6), 4, {"force_class": "SMEM"}),
         "c3_small": (W.c3(3), 2, {}), "c3_mid_pipe": (W.c3(9), 2, {"pipe": "on"}), "c2_small": (W.c2(3), 2, {}),
         "c3b_small": (W.c3b(3), 2, {}),
+        "acc8_small": (W.n2_acc_to_lhs(8, 4), 1, {}), "acc8f_small": (W.n2_acc_to_lhs(8, 4), 1, {"sigma": "faithful"}),
         "c2fsmem_small": (W.c2(3), 2, {"sigma": "faithful", "force_class": "SMEM", "smem_instr": "matrix"}),
         "c3f_small": (W.c3(3), 2, {"sigma": "faithful"}),
         "c5T": (W.c5T(0, n=15), 2, {}), "n1": (W.n1_preshuffle(14, 14), 2, {}),
@@ -41,10 +42,11 @@ if a.case.startswith("bcast"):
     import numpy as np
     from workloads import gen
     # bcast<seed>: the bench size (8 MiB -> 2 GiB); bcastS<seed>: 2 batch bits (sanitizer size)
-    small = a.case.startswith("bcastS")
+    # bcastC<seed>: small, with permuted block bits (CTA class)
+    small = a.case.startswith("bcastS") or a.case.startswith("bcastC")
     seed = int(a.case[6:] if small else a.case[5:] or 908)
     sa, sb = gen.random_broadcast_pair(np.random.default_rng(seed), 8 if not small else 5, ki=5, kj=5,
-                                       batch_bits=2 if small else 11)
+                                       batch_bits=2 if small else 11, permute_batch=a.case.startswith("bcastC"))
     import json
     p = ll.ll_plan_convert(ll.Layout.from_spec(sa), ll.Layout.from_spec(sb), 4, **json.loads(a.opts))
     A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
