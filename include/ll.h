@@ -339,10 +339,14 @@ ll_status ll_gather(const void* src, const int32_t* idx, void* dst, const ll_pla
 /* ---------------------------------------------------------------- reduce --
  * ll_plan_reduce (row a12; Table 4).  Sum (fp32; or max / min
  * with opts->reduce_op = 1 / 2) along logical dim `axis` over the non-block axis
- * bits of L (within each CTA tile): an in-register tree over Reg axis bits,
- * shfl.bfly over Lane axis bits and smem over Warp axis bits, in that fixed order
- * (reg, lane, warp ascending); broadcast (zero-column) bits are skipped, each
- * output is written once.  LL_ERR_INVALID_ARG for another reduce_op. */
+ * bits of L (within each CTA tile; they must be the low bits of the axis
+ * coordinate).  The fp32 order is fixed in logical coordinates (reading R-reduce,
+ * DESIGN.md §3): for in-tile axis bit t = 0, 1, ... ascending, v <- v(t = 0) +
+ * v(t = 1), round to nearest — the recursive pairwise sum, independent of L and of
+ * every plan option.  Each step is a register add, a shfl.bfly or a shared-memory
+ * step, whichever level of the kernel layout holds bit t; broadcast (zero-column)
+ * bits are skipped, each output is written once.  LL_ERR_INVALID_ARG for another
+ * reduce_op; LL_ERR_UNSUPPORTED when L is not distributed (Def 4.10). */
 ll_status ll_plan_reduce(const ll_layout* L, int axis, const ll_plan_opts* opts, ll_plan** plan);
 /* Number of output elements. */
 ll_status ll_plan_reduce_out_elems(const ll_plan* plan, size_t* n);

@@ -1237,8 +1237,8 @@ std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, 
           plan_bcast_store(*P, opts);
           const int nrep = int(T.rep_bits.size());
           const int gdata = int(T.grid_dst_bit.size());
-          // measured (profiles/r02_sweep_broadcast_*.jsonl): 16 unrolled replicas per
-          // store (rep_lo = 4) were the slowest plans; with the replica group as the low
+          // measured (profiles/r02_sweep_broadcast_*.jsonl): plans unrolling 16 replicas
+          // per store (rep_lo = 4) were the slowest; with the replica group as the low
           // CTA-index bits (the src tile's re-reads hit L2) at most 2 are unrolled
           T.rep_lo = std::min(2, nrep);
           while (T.rep_lo > 0 && (gdata + nrep - T.rep_lo) < 64 && (u64(1) << (gdata + nrep - T.rep_lo)) < u64(8 * 148))
