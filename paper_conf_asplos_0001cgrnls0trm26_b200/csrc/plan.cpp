@@ -1597,6 +1597,27 @@ std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const 
 // whichever level of the kernel layout L∘σ holds bit t.  The order is a property of the
 // logical tensor alone, so the fp32 bits do not depend on L, on σ or on any plan option.
 // ---------------------------------------------------------------------------
+// More warps per CTA for the single-layout kernels (reduce, scan): a register bit of the
+// kernel layout that carries no in-tile axis bit (independent rows) becomes an extra warp
+// bit, so the CTA tile (the same packed bits: TMA staging unchanged) runs on twice the
+// warps with half the registers each — latency hiding for the dependent add / shuffle
+// chains.  `thread_bytes` (ll_plan_opts) is the register budget per thread; the vector
+// bits [0, v) stay registers, at most 5 warp bits (1024 threads).
+static void widen_warps(std::vector<int>& hw_bit, int& R, int& Wb, int v, int thread_bytes,
+                        const std::function<bool(int)>& is_axis) {
+  const int Rt = std::max(v, ilog2(u64(std::max(4, thread_bytes) / 4)));
+  while (R > Rt && Wb < 5) {
+    int b = -1;
+    for (int q = R - 1; q >= v; --q) if (!is_axis(hw_bit[q])) { b = q; break; }
+    if (b < 0) break;
+    const int pk = hw_bit[b];
+    hw_bit.erase(hw_bit.begin() + b);
+    hw_bit.push_back(pk);   // after the lanes and the existing warps: the new top warp bit
+    --R;
+    ++Wb;
+  }
+}
+
 std::unique_ptr<ReducePlan> plan_reduce(const Layout& L, int axis, const ll_plan_opts* opts) {
   if (axis < 0 || axis >= int(L.out.size())) fail(LL_ERR_INVALID_ARG, "axis out of range");
   if (!L.distributed()) fail(LL_ERR_UNSUPPORTED, "reduce: L must be a distributed layout (Def 4.10)");
@@ -1608,7 +1629,7 @@ std::unique_ptr<ReducePlan> plan_reduce(const Layout& L, int axis, const ll_plan
   if (Rp->op < 0 || Rp->op > 2) fail(LL_ERR_INVALID_ARG, "reduce_op must be 0 (sum), 1 (max) or 2 (min)");
   const int sh = L.out_shift(axis), ab = L.out[axis].bits;
   const u64 amask = ((u64(1) << ab) - 1) << sh;
-  const int R = L.in_bits("reg");
+  int R = L.in_bits("reg");
   Rp->R = R;
   Rp->Wb = L.in_bits("warp");
   // K: number of in-tile (non-block) axis bits; they must be the low axis bits
@@ -1630,6 +1651,9 @@ std::unique_ptr<ReducePlan> plan_reduce(const Layout& L, int axis, const ll_plan
     Rp->sigma = SIGMA_COALESCED;
     Rp->hw_bit = sigma_line(L, Rp->v, [&](int k) { return L.cols[k] != 0 && !(L.cols[k] & amask); });
   }
+  widen_warps(Rp->hw_bit, Rp->R, Rp->Wb, Rp->v, default_int(opts, &ll_plan_opts::thread_bytes, 512),
+              [&](int k) { return (L.cols[k] & amask) != 0; });
+  R = Rp->R;
   const int n = int(Rp->hw_bit.size());
   // classify kernel bits (reduced per level, duplicate) and map each logical axis bit t
   // to the kernel bit that holds it: the steps run in t order
@@ -1722,7 +1746,7 @@ std::unique_ptr<ScanPlan> plan_scan(const Layout& L, int axis, const ll_plan_opt
   if (S->op < 0 || S->op > 2) fail(LL_ERR_INVALID_ARG, "reduce_op must be 0 (sum), 1 (max) or 2 (min)");
   const int sh = L.out_shift(axis), ab = L.out[axis].bits;
   const u64 amask = ((u64(1) << ab) - 1) << sh;
-  const int R = L.in_bits("reg");
+  int R = L.in_bits("reg");
   S->R = R;
   S->Wb = L.in_bits("warp");
   int K = 0;
@@ -1737,6 +1761,9 @@ std::unique_ptr<ScanPlan> plan_scan(const Layout& L, int axis, const ll_plan_opt
     // axis bits stay in registers where possible (register steps need no shuffle)
     S->hw_bit = sigma_line(L, S->v, [&](int k) { return L.cols[k] != 0 && !(L.cols[k] & amask); });
   }
+  widen_warps(S->hw_bit, S->R, S->Wb, S->v, default_int(opts, &ll_plan_opts::thread_bytes, 512),
+              [&](int k) { return (L.cols[k] & amask) != 0; });
+  R = S->R;
   const int n = int(S->hw_bit.size());
   for (int t = 0; t < K; ++t) {
     int b = -1;

@@ -928,3 +928,29 @@ def test_permuted_subword_shuffles_gpu():
         if done >= 24:
             break
     assert done >= 5
+
+
+@pytest.mark.parametrize("family", ["mma", "blocked"])
+@pytest.mark.parametrize("thread_bytes", [256, 128])
+def test_reduce_scan_more_warps_bitexact(family, thread_bytes):
+    """Non-axis register bits moved to extra warps (ll_plan_opts.thread_bytes: 8 / 16
+    warps per [128,128] tile): reduce bit-exact against the logical-order replica and
+    scan against the bit-doubling recurrence — the orders do not depend on the kernel
+    layout."""
+    import torch
+    L, OL = both(W.c4("reduce", family, n_i=9, n_j=9))
+    T = np.random.default_rng(1009).random(1 << OL.d_out, dtype=np.float32)
+    src = O.pack(OL, T)
+    d_src = torch.from_numpy(src).cuda()
+    p = ll.ll_plan_reduce(L, 1, thread_bytes=thread_bytes)
+    assert p.describe()["warp_bits"] > 2
+    out = torch.empty(p.out_elems(), dtype=torch.float32, device="cuda")
+    ll.ll_reduce(d_src, out, p)
+    rep = O.reduce_fixed_order_fp32(OL, 1, src)
+    assert np.array_equal(out.cpu().numpy().view(np.uint32), rep.view(np.uint32))
+    s = ll.ll_plan_scan(L, 1, thread_bytes=thread_bytes)
+    assert s.describe()["warp_bits"] > 2
+    out2 = torch.empty(src.size, dtype=torch.float32, device="cuda")
+    ll.ll_scan(d_src, out2, s)
+    rep2 = O.scan_bitdoubling_fp32(OL, 1, src)
+    assert np.array_equal(out2.cpu().numpy().view(np.uint32), rep2.view(np.uint32))

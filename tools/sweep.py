@@ -131,6 +131,29 @@ def main():
                                       "ms": round(ms, 4), "GBps": round(8 * n / ms / 1e6, 1)}), flush=True)
                     del sets
         return
+    if "warps" in only:
+        # reduce / scan with non-axis register bits moved to warps (thread_bytes)
+        for fam in ("mma", "blocked"):
+            for ni, nj in ((12, 12), (15, 13)):
+                L = ll.Layout.from_spec(W.c4("reduce", fam, n_i=ni, n_j=nj))
+                n = 1 << L.d_in
+                sets = [torch.rand(n, device="cuda") for _ in range(4 if ni == 12 else 1)]
+                for tb in (512, 256, 128):
+                    for kind in ("reduce", "scan"):
+                        p = (ll.ll_plan_reduce if kind == "reduce" else ll.ll_plan_scan)(L, 1, thread_bytes=tb)
+                        outs = [torch.empty(p.out_elems() if kind == "reduce" else n, device="cuda") for _ in sets]
+                        it = [0]
+
+                        def f():
+                            k = it[0] % len(sets)
+                            it[0] += 1
+                            (ll.ll_reduce if kind == "reduce" else ll.ll_scan)(sets[k], outs[k], p)
+                        ms = time_fn(f, batch=20 if ni == 12 else 3)
+                        nbytes = 4 * n + 4 * (p.out_elems() if kind == "reduce" else n)
+                        print(json.dumps({"case": f"{kind} {fam} [{1 << ni},{1 << nj}]", "thread_bytes": tb,
+                                          "warps": 1 << p.describe()["warp_bits"], "ms": round(ms, 4),
+                                          "GBps": round(nbytes / ms / 1e6, 1)}), flush=True)
+        return
     if "gtma" in only:
         # gather output by TMA bulk store vs per-thread STG, config size and 1 GiB
         for env in ("1", "0", None):
