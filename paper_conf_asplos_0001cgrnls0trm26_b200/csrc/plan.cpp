@@ -1651,7 +1651,10 @@ std::unique_ptr<ReducePlan> plan_reduce(const Layout& L, int axis, const ll_plan
     Rp->sigma = SIGMA_COALESCED;
     Rp->hw_bit = sigma_line(L, Rp->v, [&](int k) { return L.cols[k] != 0 && !(L.cols[k] & amask); });
   }
-  widen_warps(Rp->hw_bit, Rp->R, Rp->Wb, Rp->v, default_int(opts, &ll_plan_opts::thread_bytes, 512),
+  // default 256 bytes per thread (8 warps on a [128,128] fp32 tile): measured +5% on the
+  // config-4 MMA reduce and +1.6% at 1 GiB, neutral on the blocked one; the scan keeps 512
+  // (neutral either way; profiles/r02_sweep_reduce_scan_warps.jsonl)
+  widen_warps(Rp->hw_bit, Rp->R, Rp->Wb, Rp->v, default_int(opts, &ll_plan_opts::thread_bytes, 256),
               [&](int k) { return (L.cols[k] & amask) != 0; });
   R = Rp->R;
   const int n = int(Rp->hw_bit.size());
