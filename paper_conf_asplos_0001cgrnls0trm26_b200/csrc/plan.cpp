@@ -1464,6 +1464,27 @@ static std::vector<int> sigma_line(const Layout& L, int v, const std::function<b
   return hw;
 }
 
+// More warps per CTA for the single-layout kernels (reduce, scan): a register bit of the
+// kernel layout that carries no in-tile axis bit (independent rows) becomes an extra warp
+// bit, so the CTA tile (the same packed bits: TMA staging unchanged) runs on twice the
+// warps with half the registers each — latency hiding for the dependent add / shuffle
+// chains.  `thread_bytes` (ll_plan_opts) is the register budget per thread; the vector
+// bits [0, v) stay registers, at most 5 warp bits (1024 threads).
+static void widen_warps(std::vector<int>& hw_bit, int& R, int& Wb, int v, int thread_bytes,
+                        const std::function<bool(int)>& is_axis) {
+  const int Rt = std::max(v, ilog2(u64(std::max(4, thread_bytes) / 4)));
+  while (R > Rt && Wb < 5) {
+    int b = -1;
+    for (int q = R - 1; q >= v; --q) if (!is_axis(hw_bit[q])) { b = q; break; }
+    if (b < 0) break;
+    const int pk = hw_bit[b];
+    hw_bit.erase(hw_bit.begin() + b);
+    hw_bit.push_back(pk);   // after the lanes and the existing warps: the new top warp bit
+    --R;
+    ++Wb;
+  }
+}
+
 std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const ll_plan_opts* opts) {
   if (w != 1 && w != 2 && w != 4 && w != 8) fail(LL_ERR_INVALID_ARG, "elem_bytes must be 1, 2, 4 or 8");
   if (axis < 0 || axis >= int(L.out.size())) fail(LL_ERR_INVALID_ARG, "axis out of range");
@@ -1495,7 +1516,7 @@ std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const 
   int maxvec = default_int(opts, &ll_plan_opts::max_vec_bytes, 16);
   int v = std::min(ilog2(u64(std::max(1, maxvec / ev))), L.in_bits("reg"));
   auto regb = bits_at_level(L, 0, 0), laneb = bits_at_level(L, 1, 1), warpb = bits_at_level(L, 2, 2);
-  const int R = int(regb.size());
+  int R = int(regb.size());
 
   std::vector<int> faith;
   for (int k : regb) faith.push_back(k);
@@ -1512,6 +1533,13 @@ std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const 
   G->R = R;
   G->Wb = int(warpb.size());
   G->v = use_coal ? v : std::min(ilog2(u64(std::max(1, maxvec / ev))), R);
+  // optional extra warps from non-axis register bits (ll_plan_opts.thread_bytes; the
+  // default keeps the layout's warps — measured in profiles/r02_sweep_gather_warps.jsonl)
+  if (opts && opts->thread_bytes > 0) {
+    widen_warps(G->hw_bit, G->R, G->Wb, G->v, opts->thread_bytes / w * 4,
+                [&](int k) { return (L.cols[k] & amask) != 0; });
+    R = G->R;
+  }
   G->grid_bit = blk;
   G->lcol.resize(G->hw_bit.size());
   for (size_t b = 0; b < G->hw_bit.size(); ++b) G->lcol[b] = L.cols[G->hw_bit[b]];
@@ -1597,27 +1625,6 @@ std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const 
 // whichever level of the kernel layout L∘σ holds bit t.  The order is a property of the
 // logical tensor alone, so the fp32 bits do not depend on L, on σ or on any plan option.
 // ---------------------------------------------------------------------------
-// More warps per CTA for the single-layout kernels (reduce, scan): a register bit of the
-// kernel layout that carries no in-tile axis bit (independent rows) becomes an extra warp
-// bit, so the CTA tile (the same packed bits: TMA staging unchanged) runs on twice the
-// warps with half the registers each — latency hiding for the dependent add / shuffle
-// chains.  `thread_bytes` (ll_plan_opts) is the register budget per thread; the vector
-// bits [0, v) stay registers, at most 5 warp bits (1024 threads).
-static void widen_warps(std::vector<int>& hw_bit, int& R, int& Wb, int v, int thread_bytes,
-                        const std::function<bool(int)>& is_axis) {
-  const int Rt = std::max(v, ilog2(u64(std::max(4, thread_bytes) / 4)));
-  while (R > Rt && Wb < 5) {
-    int b = -1;
-    for (int q = R - 1; q >= v; --q) if (!is_axis(hw_bit[q])) { b = q; break; }
-    if (b < 0) break;
-    const int pk = hw_bit[b];
-    hw_bit.erase(hw_bit.begin() + b);
-    hw_bit.push_back(pk);   // after the lanes and the existing warps: the new top warp bit
-    --R;
-    ++Wb;
-  }
-}
-
 std::unique_ptr<ReducePlan> plan_reduce(const Layout& L, int axis, const ll_plan_opts* opts) {
   if (axis < 0 || axis >= int(L.out.size())) fail(LL_ERR_INVALID_ARG, "axis out of range");
   if (!L.distributed()) fail(LL_ERR_UNSUPPORTED, "reduce: L must be a distributed layout (Def 4.10)");

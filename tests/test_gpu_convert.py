@@ -954,3 +954,20 @@ def test_reduce_scan_more_warps_bitexact(family, thread_bytes):
     ll.ll_scan(d_src, out2, s)
     rep2 = O.scan_bitdoubling_fp32(OL, 1, src)
     assert np.array_equal(out2.cpu().numpy().view(np.uint32), rep2.view(np.uint32))
+
+
+@pytest.mark.parametrize("family", ["mma", "blocked"])
+@pytest.mark.parametrize("thread_bytes", [64, 32])
+def test_gather_more_warps_bitexact(family, thread_bytes):
+    """Gather with non-axis register bits moved to extra warps (thread_bytes): O10."""
+    from tests._util import from_device, to_device, empty_device
+    rng = np.random.default_rng(1010)
+    L, OL = both(W.c4("gather", family, n_i=9, n_j=7))
+    n = 1 << OL.d_in
+    src = O.pack(OL, gen.random_bits(rng, n, 4))
+    idx = O.pack(OL, rng.integers(-50, 50, size=n).astype(np.int32))
+    plan = ll.ll_plan_gather(L, 1, 4, thread_bytes=thread_bytes)
+    assert plan.describe()["warp_bits"] > 2
+    d_dst = empty_device(n, 4)
+    ll.ll_gather(to_device(src), to_device(idx.view(np.uint32)), d_dst, plan)
+    assert np.array_equal(from_device(d_dst, 4), O.gather(OL, 1, src, idx))

@@ -154,6 +154,27 @@ def main():
                                           "warps": 1 << p.describe()["warp_bits"], "ms": round(ms, 4),
                                           "GBps": round(nbytes / ms / 1e6, 1)}), flush=True)
         return
+    if "gwarps" in only:
+        for fam in ("mma", "blocked"):
+            for ni, nj in ((12, 12), (15, 13)):
+                L = ll.Layout.from_spec(W.c4("gather", fam, n_i=ni, n_j=nj))
+                n = 1 << L.d_in
+                sets = [(torch.randint(0, 1 << 30, (n,), dtype=torch.int32, device="cuda"),
+                         torch.randint(0, 32, (n,), dtype=torch.int32, device="cuda"),
+                         torch.empty(n, dtype=torch.int32, device="cuda")) for _ in range(4 if ni == 12 else 1)]
+                for tb in (0, 64, 32):
+                    p = ll.ll_plan_gather(L, 1, 4, thread_bytes=tb)
+                    it = [0]
+
+                    def f():
+                        a = sets[it[0] % len(sets)]
+                        it[0] += 1
+                        ll.ll_gather(a[0], a[1], a[2], p)
+                    ms = time_fn(f, batch=20 if ni == 12 else 3)
+                    print(json.dumps({"case": f"gather {fam} [{1 << ni},{1 << nj}]", "thread_bytes": tb,
+                                      "warps": 1 << p.describe()["warp_bits"], "ms": round(ms, 4),
+                                      "GBps": round(12 * n / ms / 1e6, 1)}), flush=True)
+        return
     if "gtma" in only:
         # gather output by TMA bulk store vs per-thread STG, config size and 1 GiB
         for env in ("1", "0", None):
