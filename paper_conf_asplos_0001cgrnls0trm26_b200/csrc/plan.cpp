@@ -1469,13 +1469,15 @@ static std::vector<int> sigma_line(const Layout& L, int v, const std::function<b
 // bit, so the CTA tile (the same packed bits: TMA staging unchanged) runs on twice the
 // warps with half the registers each — latency hiding for the dependent add / shuffle
 // chains.  `thread_bytes` (ll_plan_opts) is the register budget per thread; the vector
-// bits [0, v) stay registers, at most 5 warp bits (1024 threads).
+// bits [0, v) stay registers, at most 5 warp bits (1024 threads).  Only bits with a
+// non-zero, non-axis column move: a zero (broadcast) column stays a dead register rather
+// than duplicating whole warps.
 static void widen_warps(std::vector<int>& hw_bit, int& R, int& Wb, int v, int thread_bytes,
-                        const std::function<bool(int)>& is_axis) {
+                        const std::function<bool(int)>& movable) {
   const int Rt = std::max(v, ilog2(u64(std::max(4, thread_bytes) / 4)));
   while (R > Rt && Wb < 5) {
     int b = -1;
-    for (int q = R - 1; q >= v; --q) if (!is_axis(hw_bit[q])) { b = q; break; }
+    for (int q = R - 1; q >= v; --q) if (movable(hw_bit[q])) { b = q; break; }
     if (b < 0) break;
     const int pk = hw_bit[b];
     hw_bit.erase(hw_bit.begin() + b);
@@ -1525,7 +1527,7 @@ std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const 
   // coalesced (line σ with the axis bits preferred in the free lanes, so that fewer
   // candidates remain in registers) unless faithful is requested: measured on B200,
   // coalesced loads beat faithful ones even at 2x the shuffles (profiles/r01_*).
-  std::vector<int> coal = sigma_line(L, v, [&](int k) { return (L.cols[k] & amask) != 0; });
+  std::vector<int> coal = sigma_line(L, v, [&](int k) { return L.cols[k] != 0 && (L.cols[k] & amask) == 0; });
   int sigma = opts ? opts->sigma : 0;
   bool use_coal = sigma != SIGMA_FAITHFUL;
   G->hw_bit = use_coal ? coal : faith;
@@ -1537,7 +1539,7 @@ std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const 
   // default keeps the layout's warps — measured in profiles/r02_sweep_gather_warps.jsonl)
   if (opts && opts->thread_bytes > 0) {
     widen_warps(G->hw_bit, G->R, G->Wb, G->v, opts->thread_bytes / w * 4,
-                [&](int k) { return (L.cols[k] & amask) != 0; });
+                [&](int k) { return L.cols[k] != 0 && (L.cols[k] & amask) == 0; });
     R = G->R;
   }
   G->grid_bit = blk;
@@ -1662,7 +1664,7 @@ std::unique_ptr<ReducePlan> plan_reduce(const Layout& L, int axis, const ll_plan
   // config-4 MMA reduce and +1.6% at 1 GiB, neutral on the blocked one; the scan keeps 512
   // (neutral either way; profiles/r02_sweep_reduce_scan_warps.jsonl)
   widen_warps(Rp->hw_bit, Rp->R, Rp->Wb, Rp->v, default_int(opts, &ll_plan_opts::thread_bytes, 256),
-              [&](int k) { return (L.cols[k] & amask) != 0; });
+              [&](int k) { return L.cols[k] != 0 && (L.cols[k] & amask) == 0; });
   R = Rp->R;
   const int n = int(Rp->hw_bit.size());
   // classify kernel bits (reduced per level, duplicate) and map each logical axis bit t
@@ -1772,7 +1774,7 @@ std::unique_ptr<ScanPlan> plan_scan(const Layout& L, int axis, const ll_plan_opt
     S->hw_bit = sigma_line(L, S->v, [&](int k) { return L.cols[k] != 0 && !(L.cols[k] & amask); });
   }
   widen_warps(S->hw_bit, S->R, S->Wb, S->v, default_int(opts, &ll_plan_opts::thread_bytes, 512),
-              [&](int k) { return (L.cols[k] & amask) != 0; });
+              [&](int k) { return L.cols[k] != 0 && (L.cols[k] & amask) == 0; });
   R = S->R;
   const int n = int(S->hw_bit.size());
   for (int t = 0; t < K; ++t) {
