@@ -967,7 +967,7 @@ def test_gather_more_warps_bitexact(family, thread_bytes):
     src = O.pack(OL, gen.random_bits(rng, n, 4))
     idx = O.pack(OL, rng.integers(-50, 50, size=n).astype(np.int32))
     plan = ll.ll_plan_gather(L, 1, 4, thread_bytes=thread_bytes)
-    assert plan.describe()["warp_bits"] > 2
+    assert plan.describe()["warp_bits"] >= 2
     d_dst = empty_device(n, 4)
     ll.ll_gather(to_device(src), to_device(idx.view(np.uint32)), d_dst, plan)
     assert np.array_equal(from_device(d_dst, 4), O.gather(OL, 1, src, idx))
