@@ -1,9 +1,11 @@
-"""The CPU oracle (oracle/ll_oracle.py, as it stands, one numpy thread) timed on each
-BASELINE config, on bounded samples of the same workloads, in the GPU side's units:
-algorithmic GB/s (conversions: read + write of each element; gather: src + idx + dst;
-reduce: src + dst).  Context for BASELINE.md §3 only, like bench.py's cpu_baseline.
+"""The CPU oracles timed on each BASELINE config, on bounded samples of the same
+workloads, in the GPU side's units: algorithmic GB/s (conversions: read + write of each
+element; gather: src + idx + dst; reduce: src + dst).  Context for BASELINE.md §3 only,
+like bench.py's cpu_baseline.
 
-    python tools/oracle_rates.py > profiles/r01_oracle_rates.jsonl
+    python tools/oracle_rates.py          > profiles/r01_oracle_rates.jsonl  (numpy, 1 thread)
+    python tools/oracle_rates.py --cpp    > profiles/r02_oracle_rates_cpp.jsonl
+                                            (C++17/OpenMP oracle: all host cores and 1 core)
 """
 import json
 import os
@@ -80,7 +82,52 @@ def c4_rates(n_i=8):
     return out
 
 
+def cpp_rates():
+    """oracle/ll_oracle.cpp on every config: all host cores (os.cpu_count() threads) and
+    one; each conversion sample is 2^22 dst elements of a smaller batch of the same tiles
+    (the block bits only index tiles), gather / reduce on [256, 4096] rows."""
+    from oracle import cpp as OC
+    ncores = os.cpu_count() or 1
+    out = []
+    convs = [("1 batch (2^20 tiles)", W.c1_batched(12), 4), ("2 (65536 tiles)", W.c2(8), 2),
+             ("3 (16384 tiles)", W.c3(7), 2), ("3b (16384 tiles)", W.c3b(7), 2),
+             ("5-T / 5 at P=1 (32768^2 bf16)", W.c5T(0, n=11), 2)]
+    for name, (sa, sb), w in convs:
+        OA, OB = O.Layout(*W.spec_to_bases(sa)), O.Layout(*W.spec_to_bases(sb))
+        src = np.random.default_rng(0).integers(0, 1 << 16, size=((1 << OA.d_in) * w) // 2, dtype=np.uint16)
+        dst = np.empty((1 << OB.d_in) * w, dtype=np.uint8)
+        row = {"config": name, "impl": "oracle/ll_oracle.cpp", "cpu_model": OC.cpu_model()}
+        for th in (ncores, 1):
+            k, dt = timed(lambda: OC.convert(OA.cols, OB.cols, OA.d_out, w, src, threads=th, out=dst), budget=3.0)
+            row["GBps_%d_cores" % th] = round(2 * w * (1 << OB.d_in) * k / dt / 1e9, 5)
+        out.append(row)
+    rng = np.random.default_rng(1)
+    for fam in ("mma", "blocked"):
+        L = O.Layout(*W.spec_to_bases(W.c4("gather", fam, n_i=8)))
+        n = 1 << L.d_in
+        src = rng.random(n, dtype=np.float32)
+        idx = rng.integers(0, 32, n, dtype=np.int32)
+        row = {"config": f"4 gather {fam}", "impl": "oracle/ll_oracle.cpp"}
+        for th in (ncores, 1):
+            k, dt = timed(lambda: OC.gather(L.cols, L.d_out, 0, 5, 4, src, idx, threads=th), budget=3.0)
+            row["GBps_%d_cores" % th] = round(12 * n * k / dt / 1e9, 5)
+        out.append(row)
+        L = O.Layout(*W.spec_to_bases(W.c4("reduce", fam, n_i=8)))
+        n = 1 << L.d_in
+        src = rng.random(n, dtype=np.float32)
+        row = {"config": f"4 reduce {fam}", "impl": "oracle/ll_oracle.cpp"}
+        for th in (ncores, 1):
+            k, dt = timed(lambda: OC.reduce(L.cols, L.d_out, 0, 12, 7, src, threads=th), budget=3.0)
+            row["GBps_%d_cores" % th] = round(4 * (n + n // 128) * k / dt / 1e9, 5)
+        out.append(row)
+    return out
+
+
 def main():
+    if "--cpp" in sys.argv:
+        for r in cpp_rates():
+            print(json.dumps(r), flush=True)
+        return
     rows = [c1_single(),
             conv_rate("1 batch (2^20 tiles)", W.c1_batched(20), 4),
             conv_rate("2 (65536 tiles)", W.c2(16), 2),
