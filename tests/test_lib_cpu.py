@@ -1063,3 +1063,16 @@ def test_broadcast_cta_class_simulated(n_zero):
             os.environ.pop("LL_BCAST_CTA", None)
         else:
             os.environ["LL_BCAST_CTA"] = old
+
+
+def test_convert_pointer_checks_before_launch():
+    """ll_convert validates its pointers before touching the GPU: 16-byte alignment
+    (LL_ERR_MISALIGNED) and src / dst overlap for non-NOOP plans (LL_ERR_ALIAS) — raw
+    addresses, nothing is dereferenced."""
+    A, B = ll.Layout.from_spec(W.C1_A), ll.Layout.from_spec(W.C1_B)
+    p = ll.ll_plan_convert(A, B, 4)
+    base = 1 << 32
+    with pytest.raises(ll.LLError, match="MISALIGNED"):
+        ll.ll_convert(base + 4, base + 4096, p, stream=0)
+    with pytest.raises(ll.LLError, match="ALIAS"):
+        ll.ll_convert(base, base + 512, p, stream=0)      # 1 KiB buffers overlapping by half
