@@ -154,6 +154,23 @@ def main():
                                           "warps": 1 << p.describe()["warp_bits"], "ms": round(ms, 4),
                                           "GBps": round(nbytes / ms / 1e6, 1)}), flush=True)
         return
+    if "n2opts" in only:
+        for shape in ("16x256b", "16x128b"):
+            sa, sb = W.n2_tmem(shape, 14)
+            for opts in ({}, {"thread_bytes": 128}, {"thread_bytes": 64}, {"force_class": "SMEM"},
+                         {"sigma": "faithful"}, {"tile_bytes": 65536}):
+                conv_case(f"n2 {shape}", sa, sb, 4, **opts)
+        for rep in range(3):
+            L = ll.Layout.from_spec(W.c4("gather", "mma", n_i=15, n_j=13))
+            p = ll.ll_plan_gather(L, 1, 4)
+            n = 1 << L.d_in
+            a = torch.randint(0, 1 << 30, (n,), dtype=torch.int32, device="cuda")
+            i = torch.randint(0, 32, (n,), dtype=torch.int32, device="cuda")
+            o = torch.empty_like(a)
+            ms = time_fn(lambda: ll.ll_gather(a, i, o, p), batch=3)
+            print(json.dumps({"case": "gather mma 1 GiB repeat", "rep": rep, "ms": round(ms, 4), "GBps": round(12 * n / ms / 1e6, 1)}), flush=True)
+            del a, i, o
+        return
     if "gwarps" in only:
         for fam in ("mma", "blocked"):
             for ni, nj in ((12, 12), (15, 13)):
