@@ -36,7 +36,17 @@ if not os.environ.get("LL_NCCL_LIB"):
         pass
 
 if not os.path.exists(_LIB_PATH):
-    raise ImportError(f"{_LIB_PATH} is missing: build it with `python -c 'import __graft_entry__ as g; g.build()'`")
+    # a fresh checkout: compile the library in-tree (nvcc for sm_100a, no GPU needed);
+    # without nvcc the import fails loudly — there is no fallback implementation
+    try:
+        import importlib.util as _ilu2
+        _bspec = _ilu2.spec_from_file_location("ll_build_lib", os.path.join(_HERE, "build_lib.py"))
+        _bmod = _ilu2.module_from_spec(_bspec)
+        _bspec.loader.exec_module(_bmod)
+        _bmod.build()
+    except Exception as _e:  # noqa: BLE001 - reported as the import error
+        raise ImportError(f"{_LIB_PATH} is missing and could not be built ({_e}); build it with "
+                          f"`python -c 'import __graft_entry__ as g; g.build()'`") from None
 _lib = C.CDLL(_LIB_PATH)
 
 STATUS = ["OK", "INVALID_ARG", "DIM_MISMATCH", "NOT_SURJECTIVE", "NOT_INVERTIBLE", "NOT_DIVISIBLE",
