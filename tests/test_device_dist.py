@@ -287,3 +287,72 @@ def test_device_peers_errors():
     assert plan.device_peers(0) == ([0, 1], [0, 1])
     with pytest.raises(ll.LLError, match="INVALID_ARG"):
         plan.device_peers(2)
+
+
+def _gpu_stage_worker(rank, world, port, q):
+    """One process per virtual rank on the one GPU: the collective DEVICE plan's real
+    pack and unpack kernels (ll_convert of the stage plans) around an exchange carried
+    by gloo (NCCL refuses two ranks on one device), routed by ll_plan_device_peers;
+    every element of this rank's slice against the closed form H(B(h, dev = r))."""
+    import torch
+    import torch.distributed as dist
+    from workloads import hashfill as HF
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        torch.cuda.set_device(0)
+        p = world.bit_length() - 1
+        n = 10
+        res = []
+        for sa, sb in ([W.c5(p, n=n), W.c5T(p, n=n)] + ([W.c5_partial(p, n=n), W.c5_partial(p, n=n, swap=True)]
+                                                        if p >= 2 else [])):
+            plan = ll.ll_plan_convert(ll.Layout.from_spec(sa), ll.Layout.from_spec(sb), 2, comm=ll.Comm.loopback(world))
+            pack, unpack, chunk, nr = plan.device_stages()
+            sp, rp = plan.device_peers(rank)
+            nloc = 1 << (2 * n - p)
+            src = HF.fill(sa, 2, 5, h0=rank * nloc, n=nloc)
+            send = torch.empty_like(src)
+            if pack:
+                ll.ll_convert(src, send, pack)
+            else:
+                send.copy_(src)
+            c2 = chunk // 2
+            sv = send.view(torch.int32).view(len(sp), c2).cpu()
+            order = sorted(range(len(sp)), key=lambda j: sp[j])
+            insz = [c2 if qq in sp else 0 for qq in range(world)]
+            outsz = [c2 if qq in rp else 0 for qq in range(world)]
+            recv_t = torch.empty(len(rp) * c2, dtype=torch.int32)
+            dist.all_to_all_single(recv_t, sv[order].contiguous().view(-1), outsz, insz)
+            by_src = dict(zip(sorted(rp), recv_t.view(len(rp), c2)))
+            recv = torch.cat([by_src[rp[i]] for i in range(len(rp))]).cuda().view(torch.int16)
+            dst = torch.empty_like(src)
+            if unpack:
+                ll.ll_convert(recv, dst, unpack)
+            else:
+                dst.copy_(recv)
+            torch.cuda.synchronize()
+            res.append(HF.check(sb, 2, 5, dst, h0=rank * nloc))
+        q.put((rank, res))
+    except Exception as e:  # pragma: no cover - reported to the parent
+        q.put((rank, repr(e)))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.gpu
+@pytest.mark.timeout(600)
+@pytest.mark.parametrize("world", [2, 4])
+def test_collective_stages_multiprocess_one_gpu(world):
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_gpu_stage_worker, args=(r, world, port, q)) for r in range(world)]
+    for pr in procs:
+        pr.start()
+    res = dict(q.get(timeout=540) for _ in procs)
+    for pr in procs:
+        pr.join(timeout=60)
+    for r, v in res.items():
+        assert isinstance(v, list) and all(x == 0 for x in v), (r, v)
