@@ -17,8 +17,10 @@ OPTION_SETS = [
     {"thread_bytes": 64},
     {"thread_bytes": 128, "tile_bytes": 32768},
     {"force_class": "SHUFFLE"},
+    {"pipe": "bulk"}, {"pipe": "bulkst"}, {"pipe": "staged"},
 ]
-KINDS = ["bijective", "bijective", "broadcast", "memory", "offset_perm", "to_memory"]
+KINDS = ["bijective", "bijective", "broadcast", "memory", "offset_perm", "to_memory",
+         "broadcast_many", "subword"]
 
 
 def _out_dims(rng, d):
@@ -60,6 +62,22 @@ def fuzz_case(rng):
             sb = gen.random_distributed(rng, out, hw, zero_ok=["reg", "lane"])
         nb = int(rng.integers(0, 5))
         return kind, W.spec_to_bases(_with_batch(sa, nb)), W.spec_to_bases(_with_batch(sb, nb)), w, opts
+    if kind == "broadcast_many":
+        # up to 8 zero columns in B (replica grid bits, dst-order broadcast stores), the
+        # batch bits possibly permuted (CTA class)
+        nz = int(rng.integers(3, 9))
+        sa, sb = gen.random_broadcast_pair(rng, nz, ki=4, kj=4, batch_bits=int(rng.integers(1, 4)),
+                                           permute_batch=bool(rng.integers(0, 2)))
+        return kind, W.spec_to_bases(sa), W.spec_to_bases(sb), w, _tiling_opts(opts)
+    if kind == "subword":
+        # 1- / 2-byte elements on random SHUFFLE-class pairs (element-permuted shuffles)
+        r = int(rng.integers(3, 6))
+        hw = [("reg", r), ("lane", 5), ("warp", 10 - r - 5)]
+        out = [("i", 5), ("j", 5)]
+        sa, sb = gen.random_distributed(rng, out, hw), gen.random_distributed(rng, out, hw)
+        nb = int(rng.integers(0, 3))
+        return kind, W.spec_to_bases(_with_batch(sa, nb)), W.spec_to_bases(_with_batch(sb, nb)), \
+            [1, 2][int(rng.integers(0, 2))], {}
     if kind == "memory":
         # Def 4.14 memory layouts with 1- and 2-bit columns (swizzles, R2)
         d = int(rng.integers(6, 13))
