@@ -48,6 +48,15 @@
  *    inside the tile loop; default on for linear tiles only).
  *  - LL_LINEAR_BALANCE=0: linear CTA tiles (general invertible pull maps) take the
  *    widest store runs instead of the default balanced load/store run lengths.
+ *  - LL_BCAST=0: broadcast targets store their low replica bits per thread instead of
+ *    through the dst-order smem read-back (TilePlan::bcast).
+ *  - LL_BCAST_CTA=1|0: CTA-class broadcast maps try the CTA-tiled broadcast before (1)
+ *    or never (0) instead of after the XOR-copy tiles (default).
+ *  - LL_SCAN_TMA_STORE=0|1, LL_GATHER_TMA_STORE=0|1: scan / gather outputs stored per
+ *    thread (0) or through the stage by cp.async.bulk (1); default: bulk stores for
+ *    launches of <= 4096 tiles.
+ *  - LL_XOR_INVEC=0: XOR-copy tiles shrink the vector instead of permuting in registers.
+ *  - LL_ISOLATE_SMEM=1: diagnostic smem-exchange-only tile kernels (no global traffic).
  *  Host entry points (planning, launches) are wrapped in NVTX ranges named after
  *  the call (ll_plan_convert, ll_convert, ll_gather, ll_reduce, ll_scan).
  */
