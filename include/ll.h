@@ -57,6 +57,12 @@
  *    launches of <= 4096 tiles.
  *  - LL_XOR_INVEC=0: XOR-copy tiles shrink the vector instead of permuting in registers.
  *  - LL_ISOLATE_SMEM=1: diagnostic smem-exchange-only tile kernels (no global traffic).
+ *  - LL_GRID_PER_SM=k: cap tile-kernel grids at k CTAs per SM (persistent CTAs looping
+ *    over tiles); default / 0: one CTA per tile.
+ *  - LL_ST_HINT=wb: tile kernels store with the default write-back policy instead of
+ *    st.global.cs (evict-first streaming).
+ *  - LL_NCCL_LIB=<path>: the libnccl.so.2 dlopen'ed for DEVICE plans (the Python binding
+ *    points it at torch's NCCL).
  *  Host entry points (planning, launches) are wrapped in NVTX ranges named after
  *  the call (ll_plan_convert, ll_convert, ll_gather, ll_reduce, ll_scan).
  */
