@@ -398,6 +398,7 @@ def other_configs(ll, W, torch, peak):
         ms_t = _time_stream(tg, torch)
         out.append({"workload": f"config 4 gather: [4096,4096] fp32, {fam} [128,32] tiles", "class": "gather",
                     "executed": d["exchange"] + (" (TMA stages)" if d.get("tma") else ""), "ms": round(ms, 4),
+                    "shuffles_per_elem": d.get("shuffles_per_elem"),
                     "GBps": round(gbs, 1), "frac": round(gbs / peak, 3),
                     "torch_gather_same_bytes_GBps": round(12 * n / ms_t / 1e6, 1),
                     "size_matched_copy_GBps": size_matched_copy(torch, 12 * n)})
@@ -684,7 +685,9 @@ def main():
                        "parallelism": f"dp{world} (independent tiles, no communication)"},
             "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                          "frac": round(achieved / peak, 4), "peak_kind": peak_kind,
+                         "frac_of_nominal_8TBps": round(achieved / 8000.0, 4),
                          "traffic": traffic, "kernel": "ll_tile_kernel (shuffle)",
+                         "traffic_over_algorithmic": round(traffic / bytes_per_step, 4) if traffic else None,
                          "bytes_per_launch": bytes_per_step, "avg_launch_ms": round(avg_launch_ms, 5)},
             "e2e": {"value": round(world * bytes_per_step / (e2e_ms / 1e3) / 1e9, 2), "unit": "GB/s",
                     "h2d_bytes_per_step": n * w, "d2h_bytes_per_step": n * w, "ms_per_step": round(e2e_ms, 3),
