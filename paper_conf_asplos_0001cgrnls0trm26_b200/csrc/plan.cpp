@@ -1527,7 +1527,7 @@ std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const 
   // coalesced (line σ with the axis bits preferred in the free lanes, so that fewer
   // candidates remain in registers) unless faithful is requested: measured on B200,
   // coalesced loads beat faithful ones even at 2x the shuffles (profiles/r01_*).
-  std::vector<int> coal = sigma_line(L, v, [&](int k) { return L.cols[k] != 0 && (L.cols[k] & amask) == 0; });
+  std::vector<int> coal = sigma_line(L, v, [&](int k) { return (L.cols[k] & amask) != 0; });
   int sigma = opts ? opts->sigma : 0;
   bool use_coal = sigma != SIGMA_FAITHFUL;
   G->hw_bit = use_coal ? coal : faith;
