@@ -314,7 +314,7 @@ def other_configs(ll, W, torch, peak):
         if "tile" in d:
             ex = d["tile"]["xchg"]
         elif d.get("exchange") == "peer":
-            ex = "peer stores: one %s tile kernel per rank" % d["fused"]["tile"]["xchg"]
+            ex = "peer stores: %s tile kernel into the receivers' windows" % d["fused"]["tile"]["xchg"]
         else:
             ex = d["exec"]
         entry = {"workload": name, "class": d["class"], "executed": ex, "ms": round(ms, 4),
@@ -421,7 +421,7 @@ def other_configs(ll, W, torch, peak):
             torch.sum(s[0].view(4096, 32, 128), dim=2, out=s[1].view(4096, 32))
         ms_t = _time_stream(tr, torch)
         out.append({"workload": f"config 4 reduce: [4096,4096] fp32 -> [4096,32], {fam} [128,128] tiles",
-                    "class": "reduce", "executed": "tree + shfl.bfly" + (" (TMA stages)" if p.describe().get("tma") else ""),
+                    "class": "reduce", "executed": "logical-order steps (register / shfl.bfly / smem)" + (" (TMA stages)" if p.describe().get("tma") else ""),
                     "ms": round(ms, 4), "GBps": round(gbs, 1), "frac": round(gbs / peak, 3),
                     "torch_sum_same_bytes_GBps": round((4 * n + 4 * p.out_elems()) / ms_t / 1e6, 1),
                     "size_matched_copy_GBps": size_matched_copy(torch, 4 * n + 4 * p.out_elems())})
