@@ -145,7 +145,13 @@ typedef struct {
                          * 4 = bulk (CTA tile contiguous in src order: whole tiles by
                          * cp.async.bulk into 2-3 raw stages, mbarrier completion),
                          * 5 = bulk load + bulk store (the dst tile, contiguous in dst
-                         * order, leaves by cp.async.bulk from a dst stage)           */
+                         * order, leaves by cp.async.bulk from a dst stage).
+                         * ll_plan_reduce / ll_plan_scan: 0 = auto (reduce: TMA stages
+                         * only for >= 64 KiB tiles with an axis bit on the warps;
+                         * scan: direct loads),
+                         * 1 = direct 16-byte loads, 4 = TMA stages (cp.async.bulk of
+                         * the contiguous CTA tile), 5 = TMA stages and (scan) the
+                         * result tile out by cp.async.bulk                          */
   int min_blocks;       /* tile kernels: resident CTAs per SM requested from ptxas
                          * (__launch_bounds__ minimum): 0 = auto (2 for linear tiles,
                          * else none), -1 = none, k >= 1 = k                          */
@@ -341,10 +347,13 @@ ll_status ll_plan_autotune(const ll_layout* A, const ll_layout* B, int elem_byte
  * must be the low bits of the axis coordinate.  out[x] = src[x with the axis
  * coordinate's low bits replaced by idx[x] & (K-1)] (take_along_axis inside each
  * tile; out-of-range indices are masked).  Warp shuffles when
- * L_Wrp^axis = 0 and at most 4 candidate registers remain, else a
+ * L_Wrp^axis = 0 and at most 2 candidate registers remain, else a
  * shared-memory gather over the staged CTA tile (any axis placement; the P:519
  * crossover); opts->force_class SHUFFLE / SMEM selects one (SHUFFLE with warp axis
- * bits: LL_ERR_UNSUPPORTED). */
+ * bits: LL_ERR_UNSUPPORTED).  Direct 16-byte loads with opts->thread_bytes (default
+ * 32) bytes of data per thread (non-axis register bits become warps); opts->pipe = 4
+ * / 5 stages the src and idx tiles by cp.async.bulk (TMA) instead (5: and the dst tile
+ * leaves by cp.async.bulk). */
 ll_status ll_plan_gather(const ll_layout* L, int axis, int elem_bytes,
                          const ll_plan_opts* opts, ll_plan** plan);
 /* src, dst: packed in L; idx: int32 packed in L. */

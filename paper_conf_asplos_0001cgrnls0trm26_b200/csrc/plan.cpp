@@ -1535,10 +1535,14 @@ std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const 
   G->R = R;
   G->Wb = int(warpb.size());
   G->v = use_coal ? v : std::min(ilog2(u64(std::max(1, maxvec / ev))), R);
-  // optional extra warps from non-axis register bits (ll_plan_opts.thread_bytes; the
-  // default keeps the layout's warps — measured in profiles/r02_sweep_gather_warps.jsonl)
-  if (opts && opts->thread_bytes > 0) {
-    widen_warps(G->hw_bit, G->R, G->Wb, G->v, opts->thread_bytes / w * 4,
+  // extra warps from non-axis register bits (ll_plan_opts.thread_bytes, default 32 bytes
+  // of data per thread): measured over the config-4 gathers and Table 4 families x 3 tile
+  // shapes at 64 MiB and 1 GiB (profiles/r02_sweep_gather_families.jsonl), direct loads
+  // with 32 bytes per thread are within 3% of the best of 24 variants on every case and
+  // +5-24% over the former default (the layout's own warps and TMA stages)
+  {
+    const int tb = default_int(opts, &ll_plan_opts::thread_bytes, 32);
+    widen_warps(G->hw_bit, G->R, G->Wb, G->v, tb / w * 4,
                 [&](int k) { return L.cols[k] != 0 && (L.cols[k] & amask) == 0; });
     R = G->R;
   }
@@ -1556,12 +1560,14 @@ std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const 
     for (int l = 0; l < 5; ++l) if (G->lcol[R + l] == c) { G->axis_lane_pos[t] = l; G->axis_of_lane[l] = t; }
   }
   // shuffles vs shared memory: the paper observes the shuffle rounds lose once
-  // the gathered dimension grows; the planner switches when more than 4
-  // candidates per element remain (force_class selects either)
+  // the gathered dimension grows; the planner switches when more than 2
+  // candidates per element remain — with 4 candidates the shuffle gather measured 0.3-17%
+  // behind the smem one, with 2 even (profiles/r02_sweep_gather_families.jsonl);
+  // force_class selects either
   int force = opts ? opts->force_class : -1;
   if (warp_axis && force == LL_CLASS_SHUFFLE)
     fail(LL_ERR_UNSUPPORTED, "gather: L_Wrp^axis != 0 (P:430): the shuffle gather needs the axis off the warps");
-  G->smem = warp_axis || force == LL_CLASS_SMEM || (force != LL_CLASS_SHUFFLE && G->cand_bits > 2);
+  G->smem = warp_axis || force == LL_CLASS_SMEM || (force != LL_CLASS_SHUFFLE && G->cand_bits > 1);
   // smem layout of the staged tile: vector registers, then lanes, then the other
   // registers, then warps (offset order kreg[0,v), klane, kreg[v,R), kwarp), so the
   // staging stores are whole 16-byte vectors with consecutive lanes on consecutive
@@ -1591,7 +1597,9 @@ std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const 
   const u64 ne = u64(1) << G->lcol.size();
   const u64 gbytes = G->smem ? ne * u64(w) : 0;
   // TMA staging (cp.async.bulk of the contiguous src and idx tiles, 2 stages) with the
-  // line-coalesced σ; force_class = CTA keeps direct LDG loads (a diagnostic knob)
+  // line-coalesced σ, on request (opts->pipe = 4 bulk / 5 bulk + bulk store): the default
+  // direct loads with 32 bytes per thread beat it on every measured case
+  // (profiles/r02_sweep_gather_families.jsonl); force_class = CTA keeps direct loads
   bool contiguous = true;
   {
     int p = 0;
@@ -1602,11 +1610,12 @@ std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const 
   }
   G->stages = 2;
   const u64 stage_bytes = ne * u64(w + 4);
-  // measured (profiles/r01_sweep_gather_tma.jsonl, r01_sweep_gather_smem_vec.jsonl):
-  // the bulk-copy pipeline wins from 32 KiB stages (K = 32 smem gather: +4%; K = 64:
-  // +10-15%), direct LDG wins below (K = 16: +5-8%)
-  G->tma = G->sigma == SIGMA_COALESCED && contiguous && force != LL_CLASS_CTA &&
-           (stage_bytes >= 32768 || force == LL_CLASS_SHUFFLE || force == LL_CLASS_SMEM) &&
+  // (round 1 measured the bulk-copy pipeline ahead of direct loads at the layouts' own
+  // warp counts from 32 KiB stages, profiles/r01_sweep_gather_tma.jsonl; with extra warps
+  // the direct loads win, profiles/r02_sweep_gather_families.jsonl)
+  const int pipe = opts ? opts->pipe : 0;
+  const bool tma_want = pipe == 4 || pipe == 5;
+  G->tma = G->sigma == SIGMA_COALESCED && contiguous && force != LL_CLASS_CTA && tma_want &&
            u64(G->stages) * stage_bytes + gbytes + 16 <= 200 * 1024 && (G->v + ilog2(u64(w))) >= 2;
   G->smem_bytes = int(gbytes + (G->tma ? u64(G->stages) * stage_bytes + 8 * G->stages : 0));
   // outputs through the stage and one cp.async.bulk per tile, as for the scan: for
@@ -1615,7 +1624,7 @@ std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const 
   {
     const char* e = std::getenv("LL_GATHER_TMA_STORE");
     const bool small = G->grid_bit.size() <= 12;
-    G->tma_store = G->tma && (G->w << G->v) >= 4 && (e ? std::string(e) == "1" : small);
+    G->tma_store = G->tma && (G->w << G->v) >= 4 && (e ? std::string(e) == "1" : (pipe == 5 || small));
   }
   return G;
 }
@@ -1660,10 +1669,21 @@ std::unique_ptr<ReducePlan> plan_reduce(const Layout& L, int axis, const ll_plan
     Rp->sigma = SIGMA_COALESCED;
     Rp->hw_bit = sigma_line(L, Rp->v, [&](int k) { return L.cols[k] != 0 && !(L.cols[k] & amask); });
   }
-  // default 256 bytes per thread (8 warps on a [128,128] fp32 tile): measured +5% on the
-  // config-4 MMA reduce and +1.6% at 1 GiB, neutral on the blocked one; the scan keeps 512
-  // (neutral either way; profiles/r02_sweep_reduce_scan_warps.jsonl)
-  widen_warps(Rp->hw_bit, Rp->R, Rp->Wb, Rp->v, default_int(opts, &ll_plan_opts::thread_bytes, 256),
+  // an axis bit on the warps needs a shared-memory step; widen_warps moves only non-axis
+  // bits, so this is known before it
+  bool warp_axis = false;
+  for (size_t b = R + 5; b < Rp->hw_bit.size(); ++b)
+    if (L.cols[Rp->hw_bit[b]] & amask) warp_axis = true;
+  // default bytes per thread and load path, measured over the Table 4 families x 3 tile
+  // shapes x 2 axes at 64 MiB and 1 GiB (profiles/r02_sweep_reduce_scan_families.jsonl):
+  // direct LDG loads with 128 bytes per thread (16 warps on a 64 KiB tile, several CTAs per
+  // SM) beat the one-CTA-per-SM TMA pipeline on 38 of 48 cases (+4-8% on 64 KiB tiles, up
+  // to 2.3x on 8 KiB tiles); the TMA pipeline with 256 bytes per thread stays for 64 KiB
+  // tiles whose reduction has a shared-memory (warp) step, where it is even or ahead (up to
+  // +21%).  opts->pipe = 4 (bulk) forces the TMA stages, force_class = SHUFFLE the LDG path.
+  const bool big_tile = R + 5 + Rp->Wb >= 14;
+  const bool tma_auto = warp_axis && big_tile;
+  widen_warps(Rp->hw_bit, Rp->R, Rp->Wb, Rp->v, default_int(opts, &ll_plan_opts::thread_bytes, tma_auto ? 256 : 128),
               [&](int k) { return L.cols[k] != 0 && (L.cols[k] & amask) == 0; });
   R = Rp->R;
   const int n = int(Rp->hw_bit.size());
@@ -1729,10 +1749,12 @@ std::unique_ptr<ReducePlan> plan_reduce(const Layout& L, int axis, const ll_plan
     }
   }
   int force = opts ? opts->force_class : -1;
+  const int pipe = opts ? opts->pipe : 0;
   Rp->stages = 0;
   for (int ns = 4; ns >= 2; --ns)
     if (u64(ns) * tile_bytes + u64(Rp->wred_bytes) + 8 * ns <= 200 * 1024) { Rp->stages = ns; break; }
-  Rp->tma = Rp->sigma == SIGMA_COALESCED && Rp->v == 2 && contiguous && force != LL_CLASS_SHUFFLE && Rp->stages;
+  Rp->tma = Rp->sigma == SIGMA_COALESCED && Rp->v == 2 && contiguous && force != LL_CLASS_SHUFFLE && Rp->stages &&
+            (pipe == 4 || pipe == 5 || (pipe == 0 && tma_auto));
   Rp->smem_bytes = Rp->tma ? int(Rp->stages * tile_bytes + Rp->wred_bytes + 8 * Rp->stages) : Rp->wred_bytes;
   return Rp;
 }
@@ -1773,7 +1795,10 @@ std::unique_ptr<ScanPlan> plan_scan(const Layout& L, int axis, const ll_plan_opt
     // axis bits stay in registers where possible (register steps need no shuffle)
     S->hw_bit = sigma_line(L, S->v, [&](int k) { return L.cols[k] != 0 && !(L.cols[k] & amask); });
   }
-  widen_warps(S->hw_bit, S->R, S->Wb, S->v, default_int(opts, &ll_plan_opts::thread_bytes, 512),
+  // default 128 bytes per thread with direct LDG loads: measured over the Table 4 families
+  // (profiles/r02_sweep_reduce_scan_families.jsonl) it beats the TMA pipeline (one CTA per
+  // SM) on 46 of 48 cases, +5-14% on 64 KiB tiles and up to 1.8x on 8 KiB tiles
+  widen_warps(S->hw_bit, S->R, S->Wb, S->v, default_int(opts, &ll_plan_opts::thread_bytes, 128),
               [&](int k) { return L.cols[k] != 0 && (L.cols[k] & amask) == 0; });
   R = S->R;
   const int n = int(S->hw_bit.size());
@@ -1797,9 +1822,9 @@ std::unique_ptr<ScanPlan> plan_scan(const Layout& L, int axis, const ll_plan_opt
     else if (!hreg) lane_below = true;
     else ++low_reg_bits;
   }
-  // TMA staging as for the reduce: contiguous CTA tile (reg, lane, warp are L's lowest
-  // packed bits), line σ with 16-byte reads, 2-4 stages in smem; force_class = SHUFFLE
-  // keeps direct LDG loads
+  // TMA staging (on request, opts->pipe = 4 / 5) as for the reduce: contiguous CTA tile
+  // (reg, lane, warp are L's lowest packed bits), line σ with 16-byte reads, 2-3 stages in
+  // smem; force_class = SHUFFLE keeps direct LDG loads
   const u64 tile_bytes = u64(4) << (R + 5 + S->Wb);
   bool contiguous = true;
   {
@@ -1810,20 +1835,23 @@ std::unique_ptr<ScanPlan> plan_scan(const Layout& L, int axis, const ll_plan_opt
     }
   }
   const int force = opts ? opts->force_class : -1;
+  const int pipe = opts ? opts->pipe : 0;
   for (int ns = 3; ns >= 2; --ns)
     if (u64(ns) * tile_bytes + u64(S->xs_bytes) + 8 * ns <= 200 * 1024) { S->stages = ns; break; }
-  S->tma = S->sigma == SIGMA_COALESCED && S->v == 2 && contiguous && force != LL_CLASS_SHUFFLE && S->stages > 0;
+  // TMA stages only on request (opts->pipe = 4 bulk / 5 bulk + bulk store)
+  S->tma = S->sigma == SIGMA_COALESCED && S->v == 2 && contiguous && force != LL_CLASS_SHUFFLE && S->stages > 0 &&
+           (pipe == 4 || pipe == 5);
   // The results can go back into the stage they were read from (each thread rewrites the
   // 16-byte vectors it read) and leave by one cp.async.bulk shared -> global per tile
   // (the dst tile is contiguous like the src tile): the LSU then carries no global
   // stores.  Measured (profiles/r02_sweep_scan.jsonl): +4.5% on the config-4 size (1024
   // tiles, ramp-bound), -4% at 1 GiB (16384 tiles), where the stage held by the in-flight
-  // store shortens the load pipeline — so only for launches of <= 4096 tiles.
-  // LL_SCAN_TMA_STORE=0 / 1 forces either.
+  // store shortens the load pipeline — so with TMA stages, only for launches of <= 4096
+  // tiles, or when opts->pipe = 5 (bulkst) asks for it.  LL_SCAN_TMA_STORE=0 / 1 forces either.
   {
     const char* e = std::getenv("LL_SCAN_TMA_STORE");
     const bool small = S->grid_bit.size() <= 12;
-    S->tma_store = S->tma && (e ? std::string(e) == "1" : small);
+    S->tma_store = S->tma && (e ? std::string(e) == "1" : (pipe == 5 || small));
   }
   S->smem_bytes = S->tma ? int(S->stages * tile_bytes + S->xs_bytes + 8 * S->stages) : S->xs_bytes;
   if (S->smem_bytes > 200 * 1024) fail(LL_ERR_UNSUPPORTED, "scan: tile too large for the shared-memory exchange");

@@ -181,9 +181,12 @@ def test_gather_bitexact(family, sigma, k_bits, exchange):
     Ti = rng.integers(-1000, 1000, size=n).astype(np.int32)   # masked to [0, K) (G16)
     src, idx = O.pack(OL, T), O.pack(OL, Ti)
     ref = O.gather(OL, 1, src, idx)
-    # SHUFFLE / SMEM: forced exchange (TMA-staged when coalesced); LDG: automatic
-    # exchange with direct global loads (force_class = CTA)
-    plan = ll.ll_plan_gather(L, 1, 4, sigma=sigma, force_class="CTA" if exchange == "LDG" else exchange)
+    # SHUFFLE / SMEM: forced exchange, TMA-staged when coalesced (pipe = bulk); LDG: the
+    # default plan (automatic exchange, direct global loads)
+    if exchange == "LDG":
+        plan = ll.ll_plan_gather(L, 1, 4, sigma=sigma)
+    else:
+        plan = ll.ll_plan_gather(L, 1, 4, sigma=sigma, force_class=exchange, pipe="bulk")
     d = plan.describe()
     if exchange != "LDG":
         assert d["exchange"] == exchange.lower()
@@ -212,7 +215,7 @@ def test_gather_narrow_elements(w, exchange):
 
 
 @pytest.mark.parametrize("family", ["mma", "blocked"])
-@pytest.mark.parametrize("sigma", ["coalesced", "coalesced-ldg", "faithful"])
+@pytest.mark.parametrize("sigma", ["coalesced", "coalesced-tma", "faithful"])
 def test_reduce_tolerance_and_fixed_order(family, sigma):
     """O11: ≤ 1e-6 relative vs fp64, and bit-exact vs the fixed-order fp32 replica on
     L itself (reading R-reduce: logical axis-bit order), for every kernel layout σ and
@@ -224,10 +227,10 @@ def test_reduce_tolerance_and_fixed_order(family, sigma):
     n = 1 << OL.d_in
     T = rng.random(n, dtype=np.float32)
     src = O.pack(OL, T)
-    # "coalesced" stages tiles with cp.async.bulk (TMA), "coalesced-ldg" loads directly
-    plan = ll.ll_plan_reduce(L, 1, sigma=sigma.split("-")[0],
-                             force_class="SHUFFLE" if sigma == "coalesced-ldg" else None)
-    assert plan.describe()["tma"] == (sigma == "coalesced")
+    # "coalesced" loads directly (the default for reduces without a warp step),
+    # "coalesced-tma" stages tiles with cp.async.bulk (TMA, opts.pipe = bulk)
+    plan = ll.ll_plan_reduce(L, 1, sigma=sigma.split("-")[0], pipe="bulk" if sigma == "coalesced-tma" else "auto")
+    assert plan.describe()["tma"] == (sigma == "coalesced-tma")
     out = torch.empty(plan.out_elems(), dtype=torch.float32, device="cuda")
     ll.ll_reduce(torch.from_numpy(src).cuda(), out, plan)
     got = out.cpu().numpy()
@@ -486,9 +489,10 @@ def test_table4_reduce_families(family):
             got = out.cpu().numpy()
             ref = T.astype(np.float64).reshape(shape).sum(axis=axis)
             assert np.all(np.abs(got - ref) <= 1e-6 * np.abs(ref)), (family, shape, axis)
-            for sigma in ("coalesced", "faithful"):
-                if sigma == "faithful":
-                    plan = ll.ll_plan_reduce(L, axis, sigma="faithful")
+            for sigma in ("coalesced", "faithful", "bulk"):
+                if sigma != "coalesced":
+                    plan = (ll.ll_plan_reduce(L, axis, sigma="faithful") if sigma == "faithful" else
+                            ll.ll_plan_reduce(L, axis, pipe="bulk"))
                     out.fill_(-1.0)
                     ll.ll_reduce(torch.from_numpy(src).cuda(), out, plan)
                     got = out.cpu().numpy()
@@ -650,16 +654,21 @@ def test_scan_bitexact(family, sigma):
 
 
 @pytest.mark.parametrize("family", ["mma", "blocked"])
-def test_scan_fullsize_tma_store(family):
+@pytest.mark.parametrize("pipe", ["auto", "bulk"])
+def test_scan_fullsize_tma_store(family, pipe):
     """Config-4 scan on the whole [4096, 4096] fp32 tensor in [128, 128] tiles, in the
-    bench's launch configuration (TMA stages in, results back through the stage and out by
-    cp.async.bulk): every element bit-equal to the oracle's fixed-order recurrence."""
+    bench's launch configuration (auto: direct 16-byte loads and stores, 16 warps) and
+    with TMA stages (bulk: tiles in by cp.async.bulk, results back through the stage and
+    out by cp.async.bulk): every element bit-equal to the oracle's fixed-order recurrence."""
     import torch
     spec = W.c4("reduce", family)
     L, OL = both(spec)
-    plan = ll.ll_plan_scan(L, 1)
+    plan = ll.ll_plan_scan(L, 1, pipe=pipe)
     d = plan.describe()
-    assert d["tma"] and d["tma_store"]        # 1024 tiles: the bulk-store path
+    if pipe == "bulk":
+        assert d["tma"] and d["tma_store"]        # 1024 tiles: the bulk-store path
+    else:
+        assert not d["tma"] and d["warp_bits"] == 4
     T = np.random.default_rng(1008).random(1 << OL.d_out, dtype=np.float32)
     src = O.pack(OL, T)
     out = torch.empty(src.size, dtype=torch.float32, device="cuda")
@@ -714,11 +723,13 @@ def test_table4_scan_families(family):
                 # per thread and register) exceeds shared memory (the 512-register custom tile)
                 assert "too large" in str(e), (family, shape, axis, e)
                 continue
-            out = torch.empty(src.size, dtype=torch.float32, device="cuda")
-            ll.ll_scan(torch.from_numpy(src).cuda(), out, plan)
-            got = out.cpu().numpy()
             rep = O.scan_bitdoubling_fp32(OL, axis, src)
-            assert np.array_equal(got.view(np.uint32), rep.view(np.uint32)), (family, shape, axis)
+            # default plan (direct loads), then TMA stages with the bulk store (pipe = bulkst)
+            for p in (plan, ll.ll_plan_scan(L, axis, pipe="bulkst")):
+                out = torch.empty(src.size, dtype=torch.float32, device="cuda")
+                ll.ll_scan(torch.from_numpy(src).cuda(), out, p)
+                got = out.cpu().numpy()
+                assert np.array_equal(got.view(np.uint32), rep.view(np.uint32)), (family, shape, axis)
             ran += 1
     assert ran >= 8
 

@@ -131,6 +131,42 @@ def main():
                                       "ms": round(ms, 4), "GBps": round(8 * n / ms / 1e6, 1)}), flush=True)
                     del sets
         return
+    if "scanldg" in only:
+        # scans / reduces: TMA stages (one CTA per SM with 3 x 64 KiB stages) vs direct LDG
+        # loads (force_class = SHUFFLE: several CTAs per SM), at 512 / 256 / 128 / 64 bytes per
+        # thread; config-4 size (4 rotating buffer sets) and 1 GiB
+        for kind in ("scan", "reduce"):
+            for fam in ("mma", "blocked"):
+                for ni, nj in ((12, 12), (15, 13)):
+                    L = ll.Layout.from_spec(W.c4("reduce", fam, n_i=ni, n_j=nj))
+                    n = 1 << L.d_in
+                    nset = 4 if ni == 12 else 1
+                    sets = [torch.rand(n, device="cuda") for _ in range(nset)]
+                    for opts in ({}, {"thread_bytes": 256}, {"thread_bytes": 128}, {"force_class": "SHUFFLE"},
+                                 {"force_class": "SHUFFLE", "thread_bytes": 256},
+                                 {"force_class": "SHUFFLE", "thread_bytes": 128},
+                                 {"force_class": "SHUFFLE", "thread_bytes": 64}):
+                        p = (ll.ll_plan_scan if kind == "scan" else ll.ll_plan_reduce)(L, 1, **opts)
+                        m = n if kind == "scan" else p.out_elems()
+                        outs = [torch.empty(m, device="cuda") for _ in sets]
+                        it = [0]
+
+                        def f():
+                            k = it[0] % nset
+                            it[0] += 1
+                            (ll.ll_scan if kind == "scan" else ll.ll_reduce)(sets[k], outs[k], p)
+                        ms = time_fn(f, batch=20 if ni == 12 else 3)
+                        d = p.describe()
+                        print(json.dumps({"case": f"{kind} {fam} [{1 << ni},{1 << nj}]", "opts": opts, "tma": d["tma"],
+                                          "warps": 1 << d["warp_bits"], "R": d["R"], "ms": round(ms, 4),
+                                          "GBps": round(4 * (n + m) / ms / 1e6, 1)}), flush=True)
+                        del outs
+                    del sets
+        return
+    if "redfam" in only:
+        return reduce_scan_families()
+    if "gathfam" in only:
+        return gather_families()
     if "warps" in only:
         # reduce / scan with non-axis register bits moved to warps (thread_bytes)
         for fam in ("mma", "blocked"):
@@ -280,6 +316,118 @@ def main():
         conv_case("c1batch", sa, sb, 4, **opts)
     gather_reduce()
 
+
+
+def _batched(L, nb):
+    """L (reg, lane, warp -> 2 dims) times 2^nb CTAs on a new leading batch dim."""
+    ins, outs = L.in_dims, L.out_dims
+    vecs = L.bases()
+    bases, k = {}, 0
+    for n, b in ins:
+        bases[n] = [(0,) + tuple(v) for v in vecs[k:k + b]]
+        k += b
+    bases["block"] = [tuple([1 << q] + [0] * len(outs)) for q in range(nb)]
+    return ll.Layout(list(ins) + [("block", nb)], [("b", nb)] + list(outs), bases)
+
+
+def reduce_scan_families():
+    """Reduce and scan over Table 4 families batched to 64 MiB and 1 GiB of
+    fp32: TMA stages (one CTA per SM) vs direct LDG loads at 16 warps."""
+    import numpy as np
+    from workloads import gen
+    rng = np.random.default_rng(77)
+    fams = {
+        "blocked": lambda a, b: ll.ll_layout_blocked([a, b], [1, 4], [8, 4], [4, 1], [1, 0]),
+        "mma": lambda a, b: ll.ll_layout_mma_acc(a, b, 4),
+        "mma_input": lambda a, b: ll.ll_layout_mma_operand(0, a, b, 16, 4, 1),
+        "custom": lambda a, b: ll.Layout.from_spec(gen.random_distributed(
+            rng, [("r", a.bit_length() - 1), ("c", b.bit_length() - 1)],
+            [("reg", max(1, a.bit_length() + b.bit_length() - 2 - 7)), ("lane", 5), ("warp", 2)],
+            zero_ok=["reg", "lane", "warp"])),
+    }
+    for fam, mk in fams.items():
+        for shape in ((128, 128), (128, 16), (32, 128)):
+            T = mk(*shape)
+            for total in (24, 28):
+                L = _batched(T, total - T.d_in)
+                n = 1 << L.d_in
+                nset = 4 if total == 24 else 1
+                sets = [torch.rand(n, device="cuda") for _ in range(nset)]
+                for axis in (1, 2):
+                    for kind in ("reduce", "scan"):
+                        res = {}
+                        for tag, opts in (("default", {}), ("tma16w", {"thread_bytes": 128}),
+                                          ("ldg", {"force_class": "SHUFFLE"}),
+                                          ("ldg16w", {"force_class": "SHUFFLE", "thread_bytes": 128})):
+                            try:
+                                p = (ll.ll_plan_scan if kind == "scan" else ll.ll_plan_reduce)(L, axis, **opts)
+                            except Exception as e:   # noqa: BLE001
+                                res[tag] = str(e)[:80]
+                                continue
+                            m = n if kind == "scan" else p.out_elems()
+                            outs = [torch.empty(m, device="cuda") for _ in sets]
+                            it = [0]
+
+                            def f():
+                                k = it[0] % nset
+                                it[0] += 1
+                                (ll.ll_scan if kind == "scan" else ll.ll_reduce)(sets[k], outs[k], p)
+                            ms = time_fn(f, batch=20 if total == 24 else 3)
+                            d = p.describe()
+                            res[tag] = {"tma": d["tma"], "warps": 1 << d["warp_bits"],
+                                        "GBps": round(4 * (n + m) / ms / 1e6, 1)}
+                            del outs
+                        print(json.dumps({"kind": kind, "family": fam, "shape": shape, "axis": axis - 1,
+                                          "MiB": (4 * n) >> 20, "res": res}), flush=True)
+                del sets
+
+
+def gather_families():
+    """Gather (4-byte elements, int32 indices) over Table 4 families batched to 64 MiB and
+    1 GiB of src, and the config-4 gather layouts: load path (TMA stages: pipe = bulk;
+    direct LDG: pipe = off) x bytes per thread (extra warps) x exchange (auto / smem)."""
+    cases = []
+    fams = {
+        "blocked": lambda a, b: ll.ll_layout_blocked([a, b], [1, 4], [8, 4], [4, 1], [1, 0]),
+        "mma": lambda a, b: ll.ll_layout_mma_acc(a, b, 4),
+    }
+    for fam in ("mma", "blocked"):
+        for ni, nj in ((12, 12), (15, 13)):
+            cases.append((f"c4_{fam}", (128, 32), ll.Layout.from_spec(W.c4("gather", fam, n_i=ni, n_j=nj)), 1, 32))
+    for fam, mk in fams.items():
+        for shape in ((128, 128), (128, 16), (32, 128)):
+            T = mk(*shape)
+            for total in (24, 28):
+                for axis in (1, 2):
+                    cases.append((fam, shape, _batched(T, total - T.d_in), axis, shape[axis - 1]))
+    for fam, shape, L, axis, K in cases:
+        n = 1 << L.d_in
+        nset = 4 if n <= (1 << 24) else 1
+        sets = [(torch.randint(0, 1 << 30, (n,), dtype=torch.int32, device="cuda"),
+                 torch.randint(0, K, (n,), dtype=torch.int32, device="cuda"),
+                 torch.empty(n, dtype=torch.int32, device="cuda")) for _ in range(nset)]
+        res = {}
+        for pipe in ("auto", "bulk", "off"):
+            for tb in (0, 64, 32, 16):
+                for fc in (None, "SMEM"):
+                    tag = f"{pipe}/{tb}/{fc or 'auto'}"
+                    try:
+                        p = ll.ll_plan_gather(L, axis, 4, pipe=pipe, thread_bytes=tb, force_class=fc)
+                    except Exception as e:   # noqa: BLE001
+                        res[tag] = str(e)[:60]
+                        continue
+                    it = [0]
+
+                    def f():
+                        a = sets[it[0] % nset]
+                        it[0] += 1
+                        ll.ll_gather(a[0], a[1], a[2], p)
+                    ms = time_fn(f, batch=20 if n <= (1 << 24) else 3)
+                    d = p.describe()
+                    res[tag] = {"tma": d["tma"], "x": d["exchange"], "warps": 1 << d["warp_bits"],
+                                "GBps": round(12 * n / ms / 1e6, 1)}
+        print(json.dumps({"family": fam, "shape": shape, "axis": axis - 1, "MiB": (4 * n) >> 20, "res": res}), flush=True)
+        del sets
 
 def broadcast_sweep(permute_batch=False):
     """Broadcast targets: random bijective A -> B with 5-8 zero columns,
