@@ -37,7 +37,50 @@ conv = {"c2": (W.c2(16), 2, {}), "c2smem": (W.c2(16), 2, {"force_class": "SMEM"}
         "c2fsmemvec": (W.c2(16), 2, {"sigma": "faithful", "force_class": "SMEM", "smem_instr": "vec"}),
         "c3f": (W.c3(14), 2, {"sigma": "faithful"}),
         "c3fvec": (W.c3(14), 2, {"sigma": "faithful", "smem_instr": "vec"})}
-if a.case.startswith("bcast"):
+if a.case.startswith("t4_"):
+    # t4_<reduce|scan|gather>_<blocked|mma|custom>_<a>_<b>_<axis>: a Table 4 family tile
+    # times 8 CTAs, default plan plus --opts (sanitizer runs of the default load paths)
+    import json as _json
+    import numpy as np
+    from workloads import gen
+    _, kind, fam, ta, tb, ax = a.case.split("_")
+    ta, tb, ax = int(ta), int(tb), int(ax)
+    if fam == "blocked":
+        T = ll.ll_layout_blocked([ta, tb], [1, 4], [8, 4], [4, 1], [1, 0])
+    elif fam == "mma":
+        T = ll.ll_layout_mma_acc(ta, tb, 4)
+    else:
+        T = ll.Layout.from_spec(gen.random_distributed(
+            np.random.default_rng(77), [("r", ta.bit_length() - 1), ("c", tb.bit_length() - 1)],
+            [("reg", max(1, ta.bit_length() + tb.bit_length() - 2 - 7)), ("lane", 5), ("warp", 2)],
+            zero_ok=["reg", "lane", "warp"] if kind != "gather" else []))
+    vecs, bases, k = T.bases(), {}, 0
+    for nm, nb in T.in_dims:
+        bases[nm] = [(0,) + tuple(v) for v in vecs[k:k + nb]]
+        k += nb
+    bases["block"] = [(1, 0, 0), (2, 0, 0), (4, 0, 0)]
+    L = ll.Layout(list(T.in_dims) + [("block", 3)], [("b", 3)] + list(T.out_dims), bases)
+    n = 1 << L.d_in
+    o = _json.loads(a.opts)
+    s = torch.rand(n, device="cuda")
+    if kind == "gather":
+        p = ll.ll_plan_gather(L, ax + 1, 4, **o)
+        K = (ta, tb)[ax]
+        i = torch.randint(0, K, (n,), dtype=torch.int32, device="cuda")
+        d = torch.empty_like(s)
+        run = lambda: ll.ll_gather(s, i, d, p)   # noqa: E731
+    elif kind == "scan":
+        p = ll.ll_plan_scan(L, ax + 1, **o)
+        d = torch.empty_like(s)
+        run = lambda: ll.ll_scan(s, d, p)   # noqa: E731
+    else:
+        p = ll.ll_plan_reduce(L, ax + 1, **o)
+        d = torch.empty(p.out_elems(), device="cuda")
+        run = lambda: ll.ll_reduce(s, d, p)   # noqa: E731
+    print(p.describe())
+    for _ in range(a.iters):
+        run()
+elif a.case.startswith("bcast"):
     # the bench's broadcast row: random bijective A -> B with 8 zero columns (seed 908)
     import numpy as np
     from workloads import gen
