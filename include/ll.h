@@ -126,7 +126,9 @@ typedef struct {
   int max_vec_bytes;    /* global-memory vector bound, default 16    */
   int sigma;            /* 0 = coalesced HBM access (default), 1 = faithful      */
   int tile_bytes;       /* target CTA tile bytes when folding/choosing tiles (0 = default);
-                         * linear tiles also take it as their size cap (default 64 KiB) */
+                         * linear tiles also take it as their size cap (default 64 KiB);
+                         * gather / reduce / scan: split the layout's CTA tile down to
+                         * it (warp bits of independent rows become grid bits; 0 = keep) */
   int thread_bytes;     /* target bytes per thread (0 = default)                 */
   int generic;          /* 1 = force the runtime-generic kernel                   */
   ll_comm* comm;        /* required for DEVICE plans                              */

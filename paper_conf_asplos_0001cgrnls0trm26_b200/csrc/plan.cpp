@@ -1487,6 +1487,30 @@ static void widen_warps(std::vector<int>& hw_bit, int& R, int& Wb, int v, int th
   }
 }
 
+// The reverse step for the grid: while the CTA tile (register, lane and warp bits of the
+// kernel layout, 2^(R+5+Wb) elements of w bytes) exceeds `tile_bytes`, its top warp bit
+// that carries a non-zero, non-axis column (independent rows: no step of the gather,
+// reduction or scan crosses it) becomes a CTA-grid bit.  The CTA tile shrinks, the CTA
+// count grows, registers per thread stay.  Returns the moved layout bits in ascending
+// packed position: the caller puts them below the layout's block bits, so consecutive
+// CTAs cover neighbouring pieces of one layout tile.  0 = keep the layout's CTA tile.
+static std::vector<int> split_tile(std::vector<int>& hw_bit, int R, int& Wb, int w, int tile_bytes,
+                                   const std::function<bool(int)>& movable) {
+  std::vector<int> moved;
+  if (tile_bytes <= 0) return moved;
+  const int target = std::max(R + 5, ilog2(u64(std::max(1, tile_bytes / w))));
+  while (R + 5 + Wb > target && Wb > 0) {
+    int q = -1;
+    for (int b = int(hw_bit.size()) - 1; b >= R + 5; --b) if (movable(hw_bit[b])) { q = b; break; }
+    if (q < 0) break;
+    moved.push_back(hw_bit[q]);
+    hw_bit.erase(hw_bit.begin() + q);
+    --Wb;
+  }
+  std::sort(moved.begin(), moved.end());
+  return moved;
+}
+
 std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const ll_plan_opts* opts) {
   if (w != 1 && w != 2 && w != 4 && w != 8) fail(LL_ERR_INVALID_ARG, "elem_bytes must be 1, 2, 4 or 8");
   if (axis < 0 || axis >= int(L.out.size())) fail(LL_ERR_INVALID_ARG, "axis out of range");
@@ -1546,7 +1570,11 @@ std::unique_ptr<GatherPlan> plan_gather(const Layout& L, int axis, int w, const 
                 [&](int k) { return L.cols[k] != 0 && (L.cols[k] & amask) == 0; });
     R = G->R;
   }
-  G->grid_bit = blk;
+  // optional smaller CTA tiles (ll_plan_opts.tile_bytes): independent rows to the grid
+  const auto gmoved = split_tile(G->hw_bit, G->R, G->Wb, w, opts ? opts->tile_bytes : 0,
+                                 [&](int k) { return L.cols[k] != 0 && (L.cols[k] & amask) == 0; });
+  G->grid_bit = gmoved;
+  G->grid_bit.insert(G->grid_bit.end(), blk.begin(), blk.end());
   G->lcol.resize(G->hw_bit.size());
   for (size_t b = 0; b < G->hw_bit.size(); ++b) G->lcol[b] = L.cols[G->hw_bit[b]];
   G->axis_reg_pos.assign(G->K_bits, -1);
@@ -1686,6 +1714,9 @@ std::unique_ptr<ReducePlan> plan_reduce(const Layout& L, int axis, const ll_plan
   widen_warps(Rp->hw_bit, Rp->R, Rp->Wb, Rp->v, default_int(opts, &ll_plan_opts::thread_bytes, tma_auto ? 256 : 128),
               [&](int k) { return L.cols[k] != 0 && (L.cols[k] & amask) == 0; });
   R = Rp->R;
+  // optional smaller CTA tiles (ll_plan_opts.tile_bytes): independent rows to the grid
+  const auto rmoved = split_tile(Rp->hw_bit, R, Rp->Wb, 4, opts ? opts->tile_bytes : 0,
+                                 [&](int k) { return L.cols[k] != 0 && (L.cols[k] & amask) == 0; });
   const int n = int(Rp->hw_bit.size());
   // classify kernel bits (reduced per level, duplicate) and map each logical axis bit t
   // to the kernel bit that holds it: the steps run in t order
@@ -1714,6 +1745,10 @@ std::unique_ptr<ReducePlan> plan_reduce(const Layout& L, int axis, const ll_plan
                (b >= R && b < R + 5 && std::count(Rp->red_lane.begin(), Rp->red_lane.end(), b - R)) ||
                (b >= R + 5 && std::count(Rp->red_warp.begin(), Rp->red_warp.end(), b - R - 5));
     if (c && !red) Rp->out_col[b] = out_of(c);
+  }
+  for (int k : rmoved) {
+    Rp->grid_bit.push_back(k);
+    Rp->grid_out.push_back(out_of(L.cols[k]));
   }
   for (int k : bits_at_level(L, 3, 3)) {
     if (L.cols[k] == 0) continue;   // duplicate CTAs are not launched
@@ -1801,6 +1836,9 @@ std::unique_ptr<ScanPlan> plan_scan(const Layout& L, int axis, const ll_plan_opt
   widen_warps(S->hw_bit, S->R, S->Wb, S->v, default_int(opts, &ll_plan_opts::thread_bytes, 128),
               [&](int k) { return L.cols[k] != 0 && (L.cols[k] & amask) == 0; });
   R = S->R;
+  // optional smaller CTA tiles (ll_plan_opts.tile_bytes): independent rows to the grid
+  const auto smoved = split_tile(S->hw_bit, R, S->Wb, 4, opts ? opts->tile_bytes : 0,
+                                 [&](int k) { return L.cols[k] != 0 && (L.cols[k] & amask) == 0; });
   const int n = int(S->hw_bit.size());
   for (int t = 0; t < K; ++t) {
     int b = -1;
@@ -1808,7 +1846,8 @@ std::unique_ptr<ScanPlan> plan_scan(const Layout& L, int axis, const ll_plan_opt
     if (b < 0) fail(LL_ERR_UNSUPPORTED, "scan: in-tile axis bits must be the low axis bits");
     S->axis_hw.push_back(b);
   }
-  S->grid_bit = bits_at_level(L, 3, 3);
+  S->grid_bit = smoved;
+  for (int k : bits_at_level(L, 3, 3)) S->grid_bit.push_back(k);
   // shuffles per thread per tile: a step needs them when its bit or a lower axis bit is
   // a lane; one per distinct partner register (slots whose partners coincide share it:
   // the partner has every lower register axis bit set)

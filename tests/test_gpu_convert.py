@@ -982,3 +982,54 @@ def test_gather_more_warps_bitexact(family, thread_bytes):
     d_dst = empty_device(n, 4)
     ll.ll_gather(to_device(src), to_device(idx.view(np.uint32)), d_dst, plan)
     assert np.array_equal(from_device(d_dst, 4), O.gather(OL, 1, src, idx))
+
+
+@pytest.mark.parametrize("family", ["mma", "blocked", "sliced_mma", "custom"])
+@pytest.mark.parametrize("tile_bytes", [16384, 4096])
+def test_split_tiles_bitexact(family, tile_bytes):
+    """Smaller CTA tiles (ll_plan_opts.tile_bytes): warp bits carrying independent rows
+    become grid bits.  Reduce, scan (both axes, [128,128] Table 4 tiles x 4 CTAs) and
+    gather (config-4 tiles) stay bit-exact against the oracle: the reduction / scan /
+    gather never crosses those bits."""
+    import torch
+    from tests._util import from_device, to_device, empty_device
+    rng = np.random.default_rng(1012)
+    OT, _ = _table4_layout(family, (128, 128), rng)
+    # 4 CTAs along a new leading dim (block bits)
+    out3 = [("b", 2)] + list(OT.out_dims)
+    bases = {n: [(0,) + tuple(v) for v in OT.bases[n]] for n, _ in OT.in_dims}
+    bases["block"] = [(1, 0, 0), (2, 0, 0)]
+    OL = O.Layout(list(OT.in_dims) + [("block", 2)], out3, bases)
+    L = ll.Layout(OL.in_dims, OL.out_dims, OL.bases)
+    T = rng.random(1 << OL.d_out, dtype=np.float32)
+    src = O.pack(OL, T)
+    d_src = torch.from_numpy(src).cuda()
+    split = 0
+    for axis in (1, 2):
+        p0 = ll.ll_plan_reduce(L, axis)
+        p = ll.ll_plan_reduce(L, axis, tile_bytes=tile_bytes)
+        split += p.describe()["ctas"] > p0.describe()["ctas"]
+        out = torch.empty(p.out_elems(), dtype=torch.float32, device="cuda")
+        ll.ll_reduce(d_src, out, p)
+        rep = O.reduce_fixed_order_fp32(OL, axis, src)
+        assert np.array_equal(out.cpu().numpy().view(np.uint32), rep.view(np.uint32)), (family, axis)
+        try:
+            s = ll.ll_plan_scan(L, axis, tile_bytes=tile_bytes)
+        except ll.LLError as e:
+            assert "too large" in str(e)
+            continue
+        out2 = torch.empty(src.size, dtype=torch.float32, device="cuda")
+        ll.ll_scan(d_src, out2, s)
+        rep2 = O.scan_bitdoubling_fp32(OL, axis, src)
+        assert np.array_equal(out2.cpu().numpy().view(np.uint32), rep2.view(np.uint32)), (family, axis)
+    assert split >= 1
+    if family in ("mma", "blocked"):
+        G, OG = both(W.c4("gather", family, n_i=9, n_j=7))
+        n = 1 << OG.d_in
+        gs = O.pack(OG, gen.random_bits(rng, n, 4))
+        gi = O.pack(OG, rng.integers(-50, 50, size=n).astype(np.int32))
+        for fc in (None, "SMEM"):
+            g = ll.ll_plan_gather(G, 1, 4, tile_bytes=tile_bytes, force_class=fc)
+            d_dst = empty_device(n, 4)
+            ll.ll_gather(to_device(gs), to_device(gi.view(np.uint32)), d_dst, g)
+            assert np.array_equal(from_device(d_dst, 4), O.gather(OG, 1, gs, gi)), (family, fc)

@@ -167,6 +167,48 @@ def main():
         return reduce_scan_families()
     if "gathfam" in only:
         return gather_families()
+    if "split" in only:
+        # smaller CTA tiles (tile_bytes: independent rows to the grid) for the config-4
+        # gather / reduce / scan at the config size (4 rotating sets) and at 1 GiB
+        for fam in ("mma", "blocked"):
+            for ni, nj in ((12, 12), (15, 13)):
+                nset = 4 if ni == 12 else 1
+                for kind in ("gather", "reduce", "scan"):
+                    L = ll.Layout.from_spec(W.c4("gather" if kind == "gather" else "reduce", fam, n_i=ni, n_j=nj))
+                    n = 1 << L.d_in
+                    if kind == "gather":
+                        sets = [(torch.randint(0, 1 << 30, (n,), dtype=torch.int32, device="cuda"),
+                                 torch.randint(0, 32, (n,), dtype=torch.int32, device="cuda"),
+                                 torch.empty(n, dtype=torch.int32, device="cuda")) for _ in range(nset)]
+                    else:
+                        sets = [torch.rand(n, device="cuda") for _ in range(nset)]
+                    for tb in (0, 32768, 16384, 8192, 4096, 2048):
+                        if kind == "gather":
+                            p = ll.ll_plan_gather(L, 1, 4, tile_bytes=tb)
+                            outs = None
+                            nbytes = 12 * n
+                        else:
+                            p = (ll.ll_plan_scan if kind == "scan" else ll.ll_plan_reduce)(L, 1, tile_bytes=tb)
+                            m = n if kind == "scan" else p.out_elems()
+                            outs = [torch.empty(m, device="cuda") for _ in sets]
+                            nbytes = 4 * (n + m)
+                        it = [0]
+
+                        def f():
+                            k = it[0] % nset
+                            it[0] += 1
+                            if kind == "gather":
+                                ll.ll_gather(sets[k][0], sets[k][1], sets[k][2], p)
+                            else:
+                                (ll.ll_scan if kind == "scan" else ll.ll_reduce)(sets[k], outs[k], p)
+                        ms = time_fn(f, batch=20 if ni == 12 else 3)
+                        d = p.describe()
+                        print(json.dumps({"case": f"{kind} {fam} [{1 << ni},{1 << nj}]", "tile_bytes": tb,
+                                          "ctas": d["ctas"], "warps": 1 << d["warp_bits"], "ms": round(ms, 4),
+                                          "GBps": round(nbytes / ms / 1e6, 1)}), flush=True)
+                        del outs
+                    del sets
+        return
     if "warps" in only:
         # reduce / scan with non-axis register bits moved to warps (thread_bytes)
         for fam in ("mma", "blocked"):
