@@ -33,6 +33,7 @@ sys.path.insert(0, ROOT)
 
 PEAKS_PATH = os.path.join(ROOT, "MEASURED_PEAKS.json")
 FALLBACK_HBM = 6650.0   # B200_PROFILING.md fallback (GB/s) if MEASURED_PEAKS.json is absent
+C5_TIMEOUT_S = 300.0   # bound on the cross-GPU config-5 leg (N > 1), see main()
 METRIC = "layout-conversion GB/s per GPU and % of HBM peak; smem bank conflicts/request"
 WORKLOAD = ("config 2: [65536,128,128] bf16, wgmma m64n128 accumulator (x2 m-reps) -> "
             "blocked [8,8]/[2,16]/[4,1], warp-shuffle conversion, 65536 tiles")
@@ -660,10 +661,6 @@ def main():
     link_ms = l0.elapsed_time(l1) / args.e2e_steps
     del d_tmp
     del dev_buf
-    c5 = None
-    if world > 1 and (world & (world - 1)) == 0 and not args.no_config5:
-        c5 = config5_exchange(ll, W, torch, world, rank)
-
     if rank == 0:
         peak, peak_kind = hbm_peak()
         avg_launch_ms = statistics.mean(launch_ms)
@@ -700,8 +697,6 @@ def main():
             "smem_bank_conflicts": smem_conflicts(),
             "clocks": clk.summary(),
         }
-        if c5 is not None:
-            line["config5_nvlink"] = c5
         if world == 1 and not args.no_configs:
             # the library baseline must produce the same bytes as our kernel
             tb, y = torch_permute_baseline(torch, A_spec, B_spec, src, w)
@@ -713,6 +708,23 @@ def main():
             line["configs"] = other_configs(ll, W, torch, peak)
         if world == 1 and not args.no_cpu_baseline:   # the oracle baseline: rank 0 at N=1 only
             line["cpu_baseline"] = cpu_baseline_oracle()
+    if world > 1 and (world & (world - 1)) == 0 and not args.no_config5:
+        # config 5 across the GPUs (NCCL + peer windows).  A watchdog on every rank bounds
+        # it: should any rank stall in the exchange, rank 0 still prints the main line
+        # (config5_nvlink = the timeout) and every rank exits instead of hanging the job.
+        def _stalled():
+            if rank == 0:
+                line["config5_nvlink"] = {"error": f"timeout after {C5_TIMEOUT_S} s (exchange stalled)"}
+                print(json.dumps(line), flush=True)
+            os._exit(1 if bad else 0)
+        dog = threading.Timer(C5_TIMEOUT_S, _stalled)
+        dog.daemon = True
+        dog.start()
+        c5 = config5_exchange(ll, W, torch, world, rank)
+        dog.cancel()
+        if rank == 0:
+            line["config5_nvlink"] = c5
+    if rank == 0:
         print(json.dumps(line), flush=True)
     if world > 1:
         torch.distributed.destroy_process_group()
