@@ -80,6 +80,8 @@ def main():
         return autotune_sweep()
     if "big" in only:
         return big_configs()
+    if "ceiling" in only:
+        return ceiling_cases()
     if "small" in only:
         return small_kernels()
     if "matrix" in only:
@@ -737,6 +739,18 @@ def big_configs():
                               ("c5T", W.c5T(0), 2), ("n1", W.n1_preshuffle(14, 14), 2),
                               ("n2", W.n2_tmem_epilogue(13), 4)]:
         conv_case(name, sa, sb, w)
+
+
+def ceiling_cases():
+    """The 1-2 GiB conversions of the bench's configs list, for A/B against the plain
+    streaming ceiling (tools/smem_counter_control.cu, one tile per CTA); extra plan
+    options from $LL_SWEEP_OPTS (JSON), env hooks from the caller."""
+    extra = json.loads(os.environ.get("LL_SWEEP_OPTS", "{}"))
+    for name, (sa, sb), w in [("c2", W.c2(16), 2), ("c3", W.c3(14), 2), ("c3b", W.c3b(14), 2),
+                              ("c1b", W.c1_batched(20), 4), ("c5T", W.c5T(0), 2),
+                              ("n1", W.n1_preshuffle(15, 15), 2), ("n2_16x256b", W.n2_tmem("16x256b", 14), 4),
+                              ("n2_fp8", W.n2_acc_to_lhs(8, 18), 1), ("noop_bf16", W.n2_acc_to_lhs(16, 17), 2)]:
+        conv_case(name, sa, sb, w, **extra)
 
 
 def small_kernels():
