@@ -612,6 +612,15 @@ def main():
     ms_per_step = total_ms / args.steps
     value = world * bytes_per_step * args.steps / (total_ms / 1e3) / 1e9
 
+    # ---- context for the roofline: the library's own NOOP plan (A -> A) on the same
+    # 2+2 GiB runs ll_copy_kernel, a plain streaming copy in the tile kernels' shape —
+    # the practical read+write ceiling of a kernel on this GPU (the measured peak in
+    # MEASURED_PEAKS.json is a driver copy)
+    pc = ll.ll_plan_convert(A, A, 2)
+    ceil_ms = _time_stream(lambda: ll.ll_convert(src, dst, pc, stream), torch, samples=5)
+    ceil_gbs = bytes_per_step / (ceil_ms / 1e3) / 1e9
+    del pc
+
     # ---- end to end through the C-ABI call with HOST buffers (ll_convert_host): per
     # step the pinned host input is copied in, converted and copied back, chunked over
     # two streams so that H2D, kernels and D2H of different chunks overlap
@@ -685,7 +694,10 @@ def main():
                          "frac_of_nominal_8TBps": round(achieved / 8000.0, 4),
                          "traffic": traffic, "kernel": "ll_tile_kernel (shuffle)",
                          "traffic_over_algorithmic": round(traffic / bytes_per_step, 4) if traffic else None,
-                         "bytes_per_launch": bytes_per_step, "avg_launch_ms": round(avg_launch_ms, 5)},
+                         "bytes_per_launch": bytes_per_step, "avg_launch_ms": round(avg_launch_ms, 5),
+                         "streaming_ceiling": {"GBps": round(ceil_gbs, 1), "frac": round(achieved / ceil_gbs, 4),
+                                               "kernel": "ll_copy_kernel (NOOP plan A -> A, same 2+2 GiB, "
+                                                         "streams of 20 launches)"}},
             "e2e": {"value": round(world * bytes_per_step / (e2e_ms / 1e3) / 1e9, 2), "unit": "GB/s",
                     "h2d_bytes_per_step": n * w, "d2h_bytes_per_step": n * w, "ms_per_step": round(e2e_ms, 3),
                     "api": "ll_convert_host (chunked H2D -> kernel -> D2H over 2 streams)",

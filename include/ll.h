@@ -279,7 +279,8 @@ ll_status ll_layout_slice(const ll_layout* L, int dim, ll_layout** out);
  * ll_plan_convert (rows a2-a4, a6-a9).  Host only.
  *   A, B: same output dims; A surjective.  elem_bytes in {1, 2, 4, 8}.
  *   opts: NULL for defaults.  Computes Q = A^+ ∘ B, the paper's class (lowest
- *   hardware level Q must cross), and an execution plan: NOOP (memcpy), a
+ *   hardware level Q must cross), and an execution plan: NOOP (a streaming copy
+ *   kernel; nothing when src == dst), a
  *   specialised sm_100a tile kernel (register permutation / warp shuffles /
  *   swizzled smem round trip / cross-CTA tiled exchange), the runtime-generic
  *   kernel (broadcast and non-permutation maps), or DEVICE (pack, all-to-all over
@@ -312,8 +313,9 @@ void ll_plan_destroy(ll_plan* plan);
 
 /* ll_convert (rows a5-a10): dst[h] = src[Q(h)] on `stream` (a cudaStream_t).
  *   src: device buffer packed in A (2^{A.d_in} elements, local slice for dev);
- *   dst: device buffer packed in B; must not alias src unless the plan is NOOP
- *   (LL_ERR_ALIAS); 16-byte aligned (LL_ERR_MISALIGNED).
+ *   dst: device buffer packed in B; must not overlap src (LL_ERR_ALIAS), except
+ *   that a NOOP plan accepts dst == src (in place: nothing runs); 16-byte aligned
+ *   (LL_ERR_MISALIGNED).
  *   workspace: NULL unless ll_plan_workspace_bytes > 0.
  *   DEVICE plans are collective: every rank calls with the same plan. */
 ll_status ll_convert(const void* src, void* dst, void* workspace, const ll_plan* plan,

@@ -18,6 +18,8 @@ const std::string& last_error_ref();
 std::string jit_precompile(const std::string& plan_src, const char* name);
 int launch_generic(const void* src, void* dst, const unsigned long long* cols, int nbits, unsigned long long nelem,
                    int w, cudaStream_t stream, int sms);
+void* copy_kernel_fn();
+unsigned copy_kernel_grid(unsigned long long nbytes);
 ll_status device_convert(const ConvPlan& P, const void* src, void* dst, void* ws, cudaStream_t st);
 void plan_device(ConvPlan& P, const ll_plan_opts* opts);
 }  // namespace ll
@@ -192,12 +194,16 @@ ll_status convert_impl(const void* src, void* dst, void* ws, ConvPlan& P, cudaSt
   const size_t sbytes = P.src_elems * P.w, dbytes = P.dst_elems * P.w;
   if ((reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst)) & 15)
     fail(LL_ERR_MISALIGNED, "src and dst must be 16-byte aligned");
-  if (P.exec == EXEC_NOOP) {
-    if (src != dst) check_cuda(cudaMemcpyAsync(dst, src, dbytes, cudaMemcpyDeviceToDevice, st), "cudaMemcpyAsync");
-    return LL_OK;
-  }
   const char* s8 = static_cast<const char*>(src);
   const char* d8 = static_cast<const char*>(dst);
+  if (P.exec == EXEC_NOOP) {
+    if (src == dst) return LL_OK;   // in place: nothing moves
+    if (s8 < d8 + dbytes && d8 < s8 + sbytes) fail(LL_ERR_ALIAS, "NOOP: src and dst must be equal or disjoint");
+    unsigned long long nb = dbytes;
+    void* args[] = {const_cast<void**>(&src), &dst, &nb};
+    launch_kernel(copy_kernel_fn(), copy_kernel_grid(nb), 256, args, 0, st, "cudaLaunchKernelEx(ll_copy_kernel)");
+    return LL_OK;
+  }
   if (s8 < d8 + dbytes && d8 < s8 + sbytes) fail(LL_ERR_ALIAS, "src and dst overlap (only NOOP plans may alias)");
   if (P.exec == EXEC_TILE) {
     ensure_tile_kernel(P);

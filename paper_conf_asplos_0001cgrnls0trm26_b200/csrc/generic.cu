@@ -31,6 +31,46 @@ __global__ void __launch_bounds__(256) ll_generic_convert_kernel(const uint8_t* 
   }
 }
 
+// NOOP plans (A = B, "equivalent layouts") with dst != src: the conversion is
+// the identity on packed buffers, executed as a streaming copy in the tile kernels'
+// shape — one 32 KiB tile per CTA (256 threads x 8 16-byte vectors, 512 contiguous
+// bytes per warp instruction), all loads in flight before the stores, streaming cache
+// hints, PDL like every other kernel.  Measured faster than cudaMemcpyAsync D2D on B200
+// (profiles/r02_sweep_ceiling.jsonl).  A tail below 16 bytes (buffers < 16 bytes) is
+// copied bytewise by CTA 0.
+__global__ void __launch_bounds__(256) ll_copy_kernel(const uint4* __restrict__ src, uint4* __restrict__ dst,
+                                                      unsigned long long nbytes) {
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+  constexpr int V = 8;
+  const unsigned long long nvec = nbytes >> 4;
+  const unsigned long long base = (unsigned long long)blockIdx.x * (256ull * V) + threadIdx.x;
+  uint4 r[V];
+#pragma unroll
+  for (int k = 0; k < V; ++k) {
+    const unsigned long long i = base + 256ull * k;
+    if (i < nvec)
+      asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+                   : "=r"(r[k].x), "=r"(r[k].y), "=r"(r[k].z), "=r"(r[k].w) : "l"(src + i));
+  }
+#pragma unroll
+  for (int k = 0; k < V; ++k) {
+    const unsigned long long i = base + 256ull * k;
+    if (i < nvec)
+      asm volatile("st.global.cs.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(dst + i), "r"(r[k].x), "r"(r[k].y), "r"(r[k].z),
+                   "r"(r[k].w) : "memory");
+  }
+  const unsigned tail = unsigned(nbytes & 15);
+  if (tail && blockIdx.x == 0 && threadIdx.x < tail)
+    reinterpret_cast<uint8_t*>(dst)[(nvec << 4) + threadIdx.x] = reinterpret_cast<const uint8_t*>(src)[(nvec << 4) + threadIdx.x];
+}
+
+void* copy_kernel_fn() { return reinterpret_cast<void*>(&ll_copy_kernel); }
+unsigned copy_kernel_grid(unsigned long long nbytes) {
+  const unsigned long long tiles = ((nbytes >> 4) + 2047) / 2048;
+  return unsigned(tiles ? tiles : 1);
+}
+
 int launch_generic(const void* src, void* dst, const unsigned long long* cols, int nbits, unsigned long long nelem,
                    int w, cudaStream_t stream, int sms) {
   QCols q;

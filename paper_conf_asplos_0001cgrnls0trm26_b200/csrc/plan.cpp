@@ -754,6 +754,11 @@ static void build_tile(ConvPlan& P, const std::vector<int>& S0, const std::vecto
     // 4 -> 8 warps, profiles/r01_sweep_next_rows.jsonl)
     int dflt = 256;
     if (!in_cta) dflt = int(std::max<u64>(u64(P.w), std::min<u64>(256, ((u64(1) << Ss.size()) * u64(P.w)) / 256)));
+    // layouts whose own CTA tile is small (grid bits folded in up to tile_bytes): 8
+    // warps of 64 bytes per thread rather than 2 warps of 256 — measured +4-11% on the
+    // folded 16 KiB tiles (c1 batch, the fp8 operand, 2-byte Fig.-1 tiles), to within
+    // 1% of the plain streaming kernel (profiles/r02_sweep_small_cta.jsonl)
+    else if (!foldS.empty()) dflt = std::max(P.w, 64);
     int thread_bytes = default_int(opts, &ll_plan_opts::thread_bytes, dflt);
     assign_sigma_coalesced(T, A, B, Ss, Ds, prefer, maxvec, thread_bytes);
   }

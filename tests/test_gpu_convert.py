@@ -125,6 +125,24 @@ def test_noop_memcpy():
     assert np.array_equal(from_device(d_dst, 4), src)
 
 
+@pytest.mark.parametrize("d", [0, 1, 3, 4, 9, 12, 21])
+@pytest.mark.parametrize("w", [1, 2, 4, 8])
+def test_noop_copy_kernel_sizes(d, w):
+    """NOOP plans with dst != src run ll_copy_kernel (32 KiB per CTA): buffers from one
+    element (a bytewise tail below 16 bytes) through partial and many CTA tiles equal
+    the input; src == dst is accepted and leaves the buffer unchanged."""
+    out = [("x", d)]
+    A = ll.Layout([("offset", d)], out, {"offset": [(1 << k,) for k in range(d)]})
+    plan = ll.ll_plan_convert(A, A, w)
+    assert plan.cls == "NOOP"
+    src = gen.random_bits(np.random.default_rng(d * 8 + w), 1 << d, w)
+    d_src, d_dst = to_device(src), empty_device(1 << d, w)
+    ll.ll_convert(d_src, d_dst, plan)
+    assert np.array_equal(from_device(d_dst, w), src)
+    ll.ll_convert(d_dst, d_dst, plan)
+    assert np.array_equal(from_device(d_dst, w), src)
+
+
 def _full_size_every_element(sa, sb, w, nsample_seed):
     _full_size_every_element_opts(sa, sb, w, nsample_seed)
 

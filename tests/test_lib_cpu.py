@@ -1076,3 +1076,15 @@ def test_convert_pointer_checks_before_launch():
         ll.ll_convert(base + 4, base + 4096, p, stream=0)
     with pytest.raises(ll.LLError, match="ALIAS"):
         ll.ll_convert(base, base + 512, p, stream=0)      # 1 KiB buffers overlapping by half
+
+
+def test_noop_partial_overlap_refused():
+    """NOOP plans (A = B) run in place when src == dst and as a streaming copy kernel
+    otherwise; partially overlapping buffers are refused (LL_ERR_ALIAS) before any
+    launch — raw addresses, nothing is dereferenced."""
+    A = ll.Layout.from_spec(W.C1_A)
+    p = ll.ll_plan_convert(A, A, 4)
+    assert p.cls == "NOOP"
+    base = 1 << 32
+    with pytest.raises(ll.LLError, match="ALIAS"):
+        ll.ll_convert(base, base + 512, p, stream=0)      # 1 KiB buffers overlapping by half

@@ -42,14 +42,14 @@ def time_fn(fn, iters=20, warmup=5, batch=None):
     return ts[len(ts) // 2]
 
 
-def conv_case(name, sa, sb, w, **opts):
+def conv_case(name, sa, sb, w, batch=None, **opts):
     A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
     p = ll.ll_plan_convert(A, B, w, **opts)
     n = 1 << A.d_in
     src = torch.randint(-2 ** 15, 2 ** 15, (n * w // 2,), dtype=torch.int16, device="cuda")
     dst = torch.empty_like(src)
     p.prepare()
-    ms = time_fn(lambda: ll.ll_convert(src, dst, p))
+    ms = time_fn(lambda: ll.ll_convert(src, dst, p), batch=batch)
     gbs = 2 * n * w / ms / 1e6
     d = p.describe()
     t = d.get("tile", {})
@@ -82,6 +82,8 @@ def main():
         return big_configs()
     if "ceiling" in only:
         return ceiling_cases()
+    if "smallcta" in only:
+        return small_cta_tiles()
     if "small" in only:
         return small_kernels()
     if "matrix" in only:
@@ -750,7 +752,17 @@ def ceiling_cases():
                               ("c1b", W.c1_batched(20), 4), ("c5T", W.c5T(0), 2),
                               ("n1", W.n1_preshuffle(15, 15), 2), ("n2_16x256b", W.n2_tmem("16x256b", 14), 4),
                               ("n2_fp8", W.n2_acc_to_lhs(8, 18), 1), ("noop_bf16", W.n2_acc_to_lhs(16, 17), 2)]:
-        conv_case(name, sa, sb, w, **extra)
+        conv_case(name, sa, sb, w, batch=20, **extra)
+
+
+def small_cta_tiles():
+    """Layouts whose own CTA tile is below 16 KiB (grid bits folded up to tile_bytes):
+    tile_bytes x thread_bytes, timed as streams of 20 launches like the bench."""
+    for name, (sa, sb), w in [("c1b", W.c1_batched(20), 4), ("n2_fp8", W.n2_acc_to_lhs(8, 18), 1),
+                              ("n2_bf16_to_fp8_like_c1", W.c1_batched(21), 2)]:
+        for tile in (16384, 32768, 65536):
+            for tb in (64, 128, 256):
+                conv_case(name, sa, sb, w, batch=20, tile_bytes=tile, thread_bytes=tb)
 
 
 def small_kernels():
