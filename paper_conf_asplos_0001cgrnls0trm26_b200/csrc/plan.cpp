@@ -1149,8 +1149,9 @@ std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, 
           int tb = default_int(opts, &ll_plan_opts::tile_bytes, 16384);
           int target = std::max(v + 5, ilog2(u64(std::max(1, tb / w))));
           // the longest contiguous runs (2^c elements on both sides) whose tile fits in
-          // 64 KiB of smem: 512-byte runs, else 256, else 128 (one line)
-          const int max_bits = ilog2(u64(65536 / w));
+          // 64 KiB of smem (or ll_plan_opts.tile_bytes when larger): 512-byte runs, else
+          // 256, else 128 (one line)
+          const int max_bits = ilog2(u64(std::max(65536, tb) / w));
           for (int c_bits = v + 5; c_bits >= v + 3; --c_bits) {
             choose_cta_tile(pi, nB, c_bits, target, S, D, gS, gD, grid_only_src);
             if (int(S.size()) <= max_bits) break;

@@ -82,6 +82,8 @@ def main():
         return big_configs()
     if "ceiling" in only:
         return ceiling_cases()
+    if "ctarun" in only:
+        return cta_run_lengths()
     if "smallcta" in only:
         return small_cta_tiles()
     if "small" in only:
@@ -753,6 +755,16 @@ def ceiling_cases():
                               ("n1", W.n1_preshuffle(15, 15), 2), ("n2_16x256b", W.n2_tmem("16x256b", 14), 4),
                               ("n2_fp8", W.n2_acc_to_lhs(8, 18), 1), ("noop_bf16", W.n2_acc_to_lhs(16, 17), 2)]:
         conv_case(name, sa, sb, w, batch=20, **extra)
+
+
+def cta_run_lengths():
+    """CTA-class transposes (config 5-T, N1): 256-byte runs in 32 / 64 KiB tiles (the
+    64 KiB smem cap) vs 512-byte runs in 128 KiB tiles (tile_bytes = 131072, one CTA
+    per SM), unpipelined and pipelined; streams of 20 launches."""
+    for name, (sa, sb), w in [("c5T", W.c5T(0), 2), ("n1", W.n1_preshuffle(15, 15), 2)]:
+        for o in [{}, {"tile_bytes": 65536}, {"tile_bytes": 131072}, {"tile_bytes": 131072, "pipe": "on"},
+                  {"tile_bytes": 65536, "pipe": "on"}]:
+            conv_case(name, sa, sb, w, batch=20, **o)
 
 
 def small_cta_tiles():
