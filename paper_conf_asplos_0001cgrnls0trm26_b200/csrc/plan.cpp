@@ -862,13 +862,22 @@ static void plan_exchange(ConvPlan& P, const ll_plan_opts* opts) {
   // registers (XOR addresses that cannot fold into immediates), i.e. one CTA per SM;
   // asking for 2 trades registers for a few spills: with NOHOIST 1.07-2.2x over one
   // uncapped CTA on five of six random R2 maps (profiles/r01_sweep_linear_nohoist.jsonl);
-  // ll_plan_autotune times both.
+  // ll_plan_autotune times both.  Shuffle / smem exchanges with 256 bytes per thread
+  // (<= 8 warps): without a minimum-blocks hint ptxas compiles config 3's kernel to 62
+  // registers, fewer than the 64 that hold all 16 loads of a thread, so it splits the
+  // loads; with __launch_bounds__(threads, 2) it takes 104-110 registers and keeps every
+  // load in flight (at most 2 CTAs per SM at 8 warps).  Measured: c3 +1.7%, c3b +4.8%,
+  // c2 +0.5%, tcgen05 32x32b / 16x256b +1.4% / +1.7%, 16x64b / 16x128b unchanged
+  // (profiles/r02_sweep_smem_occupancy.jsonl, r02_sweep_shuffle_occupancy.jsonl).
   {
     const char* e = std::getenv("LL_MIN_BLOCKS");
     const int om = opts ? opts->min_blocks : 0;
     if (e) T.min_blocks = std::max(0, std::atoi(e));
     else if (om > 0) T.min_blocks = om;
     else if (om == 0 && T.ld_run >= 0 && T.xchg == X_SMEM && !T.staged) T.min_blocks = 2;
+    else if (om == 0 && (T.xchg == X_SMEM || T.xchg == X_SHUFFLE) && !T.staged && !T.bulk && !T.pipe &&
+             T.Wb <= 3 && (u64(T.w) << T.R) >= 256)
+      T.min_blocks = 2;
     else T.min_blocks = 0;
   }
   if (T.xchg == X_SMEM && (T.smem_elems * u64(T.w)) > 200 * 1024)

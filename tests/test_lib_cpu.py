@@ -844,13 +844,14 @@ def test_linear_tile_run_choice_simulated(monkeypatch, balance):
 def test_linear_tiles_default_exchange(monkeypatch):
     """Without LL_PIPE / LL_MIN_BLOCKS, linear-tile plans (random R2 memory layouts) take
     the unpipelined smem exchange with two CTAs per SM (register cap) and opaque thread
-    bases (NOHOIST); config 3 keeps the plain kernel."""
+    bases (NOHOIST); config 3 keeps the plain kernel with 2 CTAs per SM (8 warps x 256 B
+    per thread: the register cap that keeps all 16 loads of a thread in flight)."""
     monkeypatch.delenv("LL_MIN_BLOCKS", raising=False)
     monkeypatch.delenv("LL_NOHOIST", raising=False)
     monkeypatch.delenv("LL_PIPE", raising=False)
     A, B = (ll.Layout.from_spec(x) for x in W.c3(9))
     p = ll.ll_plan_convert(A, B, 2)
-    assert p.describe()["tile"]["pipe"] is False and p.describe()["tile"]["min_blocks"] == 0
+    assert p.describe()["tile"]["pipe"] is False and p.describe()["tile"]["min_blocks"] == 2
     assert "NOHOIST = false" in p.source()
     rng = np.random.default_rng(801)
     seen = 0
@@ -869,7 +870,8 @@ def test_linear_tiles_default_exchange(monkeypatch):
 def test_plan_opts_pipe_and_min_blocks():
     """ll_plan_opts.pipe / min_blocks reach the plan (describe) and the generated kernel
     (__launch_bounds__ minimum): auto = linear tiles unpipelined with two CTAs per SM;
-    explicit values override; other smem plans keep the plain kernel."""
+    explicit values override; in-CTA smem plans of 8 warps x 256 B per thread ask for
+    two CTAs per SM; other smem plans keep the plain kernel."""
     rng = np.random.default_rng(9)
     d = 16
     ca, cb = gen.random_memory_cols(rng, d), gen.random_memory_cols(rng, d)
@@ -888,8 +890,12 @@ def test_plan_opts_pipe_and_min_blocks():
         assert p.describe()["tile"]["min_blocks"] == 3 and ", 3) ll_tile_kernel" in p.source()
     Ac, Bc = (ll.Layout.from_spec(x) for x in W.c3(9))
     t = ll.ll_plan_convert(Ac, Bc, 2).describe()["tile"]
-    assert t["pipe"] is False and t["min_blocks"] == 0
-    assert ll.ll_plan_convert(Ac, Bc, 2, pipe="on").describe()["tile"]["pipe"] is True
+    assert t["pipe"] is False and t["min_blocks"] == 2     # 8 warps x 256 B per thread
+    assert ll.ll_plan_convert(Ac, Bc, 2, min_blocks=-1).describe()["tile"]["min_blocks"] == 0
+    t = ll.ll_plan_convert(Ac, Bc, 2, pipe="on").describe()["tile"]
+    assert t["pipe"] is True and t["min_blocks"] == 0
+    Ac, Bc = (ll.Layout.from_spec(x) for x in W.c5T(0, n=12))     # 128 B per thread: no cap
+    assert ll.ll_plan_convert(Ac, Bc, 2).describe()["tile"]["min_blocks"] == 0
 
 
 def test_opts_struct_matches_the_c_abi():

@@ -82,6 +82,12 @@ def main():
         return big_configs()
     if "ceiling" in only:
         return ceiling_cases()
+    if "shflocc" in only:
+        return shuffle_occupancy()
+    if "smemocc" in only:
+        return smem_occupancy()
+    if "laggards" in only:
+        return laggards()
     if "ctarun" in only:
         return cta_run_lengths()
     if "smallcta" in only:
@@ -764,6 +770,33 @@ def cta_run_lengths():
     for name, (sa, sb), w in [("c5T", W.c5T(0), 2), ("n1", W.n1_preshuffle(15, 15), 2)]:
         for o in [{}, {"tile_bytes": 65536}, {"tile_bytes": 131072}, {"tile_bytes": 131072, "pipe": "on"},
                   {"tile_bytes": 65536, "pipe": "on"}]:
+            conv_case(name, sa, sb, w, batch=20, **o)
+
+
+def laggards():
+    """The in-CTA rows furthest below the streaming ceiling (config 3b, the tcgen05
+    16x256b fragment) under the existing plan options; streams of 20 launches."""
+    for name, (sa, sb), w, extra in [("c3b", W.c3b(14), 2, [{"smem_instr": "vec"}]),
+                                     ("n2_16x256b", W.n2_tmem("16x256b", 14), 4, [{"force_class": "SMEM"}])]:
+        for o in [{}, {"pipe": "on"}, {"thread_bytes": 128}, {"tile_bytes": 131072}] + extra:
+            conv_case(name, sa, sb, w, batch=20, **o)
+
+
+def smem_occupancy():
+    """64 / 32 KiB smem-exchange tiles: CTAs per SM (registers: min_blocks) x the
+    pipelined exchange; streams of 20 launches."""
+    for name, (sa, sb), w in [("c3", W.c3(14), 2), ("c3b", W.c3b(14), 2), ("c5T", W.c5T(0), 2),
+                              ("n1", W.n1_preshuffle(15, 15), 2)]:
+        for o in [{}, {"pipe": "on"}, {"pipe": "on", "min_blocks": 2}, {"pipe": "on", "min_blocks": 3},
+                  {"min_blocks": 2}, {}]:
+            conv_case(name, sa, sb, w, batch=20, **o)
+
+
+def shuffle_occupancy():
+    """Shuffle-exchange rows under register caps (min_blocks); streams of 20 launches."""
+    cases = [("c2", W.c2(16), 2)] + [(f"n2_{sh}", W.n2_tmem(sh, 14), 4) for sh in ("32x32b", "16x64b", "16x128b", "16x256b")]
+    for name, (sa, sb), w in cases:
+        for o in [{}, {"min_blocks": 1}, {"min_blocks": 2}, {"min_blocks": 3}, {"min_blocks": 4}]:
             conv_case(name, sa, sb, w, batch=20, **o)
 
 
