@@ -176,6 +176,14 @@ std::string codegen_tile(const ConvPlan& Pl) {
   return o.str();
 }
 
+// Minimum-blocks hint for the gather / scan / reduce kernels (experiment hook,
+// LL_AUX_MIN_BLOCKS=k: __launch_bounds__(threads, k); default none).
+static std::string aux_min_blocks() {
+  const char* e = std::getenv("LL_AUX_MIN_BLOCKS");
+  const int k = e ? std::atoi(e) : 0;
+  return k > 0 ? ", " + std::to_string(k) : std::string();
+}
+
 std::string codegen_gather(const GatherPlan& G) {
   std::ostringstream o;
   const int n = int(G.hw_bit.size());
@@ -216,7 +224,7 @@ std::string codegen_gather(const GatherPlan& G) {
   o << "  template <int E, int C> static constexpr int slot_of() { int s = E;"
        " for (int i = 0; i < CBITS; ++i) { s &= ~(1 << CAND_REG[i]); if ((C >> i) & 1) s |= 1 << CAND_REG[i]; } return s; }\n";
   o << "};\n";
-  o << "extern \"C\" __global__ void __launch_bounds__(" << (32 << G.Wb)
+  o << "extern \"C\" __global__ void __launch_bounds__(" << (32 << G.Wb) << aux_min_blocks()
     << ") ll_gather_kernel(const u8* __restrict__ src, const u8* __restrict__ idx, u8* __restrict__ dst, u64 ntiles) {\n"
     << "  ll_gather_body<P>(src, idx, dst, ntiles);\n}\n";
   return o.str();
@@ -239,7 +247,7 @@ std::string codegen_scan(const ScanPlan& S) {
   o << "  static constexpr unsigned STAGES = " << std::max(1, S.stages) << "u;\n";
   o << "  static constexpr unsigned XS_BYTES = " << S.xs_bytes << "u;\n";
   o << "};\n";
-  o << "extern \"C\" __global__ void __launch_bounds__(" << (32 << S.Wb)
+  o << "extern \"C\" __global__ void __launch_bounds__(" << (32 << S.Wb) << aux_min_blocks()
     << ") ll_scan_kernel(const u8* __restrict__ src, u8* __restrict__ dst, u64 ntiles) {\n"
     << "  ll_scan_body<P>(src, dst, ntiles);\n}\n";
   return o.str();
@@ -275,7 +283,7 @@ std::string codegen_reduce(const ReducePlan& Rp) {
     << "  static constexpr u32 NOSTORE_WARP_MASK = " << nowarp << "u;\n";
   o << "  template <int E> static constexpr u64 out_of_slot() { u64 c = 0; for (int b = 0; b < R; ++b) if ((E >> b) & 1) c ^= OUT_COL[b]; return c; }\n";
   o << "};\n";
-  o << "extern \"C\" __global__ void __launch_bounds__(" << (32 << Rp.Wb)
+  o << "extern \"C\" __global__ void __launch_bounds__(" << (32 << Rp.Wb) << aux_min_blocks()
     << ") ll_reduce_kernel(const float* __restrict__ src, float* __restrict__ dst, u64 ntiles) {\n"
     << "  ll_reduce_body<P>(src, dst, ntiles);\n}\n";
   return o.str();

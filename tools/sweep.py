@@ -82,6 +82,8 @@ def main():
         return big_configs()
     if "ceiling" in only:
         return ceiling_cases()
+    if "c4rows" in only:
+        return c4_rows()
     if "shflocc" in only:
         return shuffle_occupancy()
     if "smemocc" in only:
@@ -798,6 +800,39 @@ def shuffle_occupancy():
     for name, (sa, sb), w in cases:
         for o in [{}, {"min_blocks": 1}, {"min_blocks": 2}, {"min_blocks": 3}, {"min_blocks": 4}]:
             conv_case(name, sa, sb, w, batch=20, **o)
+
+
+def c4_rows():
+    """Config-4 gather / reduce / scan at the config size (4 rotated buffer sets,
+    streams of 20 calls) and at 1 GiB (streams of 3), as the bench times them; the env
+    hooks of the caller apply (e.g. LL_AUX_MIN_BLOCKS)."""
+    tag = os.environ.get("LL_AUX_MIN_BLOCKS", "0")
+    for fam in ("mma", "blocked"):
+        for big in (False, True):
+            kw = dict(n_i=15, n_j=13) if big else {}
+            Lg = ll.Layout.from_spec(W.c4("gather", fam, **kw))
+            Lr = ll.Layout.from_spec(W.c4("reduce", fam, **kw))
+            n = 1 << Lg.d_in
+            nsets = 1 if big else 4
+            src = [torch.rand(n, device="cuda") for _ in range(nsets)]
+            idx = [torch.randint(0, 32, (n,), dtype=torch.int32, device="cuda") for _ in range(nsets)]
+            out = [torch.empty(n, device="cuda") for _ in range(nsets)]
+            pg, pr, ps = ll.ll_plan_gather(Lg, 1, 4), ll.ll_plan_reduce(Lr, 1), ll.ll_plan_scan(Lr, 1)
+            ro = [torch.empty(pr.out_elems(), device="cuda") for _ in range(nsets)]
+            it = [0]
+
+            def nxt():
+                it[0] += 1
+                return it[0] % nsets
+            rows = [("gather", lambda: (lambda k: ll.ll_gather(src[k], idx[k], out[k], pg))(nxt()), 12 * n),
+                    ("reduce", lambda: (lambda k: ll.ll_reduce(src[k], ro[k], pr))(nxt()), 4 * n + 4 * pr.out_elems()),
+                    ("scan", lambda: (lambda k: ll.ll_scan(src[k], out[k], ps))(nxt()), 8 * n)]
+            for name, fn, nbytes in rows:
+                ms = time_fn(fn, iters=10, warmup=3, batch=3 if big else 20)
+                print(json.dumps({"case": f"{name} {fam} {'1GiB' if big else 'config'}", "aux_min_blocks": tag,
+                                  "ms": round(ms, 4), "GBps": round(nbytes / ms / 1e6, 1)}), flush=True)
+            del src, idx, out, ro
+            torch.cuda.empty_cache()
 
 
 def small_cta_tiles():
