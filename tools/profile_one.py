@@ -26,6 +26,8 @@ conv = {"c2": (W.c2(16), 2, {}), "c2smem": (W.c2(16), 2, {"force_class": "SMEM"}
         "c1bsmem_small": (W.c1_batched(6), 4, {"force_class": "SMEM"}),
         "c3_small": (W.c3(3), 2, {}), "c3_mid_pipe": (W.c3(9), 2, {"pipe": "on"}), "c2_small": (W.c2(3), 2, {}),
         "c3b_small": (W.c3b(3), 2, {}),
+        # NOOP plans (ll_copy_kernel): a partial last CTA tile, and the 2 GiB copy
+        "noop_small": (W.n2_acc_to_lhs(16, 3), 2, {}), "noop": (W.n2_acc_to_lhs(16, 17), 2, {}),
         "acc8_small": (W.n2_acc_to_lhs(8, 4), 1, {}), "acc8f_small": (W.n2_acc_to_lhs(8, 4), 1, {"sigma": "faithful"}),
         "c2fsmem_small": (W.c2(3), 2, {"sigma": "faithful", "force_class": "SMEM", "smem_instr": "matrix"}),
         "c3f_small": (W.c3(3), 2, {"sigma": "faithful"}),
