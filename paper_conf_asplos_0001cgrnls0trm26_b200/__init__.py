@@ -433,9 +433,13 @@ class Plan:
 
     def check_buffers(self, src=None, dst=None, idx=None, workspace=None):
         """Raise LLError when a torch tensor is smaller than the plan's buffer (raw
-        pointers cannot be checked and pass through)."""
-        need = dict(zip(("src", "dst", "idx"), self.buffer_bytes()))
-        need["workspace"] = self.workspace_bytes() if self.kind == "convert" else 0
+        pointers cannot be checked and pass through).  Plans are immutable, so the
+        sizes are queried once and cached (keeps small launches off the host path)."""
+        need = self.__dict__.get("_need")
+        if need is None:
+            need = dict(zip(("src", "dst", "idx"), self.buffer_bytes()))
+            need["workspace"] = self.workspace_bytes() if self.kind == "convert" else 0
+            self._need = need
         for name, t in (("src", src), ("dst", dst), ("idx", idx), ("workspace", workspace)):
             if t is None or isinstance(t, int) or not hasattr(t, "numel"):
                 if name == "workspace" and t is None and need[name] > 0:

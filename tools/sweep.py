@@ -42,6 +42,32 @@ def time_fn(fn, iters=20, warmup=5, batch=None):
     return ts[len(ts) // 2]
 
 
+def time_graph(fn, batch, iters=10):
+    """Median time per call of `batch` calls captured in one CUDA graph (no host launch
+    overhead between the kernels; PDL edges are captured as programmatic dependencies)."""
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        for _ in range(3):
+            fn()
+        torch.cuda.synchronize()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=s):
+            for _ in range(batch):
+                fn()
+        g.replay()
+        torch.cuda.synchronize()
+        ts = []
+        for _ in range(iters):
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record()
+            g.replay()
+            b.record()
+            b.synchronize()
+            ts.append(a.elapsed_time(b) / batch)
+    ts.sort()
+    return ts[len(ts) // 2]
+
+
 def conv_case(name, sa, sb, w, batch=None, **opts):
     A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
     p = ll.ll_plan_convert(A, B, w, **opts)
@@ -828,9 +854,12 @@ def c4_rows():
                     ("reduce", lambda: (lambda k: ll.ll_reduce(src[k], ro[k], pr))(nxt()), 4 * n + 4 * pr.out_elems()),
                     ("scan", lambda: (lambda k: ll.ll_scan(src[k], out[k], ps))(nxt()), 8 * n)]
             for name, fn, nbytes in rows:
-                ms = time_fn(fn, iters=10, warmup=3, batch=3 if big else 20)
+                nb = 3 if big else 20
+                ms = time_fn(fn, iters=10, warmup=3, batch=nb)
+                gms = time_graph(fn, nb)
                 print(json.dumps({"case": f"{name} {fam} {'1GiB' if big else 'config'}", "aux_min_blocks": tag,
-                                  "ms": round(ms, 4), "GBps": round(nbytes / ms / 1e6, 1)}), flush=True)
+                                  "ms": round(ms, 4), "GBps": round(nbytes / ms / 1e6, 1),
+                                  "graph_ms": round(gms, 4), "graph_GBps": round(nbytes / gms / 1e6, 1)}), flush=True)
             del src, idx, out, ro
             torch.cuda.empty_cache()
 
