@@ -234,6 +234,33 @@ def _time_stream(fn, torch, samples=10, batch=20, warmup=3):
     return ts[len(ts) // 2]
 
 
+def _time_graph(fn, torch, batch=20, samples=10):
+    """Median time per call of `batch` calls captured in one CUDA graph: the small
+    config-4 kernels (12-31 us) without the Python launch path between them (the
+    production form of a launch-bound loop; PDL edges are captured)."""
+    st = torch.cuda.Stream()
+    with torch.cuda.stream(st):
+        for _ in range(3):
+            fn()
+        torch.cuda.synchronize()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=st):
+            for _ in range(batch):
+                fn()
+        g.replay()
+        torch.cuda.synchronize()
+        ts = []
+        for _ in range(samples):
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record()
+            g.replay()
+            b.record()
+            b.synchronize()
+            ts.append(a.elapsed_time(b) / batch)
+    ts.sort()
+    return ts[len(ts) // 2]
+
+
 def torch_permute_baseline(torch, A_spec, B_spec, src, w, steps=5):
     """Context for the headline: the same conversion done the way a PyTorch user would —
     the packed buffer viewed as a tensor of 2-sized dims, permuted and made contiguous
@@ -386,6 +413,7 @@ def other_configs(ll, W, torch, peak):
             it[0] += 1
             ll.ll_gather(s[0], s[1], s[2], p)
         ms = _time_stream(g1, torch)
+        gms = _time_graph(g1, torch)
         d = p.describe()
         gbs = 12 * n / ms / 1e6
         # context: PyTorch's own gather on the logical [4096*128, 32] view, same bytes,
@@ -401,6 +429,7 @@ def other_configs(ll, W, torch, peak):
                     "executed": d["exchange"] + (" (TMA stages)" if d.get("tma") else ""), "ms": round(ms, 4),
                     "shuffles_per_elem": d.get("shuffles_per_elem"),
                     "GBps": round(gbs, 1), "frac": round(gbs / peak, 3),
+                    "graph_GBps": round(12 * n / gms / 1e6, 1), "graph_frac": round(12 * n / gms / 1e6 / peak, 3),
                     "torch_gather_same_bytes_GBps": round(12 * n / ms_t / 1e6, 1),
                     "size_matched_copy_GBps": size_matched_copy(torch, 12 * n)})
         del tsets
@@ -413,7 +442,9 @@ def other_configs(ll, W, torch, peak):
             it[0] += 1
             ll.ll_reduce(s[0], s[1], p)
         ms = _time_stream(r1, torch)
+        gms = _time_graph(r1, torch)
         gbs = (4 * n + 4 * p.out_elems()) / ms / 1e6
+        ggbs = (4 * n + 4 * p.out_elems()) / gms / 1e6
 
         # context: PyTorch's own sum over the logical [4096, 32, 128] view (same bytes)
         def tr():
@@ -424,6 +455,7 @@ def other_configs(ll, W, torch, peak):
         out.append({"workload": f"config 4 reduce: [4096,4096] fp32 -> [4096,32], {fam} [128,128] tiles",
                     "class": "reduce", "executed": "logical-order steps (register / shfl.bfly / smem)" + (" (TMA stages)" if p.describe().get("tma") else ""),
                     "ms": round(ms, 4), "GBps": round(gbs, 1), "frac": round(gbs / peak, 3),
+                    "graph_GBps": round(ggbs, 1), "graph_frac": round(ggbs / peak, 3),
                     "torch_sum_same_bytes_GBps": round((4 * n + 4 * p.out_elems()) / ms_t / 1e6, 1),
                     "size_matched_copy_GBps": size_matched_copy(torch, 4 * n + 4 * p.out_elems())})
         # scan (N3): inclusive prefix sum along the axis inside each [128, 128] tile
@@ -435,6 +467,7 @@ def other_configs(ll, W, torch, peak):
             it[0] += 1
             ll.ll_scan(s[0], s[1], p)
         ms = _time_stream(s1, torch)
+        gms = _time_graph(s1, torch)
         gbs = 8 * n / ms / 1e6
 
         def ts():
@@ -446,6 +479,7 @@ def other_configs(ll, W, torch, peak):
         out.append({"workload": f"config 4 scan (N3): [4096,4096] fp32 inclusive prefix sum inside {fam} [128,128] tiles",
                     "class": "scan", "executed": f"{d['steps']} bit-doubling steps, {d['shuffles_per_elem']} shuffles/elem",
                     "ms": round(ms, 4), "GBps": round(gbs, 1), "frac": round(gbs / peak, 3),
+                    "graph_GBps": round(8 * n / gms / 1e6, 1), "graph_frac": round(8 * n / gms / 1e6 / peak, 3),
                     "torch_cumsum_same_bytes_GBps": round(8 * n / ms_t / 1e6, 1),
                     "size_matched_copy_GBps": size_matched_copy(torch, 8 * n)})
         del sets, rsets, ssets

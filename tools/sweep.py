@@ -108,6 +108,8 @@ def main():
         return big_configs()
     if "ceiling" in only:
         return ceiling_cases()
+    if "fammb" in only:
+        return families_min_blocks()
     if "c4rows" in only:
         return c4_rows()
     if "shflocc" in only:
@@ -462,6 +464,62 @@ def reduce_scan_families():
                         print(json.dumps({"kind": kind, "family": fam, "shape": shape, "axis": axis - 1,
                                           "MiB": (4 * n) >> 20, "res": res}), flush=True)
                 del sets
+
+
+def families_min_blocks():
+    """Default gather / reduce / scan plans over Table 4 families x 3 tile shapes x 2
+    axes at 64 MiB (4 rotated sets, CUDA graph of 20 calls) and 1 GiB (stream of 3),
+    under the caller's LL_AUX_MIN_BLOCKS."""
+    import numpy as np
+    from workloads import gen
+    tag = os.environ.get("LL_AUX_MIN_BLOCKS", "0")
+    rng = np.random.default_rng(77)
+    fams = {
+        "blocked": lambda a, b: ll.ll_layout_blocked([a, b], [1, 4], [8, 4], [4, 1], [1, 0]),
+        "mma": lambda a, b: ll.ll_layout_mma_acc(a, b, 4),
+        "mma_input": lambda a, b: ll.ll_layout_mma_operand(0, a, b, 16, 4, 1),
+        "custom": lambda a, b: ll.Layout.from_spec(gen.random_distributed(
+            rng, [("r", a.bit_length() - 1), ("c", b.bit_length() - 1)],
+            [("reg", max(1, a.bit_length() + b.bit_length() - 2 - 7)), ("lane", 5), ("warp", 2)],
+            zero_ok=["reg", "lane", "warp"])),
+    }
+    for fam, mk in fams.items():
+        for shape in ((128, 128), (128, 16), (32, 128)):
+            T = mk(*shape)
+            for total in (24, 28):
+                L = _batched(T, total - T.d_in)
+                n = 1 << L.d_in
+                nset = 4 if total == 24 else 1
+                sets = [torch.rand(n, device="cuda") for _ in range(nset)]
+                idx = [torch.randint(0, 1 << 20, (n,), dtype=torch.int32, device="cuda") for _ in range(nset)]
+                for axis in (1, 2):
+                    for kind in ("reduce", "scan", "gather"):
+                        try:
+                            if kind == "gather":
+                                p = ll.ll_plan_gather(L, axis, 4)
+                            else:
+                                p = (ll.ll_plan_scan if kind == "scan" else ll.ll_plan_reduce)(L, axis)
+                        except Exception as e:   # noqa: BLE001
+                            print(json.dumps({"kind": kind, "family": fam, "error": str(e)[:80]}), flush=True)
+                            continue
+                        m = p.out_elems() if kind == "reduce" else n
+                        outs = [torch.empty(m, device="cuda") for _ in sets]
+                        it = [0]
+
+                        def f():
+                            k = it[0] % nset
+                            it[0] += 1
+                            if kind == "gather":
+                                ll.ll_gather(sets[k], idx[k], outs[k], p)
+                            else:
+                                (ll.ll_scan if kind == "scan" else ll.ll_reduce)(sets[k], outs[k], p)
+                        nbytes = 4 * (n + m) + (4 * n if kind == "gather" else 0)
+                        ms = time_graph(f, 20) if total == 24 else time_fn(f, batch=3)
+                        print(json.dumps({"kind": kind, "family": fam, "shape": shape, "axis": axis - 1,
+                                          "MiB": (4 * n) >> 20, "aux_min_blocks": tag,
+                                          "GBps": round(nbytes / ms / 1e6, 1)}), flush=True)
+                        del outs
+                del sets, idx
 
 
 def gather_families():
