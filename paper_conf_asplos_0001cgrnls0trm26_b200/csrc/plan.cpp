@@ -893,15 +893,18 @@ static void plan_exchange(ConvPlan& P, const ll_plan_opts* opts) {
 // exchange, whose tiles must load from one rank).
 static void choose_cta_tile(const std::vector<int>& pi, int nloc, int c_bits,
                             int target_bits, std::vector<int>& S, std::vector<int>& D,
-                            std::vector<int>& gS, std::vector<int>& gD, u64 grid_only_src = 0) {
+                            std::vector<int>& gS, std::vector<int>& gD, u64 grid_only_src = 0,
+                            int c_ld_bits = -1) {
+  // dst runs of 2^c_bits elements, src runs of 2^c_ld_bits (default: the same)
+  if (c_ld_bits < 0) c_ld_bits = c_bits;
   std::vector<int> inv(nloc, -1);
   for (int k = 0; k < nloc; ++k) inv[pi[k]] = k;
   std::vector<char> inT(nloc, 0);
   auto ok = [&](int d) { return !((grid_only_src >> pi[d]) & 1); };
-  for (int k = 0; k < std::min(c_bits, nloc); ++k) {
+  for (int k = 0; k < std::min(c_bits, nloc); ++k)
     if (ok(k)) inT[k] = 1;
+  for (int k = 0; k < std::min(c_ld_bits, nloc); ++k)
     if (ok(inv[k])) inT[inv[k]] = 1;
-  }
   int cnt = 0;
   for (int k = 0; k < nloc; ++k) cnt += inT[k];
   for (int k = 0; k < nloc && cnt < target_bits; ++k) if (!inT[k] && ok(k)) { inT[k] = 1; ++cnt; }
@@ -1161,8 +1164,12 @@ std::unique_ptr<ConvPlan> plan_convert(const Layout& A, const Layout& B, int w, 
           // 64 KiB of smem (or ll_plan_opts.tile_bytes when larger): 512-byte runs, else
           // 256, else 128 (one line)
           const int max_bits = ilog2(u64(std::max(65536, tb) / w));
+          // experiment hook LL_CTA_RUNS=<ld extra bits>: src runs longer than the dst runs
+          const char* re = std::getenv("LL_CTA_RUNS");
+          const int ld_extra = re ? std::atoi(re) : 0;
           for (int c_bits = v + 5; c_bits >= v + 3; --c_bits) {
-            choose_cta_tile(pi, nB, c_bits, target, S, D, gS, gD, grid_only_src);
+            choose_cta_tile(pi, nB, c_bits, target, S, D, gS, gD, grid_only_src,
+                            ld_extra ? std::min(std::max(c_bits + ld_extra, v + 3), v + 6) : -1);
             if (int(S.size()) <= max_bits) break;
           }
           build_tile(*P, S, D, gS, gD, opts, false, grid_only_src);

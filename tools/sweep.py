@@ -108,6 +108,8 @@ def main():
         return big_configs()
     if "ceiling" in only:
         return ceiling_cases()
+    if "asym" in only:
+        return cta_asym_runs()
     if "fammb" in only:
         return families_min_blocks()
     if "c4rows" in only:
@@ -920,6 +922,16 @@ def c4_rows():
                                   "graph_ms": round(gms, 4), "graph_GBps": round(nbytes / gms / 1e6, 1)}), flush=True)
             del src, idx, out, ro
             torch.cuda.empty_cache()
+
+
+def cta_asym_runs():
+    """CTA-class transposes with src runs longer / shorter than dst runs (LL_CTA_RUNS=+1
+    / -1, 64 KiB tiles) vs the default symmetric 256-byte runs; streams of 20 launches."""
+    for e in ("0", "1", "-1", "0"):
+        os.environ["LL_CTA_RUNS"] = e
+        for name, (sa, sb), w in [("c5T", W.c5T(0), 2), ("n1", W.n1_preshuffle(15, 15), 2)]:
+            conv_case(f"{name} runs{e}", sa, sb, w, batch=20)
+    os.environ["LL_CTA_RUNS"] = "0"
 
 
 def small_cta_tiles():
