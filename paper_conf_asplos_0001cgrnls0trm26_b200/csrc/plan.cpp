@@ -1425,7 +1425,8 @@ std::string describe(const ConvPlan& P) {
         << ",\"F\":" << vec_json(T.F) << ",\"G\":" << vec_json(T.G) << ",\"R_basis\":" << vec_json(T.Rb)
         << ",\"rounds\":" << T.rounds << ",\"pre_stages\":" << T.pre_x.size()
         << ",\"post_stages\":" << T.post_x.size() << ",\"unit_elems\":" << T.unit_elems
-        << ",\"element_permutes\":" << (T.pre_eperm.empty() ? "false" : "true");
+        << ",\"element_permutes\":" << (T.pre_eperm.empty() ? "false" : "true")
+        << ",\"min_blocks\":" << T.min_blocks;
     if (T.xchg == X_SMEM)
       o << ",\"Vec\":" << vec_json(T.sw_vec) << ",\"Bank\":" << vec_json(T.sw_bank) << ",\"Seg\":" << vec_json(T.sw_seg)
         << ",\"H\":" << vec_json(T.sw_H) << ",\"C\":" << vec_json(T.sw_C)

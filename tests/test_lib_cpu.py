@@ -1094,3 +1094,22 @@ def test_noop_partial_overlap_refused():
     base = 1 << 32
     with pytest.raises(ll.LLError, match="ALIAS"):
         ll.ll_convert(base, base + 512, p, stream=0)      # 1 KiB buffers overlapping by half
+
+
+def test_round2_kernel_shape_defaults():
+    """Measured defaults: folded small tiles run 8 warps x 64 B per
+    thread; shuffle / smem tiles of 256 B per thread with <= 8 warps carry the 2-CTA
+    register hint (config 2, config 3); the CTA-class transpose (128 B per thread) and
+    config 2's own 4-warp shuffle keep their shapes."""
+    def tile(spec, w, **o):
+        A, B = (ll.Layout.from_spec(x) for x in spec)
+        return ll.ll_plan_convert(A, B, w, **o).describe()["tile"]
+    t = tile(W.c2(4), 2)
+    assert t["xchg"] == "shuffle" and t["threads"] == 128 and t["min_blocks"] == 2
+    t = tile(W.c3(4), 2)
+    assert t["xchg"] == "smem" and t["threads"] == 256 and t["min_blocks"] == 2
+    t = tile(W.c1_batched(12), 4)
+    assert t["threads"] == 256 and t["R"] == 4          # 16 KiB folded tile, 64 B per thread
+    assert tile(W.c1_batched(12), 4, thread_bytes=256)["threads"] == 64
+    t = tile(W.c5T(0, n=12), 2)
+    assert t["min_blocks"] == 0
