@@ -33,6 +33,7 @@ conv = {"c2": (W.c2(16), 2, {}), "c2smem": (W.c2(16), 2, {"force_class": "SMEM"}
         "c3f_small": (W.c3(3), 2, {"sigma": "faithful"}),
         "c5T": (W.c5T(0, n=15), 2, {}), "n1": (W.n1_preshuffle(14, 14), 2, {}),
         "n2": (W.n2_tmem_epilogue(13), 4, {}),
+        "n2_16x128b": (W.n2_tmem("16x128b", 14), 4, {}), "n2_16x256b": (W.n2_tmem("16x256b", 14), 4, {}),
         # Thm 5.1: stmatrix / ldmatrix vs vectorised ld/st.shared only
         "c3bvec": (W.c3b(14), 2, {"smem_instr": "vec"}),
         "c2fsmem": (W.c2(16), 2, {"sigma": "faithful", "force_class": "SMEM", "smem_instr": "matrix"}),
