@@ -285,19 +285,24 @@ def torch_permute_baseline(torch, A_spec, B_spec, src, w, steps=5):
     order = [dim_of[lo] for lo, _ in reversed(runs)]   # dst dims, most significant first
     et = {1: torch.uint8, 2: torch.int16, 4: torch.int32, 8: torch.int64}[w]
     x = src.view(et).view(*shape)
+    xp = x.permute(*order)
+    y = torch.empty(xp.shape, dtype=et, device=src.device)   # preallocated: no allocator churn
 
     def run():
-        return x.permute(*order).contiguous()
-    y = run()
+        y.copy_(xp)                      # the strided copy permute(...).contiguous() runs
+    run()
     torch.cuda.synchronize()
-    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    a.record()
+    ts = []
     for _ in range(steps):
-        y = run()
-    b.record()
-    torch.cuda.synchronize()
-    ms = a.elapsed_time(b) / steps
-    return {"impl": "torch: packed src viewed as %d dims, permute(...).contiguous()" % len(shape),
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        run()
+        b.record()
+        b.synchronize()
+        ts.append(a.elapsed_time(b))
+    ms = sorted(ts)[len(ts) // 2]
+    return {"impl": "torch: packed src viewed as %d dims, permute(...) copied into a preallocated "
+                    "contiguous tensor (the strided copy of .contiguous()), median of %d" % (len(shape), steps),
             "GBps": round(2 * src.numel() * src.element_size() / (ms / 1e3) / 1e9, 1), "ms": round(ms, 4)}, \
         y.reshape(-1).view(src.dtype)
 

@@ -11,7 +11,18 @@ from tests._fuzz import fuzz_case
 ll = pytest.importorskip("paper_conf_asplos_0001cgrnls0trm26_b200")
 
 
-@pytest.mark.parametrize("seed", [1, 2, 3, 4])
+def _seeds(default):
+    """Seeds of the fuzz cases: the default list, or LL_FUZZ_SEEDS="a-b" for an
+    extended run (e.g. the round-end robustness pass)."""
+    import os
+    e = os.environ.get("LL_FUZZ_SEEDS")
+    if not e:
+        return default
+    a, b = (int(x) for x in e.split("-"))
+    return list(range(a, b + 1))
+
+
+@pytest.mark.parametrize("seed", _seeds([1, 2, 3, 4]))
 def test_fuzz_plans_simulated(seed):
     rng = np.random.default_rng(9000 + seed)
     tiles = 0

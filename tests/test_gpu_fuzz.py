@@ -15,7 +15,18 @@ pytestmark = pytest.mark.gpu
 ll = pytest.importorskip("paper_conf_asplos_0001cgrnls0trm26_b200")
 
 
-@pytest.mark.parametrize("seed", [1, 2, 3])
+def _seeds(default):
+    """Seeds of the fuzz cases: the default list, or LL_FUZZ_SEEDS="a-b" for an
+    extended run (e.g. the round-end robustness pass)."""
+    import os
+    e = os.environ.get("LL_FUZZ_SEEDS")
+    if not e:
+        return default
+    a, b = (int(x) for x in e.split("-"))
+    return list(range(a, b + 1))
+
+
+@pytest.mark.parametrize("seed", _seeds([1, 2, 3]))
 def test_fuzz_conversions_bitexact(seed):
     import torch
     rng = np.random.default_rng(7000 + seed)
