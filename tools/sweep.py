@@ -108,6 +108,8 @@ def main():
         return big_configs()
     if "ceiling" in only:
         return ceiling_cases()
+    if "c5peer" in only:
+        return c5_peer_tiles()
     if "asym" in only:
         return cta_asym_runs()
     if "fammb" in only:
@@ -932,6 +934,24 @@ def cta_asym_runs():
         for name, (sa, sb), w in [("c5T", W.c5T(0), 2), ("n1", W.n1_preshuffle(15, 15), 2)]:
             conv_case(f"{name} runs{e}", sa, sb, w, batch=20)
     os.environ["LL_CTA_RUNS"] = "0"
+
+
+def c5_peer_tiles():
+    """Config 5 at P = 8 on one GPU (loopback windows, peer-store tile kernel): CTA tile
+    bytes x bytes per thread of the fused copy tiles; streams of 20 launches."""
+    sa, sb = W.c5(3)
+    A, B = ll.Layout.from_spec(sa), ll.Layout.from_spec(sb)
+    n = 1 << 30
+    src = torch.randint(-2 ** 15, 2 ** 15, (n,), dtype=torch.int16, device="cuda")
+    dst = torch.empty_like(src)
+    for o in [{}, {"tile_bytes": 32768}, {"tile_bytes": 65536}, {"tile_bytes": 32768, "thread_bytes": 64},
+              {"thread_bytes": 128}, {"tile_bytes": 65536, "thread_bytes": 128}, {}]:
+        p = ll.ll_plan_convert(A, B, 2, comm=ll.Comm.loopback(8), exchange="peer", **o)
+        p.prepare()
+        t = p.describe()["fused"]["tile"]
+        ms = time_fn(lambda: ll.ll_convert(src, dst, p), batch=20, iters=10)
+        print(json.dumps({"case": "c5 P=8 loopback peer", "opts": o, "n": t["n"], "threads": t["threads"],
+                          "ms": round(ms, 4), "GBps": round(4 * n / ms / 1e6, 1)}), flush=True)
 
 
 def small_cta_tiles():
