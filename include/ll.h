@@ -134,7 +134,9 @@ typedef struct {
                          * linear tiles also take it as their size cap (default 64 KiB);
                          * gather / reduce / scan: split the layout's CTA tile down to
                          * it (warp bits of independent rows become grid bits; 0 = keep) */
-  int thread_bytes;     /* target bytes per thread (0 = default)                 */
+  int thread_bytes;     /* target bytes per thread (0 = default: 256; 64 when the
+                         * layout's own CTA tile is below tile_bytes and grid bits
+                         * are folded in)                                          */
   int generic;          /* 1 = force the runtime-generic kernel                   */
   ll_comm* comm;        /* required for DEVICE plans                              */
   int exchange;         /* DEVICE plans: an ll_exchange (default AUTO)            */
@@ -160,8 +162,9 @@ typedef struct {
                          * the contiguous CTA tile), 5 = TMA stages and (scan) the
                          * result tile out by cp.async.bulk                          */
   int min_blocks;       /* tile kernels: resident CTAs per SM requested from ptxas
-                         * (__launch_bounds__ minimum): 0 = auto (2 for linear tiles,
-                         * else none), -1 = none, k >= 1 = k                          */
+                         * (__launch_bounds__ minimum): 0 = auto (2 for linear tiles and
+                         * for unpipelined shuffle / smem tiles of 256 bytes per thread
+                         * with <= 8 warps, else none), -1 = none, k >= 1 = k         */
 } ll_plan_opts;
 
 /* Fill *opts with defaults (force_class = -1, max_vec_bytes = 16, ...). */
