@@ -134,9 +134,10 @@ typedef struct {
                          * linear tiles also take it as their size cap (default 64 KiB);
                          * gather / reduce / scan: split the layout's CTA tile down to
                          * it (warp bits of independent rows become grid bits; 0 = keep) */
-  int thread_bytes;     /* target bytes per thread (0 = default: 256; 64 when the
-                         * layout's own CTA tile is below tile_bytes and grid bits
-                         * are folded in)                                          */
+  int thread_bytes;     /* target bytes per thread (0 = default: in-CTA tiles 256,
+                         * or 64 when the layout's own CTA tile is below tile_bytes
+                         * and grid bits are folded in; cross-CTA tiles: the tile's
+                         * bytes / 256, within [elem_bytes, 256])                  */
   int generic;          /* 1 = force the runtime-generic kernel                   */
   ll_comm* comm;        /* required for DEVICE plans                              */
   int exchange;         /* DEVICE plans: an ll_exchange (default AUTO)            */
