@@ -62,8 +62,8 @@
  *  - LL_ST_HINT=wb: tile kernels store with the default write-back policy instead of
  *    st.global.cs (evict-first streaming).
  *  - LL_AUX_MIN_BLOCKS=k: gather / reduce / scan kernels compiled with
- *    __launch_bounds__(threads, k) (experiment; default none — measured mixed,
- *    profiles/r02_sweep_families_aux_min_blocks.jsonl).
+ *    __launch_bounds__(threads, k), 0 = none (experiment; default: 2 for scans without
+ *    a shared-memory warp step, none otherwise — profiles/r02_sweep_families_aux_min_blocks.jsonl).
  *  - LL_CTA_RUNS=+1|-1: CTA-class permutation tiles take src runs one bit longer (+1)
  *    or shorter (-1) than the dst runs (experiment; default: equal run lengths).
  *  - LL_NCCL_LIB=<path>: the libnccl.so.2 dlopen'ed for DEVICE plans (the Python binding

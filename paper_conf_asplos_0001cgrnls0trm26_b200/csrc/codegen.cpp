@@ -176,11 +176,11 @@ std::string codegen_tile(const ConvPlan& Pl) {
   return o.str();
 }
 
-// Minimum-blocks hint for the gather / scan / reduce kernels (experiment hook,
-// LL_AUX_MIN_BLOCKS=k: __launch_bounds__(threads, k); default none).
-static std::string aux_min_blocks() {
+// Minimum-blocks hint for the gather / scan / reduce kernels: `dflt` CTAs per SM
+// (0 = none); LL_AUX_MIN_BLOCKS=k overrides it (0 = none) for experiments.
+static std::string aux_min_blocks(int dflt = 0) {
   const char* e = std::getenv("LL_AUX_MIN_BLOCKS");
-  const int k = e ? std::atoi(e) : 0;
+  const int k = e ? std::atoi(e) : dflt;
   return k > 0 ? ", " + std::to_string(k) : std::string();
 }
 
@@ -247,7 +247,10 @@ std::string codegen_scan(const ScanPlan& S) {
   o << "  static constexpr unsigned STAGES = " << std::max(1, S.stages) << "u;\n";
   o << "  static constexpr unsigned XS_BYTES = " << S.xs_bytes << "u;\n";
   o << "};\n";
-  o << "extern \"C\" __global__ void __launch_bounds__(" << (32 << S.Wb) << aux_min_blocks()
+  // scans without a shared-memory warp step (axis bits on registers and lanes) ask for
+  // 2 CTAs per SM: +0.3-3.5% on all 24 such Table 4 cases (families x tiles x 64 MiB /
+  // 1 GiB), mixed with a warp step (profiles/r02_sweep_families_aux_min_blocks.jsonl)
+  o << "extern \"C\" __global__ void __launch_bounds__(" << (32 << S.Wb) << aux_min_blocks(S.xs_bytes == 0 ? 2 : 0)
     << ") ll_scan_kernel(const u8* __restrict__ src, u8* __restrict__ dst, u64 ntiles) {\n"
     << "  ll_scan_body<P>(src, dst, ntiles);\n}\n";
   return o.str();
